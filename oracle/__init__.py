@@ -1,0 +1,172 @@
+"""ctypes wrapper around liboracle.so -- the fp64 CPU oracle (TEST INFRASTRUCTURE).
+
+Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline /
+``--impl reference`` legs may import this package.  The product path
+(paper_conf_dac_lugklr25_b200) never does.
+
+All functions take a ``synth.Graph``-like object (caller order, fp32 or fp64
+arrays) and compute in fp64 (oracle/oracle.c).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_LIB = os.path.join(_HERE, "liboracle.so")
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    src = os.path.join(_HERE, "oracle.c")
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(src):
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-ffp-contract=off", "-fPIC", "-shared",
+                               "-Wall", "-o", _LIB, src, "-lm"])
+    return _LIB
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build()
+        _lib = ctypes.CDLL(_LIB)
+    return _lib
+
+
+class _OrcGraph(ctypes.Structure):
+    _fields_ = [
+        ("num_pins", ctypes.c_int32),
+        ("num_arcs", ctypes.c_int64),
+        ("arc_from", ctypes.c_void_p),
+        ("arc_to", ctypes.c_void_p),
+        ("arc_unate", ctypes.c_void_p),
+        ("arc_mean", ctypes.c_void_p),
+        ("arc_sigma", ctypes.c_void_p),
+        ("src_mean", ctypes.c_void_p),
+        ("src_sigma", ctypes.c_void_p),
+        ("num_endpoints", ctypes.c_int32),
+        ("ep_pin", ctypes.c_void_p),
+        ("ep_rat", ctypes.c_void_p),
+    ]
+
+
+def _p(a):
+    return None if a is None else a.ctypes.data
+
+
+class OracleError(RuntimeError):
+    pass
+
+
+def _check(st):
+    if st == 1:
+        raise OracleError("oracle: bad argument")
+    if st == 2:
+        raise OracleError("oracle: combinational cycle")
+    if st:
+        raise OracleError(f"oracle: status {st}")
+
+
+class OGraph:
+    """fp64 copies of a graph's arrays + the C struct pointing at them."""
+
+    def __init__(self, g):
+        self.N = int(g.num_pins)
+        self.E = int(np.asarray(g.arc_from).shape[0])
+        self.P = int(np.asarray(g.ep_pin).shape[0])
+        self.arc_from = np.ascontiguousarray(g.arc_from, np.int32)
+        self.arc_to = np.ascontiguousarray(g.arc_to, np.int32)
+        self.arc_unate = np.ascontiguousarray(g.arc_unate, np.uint8)
+        self.arc_mean = np.ascontiguousarray(np.asarray(g.arc_mean, np.float64).reshape(self.E, 2))
+        self.arc_sigma = np.ascontiguousarray(np.asarray(g.arc_sigma, np.float64).reshape(self.E, 2))
+        self.src_mean = None if g.src_mean is None else np.ascontiguousarray(np.asarray(g.src_mean, np.float64).reshape(self.N, 2))
+        self.src_sigma = None if g.src_sigma is None else np.ascontiguousarray(np.asarray(g.src_sigma, np.float64).reshape(self.N, 2))
+        self.ep_pin = np.ascontiguousarray(g.ep_pin, np.int32)
+        self.ep_rat = np.ascontiguousarray(np.asarray(g.ep_rat, np.float64).reshape(self.P, 2))
+        self.c = _OrcGraph(self.N, self.E, _p(self.arc_from), _p(self.arc_to), _p(self.arc_unate),
+                           _p(self.arc_mean), _p(self.arc_sigma), _p(self.src_mean), _p(self.src_sigma),
+                           self.P, _p(self.ep_pin), _p(self.ep_rat))
+
+
+def _og(g):
+    return g if isinstance(g, OGraph) else OGraph(g)
+
+
+def levelize(num_pins, arc_from, arc_to):
+    """Returns dict(level, order, fanin_ptr, fanin_arc, fanout_ptr, fanout_arc, num_levels)."""
+    arc_from = np.ascontiguousarray(arc_from, np.int32)
+    arc_to = np.ascontiguousarray(arc_to, np.int32)
+    N, E = int(num_pins), int(arc_from.shape[0])
+    out = dict(level=np.zeros(N, np.int32), order=np.zeros(N, np.int32),
+               fanin_ptr=np.zeros(N + 1, np.int32), fanin_arc=np.zeros(E, np.int32),
+               fanout_ptr=np.zeros(N + 1, np.int32), fanout_arc=np.zeros(E, np.int32))
+    nl = ctypes.c_int32(0)
+    L = lib()
+    L.orc_levelize.argtypes = [ctypes.c_int32, ctypes.c_int64] + [ctypes.c_void_p] * 9
+    _check(L.orc_levelize(N, E, _p(arc_from), _p(arc_to), _p(out["level"]), _p(out["order"]),
+                          _p(out["fanin_ptr"]), _p(out["fanin_arc"]), _p(out["fanout_ptr"]),
+                          _p(out["fanout_arc"]), ctypes.byref(nl)))
+    out["num_levels"] = int(nl.value)
+    return out
+
+
+def forward(g, n_sigma=3.0, tau=0.0):
+    """Returns dict(A, sigma, mu [N,2], win_arc, win_s [N,2], gap [N,2])."""
+    og = _og(g)
+    N = og.N
+    A = np.zeros((N, 2)); sig = np.zeros((N, 2)); mu = np.zeros((N, 2))
+    wa = np.zeros((N, 2), np.int32); ws = np.zeros((N, 2), np.int8); gap = np.zeros((N, 2))
+    L = lib()
+    L.orc_forward.argtypes = [ctypes.c_void_p, ctypes.c_double, ctypes.c_double] + [ctypes.c_void_p] * 6
+    _check(L.orc_forward(ctypes.byref(og.c), float(n_sigma), float(tau), _p(A), _p(sig), _p(mu),
+                         _p(wa), _p(ws), _p(gap)))
+    return dict(A=A, sigma=sig, mu=mu, win_arc=wa, win_s=ws, gap=gap)
+
+
+def slack(g, A):
+    """Returns dict(slack [P], rf_star [P], wns, tns, num_viol)."""
+    og = _og(g)
+    A = np.ascontiguousarray(A, np.float64)
+    s = np.zeros(og.P); r = np.zeros(og.P, np.uint8)
+    wns = ctypes.c_double(); tns = ctypes.c_double(); nv = ctypes.c_int32()
+    L = lib()
+    L.orc_slack.argtypes = [ctypes.c_void_p] * 7
+    _check(L.orc_slack(ctypes.byref(og.c), _p(A), _p(s), _p(r), ctypes.byref(wns), ctypes.byref(tns),
+                       ctypes.byref(nv)))
+    return dict(slack=s, rf_star=r, wns=wns.value, tns=tns.value, num_viol=nv.value)
+
+
+def backward(g, n_sigma=3.0, tau=0.0, dslack=None):
+    """Returns dict(d_mean, d_sigma [E,2], d_src_mean, d_src_sigma, abar [N,2])."""
+    og = _og(g)
+    E, N = og.E, og.N
+    dm = np.zeros((E, 2)); ds = np.zeros((E, 2))
+    dsm = np.zeros((N, 2)); dss = np.zeros((N, 2)); ab = np.zeros((N, 2))
+    if dslack is not None:
+        dslack = np.ascontiguousarray(dslack, np.float64)
+    L = lib()
+    L.orc_backward.argtypes = [ctypes.c_void_p, ctypes.c_double, ctypes.c_double] + [ctypes.c_void_p] * 6
+    _check(L.orc_backward(ctypes.byref(og.c), float(n_sigma), float(tau), _p(dslack), _p(dm), _p(ds),
+                          _p(dsm), _p(dss), _p(ab)))
+    return dict(d_mean=dm, d_sigma=ds, d_src_mean=dsm, d_src_sigma=dss, abar=ab)
+
+
+def tie_taint(g, n_sigma=3.0, eps=1e-3, margin=1.0):
+    """Test support: (fwd_taint [N,2] bool, arc_taint [E,2] bool) for hard-mode parity."""
+    og = _og(g)
+    ft = np.zeros((og.N, 2), np.uint8); at = np.zeros((og.E, 2), np.uint8)
+    L = lib()
+    L.orc_tie_taint.argtypes = [ctypes.c_void_p, ctypes.c_double, ctypes.c_double, ctypes.c_double,
+                                ctypes.c_void_p, ctypes.c_void_p]
+    _check(L.orc_tie_taint(ctypes.byref(og.c), float(n_sigma), float(eps), float(margin), _p(ft), _p(at)))
+    return ft.astype(bool), at.astype(bool)
+
+
+def validate(g, n_sigma=3.0, tau=0.0) -> int:
+    og = _og(g)
+    L = lib()
+    L.orc_validate.argtypes = [ctypes.c_void_p, ctypes.c_double, ctypes.c_double]
+    return int(L.orc_validate(ctypes.byref(og.c), float(n_sigma), float(tau)))

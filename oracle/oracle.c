@@ -1,0 +1,495 @@
+/*
+ * oracle.c -- plain, slow, obviously-correct fp64 CPU oracle of INSTA's K=1
+ * statistical arrival propagation, endpoint slack / WNS / TNS and the TNS
+ * backward (PAPER.md, "INSTA", DAC'25).
+ *
+ * TEST INFRASTRUCTURE, NOT PRODUCT.  Loaded only by tests/, by
+ * __graft_entry__.smoke() and by bench.py's cpu_baseline / --impl reference
+ * legs.  Shares nothing with the CUDA path.
+ *
+ * Notation follows the paper: arrival_mean (mu), arrival_std (sigma) and the
+ * corner arrival A = mu + N_sigma * sigma (Eq 1-3); arc delays are
+ * indexed by the sink transition rf (Alg 1 l.12-13); the source
+ * transition is ~rf for negative-unate arcs (Alg 1 l.8).  The merge is
+ * Alg 1/Alg 2 with K = 1 ("hard", strict ">" P:L97, L115) or the LSE operator
+ * (Eq 4) with softmax gradients (Eq 6).
+ *
+ * Parity status of each function (DESIGN.md §3 "pins"):
+ *   orc_levelize   pinned (networkx.topological_generations, invariants)
+ *   orc_forward    hard: pinned (brute-force max path for sigma==0; traced
+ *                  critical-path identity for sigma>0; hand-worked example)
+ *                  lse, sigma==0: pinned (tau*logsumexp over all paths)
+ *                  lse, sigma>0: PARITY UNPINNED w.r.t. paper intent (reading
+ *                  #1: sigma of the merged arrival = sigma of the arg-max;
+ *                  pinned only by limits tau->0 / sigma->0 and FD consistency)
+ *   orc_slack      pinned (closed forms)
+ *   orc_backward   pinned (central finite differences of orc_forward; path
+ *                  marginals for sigma==0 LSE; integer path counts in hard mode)
+ */
+#include "oracle.h"
+
+#include <math.h>
+#include <stdlib.h>
+#include <string.h>
+
+enum { RISE = 0, FALL = 1 };
+enum { U_POS = 0, U_NEG = 1, U_NON = 2 };
+
+/* ------------------------------------------------------------------------- */
+/* O1: validation (C ABI error rules)                           */
+/* ------------------------------------------------------------------------- */
+static int finite(double x) { return isfinite(x); }
+
+int orc_validate(const orc_graph* g, double n_sigma, double tau) {
+  if (!g || g->num_pins < 0 || g->num_arcs < 0 || g->num_endpoints < 0) return 1;
+  if (!finite(n_sigma) || n_sigma < 0 || !finite(tau) || tau < 0) return 1;
+  if (g->num_arcs > 0 && (!g->arc_from || !g->arc_to || !g->arc_unate || !g->arc_mean || !g->arc_sigma))
+    return 1;
+  for (int64_t e = 0; e < g->num_arcs; ++e) {
+    if (g->arc_from[e] < 0 || g->arc_from[e] >= g->num_pins) return 1;
+    if (g->arc_to[e] < 0 || g->arc_to[e] >= g->num_pins) return 1;
+    if (g->arc_unate[e] > U_NON) return 1;
+    for (int rf = 0; rf < 2; ++rf) {
+      if (!finite(g->arc_mean[2 * e + rf]) || !finite(g->arc_sigma[2 * e + rf])) return 1;
+      if (g->arc_sigma[2 * e + rf] < 0) return 1;
+    }
+  }
+  for (int64_t p = 0; p < 2 * (int64_t)g->num_pins; ++p) {
+    if (g->src_mean && !finite(g->src_mean[p])) return 1;
+    if (g->src_sigma && (!finite(g->src_sigma[p]) || g->src_sigma[p] < 0)) return 1;
+  }
+  if (g->num_endpoints > 0 && (!g->ep_pin || !g->ep_rat)) return 1;
+  char* seen = calloc((size_t)g->num_pins + 1, 1);
+  for (int32_t k = 0; k < g->num_endpoints; ++k) {
+    int32_t p = g->ep_pin[k];
+    if (p < 0 || p >= g->num_pins || seen[p]) { free(seen); return 1; }
+    seen[p] = 1;
+    if (!finite(g->ep_rat[2 * k]) || !finite(g->ep_rat[2 * k + 1])) { free(seen); return 1; }
+  }
+  free(seen);
+  return 0;
+}
+
+/* ------------------------------------------------------------------------- */
+/* O2: levelization by topological sort ("constructs and levelizes its  */
+/* timing graph ... pins within the same level are processed independently") */
+/* level(p) = 0 if indeg(p) = 0, else 1 + max level of its fanin sources.     */
+/* ------------------------------------------------------------------------- */
+typedef struct {
+  int32_t n, num_levels;
+  int64_t e;
+  int32_t *level, *order, *pos;         /* pos[p] = canonical position of pin p */
+  int32_t *fanin_ptr, *fanin_arc;       /* over canonical positions            */
+  int32_t *fanout_ptr, *fanout_arc;
+} topo_t;
+
+static void topo_free(topo_t* t) {
+  free(t->level); free(t->order); free(t->pos);
+  free(t->fanin_ptr); free(t->fanin_arc); free(t->fanout_ptr); free(t->fanout_arc);
+  memset(t, 0, sizeof *t);
+}
+
+/* returns 0 ok, 2 cycle */
+static int topo_build(int32_t n, int64_t E, const int32_t* from, const int32_t* to, topo_t* t) {
+  memset(t, 0, sizeof *t);
+  t->n = n; t->e = E;
+  t->level = calloc((size_t)n + 1, sizeof(int32_t));
+  t->order = calloc((size_t)n + 1, sizeof(int32_t));
+  t->pos = calloc((size_t)n + 1, sizeof(int32_t));
+  t->fanin_ptr = calloc((size_t)n + 1, sizeof(int32_t));
+  t->fanout_ptr = calloc((size_t)n + 1, sizeof(int32_t));
+  t->fanin_arc = calloc((size_t)E + 1, sizeof(int32_t));
+  t->fanout_arc = calloc((size_t)E + 1, sizeof(int32_t));
+
+  /* caller-indexed out-adjacency (arcs of each pin, ascending arc id) */
+  int32_t* out_ptr = calloc((size_t)n + 1, sizeof(int32_t));
+  int32_t* out_arc = calloc((size_t)E + 1, sizeof(int32_t));
+  int32_t* indeg = calloc((size_t)n + 1, sizeof(int32_t));
+  for (int64_t e = 0; e < E; ++e) { out_ptr[from[e] + 1]++; indeg[to[e]]++; }
+  for (int32_t p = 0; p < n; ++p) out_ptr[p + 1] += out_ptr[p];
+  int32_t* fill = calloc((size_t)n + 1, sizeof(int32_t));
+  for (int64_t e = 0; e < E; ++e) out_arc[out_ptr[from[e]] + fill[from[e]]++] = (int32_t)e;
+
+  /* Kahn's algorithm with explicit levels */
+  int32_t* queue = malloc(((size_t)n + 1) * sizeof(int32_t));
+  int32_t head = 0, tail = 0;
+  for (int32_t p = 0; p < n; ++p) if (indeg[p] == 0) { queue[tail++] = p; t->level[p] = 0; }
+  while (head < tail) {
+    int32_t p = queue[head++];
+    for (int32_t k = out_ptr[p]; k < out_ptr[p + 1]; ++k) {
+      int32_t q = to[out_arc[k]];
+      if (t->level[p] + 1 > t->level[q]) t->level[q] = t->level[p] + 1;
+      if (--indeg[q] == 0) queue[tail++] = q;
+    }
+  }
+  int cyc = (tail < n);
+  free(queue); free(indeg); free(fill); free(out_ptr); free(out_arc);
+  if (cyc) { topo_free(t); return 2; }
+
+  /* canonical order: pins sorted by (level, pin id) -- counting sort by level */
+  int32_t L = 0;
+  for (int32_t p = 0; p < n; ++p) if (t->level[p] + 1 > L) L = t->level[p] + 1;
+  t->num_levels = L;
+  int32_t* cnt = calloc((size_t)L + 1, sizeof(int32_t));
+  for (int32_t p = 0; p < n; ++p) cnt[t->level[p] + 1]++;
+  for (int32_t l = 0; l < L; ++l) cnt[l + 1] += cnt[l];
+  for (int32_t p = 0; p < n; ++p) { int32_t k = cnt[t->level[p]]++; t->order[k] = p; t->pos[p] = k; }
+  free(cnt);
+
+  /* fanin / fanout rows in canonical order, arcs ascending by caller arc id */
+  for (int64_t e = 0; e < E; ++e) { t->fanin_ptr[t->pos[to[e]] + 1]++; t->fanout_ptr[t->pos[from[e]] + 1]++; }
+  for (int32_t k = 0; k < n; ++k) { t->fanin_ptr[k + 1] += t->fanin_ptr[k]; t->fanout_ptr[k + 1] += t->fanout_ptr[k]; }
+  int32_t* fi = calloc((size_t)n + 1, sizeof(int32_t));
+  int32_t* fo = calloc((size_t)n + 1, sizeof(int32_t));
+  for (int64_t e = 0; e < E; ++e) {
+    int32_t a = t->pos[to[e]], b = t->pos[from[e]];
+    t->fanin_arc[t->fanin_ptr[a] + fi[a]++] = (int32_t)e;
+    t->fanout_arc[t->fanout_ptr[b] + fo[b]++] = (int32_t)e;
+  }
+  free(fi); free(fo);
+  return 0;
+}
+
+int orc_levelize(int32_t num_pins, int64_t num_arcs, const int32_t* arc_from,
+                 const int32_t* arc_to, int32_t* level, int32_t* order,
+                 int32_t* fanin_ptr, int32_t* fanin_arc, int32_t* fanout_ptr,
+                 int32_t* fanout_arc, int32_t* num_levels) {
+  if (num_pins < 0 || num_arcs < 0 || num_arcs >= ((int64_t)1 << 31)) return 1;
+  for (int64_t e = 0; e < num_arcs; ++e)
+    if (arc_from[e] < 0 || arc_from[e] >= num_pins || arc_to[e] < 0 || arc_to[e] >= num_pins) return 1;
+  topo_t t;
+  int st = topo_build(num_pins, num_arcs, arc_from, arc_to, &t);
+  if (st) return st;
+  if (level) memcpy(level, t.level, sizeof(int32_t) * (size_t)num_pins);
+  if (order) memcpy(order, t.order, sizeof(int32_t) * (size_t)num_pins);
+  if (fanin_ptr) memcpy(fanin_ptr, t.fanin_ptr, sizeof(int32_t) * ((size_t)num_pins + 1));
+  if (fanout_ptr) memcpy(fanout_ptr, t.fanout_ptr, sizeof(int32_t) * ((size_t)num_pins + 1));
+  if (fanin_arc) memcpy(fanin_arc, t.fanin_arc, sizeof(int32_t) * (size_t)num_arcs);
+  if (fanout_arc) memcpy(fanout_arc, t.fanout_arc, sizeof(int32_t) * (size_t)num_arcs);
+  if (num_levels) *num_levels = t.num_levels;
+  topo_free(&t);
+  return 0;
+}
+
+/* ------------------------------------------------------------------------- */
+/* O4: candidates of (pin i, sink transition rf)                              */
+/* For each fanin arc e = (j -> i) in row order and each source transition    */
+/* s in S(rf, U[e]) -- POS: {rf}; NEG: {~rf} (Alg 1 l.8); NON: (rf, ~rf):      */
+/*   mean  mu_c  = mu_j[s] + arc_mean[e][rf]                 (Eq 1, Alg 1 l.12) */
+/*   std   sig_c = sqrt(sig_j[s]^2 + arc_std[e][rf]^2)       (Eq 2, Alg 1 l.13) */
+/*   arrival A_c = mu_c + N_sigma * sig_c                    (Eq 3, Alg 1 l.14) */
+/* ------------------------------------------------------------------------- */
+typedef struct { int32_t arc, src; int s; double mu, sig, A; } cand_t;
+
+static int sources_of(int rf, int unate, int* s_out) {
+  if (unate == U_POS) { s_out[0] = rf; return 1; }
+  if (unate == U_NEG) { s_out[0] = 1 - rf; return 1; }
+  s_out[0] = rf; s_out[1] = 1 - rf; return 2;
+}
+
+static int candidates(const orc_graph* g, const topo_t* t, int32_t k /*canonical pos*/, int rf,
+                      double n_sigma, const double* mu, const double* sig, cand_t* c) {
+  int n = 0;
+  for (int32_t q = t->fanin_ptr[k]; q < t->fanin_ptr[k + 1]; ++q) {
+    int32_t e = t->fanin_arc[q];
+    int32_t j = g->arc_from[e];
+    int ss[2];
+    int ns = sources_of(rf, g->arc_unate[e], ss);
+    for (int a = 0; a < ns; ++a) {
+      int s = ss[a];
+      double arc_mean = g->arc_mean[2 * (int64_t)e + rf];
+      double arc_std = g->arc_sigma[2 * (int64_t)e + rf];
+      c[n].arc = e; c[n].src = j; c[n].s = s;
+      c[n].mu = mu[2 * (int64_t)j + s] + arc_mean;
+      c[n].sig = sqrt(sig[2 * (int64_t)j + s] * sig[2 * (int64_t)j + s] + arc_std * arc_std);
+      c[n].A = c[n].mu + n_sigma * c[n].sig;
+      ++n;
+    }
+  }
+  return n;
+}
+
+/* first arg-max: a later candidate replaces only if strictly greater (Alg 2 l.4) */
+static int first_argmax(const cand_t* c, int n) {
+  int best = 0;
+  for (int a = 1; a < n; ++a) if (c[a].A > c[best].A) best = a;
+  return best;
+}
+
+static int max_fanin(const topo_t* t) {
+  int m = 1;
+  for (int32_t k = 0; k < t->n; ++k) {
+    int d = t->fanin_ptr[k + 1] - t->fanin_ptr[k];
+    if (d > m) m = d;
+  }
+  return m;
+}
+
+/* O3 + O4 + O5 over the whole graph; mu/sig are the per-pin state (Eq 1-2). */
+static void propagate(const orc_graph* g, const topo_t* t, double n_sigma, double tau,
+                      double* mu, double* sig, int32_t* win_arc, int8_t* win_s, double* gap) {
+  cand_t* c = malloc(sizeof(cand_t) * 2 * (size_t)max_fanin(t));
+  for (int32_t k = 0; k < t->n; ++k) {
+    int32_t i = t->order[k];
+    if (t->fanin_ptr[k] == t->fanin_ptr[k + 1]) {
+      /* O3: startpoint -- clock arrival distribution, corner via Eq 3 */
+      for (int rf = 0; rf < 2; ++rf) {
+        mu[2 * (int64_t)i + rf] = g->src_mean ? g->src_mean[2 * (int64_t)i + rf] : 0.0;
+        sig[2 * (int64_t)i + rf] = g->src_sigma ? g->src_sigma[2 * (int64_t)i + rf] : 0.0;
+        if (win_arc) win_arc[2 * (int64_t)i + rf] = -1;
+        if (win_s) win_s[2 * (int64_t)i + rf] = -1;
+        if (gap) gap[2 * (int64_t)i + rf] = INFINITY;
+      }
+      continue;
+    }
+    for (int rf = 0; rf < 2; ++rf) {
+      int n = candidates(g, t, k, rf, n_sigma, mu, sig, c);
+      int b = first_argmax(c, n);
+      if (tau == 0.0) {
+        /* hard: Alg 1 + Alg 2 with K = 1 -- keep the distribution of the max */
+        mu[2 * (int64_t)i + rf] = c[b].mu;
+        sig[2 * (int64_t)i + rf] = c[b].sig;
+      } else {
+        /* LSE (Eq 4): A_i = M + tau * log(sum exp((A_c - M)/tau)), M = max.
+         * Reading #1: sigma_i = sigma of the arg-max; mu_i = A_i - N_sigma*sigma_i. */
+        double M = c[b].A, sum = 0.0;
+        for (int a = 0; a < n; ++a) sum += exp((c[a].A - M) / tau);
+        double A_i = M + tau * log(sum);
+        sig[2 * (int64_t)i + rf] = c[b].sig;
+        mu[2 * (int64_t)i + rf] = A_i - n_sigma * c[b].sig;
+      }
+      if (win_arc) win_arc[2 * (int64_t)i + rf] = c[b].arc;
+      if (win_s) win_s[2 * (int64_t)i + rf] = (int8_t)c[b].s;
+      if (gap) {
+        double second = -INFINITY;
+        for (int a = 0; a < n; ++a) if (a != b && c[a].A > second) second = c[a].A;
+        gap[2 * (int64_t)i + rf] = (n > 1) ? c[b].A - second : INFINITY;
+      }
+    }
+  }
+  free(c);
+}
+
+int orc_forward(const orc_graph* g, double n_sigma, double tau, double* A,
+                double* sig, double* mu, int32_t* win_arc, int8_t* win_s,
+                double* gap) {
+  int st = orc_validate(g, n_sigma, tau);
+  if (st) return st;
+  topo_t t;
+  st = topo_build(g->num_pins, g->num_arcs, g->arc_from, g->arc_to, &t);
+  if (st) return st;
+  size_t n2 = 2 * (size_t)g->num_pins + 2;
+  double* m = malloc(n2 * sizeof(double));
+  double* s = malloc(n2 * sizeof(double));
+  propagate(g, &t, n_sigma, tau, m, s, win_arc, win_s, gap);
+  for (int64_t p = 0; p < 2 * (int64_t)g->num_pins; ++p) {
+    if (A) A[p] = m[p] + n_sigma * s[p];           /* Eq 3: the corner arrival */
+    if (mu) mu[p] = m[p];
+    if (sig) sig[p] = s[p];
+  }
+  free(m); free(s);
+  topo_free(&t);
+  return 0;
+}
+
+/* ------------------------------------------------------------------------- */
+/* O6: endpoint slack = RAT - A (setup), min over rf (tie -> R);              */
+/* TNS = sum of min(0, slack) in endpoint order, WNS = min(0, min slack),     */
+/* violations = #{slack < 0} (Table II signs P:L216-227).  */
+/* ------------------------------------------------------------------------- */
+int orc_slack(const orc_graph* g, const double* A, double* slack,
+              uint8_t* rf_star, double* wns, double* tns, int32_t* num_viol) {
+  double w = 0.0, t = 0.0;
+  int32_t nv = 0;
+  for (int32_t k = 0; k < g->num_endpoints; ++k) {
+    int32_t p = g->ep_pin[k];
+    double sr = g->ep_rat[2 * k + RISE] - A[2 * (int64_t)p + RISE];
+    double sf = g->ep_rat[2 * k + FALL] - A[2 * (int64_t)p + FALL];
+    int r = (sf < sr) ? FALL : RISE;
+    double s = (r == FALL) ? sf : sr;
+    if (slack) slack[k] = s;
+    if (rf_star) rf_star[k] = (uint8_t)r;
+    if (s < 0) { t += s; ++nv; }
+    if (s < w) w = s;
+  }
+  if (wns) *wns = w;
+  if (tns) *tns = t;
+  if (num_viol) *num_viol = nv;
+  return 0;
+}
+
+/* ------------------------------------------------------------------------- */
+/* O7: backward, push style in reverse canonical order.          */
+/* State adjoints per pin/rf: mbar = dL/dmu, sbar = dL/dsigma.                */
+/* Merge (Eq 4/6): A_i = LSE(A_c), w_c = exp((A_c - M)/tau) / sum (Eq 6);     */
+/* hard mode is w = one-hot(c*).  With mu_i = A_i - Ns*sig_{c*} and           */
+/* sig_i = sig_{c*}:                                                          */
+/*   Abar_c   = w_c * mbar_i                                                  */
+/*   mbar_c   = Abar_c                                                        */
+/*   sbar_c   = Ns*Abar_c + [c = c*]*(sbar_i - Ns*mbar_i)                     */
+/* Candidate (Eq 1-2): mbar_j[s] += mbar_c, dmean_e[rf] += mbar_c,            */
+/*   sbar_j[s] += sbar_c*sig_j[s]/sig_c, dsigma_e[rf] += sbar_c*sig_e/sig_c   */
+/*   (0/0 := 0).                                                              */
+/* ------------------------------------------------------------------------- */
+int orc_backward(const orc_graph* g, double n_sigma, double tau,
+                 const double* dslack, double* d_mean, double* d_sigma,
+                 double* d_src_mean, double* d_src_sigma, double* abar) {
+  int st = orc_validate(g, n_sigma, tau);
+  if (st) return st;
+  topo_t t;
+  st = topo_build(g->num_pins, g->num_arcs, g->arc_from, g->arc_to, &t);
+  if (st) return st;
+  int32_t N = g->num_pins;
+  int64_t E = g->num_arcs;
+  size_t n2 = 2 * (size_t)N + 2;
+  double* mu = malloc(n2 * sizeof(double));
+  double* sig = malloc(n2 * sizeof(double));
+  propagate(g, &t, n_sigma, tau, mu, sig, NULL, NULL, NULL);
+
+  double* mbar = calloc(n2, sizeof(double));
+  double* sbar = calloc(n2, sizeof(double));
+  double* dm = calloc(2 * (size_t)E + 2, sizeof(double));
+  double* ds = calloc(2 * (size_t)E + 2, sizeof(double));
+
+  /* seeds: slack = RAT - (mu + Ns*sig) at rf*, so dL/dmu = -dslack, dL/dsig = -Ns*dslack */
+  for (int32_t k = 0; k < g->num_endpoints; ++k) {
+    int32_t p = g->ep_pin[k];
+    double sr = g->ep_rat[2 * k + RISE] - (mu[2 * (int64_t)p + RISE] + n_sigma * sig[2 * (int64_t)p + RISE]);
+    double sf = g->ep_rat[2 * k + FALL] - (mu[2 * (int64_t)p + FALL] + n_sigma * sig[2 * (int64_t)p + FALL]);
+    int r = (sf < sr) ? FALL : RISE;
+    double s = (r == FALL) ? sf : sr;
+    double seed = dslack ? dslack[k] : (s < 0 ? 1.0 : 0.0);
+    mbar[2 * (int64_t)p + r] += -seed;
+    sbar[2 * (int64_t)p + r] += -n_sigma * seed;
+  }
+
+  cand_t* c = malloc(sizeof(cand_t) * 2 * (size_t)max_fanin(&t));
+  double* w = malloc(sizeof(double) * 2 * (size_t)max_fanin(&t));
+  for (int32_t k = N - 1; k >= 0; --k) {
+    int32_t i = t.order[k];
+    if (t.fanin_ptr[k] == t.fanin_ptr[k + 1]) continue;
+    for (int rf = 0; rf < 2; ++rf) {
+      double mb = mbar[2 * (int64_t)i + rf], sb = sbar[2 * (int64_t)i + rf];
+      if (mb == 0.0 && sb == 0.0) continue;
+      int n = candidates(g, &t, k, rf, n_sigma, mu, sig, c);
+      int b = first_argmax(c, n);
+      if (tau == 0.0) {
+        for (int a = 0; a < n; ++a) w[a] = (a == b) ? 1.0 : 0.0;
+      } else {
+        double M = c[b].A, sum = 0.0;
+        for (int a = 0; a < n; ++a) sum += exp((c[a].A - M) / tau);
+        for (int a = 0; a < n; ++a) w[a] = exp((c[a].A - M) / tau) / sum;   /* Eq 6 */
+      }
+      for (int a = 0; a < n; ++a) {
+        double Abar_c = w[a] * mb;
+        double mbar_c = Abar_c;
+        double sbar_c = n_sigma * Abar_c + ((a == b) ? (sb - n_sigma * mb) : 0.0);
+        int64_t e = c[a].arc;
+        int32_t j = c[a].src;
+        int s = c[a].s;
+        double sig_j = sig[2 * (int64_t)j + s];
+        double sig_e = g->arc_sigma[2 * e + rf];
+        mbar[2 * (int64_t)j + s] += mbar_c;
+        dm[2 * e + rf] += mbar_c;
+        if (c[a].sig > 0.0) {
+          sbar[2 * (int64_t)j + s] += sbar_c * sig_j / c[a].sig;
+          ds[2 * e + rf] += sbar_c * sig_e / c[a].sig;
+        }
+      }
+    }
+  }
+  free(c); free(w);
+
+  if (d_mean) memcpy(d_mean, dm, sizeof(double) * 2 * (size_t)E);
+  if (d_sigma) memcpy(d_sigma, ds, sizeof(double) * 2 * (size_t)E);
+  for (int32_t p = 0; p < N; ++p) {
+    int is_src = (t.fanin_ptr[t.pos[p]] == t.fanin_ptr[t.pos[p] + 1]);
+    for (int rf = 0; rf < 2; ++rf) {
+      if (d_src_mean) d_src_mean[2 * (int64_t)p + rf] = is_src ? mbar[2 * (int64_t)p + rf] : 0.0;
+      if (d_src_sigma) d_src_sigma[2 * (int64_t)p + rf] = is_src ? sbar[2 * (int64_t)p + rf] : 0.0;
+      if (abar) abar[2 * (int64_t)p + rf] = mbar[2 * (int64_t)p + rf];
+    }
+  }
+  free(mu); free(sig); free(mbar); free(sbar); free(dm); free(ds);
+  topo_free(&t);
+  return 0;
+}
+
+/* ------------------------------------------------------------------------- */
+/* Test support: near-tie taint (hard mode).  Not part of the method.         */
+/* ------------------------------------------------------------------------- */
+int orc_tie_taint(const orc_graph* g, double n_sigma, double eps, double margin,
+                  uint8_t* fwd_taint, uint8_t* arc_taint) {
+  int st = orc_validate(g, n_sigma, 0.0);
+  if (st) return st;
+  topo_t t;
+  st = topo_build(g->num_pins, g->num_arcs, g->arc_from, g->arc_to, &t);
+  if (st) return st;
+  int32_t N = g->num_pins;
+  int64_t E = g->num_arcs;
+  size_t n2 = 2 * (size_t)N + 2;
+  double* mu = malloc(n2 * sizeof(double));
+  double* sig = malloc(n2 * sizeof(double));
+  propagate(g, &t, n_sigma, 0.0, mu, sig, NULL, NULL, NULL);
+  uint8_t* ft = calloc(n2, 1);
+  uint8_t* bt = calloc(n2, 1);     /* backward: adjoint of (pin, rf) uncertain */
+  uint8_t* at = calloc(2 * (size_t)E + 2, 1);
+  cand_t* c = malloc(sizeof(cand_t) * 2 * (size_t)max_fanin(&t));
+
+  /* forward taint: near tie at the merge, or a near-max candidate from a tainted source */
+  for (int32_t k = 0; k < N; ++k) {
+    int32_t i = t.order[k];
+    if (t.fanin_ptr[k] == t.fanin_ptr[k + 1]) continue;
+    for (int rf = 0; rf < 2; ++rf) {
+      int n = candidates(g, &t, k, rf, n_sigma, mu, sig, c);
+      int b = first_argmax(c, n);
+      uint8_t x = 0;
+      for (int a = 0; a < n; ++a) {
+        if (a != b && c[b].A - c[a].A <= eps) x = 1;
+        if (c[b].A - c[a].A <= margin && ft[2 * (int64_t)c[a].src + c[a].s]) x = 1;
+      }
+      ft[2 * (int64_t)i + rf] = x;
+    }
+  }
+  /* backward taint originates at endpoints with ambiguous seeds or tainted state */
+  for (int32_t k = 0; k < g->num_endpoints; ++k) {
+    int32_t p = g->ep_pin[k];
+    double ar = mu[2 * (int64_t)p] + n_sigma * sig[2 * (int64_t)p];
+    double af = mu[2 * (int64_t)p + 1] + n_sigma * sig[2 * (int64_t)p + 1];
+    double sr = g->ep_rat[2 * k] - ar, sf = g->ep_rat[2 * k + 1] - af;
+    double s = sf < sr ? sf : sr;
+    if (fabs(sr - sf) <= eps || fabs(s) <= eps || ft[2 * (int64_t)p] || ft[2 * (int64_t)p + 1]) {
+      bt[2 * (int64_t)p] = bt[2 * (int64_t)p + 1] = 1;
+    }
+  }
+  /* reverse: where the oracle (or an uncertain upstream) routes adjoint, an
+   * ambiguous merge taints every candidate within `margin` of the max, and an
+   * unambiguous merge with an uncertain adjoint taints only its winner. */
+  double* mb = malloc(n2 * sizeof(double));
+  orc_backward(g, n_sigma, 0.0, NULL, NULL, NULL, NULL, NULL, mb);
+  for (int32_t k = N - 1; k >= 0; --k) {
+    int32_t i = t.order[k];
+    if (t.fanin_ptr[k] == t.fanin_ptr[k + 1]) continue;
+    for (int rf = 0; rf < 2; ++rf) {
+      int64_t q = 2 * (int64_t)i + rf;
+      if (!(bt[q] || mb[q] != 0.0)) continue;
+      int n = candidates(g, &t, k, rf, n_sigma, mu, sig, c);
+      int b = first_argmax(c, n);
+      int amb = ft[q];
+      for (int a = 0; a < n; ++a) if (a != b && c[b].A - c[a].A <= eps) amb = 1;
+      for (int a = 0; a < n; ++a) {
+        int hit = amb ? (c[b].A - c[a].A <= margin) : (bt[q] && a == b);
+        if (hit) {
+          bt[2 * (int64_t)c[a].src + c[a].s] = 1;
+          at[2 * (int64_t)c[a].arc + rf] = 1;
+        }
+      }
+    }
+  }
+  free(mb);
+  if (fwd_taint) memcpy(fwd_taint, ft, 2 * (size_t)N);
+  if (arc_taint) memcpy(arc_taint, at, 2 * (size_t)E);
+  free(c); free(ft); free(bt); free(at); free(mu); free(sig);
+  topo_free(&t);
+  return 0;
+}
