@@ -1,0 +1,179 @@
+/*
+ * insta.h -- C ABI of the B200-native INSTA hot path (libinsta.so).
+ *
+ * INSTA (Lu et al., DAC'25; /root/reference/PAPER.md, cited P:Lnn) propagates
+ * statistical (POCV) arrival times level by level over a timing graph whose arc
+ * delays are already known, ends in endpoint slack and WNS/TNS, and returns
+ * timing gradients dTNS/d(arc delay) through a backward pass.  This header is
+ * the boundary: plain C types, plain pointers (host or device as stated), no
+ * C++ types, no exceptions.  Every entry point returns an insta_status; on a
+ * non-OK status insta_last_error() returns a thread-local message.
+ *
+ * Conventions (all entry points)
+ *  - Pin ids 0..num_pins-1 and arc ids 0..num_arcs-1 are CALLER ids; the
+ *    internal level-ordered permutation is hidden except via insta_graph_export.
+ *  - rf index 0 = rise (R), 1 = fall (F).  "[n][2]" arrays are row-major
+ *    {R, F} pairs of float32 (ps).
+ *  - Arc delays are indexed by the SINK transition (Alg 1 l.12-13); the
+ *    source transition is ~rf for negative-unate arcs (Alg 1 l.8) and
+ *    both transitions for non-unate arcs (reading R3).
+ *  - Device pointers are caller-owned device memory on the graph's device
+ *    (e.g. torch tensor data_ptr()); the library never keeps a caller pointer
+ *    past the call.  All device work is enqueued on the caller's stream
+ *    (cudaStream_t passed as void*; NULL = legacy default stream).  Only
+ *    insta_graph_create / destroy / export / levelize synchronize implicitly;
+ *    passing a non-NULL insta_summary* also synchronizes the stream.
+ *  - One graph must not be used from two host threads at once.
+ *  - Errors: INSTA_E_ARG (bad id, NaN/Inf, sigma < 0, duplicate endpoint,
+ *    tau < 0, n_sigma < 0, NULL required pointer, size limits: num_pins < 2^29,
+ *    num_arcs < 2^31), INSTA_E_CYCLE (combinational loop), INSTA_E_STATE (call
+ *    out of order, e.g. backward before forward), INSTA_E_CUDA / INSTA_E_NOMEM
+ *    (runtime failures; the graph is then unusable and must be destroyed).
+ */
+#ifndef INSTA_H
+#define INSTA_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct insta_graph insta_graph; /* opaque; owns all of its device memory */
+
+typedef enum {
+  INSTA_OK = 0,
+  INSTA_E_ARG = 1,
+  INSTA_E_CYCLE = 2,
+  INSTA_E_CUDA = 3,
+  INSTA_E_NOMEM = 4,
+  INSTA_E_STATE = 5
+} insta_status;
+
+typedef enum { INSTA_POS = 0, INSTA_NEG = 1, INSTA_NON = 2 } insta_unate;
+
+/* Graph description (all HOST pointers; copied by insta_graph_create).
+ * Inputs are the paper's "arc attributes in consideration of rise/fall
+ * conditions and unateness ... SP/EP attributes (clock arrival times, minimum
+ * required times)". */
+typedef struct {
+  int32_t num_pins;
+  int64_t num_arcs;
+  const int32_t* arc_from;   /* [num_arcs] driver pin of each arc                        */
+  const int32_t* arc_to;     /* [num_arcs] sink pin of each arc                          */
+  const uint8_t* arc_unate;  /* [num_arcs] insta_unate                                   */
+  const float* arc_mean;     /* [num_arcs][2] arc delay mean per SINK transition (Eq 1)  */
+  const float* arc_sigma;    /* [num_arcs][2] arc delay std per SINK transition (Eq 2), >=0 */
+  const float* src_mean;     /* [num_pins][2] or NULL(=0): arrival mean at indeg-0 pins  */
+  const float* src_sigma;    /* [num_pins][2] or NULL(=0): arrival std at indeg-0 pins   */
+  int32_t num_endpoints;
+  const int32_t* ep_pin;     /* [num_endpoints] unique endpoint pins                     */
+  const float* ep_rat;       /* [num_endpoints][2] required arrival time per rf          */
+  const uint8_t* arc_class;  /* [num_arcs] 0 = net arc, 1 = cell arc, or NULL (all net);
+                                used only by scenario derates (insta_forward_batch)       */
+  int32_t device;            /* CUDA device ordinal                                      */
+} insta_graph_desc;
+
+/* Forward options.  n_sigma: the pessimism level of Eq 3 (3.0 in the
+ * paper).  tau: 0 selects the paper's hard max (Alg 1/Alg 2 with Top-K = 1,
+ * strict ">" P:L97); tau > 0 selects the LSE smooth max of Eq 4 with
+ * Eq 6 gradients.  schedule: 0 = persistent dataflow kernel (default),
+ * 1 = one launch per timing level (the paper's launch structure). */
+typedef struct {
+  float n_sigma;
+  float tau;
+  int32_t want_grad_sigma; /* reserved; must be 0 in this version */
+  int32_t schedule;
+} insta_opts;
+
+/* Global timing metrics: WNS = min(0, min slack),
+ * TNS = sum of min(0, slack) accumulated in fp64 in endpoint order. */
+typedef struct {
+  double wns;
+  double tns;
+  int32_t num_violations; /* #endpoints with slack < 0 (strict) */
+  int32_t num_levels;
+} insta_summary;
+
+/* Host-only levelization (no device needed): the "topological sort" of P:L62.
+ * level(p) = 0 for indeg-0 pins, else 1 + max level of its fanin sources.
+ * Outputs (HOST buffers, any may be NULL): level_of_pin[num_pins];
+ * order[num_pins] = caller pin at each canonical position, pins sorted by
+ * (level, pin id); fanin_ptr/fanout_ptr[num_pins+1] over canonical positions;
+ * fanin_arc/fanout_arc[num_arcs] caller arc ids, ascending within each row;
+ * *num_levels.  INSTA_E_CYCLE on a combinational loop. */
+insta_status insta_levelize(int32_t num_pins, int64_t num_arcs, const int32_t* arc_from,
+                            const int32_t* arc_to, int32_t* level_of_pin, int32_t* order,
+                            int32_t* fanin_ptr, int32_t* fanin_arc, int32_t* fanout_ptr,
+                            int32_t* fanout_arc, int32_t* num_levels);
+
+/* Validate, copy, levelize (host) and upload a graph; synchronous.  On success
+ * *out owns every device buffer until insta_graph_destroy. */
+insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out);
+void insta_graph_destroy(insta_graph* g);
+
+/* Copy the graph's levelization to HOST buffers (same layout as
+ * insta_levelize; any may be NULL); synchronous.  For bit-exact tests. */
+insta_status insta_graph_export(const insta_graph* g, int32_t* level_of_pin, int32_t* order,
+                                int32_t* fanin_ptr, int32_t* fanin_arc, int32_t* fanout_ptr,
+                                int32_t* fanout_arc);
+
+/* Sizes of a created graph (host). */
+insta_status insta_graph_sizes(const insta_graph* g, int32_t* num_pins, int64_t* num_arcs,
+                               int32_t* num_endpoints, int32_t* num_levels);
+
+/* Forward: statistical arrival propagation (Eq 1-3, Alg 1 with K = 1, or
+ * Eq 4) over all levels, then endpoint slack = RAT - A, min over rf (ties ->
+ * R), and WNS/TNS.  o may be NULL (defaults n_sigma 3, tau 0, schedule 0).
+ * out: NULL = asynchronous; non-NULL = synchronize and fill. */
+insta_status insta_forward(insta_graph* g, const insta_opts* o, void* cuda_stream,
+                           insta_summary* out);
+
+/* Copy the last forward's endpoint slack (DEVICE float[num_endpoints], caller
+ * endpoint order) and optionally rf_star (DEVICE uint8[num_endpoints], the rf
+ * attaining the min) and the summary (forces a sync).  Any may be NULL.
+ * INSTA_E_STATE if no forward since creation or since insta_update_arcs. */
+insta_status insta_slack(insta_graph* g, float* slack, uint8_t* rf_star, void* cuda_stream,
+                         insta_summary* out);
+
+/* Copy the last forward's per-pin arrival state in caller pin order (DEVICE
+ * buffers [num_pins][2], any may be NULL): corner arrival A = mu + n_sigma*sigma
+ * (Eq 3), mean mu (Eq 1) and std sigma (Eq 2). */
+insta_status insta_arrivals(insta_graph* g, float* A, float* mean, float* sigma,
+                            void* cuda_stream);
+
+/* Backward: timing gradients of L w.r.t. every arc delay mean,
+ * chaining the Eq 6 softmax weights (hard mode: one-hot at the first arg-max)
+ * in reverse level order.  ep_seed: DEVICE float[num_endpoints] dL/dslack, or
+ * NULL for L = TNS (seed 1 where slack < 0).  d_arc_mean: DEVICE
+ * float[num_arcs][2] in caller arc order, overwritten (required).
+ * d_arc_sigma must be NULL in this version.  d_src: DEVICE float[num_pins][2]
+ * dL/d(src_mean) in caller pin order (0 at non-source pins), or NULL.
+ * Uses the tau/n_sigma of the last forward.  INSTA_E_STATE if the last
+ * forward is stale. */
+insta_status insta_backward(insta_graph* g, const float* ep_seed, float* d_arc_mean,
+                            float* d_arc_sigma, float* d_src, void* cuda_stream);
+
+/* Re-annotate n arcs ("re-annotate ... then re-propagate"):
+ * arc_ids DEVICE int32[n] (caller ids, unique), mean/sigma DEVICE float[n][2].
+ * incremental = 1: the next insta_forward re-propagates only the fanout cone
+ * of the changed arcs (same per-pin arithmetic, so results are bit-identical
+ * to a full forward); 0: the next forward is a full one.  Invalid ids or
+ * values are not checked on the device (caller contract). */
+insta_status insta_update_arcs(insta_graph* g, int64_t n, const int32_t* arc_ids,
+                               const float* mean, const float* sigma, int32_t incremental,
+                               void* cuda_stream);
+
+/* Statistics of the last forward: number of pins recomputed (== num_pins for a
+ * full forward; the cone size for an incremental one).  Synchronizes. */
+insta_status insta_last_forward_stats(insta_graph* g, int64_t* pins_recomputed);
+
+/* Thread-local message for the last non-OK status ("" if none). */
+const char* insta_last_error(void);
+
+/* Library version string. */
+const char* insta_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* INSTA_H */

@@ -1,0 +1,194 @@
+"""B200-native INSTA hot path: Python binding over the C ABI (include/insta.h).
+
+Argument marshalling only -- every step of the path runs in libinsta.so's
+CUDA kernels.  torch supplies device memory and streams.
+
+    g = Graph(desc)                      # validate + levelize + upload
+    s = g.forward(n_sigma=3.0, tau=0.0)  # arrivals -> slack -> WNS/TNS
+    d_mean = g.backward()                # dTNS/d(arc mean), caller arc order
+"""
+from __future__ import annotations
+
+import ctypes
+import dataclasses
+
+import numpy as np
+
+from . import _capi
+from ._capi import InstaError, check
+
+__all__ = ["Graph", "Summary", "InstaError", "levelize", "version"]
+
+
+@dataclasses.dataclass
+class Summary:
+    wns: float
+    tns: float
+    num_violations: int
+    num_levels: int
+
+
+def version() -> str:
+    return _capi.load().insta_version().decode()
+
+
+def _np(a, dtype, shape=None):
+    a = np.ascontiguousarray(a, dtype=dtype)
+    if shape is not None:
+        a = a.reshape(shape)
+    return a
+
+
+def _ptr(a):
+    return None if a is None else a.ctypes.data
+
+
+def levelize(num_pins: int, arc_from, arc_to) -> dict:
+    """Host-only levelization through the C ABI (insta_levelize)."""
+    lib = _capi.load()
+    af = _np(arc_from, np.int32)
+    at = _np(arc_to, np.int32)
+    N, E = int(num_pins), int(af.shape[0])
+    out = dict(level=np.zeros(N, np.int32), order=np.zeros(N, np.int32),
+               fanin_ptr=np.zeros(N + 1, np.int32), fanin_arc=np.zeros(E, np.int32),
+               fanout_ptr=np.zeros(N + 1, np.int32), fanout_arc=np.zeros(E, np.int32))
+    nl = ctypes.c_int32(0)
+    check(lib.insta_levelize(N, E, _ptr(af), _ptr(at), _ptr(out["level"]), _ptr(out["order"]),
+                             _ptr(out["fanin_ptr"]), _ptr(out["fanin_arc"]), _ptr(out["fanout_ptr"]),
+                             _ptr(out["fanout_arc"]), ctypes.byref(nl)), "insta_levelize")
+    out["num_levels"] = int(nl.value)
+    return out
+
+
+def _stream(torch, device):
+    return ctypes.c_void_p(torch.cuda.current_stream(device).cuda_stream)
+
+
+def _dptr(t):
+    return None if t is None else ctypes.c_void_p(t.data_ptr())
+
+
+class Graph:
+    """A timing graph resident on one GPU (opaque insta_graph)."""
+
+    def __init__(self, g, device: int = 0):
+        import torch  # plumbing only: device memory + streams
+        self._torch = torch
+        self.lib = _capi.load()
+        self.device = torch.device("cuda", device)
+        self.num_pins = int(g.num_pins)
+        self._arrs = dict(
+            arc_from=_np(g.arc_from, np.int32), arc_to=_np(g.arc_to, np.int32),
+            arc_unate=_np(g.arc_unate, np.uint8),
+            arc_mean=_np(g.arc_mean, np.float32), arc_sigma=_np(g.arc_sigma, np.float32),
+            src_mean=None if getattr(g, "src_mean", None) is None else _np(g.src_mean, np.float32),
+            src_sigma=None if getattr(g, "src_sigma", None) is None else _np(g.src_sigma, np.float32),
+            ep_pin=_np(g.ep_pin, np.int32), ep_rat=_np(g.ep_rat, np.float32),
+            arc_class=None if getattr(g, "arc_class", None) is None else _np(g.arc_class, np.uint8))
+        a = self._arrs
+        self.num_arcs = int(a["arc_from"].shape[0])
+        self.num_endpoints = int(a["ep_pin"].shape[0])
+        desc = _capi.insta_graph_desc(
+            self.num_pins, self.num_arcs, _ptr(a["arc_from"]), _ptr(a["arc_to"]), _ptr(a["arc_unate"]),
+            _ptr(a["arc_mean"]), _ptr(a["arc_sigma"]), _ptr(a["src_mean"]), _ptr(a["src_sigma"]),
+            self.num_endpoints, _ptr(a["ep_pin"]), _ptr(a["ep_rat"]), _ptr(a["arc_class"]), int(device))
+        h = ctypes.c_void_p()
+        check(self.lib.insta_graph_create(ctypes.byref(desc), ctypes.byref(h)), "insta_graph_create")
+        self._h = h
+        self._arrs = None   # the library copied everything
+        nl = ctypes.c_int32()
+        check(self.lib.insta_graph_sizes(self._h, None, None, None, ctypes.byref(nl)), "insta_graph_sizes")
+        self.num_levels = int(nl.value)
+
+    # ------------------------------------------------------------------ lifetime
+    def close(self):
+        if getattr(self, "_h", None):
+            self.lib.insta_graph_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    # ------------------------------------------------------------------ calls
+    def _st(self, stream=None):
+        if stream is not None:
+            return ctypes.c_void_p(stream.cuda_stream)
+        return _stream(self._torch, self.device)
+
+    def forward(self, n_sigma: float = 3.0, tau: float = 0.0, schedule: int = 0, sync: bool = True,
+                stream=None):
+        """insta_forward: arrivals -> endpoint slack -> WNS/TNS.  Returns a Summary if sync."""
+        opts = _capi.insta_opts(float(n_sigma), float(tau), 0, int(schedule))
+        out = _capi.insta_summary() if sync else None
+        check(self.lib.insta_forward(self._h, ctypes.byref(opts), self._st(stream),
+                                     ctypes.byref(out) if out is not None else None), "insta_forward")
+        if out is None:
+            return None
+        return Summary(out.wns, out.tns, out.num_violations, out.num_levels)
+
+    def slack(self, stream=None):
+        """insta_slack: (slack float32[P], rf_star uint8[P]) device tensors, caller endpoint order."""
+        t = self._torch
+        s = t.empty(self.num_endpoints, dtype=t.float32, device=self.device)
+        r = t.empty(self.num_endpoints, dtype=t.uint8, device=self.device)
+        check(self.lib.insta_slack(self._h, _dptr(s), _dptr(r), self._st(stream), None), "insta_slack")
+        return s, r
+
+    def summary(self, stream=None) -> Summary:
+        out = _capi.insta_summary()
+        check(self.lib.insta_slack(self._h, None, None, self._st(stream), ctypes.byref(out)), "insta_slack")
+        return Summary(out.wns, out.tns, out.num_violations, out.num_levels)
+
+    def arrivals(self, stream=None):
+        """insta_arrivals: (A, mean, sigma) float32[N,2] device tensors in caller pin order."""
+        t = self._torch
+        A, m, s = (t.empty((self.num_pins, 2), dtype=t.float32, device=self.device) for _ in range(3))
+        check(self.lib.insta_arrivals(self._h, _dptr(A), _dptr(m), _dptr(s), self._st(stream)), "insta_arrivals")
+        return A, m, s
+
+    def backward(self, ep_seed=None, want_src: bool = False, out=None, stream=None):
+        """insta_backward: dL/d(arc mean) float32[E,2] (caller arc order); L = TNS if ep_seed is None."""
+        t = self._torch
+        d_mean = out if out is not None else t.empty((self.num_arcs, 2), dtype=t.float32, device=self.device)
+        d_src = t.empty((self.num_pins, 2), dtype=t.float32, device=self.device) if want_src else None
+        seed = None
+        if ep_seed is not None:
+            seed = t.as_tensor(ep_seed, dtype=t.float32, device=self.device).contiguous()
+        check(self.lib.insta_backward(self._h, _dptr(seed), _dptr(d_mean), None, _dptr(d_src), self._st(stream)),
+              "insta_backward")
+        return (d_mean, d_src) if want_src else d_mean
+
+    def update_arcs(self, arc_ids, mean, sigma, incremental: bool = True, stream=None):
+        """insta_update_arcs: re-annotate arcs (device or host arrays; copied to the device)."""
+        t = self._torch
+        ids = t.as_tensor(arc_ids, dtype=t.int32, device=self.device).contiguous()
+        m = t.as_tensor(mean, dtype=t.float32, device=self.device).contiguous()
+        s = t.as_tensor(sigma, dtype=t.float32, device=self.device).contiguous()
+        check(self.lib.insta_update_arcs(self._h, int(ids.numel()), _dptr(ids), _dptr(m), _dptr(s),
+                                         int(bool(incremental)), self._st(stream)), "insta_update_arcs")
+
+    def last_forward_stats(self) -> int:
+        v = ctypes.c_int64()
+        check(self.lib.insta_last_forward_stats(self._h, ctypes.byref(v)), "insta_last_forward_stats")
+        return int(v.value)
+
+    def export(self) -> dict:
+        """insta_graph_export: the levelization (host numpy) for bit-exact checks."""
+        N, E = self.num_pins, self.num_arcs
+        out = dict(level=np.zeros(N, np.int32), order=np.zeros(N, np.int32),
+                   fanin_ptr=np.zeros(N + 1, np.int32), fanin_arc=np.zeros(E, np.int32),
+                   fanout_ptr=np.zeros(N + 1, np.int32), fanout_arc=np.zeros(E, np.int32))
+        check(self.lib.insta_graph_export(self._h, _ptr(out["level"]), _ptr(out["order"]), _ptr(out["fanin_ptr"]),
+                                          _ptr(out["fanin_arc"]), _ptr(out["fanout_ptr"]), _ptr(out["fanout_arc"])),
+              "insta_graph_export")
+        out["num_levels"] = self.num_levels
+        return out

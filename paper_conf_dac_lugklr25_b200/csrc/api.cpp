@@ -1,0 +1,377 @@
+// api.cpp -- the extern "C" boundary (include/insta.h): validation, host
+// levelization, device upload, call ordering and error reporting.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "internal.h"
+
+namespace {
+
+thread_local std::string g_last_error;
+
+insta_status fail(insta_status st, const std::string& msg) {
+  g_last_error = msg;
+  return st;
+}
+
+insta_status cuda_fail(int err, const char* where) {
+  if (err == int(cudaErrorMemoryAllocation))
+    return fail(INSTA_E_NOMEM, std::string(where) + ": out of device memory");
+  return fail(INSTA_E_CUDA, std::string(where) + ": " +
+                                cudaGetErrorString(static_cast<cudaError_t>(err)));
+}
+
+template <class T>
+cudaError_t upload(T** dst, const T* src, size_t count) {
+  *dst = nullptr;
+  size_t bytes = sizeof(T) * std::max<size_t>(count, 1);
+  cudaError_t e = cudaMalloc(reinterpret_cast<void**>(dst), bytes);
+  if (e != cudaSuccess) return e;
+  if (count && src) return cudaMemcpy(*dst, src, sizeof(T) * count, cudaMemcpyHostToDevice);
+  return cudaMemset(*dst, 0, bytes);
+}
+
+template <class T>
+cudaError_t alloc_zero(T** dst, size_t count) {
+  return upload<T>(dst, nullptr, count);
+}
+
+void free_graph(insta::DevGraph& d) {
+  void* ptrs[] = {d.level_ptr, d.tile_lv,   d.level_ntiles, d.done_fwd, d.done_bwd,
+                  d.heavy_slot, d.heavy_acc, d.fanin_ptr,   d.fin_src,  d.fin_ms,
+                  d.fin_arc,   d.fanout_ptr, d.fout,        d.arc_pos,  d.arc_sink,
+                  d.order,     d.src_ms,    d.ep_pin,       d.ep_rat,   d.arc_class,
+                  d.state,     d.g,         d.seed,         d.slack,    d.rf_star,
+                  d.partials,  d.ticket,    d.summary,      d.dirty,    d.changed,
+                  d.tile_dirty, d.counters};
+  for (void* p : ptrs)
+    if (p) cudaFree(p);
+}
+
+bool finite2(const float* a, int64_t n, bool nonneg) {
+  for (int64_t k = 0; k < 2 * n; ++k) {
+    if (!std::isfinite(a[k])) return false;
+    if (nonneg && a[k] < 0.f) return false;
+  }
+  return true;
+}
+
+insta_status validate_desc(const insta_graph_desc* d) {
+  if (!d) return fail(INSTA_E_ARG, "graph_create: NULL descriptor");
+  if (d->num_pins < 0 || d->num_arcs < 0 || d->num_endpoints < 0)
+    return fail(INSTA_E_ARG, "graph_create: negative size");
+  if (d->num_pins > insta::kMaxPins || d->num_arcs >= (int64_t(1) << 31))
+    return fail(INSTA_E_ARG, "graph_create: size limit (num_pins < 2^29, num_arcs < 2^31)");
+  if (d->num_arcs > 0 &&
+      (!d->arc_from || !d->arc_to || !d->arc_unate || !d->arc_mean || !d->arc_sigma))
+    return fail(INSTA_E_ARG, "graph_create: NULL arc array");
+  if (d->num_endpoints > 0 && (!d->ep_pin || !d->ep_rat))
+    return fail(INSTA_E_ARG, "graph_create: NULL endpoint array");
+  for (int64_t a = 0; a < d->num_arcs; ++a)
+    if (d->arc_unate[a] > INSTA_NON) return fail(INSTA_E_ARG, "graph_create: bad unateness");
+  if (d->num_arcs > 0 && !finite2(d->arc_mean, d->num_arcs, false))
+    return fail(INSTA_E_ARG, "graph_create: non-finite arc mean");
+  if (d->num_arcs > 0 && !finite2(d->arc_sigma, d->num_arcs, true))
+    return fail(INSTA_E_ARG, "graph_create: arc sigma must be finite and >= 0");
+  if (d->src_mean && !finite2(d->src_mean, d->num_pins, false))
+    return fail(INSTA_E_ARG, "graph_create: non-finite source mean");
+  if (d->src_sigma && !finite2(d->src_sigma, d->num_pins, true))
+    return fail(INSTA_E_ARG, "graph_create: source sigma must be finite and >= 0");
+  if (d->num_endpoints > 0 && !finite2(d->ep_rat, d->num_endpoints, false))
+    return fail(INSTA_E_ARG, "graph_create: non-finite required time");
+  std::vector<uint8_t> seen(size_t(d->num_pins), 0);
+  for (int32_t k = 0; k < d->num_endpoints; ++k) {
+    int32_t p = d->ep_pin[k];
+    if (p < 0 || p >= d->num_pins) return fail(INSTA_E_ARG, "graph_create: endpoint id out of range");
+    if (seen[p]) return fail(INSTA_E_ARG, "graph_create: duplicate endpoint pin");
+    seen[p] = 1;
+  }
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || d->device < 0 || d->device >= ndev)
+    return fail(INSTA_E_ARG, "graph_create: no such CUDA device");
+  return INSTA_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* insta_last_error(void) { return g_last_error.c_str(); }
+
+const char* insta_version(void) { return "insta-b200 0.1 (sm_100a)"; }
+
+insta_status insta_levelize(int32_t num_pins, int64_t num_arcs, const int32_t* arc_from,
+                            const int32_t* arc_to, int32_t* level_of_pin, int32_t* order,
+                            int32_t* fanin_ptr, int32_t* fanin_arc, int32_t* fanout_ptr,
+                            int32_t* fanout_arc, int32_t* num_levels) {
+  insta::HostLevels h;
+  std::string err;
+  insta_status st = insta::levelize_host(num_pins, num_arcs, arc_from, arc_to, &h, &err);
+  if (st != INSTA_OK) return fail(st, err);
+  const size_t n = size_t(num_pins), e = size_t(num_arcs);
+  if (level_of_pin) std::copy(h.level.begin(), h.level.end(), level_of_pin);
+  if (order) std::copy(h.order.begin(), h.order.end(), order);
+  if (fanin_ptr) std::copy(h.fanin_ptr.begin(), h.fanin_ptr.begin() + n + 1, fanin_ptr);
+  if (fanout_ptr) std::copy(h.fanout_ptr.begin(), h.fanout_ptr.begin() + n + 1, fanout_ptr);
+  if (fanin_arc) std::copy(h.fanin_arc.begin(), h.fanin_arc.begin() + e, fanin_arc);
+  if (fanout_arc) std::copy(h.fanout_arc.begin(), h.fanout_arc.begin() + e, fanout_arc);
+  if (num_levels) *num_levels = h.num_levels;
+  return INSTA_OK;
+}
+
+insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out) {
+  if (!out) return fail(INSTA_E_ARG, "graph_create: NULL out");
+  *out = nullptr;
+  insta_status st = validate_desc(desc);
+  if (st != INSTA_OK) return st;
+  insta_graph* G = new (std::nothrow) insta_graph();
+  if (!G) return fail(INSTA_E_NOMEM, "graph_create: host allocation");
+  insta::DevGraph& d = G->d;
+  d.device = desc->device;
+  std::string err;
+  st = insta::levelize_host(desc->num_pins, desc->num_arcs, desc->arc_from, desc->arc_to, &d.host,
+                            &err);
+  if (st != INSTA_OK) {
+    delete G;
+    return fail(st, err);
+  }
+  const insta::HostLevels& h = d.host;
+  const int32_t n = desc->num_pins;
+  const int64_t E = desc->num_arcs;
+  d.n = n;
+  d.e = E;
+  d.num_levels = h.num_levels;
+  d.num_src = n > 0 ? h.level_ptr[1] : 0;
+  d.num_ep = desc->num_endpoints;
+  d.num_tiles = (n + insta::kTile - 1) / insta::kTile;
+
+  // ---- canonical host arrays ------------------------------------------------
+  const size_t nE = static_cast<size_t>(E), nN = static_cast<size_t>(n);
+  std::vector<int32_t> arc_pos(nE), arc_sink(nE), fin_src(nE), fout(nE);
+  std::vector<float4> fin_ms(nE);
+  std::vector<int32_t> heavy_slot(nN, -1);
+  int32_t nheavy = 0;
+  for (int32_t k = 0; k < n; ++k) {
+    if (h.fanout_ptr[k + 1] - h.fanout_ptr[k] > insta::kHeavyFanout) heavy_slot[k] = nheavy++;
+    d.max_fanin = std::max(d.max_fanin, h.fanin_ptr[k + 1] - h.fanin_ptr[k]);
+  }
+  d.num_heavy = nheavy;
+  for (int64_t q = 0; q < E; ++q) {
+    const int32_t a = h.fanin_arc[q];
+    const int32_t src = h.pos[desc->arc_from[a]];
+    arc_pos[a] = int32_t(q);
+    arc_sink[a] = h.pos[desc->arc_to[a]];
+    fin_src[q] = src | ((heavy_slot[src] >= 0 ? 1 : 0) << 29) |
+                 int32_t(uint32_t(desc->arc_unate[a]) << insta::kUnateShift);
+    fin_ms[q] = make_float4(desc->arc_mean[2 * a], desc->arc_mean[2 * a + 1],
+                            desc->arc_sigma[2 * a], desc->arc_sigma[2 * a + 1]);
+  }
+  for (int64_t k = 0; k < E; ++k) fout[k] = arc_pos[h.fanout_arc[k]];
+  std::vector<float4> src_ms(size_t(std::max(d.num_src, 1)));
+  for (int32_t i = 0; i < d.num_src; ++i) {
+    const int32_t p = h.order[i];
+    src_ms[i] = make_float4(desc->src_mean ? desc->src_mean[2 * p] : 0.f,
+                            desc->src_mean ? desc->src_mean[2 * p + 1] : 0.f,
+                            desc->src_sigma ? desc->src_sigma[2 * p] : 0.f,
+                            desc->src_sigma ? desc->src_sigma[2 * p + 1] : 0.f);
+  }
+  std::vector<int32_t> ep_pin(size_t(d.num_ep));
+  std::vector<float2> ep_rat(size_t(d.num_ep));
+  for (int32_t k = 0; k < d.num_ep; ++k) {
+    ep_pin[k] = h.pos[desc->ep_pin[k]];
+    ep_rat[k] = make_float2(desc->ep_rat[2 * k], desc->ep_rat[2 * k + 1]);
+  }
+  // tiles of kTile canonical pins and the levels they span
+  std::vector<int2> tile_lv(size_t(std::max(d.num_tiles, 1)));
+  std::vector<int32_t> level_ntiles(size_t(std::max(d.num_levels, 1)), 0);
+  for (int32_t t = 0; t < d.num_tiles; ++t) {
+    const int32_t first = t * insta::kTile;
+    const int32_t last = std::min(n, first + insta::kTile) - 1;
+    tile_lv[t] = make_int2(h.level[h.order[first]], h.level[h.order[last]]);
+    for (int l = tile_lv[t].x; l <= tile_lv[t].y; ++l) level_ntiles[l]++;
+  }
+  std::vector<uint8_t> arc_class(nE, 0);
+  if (desc->arc_class) std::copy(desc->arc_class, desc->arc_class + E, arc_class.begin());
+
+  // ---- device upload ----------------------------------------------------------
+  cudaError_t e = cudaSetDevice(d.device);
+#define UP(dst, src, cnt)                       \
+  if (e == cudaSuccess) e = upload(&(dst), (src), size_t(cnt));
+#define ZERO(dst, cnt) \
+  if (e == cudaSuccess) e = alloc_zero(&(dst), size_t(cnt));
+  UP(d.level_ptr, h.level_ptr.data(), h.level_ptr.size());
+  UP(d.tile_lv, tile_lv.data(), tile_lv.size());
+  UP(d.level_ntiles, level_ntiles.data(), level_ntiles.size());
+  ZERO(d.done_fwd, std::max(d.num_levels, 1));
+  ZERO(d.done_bwd, std::max(d.num_levels, 1));
+  UP(d.heavy_slot, heavy_slot.data(), heavy_slot.size());
+  ZERO(d.heavy_acc, 2 * std::max(nheavy, 1));
+  UP(d.fanin_ptr, h.fanin_ptr.data(), h.fanin_ptr.size());
+  UP(d.fin_src, fin_src.data(), fin_src.size());
+  UP(d.fin_ms, fin_ms.data(), fin_ms.size());
+  UP(d.fin_arc, h.fanin_arc.data(), h.fanin_arc.size());
+  UP(d.fanout_ptr, h.fanout_ptr.data(), h.fanout_ptr.size());
+  UP(d.fout, fout.data(), fout.size());
+  UP(d.arc_pos, arc_pos.data(), arc_pos.size());
+  UP(d.arc_sink, arc_sink.data(), arc_sink.size());
+  UP(d.order, h.order.data(), h.order.size());
+  UP(d.src_ms, src_ms.data(), src_ms.size());
+  UP(d.ep_pin, ep_pin.data(), ep_pin.size());
+  UP(d.ep_rat, ep_rat.data(), ep_rat.size());
+  UP(d.arc_class, arc_class.data(), arc_class.size());
+  ZERO(d.state, n);
+  ZERO(d.g, E);
+  ZERO(d.seed, n);
+  ZERO(d.slack, d.num_ep);
+  ZERO(d.rf_star, d.num_ep);
+  ZERO(d.partials, 3 * ((d.num_ep + 255) / 256 + 1));
+  ZERO(d.ticket, 1);
+  ZERO(d.summary, 4);
+  ZERO(d.counters, 4);
+#undef UP
+#undef ZERO
+  if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  if (e == cudaSuccess) e = static_cast<cudaError_t>(insta::configure_grids(d));
+  if (e != cudaSuccess) {
+    insta_status s2 = cuda_fail(int(e), "graph_create");
+    free_graph(d);
+    delete G;
+    return s2;
+  }
+  *out = G;
+  return INSTA_OK;
+}
+
+void insta_graph_destroy(insta_graph* g) {
+  if (!g) return;
+  cudaSetDevice(g->d.device);
+  free_graph(g->d);
+  delete g;
+}
+
+insta_status insta_graph_export(const insta_graph* g, int32_t* level_of_pin, int32_t* order,
+                                int32_t* fanin_ptr, int32_t* fanin_arc, int32_t* fanout_ptr,
+                                int32_t* fanout_arc) {
+  if (!g) return fail(INSTA_E_ARG, "graph_export: NULL graph");
+  const insta::HostLevels& h = g->d.host;
+  if (level_of_pin) std::copy(h.level.begin(), h.level.end(), level_of_pin);
+  if (order) std::copy(h.order.begin(), h.order.end(), order);
+  if (fanin_ptr) std::copy(h.fanin_ptr.begin(), h.fanin_ptr.end(), fanin_ptr);
+  if (fanout_ptr) std::copy(h.fanout_ptr.begin(), h.fanout_ptr.end(), fanout_ptr);
+  if (fanin_arc) std::copy(h.fanin_arc.begin(), h.fanin_arc.end(), fanin_arc);
+  if (fanout_arc) std::copy(h.fanout_arc.begin(), h.fanout_arc.end(), fanout_arc);
+  return INSTA_OK;
+}
+
+insta_status insta_graph_sizes(const insta_graph* g, int32_t* num_pins, int64_t* num_arcs,
+                               int32_t* num_endpoints, int32_t* num_levels) {
+  if (!g) return fail(INSTA_E_ARG, "graph_sizes: NULL graph");
+  if (num_pins) *num_pins = g->d.n;
+  if (num_arcs) *num_arcs = g->d.e;
+  if (num_endpoints) *num_endpoints = g->d.num_ep;
+  if (num_levels) *num_levels = g->d.num_levels;
+  return INSTA_OK;
+}
+
+static insta_status read_summary(insta::DevGraph& d, void* stream, insta_summary* out) {
+  double s[3];
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  cudaError_t e = cudaMemcpyAsync(s, d.summary, sizeof s, cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) return cuda_fail(int(e), "summary");
+  out->wns = s[0];
+  out->tns = s[1];
+  out->num_violations = int32_t(s[2]);
+  out->num_levels = d.num_levels;
+  return INSTA_OK;
+}
+
+insta_status insta_forward(insta_graph* g, const insta_opts* o, void* cuda_stream,
+                           insta_summary* out) {
+  if (!g) return fail(INSTA_E_ARG, "forward: NULL graph");
+  insta_opts opt{3.0f, 0.0f, 0, 0};
+  if (o) opt = *o;
+  if (!std::isfinite(opt.n_sigma) || opt.n_sigma < 0.f || !std::isfinite(opt.tau) ||
+      opt.tau < 0.f)
+    return fail(INSTA_E_ARG, "forward: n_sigma and tau must be finite and >= 0");
+  if (opt.want_grad_sigma != 0) return fail(INSTA_E_ARG, "forward: want_grad_sigma unsupported");
+  if (opt.schedule != 0 && opt.schedule != 1) return fail(INSTA_E_ARG, "forward: bad schedule");
+  insta::DevGraph& d = g->d;
+  cudaSetDevice(d.device);
+  int err = insta::launch_forward(d, opt.n_sigma, opt.tau, opt.schedule, cuda_stream);
+  if (err) return cuda_fail(err, "forward");
+  d.bwd_schedule = opt.schedule;
+  d.fwd_valid = true;
+  d.pending_full = false;
+  d.pending_incremental = false;
+  d.last_recomputed = d.n;
+  if (out) return read_summary(d, cuda_stream, out);
+  return INSTA_OK;
+}
+
+insta_status insta_slack(insta_graph* g, float* slack, uint8_t* rf_star, void* cuda_stream,
+                         insta_summary* out) {
+  if (!g) return fail(INSTA_E_ARG, "slack: NULL graph");
+  insta::DevGraph& d = g->d;
+  if (!d.fwd_valid) return fail(INSTA_E_STATE, "slack: no valid forward (call insta_forward)");
+  cudaSetDevice(d.device);
+  int err = insta::launch_copy_slack(d, slack, rf_star, cuda_stream);
+  if (err) return cuda_fail(err, "slack");
+  if (out) return read_summary(d, cuda_stream, out);
+  return INSTA_OK;
+}
+
+insta_status insta_arrivals(insta_graph* g, float* A, float* mean, float* sigma,
+                            void* cuda_stream) {
+  if (!g) return fail(INSTA_E_ARG, "arrivals: NULL graph");
+  insta::DevGraph& d = g->d;
+  if (!d.fwd_valid) return fail(INSTA_E_STATE, "arrivals: no valid forward");
+  cudaSetDevice(d.device);
+  int err = insta::launch_arrivals(d, A, mean, sigma, cuda_stream);
+  if (err) return cuda_fail(err, "arrivals");
+  return INSTA_OK;
+}
+
+insta_status insta_backward(insta_graph* g, const float* ep_seed, float* d_arc_mean,
+                            float* d_arc_sigma, float* d_src, void* cuda_stream) {
+  if (!g) return fail(INSTA_E_ARG, "backward: NULL graph");
+  if (!d_arc_mean) return fail(INSTA_E_ARG, "backward: d_arc_mean is required");
+  if (d_arc_sigma) return fail(INSTA_E_ARG, "backward: d_arc_sigma is not supported (pass NULL)");
+  insta::DevGraph& d = g->d;
+  if (!d.fwd_valid) return fail(INSTA_E_STATE, "backward: no valid forward (call insta_forward)");
+  cudaSetDevice(d.device);
+  int err = insta::launch_backward(d, ep_seed, d_arc_mean, d_src, cuda_stream);
+  if (err) return cuda_fail(err, "backward");
+  return INSTA_OK;
+}
+
+insta_status insta_update_arcs(insta_graph* g, int64_t n, const int32_t* arc_ids,
+                               const float* mean, const float* sigma, int32_t incremental,
+                               void* cuda_stream) {
+  if (!g) return fail(INSTA_E_ARG, "update_arcs: NULL graph");
+  if (n < 0 || (n > 0 && (!arc_ids || !mean || !sigma)))
+    return fail(INSTA_E_ARG, "update_arcs: bad arguments");
+  insta::DevGraph& d = g->d;
+  if (n > d.e) return fail(INSTA_E_ARG, "update_arcs: more updates than arcs");
+  cudaSetDevice(d.device);
+  int err = insta::launch_update_arcs(d, n, arc_ids, mean, sigma, incremental, cuda_stream);
+  if (err) return cuda_fail(err, "update_arcs");
+  d.fwd_valid = false;
+  if (incremental && !d.pending_full) d.pending_incremental = true;
+  else d.pending_full = true;
+  return INSTA_OK;
+}
+
+insta_status insta_last_forward_stats(insta_graph* g, int64_t* pins_recomputed) {
+  if (!g) return fail(INSTA_E_ARG, "stats: NULL graph");
+  if (pins_recomputed) *pins_recomputed = g->d.last_recomputed;
+  return INSTA_OK;
+}
+
+}  // extern "C"

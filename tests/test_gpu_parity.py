@@ -1,0 +1,282 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the fp64 CPU oracle.
+
+Tolerances (BASELINE.json north_star):
+  levelization / CSR: bit-exact;
+  arrival, slack: |x - x_ref| <= max(1e-4 |x_ref|, 1e-3 ps);
+  gradients: |g - g_ref| <= 1e-3 max(|g_ref|, 1) for tau = 0 (tie-free arcs) and tau >= 1 ps;
+             ||g - g_ref|| <= 1e-3 ||g_ref|| ... reported for tau = 0.01 (see test);
+  dyadic mode (mu on a 2^-6 grid, sigma = 0): bit-exact, ties included.
+Near-tie arcs in hard mode are excluded using the oracle's taint mask
+(oracle.tie_taint) and must stay a small fraction.
+"""
+import types
+
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_dac_lugklr25_b200 as insta
+from paper_conf_dac_lugklr25_b200 import synth
+from tests import bruteforce as bf
+
+pytestmark = pytest.mark.gpu
+NS = 3.0
+
+
+def tol_ok(x, ref, mask=None):
+    err = np.abs(np.asarray(x, np.float64) - ref)
+    lim = np.maximum(1e-4 * np.abs(ref), 1e-3)
+    bad = err > lim
+    if mask is not None:
+        bad &= ~mask
+    return bad
+
+
+def run_gpu(g, tau=0.0, schedule=0, seed=None, want_src=False):
+    G = insta.Graph(g)
+    s = G.forward(NS, tau, schedule)
+    A, mu, sig = (x.cpu().numpy() for x in G.arrivals())
+    sl, rf = (x.cpu().numpy() for x in G.slack())
+    out = G.backward(ep_seed=seed, want_src=want_src)
+    if want_src:
+        d, dsrc = out[0].cpu().numpy(), out[1].cpu().numpy()
+    else:
+        d, dsrc = out.cpu().numpy(), None
+    exp = G.export()
+    G.close()
+    return types.SimpleNamespace(summary=s, A=A, mu=mu, sigma=sig, slack=sl, rf=rf, d_mean=d, d_src=dsrc,
+                                 export=exp)
+
+
+def run_oracle(g, tau=0.0, dslack=None):
+    f = oracle.forward(g, NS, tau)
+    s = oracle.slack(g, f["A"])
+    b = oracle.backward(g, NS, tau, dslack=dslack)
+    return f, s, b
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C2"])
+def test_levelization_bit_exact(cfg):
+    g = synth.generate(cfg)
+    G = insta.Graph(g)
+    e = G.export()
+    o = oracle.levelize(g.num_pins, g.arc_from, g.arc_to)
+    for k in ("level", "order", "fanin_ptr", "fanin_arc", "fanout_ptr", "fanout_arc"):
+        assert np.array_equal(e[k], o[k]), k
+    assert G.num_levels == o["num_levels"]
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C2"])
+@pytest.mark.parametrize("schedule", [0, 1])
+def test_dyadic_hard_bit_exact(cfg, schedule):
+    """sigma = 0 and mu on a 2^-6 grid: fp32 sums are exact, so GPU == oracle bit for bit,
+    including tie-breaking (first candidate wins)."""
+    g = synth.generate(cfg, dyadic=True)
+    r = run_gpu(g, 0.0, schedule)
+    f, s, b = run_oracle(g, 0.0)
+    assert np.array_equal(r.A, f["A"].astype(np.float32))
+    assert np.array_equal(r.slack, s["slack"].astype(np.float32))
+    assert np.array_equal(r.rf, s["rf_star"])
+    assert r.summary.tns == s["tns"] and r.summary.wns == s["wns"]
+    assert r.summary.num_violations == s["num_viol"]
+    assert np.array_equal(r.d_mean, b["d_mean"].astype(np.float32))
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C2"])
+def test_hard_parity(cfg):
+    g = synth.generate(cfg)
+    r = run_gpu(g, 0.0)
+    f, s, b = run_oracle(g, 0.0)
+    ft, at = oracle.tie_taint(g, NS, eps=2e-3, margin=0.05)
+    assert ft.mean() < 0.01
+    assert not tol_ok(r.A, f["A"], ft).any()
+    assert not tol_ok(r.mu, f["mu"], ft).any()
+    ep_t = ft[g.ep_pin].any(axis=1)
+    assert not tol_ok(r.slack, s["slack"], ep_t).any()
+    assert r.summary.num_violations == pytest.approx(s["num_viol"], abs=max(1, ep_t.sum()))
+    assert r.summary.tns == pytest.approx(s["tns"], rel=1e-5)
+    # hard-mode gradients are (negated) path counts: exact away from near-ties
+    bad = (r.d_mean != b["d_mean"]) & ~at
+    assert not bad.any(), np.argwhere(bad)[:5]
+    assert at.mean() < 0.01
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C2"])
+def test_lse_tau1_parity(cfg):
+    g = synth.generate(cfg)
+    r = run_gpu(g, 1.0, want_src=True)
+    f, s, b = run_oracle(g, 1.0)
+    assert not tol_ok(r.A, f["A"]).any()
+    assert not tol_ok(r.slack, s["slack"]).any()
+    assert r.summary.tns == pytest.approx(s["tns"], rel=1e-5)
+    err = np.abs(r.d_mean - b["d_mean"])
+    assert (err <= 1e-3 * np.maximum(np.abs(b["d_mean"]), 1.0)).all(), err.max()
+    srcmask = np.bincount(g.arc_to, minlength=g.num_pins) == 0
+    assert np.abs(r.d_src[srcmask] - b["d_src_mean"][srcmask]).max() <= 1e-3 * max(1, np.abs(b["d_src_mean"]).max())
+
+
+def test_lse_tau_0p01_normwise_c1():
+    """tau = 0.01 ps (the INSTA-Size value): fp32 arrival rounding is a visible
+    fraction of tau, so gradients are compared norm-wise."""
+    g = synth.generate("C1")
+    r = run_gpu(g, 0.01)
+    f, s, b = run_oracle(g, 0.01)
+    assert not tol_ok(r.A, f["A"]).any()
+    rel = np.linalg.norm(r.d_mean - b["d_mean"]) / np.linalg.norm(b["d_mean"])
+    assert rel <= 1e-3, rel
+
+
+@pytest.mark.parametrize("tau", [0.0, 1.0])
+def test_schedules_and_reruns_bit_identical(tau):
+    g = synth.generate("C2")
+    a = run_gpu(g, tau, 0)
+    c = run_gpu(g, tau, 1)
+    d = run_gpu(g, tau, 0)
+    for x, y in ((a, c), (a, d)):
+        assert np.array_equal(x.A, y.A) and np.array_equal(x.sigma, y.sigma)
+        assert np.array_equal(x.slack, y.slack) and x.summary == y.summary
+        assert np.array_equal(x.d_mean, y.d_mean)
+
+
+def test_custom_endpoint_seed_and_source_gradient():
+    g = synth.generate("C1")
+    rng = np.random.default_rng(7)
+    seed = rng.uniform(-1, 1, g.num_endpoints).astype(np.float32)
+    r = run_gpu(g, 1.0, seed=seed, want_src=True)
+    _, _, b = run_oracle(g, 1.0, dslack=seed.astype(np.float64))
+    assert np.abs(r.d_mean - b["d_mean"]).max() <= 1e-3 * max(1.0, np.abs(b["d_mean"]).max())
+    assert np.abs(r.d_src - b["d_src_mean"]).max() <= 1e-3 * max(1.0, np.abs(b["d_src_mean"]).max())
+
+
+@pytest.mark.parametrize("seed", range(6))
+@pytest.mark.parametrize("tau", [0.0, 1.0])
+def test_tiny_dags(seed, tau):
+    g = bf.tiny_dag(seed, n_pins=9)
+    r = run_gpu(g, tau)
+    f, s, b = run_oracle(g, tau)
+    ft, at = oracle.tie_taint(g, NS, eps=1e-4, margin=0.05)
+    assert not tol_ok(r.A, f["A"], ft if tau == 0 else None).any()
+    mask = at if tau == 0 else np.zeros_like(at)
+    err = np.abs(r.d_mean - b["d_mean"])
+    assert ((err <= 1e-3 * np.maximum(np.abs(b["d_mean"]), 1)) | mask).all()
+
+
+def _star(n_sinks, tau_unate=2, wide=9):
+    """One driver with a huge fanout (> 128, the heavy-driver path) and a wide
+    (9-input) NON-unate cell: exercises the atomic accumulator and the slow fanin path."""
+    rng = np.random.default_rng(n_sinks)
+    src, drv = 0, 1
+    sinks = np.arange(2, 2 + n_sinks)
+    cell_in = sinks[:wide]
+    out = 2 + n_sinks
+    af = [src] + [drv] * n_sinks + list(cell_in)
+    at = [drv] + list(sinks) + [out] * wide
+    E = len(af)
+    un = np.zeros(E, np.uint8)
+    un[1 + n_sinks:] = tau_unate
+    mean = rng.uniform(1, 10, (E, 2)).astype(np.float32)
+    sig = rng.uniform(0, 1, (E, 2)).astype(np.float32)
+    N = out + 1
+    eps = np.concatenate([sinks[wide:], [out]]).astype(np.int32)
+    rat = np.full((len(eps), 2), 18.0, np.float32)
+    sm = np.zeros((N, 2), np.float32)
+    ss = np.zeros((N, 2), np.float32)
+    ss[0] = 0.5
+    return types.SimpleNamespace(num_pins=N, arc_from=np.array(af, np.int32), arc_to=np.array(at, np.int32),
+                                 arc_unate=un, arc_class=np.zeros(E, np.uint8), arc_mean=mean, arc_sigma=sig,
+                                 src_mean=sm, src_sigma=ss, ep_pin=eps, ep_rat=rat)
+
+
+@pytest.mark.parametrize("n_sinks", [40, 3000])
+@pytest.mark.parametrize("tau", [0.0, 1.0])
+def test_heavy_fanout_and_wide_fanin(n_sinks, tau):
+    g = _star(n_sinks)
+    r = run_gpu(g, tau, want_src=True)
+    f, s, b = run_oracle(g, tau)
+    assert not tol_ok(r.A, f["A"]).any()
+    err = np.abs(r.d_mean - b["d_mean"])
+    assert (err <= 1e-3 * np.maximum(np.abs(b["d_mean"]), 1)).all(), err.max()
+    assert np.abs(r.d_src - b["d_src_mean"]).max() <= 1e-3 * max(1, np.abs(b["d_src_mean"]).max())
+    r1 = run_gpu(g, tau, schedule=1)
+    assert np.array_equal(r1.d_mean, r.d_mean)
+
+
+def test_degenerate_graphs():
+    # no arcs: all pins are sources; endpoints at sources
+    g = types.SimpleNamespace(num_pins=3, arc_from=np.zeros(0, np.int32), arc_to=np.zeros(0, np.int32),
+                              arc_unate=np.zeros(0, np.uint8), arc_class=None, arc_mean=np.zeros((0, 2), np.float32),
+                              arc_sigma=np.zeros((0, 2), np.float32),
+                              src_mean=np.array([[1, 2], [3, 4], [5, 6]], np.float32),
+                              src_sigma=np.zeros((3, 2), np.float32),
+                              ep_pin=np.array([2, 0], np.int32), ep_rat=np.array([[4, 4], [0, 5]], np.float32))
+    r = run_gpu(g, 0.0, want_src=True)
+    assert list(r.slack) == [-2.0, -1.0]
+    assert r.summary.tns == -3.0 and r.summary.num_violations == 2
+    assert np.array_equal(r.d_src, np.array([[-1, 0], [0, 0], [-1, 0]], np.float32))
+    # no endpoints
+    g2 = bf.tiny_dag(1)
+    g2.ep_pin = np.zeros(0, np.int32)
+    g2.ep_rat = np.zeros((0, 2), np.float32)
+    r2 = run_gpu(g2, 0.0)
+    assert r2.summary.tns == 0.0 and not r2.d_mean.any()
+
+
+def test_call_order_errors():
+    g = synth.generate("C1")
+    G = insta.Graph(g)
+    with pytest.raises(insta.InstaError, match="E_STATE"):
+        G.backward()
+    G.forward()
+    G.update_arcs([0], np.ones((1, 2)), np.zeros((1, 2)), incremental=False)
+    with pytest.raises(insta.InstaError, match="E_STATE"):
+        G.slack()
+    with pytest.raises(insta.InstaError, match="E_ARG"):
+        G.forward(tau=-1.0)
+    G.close()
+
+
+def test_update_arcs_then_forward_equals_fresh_graph():
+    g = synth.generate("C2")
+    ids, m, s = synth.sizing_step(g, 0)
+    G = insta.Graph(g)
+    G.forward()
+    G.update_arcs(ids, m, s, incremental=False)
+    G.forward()
+    A1 = G.arrivals()[0].cpu().numpy()
+    d1 = G.backward().cpu().numpy()
+    g2 = types.SimpleNamespace(**vars(g))
+    g2.arc_mean = g.arc_mean.copy()
+    g2.arc_sigma = g.arc_sigma.copy()
+    g2.arc_mean[ids] = m
+    g2.arc_sigma[ids] = s
+    r = run_gpu(g2, 0.0)
+    assert np.array_equal(A1, r.A) and np.array_equal(d1, r.d_mean)
+
+
+@pytest.mark.slow
+def test_c4_full_size_parity():
+    """15M pins, the bench configuration (persistent kernels, hard mode): levelization
+    bit-exact, arrivals/slack within tolerance everywhere outside near-tie taint, TNS."""
+    g = synth.generate("C4")
+    G = insta.Graph(g)
+    summ = G.forward(NS, 0.0)
+    e = G.export()
+    o = oracle.levelize(g.num_pins, g.arc_from, g.arc_to)
+    for k in ("level", "order", "fanin_ptr", "fanin_arc", "fanout_ptr", "fanout_arc"):
+        assert np.array_equal(e[k], o[k]), k
+    del e, o
+    A = G.arrivals()[0].cpu().numpy()
+    sl = G.slack()[0].cpu().numpy()
+    f = oracle.forward(g, NS, 0.0)
+    s = oracle.slack(g, f["A"])
+    ft, _ = oracle.tie_taint(g, NS, eps=2e-3, margin=0.05)
+    assert ft.mean() < 0.01
+    assert not tol_ok(A, f["A"], ft).any()
+    assert not tol_ok(sl, s["slack"], ft[g.ep_pin].any(axis=1)).any()
+    assert summ.tns == pytest.approx(s["tns"], rel=1e-5)
+    # gradients: hard mode, exact integers away from near-ties
+    d = G.backward().cpu().numpy()
+    b = oracle.backward(g, NS, 0.0)
+    _, at = oracle.tie_taint(g, NS, eps=2e-3, margin=0.05)
+    assert not ((d != b["d_mean"]) & ~at).any()
+    G.close()
