@@ -101,22 +101,29 @@ class ClockSampler:
 # ---------------------------------------------------------------------------
 # byte model: algorithmic bytes per launch
 # ---------------------------------------------------------------------------
-def fwd_bytes(N, E, n_src, P):
-    return (4 * (N - n_src) + 4          # fanin row pointers
-            + 36 * E                      # fin_src 4 + arc {mu,sigma}x{R,F} 16 + source state gather 16
-            + 16 * N                      # state write
-            + 16 * n_src                  # source (clock) arrival read
-            + 33 * P)                     # slack: ep pin 4 + RAT 8 + state 16 + slack 4 + rf 1
+HEAVY_FANOUT = 256   # csrc/internal.h kHeavyFanout: drivers above it use the atomic path
 
 
-def bwd_bytes(N, E, n_src, P, E_active):
+def fwd_bytes(N, E, n_src, P, lse):
+    """insta_forward: propagation kernel + slack/TNS kernel."""
+    return (4 * (N - n_src) + 4           # fanin row pointers
+            + 20 * E                      # per arc: source word 4 + {mu,sigma}x{R,F} 16 (TMA-staged)
+            + 24 * E                      # per arc: source state gather {mu_R, mu_F (f64), sigma_R, sigma_F}
+            + 24 * N                      # state write
+            + 16 * n_src                  # startpoint (clock) arrival read
+            + (16 * E if lse else 4 * (N - n_src))   # Eq 6 weights per arc (LSE) / arg-max per pin (hard)
+            + 41 * P)                     # slack: ep pin 4 + RAT 8 + state 24 + slack 4 + rf 1
+
+
+def bwd_bytes(N, E, E_light, P, nnz_arcs, lse):
+    """insta_backward: zero fill + seed kernel + propagation kernel."""
     return (8 * E                         # d_mean zero fill
             + 17 * P                      # seeds: ep pin 4 + slack 4 + rf 1 + seed write 8
-            + 12 * N + 4 * (N - n_src)    # fanout ptr + seed read + fanin ptr
-            + 12 * E                      # pull: fanout entry 4 + per-arc adjoint gather 8
-            + 8 * E                       # per-arc adjoint write
-            + 48 * E_active)              # arcs of pins with nonzero adjoint: topology 20 + src state 16
-                                          # + arc id 4 + d_mean write 8
+            + 24 * N                      # per pin: light-fanout ptr 4, fanin ptr 4, seed 8, heavy slot 4, + 4
+            + (16 * E if lse else 0)      # Eq 6 weights (LSE); the hard arg-max is in the 24 B/pin above
+            + 12 * E_light                # pull: fanout entry 4 + per-arc adjoint gather 8
+            + 16 * E                      # per arc: source word 4 + arc id 4 + per-arc adjoint write 8
+            + 8 * nnz_arcs)               # nonzero d_mean scatter
 
 
 def cpu_oracle_sample(cfg_name, sample_pins, tau):
@@ -239,15 +246,14 @@ def main():
     ms_step = total_ms / args.steps
     value = world * N / (ms_step * 1e-3)
 
-    # active arcs of the backward (pins with nonzero adjoint) for the byte model
+    # byte model inputs: nonzero gradient arcs and light (pulled) fanout entries
     dm = d_mean.cpu().numpy()
-    nz_arcs = np.nonzero((dm != 0).any(axis=1))[0]
-    active = np.zeros(N, bool)
-    active[g.arc_to[nz_arcs]] = True
-    indeg = np.bincount(g.arc_to, minlength=N)
-    E_active = int(indeg[active].sum())
-    fb = fwd_bytes(N, E, n_src, P)
-    bb = bwd_bytes(N, E, n_src, P, E_active)
+    nnz_arcs = int(np.count_nonzero((dm != 0).any(axis=1)))
+    fo = np.bincount(g.arc_from, minlength=N)
+    E_light = int(fo[fo <= HEAVY_FANOUT].sum())
+    lse = args.tau > 0
+    fb = fwd_bytes(N, E, n_src, P, lse)
+    bb = bwd_bytes(N, E, E_light, P, nnz_arcs, lse)
     peak, peak_kind = _peaks()
     fwd_gbs = fb / (fwd_ms * 1e-3) / 1e9
     bwd_gbs = bb / (bwd_ms * 1e-3) / 1e9

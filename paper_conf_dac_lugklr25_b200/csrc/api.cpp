@@ -27,10 +27,12 @@ insta_status cuda_fail(int err, const char* where) {
                                 cudaGetErrorString(static_cast<cudaError_t>(err)));
 }
 
+// Every device array is padded by 64 bytes: TMA bulk copies read 16-byte
+// aligned windows that may extend past the last element.
 template <class T>
 cudaError_t upload(T** dst, const T* src, size_t count) {
   *dst = nullptr;
-  size_t bytes = sizeof(T) * std::max<size_t>(count, 1);
+  size_t bytes = sizeof(T) * std::max<size_t>(count, 1) + 64;
   cudaError_t e = cudaMalloc(reinterpret_cast<void**>(dst), bytes);
   if (e != cudaSuccess) return e;
   if (count && src) return cudaMemcpy(*dst, src, sizeof(T) * count, cudaMemcpyHostToDevice);
@@ -43,13 +45,12 @@ cudaError_t alloc_zero(T** dst, size_t count) {
 }
 
 void free_graph(insta::DevGraph& d) {
-  void* ptrs[] = {d.level_ptr, d.tile_lv,   d.level_ntiles, d.done_fwd, d.done_bwd,
-                  d.heavy_slot, d.heavy_acc, d.fanin_ptr,   d.fin_src,  d.fin_ms,
-                  d.fin_arc,   d.fanout_ptr, d.fout,        d.arc_pos,  d.arc_sink,
-                  d.order,     d.src_ms,    d.ep_pin,       d.ep_rat,   d.arc_class,
-                  d.state,     d.g,         d.seed,         d.slack,    d.rf_star,
-                  d.partials,  d.ticket,    d.summary,      d.dirty,    d.changed,
-                  d.tile_dirty, d.counters};
+  void* ptrs[] = {d.level_ptr, d.fanin_ptr, d.fin_src,   d.fin_ms,     d.fin_arc,   d.lfo_ptr,
+                  d.lfo,       d.fanout_ptr, d.fout_sink, d.heavy_slot, d.heavy_acc, d.arc_pos,
+                  d.arc_sink,  d.order,     d.src_ms,    d.ep_pin,     d.ep_rat,    d.arc_class,
+                  d.fwd_a,     d.fwd_b,     d.bwd_a,     d.bwd_b,      d.done_fwd,  d.done_bwd,
+                  d.state,     d.win,       d.wts,       d.g,          d.seed,      d.slack,
+                  d.rf_star,   d.partials,  d.ticket,    d.summary,    d.dirty,     d.counters};
   for (void* p : ptrs)
     if (p) cudaFree(p);
 }
@@ -149,17 +150,20 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   d.num_levels = h.num_levels;
   d.num_src = n > 0 ? h.level_ptr[1] : 0;
   d.num_ep = desc->num_endpoints;
-  d.num_tiles = (n + insta::kTile - 1) / insta::kTile;
 
   // ---- canonical host arrays ------------------------------------------------
   const size_t nE = static_cast<size_t>(E), nN = static_cast<size_t>(n);
-  std::vector<int32_t> arc_pos(nE), arc_sink(nE), fin_src(nE), fout(nE);
+  std::vector<int32_t> arc_pos(nE), arc_sink(nE), fin_src(nE), fout_sink(nE);
   std::vector<float4> fin_ms(nE);
   std::vector<int32_t> heavy_slot(nN, -1);
-  int32_t nheavy = 0;
+  int32_t nheavy = 0, max_fanin = 0;
   for (int32_t k = 0; k < n; ++k) {
     if (h.fanout_ptr[k + 1] - h.fanout_ptr[k] > insta::kHeavyFanout) heavy_slot[k] = nheavy++;
-    d.max_fanin = std::max(d.max_fanin, h.fanin_ptr[k + 1] - h.fanin_ptr[k]);
+    max_fanin = std::max(max_fanin, h.fanin_ptr[k + 1] - h.fanin_ptr[k]);
+  }
+  if (max_fanin >= 32768) {
+    delete G;
+    return fail(INSTA_E_ARG, "graph_create: a pin has >= 32768 fanin arcs");
   }
   d.num_heavy = nheavy;
   for (int64_t q = 0; q < E; ++q) {
@@ -167,12 +171,23 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
     const int32_t src = h.pos[desc->arc_from[a]];
     arc_pos[a] = int32_t(q);
     arc_sink[a] = h.pos[desc->arc_to[a]];
-    fin_src[q] = src | ((heavy_slot[src] >= 0 ? 1 : 0) << 29) |
+    fin_src[q] = src | ((heavy_slot[src] >= 0 ? 1 : 0) << insta::kHeavyBit) |
                  int32_t(uint32_t(desc->arc_unate[a]) << insta::kUnateShift);
     fin_ms[q] = make_float4(desc->arc_mean[2 * a], desc->arc_mean[2 * a + 1],
                             desc->arc_sigma[2 * a], desc->arc_sigma[2 * a + 1]);
   }
-  for (int64_t k = 0; k < E; ++k) fout[k] = arc_pos[h.fanout_arc[k]];
+  // light fanout CSR (rows of heavy drivers left empty) and full fanout sinks
+  std::vector<int32_t> lfo_ptr(nN + 1, 0), lfo;
+  lfo.reserve(nE);
+  for (int32_t k = 0; k < n; ++k) {
+    for (int32_t r = h.fanout_ptr[k]; r < h.fanout_ptr[k + 1]; ++r) {
+      const int32_t a = h.fanout_arc[r];
+      fout_sink[r] = arc_sink[a];
+      if (heavy_slot[k] < 0) lfo.push_back(arc_pos[a]);
+    }
+    lfo_ptr[k + 1] = int32_t(lfo.size());
+  }
+  d.e_light = int64_t(lfo.size());
   std::vector<float4> src_ms(size_t(std::max(d.num_src, 1)));
   for (int32_t i = 0; i < d.num_src; ++i) {
     const int32_t p = h.order[i];
@@ -187,57 +202,56 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
     ep_pin[k] = h.pos[desc->ep_pin[k]];
     ep_rat[k] = make_float2(desc->ep_rat[2 * k], desc->ep_rat[2 * k + 1]);
   }
-  // tiles of kTile canonical pins and the levels they span
-  std::vector<int2> tile_lv(size_t(std::max(d.num_tiles, 1)));
-  std::vector<int32_t> level_ntiles(size_t(std::max(d.num_levels, 1)), 0);
-  for (int32_t t = 0; t < d.num_tiles; ++t) {
-    const int32_t first = t * insta::kTile;
-    const int32_t last = std::min(n, first + insta::kTile) - 1;
-    tile_lv[t] = make_int2(h.level[h.order[first]], h.level[h.order[last]]);
-    for (int l = tile_lv[t].x; l <= tile_lv[t].y; ++l) level_ntiles[l]++;
-  }
   std::vector<uint8_t> arc_class(nE, 0);
   if (desc->arc_class) std::copy(desc->arc_class, desc->arc_class + E, arc_class.begin());
 
-  // ---- device upload ----------------------------------------------------------
+  // ---- device: grid, items, upload ------------------------------------------------
   cudaError_t e = cudaSetDevice(d.device);
+  if (e == cudaSuccess) e = static_cast<cudaError_t>(insta::query_grid(d.device, &d.grid));
+  if (e == cudaSuccess) insta::build_items(d, lfo_ptr);
 #define UP(dst, src, cnt)                       \
   if (e == cudaSuccess) e = upload(&(dst), (src), size_t(cnt));
 #define ZERO(dst, cnt) \
   if (e == cudaSuccess) e = alloc_zero(&(dst), size_t(cnt));
   UP(d.level_ptr, h.level_ptr.data(), h.level_ptr.size());
-  UP(d.tile_lv, tile_lv.data(), tile_lv.size());
-  UP(d.level_ntiles, level_ntiles.data(), level_ntiles.size());
-  ZERO(d.done_fwd, std::max(d.num_levels, 1));
-  ZERO(d.done_bwd, std::max(d.num_levels, 1));
-  UP(d.heavy_slot, heavy_slot.data(), heavy_slot.size());
-  ZERO(d.heavy_acc, 2 * std::max(nheavy, 1));
   UP(d.fanin_ptr, h.fanin_ptr.data(), h.fanin_ptr.size());
-  UP(d.fin_src, fin_src.data(), fin_src.size());
-  UP(d.fin_ms, fin_ms.data(), fin_ms.size());
-  UP(d.fin_arc, h.fanin_arc.data(), h.fanin_arc.size());
+  UP(d.fin_src, fin_src.data(), nE);
+  UP(d.fin_ms, fin_ms.data(), nE);
+  UP(d.fin_arc, h.fanin_arc.data(), nE);
+  UP(d.lfo_ptr, lfo_ptr.data(), lfo_ptr.size());
+  UP(d.lfo, lfo.data(), lfo.size());
   UP(d.fanout_ptr, h.fanout_ptr.data(), h.fanout_ptr.size());
-  UP(d.fout, fout.data(), fout.size());
-  UP(d.arc_pos, arc_pos.data(), arc_pos.size());
-  UP(d.arc_sink, arc_sink.data(), arc_sink.size());
-  UP(d.order, h.order.data(), h.order.size());
+  UP(d.fout_sink, fout_sink.data(), nE);
+  UP(d.heavy_slot, heavy_slot.data(), nN);
+  ZERO(d.heavy_acc, 2 * std::max(nheavy, 1));
+  UP(d.arc_pos, arc_pos.data(), nE);
+  UP(d.arc_sink, arc_sink.data(), nE);
+  UP(d.order, h.order.data(), nN);
   UP(d.src_ms, src_ms.data(), src_ms.size());
   UP(d.ep_pin, ep_pin.data(), ep_pin.size());
   UP(d.ep_rat, ep_rat.data(), ep_rat.size());
-  UP(d.arc_class, arc_class.data(), arc_class.size());
-  ZERO(d.state, n);
-  ZERO(d.g, E);
-  ZERO(d.seed, n);
+  UP(d.arc_class, arc_class.data(), nE);
+  UP(d.fwd_a, d.fwd_items.a.data(), d.fwd_items.a.size());
+  UP(d.fwd_b, d.fwd_items.b.data(), d.fwd_items.b.size());
+  UP(d.bwd_a, d.bwd_items.a.data(), d.bwd_items.a.size());
+  UP(d.bwd_b, d.bwd_items.b.data(), d.bwd_items.b.size());
+  ZERO(d.done_fwd, std::max(d.num_levels, 1));
+  ZERO(d.done_bwd, std::max(d.num_levels, 1));
+  ZERO(d.state, nN);
+  ZERO(d.win, nN);
+  ZERO(d.wts, nE);
+  ZERO(d.g, nE);
+  ZERO(d.seed, nN);
   ZERO(d.slack, d.num_ep);
   ZERO(d.rf_star, d.num_ep);
   ZERO(d.partials, 3 * ((d.num_ep + 255) / 256 + 1));
   ZERO(d.ticket, 1);
   ZERO(d.summary, 4);
+  ZERO(d.dirty, nN);
   ZERO(d.counters, 4);
 #undef UP
 #undef ZERO
   if (e == cudaSuccess) e = cudaDeviceSynchronize();
-  if (e == cudaSuccess) e = static_cast<cudaError_t>(insta::configure_grids(d));
   if (e != cudaSuccess) {
     insta_status s2 = cuda_fail(int(e), "graph_create");
     free_graph(d);
@@ -341,9 +355,9 @@ insta_status insta_arrivals(insta_graph* g, float* A, float* mean, float* sigma,
 insta_status insta_backward(insta_graph* g, const float* ep_seed, float* d_arc_mean,
                             float* d_arc_sigma, float* d_src, void* cuda_stream) {
   if (!g) return fail(INSTA_E_ARG, "backward: NULL graph");
-  if (!d_arc_mean) return fail(INSTA_E_ARG, "backward: d_arc_mean is required");
   if (d_arc_sigma) return fail(INSTA_E_ARG, "backward: d_arc_sigma is not supported (pass NULL)");
   insta::DevGraph& d = g->d;
+  if (!d_arc_mean && d.e > 0) return fail(INSTA_E_ARG, "backward: d_arc_mean is required");
   if (!d.fwd_valid) return fail(INSTA_E_STATE, "backward: no valid forward (call insta_forward)");
   cudaSetDevice(d.device);
   int err = insta::launch_backward(d, ep_seed, d_arc_mean, d_src, cuda_stream);

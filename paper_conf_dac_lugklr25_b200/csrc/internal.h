@@ -6,9 +6,17 @@
 // in canonical order ("fanin position" q), sorted by caller arc id within a
 // row; this is the order the forward walks (Alg 1 l.5-7 "outPin_parent_start").
 //
-// Per-pin state is float4 {mu_R, mu_F, sigma_R, sigma_F} (Eq 1-2 state; the
-// corner arrival A = mu + n_sigma*sigma of Eq 3 is formed on the fly), the
-// same layout as an arc record {arc_mean_R, arc_mean_F, arc_std_R, arc_std_F}.
+// Per-pin state is 32 bytes: {double mu_R, double mu_F, float sigma_R,
+// float sigma_F, pad} -- the Eq 1-2 state with the mean accumulated in fp64
+// (a random 32-byte gather costs one DRAM sector either way, and
+// fp64 means keep 15M-pin slacks within 1e-3 ps of the fp64 oracle).  Arc
+// records are float4 {arc_mean_R, arc_mean_F, arc_std_R, arc_std_F}.
+//
+// Work decomposition: every level is cut into `rounds x G`
+// contiguous pin chunks of balanced work (G = resident CTAs); chunk j of level
+// l is "item" (round j / G, CTA j % G).  Item descriptors are precomputed on
+// the host so a CTA can prefetch the next item's topology with TMA bulk copies
+// while it works on the current one.
 #pragma once
 #include <cstdint>
 #include <string>
@@ -21,10 +29,28 @@
 namespace insta {
 
 // fin_src word: bits 0..28 canonical source pin, bit 29 "source is a heavy
-// driver" (fanout > kHeavy), bits 30..31 unateness.  Hence num_pins < 2^29.
+// driver" (fanout > kHeavyFanout), bits 30..31 unateness.  num_pins < 2^29.
 constexpr int kUnateShift = 30;
-constexpr int kHeavyFanout = 128;
+constexpr int kHeavyBit = 29;
+constexpr int32_t kSrcMask = (1 << kHeavyBit) - 1;
 constexpr int32_t kMaxPins = (1 << 29) - 1;
+constexpr int kHeavyFanout = 256;
+
+// CTA shape and shared-memory stage capacities (per item)
+constexpr int kThreads = 1024;
+constexpr int kFwdPins = 2048, kFwdArcs = 2560;                     // forward item caps
+constexpr int kBwdPins = 1024, kBwdFanout = 2048, kBwdArcs = 2048;  // backward item caps
+static_assert(kHeavyFanout <= kBwdFanout, "a light pin's fanout row must fit one item");
+
+struct alignas(32) PinState {
+  double mu[2];
+  float sig[2];
+  float pad[2];
+};
+
+// item flags
+constexpr int kItemDirect = 1;   // does not fit the smem stage: read topology from global
+constexpr int kItemLast = 2;     // last round of its level: publish after it
 
 // Host result of levelization (canonical layout), also what export returns.
 struct HostLevels {
@@ -45,29 +71,34 @@ struct HostLevels {
 insta_status levelize_host(int32_t n, int64_t e, const int32_t* from, const int32_t* to,
                            HostLevels* out, std::string* err);
 
-// Tiles of the persistent dataflow kernels: TILE consecutive canonical pins.
-constexpr int kTile = 128;
+// Item table: step s of CTA c is entry s * G + c.
+//  forward:  a = {pin_lo, pin_hi, arc_lo, arc_hi}, b = {level, flags, 0, 0}
+//  backward: a = {pin_lo, pin_hi, lfo_lo, lfo_hi}, b = {arc_lo, arc_hi, level, flags}
+struct ItemTable {
+  int32_t num_steps = 0;
+  std::vector<int32_t> level_step0;  // [L] first step of each level (in table order)
+  std::vector<int32_t> level_steps;  // [L] rounds of each level
+  std::vector<int4> a, b;
+};
 
 struct DevGraph {
   int device = 0;
-  int32_t n = 0, num_levels = 0, num_src = 0, num_ep = 0, num_tiles = 0;
-  int64_t e = 0;
-  int max_fanin = 0;
-  // topology (canonical)
+  int32_t n = 0, num_levels = 0, num_src = 0, num_ep = 0;
+  int64_t e = 0, e_light = 0;
+  int grid = 0;                    // resident CTAs (cooperative grid)
+  // topology (canonical); every array is padded by >= 64 bytes for bulk copies
   int32_t* level_ptr = nullptr;    // [L+1]
-  int2* tile_lv = nullptr;         // [T] {level of first pin, level of last pin}
-  int32_t* level_ntiles = nullptr; // [L] tiles intersecting each level
-  uint32_t* done_fwd = nullptr;    // [L] level completion counters (forward)
-  uint32_t* done_bwd = nullptr;    // [L] level completion counters (backward)
+  int32_t* fanin_ptr = nullptr;    // [n+1]
+  int32_t* fin_src = nullptr;      // [e] canonical source | heavy << 29 | unate << 30
+  float4* fin_ms = nullptr;        // [e] {mean_R, mean_F, std_R, std_F}
+  int32_t* fin_arc = nullptr;      // [e] caller arc id
+  int32_t* lfo_ptr = nullptr;      // [n+1] light fanout rows (heavy drivers' rows empty)
+  int32_t* lfo = nullptr;          // [e_light] fanin position of each light fanout entry
+  int32_t* fanout_ptr = nullptr;   // [n+1] full fanout rows (incremental marking)
+  int32_t* fout_sink = nullptr;    // [e] canonical sink of each full fanout entry
   int32_t* heavy_slot = nullptr;   // [n] accumulator slot of heavy drivers, -1 otherwise
   unsigned long long* heavy_acc = nullptr;  // [num_heavy][2] fixed-point adjoints
   int32_t num_heavy = 0;
-  int32_t* fanin_ptr = nullptr;    // [n+1]
-  int32_t* fin_src = nullptr;      // [e] canonical source | unate << 30
-  float4* fin_ms = nullptr;        // [e] {mean_R, mean_F, std_R, std_F}
-  int32_t* fin_arc = nullptr;      // [e] caller arc id
-  int32_t* fanout_ptr = nullptr;   // [n+1]
-  int32_t* fout = nullptr;         // [e] fanin position of each fanout entry
   int32_t* arc_pos = nullptr;      // [e] caller arc id -> fanin position
   int32_t* arc_sink = nullptr;     // [e] caller arc id -> canonical sink
   int32_t* order = nullptr;        // [n] canonical -> caller pin
@@ -75,8 +106,18 @@ struct DevGraph {
   int32_t* ep_pin = nullptr;       // [P] canonical
   float2* ep_rat = nullptr;        // [P]
   uint8_t* arc_class = nullptr;    // [e] caller order (derates)
+  // item tables
+  int4* fwd_a = nullptr;
+  int4* fwd_b = nullptr;
+  int4* bwd_a = nullptr;
+  int4* bwd_b = nullptr;
+  ItemTable fwd_items, bwd_items;
+  uint32_t* done_fwd = nullptr;    // [L] level completion counters (forward)
+  uint32_t* done_bwd = nullptr;    // [L] level completion counters (backward)
   // state
-  float4* state = nullptr;         // [n]
+  PinState* state = nullptr;       // [n]
+  int32_t* win = nullptr;          // [n] hard-mode winners {R: k | s<<15, F: << 16}
+  float4* wts = nullptr;           // [e] LSE weights w[rf][s] per fanin arc
   float2* g = nullptr;             // [e] per-fanin-arc adjoint to its source's {R, F}
   float2* seed = nullptr;          // [n] endpoint seeds (zero at non-endpoints)
   float* slack = nullptr;          // [P]
@@ -85,14 +126,11 @@ struct DevGraph {
   uint32_t* ticket = nullptr;      // last-block ticket
   double* summary = nullptr;       // {wns, tns, nviol} on device
   // incremental
-  uint32_t* dirty = nullptr;       // [n] stamp: pin must be recomputed in pass `inc_epoch`
-  uint32_t* changed = nullptr;     // [n] stamp: pin state changed in pass `inc_epoch`
-  uint32_t* tile_dirty = nullptr;  // [T] stamp: tile holds a dirty pin / produced a change
+  uint32_t* dirty = nullptr;       // [n] stamp == inc_epoch: pin must be recomputed
   unsigned long long* counters = nullptr;  // [4] recomputed pins etc.
   // host-side bookkeeping
   HostLevels host;
-  uint32_t epoch_fwd = 0, epoch_bwd = 0, inc_epoch = 1;
-  int grid_fwd = 0, grid_bwd = 0, grid_inc = 0;
+  uint32_t epoch_fwd = 0, epoch_bwd = 0, inc_epoch = 0;
   int bwd_schedule = 0;            // schedule of the last forward (backward mirrors it)
   bool fwd_valid = false;          // a forward ran since the last update
   bool pending_incremental = false;
@@ -100,6 +138,9 @@ struct DevGraph {
   float last_n_sigma = 3.0f, last_tau = 0.0f;
   int64_t last_recomputed = 0;
 };
+
+// item tables (items.cpp)
+void build_items(DevGraph& d, const std::vector<int32_t>& lfo_ptr);
 
 }  // namespace insta
 
@@ -109,6 +150,7 @@ struct insta_graph {
 
 namespace insta {
 // kernels.cu launchers; return cudaError_t as int
+int query_grid(int device, int* grid);
 int launch_forward(DevGraph& g, float n_sigma, float tau, int schedule, void* stream);
 int launch_forward_incremental(DevGraph& g, float n_sigma, float tau, void* stream);
 int launch_slack(DevGraph& g, void* stream);
@@ -118,5 +160,4 @@ int launch_update_arcs(DevGraph& g, int64_t n, const int32_t* ids, const float* 
                        const float* sigma, int incremental, void* stream);
 int launch_arrivals(DevGraph& g, float* A, float* mean, float* sigma, void* stream);
 int launch_copy_slack(DevGraph& g, float* slack, uint8_t* rf, void* stream);
-int configure_grids(DevGraph& g);
 }  // namespace insta

@@ -2,65 +2,66 @@
 //
 //  * forward: statistical arrival propagation, Eq 1-3 with the
 //    Alg 1 / Alg 2 K = 1 merge (strict ">") or the LSE smooth max
-//    of Eq 4.  Thread per pin (Alg 1 l.3 "outPinID"), both rf in one
-//    pass, fanin rows read as one coalesced CSR slice (Alg 1 l.5-7).
+//    of Eq 4; both rf per pin in one pass (Alg 1 l.7).
 //  * slack / WNS / TNS: deterministic two-level fp64 reduction.
 //  * backward: Eq 6 softmax weights chained in reverse level order
-//    (P:L152).  Pull-style: a pin's adjoint is the sum of the per-arc adjoints
-//    its fanout sinks wrote (warp-cooperative segmented reduction over the
-//    warp's concatenated fanout rows; no float atomics).  High-fanout drivers
-//    (> kHeavy sinks) instead receive int64 fixed-point atomic adds from their
-//    sinks (order-independent, hence still deterministic).
+//    (P:L152).  The forward stores what the backward needs (hard mode: the
+//    arg-max candidate per pin and rf; LSE: the Eq 6 weights per fanin arc), so
+//    the backward never re-reads arrival states.  A pin's adjoint is pulled
+//    from the per-arc adjoints its fanout sinks wrote (no float atomics); very
+//    high-fanout drivers (> kHeavyFanout sinks) instead receive int64
+//    fixed-point atomic adds (order-independent, hence deterministic).
 //
-// Launch structure: the paper launches one kernel per timing
-// level.  Here the default is ONE persistent cooperative kernel per
-// pass: each CTA walks tiles of kTile consecutive canonical pins; before the
-// pins of level l are computed the CTA waits on a device counter until every
-// tile that intersects level l-1 has published (release/acquire), so the level
-// barrier is a per-CTA wait, not a grid-wide sync, and topology loads for the
-// next tile are issued before the wait.  schedule=1 keeps the per-level
-// launch chain for comparison; both call the same __device__ pin functions
-// with the same warp alignment, so they are bit-identical.
+// Execution.  The paper launches one kernel per timing level
+// (P:L113).  Here one persistent cooperative kernel per pass runs every level:
+// each level is pre-cut into balanced contiguous pin chunks ("items"), one per
+// resident CTA per round.  While a CTA works on item k, one thread has already
+// issued TMA bulk copies (cp.async.bulk + mbarrier) that stage item k+1's CSR
+// slice (row pointers, source ids, arc mean/sigma, weights) in shared memory.
+// The level dependency is a per-level device counter: a CTA publishes level l
+// with fence.acq_rel + red.relaxed after its last item of l, and waits with
+// ld.acquire before its first item of l+1 -- no grid-wide barrier, and CTAs
+// with no pins in a level never wait.  After the wait the only random accesses
+// are the source-state gathers (forward) / per-arc adjoint gathers (backward),
+// issued arc-parallel by all 1024 threads into shared memory.
 //
-// Arithmetic: fp32, IEEE sqrt/div/exp/log, compiled with --fmad=false so that
-// every kernel evaluates a candidate with the same rounding (bitwise
-// reproducible; incremental == full).
+// schedule = 1 launches the same item code once per level (no counters); both
+// schedules are bit-identical.  Arithmetic: fp64 means, fp32 sigmas, IEEE
+// sqrt/div/exp/log, --fmad=false: deterministic and bit-reproducible.
 #include <cuda_runtime.h>
 
-#include <cfloat>
-#include <cmath>
 #include <algorithm>
+#include <cmath>
 #include <cstdint>
 
 #include "internal.h"
 
 namespace insta {
 
-constexpr int kMaxF = 4;          // fanin arcs cached in registers per pin
-constexpr int kHeavy = kHeavyFanout;  // fanout above which a driver uses atomic accumulation
-constexpr int kHeavyBit = 29;     // fin_src bit: the source pin is a heavy driver
-constexpr int32_t kSrcMask = (1 << kHeavyBit) - 1;
-constexpr double kFix = 4294967296.0;  // 2^32 fixed-point scale of heavy accumulators
+constexpr double kFix = 4294967296.0;  // 2^32: fixed-point scale of heavy accumulators
 
 struct KParams {
-  int32_t n, num_tiles, num_levels, num_src, num_ep;
-  const int32_t* __restrict__ level_ptr;
-  const int2* __restrict__ tile_lv;       // {first level, last level} of each tile
-  const int32_t* __restrict__ level_ntiles;
+  int32_t n, num_levels, grid;
+  int32_t step_begin, step_end;  // item steps this launch runs
+  int32_t wait;                  // 1 = persistent (level counters), 0 = per-level launch
+  const int4* __restrict__ item_a;
+  const int4* __restrict__ item_b;
   const int32_t* __restrict__ fanin_ptr;
   const int32_t* __restrict__ fin_src;
   const float4* __restrict__ fin_ms;
   const int32_t* __restrict__ fin_arc;
-  const int32_t* __restrict__ fanout_ptr;
-  const int32_t* __restrict__ fout;       // fanin position of each fanout entry
-  const int32_t* __restrict__ heavy_slot; // [n] slot of heavy drivers, -1 otherwise
+  const int32_t* __restrict__ lfo_ptr;
+  const int32_t* __restrict__ lfo;
+  const int32_t* __restrict__ heavy_slot;
   const float4* __restrict__ src_ms;
   const int32_t* __restrict__ order;
-  float4* state;
+  PinState* state;
+  int32_t* win;
+  float4* wts;
   float2* g;
   const float2* seed;
-  unsigned long long* heavy_acc;          // [slots][2] fixed point
-  uint32_t* done;                         // [L] per-level completion counters
+  unsigned long long* heavy_acc;
+  uint32_t* done;
   float* d_mean;
   float* d_src;
   float n_sigma, tau;
@@ -68,467 +69,518 @@ struct KParams {
 };
 
 // --------------------------------------------------------------------------
-// memory-model helpers
+// PTX helpers: memory model, mbarrier, TMA bulk copy
 // --------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
 __device__ __forceinline__ uint32_t ld_acquire(const uint32_t* p) {
   uint32_t v;
   asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
 
-// Thread 0 of the CTA waits until level `l` has been published by all tiles
-// that intersect it in pass `epoch`, then the CTA proceeds.
-__device__ __forceinline__ void cta_wait_level(const KParams& P, int l) {
-  if (threadIdx.x == 0) {
-    const uint32_t target = P.epoch * uint32_t(P.level_ntiles[l]);
-    if (ld_acquire(P.done + l) != target) {
-      int ns = 20;
-      while (ld_acquire(P.done + l) != target) {
-        __nanosleep(ns);
-        ns = ns < 160 ? ns * 2 : 160;
-      }
-    }
-    __threadfence();
-  }
-  __syncthreads();
+__device__ __forceinline__ void red_release(uint32_t* p) {
+  asm volatile("fence.acq_rel.gpu;\n\tred.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(p) : "memory");
 }
 
-__device__ __forceinline__ void cta_publish_level(const KParams& P, int l) {
-  __syncthreads();
+__device__ __forceinline__ void mbar_init(uint64_t* bar) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(bar)) : "memory");
+}
+
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAIT_%=;\n}" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+
+__device__ __forceinline__ void bulk_g2s(void* sdst, const void* gsrc, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(sdst)),
+      "l"(gsrc), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+// 16-byte aligned window covering elements [a, b) of an array of esz-byte items
+struct Window {
+  int32_t off;     // element offset of a inside the window
+  uint32_t bytes;  // bytes to copy
+  int64_t start;   // first element copied
+};
+
+__device__ __forceinline__ Window window(int64_t a, int64_t b, int esz) {
+  const int per = 16 / esz;
+  Window w;
+  w.start = a - (a % per);
+  const int64_t end = ((b + per - 1) / per) * per;
+  w.off = int32_t(a - w.start);
+  w.bytes = b > a ? uint32_t((end - w.start) * esz) : 0u;
+  return w;
+}
+
+// Level dependency: thread 0 spins on the counter, then the CTA proceeds.
+__device__ __forceinline__ void wait_level(const KParams& P, int l) {
   if (threadIdx.x == 0) {
-    __threadfence();
-    atomicAdd(P.done + l, 1u);
+    const uint32_t target = P.epoch * uint32_t(P.grid);
+    while (ld_acquire(P.done + l) != target) __nanosleep(20);
   }
+  __syncthreads();
 }
 
 // --------------------------------------------------------------------------
-// Eq 1-3 for one candidate.  st/ms layout {mu_R, mu_F, sig_R, sig_F}.
+// Eq 1-3 for one candidate: arc e = (j -> i), sink transition rf, source
+// transition s.
 //   mu_c  = mu_j[s] + arc_mean[rf]                 (Eq 1, Alg 1 l.12)
 //   sig_c = sqrt(sig_j[s]^2 + arc_std[rf]^2)       (Eq 2, Alg 1 l.13)
 //   A_c   = mu_c + n_sigma * sig_c                 (Eq 3, Alg 1 l.14)
 // --------------------------------------------------------------------------
-struct Cand {
-  float mu, sig, A;
+struct Gath {
+  double mu0, mu1;
+  float s0, s1;
 };
 
-__device__ __forceinline__ float comp_mu(const float4& v, int s) { return s ? v.y : v.x; }
-__device__ __forceinline__ float comp_sig(const float4& v, int s) { return s ? v.w : v.z; }
+struct Cand {
+  double mu, A;
+  float sig;
+};
 
-__device__ __forceinline__ Cand make_cand(const float4& sj, const float4& ms, int rf, int s,
-                                          float ns) {
+__device__ __forceinline__ Gath load_state_cg(const PinState* p) {
+  const double2 m = __ldcg(reinterpret_cast<const double2*>(p));
+  const float2 s = __ldcg(reinterpret_cast<const float2*>(p) + 2);
+  Gath g;
+  g.mu0 = m.x;
+  g.mu1 = m.y;
+  g.s0 = s.x;
+  g.s1 = s.y;
+  return g;
+}
+
+__device__ __forceinline__ Cand make_cand(const Gath& st, const float4& ms, int rf, int s, double ns) {
+  const float sj = s ? st.s1 : st.s0;
+  const float se = rf ? ms.w : ms.z;
   Cand c;
-  const float sgj = comp_sig(sj, s), sge = comp_sig(ms, rf);
-  c.mu = comp_mu(sj, s) + comp_mu(ms, rf);
-  c.sig = sqrtf(sgj * sgj + sge * sge);
-  c.A = c.mu + ns * c.sig;
+  c.mu = (s ? st.mu1 : st.mu0) + double(rf ? ms.y : ms.x);
+  c.sig = sqrtf(sj * sj + se * se);
+  c.A = c.mu + ns * double(c.sig);
   return c;
 }
 
-// number of source transitions of an arc for sink transition rf, and the k-th
-// one: POS {rf}; NEG {~rf} (Alg 1 l.8); NON (rf, ~rf) (reading R3).
+// source transitions of an arc for sink transition rf: POS {rf}; NEG {~rf}
+// (Alg 1 l.8); NON (rf, ~rf) (reading R3).
 __device__ __forceinline__ int n_src_tr(int u) { return u == 2 ? 2 : 1; }
-__device__ __forceinline__ int src_tr(int rf, int u, int k) { return (u == 1 || k == 1) ? (rf ^ 1) : rf; }
+__device__ __forceinline__ int src_tr(int rf, int u, int a) { return (u == 1 || a == 1) ? (rf ^ 1) : rf; }
 
-// Per-pin fanin view: the first kMaxF arcs live in registers, the rest are
-// read from memory on demand (rare slow path for wide cells).
-struct Fanin {
-  int beg, nf;
-  int32_t src[kMaxF];
-  float4 ms[kMaxF];
-  float4 st[kMaxF];
-};
-
-__device__ __forceinline__ void fanin_load_topology(const KParams& P, int i, Fanin& F) {
-  F.beg = __ldg(P.fanin_ptr + i);
-  F.nf = __ldg(P.fanin_ptr + i + 1) - F.beg;
-#pragma unroll
-  for (int k = 0; k < kMaxF; ++k) {
-    if (k < F.nf) {
-      F.src[k] = __ldg(P.fin_src + F.beg + k);
-      F.ms[k] = __ldg(P.fin_ms + F.beg + k);
-    }
-  }
-}
-
-// Source states: written by this kernel in earlier levels, so read at L2 (.cg).
-template <bool kVolatileState>
-__device__ __forceinline__ void fanin_load_state(const KParams& P, Fanin& F) {
-#pragma unroll
-  for (int k = 0; k < kMaxF; ++k) {
-    if (k < F.nf) {
-      const float4* p = P.state + (F.src[k] & kSrcMask);
-      F.st[k] = kVolatileState ? __ldcg(p) : __ldg(p);
-    }
-  }
-}
-
-template <bool kVolatileState, class Fn>
-__device__ __forceinline__ void fanin_arc(const KParams& P, const Fanin& F, int k, Fn&& fn) {
-  if (k < kMaxF) {
-    fn(F.src[k], F.ms[k], F.st[k]);
-  } else {
-    const int32_t s = __ldg(P.fin_src + F.beg + k);
-    const float4 ms = __ldg(P.fin_ms + F.beg + k);
-    const float4* p = P.state + (s & kSrcMask);
-    const float4 st = kVolatileState ? __ldcg(p) : __ldg(p);
-    fn(s, ms, st);
-  }
-}
-
-// Visit the candidates of (pin, rf) in canonical order: fanin row order, then
-// source transition rf before ~rf.  fn(k, s, cand).
-template <bool kVolatileState, class Fn>
-__device__ __forceinline__ void for_each_cand(const KParams& P, const Fanin& F, int rf, Fn&& fn) {
-  const float ns = P.n_sigma;
-#pragma unroll
-  for (int k = 0; k < kMaxF; ++k) {
-    if (k < F.nf) {
-      const int u = int(uint32_t(F.src[k]) >> kUnateShift);
-      const int m = n_src_tr(u);
-      for (int a = 0; a < m; ++a) {
-        const int s = src_tr(rf, u, a);
-        fn(k, s, make_cand(F.st[k], F.ms[k], rf, s, ns));
-      }
-    }
-  }
-  for (int k = kMaxF; k < F.nf; ++k) {
-    fanin_arc<kVolatileState>(P, F, k, [&](int32_t srcw, const float4& ms, const float4& st) {
-      const int u = int(uint32_t(srcw) >> kUnateShift);
-      const int m = n_src_tr(u);
-      for (int a = 0; a < m; ++a) {
-        const int s = src_tr(rf, u, a);
-        fn(k, s, make_cand(st, ms, rf, s, ns));
-      }
-    });
-  }
-}
-
-// Merge result for one (pin, rf): first arg-max (strict ">") and, in LSE mode,
-// the log-sum-exp normalizer S = sum exp((A_c - M)/tau).
-struct Merge {
-  float M, mu_best, sig_best, S;
-  int k_best, s_best;
-};
-
-template <bool kLSE, bool kVolatileState>
-__device__ __forceinline__ Merge merge_pin(const KParams& P, const Fanin& F, int rf) {
-  Merge r;
-  r.M = -INFINITY;
-  r.mu_best = 0.f;
-  r.sig_best = 0.f;
-  r.k_best = -1;
-  r.s_best = 0;
-  r.S = 1.f;
-  for_each_cand<kVolatileState>(P, F, rf, [&](int k, int s, const Cand& c) {
-    if (r.k_best < 0 || c.A > r.M) {   // Alg 2 l.4: replace only if strictly greater
-      r.M = c.A;
-      r.mu_best = c.mu;
-      r.sig_best = c.sig;
-      r.k_best = k;
-      r.s_best = s;
-    }
-  });
-  if (kLSE) {
-    float S = 0.f;
-    const float tau = P.tau;
-    const float M = r.M;
-    for_each_cand<kVolatileState>(P, F, rf, [&](int, int, const Cand& c) { S += expf((c.A - M) / tau); });
-    r.S = S;
-  }
-  return r;
-}
-
-// Forward for one non-source pin; returns the new state.
-template <bool kLSE, bool kVolatileState>
-__device__ __forceinline__ float4 forward_pin(const KParams& P, const Fanin& F) {
-  float mu[2], sg[2];
+// Forward of one non-source pin i with nf fanin arcs (first at fanin position
+// q0); arc(k, srcw, ms, state) yields the k-th arc record and source state.
+template <bool kLSE, class ArcFn>
+__device__ __forceinline__ void fwd_pin(const KParams& P, int i, int nf, int q0, ArcFn&& arc) {
+  const double ns = double(P.n_sigma);
+  const double tau = double(P.tau);
+  double mu_out[2], M[2];
+  float sg_out[2], S[2];
+  int win = 0;
 #pragma unroll
   for (int rf = 0; rf < 2; ++rf) {
-    const Merge m = merge_pin<kLSE, kVolatileState>(P, F, rf);
-    sg[rf] = m.sig_best;
-    if (kLSE) {
-      // Eq 4: A_i = M + tau*log(sum exp((A_c - M)/tau)); reading R1: sigma_i =
-      // sigma of the arg-max, mu_i = A_i - n_sigma*sigma_i.
-      const float A = m.M + P.tau * logf(m.S);
-      mu[rf] = A - P.n_sigma * m.sig_best;
-    } else {
-      mu[rf] = m.mu_best;   // Alg 1 l.15 / Alg 2 l.6 with K = 1
-    }
-  }
-  return make_float4(mu[0], mu[1], sg[0], sg[1]);
-}
-
-__device__ __forceinline__ float4 source_state(const KParams& P, int i) {
-  // P:L62 clock arrival of a startpoint: its (mean, std) per rf.
-  return __ldg(P.src_ms + i);
-}
-
-// --------------------------------------------------------------------------
-// Forward: persistent cooperative kernel
-// --------------------------------------------------------------------------
-__device__ __forceinline__ int pin_level(const KParams& P, int i, int lvl0) {
-  int l = lvl0;
-  while (__ldg(P.level_ptr + l + 1) <= i) ++l;
-  return l;
-}
-
-template <bool kLSE>
-__global__ void __launch_bounds__(kTile) fwd_persistent(KParams P) {
-  for (int t = blockIdx.x; t < P.num_tiles; t += gridDim.x) {
-    const int i = t * kTile + threadIdx.x;
-    const bool valid = i < P.n;
-    const int2 lv = __ldg(P.tile_lv + t);
-    const int my_l = valid ? pin_level(P, i, lv.x) : -1;
-    Fanin F;
-    F.nf = 0;
-    if (valid && my_l > 0) fanin_load_topology(P, i, F);   // issued before the wait
-    for (int l = lv.x; l <= lv.y; ++l) {
-      if (l > 0) cta_wait_level(P, l - 1);
-      if (my_l == l) {
-        if (l == 0) {
-          P.state[i] = source_state(P, i);
-        } else {
-          fanin_load_state<true>(P, F);
-          P.state[i] = forward_pin<kLSE, true>(P, F);
+    double best = 0.0, bmu = 0.0;
+    float bsg = 0.f;
+    int bk = -1, bs = 0;
+    for (int k = 0; k < nf; ++k) {
+      int32_t w;
+      float4 ms;
+      Gath st;
+      arc(k, w, ms, st);
+      const int u = int(uint32_t(w) >> kUnateShift);
+      for (int a = 0; a < n_src_tr(u); ++a) {
+        const int s = src_tr(rf, u, a);
+        const Cand c = make_cand(st, ms, rf, s, ns);
+        if (bk < 0 || c.A > best) {   // Alg 2 l.4: replace only if strictly greater
+          best = c.A;
+          bmu = c.mu;
+          bsg = c.sig;
+          bk = k;
+          bs = s;
         }
       }
-      cta_publish_level(P, l);
     }
-  }
-}
-
-// One launch per level (schedule = 1): pins [lo, hi) of one level.
-template <bool kLSE>
-__global__ void __launch_bounds__(kTile) fwd_level(KParams P, int lo, int hi, int level) {
-  const int i = lo + blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= hi) return;
-  if (level == 0) {
-    P.state[i] = source_state(P, i);
-    return;
-  }
-  Fanin F;
-  fanin_load_topology(P, i, F);
-  fanin_load_state<false>(P, F);
-  P.state[i] = forward_pin<kLSE, false>(P, F);
-}
-
-// --------------------------------------------------------------------------
-// Backward
-// --------------------------------------------------------------------------
-// Warp-cooperative pull: lane's pin i in [seg_lo, seg_hi) owns fanout row
-// [row_beg, row_end) (empty for inactive lanes and heavy drivers).  The warp
-// walks the concatenated rows in chunks of 32 entries; each entry's owner is
-// found by a shuffle binary search and summed by a segmented shuffle scan;
-// segment tails accumulate into the owner lane.  Fixed order => deterministic.
-__device__ __forceinline__ float2 warp_pull(const KParams& P, int row_beg, int row_end) {
-  const unsigned full = 0xffffffffu;
-  const int lane = threadIdx.x & 31;
-  const int r0 = __shfl_sync(full, row_beg, 0);
-  const int r1 = __shfl_sync(full, row_end, 31);
-  float ax = 0.f, ay = 0.f;
-  for (int c = r0; c < r1; c += 32) {
-    const int k = c + lane;
-    // owner = last lane whose row_beg <= k (row_beg is non-decreasing over lanes)
-    int o = 0;
-#pragma unroll
-    for (int step = 16; step >= 1; step >>= 1) {
-      const int probe = o + step;
-      const int rb = __shfl_sync(full, row_beg, probe);
-      if (rb <= k) o = probe;
-    }
-    const int oend = __shfl_sync(full, row_end, o);
-    const bool live = k < oend;   // also false for k >= r1 and inside skipped rows
-    float vx = 0.f, vy = 0.f;
-    if (live) {
-      const float2 gv = __ldcg(P.g + __ldg(P.fout + k));
-      vx = gv.x;
-      vy = gv.y;
-    }
-    const int owner = live ? o : -1 - lane;   // dead entries are singleton segments
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      const float tx = __shfl_up_sync(full, vx, d);
-      const float ty = __shfl_up_sync(full, vy, d);
-      const int to = __shfl_up_sync(full, owner, d);
-      if (lane >= d && to == owner) {
-        vx += tx;
-        vy += ty;
+    M[rf] = best;
+    sg_out[rf] = bsg;
+    win |= (bk | (bs << 15)) << (16 * rf);
+    if (kLSE) {
+      // Eq 4: A_i = M + tau * log(sum_c exp((A_c - M) / tau)); reading R1:
+      // sigma_i = sigma of the arg-max, mu_i = A_i - n_sigma * sigma_i.
+      float sum = 0.f;
+      for (int k = 0; k < nf; ++k) {
+        int32_t w;
+        float4 ms;
+        Gath st;
+        arc(k, w, ms, st);
+        const int u = int(uint32_t(w) >> kUnateShift);
+        for (int a = 0; a < n_src_tr(u); ++a) {
+          const Cand c = make_cand(st, ms, rf, src_tr(rf, u, a), ns);
+          sum += expf(float((c.A - best) / tau));
+        }
       }
-    }
-    // each owner lane takes the inclusive-scan value at its last entry in this chunk
-    const int lo = max(row_beg, c), hi = min(row_end, c + 32);
-    const int tail = (hi - 1 - c) & 31;
-    const float sx = __shfl_sync(full, vx, tail);
-    const float sy = __shfl_sync(full, vy, tail);
-    if (hi > lo) {
-      ax += sx;
-      ay += sy;
+      S[rf] = sum;
+      mu_out[rf] = (best + tau * double(logf(sum))) - ns * double(bsg);
+    } else {
+      mu_out[rf] = bmu;   // Alg 1 l.15 / Alg 2 l.6 with K = 1
     }
   }
-  return make_float2(ax, ay);
+  PinState* o = P.state + i;
+  reinterpret_cast<double2*>(o)[0] = make_double2(mu_out[0], mu_out[1]);
+  reinterpret_cast<float4*>(o)[1] = make_float4(sg_out[0], sg_out[1], 0.f, 0.f);
+  if (!kLSE) {
+    P.win[i] = win;
+  } else {
+    // Eq 6 weights w[rf][s] of every candidate, stored per fanin arc
+    for (int k = 0; k < nf; ++k) {
+      int32_t w;
+      float4 ms;
+      Gath st;
+      arc(k, w, ms, st);
+      const int u = int(uint32_t(w) >> kUnateShift);
+      float wt[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
+#pragma unroll
+      for (int rf = 0; rf < 2; ++rf) {
+        for (int a = 0; a < n_src_tr(u); ++a) {
+          const int s = src_tr(rf, u, a);
+          const Cand c = make_cand(st, ms, rf, s, ns);
+          wt[rf][s] = expf(float((c.A - M[rf]) / tau)) / S[rf];
+        }
+      }
+      P.wts[q0 + k] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
+    }
+  }
 }
 
-// Backward for one pin i at level l (>0 => has fanin) with adjoint abar of its
-// corner arrival per rf (dL/dA_i = dL/dmu_i, reading R1).  Writes, for each
-// fanin arc q, g[q] = per-source-transition adjoint and d_mean[arc] (Eq 6
-// chain; hard mode: one-hot at the first arg-max).
+// --------------------------------------------------------------------------
+// Forward kernel
+// --------------------------------------------------------------------------
+struct FwdStage {
+  int32_t ptr[kFwdPins + 8];
+  int32_t src[kFwdArcs + 8];
+  float4 ms[kFwdArcs];
+};
+constexpr size_t kFwdSmem = 2 * sizeof(FwdStage) + sizeof(Gath) * kFwdArcs;
+
+__device__ __forceinline__ bool fwd_staged(const int4& A, const int4& B) {
+  return A.y > A.x && B.x > 0 && !(B.y & kItemDirect);
+}
+
+// thread 0: issue the bulk copies staging item (step, c) into `st`
+__device__ __forceinline__ void fwd_prefetch(const KParams& P, FwdStage* st, uint64_t* bar, int step,
+                                             int c) {
+  const int4 A = __ldg(P.item_a + size_t(step) * P.grid + c);
+  const int4 B = __ldg(P.item_b + size_t(step) * P.grid + c);
+  if (!fwd_staged(A, B)) return;
+  const Window wp = window(A.x, A.y + 1, 4);
+  const Window ws = window(A.z, A.w, 4);
+  const uint32_t bms = uint32_t(A.w - A.z) * 16u;
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  mbar_expect_tx(bar, wp.bytes + ws.bytes + bms);
+  bulk_g2s(st->ptr, P.fanin_ptr + wp.start, wp.bytes, bar);
+  if (ws.bytes) bulk_g2s(st->src, P.fin_src + ws.start, ws.bytes, bar);
+  if (bms) bulk_g2s(st->ms, P.fin_ms + A.z, bms, bar);
+}
+
 template <bool kLSE>
-__device__ __forceinline__ void backward_fanin(const KParams& P, int i, float2 abar) {
-  Fanin F;
-  fanin_load_topology(P, i, F);
-  if (abar.x == 0.f && abar.y == 0.f) {
-    for (int k = 0; k < F.nf; ++k) P.g[F.beg + k] = make_float2(0.f, 0.f);
-    return;   // d_mean was zero-filled by the launcher
+__global__ void __launch_bounds__(kThreads, 1) fwd_kernel(KParams P) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  FwdStage* stage = reinterpret_cast<FwdStage*>(smem);
+  Gath* gath = reinterpret_cast<Gath*>(smem + 2 * sizeof(FwdStage));
+  __shared__ __align__(8) uint64_t bar[2];
+  const int c = blockIdx.x;
+  const int tid = threadIdx.x;
+  if (tid == 0) {
+    mbar_init(&bar[0]);
+    mbar_init(&bar[1]);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  fanin_load_state<false>(P, F);
-  float gs[kMaxF][2], gm[kMaxF][2];
-#pragma unroll
-  for (int k = 0; k < kMaxF; ++k) gs[k][0] = gs[k][1] = gm[k][0] = gm[k][1] = 0.f;
-  const bool wide = F.nf > kMaxF;
-#pragma unroll
-  for (int rf = 0; rf < 2; ++rf) {
-    const float ab = rf ? abar.y : abar.x;
-    if (ab == 0.f) continue;
-    const Merge m = merge_pin<kLSE, false>(P, F, rf);
-    const float tau = P.tau, M = m.M, S = m.S;
-    for_each_cand<false>(P, F, rf, [&](int k, int s, const Cand& c) {
-      float w;
-      if (kLSE) {
-        w = expf((c.A - M) / tau) / S;                    // Eq 6
+  __syncthreads();
+  uint32_t phase0 = 0, phase1 = 0;
+  int waited = -1;
+  if (tid == 0 && P.step_begin < P.step_end) fwd_prefetch(P, &stage[0], &bar[0], P.step_begin, c);
+  for (int k = P.step_begin; k < P.step_end; ++k) {
+    const int buf = (k - P.step_begin) & 1;
+    const int4 A = __ldg(P.item_a + size_t(k) * P.grid + c);   // {pin_lo, pin_hi, arc_lo, arc_hi}
+    const int4 B = __ldg(P.item_b + size_t(k) * P.grid + c);   // {level, flags}
+    const int l = B.x;
+    if (tid == 0 && k + 1 < P.step_end) fwd_prefetch(P, &stage[buf ^ 1], &bar[buf ^ 1], k + 1, c);
+    if (A.y > A.x) {
+      if (l == 0) {
+        // startpoints: clock arrival distribution, mean and std per rf
+        for (int i = A.x + tid; i < A.y; i += kThreads) {
+          const float4 s = __ldg(P.src_ms + i);
+          PinState* o = P.state + i;
+          reinterpret_cast<double2*>(o)[0] = make_double2(double(s.x), double(s.y));
+          reinterpret_cast<float4*>(o)[1] = make_float4(s.z, s.w, 0.f, 0.f);
+        }
+      } else if (!(B.y & kItemDirect)) {
+        if (buf == 0) {
+          mbar_wait(&bar[0], phase0);
+          phase0 ^= 1;
+        } else {
+          mbar_wait(&bar[1], phase1);
+          phase1 ^= 1;
+        }
+        if (P.wait && waited != l) {
+          wait_level(P, l - 1);
+          waited = l;
+        }
+        const FwdStage& S = stage[buf];
+        const int po = A.x & 3, so = A.z & 3;
+        const int na = A.w - A.z;
+        for (int a = tid; a < na; a += kThreads)
+          gath[a] = load_state_cg(P.state + (S.src[so + a] & kSrcMask));
+        __syncthreads();
+        for (int p = tid; p < A.y - A.x; p += kThreads) {
+          const int b0 = S.ptr[po + p] - A.z;
+          const int b1 = S.ptr[po + p + 1] - A.z;
+          fwd_pin<kLSE>(P, A.x + p, b1 - b0, A.z + b0,
+                        [&](int kk, int32_t& w, float4& ms, Gath& st) {
+                          w = S.src[so + b0 + kk];
+                          ms = S.ms[b0 + kk];
+                          st = gath[b0 + kk];
+                        });
+        }
       } else {
-        w = (k == m.k_best && s == m.s_best) ? 1.f : 0.f; // hard: one-hot at c*
+        if (P.wait && waited != l) {
+          wait_level(P, l - 1);
+          waited = l;
+        }
+        for (int i = A.x + tid; i < A.y; i += kThreads) {
+          const int b0 = __ldg(P.fanin_ptr + i), b1 = __ldg(P.fanin_ptr + i + 1);
+          fwd_pin<kLSE>(P, i, b1 - b0, b0, [&](int kk, int32_t& w, float4& ms, Gath& st) {
+            w = __ldg(P.fin_src + b0 + kk);
+            ms = __ldg(P.fin_ms + b0 + kk);
+            st = load_state_cg(P.state + (w & kSrcMask));
+          });
+        }
       }
-      const float a = w * ab;
-      if (k < kMaxF) {
+    }
+    __syncthreads();
+    if ((B.y & kItemLast) && P.wait && tid == 0) red_release(P.done + l);
+  }
+}
+
+// --------------------------------------------------------------------------
+// Backward kernel
+// --------------------------------------------------------------------------
+struct BwdStage {
+  int32_t lptr[kBwdPins + 8];   // light fanout row pointers
+  int32_t lfo[kBwdFanout + 8];  // fanin position of each light fanout entry
+  int32_t fptr[kBwdPins + 8];   // fanin row pointers
+  int32_t src[kBwdArcs + 8];    // fin_src
+  int32_t arc[kBwdArcs + 8];    // caller arc ids
+  int32_t win[kBwdPins + 8];    // hard-mode winners
+  float2 seed[kBwdPins + 8];
+  float4 wts[kBwdArcs];         // LSE weights
+};
+constexpr size_t kBwdSmem = 2 * sizeof(BwdStage) + sizeof(float2) * kBwdFanout;
+
+__device__ __forceinline__ bool bwd_staged(const int4& A, const int4& B) {
+  return A.y > A.x && !(B.w & kItemDirect);
+}
+
+template <bool kLSE>
+__device__ __forceinline__ void bwd_prefetch(const KParams& P, BwdStage* st, uint64_t* bar, int step,
+                                             int c) {
+  const int4 A = __ldg(P.item_a + size_t(step) * P.grid + c);   // {pin_lo, pin_hi, lfo_lo, lfo_hi}
+  const int4 B = __ldg(P.item_b + size_t(step) * P.grid + c);   // {arc_lo, arc_hi, level, flags}
+  if (!bwd_staged(A, B)) return;
+  const Window wl = window(A.x, A.y + 1, 4);   // lfo_ptr and fanin_ptr: same pin window
+  const Window wf = window(A.z, A.w, 4);
+  const Window wa = window(B.x, B.y, 4);
+  const Window wsd = window(A.x, A.y, 8);
+  const Window ww = window(A.x, A.y, 4);
+  const uint32_t bw = kLSE ? uint32_t(B.y - B.x) * 16u : 0u;
+  const uint32_t total = 2 * wl.bytes + wf.bytes + 2 * wa.bytes + wsd.bytes + (kLSE ? bw : ww.bytes);
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  mbar_expect_tx(bar, total);
+  bulk_g2s(st->lptr, P.lfo_ptr + wl.start, wl.bytes, bar);
+  if (wf.bytes) bulk_g2s(st->lfo, P.lfo + wf.start, wf.bytes, bar);
+  bulk_g2s(st->fptr, P.fanin_ptr + wl.start, wl.bytes, bar);
+  if (wa.bytes) {
+    bulk_g2s(st->src, P.fin_src + wa.start, wa.bytes, bar);
+    bulk_g2s(st->arc, P.fin_arc + wa.start, wa.bytes, bar);
+  }
+  bulk_g2s(st->seed, P.seed + wsd.start, wsd.bytes, bar);
+  if (kLSE) {
+    if (bw) bulk_g2s(st->wts, P.wts + B.x, bw, bar);
+  } else {
+    bulk_g2s(st->win, P.win + ww.start, ww.bytes, bar);
+  }
+}
+
+__device__ __forceinline__ void heavy_add(const KParams& P, int32_t srcw, float gx, float gy) {
+  if (!((srcw >> kHeavyBit) & 1)) return;
+  const int slot = __ldg(P.heavy_slot + (srcw & kSrcMask));
+  if (gx != 0.f) atomicAdd(P.heavy_acc + 2 * slot, (unsigned long long)__double2ll_rn(double(gx) * kFix));
+  if (gy != 0.f) atomicAdd(P.heavy_acc + 2 * slot + 1, (unsigned long long)__double2ll_rn(double(gy) * kFix));
+}
+
+// Sink side of a pin (nf fanin arcs from fanin position q0) with adjoint ab:
+// per arc, g = adjoint to the source's {R, F} and dL/d(arc mean) (Eq 6 chain;
+// hard mode: one-hot at the recorded arg-max).
+template <bool kLSE, class ArcFn>
+__device__ __forceinline__ void bwd_sink(const KParams& P, int nf, int q0, float2 ab, int32_t win,
+                                         ArcFn&& arc) {
+  const float abr[2] = {ab.x, ab.y};
+  for (int k = 0; k < nf; ++k) {
+    int32_t srcw, arcid;
+    float4 w4;
+    arc(k, srcw, arcid, w4);
+    float w[2][2];
+    if (kLSE) {
+      w[0][0] = w4.x;
+      w[0][1] = w4.y;
+      w[1][0] = w4.z;
+      w[1][1] = w4.w;
+    } else {
 #pragma unroll
-        for (int kk = 0; kk < kMaxF; ++kk) {
-          if (kk == k) {
-            gm[kk][rf] += a;
-            gs[kk][s] += a;
+      for (int rf = 0; rf < 2; ++rf) {
+        const int wv = (win >> (16 * rf)) & 0xffff;
+        const bool hit = (wv & 0x7fff) == k;
+        w[rf][0] = (hit && (wv >> 15) == 0) ? 1.f : 0.f;
+        w[rf][1] = (hit && (wv >> 15) == 1) ? 1.f : 0.f;
+      }
+    }
+    float gm[2], gs[2] = {0.f, 0.f};
+#pragma unroll
+    for (int rf = 0; rf < 2; ++rf) {
+      const float a0 = w[rf][0] * abr[rf], a1 = w[rf][1] * abr[rf];
+      gm[rf] = a0 + a1;
+      gs[0] += a0;
+      gs[1] += a1;
+    }
+    P.g[q0 + k] = make_float2(gs[0], gs[1]);
+    if (gm[0] != 0.f || gm[1] != 0.f)
+      reinterpret_cast<float2*>(P.d_mean)[arcid] = make_float2(gm[0], gm[1]);
+    heavy_add(P, srcw, gs[0], gs[1]);
+  }
+}
+
+__device__ __forceinline__ float2 heavy_take(const KParams& P, int i) {
+  const int slot = __ldg(P.heavy_slot + i);
+  if (slot < 0) return make_float2(0.f, 0.f);
+  // every sink of i is at a deeper, completed level: read and reset
+  const long long hx = (long long)atomicExch(P.heavy_acc + 2 * slot, 0ull);
+  const long long hy = (long long)atomicExch(P.heavy_acc + 2 * slot + 1, 0ull);
+  return make_float2(float(double(hx) / kFix), float(double(hy) / kFix));
+}
+
+template <bool kLSE>
+__global__ void __launch_bounds__(kThreads, 1) bwd_kernel(KParams P) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  BwdStage* stage = reinterpret_cast<BwdStage*>(smem);
+  float2* gg = reinterpret_cast<float2*>(smem + 2 * sizeof(BwdStage));
+  __shared__ __align__(8) uint64_t bar[2];
+  const int c = blockIdx.x;
+  const int tid = threadIdx.x;
+  if (tid == 0) {
+    mbar_init(&bar[0]);
+    mbar_init(&bar[1]);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  uint32_t phase0 = 0, phase1 = 0;
+  int waited = -1;
+  if (tid == 0 && P.step_begin < P.step_end) bwd_prefetch<kLSE>(P, &stage[0], &bar[0], P.step_begin, c);
+  for (int k = P.step_begin; k < P.step_end; ++k) {
+    const int buf = (k - P.step_begin) & 1;
+    const int4 A = __ldg(P.item_a + size_t(k) * P.grid + c);   // {pin_lo, pin_hi, lfo_lo, lfo_hi}
+    const int4 B = __ldg(P.item_b + size_t(k) * P.grid + c);   // {arc_lo, arc_hi, level, flags}
+    const int l = B.z;
+    if (tid == 0 && k + 1 < P.step_end) bwd_prefetch<kLSE>(P, &stage[buf ^ 1], &bar[buf ^ 1], k + 1, c);
+    if (A.y > A.x) {
+      const bool wait_needed = P.wait && l + 1 < P.num_levels && waited != l;
+      if (!(B.w & kItemDirect)) {
+        if (buf == 0) {
+          mbar_wait(&bar[0], phase0);
+          phase0 ^= 1;
+        } else {
+          mbar_wait(&bar[1], phase1);
+          phase1 ^= 1;
+        }
+        if (wait_needed) {
+          wait_level(P, l + 1);
+          waited = l;
+        }
+        const BwdStage& S = stage[buf];
+        const int lo = A.x & 3, fo = A.z & 3, ao = B.x & 3, so = A.x & 1;
+        const int nfo = A.w - A.z;
+        for (int e = tid; e < nfo; e += kThreads) gg[e] = __ldcg(P.g + S.lfo[fo + e]);
+        __syncthreads();
+        for (int p = tid; p < A.y - A.x; p += kThreads) {
+          const int i = A.x + p;
+          // pull: seed + sum of the sinks' per-arc adjoints (+ heavy accumulator)
+          const int r0 = S.lptr[lo + p] - A.z, r1 = S.lptr[lo + p + 1] - A.z;
+          float2 ab = S.seed[so + p];
+          float sx = 0.f, sy = 0.f;
+          for (int r = r0; r < r1; ++r) {
+            sx += gg[r].x;
+            sy += gg[r].y;
+          }
+          const float2 h = heavy_take(P, i);
+          ab.x += sx + h.x;
+          ab.y += sy + h.y;
+          if (l == 0) {
+            if (P.d_src) reinterpret_cast<float2*>(P.d_src)[__ldg(P.order + i)] = ab;
+          } else {
+            const int b0 = S.fptr[lo + p] - B.x, b1 = S.fptr[lo + p + 1] - B.x;
+            bwd_sink<kLSE>(P, b1 - b0, B.x + b0, ab, S.win[lo + p],
+                           [&](int kk, int32_t& srcw, int32_t& arcid, float4& w4) {
+                             srcw = S.src[ao + b0 + kk];
+                             arcid = S.arc[ao + b0 + kk];
+                             if (kLSE) w4 = S.wts[b0 + kk];
+                           });
+          }
+        }
+      } else {
+        if (wait_needed) {
+          wait_level(P, l + 1);
+          waited = l;
+        }
+        for (int i = A.x + tid; i < A.y; i += kThreads) {
+          float2 ab = P.seed[i];
+          float sx = 0.f, sy = 0.f;
+          const int r0 = __ldg(P.lfo_ptr + i), r1 = __ldg(P.lfo_ptr + i + 1);
+          for (int r = r0; r < r1; ++r) {
+            const float2 v = __ldcg(P.g + __ldg(P.lfo + r));
+            sx += v.x;
+            sy += v.y;
+          }
+          const float2 h = heavy_take(P, i);
+          ab.x += sx + h.x;
+          ab.y += sy + h.y;
+          if (l == 0) {
+            if (P.d_src) reinterpret_cast<float2*>(P.d_src)[__ldg(P.order + i)] = ab;
+          } else {
+            const int b0 = __ldg(P.fanin_ptr + i), b1 = __ldg(P.fanin_ptr + i + 1);
+            bwd_sink<kLSE>(P, b1 - b0, b0, ab, kLSE ? 0 : P.win[i],
+                           [&](int kk, int32_t& srcw, int32_t& arcid, float4& w4) {
+                             srcw = __ldg(P.fin_src + b0 + kk);
+                             arcid = __ldg(P.fin_arc + b0 + kk);
+                             if (kLSE) w4 = P.wts[b0 + kk];
+                           });
           }
         }
       }
-    });
-    (void)wide;
-  }
-#pragma unroll
-  for (int k = 0; k < kMaxF; ++k) {
-    if (k < F.nf) {
-      const int q = F.beg + k;
-      P.g[q] = make_float2(gs[k][0], gs[k][1]);
-      if (gm[k][0] != 0.f || gm[k][1] != 0.f)
-        reinterpret_cast<float2*>(P.d_mean)[__ldg(P.fin_arc + q)] = make_float2(gm[k][0], gm[k][1]);
-      if ((F.src[k] >> kHeavyBit) & 1) {
-        const int slot = __ldg(P.heavy_slot + (F.src[k] & kSrcMask));
-        if (gs[k][0] != 0.f)
-          atomicAdd(P.heavy_acc + 2 * slot, (unsigned long long)__double2ll_rn(double(gs[k][0]) * kFix));
-        if (gs[k][1] != 0.f)
-          atomicAdd(P.heavy_acc + 2 * slot + 1, (unsigned long long)__double2ll_rn(double(gs[k][1]) * kFix));
-      }
     }
+    __syncthreads();
+    if ((B.w & kItemLast) && P.wait && tid == 0) red_release(P.done + l);
   }
-  // slow path: arcs beyond the register cache, one at a time
-  for (int k = kMaxF; k < F.nf; ++k) {
-    float ks[2] = {0.f, 0.f}, km[2] = {0.f, 0.f};
-#pragma unroll
-    for (int rf = 0; rf < 2; ++rf) {
-      const float ab = rf ? abar.y : abar.x;
-      if (ab == 0.f) continue;
-      const Merge m = merge_pin<kLSE, false>(P, F, rf);
-      const float tau = P.tau, M = m.M, S = m.S;
-      for_each_cand<false>(P, F, rf, [&](int kc, int s, const Cand& c) {
-        if (kc != k) return;
-        const float w = kLSE ? expf((c.A - M) / tau) / S
-                             : ((kc == m.k_best && s == m.s_best) ? 1.f : 0.f);
-        const float a = w * ab;
-        km[rf] += a;
-        ks[s] += a;
-      });
-    }
-    const int q = F.beg + k;
-    const int32_t srcw = __ldg(P.fin_src + q);
-    P.g[q] = make_float2(ks[0], ks[1]);
-    if (km[0] != 0.f || km[1] != 0.f)
-      reinterpret_cast<float2*>(P.d_mean)[__ldg(P.fin_arc + q)] = make_float2(km[0], km[1]);
-    if ((srcw >> kHeavyBit) & 1) {
-      const int slot = __ldg(P.heavy_slot + (srcw & kSrcMask));
-      if (ks[0] != 0.f) atomicAdd(P.heavy_acc + 2 * slot, (unsigned long long)__double2ll_rn(double(ks[0]) * kFix));
-      if (ks[1] != 0.f) atomicAdd(P.heavy_acc + 2 * slot + 1, (unsigned long long)__double2ll_rn(double(ks[1]) * kFix));
-    }
-  }
-}
-
-// Adjoint of pin i (seg_lo <= i < seg_hi are this warp's pins of the current
-// level; lanes outside contribute empty rows): seed + pulled fanout sum, or
-// the heavy accumulator for high-fanout drivers.
-__device__ __forceinline__ float2 pin_adjoint(const KParams& P, int i, bool active, int seg_lo,
-                                              int seg_hi) {
-  const int ci = min(max(i, seg_lo), seg_hi);
-  const int ci1 = min(max(i + 1, seg_lo), seg_hi);
-  int rb = __ldg(P.fanout_ptr + ci);
-  int re = __ldg(P.fanout_ptr + ci1);
-  int slot = -1;
-  if (active && re - rb > kHeavy) {
-    slot = __ldg(P.heavy_slot + i);
-    rb = re;   // skipped row (contributions arrive through the accumulator)
-  }
-  float2 a = warp_pull(P, rb, re);
-  if (!active) return make_float2(0.f, 0.f);
-  if (slot >= 0) {
-    // all sinks are at deeper, completed levels: read and reset the accumulator
-    unsigned long long* acc = P.heavy_acc + 2 * slot;
-    const long long hx = (long long)atomicExch(acc, 0ull);
-    const long long hy = (long long)atomicExch(acc + 1, 0ull);
-    a.x = float(double(hx) / kFix);
-    a.y = float(double(hy) / kFix);
-  }
-  const float2 sd = P.seed[i];
-  return make_float2(sd.x + a.x, sd.y + a.y);
-}
-
-template <bool kLSE>
-__device__ __forceinline__ void backward_pin(const KParams& P, int i, int l, float2 abar) {
-  if (l == 0) {
-    if (P.d_src) reinterpret_cast<float2*>(P.d_src)[__ldg(P.order + i)] = abar;
-  } else {
-    backward_fanin<kLSE>(P, i, abar);
-  }
-}
-
-template <bool kLSE>
-__global__ void __launch_bounds__(kTile) bwd_persistent(KParams P) {
-  for (int r = blockIdx.x; r < P.num_tiles; r += gridDim.x) {
-    const int t = P.num_tiles - 1 - r;
-    const int base = t * kTile;
-    const int i = base + threadIdx.x;
-    const bool valid = i < P.n;
-    const int2 lv = __ldg(P.tile_lv + t);
-    const int my_l = valid ? pin_level(P, i, lv.x) : -1;
-    const int wbase = base + (threadIdx.x & ~31);
-    for (int l = lv.y; l >= lv.x; --l) {
-      if (l + 1 < P.num_levels) cta_wait_level(P, l + 1);
-      const int seg_lo = max(__ldg(P.level_ptr + l), wbase);
-      const int seg_hi = max(min(__ldg(P.level_ptr + l + 1), wbase + 32), seg_lo);
-      const bool active = my_l == l;
-      const float2 abar = pin_adjoint(P, i, active, seg_lo, seg_hi);
-      if (active) backward_pin<kLSE>(P, i, l, abar);
-      cta_publish_level(P, l);
-    }
-  }
-}
-
-// One launch per level (schedule = 1).  Threads are aligned to global
-// multiples of 32 pins so that warps see the same pins as in bwd_persistent.
-template <bool kLSE>
-__global__ void __launch_bounds__(kTile) bwd_level(KParams P, int lo, int hi, int level) {
-  const int i = (lo & ~31) + blockIdx.x * blockDim.x + threadIdx.x;
-  const int wbase = i & ~31;
-  const int seg_lo = max(lo, wbase);
-  const int seg_hi = max(min(hi, wbase + 32), seg_lo);
-  const bool active = i >= lo && i < hi;
-  if (wbase >= hi) return;   // whole warp outside the level
-  const float2 abar = pin_adjoint(P, i, active, seg_lo, seg_hi);
-  if (active) backward_pin<kLSE>(P, i, level, abar);
 }
 
 // Endpoint seeds: dL/dA_ep[rf*] = -dL/dslack (slack = RAT - A); TNS: dL/dslack
@@ -551,7 +603,7 @@ constexpr int kRedThreads = 256;
 
 __global__ void __launch_bounds__(kRedThreads)
 slack_kernel(int num_ep, const int32_t* __restrict__ ep_pin, const float2* __restrict__ ep_rat,
-             const float4* __restrict__ state, float n_sigma, float* slack, uint8_t* rf_star,
+             const PinState* __restrict__ state, float n_sigma, float* slack, uint8_t* rf_star,
              double* partials, uint32_t* ticket, double* summary) {
   __shared__ double s_tns[kRedThreads];
   __shared__ double s_wns[kRedThreads];
@@ -560,20 +612,20 @@ slack_kernel(int num_ep, const int32_t* __restrict__ ep_pin, const float2* __res
   const int k = blockIdx.x * kRedThreads + threadIdx.x;
   double tns = 0.0, wns = 0.0, nv = 0.0;
   if (k < num_ep) {
-    const float4 st = __ldcg(state + ep_pin[k]);
+    const Gath st = load_state_cg(state + ep_pin[k]);
     const float2 rat = ep_rat[k];
-    const float aR = st.x + n_sigma * st.z;   // Eq 3
-    const float aF = st.y + n_sigma * st.w;
-    const float sR = rat.x - aR, sF = rat.y - aF;
+    const double ns = double(n_sigma);
+    const double sR = double(rat.x) - (st.mu0 + ns * double(st.s0));   // Eq 3 corner
+    const double sF = double(rat.y) - (st.mu1 + ns * double(st.s1));
     const bool fall = sF < sR;
-    const float s = fall ? sF : sR;
-    slack[k] = s;
+    const double s = fall ? sF : sR;
+    slack[k] = float(s);
     rf_star[k] = fall ? 1 : 0;
-    if (s < 0.f) {
-      tns = double(s);
+    if (s < 0.0) {
+      tns = s;
       nv = 1.0;
+      wns = s;
     }
-    wns = s < 0.f ? double(s) : 0.0;
   }
   s_tns[threadIdx.x] = tns;
   s_wns[threadIdx.x] = wns;
@@ -629,16 +681,17 @@ slack_kernel(int num_ep, const int32_t* __restrict__ ep_pin, const float2* __res
 // --------------------------------------------------------------------------
 // Small utility kernels
 // --------------------------------------------------------------------------
-__global__ void arrivals_kernel(int n, const float4* __restrict__ state,
+__global__ void arrivals_kernel(int n, const PinState* __restrict__ state,
                                 const int32_t* __restrict__ order, float n_sigma, float2* A,
                                 float2* mean, float2* sigma) {
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
-  const float4 st = state[i];
+  const Gath st = load_state_cg(state + i);
   const int p = order[i];
-  if (A) A[p] = make_float2(st.x + n_sigma * st.z, st.y + n_sigma * st.w);
-  if (mean) mean[p] = make_float2(st.x, st.y);
-  if (sigma) sigma[p] = make_float2(st.z, st.w);
+  const double ns = double(n_sigma);
+  if (A) A[p] = make_float2(float(st.mu0 + ns * double(st.s0)), float(st.mu1 + ns * double(st.s1)));
+  if (mean) mean[p] = make_float2(float(st.mu0), float(st.mu1));
+  if (sigma) sigma[p] = make_float2(st.s0, st.s1);
 }
 
 __global__ void update_arcs_kernel(int64_t n, const int32_t* __restrict__ ids,
@@ -655,74 +708,89 @@ __global__ void update_arcs_kernel(int64_t n, const int32_t* __restrict__ ids,
 // --------------------------------------------------------------------------
 // Launchers
 // --------------------------------------------------------------------------
-static KParams make_params(DevGraph& g) {
-  KParams P;
+static KParams make_params(DevGraph& g, bool bwd) {
+  KParams P{};
   P.n = g.n;
-  P.num_tiles = g.num_tiles;
   P.num_levels = g.num_levels;
-  P.num_src = g.num_src;
-  P.num_ep = g.num_ep;
-  P.level_ptr = g.level_ptr;
-  P.tile_lv = g.tile_lv;
-  P.level_ntiles = g.level_ntiles;
+  P.grid = g.grid;
+  P.item_a = bwd ? g.bwd_a : g.fwd_a;
+  P.item_b = bwd ? g.bwd_b : g.fwd_b;
   P.fanin_ptr = g.fanin_ptr;
   P.fin_src = g.fin_src;
   P.fin_ms = g.fin_ms;
   P.fin_arc = g.fin_arc;
-  P.fanout_ptr = g.fanout_ptr;
-  P.fout = g.fout;
+  P.lfo_ptr = g.lfo_ptr;
+  P.lfo = g.lfo;
   P.heavy_slot = g.heavy_slot;
   P.src_ms = g.src_ms;
   P.order = g.order;
   P.state = g.state;
+  P.win = g.win;
+  P.wts = g.wts;
   P.g = g.g;
   P.seed = g.seed;
   P.heavy_acc = g.heavy_acc;
-  P.done = nullptr;
-  P.d_mean = nullptr;
-  P.d_src = nullptr;
+  P.done = bwd ? g.done_bwd : g.done_fwd;
   P.n_sigma = 3.f;
   P.tau = 0.f;
-  P.epoch = 0;
   return P;
 }
 
 template <class K>
-static int occupancy(K kernel, int sms) {
-  int b = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kernel, kTile, 0);
-  return b * sms;
+static int set_smem(K kernel, size_t bytes) {
+  return int(cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(bytes)));
 }
 
-int configure_grids(DevGraph& g) {
+int query_grid(int device, int* grid) {
   int sms = 0, coop = 0;
-  cudaError_t e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g.device);
+  cudaError_t e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
   if (e != cudaSuccess) return int(e);
-  cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, g.device);
+  cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, device);
   if (!coop) return int(cudaErrorNotSupported);
-  int f = std::min(occupancy(fwd_persistent<false>, sms), occupancy(fwd_persistent<true>, sms));
-  int b = std::min(occupancy(bwd_persistent<false>, sms), occupancy(bwd_persistent<true>, sms));
-  if (f <= 0 || b <= 0) return int(cudaErrorLaunchOutOfResources);
-  g.grid_fwd = std::max(1, std::min(f, g.num_tiles));
-  g.grid_bwd = std::max(1, std::min(b, g.num_tiles));
+  int err = set_smem(fwd_kernel<false>, kFwdSmem);
+  if (!err) err = set_smem(fwd_kernel<true>, kFwdSmem);
+  if (!err) err = set_smem(bwd_kernel<false>, kBwdSmem);
+  if (!err) err = set_smem(bwd_kernel<true>, kBwdSmem);
+  if (err) return err;
+  int occ = 1 << 30, b = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<false>, kThreads, kFwdSmem);
+  occ = std::min(occ, b);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<true>, kThreads, kFwdSmem);
+  occ = std::min(occ, b);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bwd_kernel<false>, kThreads, kBwdSmem);
+  occ = std::min(occ, b);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bwd_kernel<true>, kThreads, kBwdSmem);
+  occ = std::min(occ, b);
+  if (occ <= 0) return int(cudaErrorLaunchOutOfResources);
+  *grid = occ * sms;
   return int(cudaGetLastError());
 }
 
-static int coop_launch(const void* fn, int grid, KParams& P, cudaStream_t st) {
-  void* args[] = {&P};
-  return int(cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kTile), args, 0, st));
+static int launch_items(const void* fn, size_t smem, KParams& P, const ItemTable& T, bool bwd,
+                        int schedule, cudaStream_t st) {
+  if (schedule == 0) {
+    P.wait = 1;
+    P.step_begin = 0;
+    P.step_end = T.num_steps;
+    void* args[] = {&P};
+    return int(cudaLaunchCooperativeKernel(fn, dim3(P.grid), dim3(kThreads), args, smem, st));
+  }
+  P.wait = 0;
+  const int L = P.num_levels;
+  for (int li = 0; li < L; ++li) {
+    const int l = bwd ? L - 1 - li : li;
+    P.step_begin = T.level_step0[l];
+    P.step_end = T.level_step0[l] + T.level_steps[l];
+    void* args[] = {&P};
+    int err = int(cudaLaunchKernel(fn, dim3(P.grid), dim3(kThreads), args, smem, st));
+    if (err) return err;
+  }
+  return 0;
 }
-
-// Level counters are never reset: pass e leaves done[l] == e * ntiles[l] (mod 2^32)
-// and, within a pass, the counter only takes values (e-1)*ntiles[l] + j with
-// j < ntiles[l], so modular equality with the target is exact across wrap-around.
-static void bump_epoch(uint32_t& epoch) { ++epoch; }
 
 int launch_slack(DevGraph& g, void* stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  if (g.num_ep == 0) {
-    return int(cudaMemsetAsync(g.summary, 0, sizeof(double) * 3, st));
-  }
+  if (g.num_ep == 0) return int(cudaMemsetAsync(g.summary, 0, sizeof(double) * 3, st));
   const int blocks = (g.num_ep + kRedThreads - 1) / kRedThreads;
   slack_kernel<<<blocks, kRedThreads, 0, st>>>(g.num_ep, g.ep_pin, g.ep_rat, g.state,
                                               g.last_n_sigma, g.slack, g.rf_star, g.partials,
@@ -732,30 +800,16 @@ int launch_slack(DevGraph& g, void* stream) {
 
 int launch_forward(DevGraph& g, float n_sigma, float tau, int schedule, void* stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  KParams P = make_params(g);
+  KParams P = make_params(g, false);
   P.n_sigma = n_sigma;
   P.tau = tau;
   const bool lse = tau > 0.f;
-  int err = 0;
   if (g.n > 0) {
-    if (schedule == 0) {
-      bump_epoch(g.epoch_fwd);
-      P.epoch = g.epoch_fwd;
-      P.done = g.done_fwd;
-      err = coop_launch(lse ? (const void*)fwd_persistent<true> : (const void*)fwd_persistent<false>,
-                        g.grid_fwd, P, st);
-    } else {
-      const auto& lp = g.host.level_ptr;
-      for (int l = 0; l < g.num_levels && !err; ++l) {
-        const int lo = lp[l], hi = lp[l + 1];
-        const int blocks = (hi - lo + kTile - 1) / kTile;
-        if (lse) fwd_level<true><<<blocks, kTile, 0, st>>>(P, lo, hi, l);
-        else fwd_level<false><<<blocks, kTile, 0, st>>>(P, lo, hi, l);
-        err = int(cudaGetLastError());
-      }
-    }
+    if (schedule == 0) P.epoch = ++g.epoch_fwd;
+    int err = launch_items(lse ? (const void*)fwd_kernel<true> : (const void*)fwd_kernel<false>,
+                           kFwdSmem, P, g.fwd_items, false, schedule, st);
+    if (err) return err;
   }
-  if (err) return err;
   g.last_n_sigma = n_sigma;
   g.last_tau = tau;
   return launch_slack(g, stream);
@@ -764,8 +818,11 @@ int launch_forward(DevGraph& g, float n_sigma, float tau, int schedule, void* st
 int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float* d_src,
                     void* stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  cudaError_t e = cudaMemsetAsync(d_arc_mean, 0, sizeof(float) * 2 * size_t(g.e), st);
-  if (e != cudaSuccess) return int(e);
+  cudaError_t e = cudaSuccess;
+  if (g.e > 0) {
+    e = cudaMemsetAsync(d_arc_mean, 0, sizeof(float) * 2 * size_t(g.e), st);
+    if (e != cudaSuccess) return int(e);
+  }
   if (d_src) {
     e = cudaMemsetAsync(d_src, 0, sizeof(float) * 2 * size_t(g.n), st);
     if (e != cudaSuccess) return int(e);
@@ -777,30 +834,15 @@ int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float*
     if (err) return err;
   }
   if (g.n == 0) return 0;
-  KParams P = make_params(g);
+  KParams P = make_params(g, true);
   P.n_sigma = g.last_n_sigma;
   P.tau = g.last_tau;
   P.d_mean = d_arc_mean;
   P.d_src = d_src;
   const bool lse = g.last_tau > 0.f;
-  if (g.bwd_schedule == 0) {
-    bump_epoch(g.epoch_bwd);
-    P.epoch = g.epoch_bwd;
-    P.done = g.done_bwd;
-    return coop_launch(lse ? (const void*)bwd_persistent<true> : (const void*)bwd_persistent<false>,
-                       g.grid_bwd, P, st);
-  }
-  const auto& lp = g.host.level_ptr;
-  for (int l = g.num_levels - 1; l >= 0; --l) {
-    const int lo = lp[l], hi = lp[l + 1];
-    const int span = hi - (lo & ~31);
-    const int blocks = (span + kTile - 1) / kTile;
-    if (lse) bwd_level<true><<<blocks, kTile, 0, st>>>(P, lo, hi, l);
-    else bwd_level<false><<<blocks, kTile, 0, st>>>(P, lo, hi, l);
-    int err = int(cudaGetLastError());
-    if (err) return err;
-  }
-  return 0;
+  if (g.bwd_schedule == 0) P.epoch = ++g.epoch_bwd;
+  return launch_items(lse ? (const void*)bwd_kernel<true> : (const void*)bwd_kernel<false>, kBwdSmem,
+                      P, g.bwd_items, true, g.bwd_schedule, st);
 }
 
 int launch_update_arcs(DevGraph& g, int64_t n, const int32_t* ids, const float* mean,
