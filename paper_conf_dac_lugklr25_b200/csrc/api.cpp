@@ -47,6 +47,7 @@ cudaError_t alloc_zero(T** dst, size_t count) {
 void free_graph(insta::DevGraph& d) {
   void* ptrs[] = {d.level_ptr, d.fanin_ptr, d.fin_src,   d.fin_ms,     d.fin_arc,   d.lfo_ptr,
                   d.lfo,       d.fanout_ptr, d.fout_sink, d.heavy_slot, d.heavy_acc, d.arc_pos,
+                  d.heavy_cnt, d.heavy_fo,
                   d.arc_sink,  d.order,     d.src_ms,    d.ep_pin,     d.ep_rat,    d.arc_class,
                   d.fwd_a,     d.fwd_b,     d.bwd_a,     d.bwd_b,      d.done_fwd,  d.done_bwd,
                   d.state,     d.win,       d.wts,       d.g,          d.seed,      d.slack,
@@ -157,9 +158,19 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   std::vector<float4> fin_ms(nE);
   std::vector<int32_t> heavy_slot(nN, -1);
   int32_t nheavy = 0, max_fanin = 0;
+  std::vector<int32_t> heavy_fo;
   for (int32_t k = 0; k < n; ++k) {
-    if (h.fanout_ptr[k + 1] - h.fanout_ptr[k] > insta::kHeavyFanout) heavy_slot[k] = nheavy++;
+    if (h.fanout_ptr[k + 1] - h.fanout_ptr[k] > insta::kHeavyFanout) {
+      heavy_slot[k] = nheavy++;
+      heavy_fo.push_back(h.fanout_ptr[k + 1] - h.fanout_ptr[k]);
+    }
     max_fanin = std::max(max_fanin, h.fanin_ptr[k + 1] - h.fanin_ptr[k]);
+  }
+  for (int32_t f : heavy_fo) {
+    if (f >= (1 << 19)) {
+      delete G;
+      return fail(INSTA_E_ARG, "graph_create: a pin has >= 2^19 fanout arcs");
+    }
   }
   if (max_fanin >= 32768) {
     delete G;
@@ -224,6 +235,8 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   UP(d.fout_sink, fout_sink.data(), nE);
   UP(d.heavy_slot, heavy_slot.data(), nN);
   ZERO(d.heavy_acc, 2 * std::max(nheavy, 1));
+  ZERO(d.heavy_cnt, std::max(nheavy, 1));
+  UP(d.heavy_fo, heavy_fo.data(), heavy_fo.size());
   UP(d.arc_pos, arc_pos.data(), nE);
   UP(d.arc_sink, arc_sink.data(), nE);
   UP(d.order, h.order.data(), nN);

@@ -6,11 +6,13 @@
 // in canonical order ("fanin position" q), sorted by caller arc id within a
 // row; this is the order the forward walks (Alg 1 l.5-7 "outPin_parent_start").
 //
-// Per-pin state is 32 bytes: {double mu_R, double mu_F, float sigma_R,
-// float sigma_F, pad} -- the Eq 1-2 state with the mean accumulated in fp64
-// (a random 32-byte gather costs one DRAM sector either way, and
-// fp64 means keep 15M-pin slacks within 1e-3 ps of the fp64 oracle).  Arc
-// records are float4 {arc_mean_R, arc_mean_F, arc_std_R, arc_std_F}.
+// Per-pin state is 32 bytes: {double mu_R, mu_F, var_R, var_F} -- the Eq 1-2
+// state (mean and variance, sigma = sqrt(var)) accumulated in fp64 (a random 32-byte gather costs
+// one DRAM sector either way, and fp64 keeps 15M-pin slacks within 1e-3 ps of
+// the fp64 oracle).  The least significant mantissa bit of every word carries
+// the parity of the pass that wrote it (DESIGN.md §4 "dataflow"), so a reader
+// knows, word by word, whether a value is from the current pass.  Arc records
+// are float4 {arc_mean_R, arc_mean_F, arc_std_R, arc_std_F}.
 //
 // Work decomposition: every level is cut into `rounds x G`
 // contiguous pin chunks of balanced work (G = resident CTAs); chunk j of level
@@ -36,16 +38,16 @@ constexpr int32_t kSrcMask = (1 << kHeavyBit) - 1;
 constexpr int32_t kMaxPins = (1 << 29) - 1;
 constexpr int kHeavyFanout = 256;
 
-// CTA shape and shared-memory stage capacities (per item)
+// CTA shape (one 1024-thread CTA per SM) and shared-memory stage capacities
+// (per item; two stages are double-buffered)
 constexpr int kThreads = 1024;
-constexpr int kFwdPins = 2048, kFwdArcs = 2560;                     // forward item caps
+constexpr int kFwdPins = 2048, kFwdArcs = 2048;                     // forward item caps
 constexpr int kBwdPins = 1024, kBwdFanout = 2048, kBwdArcs = 2048;  // backward item caps
 static_assert(kHeavyFanout <= kBwdFanout, "a light pin's fanout row must fit one item");
 
 struct alignas(32) PinState {
   double mu[2];
-  float sig[2];
-  float pad[2];
+  double var[2];
 };
 
 // item flags
@@ -98,6 +100,8 @@ struct DevGraph {
   int32_t* fout_sink = nullptr;    // [e] canonical sink of each full fanout entry
   int32_t* heavy_slot = nullptr;   // [n] accumulator slot of heavy drivers, -1 otherwise
   unsigned long long* heavy_acc = nullptr;  // [num_heavy][2] fixed-point adjoints
+  uint32_t* heavy_cnt = nullptr;   // [num_heavy] sink arcs that have contributed this pass
+  int32_t* heavy_fo = nullptr;     // [num_heavy] fanout of each heavy driver
   int32_t num_heavy = 0;
   int32_t* arc_pos = nullptr;      // [e] caller arc id -> fanin position
   int32_t* arc_sink = nullptr;     // [e] caller arc id -> canonical sink
@@ -118,7 +122,7 @@ struct DevGraph {
   PinState* state = nullptr;       // [n]
   int32_t* win = nullptr;          // [n] hard-mode winners {R: k | s<<15, F: << 16}
   float4* wts = nullptr;           // [e] LSE weights w[rf][s] per fanin arc
-  float2* g = nullptr;             // [e] per-fanin-arc adjoint to its source's {R, F}
+  float2* g = nullptr;             // [e] per-fanin-arc adjoint to its source's {R, F} (parity LSB)
   float2* seed = nullptr;          // [n] endpoint seeds (zero at non-endpoints)
   float* slack = nullptr;          // [P]
   uint8_t* rf_star = nullptr;      // [P]
@@ -131,6 +135,7 @@ struct DevGraph {
   // host-side bookkeeping
   HostLevels host;
   uint32_t epoch_fwd = 0, epoch_bwd = 0, inc_epoch = 0;
+  uint32_t pass_fwd = 0, pass_bwd = 0;   // full passes so far; parity = pass & 1
   int bwd_schedule = 0;            // schedule of the last forward (backward mirrors it)
   bool fwd_valid = false;          // a forward ran since the last update
   bool pending_incremental = false;

@@ -18,32 +18,39 @@
 // resident CTA per round.  While a CTA works on item k, one thread has already
 // issued TMA bulk copies (cp.async.bulk + mbarrier) that stage item k+1's CSR
 // slice (row pointers, source ids, arc mean/sigma, weights) in shared memory.
-// The level dependency is a per-level device counter: a CTA publishes level l
-// with fence.acq_rel + red.relaxed after its last item of l, and waits with
-// ld.acquire before its first item of l+1 -- no grid-wide barrier, and CTAs
-// with no pins in a level never wait.  After the wait the only random accesses
-// are the source-state gathers (forward) / per-arc adjoint gathers (backward),
-// issued arc-parallel by all 1024 threads into shared memory.
-//
-// schedule = 1 launches the same item code once per level (no counters); both
-// schedules are bit-identical.  Arithmetic: fp64 means, fp32 sigmas, IEEE
-// sqrt/div/exp/log, --fmad=false: deterministic and bit-reproducible.
+// Dependencies are dataflow, not barriers (mode 2, the default): every 64-bit
+// state word and every 32-bit adjoint word carries the parity of the pass that
+// wrote it in its least significant mantissa bit, so the arc-parallel gathers
+// (source states in the forward, per-arc adjoints in the backward) simply
+// re-poll a word until its parity is the current pass's.  Naturally aligned
+// 64/32-bit accesses are single-copy atomic, so no fence, counter or grid
+// barrier sits on the level-to-level critical path; a CTA waits for exactly
+// the words it consumes.  Heavy drivers wait on a release/acquire arrival
+// count.  mode 1 keeps per-level completion counters (used where parity cannot
+// tell old from new values: incremental passes); mode 0 is one launch per
+// level (schedule = 1).  All modes run the same item code and are
+// bit-identical.  Arithmetic: fp64 state, fp32 inputs, IEEE sqrt/div/exp/log,
+// --fmad=false: deterministic and bit-reproducible.
 #include <cuda_runtime.h>
 
 #include <algorithm>
 #include <cmath>
 #include <cstdint>
+#include <cstdio>
+#include <cstdlib>
+#include <string>
+#include <vector>
 
 #include "internal.h"
 
 namespace insta {
 
-constexpr double kFix = 4294967296.0;  // 2^32: fixed-point scale of heavy accumulators
 
 struct KParams {
   int32_t n, num_levels, grid;
   int32_t step_begin, step_end;  // item steps this launch runs
-  int32_t wait;                  // 1 = persistent (level counters), 0 = per-level launch
+  int32_t mode;                  // 0 per-level launch, 1 level counters, 2 dataflow (parity)
+  uint32_t par;                  // parity written (and awaited) by this pass
   const int4* __restrict__ item_a;
   const int4* __restrict__ item_b;
   const int32_t* __restrict__ fanin_ptr;
@@ -61,11 +68,12 @@ struct KParams {
   float2* g;
   const float2* seed;
   unsigned long long* heavy_acc;
-  uint32_t* done;
+  uint32_t* heavy_cnt;
+  const int32_t* __restrict__ heavy_fo;
   float* d_mean;
   float* d_src;
   float n_sigma, tau;
-  uint32_t epoch;
+  unsigned long long* trace;     // optional per-(CTA, step, warp) {start, end} globaltimer (debug)
 };
 
 // --------------------------------------------------------------------------
@@ -81,12 +89,33 @@ __device__ __forceinline__ uint32_t ld_acquire(const uint32_t* p) {
   return v;
 }
 
-__device__ __forceinline__ void red_release(uint32_t* p) {
-  asm volatile("fence.acq_rel.gpu;\n\tred.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(p) : "memory");
+// ---- parity-tagged words ----
+__device__ __forceinline__ double with_par(double x, uint32_t par) {
+  return __longlong_as_double((__double_as_longlong(x) & ~1ll) | (long long)par);
+}
+__device__ __forceinline__ double strip(unsigned long long b) { return __longlong_as_double((long long)(b & ~1ull)); }
+__device__ __forceinline__ float with_parf(float x, uint32_t par) {
+  return __uint_as_float((__float_as_uint(x) & ~1u) | par);
+}
+__device__ __forceinline__ float stripf(uint32_t b) { return __uint_as_float(b & ~1u); }
+
+__device__ __forceinline__ void ld2_u64(const void* p, unsigned long long& a, unsigned long long& b) {
+  asm volatile("ld.relaxed.gpu.global.v2.b64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
+}
+__device__ __forceinline__ void st2_u64(void* p, double a, double b) {
+  asm volatile("st.relaxed.gpu.global.v2.f64 [%0], {%1, %2};" ::"l"(p), "d"(a), "d"(b) : "memory");
+}
+__device__ __forceinline__ void ld2_u32(const void* p, uint32_t& a, uint32_t& b) {
+  asm volatile("ld.relaxed.gpu.global.v2.b32 {%0, %1}, [%2];" : "=r"(a), "=r"(b) : "l"(p) : "memory");
+}
+__device__ __forceinline__ void st2_f32(void* p, float a, float b) {
+  asm volatile("st.relaxed.gpu.global.v2.f32 [%0], {%1, %2};" ::"l"(p), "f"(a), "f"(b) : "memory");
 }
 
-__device__ __forceinline__ void mbar_init(uint64_t* bar) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(bar)) : "memory");
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
 }
 
 __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
@@ -129,49 +158,84 @@ __device__ __forceinline__ Window window(int64_t a, int64_t b, int esz) {
   return w;
 }
 
-// Level dependency: thread 0 spins on the counter, then the CTA proceeds.
-__device__ __forceinline__ void wait_level(const KParams& P, int l) {
-  if (threadIdx.x == 0) {
-    const uint32_t target = P.epoch * uint32_t(P.grid);
-    while (ld_acquire(P.done + l) != target) __nanosleep(20);
-  }
-  __syncthreads();
-}
-
 // --------------------------------------------------------------------------
 // Eq 1-3 for one candidate: arc e = (j -> i), sink transition rf, source
-// transition s.
+// transition s.  State carries the variance (Eq 2 is additive in it):
 //   mu_c  = mu_j[s] + arc_mean[rf]                 (Eq 1, Alg 1 l.12)
-//   sig_c = sqrt(sig_j[s]^2 + arc_std[rf]^2)       (Eq 2, Alg 1 l.13)
-//   A_c   = mu_c + n_sigma * sig_c                 (Eq 3, Alg 1 l.14)
+//   var_c = var_j[s] + arc_std[rf]^2               (Eq 2, Alg 1 l.13)
+//   A_c   = mu_c + n_sigma * sqrt(var_c)           (Eq 3, Alg 1 l.14)
+// mean and variance accumulate in fp64; the sqrt of the corner is fp32.
 // --------------------------------------------------------------------------
 struct Gath {
-  double mu0, mu1;
-  float s0, s1;
+  double mu0, mu1, v0, v1;
 };
 
 struct Cand {
-  double mu, A;
+  double mu, var, A;
   float sig;
 };
 
-__device__ __forceinline__ Gath load_state_cg(const PinState* p) {
-  const double2 m = __ldcg(reinterpret_cast<const double2*>(p));
-  const float2 s = __ldcg(reinterpret_cast<const float2*>(p) + 2);
+__device__ __forceinline__ float sigma_of(double var) { return sqrtf(float(var)); }
+
+// Pin state words as loaded (parity bits still in place).
+struct Raw {
+  unsigned long long a, b, c, d;
+};
+
+// one 256-bit access per 32-byte pin record (LDG/STG .256 on sm_100a)
+__device__ __forceinline__ Raw ld_state_raw(const KParams& P, int j) {
+  Raw r;
+  asm volatile("ld.relaxed.gpu.global.v4.b64 {%0, %1, %2, %3}, [%4];"
+               : "=l"(r.a), "=l"(r.b), "=l"(r.c), "=l"(r.d)
+               : "l"(P.state + j)
+               : "memory");
+  return r;
+}
+
+__device__ __forceinline__ bool raw_ready(const Raw& r, uint32_t par) {
+  return (((r.a & r.b & r.c & r.d) & 1ull) == par) && (((r.a | r.b | r.c | r.d) & 1ull) == par);
+}
+
+// Complete a state read issued earlier: in dataflow mode re-poll until every
+// word carries this pass's parity.
+__device__ __forceinline__ void await_raw(const KParams& P, int j, Raw& r) {
+  if (P.mode == 2) {
+    while (!raw_ready(r, P.par)) {
+      __nanosleep(20);
+      r = ld_state_raw(P, j);
+    }
+  }
+}
+
+__device__ __forceinline__ Gath unpack(const Raw& r) {
   Gath g;
-  g.mu0 = m.x;
-  g.mu1 = m.y;
-  g.s0 = s.x;
-  g.s1 = s.y;
+  g.mu0 = strip(r.a);
+  g.mu1 = strip(r.b);
+  g.v0 = strip(r.c);
+  g.v1 = strip(r.d);
   return g;
 }
 
+__device__ __forceinline__ Gath load_state(const KParams& P, int j) {
+  Raw r = ld_state_raw(P, j);
+  await_raw(P, j, r);
+  return unpack(r);
+}
+
+__device__ __forceinline__ void store_state(const KParams& P, int i, double m0, double m1, double v0,
+                                            double v1) {
+  asm volatile("st.relaxed.gpu.global.v4.f64 [%0], {%1, %2, %3, %4};" ::"l"(P.state + i),
+               "d"(with_par(m0, P.par)), "d"(with_par(m1, P.par)), "d"(with_par(v0, P.par)),
+               "d"(with_par(v1, P.par))
+               : "memory");
+}
+
 __device__ __forceinline__ Cand make_cand(const Gath& st, const float4& ms, int rf, int s, double ns) {
-  const float sj = s ? st.s1 : st.s0;
-  const float se = rf ? ms.w : ms.z;
+  const double se = double(rf ? ms.w : ms.z);
   Cand c;
   c.mu = (s ? st.mu1 : st.mu0) + double(rf ? ms.y : ms.x);
-  c.sig = sqrtf(sj * sj + se * se);
+  c.var = (s ? st.v1 : st.v0) + se * se;
+  c.sig = sigma_of(c.var);
   c.A = c.mu + ns * double(c.sig);
   return c;
 }
@@ -181,105 +245,82 @@ __device__ __forceinline__ Cand make_cand(const Gath& st, const float4& ms, int 
 __device__ __forceinline__ int n_src_tr(int u) { return u == 2 ? 2 : 1; }
 __device__ __forceinline__ int src_tr(int rf, int u, int a) { return (u == 1 || a == 1) ? (rf ^ 1) : rf; }
 
-// Forward of one non-source pin i with nf fanin arcs (first at fanin position
-// q0); arc(k, srcw, ms, state) yields the k-th arc record and source state.
-template <bool kLSE, class ArcFn>
-__device__ __forceinline__ void fwd_pin(const KParams& P, int i, int nf, int q0, ArcFn&& arc) {
-  const double ns = double(P.n_sigma);
-  const double tau = double(P.tau);
-  double mu_out[2], M[2];
-  float sg_out[2], S[2];
-  int win = 0;
-#pragma unroll
-  for (int rf = 0; rf < 2; ++rf) {
-    double best = 0.0, bmu = 0.0;
-    float bsg = 0.f;
-    int bk = -1, bs = 0;
-    for (int k = 0; k < nf; ++k) {
-      int32_t w;
-      float4 ms;
-      Gath st;
-      arc(k, w, ms, st);
-      const int u = int(uint32_t(w) >> kUnateShift);
-      for (int a = 0; a < n_src_tr(u); ++a) {
-        const int s = src_tr(rf, u, a);
-        const Cand c = make_cand(st, ms, rf, s, ns);
-        if (bk < 0 || c.A > best) {   // Alg 2 l.4: replace only if strictly greater
-          best = c.A;
-          bmu = c.mu;
-          bsg = c.sig;
-          bk = k;
-          bs = s;
-        }
-      }
-    }
-    M[rf] = best;
-    sg_out[rf] = bsg;
-    win |= (bk | (bs << 15)) << (16 * rf);
-    if (kLSE) {
-      // Eq 4: A_i = M + tau * log(sum_c exp((A_c - M) / tau)); reading R1:
-      // sigma_i = sigma of the arg-max, mu_i = A_i - n_sigma * sigma_i.
-      float sum = 0.f;
-      for (int k = 0; k < nf; ++k) {
-        int32_t w;
-        float4 ms;
-        Gath st;
-        arc(k, w, ms, st);
-        const int u = int(uint32_t(w) >> kUnateShift);
-        for (int a = 0; a < n_src_tr(u); ++a) {
-          const Cand c = make_cand(st, ms, rf, src_tr(rf, u, a), ns);
-          sum += expf(float((c.A - best) / tau));
-        }
-      }
-      S[rf] = sum;
-      mu_out[rf] = (best + tau * double(logf(sum))) - ns * double(bsg);
-    } else {
-      mu_out[rf] = bmu;   // Alg 1 l.15 / Alg 2 l.6 with K = 1
-    }
-  }
-  PinState* o = P.state + i;
-  reinterpret_cast<double2*>(o)[0] = make_double2(mu_out[0], mu_out[1]);
-  reinterpret_cast<float4*>(o)[1] = make_float4(sg_out[0], sg_out[1], 0.f, 0.f);
-  if (!kLSE) {
-    P.win[i] = win;
-  } else {
-    // Eq 6 weights w[rf][s] of every candidate, stored per fanin arc
-    for (int k = 0; k < nf; ++k) {
-      int32_t w;
-      float4 ms;
-      Gath st;
-      arc(k, w, ms, st);
-      const int u = int(uint32_t(w) >> kUnateShift);
-      float wt[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
-#pragma unroll
-      for (int rf = 0; rf < 2; ++rf) {
-        for (int a = 0; a < n_src_tr(u); ++a) {
-          const int s = src_tr(rf, u, a);
-          const Cand c = make_cand(st, ms, rf, s, ns);
-          wt[rf][s] = expf(float((c.A - M[rf]) / tau)) / S[rf];
-        }
-      }
-      P.wts[q0 + k] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
-    }
+// Merge of one (pin, rf): first arg-max (strict ">"), LSE normalizer.
+struct Merge {
+  double best, mu, var;
+  float sig, sum;
+  int k, s;
+};
+
+__device__ __forceinline__ void merge_init(Merge& m) {
+  m.best = 0.0;
+  m.mu = 0.0;
+  m.var = 0.0;
+  m.sig = 0.f;
+  m.sum = 0.f;
+  m.k = -1;
+  m.s = 0;
+}
+
+__device__ __forceinline__ void merge_max(Merge& m, const Cand& c, int k, int s) {
+  if (m.k < 0 || c.A > m.best) {   // Alg 2 l.4: replace only if strictly greater
+    m.best = c.A;
+    m.mu = c.mu;
+    m.var = c.var;
+    m.sig = c.sig;
+    m.k = k;
+    m.s = s;
   }
 }
 
+// Eq 6 weight of a candidate given its merge (LSE)
+__device__ __forceinline__ float lse_term(const Cand& c, const Merge& m, double tau) {
+  return expf(float((c.A - m.best) / tau));
+}
+
+// Write the merged pin state and what the backward needs.
+template <bool kLSE>
+__device__ __forceinline__ void fwd_store(const KParams& P, int i, const Merge* m) {
+  double mu[2];
+#pragma unroll
+  for (int rf = 0; rf < 2; ++rf) {
+    // hard: Alg 1 l.15 / Alg 2 l.6 with K = 1.  LSE (Eq 4): A_i = M + tau*log(sum);
+    // reading R1: sigma_i = sigma of the arg-max, mu_i = A_i - n_sigma * sigma_i.
+    mu[rf] = kLSE ? (m[rf].best + double(P.tau) * double(logf(m[rf].sum))) - double(P.n_sigma) * double(m[rf].sig)
+                  : m[rf].mu;
+  }
+  store_state(P, i, mu[0], mu[1], m[0].var, m[1].var);
+  if (!kLSE) P.win[i] = (m[0].k | (m[0].s << 15)) | ((m[1].k | (m[1].s << 15)) << 16);
+}
+
 // --------------------------------------------------------------------------
-// Forward kernel
+// Level-synchronous item loop.  Each CTA walks its item list in
+// level order.  Thread 0 stages item t+1's CSR slice with TMA bulk copies
+// (double-buffered, mbarrier completion) while the CTA works on item t.  An
+// item runs in two phases separated by one CTA barrier: (1) arc-parallel
+// gathers of the source words -- every thread issues all of its loads before
+// checking any, and re-polls only words whose parity is not yet this pass's --
+// into shared memory; (2) pin-parallel compute from shared memory and stores
+// of the new words (with this pass's parity).  No grid barrier, counter or
+// fence: the parity bits are the only synchronization between CTAs.
 // --------------------------------------------------------------------------
+__device__ __forceinline__ void mbar_init1(uint64_t* bar) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(bar)) : "memory");
+}
+
 struct FwdStage {
   int32_t ptr[kFwdPins + 8];
   int32_t src[kFwdArcs + 8];
   float4 ms[kFwdArcs];
 };
-constexpr size_t kFwdSmem = 2 * sizeof(FwdStage) + sizeof(Gath) * kFwdArcs;
+constexpr size_t kFwdSmem = 2 * sizeof(FwdStage) + sizeof(Raw) * kFwdArcs;
 
 __device__ __forceinline__ bool fwd_staged(const int4& A, const int4& B) {
   return A.y > A.x && B.x > 0 && !(B.y & kItemDirect);
 }
 
-// thread 0: issue the bulk copies staging item (step, c) into `st`
-__device__ __forceinline__ void fwd_prefetch(const KParams& P, FwdStage* st, uint64_t* bar, int step,
+// thread 0: issue the bulk copies staging item `step` into `st`
+__device__ __forceinline__ void fwd_prefetch(const KParams& P, FwdStage* st, uint64_t* full, int step,
                                              int c) {
   const int4 A = __ldg(P.item_a + size_t(step) * P.grid + c);
   const int4 B = __ldg(P.item_b + size_t(step) * P.grid + c);
@@ -288,89 +329,158 @@ __device__ __forceinline__ void fwd_prefetch(const KParams& P, FwdStage* st, uin
   const Window ws = window(A.z, A.w, 4);
   const uint32_t bms = uint32_t(A.w - A.z) * 16u;
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-  mbar_expect_tx(bar, wp.bytes + ws.bytes + bms);
-  bulk_g2s(st->ptr, P.fanin_ptr + wp.start, wp.bytes, bar);
-  if (ws.bytes) bulk_g2s(st->src, P.fin_src + ws.start, ws.bytes, bar);
-  if (bms) bulk_g2s(st->ms, P.fin_ms + A.z, bms, bar);
+  mbar_expect_tx(full, wp.bytes + ws.bytes + bms);
+  bulk_g2s(st->ptr, P.fanin_ptr + wp.start, wp.bytes, full);
+  if (ws.bytes) bulk_g2s(st->src, P.fin_src + ws.start, ws.bytes, full);
+  if (bms) bulk_g2s(st->ms, P.fin_ms + A.z, bms, full);
+}
+
+// Forward of one non-source pin whose arc records and gathered source words
+// are addressable by arc(k, w, ms, raw) for k < nf.  Candidates are visited in
+// canonical order: fanin row, then s = rf before ~rf.
+template <bool kLSE, class ArcFn>
+__device__ __forceinline__ void fwd_pin(const KParams& P, int i, int nf, int q0, ArcFn&& arc) {
+  const double ns = double(P.n_sigma), tau = double(P.tau);
+  Merge m[2];
+  merge_init(m[0]);
+  merge_init(m[1]);
+  for (int k = 0; k < nf; ++k) {
+    int32_t w;
+    float4 ms;
+    Raw r;
+    arc(k, w, ms, r);
+    const Gath st = unpack(r);
+    const int u = int(uint32_t(w) >> kUnateShift);
+#pragma unroll
+    for (int rf = 0; rf < 2; ++rf) {
+      const int s0 = src_tr(rf, u, 0);
+      merge_max(m[rf], make_cand(st, ms, rf, s0, ns), k, s0);
+      if (u == 2) merge_max(m[rf], make_cand(st, ms, rf, rf ^ 1, ns), k, rf ^ 1);
+    }
+  }
+  if (kLSE) {
+    for (int k = 0; k < nf; ++k) {
+      int32_t w;
+      float4 ms;
+      Raw r;
+      arc(k, w, ms, r);
+      const Gath st = unpack(r);
+      const int u = int(uint32_t(w) >> kUnateShift);
+#pragma unroll
+      for (int rf = 0; rf < 2; ++rf) {
+        m[rf].sum += lse_term(make_cand(st, ms, rf, src_tr(rf, u, 0), ns), m[rf], tau);
+        if (u == 2) m[rf].sum += lse_term(make_cand(st, ms, rf, rf ^ 1, ns), m[rf], tau);
+      }
+    }
+    // Eq 6 weights w[rf][s] per fanin arc
+    for (int k = 0; k < nf; ++k) {
+      int32_t w;
+      float4 ms;
+      Raw r;
+      arc(k, w, ms, r);
+      const Gath st = unpack(r);
+      const int u = int(uint32_t(w) >> kUnateShift);
+      float wt[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
+#pragma unroll
+      for (int rf = 0; rf < 2; ++rf) {
+        const int s0 = src_tr(rf, u, 0);
+        wt[rf][s0] = lse_term(make_cand(st, ms, rf, s0, ns), m[rf], tau) / m[rf].sum;
+        if (u == 2) wt[rf][rf ^ 1] = lse_term(make_cand(st, ms, rf, rf ^ 1, ns), m[rf], tau) / m[rf].sum;
+      }
+      P.wts[q0 + k] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
+    }
+  }
+  fwd_store<kLSE>(P, i, m);
+}
+
+__device__ __forceinline__ void trace_stamp(const KParams& P, int c, int nsteps, int t, int slot) {
+  if (P.trace && threadIdx.x == 0) P.trace[(size_t(c) * nsteps + t) * 4 + slot] = gtimer();
 }
 
 template <bool kLSE>
 __global__ void __launch_bounds__(kThreads, 1) fwd_kernel(KParams P) {
   extern __shared__ __align__(128) unsigned char smem[];
   FwdStage* stage = reinterpret_cast<FwdStage*>(smem);
-  Gath* gath = reinterpret_cast<Gath*>(smem + 2 * sizeof(FwdStage));
-  __shared__ __align__(8) uint64_t bar[2];
+  Raw* gath = reinterpret_cast<Raw*>(smem + 2 * sizeof(FwdStage));
+  __shared__ __align__(8) uint64_t full[2];
   const int c = blockIdx.x;
   const int tid = threadIdx.x;
   if (tid == 0) {
-    mbar_init(&bar[0]);
-    mbar_init(&bar[1]);
+    mbar_init1(&full[0]);
+    mbar_init1(&full[1]);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
-  uint32_t phase0 = 0, phase1 = 0;
-  int waited = -1;
-  if (tid == 0 && P.step_begin < P.step_end) fwd_prefetch(P, &stage[0], &bar[0], P.step_begin, c);
-  for (int k = P.step_begin; k < P.step_end; ++k) {
-    const int buf = (k - P.step_begin) & 1;
+  uint32_t phase[2] = {0u, 0u};
+  const int nsteps = P.step_end - P.step_begin;
+  if (tid == 0 && nsteps > 0) fwd_prefetch(P, &stage[0], &full[0], P.step_begin, c);
+  for (int t = 0; t < nsteps; ++t) {
+    const int buf = t & 1;
+    const int k = P.step_begin + t;
     const int4 A = __ldg(P.item_a + size_t(k) * P.grid + c);   // {pin_lo, pin_hi, arc_lo, arc_hi}
     const int4 B = __ldg(P.item_b + size_t(k) * P.grid + c);   // {level, flags}
-    const int l = B.x;
-    if (tid == 0 && k + 1 < P.step_end) fwd_prefetch(P, &stage[buf ^ 1], &bar[buf ^ 1], k + 1, c);
+    if (tid == 0 && t + 1 < nsteps) fwd_prefetch(P, &stage[buf ^ 1], &full[buf ^ 1], k + 1, c);
+    trace_stamp(P, c, nsteps, t, 0);
     if (A.y > A.x) {
-      if (l == 0) {
-        // startpoints: clock arrival distribution, mean and std per rf
+      if (B.x == 0) {
+        // startpoints: clock arrival distribution, mean and variance per rf
         for (int i = A.x + tid; i < A.y; i += kThreads) {
-          const float4 s = __ldg(P.src_ms + i);
-          PinState* o = P.state + i;
-          reinterpret_cast<double2*>(o)[0] = make_double2(double(s.x), double(s.y));
-          reinterpret_cast<float4*>(o)[1] = make_float4(s.z, s.w, 0.f, 0.f);
+          const float4 v = __ldg(P.src_ms + i);
+          store_state(P, i, double(v.x), double(v.y), double(v.z) * double(v.z), double(v.w) * double(v.w));
         }
       } else if (!(B.y & kItemDirect)) {
-        if (buf == 0) {
-          mbar_wait(&bar[0], phase0);
-          phase0 ^= 1;
-        } else {
-          mbar_wait(&bar[1], phase1);
-          phase1 ^= 1;
-        }
-        if (P.wait && waited != l) {
-          wait_level(P, l - 1);
-          waited = l;
-        }
+        mbar_wait(&full[buf], phase[buf]);
+        phase[buf] ^= 1u;
         const FwdStage& S = stage[buf];
         const int po = A.x & 3, so = A.z & 3;
         const int na = A.w - A.z;
-        for (int a = tid; a < na; a += kThreads)
-          gath[a] = load_state_cg(P.state + (S.src[so + a] & kSrcMask));
+        // (1) gathers: asynchronous global->shared copies (LDGSTS, through L2)
+        // of every source record of this thread, then complete them: re-poll
+        // only records whose words do not all carry this pass's parity.
+        for (int a = tid; a < na; a += kThreads) {
+          const PinState* src = P.state + (S.src[so + a] & kSrcMask);
+          const uint32_t d = smem_u32(gath + a);
+          asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n\t"
+                       "cp.async.cg.shared.global [%2], [%3], 16;" ::"r"(d),
+                       "l"(src), "r"(d + 16u), "l"(reinterpret_cast<const char*>(src) + 16)
+                       : "memory");
+        }
+        asm volatile("cp.async.wait_all;" ::: "memory");
+        for (int a = tid; a < na; a += kThreads) {
+          Raw r = gath[a];
+          if (P.mode == 2 && !raw_ready(r, P.par)) {
+            const int j = S.src[so + a] & kSrcMask;
+            await_raw(P, j, r);
+            gath[a] = r;
+          }
+        }
         __syncthreads();
+        trace_stamp(P, c, nsteps, t, 1);
+        // (2) compute
         for (int p = tid; p < A.y - A.x; p += kThreads) {
           const int b0 = S.ptr[po + p] - A.z;
-          const int b1 = S.ptr[po + p + 1] - A.z;
-          fwd_pin<kLSE>(P, A.x + p, b1 - b0, A.z + b0,
-                        [&](int kk, int32_t& w, float4& ms, Gath& st) {
-                          w = S.src[so + b0 + kk];
-                          ms = S.ms[b0 + kk];
-                          st = gath[b0 + kk];
-                        });
+          const int nf = S.ptr[po + p + 1] - A.z - b0;
+          fwd_pin<kLSE>(P, A.x + p, nf, A.z + b0, [&](int kk, int32_t& w, float4& ms, Raw& rr) {
+            w = S.src[so + b0 + kk];
+            ms = S.ms[b0 + kk];
+            rr = gath[b0 + kk];
+          });
         }
       } else {
-        if (P.wait && waited != l) {
-          wait_level(P, l - 1);
-          waited = l;
-        }
         for (int i = A.x + tid; i < A.y; i += kThreads) {
-          const int b0 = __ldg(P.fanin_ptr + i), b1 = __ldg(P.fanin_ptr + i + 1);
-          fwd_pin<kLSE>(P, i, b1 - b0, b0, [&](int kk, int32_t& w, float4& ms, Gath& st) {
+          const int b0 = __ldg(P.fanin_ptr + i);
+          const int nf = __ldg(P.fanin_ptr + i + 1) - b0;
+          fwd_pin<kLSE>(P, i, nf, b0, [&](int kk, int32_t& w, float4& ms, Raw& rr) {
             w = __ldg(P.fin_src + b0 + kk);
             ms = __ldg(P.fin_ms + b0 + kk);
-            st = load_state_cg(P.state + (w & kSrcMask));
+            rr = ld_state_raw(P, w & kSrcMask);
+            await_raw(P, w & kSrcMask, rr);
           });
         }
       }
     }
-    __syncthreads();
-    if ((B.y & kItemLast) && P.wait && tid == 0) red_release(P.done + l);
+    __syncthreads();   // stage[buf] and gath are free for reuse
+    trace_stamp(P, c, nsteps, t, 2);
   }
 }
 
@@ -394,7 +504,7 @@ __device__ __forceinline__ bool bwd_staged(const int4& A, const int4& B) {
 }
 
 template <bool kLSE>
-__device__ __forceinline__ void bwd_prefetch(const KParams& P, BwdStage* st, uint64_t* bar, int step,
+__device__ __forceinline__ void bwd_prefetch(const KParams& P, BwdStage* st, uint64_t* full, int step,
                                              int c) {
   const int4 A = __ldg(P.item_a + size_t(step) * P.grid + c);   // {pin_lo, pin_hi, lfo_lo, lfo_hi}
   const int4 B = __ldg(P.item_b + size_t(step) * P.grid + c);   // {arc_lo, arc_hi, level, flags}
@@ -407,27 +517,54 @@ __device__ __forceinline__ void bwd_prefetch(const KParams& P, BwdStage* st, uin
   const uint32_t bw = kLSE ? uint32_t(B.y - B.x) * 16u : 0u;
   const uint32_t total = 2 * wl.bytes + wf.bytes + 2 * wa.bytes + wsd.bytes + (kLSE ? bw : ww.bytes);
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-  mbar_expect_tx(bar, total);
-  bulk_g2s(st->lptr, P.lfo_ptr + wl.start, wl.bytes, bar);
-  if (wf.bytes) bulk_g2s(st->lfo, P.lfo + wf.start, wf.bytes, bar);
-  bulk_g2s(st->fptr, P.fanin_ptr + wl.start, wl.bytes, bar);
+  mbar_expect_tx(full, total);
+  bulk_g2s(st->lptr, P.lfo_ptr + wl.start, wl.bytes, full);
+  if (wf.bytes) bulk_g2s(st->lfo, P.lfo + wf.start, wf.bytes, full);
+  bulk_g2s(st->fptr, P.fanin_ptr + wl.start, wl.bytes, full);
   if (wa.bytes) {
-    bulk_g2s(st->src, P.fin_src + wa.start, wa.bytes, bar);
-    bulk_g2s(st->arc, P.fin_arc + wa.start, wa.bytes, bar);
+    bulk_g2s(st->src, P.fin_src + wa.start, wa.bytes, full);
+    bulk_g2s(st->arc, P.fin_arc + wa.start, wa.bytes, full);
   }
-  bulk_g2s(st->seed, P.seed + wsd.start, wsd.bytes, bar);
+  bulk_g2s(st->seed, P.seed + wsd.start, wsd.bytes, full);
   if (kLSE) {
-    if (bw) bulk_g2s(st->wts, P.wts + B.x, bw, bar);
+    if (bw) bulk_g2s(st->wts, P.wts + B.x, bw, full);
   } else {
-    bulk_g2s(st->win, P.win + ww.start, ww.bytes, bar);
+    bulk_g2s(st->win, P.win + ww.start, ww.bytes, full);
   }
 }
+
+// Heavy drivers (fanout > kHeavyFanout) accumulate their adjoint from their
+// sinks by integer atomics, so the sum is order-independent (deterministic).
+// Each contribution adds kCountUnit + round(g * kFixH) to both words: the
+// arrival count travels inside the same atomic word as the value, so the
+// driver knows the sum is complete when both counts reach its fanout -- no
+// release fence is needed.  |adjoint| < 2^19 and fanout < 2^19 (checked).
+constexpr double kFixH = 16777216.0;                    // 2^24
+constexpr long long kCountUnit = 1ll << 44;
 
 __device__ __forceinline__ void heavy_add(const KParams& P, int32_t srcw, float gx, float gy) {
   if (!((srcw >> kHeavyBit) & 1)) return;
   const int slot = __ldg(P.heavy_slot + (srcw & kSrcMask));
-  if (gx != 0.f) atomicAdd(P.heavy_acc + 2 * slot, (unsigned long long)__double2ll_rn(double(gx) * kFix));
-  if (gy != 0.f) atomicAdd(P.heavy_acc + 2 * slot + 1, (unsigned long long)__double2ll_rn(double(gy) * kFix));
+  atomicAdd(P.heavy_acc + 2 * slot, (unsigned long long)(kCountUnit + __double2ll_rn(double(gx) * kFixH)));
+  atomicAdd(P.heavy_acc + 2 * slot + 1, (unsigned long long)(kCountUnit + __double2ll_rn(double(gy) * kFixH)));
+}
+
+__device__ __forceinline__ long long heavy_count(long long acc) { return (acc + (kCountUnit >> 1)) >> 44; }
+
+__device__ __forceinline__ float2 heavy_take(const KParams& P, int i) {
+  const int slot = __ldg(P.heavy_slot + i);
+  if (slot < 0) return make_float2(0.f, 0.f);
+  // wait until every sink arc has arrived in both words, then decode and reset
+  const long long target = __ldg(P.heavy_fo + slot);
+  unsigned long long x, y;
+  ld2_u64(P.heavy_acc + 2 * slot, x, y);
+  while (heavy_count((long long)x) != target || heavy_count((long long)y) != target) {
+    __nanosleep(32);
+    ld2_u64(P.heavy_acc + 2 * slot, x, y);
+  }
+  asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %1};" ::"l"(P.heavy_acc + 2 * slot), "l"(0ull) : "memory");
+  const long long vx = (long long)x - target * kCountUnit, vy = (long long)y - target * kCountUnit;
+  return make_float2(float(double(vx) / kFixH), float(double(vy) / kFixH));
 }
 
 // Sink side of a pin (nf fanin arcs from fanin position q0) with adjoint ab:
@@ -464,20 +601,28 @@ __device__ __forceinline__ void bwd_sink(const KParams& P, int nf, int q0, float
       gs[0] += a0;
       gs[1] += a1;
     }
-    P.g[q0 + k] = make_float2(gs[0], gs[1]);
+    st2_f32(P.g + q0 + k, with_parf(gs[0], P.par), with_parf(gs[1], P.par));
     if (gm[0] != 0.f || gm[1] != 0.f)
       reinterpret_cast<float2*>(P.d_mean)[arcid] = make_float2(gm[0], gm[1]);
     heavy_add(P, srcw, gs[0], gs[1]);
   }
 }
 
-__device__ __forceinline__ float2 heavy_take(const KParams& P, int i) {
-  const int slot = __ldg(P.heavy_slot + i);
-  if (slot < 0) return make_float2(0.f, 0.f);
-  // every sink of i is at a deeper, completed level: read and reset
-  const long long hx = (long long)atomicExch(P.heavy_acc + 2 * slot, 0ull);
-  const long long hy = (long long)atomicExch(P.heavy_acc + 2 * slot + 1, 0ull);
-  return make_float2(float(double(hx) / kFix), float(double(hy) / kFix));
+// Per-arc adjoint words written by a sink (fanin position q)
+__device__ __forceinline__ void await_g(const KParams& P, int q, uint32_t& a, uint32_t& b) {
+  if (P.mode == 2) {
+    while (((a & 1u) != P.par) || ((b & 1u) != P.par)) {
+      __nanosleep(20);
+      ld2_u32(P.g + q, a, b);
+    }
+  }
+}
+
+__device__ __forceinline__ float2 load_g(const KParams& P, int q) {
+  uint32_t a, b;
+  ld2_u32(P.g + q, a, b);
+  await_g(P, q, a, b);
+  return make_float2(stripf(a), stripf(b));
 }
 
 template <bool kLSE>
@@ -485,61 +630,69 @@ __global__ void __launch_bounds__(kThreads, 1) bwd_kernel(KParams P) {
   extern __shared__ __align__(128) unsigned char smem[];
   BwdStage* stage = reinterpret_cast<BwdStage*>(smem);
   float2* gg = reinterpret_cast<float2*>(smem + 2 * sizeof(BwdStage));
-  __shared__ __align__(8) uint64_t bar[2];
+  __shared__ __align__(8) uint64_t full[2];
   const int c = blockIdx.x;
   const int tid = threadIdx.x;
   if (tid == 0) {
-    mbar_init(&bar[0]);
-    mbar_init(&bar[1]);
+    mbar_init1(&full[0]);
+    mbar_init1(&full[1]);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
-  uint32_t phase0 = 0, phase1 = 0;
-  int waited = -1;
-  if (tid == 0 && P.step_begin < P.step_end) bwd_prefetch<kLSE>(P, &stage[0], &bar[0], P.step_begin, c);
-  for (int k = P.step_begin; k < P.step_end; ++k) {
-    const int buf = (k - P.step_begin) & 1;
+  uint32_t phase[2] = {0u, 0u};
+  const int nsteps = P.step_end - P.step_begin;
+  if (tid == 0 && nsteps > 0) bwd_prefetch<kLSE>(P, &stage[0], &full[0], P.step_begin, c);
+  for (int t = 0; t < nsteps; ++t) {
+    const int buf = t & 1;
+    const int k = P.step_begin + t;
     const int4 A = __ldg(P.item_a + size_t(k) * P.grid + c);   // {pin_lo, pin_hi, lfo_lo, lfo_hi}
     const int4 B = __ldg(P.item_b + size_t(k) * P.grid + c);   // {arc_lo, arc_hi, level, flags}
     const int l = B.z;
-    if (tid == 0 && k + 1 < P.step_end) bwd_prefetch<kLSE>(P, &stage[buf ^ 1], &bar[buf ^ 1], k + 1, c);
-    if (A.y > A.x) {
-      const bool wait_needed = P.wait && l + 1 < P.num_levels && waited != l;
+    if (tid == 0 && t + 1 < nsteps) bwd_prefetch<kLSE>(P, &stage[buf ^ 1], &full[buf ^ 1], k + 1, c);
+    trace_stamp(P, c, nsteps, t, 0);
+    const int np = A.y - A.x;
+    if (np > 0) {
       if (!(B.w & kItemDirect)) {
-        if (buf == 0) {
-          mbar_wait(&bar[0], phase0);
-          phase0 ^= 1;
-        } else {
-          mbar_wait(&bar[1], phase1);
-          phase1 ^= 1;
-        }
-        if (wait_needed) {
-          wait_level(P, l + 1);
-          waited = l;
-        }
+        mbar_wait(&full[buf], phase[buf]);
+        phase[buf] ^= 1u;
         const BwdStage& S = stage[buf];
         const int lo = A.x & 3, fo = A.z & 3, ao = B.x & 3, so = A.x & 1;
         const int nfo = A.w - A.z;
-        for (int e = tid; e < nfo; e += kThreads) gg[e] = __ldcg(P.g + S.lfo[fo + e]);
+        // (1) gather the sinks' per-arc adjoints of every light fanout entry:
+        // asynchronous 8-byte global->shared copies, then re-poll stale words
+        for (int e = tid; e < nfo; e += kThreads)
+          asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(gg + e)),
+                       "l"(P.g + S.lfo[fo + e])
+                       : "memory");
+        asm volatile("cp.async.wait_all;" ::: "memory");
+        for (int e = tid; e < nfo; e += kThreads) {
+          uint32_t a = __float_as_uint(gg[e].x), b = __float_as_uint(gg[e].y);
+          if (P.mode == 2 && (((a & 1u) != P.par) || ((b & 1u) != P.par))) {
+            const int q = S.lfo[fo + e];
+            ld2_u32(P.g + q, a, b);
+            await_g(P, q, a, b);
+          }
+          gg[e] = make_float2(stripf(a), stripf(b));
+        }
         __syncthreads();
-        for (int p = tid; p < A.y - A.x; p += kThreads) {
+        trace_stamp(P, c, nsteps, t, 1);
+        // (2) per pin: pull + seed (+ heavy accumulator), then the sink side
+        for (int p = tid; p < np; p += kThreads) {
           const int i = A.x + p;
-          // pull: seed + sum of the sinks' per-arc adjoints (+ heavy accumulator)
           const int r0 = S.lptr[lo + p] - A.z, r1 = S.lptr[lo + p + 1] - A.z;
-          float2 ab = S.seed[so + p];
           float sx = 0.f, sy = 0.f;
           for (int r = r0; r < r1; ++r) {
             sx += gg[r].x;
             sy += gg[r].y;
           }
           const float2 h = heavy_take(P, i);
-          ab.x += sx + h.x;
-          ab.y += sy + h.y;
+          const float2 sd = S.seed[so + p];
+          const float2 ab = make_float2(sd.x + (sx + h.x), sd.y + (sy + h.y));
           if (l == 0) {
             if (P.d_src) reinterpret_cast<float2*>(P.d_src)[__ldg(P.order + i)] = ab;
           } else {
             const int b0 = S.fptr[lo + p] - B.x, b1 = S.fptr[lo + p + 1] - B.x;
-            bwd_sink<kLSE>(P, b1 - b0, B.x + b0, ab, S.win[lo + p],
+            bwd_sink<kLSE>(P, b1 - b0, B.x + b0, ab, kLSE ? 0 : S.win[lo + p],
                            [&](int kk, int32_t& srcw, int32_t& arcid, float4& w4) {
                              srcw = S.src[ao + b0 + kk];
                              arcid = S.arc[ao + b0 + kk];
@@ -548,22 +701,17 @@ __global__ void __launch_bounds__(kThreads, 1) bwd_kernel(KParams P) {
           }
         }
       } else {
-        if (wait_needed) {
-          wait_level(P, l + 1);
-          waited = l;
-        }
         for (int i = A.x + tid; i < A.y; i += kThreads) {
-          float2 ab = P.seed[i];
-          float sx = 0.f, sy = 0.f;
           const int r0 = __ldg(P.lfo_ptr + i), r1 = __ldg(P.lfo_ptr + i + 1);
+          float sx = 0.f, sy = 0.f;
           for (int r = r0; r < r1; ++r) {
-            const float2 v = __ldcg(P.g + __ldg(P.lfo + r));
+            const float2 v = load_g(P, __ldg(P.lfo + r));
             sx += v.x;
             sy += v.y;
           }
           const float2 h = heavy_take(P, i);
-          ab.x += sx + h.x;
-          ab.y += sy + h.y;
+          const float2 sd = P.seed[i];
+          const float2 ab = make_float2(sd.x + (sx + h.x), sd.y + (sy + h.y));
           if (l == 0) {
             if (P.d_src) reinterpret_cast<float2*>(P.d_src)[__ldg(P.order + i)] = ab;
           } else {
@@ -579,8 +727,20 @@ __global__ void __launch_bounds__(kThreads, 1) bwd_kernel(KParams P) {
       }
     }
     __syncthreads();
-    if ((B.w & kItemLast) && P.wait && tid == 0) red_release(P.done + l);
+    trace_stamp(P, c, nsteps, t, 2);
   }
+}
+
+// State read outside a propagation pass (parity stripped, no waiting).
+__device__ __forceinline__ Gath load_state_plain(const PinState* p) {
+  const double2 m = __ldcg(reinterpret_cast<const double2*>(p));
+  const double2 v = __ldcg(reinterpret_cast<const double2*>(p) + 1);
+  Gath g;
+  g.mu0 = strip((unsigned long long)__double_as_longlong(m.x));
+  g.mu1 = strip((unsigned long long)__double_as_longlong(m.y));
+  g.v0 = strip((unsigned long long)__double_as_longlong(v.x));
+  g.v1 = strip((unsigned long long)__double_as_longlong(v.y));
+  return g;
 }
 
 // Endpoint seeds: dL/dA_ep[rf*] = -dL/dslack (slack = RAT - A); TNS: dL/dslack
@@ -612,11 +772,11 @@ slack_kernel(int num_ep, const int32_t* __restrict__ ep_pin, const float2* __res
   const int k = blockIdx.x * kRedThreads + threadIdx.x;
   double tns = 0.0, wns = 0.0, nv = 0.0;
   if (k < num_ep) {
-    const Gath st = load_state_cg(state + ep_pin[k]);
+    const Gath st = load_state_plain(state + ep_pin[k]);
     const float2 rat = ep_rat[k];
     const double ns = double(n_sigma);
-    const double sR = double(rat.x) - (st.mu0 + ns * double(st.s0));   // Eq 3 corner
-    const double sF = double(rat.y) - (st.mu1 + ns * double(st.s1));
+    const double sR = double(rat.x) - (st.mu0 + ns * double(sigma_of(st.v0)));   // Eq 3 corner
+    const double sF = double(rat.y) - (st.mu1 + ns * double(sigma_of(st.v1)));
     const bool fall = sF < sR;
     const double s = fall ? sF : sR;
     slack[k] = float(s);
@@ -686,12 +846,13 @@ __global__ void arrivals_kernel(int n, const PinState* __restrict__ state,
                                 float2* mean, float2* sigma) {
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
-  const Gath st = load_state_cg(state + i);
+  const Gath st = load_state_plain(state + i);
   const int p = order[i];
   const double ns = double(n_sigma);
-  if (A) A[p] = make_float2(float(st.mu0 + ns * double(st.s0)), float(st.mu1 + ns * double(st.s1)));
+  const float s0 = sigma_of(st.v0), s1 = sigma_of(st.v1);
+  if (A) A[p] = make_float2(float(st.mu0 + ns * double(s0)), float(st.mu1 + ns * double(s1)));
   if (mean) mean[p] = make_float2(float(st.mu0), float(st.mu1));
-  if (sigma) sigma[p] = make_float2(st.s0, st.s1);
+  if (sigma) sigma[p] = make_float2(s0, s1);
 }
 
 __global__ void update_arcs_kernel(int64_t n, const int32_t* __restrict__ ids,
@@ -730,7 +891,8 @@ static KParams make_params(DevGraph& g, bool bwd) {
   P.g = g.g;
   P.seed = g.seed;
   P.heavy_acc = g.heavy_acc;
-  P.done = bwd ? g.done_bwd : g.done_fwd;
+  P.heavy_cnt = g.heavy_cnt;
+  P.heavy_fo = g.heavy_fo;
   P.n_sigma = 3.f;
   P.tau = 0.f;
   return P;
@@ -766,16 +928,47 @@ int query_grid(int device, int* grid) {
   return int(cudaGetLastError());
 }
 
+// mode 2 (dataflow) / 1 (level counters): one cooperative launch over all
+// items; mode 0: one launch per level (kernel boundaries order the levels).
+// Debug: with INSTA_TRACE_DIR set, persistent launches record per-(CTA, step)
+// globaltimer stamps {item start, gathers done, item done, -} and dump them to
+// a binary file (int32 header: grid, steps, 4; then uint64).  Synchronizes.
+static int dump_trace(const char* name, unsigned long long* d, int grid, int steps, cudaStream_t st) {
+  const size_t n = size_t(grid) * steps * 4;
+  std::vector<unsigned long long> h(n);
+  cudaError_t e = cudaMemcpyAsync(h.data(), d, n * 8, cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  cudaFree(d);
+  if (e != cudaSuccess) return int(e);
+  std::string path = std::string(getenv("INSTA_TRACE_DIR")) + "/" + name;
+  FILE* f = fopen(path.c_str(), "wb");
+  if (f) {
+    int32_t hdr[3] = {grid, steps, 4};
+    fwrite(hdr, 4, 3, f);
+    fwrite(h.data(), 8, n, f);
+    fclose(f);
+  }
+  return 0;
+}
+
+// mode 2 (dataflow): one cooperative launch over all items; mode 0: one launch
+// per level (kernel boundaries order the levels).
 static int launch_items(const void* fn, size_t smem, KParams& P, const ItemTable& T, bool bwd,
-                        int schedule, cudaStream_t st) {
-  if (schedule == 0) {
-    P.wait = 1;
+                        cudaStream_t st) {
+  P.trace = nullptr;
+  if (P.mode != 0) {
     P.step_begin = 0;
     P.step_end = T.num_steps;
+    const bool tracing = getenv("INSTA_TRACE_DIR") != nullptr;
+    if (tracing) {
+      cudaMalloc(&P.trace, size_t(P.grid) * T.num_steps * 32);
+      cudaMemsetAsync(P.trace, 0, size_t(P.grid) * T.num_steps * 32, st);
+    }
     void* args[] = {&P};
-    return int(cudaLaunchCooperativeKernel(fn, dim3(P.grid), dim3(kThreads), args, smem, st));
+    int err = int(cudaLaunchCooperativeKernel(fn, dim3(P.grid), dim3(kThreads), args, smem, st));
+    if (!err && tracing) err = dump_trace(bwd ? "bwd_trace.bin" : "fwd_trace.bin", P.trace, P.grid, T.num_steps, st);
+    return err;
   }
-  P.wait = 0;
   const int L = P.num_levels;
   for (int li = 0; li < L; ++li) {
     const int l = bwd ? L - 1 - li : li;
@@ -805,9 +998,10 @@ int launch_forward(DevGraph& g, float n_sigma, float tau, int schedule, void* st
   P.tau = tau;
   const bool lse = tau > 0.f;
   if (g.n > 0) {
-    if (schedule == 0) P.epoch = ++g.epoch_fwd;
+    P.mode = schedule == 0 ? 2 : 0;   // dataflow persistent / one launch per level
+    P.par = (++g.pass_fwd) & 1u;
     int err = launch_items(lse ? (const void*)fwd_kernel<true> : (const void*)fwd_kernel<false>,
-                           kFwdSmem, P, g.fwd_items, false, schedule, st);
+                           kFwdSmem, P, g.fwd_items, false, st);
     if (err) return err;
   }
   g.last_n_sigma = n_sigma;
@@ -840,9 +1034,10 @@ int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float*
   P.d_mean = d_arc_mean;
   P.d_src = d_src;
   const bool lse = g.last_tau > 0.f;
-  if (g.bwd_schedule == 0) P.epoch = ++g.epoch_bwd;
+  P.mode = g.bwd_schedule == 0 ? 2 : 0;
+  P.par = (++g.pass_bwd) & 1u;
   return launch_items(lse ? (const void*)bwd_kernel<true> : (const void*)bwd_kernel<false>, kBwdSmem,
-                      P, g.bwd_items, true, g.bwd_schedule, st);
+                      P, g.bwd_items, true, st);
 }
 
 int launch_update_arcs(DevGraph& g, int64_t n, const int32_t* ids, const float* mean,
