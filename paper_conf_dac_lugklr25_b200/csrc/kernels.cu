@@ -73,6 +73,7 @@ struct KParams {
   float* d_mean;
   float* d_src;
   float n_sigma, tau;
+  double inv_tau;                // 1 / tau (LSE exponent scale)
   unsigned long long* trace;     // optional per-(CTA, step, warp) {start, end} globaltimer (debug)
 };
 
@@ -275,22 +276,77 @@ __device__ __forceinline__ void merge_max(Merge& m, const Cand& c, int k, int s)
 
 // Eq 6 weight of a candidate given its merge (LSE)
 __device__ __forceinline__ float lse_term(const Cand& c, const Merge& m, double tau) {
-  return expf(float((c.A - m.best) / tau));
+  return expf(float((c.A - m.best) * tau));   // tau: the inverse temperature 1/tau
 }
 
-// Write the merged pin state and what the backward needs.
-template <bool kLSE>
-__device__ __forceinline__ void fwd_store(const KParams& P, int i, const Merge* m) {
-  double mu[2];
-#pragma unroll
-  for (int rf = 0; rf < 2; ++rf) {
-    // hard: Alg 1 l.15 / Alg 2 l.6 with K = 1.  LSE (Eq 4): A_i = M + tau*log(sum);
-    // reading R1: sigma_i = sigma of the arg-max, mu_i = A_i - n_sigma * sigma_i.
-    mu[rf] = kLSE ? (m[rf].best + double(P.tau) * double(logf(m[rf].sum))) - double(P.n_sigma) * double(m[rf].sig)
-                  : m[rf].mu;
+// Merge of one (pin, rf) (Alg 1 / Alg 2 with K = 1, or Eq 4) over its
+// candidates in canonical order: fanin row, then s = rf before ~rf.
+// arc(k, w, ms, raw) yields arc k's record and gathered source words.
+struct RfOut {
+  double mu, var, best;
+  float sum;
+  int win;   // arg-max: k | s << 15
+};
+
+template <bool kLSE, class ArcFn>
+__device__ __forceinline__ RfOut pin_rf(const KParams& P, int rf, int nf, ArcFn&& arc) {
+  const double ns = double(P.n_sigma);
+  Merge m;
+  merge_init(m);
+  for (int k = 0; k < nf; ++k) {
+    int32_t w;
+    float4 ms;
+    Raw r;
+    arc(k, w, ms, r);
+    const Gath st = unpack(r);
+    const int u = int(uint32_t(w) >> kUnateShift);
+    const int s0 = src_tr(rf, u, 0);
+    merge_max(m, make_cand(st, ms, rf, s0, ns), k, s0);
+    if (u == 2) merge_max(m, make_cand(st, ms, rf, rf ^ 1, ns), k, rf ^ 1);
   }
-  store_state(P, i, mu[0], mu[1], m[0].var, m[1].var);
-  if (!kLSE) P.win[i] = (m[0].k | (m[0].s << 15)) | ((m[1].k | (m[1].s << 15)) << 16);
+  RfOut o;
+  o.best = m.best;
+  o.var = m.var;
+  o.win = m.k | (m.s << 15);
+  o.sum = 0.f;
+  o.mu = m.mu;   // hard: Alg 1 l.15 / Alg 2 l.6 (the winner's distribution)
+  if (kLSE) {
+    // Eq 4: A_i = M + tau * log(sum_c exp((A_c - M) / tau)); reading R1:
+    // sigma_i = sigma of the arg-max, mu_i = A_i - n_sigma * sigma_i.
+    float sum = 0.f;
+    for (int k = 0; k < nf; ++k) {
+      int32_t w;
+      float4 ms;
+      Raw r;
+      arc(k, w, ms, r);
+      const Gath st = unpack(r);
+      const int u = int(uint32_t(w) >> kUnateShift);
+      sum += lse_term(make_cand(st, ms, rf, src_tr(rf, u, 0), ns), m, P.inv_tau);
+      if (u == 2) sum += lse_term(make_cand(st, ms, rf, rf ^ 1, ns), m, P.inv_tau);
+    }
+    o.sum = sum;
+    o.mu = (m.best + double(P.tau) * double(logf(sum))) - ns * double(m.sig);
+  }
+  return o;
+}
+
+// Eq 6 weights {w[rf][s=R], w[rf][s=F]} of arc k's candidates for transition rf
+template <class ArcFn>
+__device__ __forceinline__ float2 arc_rf_weights(const KParams& P, int rf, int k, const RfOut& o, ArcFn&& arc) {
+  const double ns = double(P.n_sigma);
+  int32_t w;
+  float4 ms;
+  Raw r;
+  arc(k, w, ms, r);
+  const Gath st = unpack(r);
+  const int u = int(uint32_t(w) >> kUnateShift);
+  float wt[2] = {0.f, 0.f};
+  const int s0 = src_tr(rf, u, 0);
+  Merge m;
+  m.best = o.best;
+  wt[s0] = lse_term(make_cand(st, ms, rf, s0, ns), m, P.inv_tau) / o.sum;
+  if (u == 2) wt[rf ^ 1] = lse_term(make_cand(st, ms, rf, rf ^ 1, ns), m, P.inv_tau) / o.sum;
+  return make_float2(wt[0], wt[1]);
 }
 
 // --------------------------------------------------------------------------
@@ -335,62 +391,44 @@ __device__ __forceinline__ void fwd_prefetch(const KParams& P, FwdStage* st, uin
   if (bms) bulk_g2s(st->ms, P.fin_ms + A.z, bms, full);
 }
 
-// Forward of one non-source pin whose arc records and gathered source words
-// are addressable by arc(k, w, ms, raw) for k < nf.  Candidates are visited in
-// canonical order: fanin row, then s = rf before ~rf.
+// Forward of one non-source pin by one thread (both rf).
 template <bool kLSE, class ArcFn>
 __device__ __forceinline__ void fwd_pin(const KParams& P, int i, int nf, int q0, ArcFn&& arc) {
-  const double ns = double(P.n_sigma), tau = double(P.tau);
-  Merge m[2];
-  merge_init(m[0]);
-  merge_init(m[1]);
-  for (int k = 0; k < nf; ++k) {
-    int32_t w;
-    float4 ms;
-    Raw r;
-    arc(k, w, ms, r);
-    const Gath st = unpack(r);
-    const int u = int(uint32_t(w) >> kUnateShift);
-#pragma unroll
-    for (int rf = 0; rf < 2; ++rf) {
-      const int s0 = src_tr(rf, u, 0);
-      merge_max(m[rf], make_cand(st, ms, rf, s0, ns), k, s0);
-      if (u == 2) merge_max(m[rf], make_cand(st, ms, rf, rf ^ 1, ns), k, rf ^ 1);
+  const RfOut R = pin_rf<kLSE>(P, 0, nf, arc);
+  const RfOut F = pin_rf<kLSE>(P, 1, nf, arc);
+  store_state(P, i, R.mu, F.mu, R.var, F.var);
+  if (!kLSE) {
+    P.win[i] = R.win | (F.win << 16);
+  } else {
+    for (int k = 0; k < nf; ++k) {
+      const float2 wr = arc_rf_weights(P, 0, k, R, arc);
+      const float2 wf = arc_rf_weights(P, 1, k, F, arc);
+      P.wts[q0 + k] = make_float4(wr.x, wr.y, wf.x, wf.y);
     }
+  }
+}
+
+// Forward of one pin by a lane pair: the even lane computes rf = R, the odd
+// lane rf = F (halving the dependent arithmetic per thread); the even lane
+// writes the record.  Same functions as fwd_pin, hence bit-identical.
+template <bool kLSE, class ArcFn>
+__device__ __forceinline__ void fwd_pin_pair(const KParams& P, int i, int rf, int nf, int q0, ArcFn&& arc) {
+  const unsigned pair = 3u << ((threadIdx.x & 31) & ~1);
+  const RfOut o = pin_rf<kLSE>(P, rf, nf, arc);
+  const double mu_o = __shfl_xor_sync(pair, o.mu, 1);
+  const double var_o = __shfl_xor_sync(pair, o.var, 1);
+  const int win_o = __shfl_xor_sync(pair, o.win, 1);
+  if (rf == 0) {
+    store_state(P, i, o.mu, mu_o, o.var, var_o);
+    if (!kLSE) P.win[i] = o.win | (win_o << 16);
   }
   if (kLSE) {
     for (int k = 0; k < nf; ++k) {
-      int32_t w;
-      float4 ms;
-      Raw r;
-      arc(k, w, ms, r);
-      const Gath st = unpack(r);
-      const int u = int(uint32_t(w) >> kUnateShift);
-#pragma unroll
-      for (int rf = 0; rf < 2; ++rf) {
-        m[rf].sum += lse_term(make_cand(st, ms, rf, src_tr(rf, u, 0), ns), m[rf], tau);
-        if (u == 2) m[rf].sum += lse_term(make_cand(st, ms, rf, rf ^ 1, ns), m[rf], tau);
-      }
-    }
-    // Eq 6 weights w[rf][s] per fanin arc
-    for (int k = 0; k < nf; ++k) {
-      int32_t w;
-      float4 ms;
-      Raw r;
-      arc(k, w, ms, r);
-      const Gath st = unpack(r);
-      const int u = int(uint32_t(w) >> kUnateShift);
-      float wt[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
-#pragma unroll
-      for (int rf = 0; rf < 2; ++rf) {
-        const int s0 = src_tr(rf, u, 0);
-        wt[rf][s0] = lse_term(make_cand(st, ms, rf, s0, ns), m[rf], tau) / m[rf].sum;
-        if (u == 2) wt[rf][rf ^ 1] = lse_term(make_cand(st, ms, rf, rf ^ 1, ns), m[rf], tau) / m[rf].sum;
-      }
-      P.wts[q0 + k] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
+      const float2 w = arc_rf_weights(P, rf, k, o, arc);
+      const float wx = __shfl_xor_sync(pair, w.x, 1), wy = __shfl_xor_sync(pair, w.y, 1);
+      if (rf == 0) P.wts[q0 + k] = make_float4(w.x, w.y, wx, wy);
     }
   }
-  fwd_store<kLSE>(P, i, m);
 }
 
 __device__ __forceinline__ void trace_stamp(const KParams& P, int c, int nsteps, int t, int slot) {
@@ -456,11 +494,12 @@ __global__ void __launch_bounds__(kThreads, 1) fwd_kernel(KParams P) {
         }
         __syncthreads();
         trace_stamp(P, c, nsteps, t, 1);
-        // (2) compute
-        for (int p = tid; p < A.y - A.x; p += kThreads) {
+        // (2) compute: work unit = (pin, rf), a lane pair per pin
+        for (int un = tid; un < 2 * (A.y - A.x); un += kThreads) {
+          const int p = un >> 1;
           const int b0 = S.ptr[po + p] - A.z;
           const int nf = S.ptr[po + p + 1] - A.z - b0;
-          fwd_pin<kLSE>(P, A.x + p, nf, A.z + b0, [&](int kk, int32_t& w, float4& ms, Raw& rr) {
+          fwd_pin_pair<kLSE>(P, A.x + p, un & 1, nf, A.z + b0, [&](int kk, int32_t& w, float4& ms, Raw& rr) {
             w = S.src[so + b0 + kk];
             ms = S.ms[b0 + kk];
             rr = gath[b0 + kk];
@@ -494,6 +533,7 @@ struct BwdStage {
   int32_t src[kBwdArcs + 8];    // fin_src
   int32_t arc[kBwdArcs + 8];    // caller arc ids
   int32_t win[kBwdPins + 8];    // hard-mode winners
+  int32_t hslot[kBwdPins + 8];  // heavy accumulator slot per pin (-1: light)
   float2 seed[kBwdPins + 8];
   float4 wts[kBwdArcs];         // LSE weights
 };
@@ -515,7 +555,7 @@ __device__ __forceinline__ void bwd_prefetch(const KParams& P, BwdStage* st, uin
   const Window wsd = window(A.x, A.y, 8);
   const Window ww = window(A.x, A.y, 4);
   const uint32_t bw = kLSE ? uint32_t(B.y - B.x) * 16u : 0u;
-  const uint32_t total = 2 * wl.bytes + wf.bytes + 2 * wa.bytes + wsd.bytes + (kLSE ? bw : ww.bytes);
+  const uint32_t total = 2 * wl.bytes + wf.bytes + 2 * wa.bytes + wsd.bytes + ww.bytes + (kLSE ? bw : ww.bytes);
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   mbar_expect_tx(full, total);
   bulk_g2s(st->lptr, P.lfo_ptr + wl.start, wl.bytes, full);
@@ -526,6 +566,7 @@ __device__ __forceinline__ void bwd_prefetch(const KParams& P, BwdStage* st, uin
     bulk_g2s(st->arc, P.fin_arc + wa.start, wa.bytes, full);
   }
   bulk_g2s(st->seed, P.seed + wsd.start, wsd.bytes, full);
+  bulk_g2s(st->hslot, P.heavy_slot + ww.start, ww.bytes, full);
   if (kLSE) {
     if (bw) bulk_g2s(st->wts, P.wts + B.x, bw, full);
   } else {
@@ -551,8 +592,7 @@ __device__ __forceinline__ void heavy_add(const KParams& P, int32_t srcw, float 
 
 __device__ __forceinline__ long long heavy_count(long long acc) { return (acc + (kCountUnit >> 1)) >> 44; }
 
-__device__ __forceinline__ float2 heavy_take(const KParams& P, int i) {
-  const int slot = __ldg(P.heavy_slot + i);
+__device__ __forceinline__ float2 heavy_take(const KParams& P, int slot) {
   if (slot < 0) return make_float2(0.f, 0.f);
   // wait until every sink arc has arrived in both words, then decode and reset
   const long long target = __ldg(P.heavy_fo + slot);
@@ -685,7 +725,7 @@ __global__ void __launch_bounds__(kThreads, 1) bwd_kernel(KParams P) {
             sx += gg[r].x;
             sy += gg[r].y;
           }
-          const float2 h = heavy_take(P, i);
+          const float2 h = heavy_take(P, S.hslot[lo + p]);
           const float2 sd = S.seed[so + p];
           const float2 ab = make_float2(sd.x + (sx + h.x), sd.y + (sy + h.y));
           if (l == 0) {
@@ -709,7 +749,7 @@ __global__ void __launch_bounds__(kThreads, 1) bwd_kernel(KParams P) {
             sx += v.x;
             sy += v.y;
           }
-          const float2 h = heavy_take(P, i);
+          const float2 h = heavy_take(P, __ldg(P.heavy_slot + i));
           const float2 sd = P.seed[i];
           const float2 ab = make_float2(sd.x + (sx + h.x), sd.y + (sy + h.y));
           if (l == 0) {
@@ -996,6 +1036,7 @@ int launch_forward(DevGraph& g, float n_sigma, float tau, int schedule, void* st
   KParams P = make_params(g, false);
   P.n_sigma = n_sigma;
   P.tau = tau;
+  P.inv_tau = tau > 0.f ? 1.0 / double(tau) : 0.0;
   const bool lse = tau > 0.f;
   if (g.n > 0) {
     P.mode = schedule == 0 ? 2 : 0;   // dataflow persistent / one launch per level
@@ -1031,6 +1072,7 @@ int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float*
   KParams P = make_params(g, true);
   P.n_sigma = g.last_n_sigma;
   P.tau = g.last_tau;
+  P.inv_tau = g.last_tau > 0.f ? 1.0 / double(g.last_tau) : 0.0;
   P.d_mean = d_arc_mean;
   P.d_src = d_src;
   const bool lse = g.last_tau > 0.f;
