@@ -163,6 +163,33 @@ insta_status insta_update_arcs(insta_graph* g, int64_t n, const int32_t* arc_ids
                                const float* mean, const float* sigma, int32_t incremental,
                                void* cuda_stream);
 
+/* One scenario of a batched evaluation: the graph's arc
+ * delays with mean and sigma of cell arcs (arc_class 1) multiplied by
+ * derate_cell and of net arcs by derate_net -- materialized in fp32 as
+ * fl32(x * d) -- then the listed arcs' {mean, sigma} replaced by the given
+ * values (sparse overrides, e.g. a gate-sizing candidate); n_sigma is the
+ * scenario's pessimism (Eq 3).  delta_* are HOST arrays, copied by the call;
+ * delta arc ids must be unique within a scenario. */
+typedef struct {
+  float n_sigma;
+  float derate_cell;
+  float derate_net;
+  int32_t n_delta;
+  const int32_t* delta_arc;   /* HOST [n_delta] caller arc ids */
+  const float* delta_mean;    /* HOST [n_delta][2] */
+  const float* delta_sigma;   /* HOST [n_delta][2], >= 0 */
+} insta_scenario;
+
+/* Batched evaluation of num_scenarios independent scenarios (forward, slack,
+ * WNS/TNS; optionally the TNS backward), 32 per pass with scenario-minor state.
+ * Each scenario's arrivals equal insta_forward on its materialized graph bit
+ * for bit.  summaries: DEVICE double[num_scenarios][3] {wns, tns,
+ * num_violations}.  d_arc_mean_sum: DEVICE float[num_arcs][2], overwritten
+ * with sum_s dTNS_s/d(arc mean of scenario s), or NULL for forward only.
+ * tau as in insta_opts.  Does not change the graph's single-scenario state. */
+insta_status insta_forward_batch(insta_graph* g, int32_t num_scenarios, const insta_scenario* sc, float tau,
+                                 double* summaries, float* d_arc_mean_sum, void* cuda_stream);
+
 /* Statistics of the last forward: number of pins recomputed (== num_pins for a
  * full forward; the cone size for an incremental one).  Synchronizes. */
 insta_status insta_last_forward_stats(insta_graph* g, int64_t* pins_recomputed);

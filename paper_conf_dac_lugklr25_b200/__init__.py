@@ -176,6 +176,37 @@ class Graph:
         check(self.lib.insta_update_arcs(self._h, int(ids.numel()), _dptr(ids), _dptr(m), _dptr(s),
                                          int(bool(incremental)), self._st(stream)), "insta_update_arcs")
 
+    def forward_batch(self, scenarios, tau: float = 0.0, want_grad: bool = False, summaries=None, d_mean_sum=None,
+                      stream=None):
+        """insta_forward_batch: evaluate independent scenarios (dicts with n_sigma, derate_cell, derate_net and
+        optional delta_arc / delta_mean / delta_sigma host arrays).  Returns (summaries float64[B,3] {wns, tns,
+        num_violations} device tensor, d_mean_sum float32[E,2] or None)."""
+        t = self._torch
+        B = len(scenarios)
+        arr = (_capi.insta_scenario * max(B, 1))()
+        keep = []
+        for k, sc in enumerate(scenarios):
+            da = sc.get("delta_arc")
+            n = 0 if da is None else len(da)
+            if n:
+                ids = _np(da, np.int32)
+                dm = _np(sc["delta_mean"], np.float32, (n, 2))
+                ds = _np(sc["delta_sigma"], np.float32, (n, 2))
+                keep += [ids, dm, ds]
+                arr[k] = _capi.insta_scenario(float(sc.get("n_sigma", 3.0)), float(sc.get("derate_cell", 1.0)),
+                                              float(sc.get("derate_net", 1.0)), n, _ptr(ids), _ptr(dm), _ptr(ds))
+            else:
+                arr[k] = _capi.insta_scenario(float(sc.get("n_sigma", 3.0)), float(sc.get("derate_cell", 1.0)),
+                                              float(sc.get("derate_net", 1.0)), 0, None, None, None)
+        summ = summaries if summaries is not None else t.empty((B, 3), dtype=t.float64, device=self.device)
+        dsum = None
+        if want_grad:
+            dsum = d_mean_sum if d_mean_sum is not None else t.empty((self.num_arcs, 2), dtype=t.float32,
+                                                                      device=self.device)
+        check(self.lib.insta_forward_batch(self._h, B, arr, float(tau), _dptr(summ), _dptr(dsum), self._st(stream)),
+              "insta_forward_batch")
+        return summ, dsum
+
     def last_forward_stats(self) -> int:
         v = ctypes.c_int64()
         check(self.lib.insta_last_forward_stats(self._h, ctypes.byref(v)), "insta_last_forward_stats")

@@ -43,6 +43,11 @@ class insta_summary(ctypes.Structure):
                 ("num_violations", ctypes.c_int32), ("num_levels", ctypes.c_int32)]
 
 
+class insta_scenario(ctypes.Structure):
+    _fields_ = [("n_sigma", ctypes.c_float), ("derate_cell", ctypes.c_float), ("derate_net", ctypes.c_float),
+                ("n_delta", ctypes.c_int32), ("delta_arc", c_vp), ("delta_mean", c_vp), ("delta_sigma", c_vp)]
+
+
 # name -> (restype, argtypes); every symbol declared in include/insta.h
 SIGNATURES = {
     "insta_levelize": (ctypes.c_int, [ctypes.c_int32, ctypes.c_int64, c_vp, c_vp, c_vp, c_vp, c_vp, c_vp,
@@ -57,6 +62,8 @@ SIGNATURES = {
     "insta_backward": (ctypes.c_int, [c_vp, c_vp, c_vp, c_vp, c_vp, c_vp]),
     "insta_update_arcs": (ctypes.c_int, [c_vp, ctypes.c_int64, c_vp, c_vp, c_vp, ctypes.c_int32, c_vp]),
     "insta_last_forward_stats": (ctypes.c_int, [c_vp, c_vp]),
+    "insta_forward_batch": (ctypes.c_int, [c_vp, ctypes.c_int32, ctypes.POINTER(insta_scenario), ctypes.c_float,
+                                           c_vp, c_vp, c_vp]),
     "insta_last_error": (ctypes.c_char_p, []),
     "insta_version": (ctypes.c_char_p, []),
 }

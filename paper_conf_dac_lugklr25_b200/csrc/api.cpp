@@ -51,7 +51,10 @@ void free_graph(insta::DevGraph& d) {
                   d.arc_sink,  d.order,     d.src_ms,    d.ep_pin,     d.ep_rat,    d.arc_class,
                   d.fwd_a,     d.fwd_b,     d.bwd_a,     d.bwd_b,      d.done_fwd,  d.done_bwd,
                   d.state,     d.win,       d.wts,       d.g,          d.seed,      d.slack,
-                  d.rf_star,   d.partials,  d.ticket,    d.summary,    d.dirty,     d.counters};
+                  d.rf_star,   d.partials,  d.ticket,    d.summary,    d.dirty,     d.counters,
+                  d.fin_flags, d.ep_of_pin, d.b_state,   d.b_win,      d.b_wts,     d.b_g,
+                  d.b_heavy,   d.b_sc,      d.b_ov_ptr,  d.b_ov_pos,   d.b_ov_ms,   d.b_slack,
+                  d.b_rf,      d.b_partials, d.b_ticket};
   for (void* p : ptrs)
     if (p) cudaFree(p);
 }
@@ -215,6 +218,11 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   }
   std::vector<uint8_t> arc_class(nE, 0);
   if (desc->arc_class) std::copy(desc->arc_class, desc->arc_class + E, arc_class.begin());
+  std::vector<uint8_t> fin_flags(nE, 0);
+  for (int64_t q = 0; q < E; ++q) fin_flags[q] = arc_class[h.fanin_arc[q]] ? 1 : 0;
+  std::vector<int32_t> ep_of_pin(nN, -1);
+  for (int32_t k = 0; k < d.num_ep; ++k) ep_of_pin[ep_pin[k]] = k;
+  d.h_arc_pos = arc_pos;
 
   // ---- device: grid, items, upload ------------------------------------------------
   cudaError_t e = cudaSetDevice(d.device);
@@ -244,6 +252,8 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   UP(d.ep_pin, ep_pin.data(), ep_pin.size());
   UP(d.ep_rat, ep_rat.data(), ep_rat.size());
   UP(d.arc_class, arc_class.data(), nE);
+  UP(d.fin_flags, fin_flags.data(), nE);
+  UP(d.ep_of_pin, ep_of_pin.data(), nN);
   UP(d.fwd_a, d.fwd_items.a.data(), d.fwd_items.a.size());
   UP(d.fwd_b, d.fwd_items.b.data(), d.fwd_items.b.size());
   UP(d.bwd_a, d.bwd_items.a.data(), d.bwd_items.a.size());
@@ -392,6 +402,61 @@ insta_status insta_update_arcs(insta_graph* g, int64_t n, const int32_t* arc_ids
   d.fwd_valid = false;
   if (incremental && !d.pending_full) d.pending_incremental = true;
   else d.pending_full = true;
+  return INSTA_OK;
+}
+
+insta_status insta_forward_batch(insta_graph* g, int32_t num_scenarios, const insta_scenario* sc, float tau,
+                                 double* summaries, float* d_arc_mean_sum, void* cuda_stream) {
+  if (!g) return fail(INSTA_E_ARG, "forward_batch: NULL graph");
+  if (num_scenarios < 0 || (num_scenarios > 0 && (!sc || !summaries)))
+    return fail(INSTA_E_ARG, "forward_batch: bad arguments");
+  if (!std::isfinite(tau) || tau < 0.f) return fail(INSTA_E_ARG, "forward_batch: tau must be >= 0");
+  insta::DevGraph& d = g->d;
+  for (int32_t s = 0; s < num_scenarios; ++s) {
+    const insta_scenario& x = sc[s];
+    if (!std::isfinite(x.n_sigma) || x.n_sigma < 0.f || !std::isfinite(x.derate_cell) || x.derate_cell < 0.f ||
+        !std::isfinite(x.derate_net) || x.derate_net < 0.f)
+      return fail(INSTA_E_ARG, "forward_batch: scenario n_sigma and derates must be finite and >= 0");
+    if (x.n_delta < 0 || (x.n_delta > 0 && (!x.delta_arc || !x.delta_mean || !x.delta_sigma)))
+      return fail(INSTA_E_ARG, "forward_batch: bad scenario delta list");
+    for (int32_t k = 0; k < x.n_delta; ++k) {
+      if (x.delta_arc[k] < 0 || x.delta_arc[k] >= d.e) return fail(INSTA_E_ARG, "forward_batch: delta arc out of range");
+      for (int r = 0; r < 2; ++r)
+        if (!std::isfinite(x.delta_mean[2 * k + r]) || !std::isfinite(x.delta_sigma[2 * k + r]) ||
+            x.delta_sigma[2 * k + r] < 0.f)
+          return fail(INSTA_E_ARG, "forward_batch: bad delta value");
+    }
+  }
+  cudaSetDevice(d.device);
+  cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+  if (d_arc_mean_sum && d.e > 0) {
+    cudaError_t e = cudaMemsetAsync(d_arc_mean_sum, 0, sizeof(float) * 2 * size_t(d.e), st);
+    if (e != cudaSuccess) return cuda_fail(int(e), "forward_batch");
+  }
+  constexpr int kL = 32;
+  for (int32_t b0 = 0; b0 < num_scenarios; b0 += kL) {
+    const int nb = std::min(kL, num_scenarios - b0);
+    float par[3 * kL];
+    std::vector<int32_t> ov_ptr(kL + 1, 0), ov_pos;
+    std::vector<float4> ov_ms;
+    for (int s = 0; s < kL; ++s) {
+      const insta_scenario* x = s < nb ? &sc[b0 + s] : nullptr;
+      par[s] = x ? x->n_sigma : 0.f;
+      par[kL + s] = x ? x->derate_cell : 1.f;
+      par[2 * kL + s] = x ? x->derate_net : 1.f;
+      if (x) {
+        for (int32_t k = 0; k < x->n_delta; ++k) {
+          ov_pos.push_back(d.h_arc_pos[x->delta_arc[k]]);
+          ov_ms.push_back(make_float4(x->delta_mean[2 * k], x->delta_mean[2 * k + 1], x->delta_sigma[2 * k],
+                                      x->delta_sigma[2 * k + 1]));
+        }
+      }
+      ov_ptr[s + 1] = int32_t(ov_pos.size());
+    }
+    int err = insta::launch_forward_batch(d, nb, par, ov_ptr, ov_pos, ov_ms, tau, summaries + 3 * size_t(b0),
+                                          d_arc_mean_sum, cuda_stream);
+    if (err) return cuda_fail(err, "forward_batch");
+  }
   return INSTA_OK;
 }
 

@@ -1,0 +1,711 @@
+// batch.cu -- batched scenario evaluation (BASELINE north
+// star: "independent evaluations ... batches of candidate gate-sizing
+// perturbations or PVT/OCV scenarios").
+//
+// Up to kLanes = 32 scenarios are evaluated in one pass over the graph.  The
+// per-pin state is scenario-minor ([pin][scenario], 32 B per entry), so the 32
+// lanes of a warp are the 32 scenarios of ONE pin: every source-state gather
+// is a contiguous 1 KB access, and the topology (row pointers, source words,
+// arc records -- TMA-staged per item exactly as in kernels.cu) is read once
+// for all scenarios.  Scenario s materializes its arc table in fp32 as the
+// oracle does: mean' = fl32(mean * d), sigma' = fl32(sigma *
+// d) with d = derate_cell or derate_net by arc class, then sparse overrides
+// replace whole arc records; N_sigma is per scenario.  Candidate arithmetic,
+// merge order and LSE are the same device functions as the single-scenario
+// path, so each scenario's arrivals are bit-identical to insta_forward on the
+// materialized graph.  Synchronization is the same parity dataflow.
+//
+// The optional backward accumulates sum_s dTNS_s / d(arc mean') into one
+// [E][2] buffer: per arc, the 32 lanes' contributions are summed by a fixed
+// xor-shuffle tree and added by lane 0 (each arc is written by exactly one
+// warp per pass, so the read-modify-write needs no atomics).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdint>
+#include <vector>
+
+#include "device_common.cuh"
+#include "internal.h"
+
+namespace insta {
+
+constexpr int kLanes = 32;
+constexpr double kFixB = 16777216.0;          // 2^24 (heavy accumulators, as kernels.cu)
+constexpr long long kCountUnitB = 1ll << 44;
+
+struct BParams {
+  int32_t n, num_levels, grid, step_begin, step_end, nb;
+  uint32_t par;
+  float tau;
+  double inv_tau;
+  const int4* __restrict__ item_a;
+  const int4* __restrict__ item_b;
+  const int32_t* __restrict__ fanin_ptr;
+  const int32_t* __restrict__ fin_src;
+  const float4* __restrict__ fin_ms;
+  const uint8_t* __restrict__ fin_flags;   // bit 0: cell arc, bit 1: overridden in this batch
+  const int32_t* __restrict__ fin_arc;
+  const int32_t* __restrict__ lfo_ptr;
+  const int32_t* __restrict__ lfo;
+  const int32_t* __restrict__ heavy_slot;
+  const int32_t* __restrict__ heavy_fo;
+  const int32_t* __restrict__ ep_of_pin;
+  const float4* __restrict__ src_ms;
+  const float* __restrict__ sc;            // [3][32]: n_sigma, derate_cell, derate_net
+  const int32_t* __restrict__ ov_ptr;      // [33] overrides of scenario s: [ov_ptr[s], ov_ptr[s+1])
+  const int32_t* __restrict__ ov_pos;      // fanin positions, ascending within a scenario
+  const float4* __restrict__ ov_ms;        // override arc records
+  PinState* bstate;                        // [n][32]
+  int32_t* bwin;                           // [n][32]
+  float4* bwts;                            // [e][32]
+  float2* bg;                              // [e][32]
+  unsigned long long* bheavy;              // [heavy][32][2]
+  const float* bslack;                     // [P][32]
+  const uint8_t* brf;                      // [P][32]
+  float* d_mean_sum;                       // [e][2] (accumulated)
+};
+
+// ---------------------------------------------------------------- scenario arcs
+__device__ __forceinline__ float4 scen_arc(const BParams& P, float4 ms, uint32_t flags, int q, int s,
+                                           float dcell, float dnet) {
+  if (flags & 2u) {
+    for (int o = __ldg(P.ov_ptr + s); o < __ldg(P.ov_ptr + s + 1); ++o)
+      if (__ldg(P.ov_pos + o) == q) return __ldg(P.ov_ms + o);
+  }
+  const float d = (flags & 1u) ? dcell : dnet;
+  return make_float4(ms.x * d, ms.y * d, ms.z * d, ms.w * d);
+}
+
+__device__ __forceinline__ Raw ldb_raw(const BParams& P, int j, int s) {
+  Raw r;
+  asm volatile("ld.relaxed.gpu.global.v4.b64 {%0, %1, %2, %3}, [%4];"
+               : "=l"(r.a), "=l"(r.b), "=l"(r.c), "=l"(r.d)
+               : "l"(P.bstate + size_t(j) * kLanes + s)
+               : "memory");
+  return r;
+}
+
+__device__ __forceinline__ void awaitb(const BParams& P, int j, int s, Raw& r) {
+  while (!raw_ready(r, P.par)) {
+    __nanosleep(20);
+    r = ldb_raw(P, j, s);
+  }
+}
+
+__device__ __forceinline__ void storeb(const BParams& P, int i, int s, double m0, double m1, double v0,
+                                       double v1) {
+  asm volatile("st.relaxed.gpu.global.v4.f64 [%0], {%1, %2, %3, %4};" ::"l"(P.bstate + size_t(i) * kLanes + s),
+               "d"(with_par(m0, P.par)), "d"(with_par(m1, P.par)), "d"(with_par(v0, P.par)),
+               "d"(with_par(v1, P.par))
+               : "memory");
+}
+
+// ---------------------------------------------------------------- forward
+struct BFwdStage {
+  int32_t ptr[kFwdPins + 8];
+  int32_t src[kFwdArcs + 8];
+  uint8_t flags[kFwdArcs + 32];
+  float4 ms[kFwdArcs];
+};
+constexpr size_t kBFwdSmem = 2 * sizeof(BFwdStage);
+
+__device__ __forceinline__ bool bfwd_staged(const int4& A, const int4& B) {
+  return A.y > A.x && B.x > 0 && !(B.y & kItemDirect);
+}
+
+__device__ __forceinline__ void bfwd_prefetch(const BParams& P, BFwdStage* st, uint64_t* full, int step, int c) {
+  const int4 A = __ldg(P.item_a + size_t(step) * P.grid + c);
+  const int4 B = __ldg(P.item_b + size_t(step) * P.grid + c);
+  if (!bfwd_staged(A, B)) return;
+  const Window wp = window(A.x, A.y + 1, 4);
+  const Window ws = window(A.z, A.w, 4);
+  const Window wf = window(A.z, A.w, 1);
+  const uint32_t bms = uint32_t(A.w - A.z) * 16u;
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  mbar_expect_tx(full, wp.bytes + ws.bytes + wf.bytes + bms);
+  bulk_g2s(st->ptr, P.fanin_ptr + wp.start, wp.bytes, full);
+  if (ws.bytes) {
+    bulk_g2s(st->src, P.fin_src + ws.start, ws.bytes, full);
+    bulk_g2s(st->flags, P.fin_flags + wf.start, wf.bytes, full);
+    bulk_g2s(st->ms, P.fin_ms + A.z, bms, full);
+  }
+}
+
+// Merge of (pin, rf) for scenario lane s over nf arcs; arc(k, w, ms_s, raw).
+struct RfOutB {
+  double mu, var, best;
+  float sum;
+  int win;
+};
+
+template <bool kLSE, class ArcFn>
+__device__ __forceinline__ RfOutB pin_rf_b(const BParams& P, double ns, int rf, int nf, ArcFn&& arc) {
+  Merge m;
+  merge_init(m);
+  for (int k = 0; k < nf; ++k) {
+    int32_t w;
+    float4 ms;
+    Raw r;
+    arc(k, w, ms, r);
+    const Gath st = unpack(r);
+    const int u = int(uint32_t(w) >> kUnateShift);
+    const int s0 = src_tr(rf, u, 0);
+    merge_max(m, make_cand(st, ms, rf, s0, ns), k, s0);
+    if (u == 2) merge_max(m, make_cand(st, ms, rf, rf ^ 1, ns), k, rf ^ 1);
+  }
+  RfOutB o;
+  o.best = m.best;
+  o.var = m.var;
+  o.win = m.k | (m.s << 15);
+  o.sum = 0.f;
+  o.mu = m.mu;
+  if (kLSE) {
+    float sum = 0.f;
+    for (int k = 0; k < nf; ++k) {
+      int32_t w;
+      float4 ms;
+      Raw r;
+      arc(k, w, ms, r);
+      const Gath st = unpack(r);
+      const int u = int(uint32_t(w) >> kUnateShift);
+      sum += lse_term(make_cand(st, ms, rf, src_tr(rf, u, 0), ns), m, P.inv_tau);
+      if (u == 2) sum += lse_term(make_cand(st, ms, rf, rf ^ 1, ns), m, P.inv_tau);
+    }
+    o.sum = sum;
+    o.mu = (m.best + double(P.tau) * double(logf(sum))) - ns * double(m.sig);
+  }
+  return o;
+}
+
+template <class ArcFn>
+__device__ __forceinline__ float2 arc_rf_weights_b(const BParams& P, double ns, int rf, int k, const RfOutB& o,
+                                                   ArcFn&& arc) {
+  int32_t w;
+  float4 ms;
+  Raw r;
+  arc(k, w, ms, r);
+  const Gath st = unpack(r);
+  const int u = int(uint32_t(w) >> kUnateShift);
+  float wt[2] = {0.f, 0.f};
+  const int s0 = src_tr(rf, u, 0);
+  Merge m;
+  m.best = o.best;
+  wt[s0] = lse_term(make_cand(st, ms, rf, s0, ns), m, P.inv_tau) / o.sum;
+  if (u == 2) wt[rf ^ 1] = lse_term(make_cand(st, ms, rf, rf ^ 1, ns), m, P.inv_tau) / o.sum;
+  return make_float2(wt[0], wt[1]);
+}
+
+constexpr int kRegArcsB = 4;
+
+template <bool kLSE>
+__global__ void __launch_bounds__(kThreads, 1) fwdb_kernel(BParams P) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  BFwdStage* stage = reinterpret_cast<BFwdStage*>(smem);
+  __shared__ __align__(8) uint64_t full[2];
+  const int c = blockIdx.x, tid = threadIdx.x;
+  const int warp = tid >> 5, s = tid & 31;
+  const bool lane_on = s < P.nb;
+  const double ns = double(__ldg(P.sc + s));
+  const float dcell = __ldg(P.sc + kLanes + s), dnet = __ldg(P.sc + 2 * kLanes + s);
+  if (tid == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&full[0])) : "memory");
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&full[1])) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  uint32_t phase[2] = {0u, 0u};
+  const int nsteps = P.step_end - P.step_begin;
+  if (tid == 0 && nsteps > 0) bfwd_prefetch(P, &stage[0], &full[0], P.step_begin, c);
+  for (int t = 0; t < nsteps; ++t) {
+    const int buf = t & 1, k = P.step_begin + t;
+    const int4 A = __ldg(P.item_a + size_t(k) * P.grid + c);
+    const int4 B = __ldg(P.item_b + size_t(k) * P.grid + c);
+    if (tid == 0 && t + 1 < nsteps) bfwd_prefetch(P, &stage[buf ^ 1], &full[buf ^ 1], k + 1, c);
+    if (A.y > A.x) {
+      if (B.x == 0) {
+        for (int i = A.x + warp; i < A.y; i += kThreads / 32) {
+          if (!lane_on) continue;
+          const float4 v = __ldg(P.src_ms + i);
+          storeb(P, i, s, double(v.x), double(v.y), double(v.z) * double(v.z), double(v.w) * double(v.w));
+        }
+      } else {
+        const bool staged = !(B.y & kItemDirect);
+        if (staged) {
+          mbar_wait(&full[buf], phase[buf]);
+          phase[buf] ^= 1u;
+        }
+        const BFwdStage& S = stage[buf];
+        const int po = A.x & 3, so = A.z & 3, fo = A.z & 15;
+        for (int p = warp; p < A.y - A.x && lane_on; p += kThreads / 32) {
+          const int i = A.x + p;
+          int b0, nf;
+          if (staged) {
+            b0 = S.ptr[po + p] - A.z;
+            nf = S.ptr[po + p + 1] - A.z - b0;
+          } else {
+            b0 = __ldg(P.fanin_ptr + i) - A.z;
+            nf = __ldg(P.fanin_ptr + i + 1) - A.z - b0;
+          }
+          // gather the first kRegArcsB source entries of this scenario together
+          Raw rr[kRegArcsB];
+          int32_t ww[kRegArcsB];
+#pragma unroll
+          for (int kk = 0; kk < kRegArcsB; ++kk) {
+            if (kk < nf) {
+              ww[kk] = staged ? S.src[so + b0 + kk] : __ldg(P.fin_src + A.z + b0 + kk);
+              rr[kk] = ldb_raw(P, ww[kk] & kSrcMask, s);
+            }
+          }
+#pragma unroll
+          for (int kk = 0; kk < kRegArcsB; ++kk)
+            if (kk < nf) awaitb(P, ww[kk] & kSrcMask, s, rr[kk]);
+          auto arc = [&](int kk, int32_t& w, float4& ms, Raw& r) {
+            const int q = A.z + b0 + kk;
+            float4 m0;
+            uint32_t fl;
+            if (staged) {
+              w = S.src[so + b0 + kk];
+              m0 = S.ms[b0 + kk];
+              fl = S.flags[fo + b0 + kk];
+            } else {
+              w = __ldg(P.fin_src + q);
+              m0 = __ldg(P.fin_ms + q);
+              fl = __ldg(P.fin_flags + q);
+            }
+            ms = scen_arc(P, m0, fl, q, s, dcell, dnet);
+            if (kk < kRegArcsB) {
+              r = rr[0];
+#pragma unroll
+              for (int x = 1; x < kRegArcsB; ++x)
+                if (x == kk) r = rr[x];
+            } else {
+              r = ldb_raw(P, w & kSrcMask, s);
+              awaitb(P, w & kSrcMask, s, r);
+            }
+          };
+          const RfOutB R = pin_rf_b<kLSE>(P, ns, 0, nf, arc);
+          const RfOutB F = pin_rf_b<kLSE>(P, ns, 1, nf, arc);
+          storeb(P, i, s, R.mu, F.mu, R.var, F.var);
+          if (!kLSE) {
+            P.bwin[size_t(i) * kLanes + s] = R.win | (F.win << 16);
+          } else {
+            for (int kk = 0; kk < nf; ++kk) {
+              const float2 wr = arc_rf_weights_b(P, ns, 0, kk, R, arc);
+              const float2 wf = arc_rf_weights_b(P, ns, 1, kk, F, arc);
+              P.bwts[size_t(A.z + b0 + kk) * kLanes + s] = make_float4(wr.x, wr.y, wf.x, wf.y);
+            }
+          }
+        }
+      }
+    }
+    __syncthreads();
+  }
+}
+
+// ---------------------------------------------------------------- slack
+// slack[ep][s] = RAT - A (min over rf, tie -> R); per-scenario WNS/TNS/#viol
+// via fixed-order reductions (block partials over endpoints, then the last block).
+constexpr int kSlackEps = 8;   // endpoint rows per 256-thread block iteration
+
+__global__ void __launch_bounds__(256) slackb_kernel(int num_ep, int nb, const int32_t* __restrict__ ep_pin,
+                                                     const float2* __restrict__ ep_rat,
+                                                     const PinState* __restrict__ bstate,
+                                                     const float* __restrict__ sc, float* bslack, uint8_t* brf,
+                                                     double* partials, uint32_t* ticket, double* summaries) {
+  __shared__ double st[3][kSlackEps][kLanes];
+  __shared__ bool s_last;
+  const int s = threadIdx.x & 31, row = threadIdx.x >> 5;
+  const double ns = double(sc[s]);
+  double tns = 0.0, wns = 0.0, nv = 0.0;
+  const int per_block = kSlackEps * 64;
+  const int e0 = blockIdx.x * per_block;
+  for (int e = e0 + row; e < min(num_ep, e0 + per_block); e += kSlackEps) {
+    if (s >= nb) continue;
+    const double2 m = __ldcg(reinterpret_cast<const double2*>(bstate + size_t(ep_pin[e]) * kLanes + s));
+    const double2 v = __ldcg(reinterpret_cast<const double2*>(bstate + size_t(ep_pin[e]) * kLanes + s) + 1);
+    const float2 rat = ep_rat[e];
+    const double aR = strip((unsigned long long)__double_as_longlong(m.x)) +
+                      ns * double(sigma_of(strip((unsigned long long)__double_as_longlong(v.x))));
+    const double aF = strip((unsigned long long)__double_as_longlong(m.y)) +
+                      ns * double(sigma_of(strip((unsigned long long)__double_as_longlong(v.y))));
+    const double sR = double(rat.x) - aR, sF = double(rat.y) - aF;
+    const bool fall = sF < sR;
+    const double sl = fall ? sF : sR;
+    bslack[size_t(e) * kLanes + s] = float(sl);
+    brf[size_t(e) * kLanes + s] = fall ? 1 : 0;
+    if (sl < 0.0) {
+      tns += sl;
+      nv += 1.0;
+      wns = fmin(wns, sl);
+    }
+  }
+  st[0][row][s] = tns;
+  st[1][row][s] = wns;
+  st[2][row][s] = nv;
+  __syncthreads();
+  if (row == 0) {
+    for (int r = 1; r < kSlackEps; ++r) {
+      tns += st[0][r][s];
+      wns = fmin(wns, st[1][r][s]);
+      nv += st[2][r][s];
+    }
+    partials[(size_t(blockIdx.x) * 3 + 0) * kLanes + s] = tns;
+    partials[(size_t(blockIdx.x) * 3 + 1) * kLanes + s] = wns;
+    partials[(size_t(blockIdx.x) * 3 + 2) * kLanes + s] = nv;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    s_last = atomicAdd(ticket, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (!s_last || row != 0) return;
+  __threadfence();
+  tns = 0.0;
+  wns = 0.0;
+  nv = 0.0;
+  for (int b = 0; b < int(gridDim.x); ++b) {
+    tns += __ldcg(partials + (size_t(b) * 3 + 0) * kLanes + s);
+    wns = fmin(wns, __ldcg(partials + (size_t(b) * 3 + 1) * kLanes + s));
+    nv += __ldcg(partials + (size_t(b) * 3 + 2) * kLanes + s);
+  }
+  if (s < nb) {
+    summaries[size_t(s) * 3 + 0] = wns;
+    summaries[size_t(s) * 3 + 1] = tns;
+    summaries[size_t(s) * 3 + 2] = nv;
+  }
+  if (s == 0) *ticket = 0u;
+}
+
+// ---------------------------------------------------------------- backward
+struct BBwdStage {
+  int32_t lptr[kBwdPins + 8];
+  int32_t lfo[kBwdFanout + 8];
+  int32_t fptr[kBwdPins + 8];
+  int32_t src[kBwdArcs + 8];
+  int32_t arc[kBwdArcs + 8];
+  int32_t hslot[kBwdPins + 8];
+  int32_t eop[kBwdPins + 8];
+};
+constexpr size_t kBBwdSmem = 2 * sizeof(BBwdStage);
+
+__device__ __forceinline__ void bbwd_prefetch(const BParams& P, BBwdStage* st, uint64_t* full, int step, int c) {
+  const int4 A = __ldg(P.item_a + size_t(step) * P.grid + c);   // {pin_lo, pin_hi, lfo_lo, lfo_hi}
+  const int4 B = __ldg(P.item_b + size_t(step) * P.grid + c);   // {arc_lo, arc_hi, level, flags}
+  if (!(A.y > A.x && !(B.w & kItemDirect))) return;
+  const Window wl = window(A.x, A.y + 1, 4);
+  const Window wf = window(A.z, A.w, 4);
+  const Window wa = window(B.x, B.y, 4);
+  const Window ww = window(A.x, A.y, 4);
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  mbar_expect_tx(full, 2 * wl.bytes + wf.bytes + 2 * wa.bytes + 2 * ww.bytes);
+  bulk_g2s(st->lptr, P.lfo_ptr + wl.start, wl.bytes, full);
+  if (wf.bytes) bulk_g2s(st->lfo, P.lfo + wf.start, wf.bytes, full);
+  bulk_g2s(st->fptr, P.fanin_ptr + wl.start, wl.bytes, full);
+  if (wa.bytes) {
+    bulk_g2s(st->src, P.fin_src + wa.start, wa.bytes, full);
+    bulk_g2s(st->arc, P.fin_arc + wa.start, wa.bytes, full);
+  }
+  bulk_g2s(st->hslot, P.heavy_slot + ww.start, ww.bytes, full);
+  bulk_g2s(st->eop, P.ep_of_pin + ww.start, ww.bytes, full);
+}
+
+__device__ __forceinline__ float2 loadb_g(const BParams& P, int q, int s) {
+  uint32_t a, b;
+  const float2* p = P.bg + size_t(q) * kLanes + s;
+  ld2_u32(p, a, b);
+  while (((a & 1u) != P.par) || ((b & 1u) != P.par)) {
+    __nanosleep(20);
+    ld2_u32(p, a, b);
+  }
+  return make_float2(stripf(a), stripf(b));
+}
+
+__device__ __forceinline__ float warp_sum(float v) {
+#pragma unroll
+  for (int d = 16; d >= 1; d >>= 1) v += __shfl_xor_sync(0xffffffffu, v, d);
+  return v;
+}
+
+template <bool kLSE>
+__global__ void __launch_bounds__(kThreads, 1) bwdb_kernel(BParams P) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  BBwdStage* stage = reinterpret_cast<BBwdStage*>(smem);
+  __shared__ __align__(8) uint64_t full[2];
+  const int c = blockIdx.x, tid = threadIdx.x;
+  const int warp = tid >> 5, s = tid & 31;
+  const bool lane_on = s < P.nb;
+  if (tid == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&full[0])) : "memory");
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&full[1])) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  uint32_t phase[2] = {0u, 0u};
+  const int nsteps = P.step_end - P.step_begin;
+  if (tid == 0 && nsteps > 0) bbwd_prefetch(P, &stage[0], &full[0], P.step_begin, c);
+  for (int t = 0; t < nsteps; ++t) {
+    const int buf = t & 1, k = P.step_begin + t;
+    const int4 A = __ldg(P.item_a + size_t(k) * P.grid + c);
+    const int4 B = __ldg(P.item_b + size_t(k) * P.grid + c);
+    const int l = B.z;
+    if (tid == 0 && t + 1 < nsteps) bbwd_prefetch(P, &stage[buf ^ 1], &full[buf ^ 1], k + 1, c);
+    if (A.y > A.x) {
+      const bool staged = !(B.w & kItemDirect);
+      if (staged) {
+        mbar_wait(&full[buf], phase[buf]);
+        phase[buf] ^= 1u;
+      }
+      const BBwdStage& S = stage[buf];
+      const int lo = A.x & 3, fo = A.z & 3, ao = B.x & 3;
+      for (int p = warp; p < A.y - A.x; p += kThreads / 32) {
+        const int i = A.x + p;
+        const int r0 = (staged ? S.lptr[lo + p] : __ldg(P.lfo_ptr + i)) - (staged ? A.z : 0);
+        const int r1 = (staged ? S.lptr[lo + p + 1] : __ldg(P.lfo_ptr + i + 1)) - (staged ? A.z : 0);
+        const int slot = staged ? S.hslot[lo + p] : __ldg(P.heavy_slot + i);
+        const int ep = staged ? S.eop[lo + p] : __ldg(P.ep_of_pin + i);
+        float ax = 0.f, ay = 0.f;
+        if (lane_on) {
+          // pull (row order, fixed) + seed + heavy accumulator
+          for (int r = r0; r < r1; ++r) {
+            const int q = staged ? S.lfo[fo + r] : __ldg(P.lfo + r);
+            const float2 v = loadb_g(P, q, s);
+            ax += v.x;
+            ay += v.y;
+          }
+          if (slot >= 0) {
+            unsigned long long* acc = P.bheavy + (size_t(slot) * kLanes + s) * 2;
+            const long long target = __ldg(P.heavy_fo + slot);
+            unsigned long long x, y;
+            ld2_u64(acc, x, y);
+            while (((long long)x + (kCountUnitB >> 1)) >> 44 != target ||
+                   ((long long)y + (kCountUnitB >> 1)) >> 44 != target) {
+              __nanosleep(32);
+              ld2_u64(acc, x, y);
+            }
+            asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %1};" ::"l"(acc), "l"(0ull) : "memory");
+            ax += float(double((long long)x - target * kCountUnitB) / kFixB);
+            ay += float(double((long long)y - target * kCountUnitB) / kFixB);
+          }
+          float sx = 0.f, sy = 0.f;
+          if (ep >= 0) {   // TNS seed: dL/dA[rf*] = -1 where slack < 0
+            const float sl = P.bslack[size_t(ep) * kLanes + s];
+            if (sl < 0.f) {
+              if (P.brf[size_t(ep) * kLanes + s]) sy = -1.f;
+              else sx = -1.f;
+            }
+          }
+          ax = sx + ax;
+          ay = sy + ay;
+        }
+        if (l == 0) continue;
+        const int b0 = staged ? S.fptr[lo + p] - B.x : __ldg(P.fanin_ptr + i) - B.x;
+        const int nf = (staged ? S.fptr[lo + p + 1] : __ldg(P.fanin_ptr + i + 1)) - B.x - b0;
+        const int32_t win = (!kLSE && lane_on) ? P.bwin[size_t(i) * kLanes + s] : 0;
+        for (int kk = 0; kk < nf; ++kk) {   // warp-uniform loop (same pin in all lanes)
+          const int q = B.x + b0 + kk;
+          const int32_t srcw = staged ? S.src[ao + b0 + kk] : __ldg(P.fin_src + q);
+          const int32_t arcid = staged ? S.arc[ao + b0 + kk] : __ldg(P.fin_arc + q);
+          float w[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
+          if (lane_on) {
+            if (kLSE) {
+              const float4 w4 = P.bwts[size_t(q) * kLanes + s];
+              w[0][0] = w4.x;
+              w[0][1] = w4.y;
+              w[1][0] = w4.z;
+              w[1][1] = w4.w;
+            } else {
+#pragma unroll
+              for (int rf = 0; rf < 2; ++rf) {
+                const int wv = (win >> (16 * rf)) & 0xffff;
+                const bool hit = (wv & 0x7fff) == kk;
+                w[rf][0] = (hit && (wv >> 15) == 0) ? 1.f : 0.f;
+                w[rf][1] = (hit && (wv >> 15) == 1) ? 1.f : 0.f;
+              }
+            }
+          }
+          const float abr[2] = {ax, ay};
+          float gm[2], gs[2] = {0.f, 0.f};
+#pragma unroll
+          for (int rf = 0; rf < 2; ++rf) {
+            const float a0 = w[rf][0] * abr[rf], a1 = w[rf][1] * abr[rf];
+            gm[rf] = a0 + a1;
+            gs[0] += a0;
+            gs[1] += a1;
+          }
+          if (lane_on) {
+            st2_f32(P.bg + size_t(q) * kLanes + s, with_parf(gs[0], P.par), with_parf(gs[1], P.par));
+            if ((srcw >> kHeavyBit) & 1) {
+              const int hs = __ldg(P.heavy_slot + (srcw & kSrcMask));
+              unsigned long long* acc = P.bheavy + (size_t(hs) * kLanes + s) * 2;
+              atomicAdd(acc, (unsigned long long)(kCountUnitB + __double2ll_rn(double(gs[0]) * kFixB)));
+              atomicAdd(acc + 1, (unsigned long long)(kCountUnitB + __double2ll_rn(double(gs[1]) * kFixB)));
+            }
+          }
+          // sum over scenarios of dTNS_s/d(arc mean'), fixed xor tree
+          const float t0 = warp_sum(gm[0]), t1 = warp_sum(gm[1]);
+          if (s == 0 && (t0 != 0.f || t1 != 0.f)) {
+            float2* o = reinterpret_cast<float2*>(P.d_mean_sum) + arcid;
+            const float2 prev = *o;
+            *o = make_float2(prev.x + t0, prev.y + t1);
+          }
+        }
+      }
+    }
+    __syncthreads();
+  }
+}
+
+// ---------------------------------------------------------------- flags scatter
+__global__ void set_flag_kernel(int n, const int32_t* __restrict__ pos, uint8_t* flags, uint8_t bit, int on) {
+  const int k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k >= n) return;
+  if (on) flags[pos[k]] |= bit;
+  else flags[pos[k]] &= uint8_t(~bit);
+}
+
+// ---------------------------------------------------------------- host side
+template <class K>
+static int set_smem_b(K kernel, size_t bytes) {
+  return int(cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(bytes)));
+}
+
+static int ensure_batch(DevGraph& g, bool lse, bool grad) {
+  static bool attrs = false;
+  if (!attrs) {
+    int err = set_smem_b(fwdb_kernel<false>, kBFwdSmem);
+    if (!err) err = set_smem_b(fwdb_kernel<true>, kBFwdSmem);
+    if (!err) err = set_smem_b(bwdb_kernel<false>, kBBwdSmem);
+    if (!err) err = set_smem_b(bwdb_kernel<true>, kBBwdSmem);
+    if (err) return err;
+    attrs = true;
+  }
+  auto alloc = [](void** p, size_t bytes) -> int {
+    if (*p) return 0;
+    cudaError_t e = cudaMalloc(p, bytes + 64);
+    if (e != cudaSuccess) return int(e);
+    return int(cudaMemset(*p, 0, bytes + 64));
+  };
+  const size_t n = size_t(std::max(g.n, 1)), e = size_t(std::max<int64_t>(g.e, 1));
+  int err = alloc(reinterpret_cast<void**>(&g.b_state), n * kLanes * sizeof(PinState));
+  if (!err) err = alloc(reinterpret_cast<void**>(&g.b_sc), 3 * kLanes * sizeof(float));
+  if (!err) err = alloc(reinterpret_cast<void**>(&g.b_ov_ptr), (kLanes + 1) * sizeof(int32_t));
+  if (!err) err = alloc(reinterpret_cast<void**>(&g.b_slack), size_t(std::max(g.num_ep, 1)) * kLanes * sizeof(float));
+  if (!err) err = alloc(reinterpret_cast<void**>(&g.b_rf), size_t(std::max(g.num_ep, 1)) * kLanes);
+  if (!err) err = alloc(reinterpret_cast<void**>(&g.b_partials),
+                        size_t((g.num_ep + kSlackEps * 64 - 1) / (kSlackEps * 64) + 1) * 3 * kLanes * sizeof(double));
+  if (!err) err = alloc(reinterpret_cast<void**>(&g.b_ticket), sizeof(uint32_t));
+  if (!err && !lse) err = alloc(reinterpret_cast<void**>(&g.b_win), n * kLanes * sizeof(int32_t));
+  if (!err && lse) err = alloc(reinterpret_cast<void**>(&g.b_wts), e * kLanes * sizeof(float4));
+  if (!err && grad) err = alloc(reinterpret_cast<void**>(&g.b_g), e * kLanes * sizeof(float2));
+  if (!err && grad) err = alloc(reinterpret_cast<void**>(&g.b_heavy),
+                                size_t(std::max(g.num_heavy, 1)) * kLanes * 2 * sizeof(unsigned long long));
+  return err;
+}
+
+static BParams make_bparams(DevGraph& g, bool bwd) {
+  BParams P{};
+  P.n = g.n;
+  P.num_levels = g.num_levels;
+  P.grid = g.grid;
+  P.item_a = bwd ? g.bwd_a : g.fwd_a;
+  P.item_b = bwd ? g.bwd_b : g.fwd_b;
+  P.fanin_ptr = g.fanin_ptr;
+  P.fin_src = g.fin_src;
+  P.fin_ms = g.fin_ms;
+  P.fin_flags = g.fin_flags;
+  P.fin_arc = g.fin_arc;
+  P.lfo_ptr = g.lfo_ptr;
+  P.lfo = g.lfo;
+  P.heavy_slot = g.heavy_slot;
+  P.heavy_fo = g.heavy_fo;
+  P.ep_of_pin = g.ep_of_pin;
+  P.src_ms = g.src_ms;
+  P.sc = g.b_sc;
+  P.ov_ptr = g.b_ov_ptr;
+  P.ov_pos = g.b_ov_pos;
+  P.ov_ms = g.b_ov_ms;
+  P.bstate = g.b_state;
+  P.bwin = g.b_win;
+  P.bwts = g.b_wts;
+  P.bg = g.b_g;
+  P.bheavy = g.b_heavy;
+  P.bslack = g.b_slack;
+  P.brf = g.b_rf;
+  return P;
+}
+
+int launch_forward_batch(DevGraph& g, int nb, const float* sc_host /*[3][32]*/, const std::vector<int32_t>& ov_ptr,
+                         const std::vector<int32_t>& ov_pos, const std::vector<float4>& ov_ms, float tau,
+                         double* summaries, float* d_mean_sum, void* stream) {
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  const bool lse = tau > 0.f, grad = d_mean_sum != nullptr;
+  int err = ensure_batch(g, lse, grad);
+  if (err) return err;
+  cudaError_t e = cudaMemcpyAsync(g.b_sc, sc_host, 3 * kLanes * sizeof(float), cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(g.b_ov_ptr, ov_ptr.data(), (kLanes + 1) * sizeof(int32_t), cudaMemcpyHostToDevice, st);
+  const int nov = int(ov_pos.size());
+  if (e == cudaSuccess && nov > g.b_ov_cap) {
+    cudaFree(g.b_ov_pos);
+    cudaFree(g.b_ov_ms);
+    g.b_ov_pos = nullptr;
+    g.b_ov_ms = nullptr;
+    e = cudaMalloc(&g.b_ov_pos, sizeof(int32_t) * nov + 64);
+    if (e == cudaSuccess) e = cudaMalloc(&g.b_ov_ms, sizeof(float4) * nov + 64);
+    g.b_ov_cap = nov;
+  }
+  if (e == cudaSuccess && nov > 0) {
+    e = cudaMemcpyAsync(g.b_ov_pos, ov_pos.data(), sizeof(int32_t) * nov, cudaMemcpyHostToDevice, st);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(g.b_ov_ms, ov_ms.data(), sizeof(float4) * nov, cudaMemcpyHostToDevice, st);
+    if (e == cudaSuccess) {
+      set_flag_kernel<<<(nov + 255) / 256, 256, 0, st>>>(nov, g.b_ov_pos, g.fin_flags, 2, 1);
+      e = cudaGetLastError();
+    }
+  }
+  if (e != cudaSuccess) return int(e);
+  BParams P = make_bparams(g, false);
+  P.nb = nb;
+  P.tau = tau;
+  P.inv_tau = lse ? 1.0 / double(tau) : 0.0;
+  P.par = (++g.pass_bfwd) & 1u;
+  P.step_begin = 0;
+  P.step_end = g.fwd_items.num_steps;
+  if (g.n > 0) {
+    void* args[] = {&P};
+    e = cudaLaunchCooperativeKernel(lse ? (const void*)fwdb_kernel<true> : (const void*)fwdb_kernel<false>,
+                                    dim3(g.grid), dim3(kThreads), args, kBFwdSmem, st);
+    if (e != cudaSuccess) return int(e);
+  }
+  if (g.num_ep > 0) {
+    const int blocks = (g.num_ep + kSlackEps * 64 - 1) / (kSlackEps * 64);
+    slackb_kernel<<<blocks, 256, 0, st>>>(g.num_ep, nb, g.ep_pin, g.ep_rat, g.b_state, g.b_sc, g.b_slack, g.b_rf,
+                                          g.b_partials, g.b_ticket, summaries);
+    e = cudaGetLastError();
+  } else {
+    e = cudaMemsetAsync(summaries, 0, sizeof(double) * 3 * nb, st);
+  }
+  if (e != cudaSuccess) return int(e);
+  if (grad && g.n > 0) {
+    BParams Q = make_bparams(g, true);
+    Q.nb = nb;
+    Q.tau = tau;
+    Q.inv_tau = P.inv_tau;
+    Q.par = (++g.pass_bbwd) & 1u;
+    Q.d_mean_sum = d_mean_sum;
+    Q.step_begin = 0;
+    Q.step_end = g.bwd_items.num_steps;
+    void* args[] = {&Q};
+    e = cudaLaunchCooperativeKernel(lse ? (const void*)bwdb_kernel<true> : (const void*)bwdb_kernel<false>,
+                                    dim3(g.grid), dim3(kThreads), args, kBBwdSmem, st);
+    if (e != cudaSuccess) return int(e);
+  }
+  if (nov > 0) {
+    set_flag_kernel<<<(nov + 255) / 256, 256, 0, st>>>(nov, g.b_ov_pos, g.fin_flags, 2, 0);
+    e = cudaGetLastError();
+  }
+  return int(e);
+}
+
+}  // namespace insta

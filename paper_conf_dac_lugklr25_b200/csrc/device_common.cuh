@@ -1,0 +1,182 @@
+// device_common.cuh -- PTX helpers shared by the single-scenario (kernels.cu)
+// and batched (batch.cu) propagation kernels: memory-model accesses, the
+// parity-tagged words of the dataflow synchronization, mbarrier + TMA bulk
+// copies, and the per-candidate primitives of Eq 1-3.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+namespace insta {
+
+// --------------------------------------------------------------------------
+// PTX helpers: memory model, mbarrier, TMA bulk copy
+// --------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ uint32_t ld_acquire(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+// ---- parity-tagged words ----
+__device__ __forceinline__ double with_par(double x, uint32_t par) {
+  return __longlong_as_double((__double_as_longlong(x) & ~1ll) | (long long)par);
+}
+__device__ __forceinline__ double strip(unsigned long long b) { return __longlong_as_double((long long)(b & ~1ull)); }
+__device__ __forceinline__ float with_parf(float x, uint32_t par) {
+  return __uint_as_float((__float_as_uint(x) & ~1u) | par);
+}
+__device__ __forceinline__ float stripf(uint32_t b) { return __uint_as_float(b & ~1u); }
+
+__device__ __forceinline__ void ld2_u64(const void* p, unsigned long long& a, unsigned long long& b) {
+  asm volatile("ld.relaxed.gpu.global.v2.b64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
+}
+__device__ __forceinline__ void st2_u64(void* p, double a, double b) {
+  asm volatile("st.relaxed.gpu.global.v2.f64 [%0], {%1, %2};" ::"l"(p), "d"(a), "d"(b) : "memory");
+}
+__device__ __forceinline__ void ld2_u32(const void* p, uint32_t& a, uint32_t& b) {
+  asm volatile("ld.relaxed.gpu.global.v2.b32 {%0, %1}, [%2];" : "=r"(a), "=r"(b) : "l"(p) : "memory");
+}
+__device__ __forceinline__ void st2_f32(void* p, float a, float b) {
+  asm volatile("st.relaxed.gpu.global.v2.f32 [%0], {%1, %2};" ::"l"(p), "f"(a), "f"(b) : "memory");
+}
+
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAIT_%=;\n}" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+
+__device__ __forceinline__ void bulk_g2s(void* sdst, const void* gsrc, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(sdst)),
+      "l"(gsrc), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+// 16-byte aligned window covering elements [a, b) of an array of esz-byte items
+struct Window {
+  int32_t off;     // element offset of a inside the window
+  uint32_t bytes;  // bytes to copy
+  int64_t start;   // first element copied
+};
+
+__device__ __forceinline__ Window window(int64_t a, int64_t b, int esz) {
+  const int per = 16 / esz;
+  Window w;
+  w.start = a - (a % per);
+  const int64_t end = ((b + per - 1) / per) * per;
+  w.off = int32_t(a - w.start);
+  w.bytes = b > a ? uint32_t((end - w.start) * esz) : 0u;
+  return w;
+}
+
+__device__ __forceinline__ float sigma_of(double var) { return sqrtf(float(var)); }
+
+// source transitions of an arc for sink transition rf: POS {rf}; NEG {~rf}
+// (Alg 1 l.8); NON (rf, ~rf) (reading R3).
+__device__ __forceinline__ int n_src_tr(int u) { return u == 2 ? 2 : 1; }
+__device__ __forceinline__ int src_tr(int rf, int u, int a) { return (u == 1 || a == 1) ? (rf ^ 1) : rf; }
+
+// --------------------------------------------------------------------------
+// Eq 1-3 for one candidate: arc e = (j -> i), sink transition rf, source
+// transition s.  State carries the variance (Eq 2 is additive in it):
+//   mu_c  = mu_j[s] + arc_mean[rf]                 (Eq 1, Alg 1 l.12)
+//   var_c = var_j[s] + arc_std[rf]^2               (Eq 2, Alg 1 l.13)
+//   A_c   = mu_c + n_sigma * sqrt(var_c)           (Eq 3, Alg 1 l.14)
+// mean and variance accumulate in fp64; the sqrt of the corner is fp32.
+// --------------------------------------------------------------------------
+struct Gath {
+  double mu0, mu1, v0, v1;
+};
+
+struct Cand {
+  double mu, var, A;
+  float sig;
+};
+
+
+// Pin state words as loaded (parity bits still in place).
+struct Raw {
+  unsigned long long a, b, c, d;
+};
+
+// one 256-bit access per 32-byte pin record (LDG/STG .256 on sm_100a)
+__device__ __forceinline__ bool raw_ready(const Raw& r, uint32_t par) {
+  return (((r.a & r.b & r.c & r.d) & 1ull) == par) && (((r.a | r.b | r.c | r.d) & 1ull) == par);
+}
+
+__device__ __forceinline__ Gath unpack(const Raw& r) {
+  Gath g;
+  g.mu0 = strip(r.a);
+  g.mu1 = strip(r.b);
+  g.v0 = strip(r.c);
+  g.v1 = strip(r.d);
+  return g;
+}
+
+__device__ __forceinline__ Cand make_cand(const Gath& st, const float4& ms, int rf, int s, double ns) {
+  const double se = double(rf ? ms.w : ms.z);
+  Cand c;
+  c.mu = (s ? st.mu1 : st.mu0) + double(rf ? ms.y : ms.x);
+  c.var = (s ? st.v1 : st.v0) + se * se;
+  c.sig = sigma_of(c.var);
+  c.A = c.mu + ns * double(c.sig);
+  return c;
+}
+
+
+// Merge of one (pin, rf): first arg-max (strict ">"), LSE normalizer.
+struct Merge {
+  double best, mu, var;
+  float sig, sum;
+  int k, s;
+};
+
+__device__ __forceinline__ void merge_init(Merge& m) {
+  m.best = 0.0;
+  m.mu = 0.0;
+  m.var = 0.0;
+  m.sig = 0.f;
+  m.sum = 0.f;
+  m.k = -1;
+  m.s = 0;
+}
+
+__device__ __forceinline__ void merge_max(Merge& m, const Cand& c, int k, int s) {
+  if (m.k < 0 || c.A > m.best) {   // Alg 2 l.4: replace only if strictly greater
+    m.best = c.A;
+    m.mu = c.mu;
+    m.var = c.var;
+    m.sig = c.sig;
+    m.k = k;
+    m.s = s;
+  }
+}
+
+// Eq 6 weight of a candidate given its merge (LSE)
+__device__ __forceinline__ float lse_term(const Cand& c, const Merge& m, double tau) {
+  return expf(float((c.A - m.best) * tau));   // tau: the inverse temperature 1/tau
+}
+
+}  // namespace insta

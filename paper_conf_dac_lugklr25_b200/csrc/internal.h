@@ -110,6 +110,25 @@ struct DevGraph {
   int32_t* ep_pin = nullptr;       // [P] canonical
   float2* ep_rat = nullptr;        // [P]
   uint8_t* arc_class = nullptr;    // [e] caller order (derates)
+  uint8_t* fin_flags = nullptr;    // [e] fanin order: bit 0 cell arc, bit 1 overridden in the current batch
+  int32_t* ep_of_pin = nullptr;    // [n] endpoint index of a canonical pin, -1 otherwise
+  std::vector<int32_t> h_arc_pos;  // host copy of arc_pos (batch overrides)
+  // batched scenarios (allocated on first use; scenario-minor, 32 lanes)
+  PinState* b_state = nullptr;
+  int32_t* b_win = nullptr;
+  float4* b_wts = nullptr;
+  float2* b_g = nullptr;
+  unsigned long long* b_heavy = nullptr;
+  float* b_sc = nullptr;
+  int32_t* b_ov_ptr = nullptr;
+  int32_t* b_ov_pos = nullptr;
+  float4* b_ov_ms = nullptr;
+  int32_t b_ov_cap = 0;
+  float* b_slack = nullptr;
+  uint8_t* b_rf = nullptr;
+  double* b_partials = nullptr;
+  uint32_t* b_ticket = nullptr;
+  uint32_t pass_bfwd = 0, pass_bbwd = 0;
   // item tables
   int4* fwd_a = nullptr;
   int4* fwd_b = nullptr;
@@ -165,4 +184,8 @@ int launch_update_arcs(DevGraph& g, int64_t n, const int32_t* ids, const float* 
                        const float* sigma, int incremental, void* stream);
 int launch_arrivals(DevGraph& g, float* A, float* mean, float* sigma, void* stream);
 int launch_copy_slack(DevGraph& g, float* slack, uint8_t* rf, void* stream);
+// batch.cu: up to 32 scenarios in one pass; sc = [3][32] {n_sigma, derate_cell, derate_net}
+int launch_forward_batch(DevGraph& g, int nb, const float* sc_host, const std::vector<int32_t>& ov_ptr,
+                         const std::vector<int32_t>& ov_pos, const std::vector<float4>& ov_ms, float tau,
+                         double* summaries, float* d_mean_sum, void* stream);
 }  // namespace insta

@@ -322,6 +322,45 @@ def sizing_step(g: Graph, step: int, frac: float = 0.01, base_seed: int = 3030):
     return ids, (g.arc_mean[ids] * fac).astype(np.float32), (g.arc_sigma[ids] * fac).astype(np.float32)
 
 
+def sizing_scenario(g: Graph, s: int, seed: int = 505, _cache={}):
+    """Sizing-candidate scenario s (C5 scenarios 512..1023): one random cell's arcs
+    scaled by U(.75, 1.05) and its input net arcs by U(1.0, 1.1) (mean and sigma
+    alike), as a scenario dict for insta_forward_batch (fp32 override values)."""
+    key = id(g)
+    if key not in _cache:
+        order, starts = _cell_groups(g)
+        net = np.nonzero(g.arc_class == NET)[0]
+        net_by_to = np.full(g.num_pins, -1, np.int64)
+        net_by_to[g.arc_to[net]] = net
+        _cache.clear()
+        _cache[key] = (order, starts, net_by_to)
+    order, starts, net_by_to = _cache[key]
+    rng = np.random.default_rng([seed, s])
+    c = int(rng.integers(starts.size - 1))
+    arcs = order[starts[c]:starts[c + 1]]
+    nets = net_by_to[g.arc_from[arcs]]
+    nets = nets[nets >= 0]
+    ids = np.concatenate([arcs, nets]).astype(np.int32)
+    fac = np.concatenate([np.full(arcs.size, rng.uniform(0.75, 1.05)), rng.uniform(1.0, 1.1, nets.size)])[:, None]
+    ids, first = np.unique(ids, return_index=True)
+    fac = fac[first]
+    return dict(n_sigma=3.0, derate_cell=1.0, derate_net=1.0, delta_arc=ids,
+                delta_mean=(g.arc_mean[ids] * fac).astype(np.float32),
+                delta_sigma=(g.arc_sigma[ids] * fac).astype(np.float32))
+
+
+def c5_scenarios(g: Graph, n: int = 1024, n_ocv: int = 512, seed: int = 505):
+    """The C5 workload: scenarios 0..n_ocv-1 are OCV (N_sigma, derates), the rest sizing candidates."""
+    out = []
+    for s in range(n):
+        if s < n_ocv:
+            ns, dc, dn = ocv_scenario(s, seed)
+            out.append(dict(n_sigma=ns, derate_cell=dc, derate_net=dn))
+        else:
+            out.append(sizing_scenario(g, s, seed))
+    return out
+
+
 def ocv_scenario(s: int, seed: int = 505):
     """OCV scenario s (C5 scenarios 0..511): (n_sigma, derate_cell, derate_net)."""
     rng = np.random.default_rng([seed, s])
