@@ -54,7 +54,7 @@ void free_graph(insta::DevGraph& d) {
                   d.rf_star,   d.partials,  d.ticket,    d.summary,    d.dirty,     d.counters,
                   d.fin_flags, d.ep_of_pin, d.b_state,   d.b_win,      d.b_wts,     d.b_g,
                   d.b_heavy,   d.b_sc,      d.b_ov_ptr,  d.b_ov_pos,   d.b_ov_ms,   d.b_slack,
-                  d.b_rf,      d.b_partials, d.b_ticket};
+                  d.b_rf,      d.b_partials, d.b_ticket,  d.pin_level,  d.lvl_range};
   for (void* p : ptrs)
     if (p) cudaFree(p);
 }
@@ -220,6 +220,9 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   if (desc->arc_class) std::copy(desc->arc_class, desc->arc_class + E, arc_class.begin());
   std::vector<uint8_t> fin_flags(nE, 0);
   for (int64_t q = 0; q < E; ++q) fin_flags[q] = arc_class[h.fanin_arc[q]] ? 1 : 0;
+  std::vector<int32_t> pin_level(nN);
+  for (int32_t k = 0; k < n; ++k) pin_level[k] = h.level[h.order[k]];
+  const int32_t lvl_init[2] = {0x7fffffff, -1};
   std::vector<int32_t> ep_of_pin(nN, -1);
   for (int32_t k = 0; k < d.num_ep; ++k) ep_of_pin[ep_pin[k]] = k;
   d.h_arc_pos = arc_pos;
@@ -254,6 +257,8 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   UP(d.arc_class, arc_class.data(), nE);
   UP(d.fin_flags, fin_flags.data(), nE);
   UP(d.ep_of_pin, ep_of_pin.data(), nN);
+  UP(d.pin_level, pin_level.data(), nN);
+  UP(d.lvl_range, lvl_init, 2);
   UP(d.fwd_a, d.fwd_items.a.data(), d.fwd_items.a.size());
   UP(d.fwd_b, d.fwd_items.b.data(), d.fwd_items.b.size());
   UP(d.bwd_a, d.bwd_items.a.data(), d.bwd_items.a.size());
@@ -341,12 +346,18 @@ insta_status insta_forward(insta_graph* g, const insta_opts* o, void* cuda_strea
   if (opt.schedule != 0 && opt.schedule != 1) return fail(INSTA_E_ARG, "forward: bad schedule");
   insta::DevGraph& d = g->d;
   cudaSetDevice(d.device);
-  int err = insta::launch_forward(d, opt.n_sigma, opt.tau, opt.schedule, cuda_stream);
+  // incremental cone pass when only incremental updates happened since a
+  // forward with the same options (persistent schedule)
+  const bool inc = d.pending_incremental && !d.pending_full && opt.schedule == 0 &&
+                   opt.n_sigma == d.last_n_sigma && opt.tau == d.last_tau;
+  int err = inc ? insta::launch_forward_incremental(d, opt.n_sigma, opt.tau, cuda_stream)
+                : insta::launch_forward(d, opt.n_sigma, opt.tau, opt.schedule, cuda_stream);
   if (err) return cuda_fail(err, "forward");
   d.bwd_schedule = opt.schedule;
   d.fwd_valid = true;
   d.pending_full = false;
   d.pending_incremental = false;
+  d.last_incremental = inc;
   d.last_recomputed = d.n;
   if (out) return read_summary(d, cuda_stream, out);
   return INSTA_OK;
@@ -462,7 +473,17 @@ insta_status insta_forward_batch(insta_graph* g, int32_t num_scenarios, const in
 
 insta_status insta_last_forward_stats(insta_graph* g, int64_t* pins_recomputed) {
   if (!g) return fail(INSTA_E_ARG, "stats: NULL graph");
-  if (pins_recomputed) *pins_recomputed = g->d.last_recomputed;
+  insta::DevGraph& d = g->d;
+  if (pins_recomputed) {
+    if (d.last_incremental) {
+      unsigned long long c[2] = {0, 0};
+      cudaError_t e = cudaMemcpy(c, d.counters, sizeof c, cudaMemcpyDeviceToHost);
+      if (e != cudaSuccess) return cuda_fail(int(e), "stats");
+      *pins_recomputed = int64_t(c[0]);
+    } else {
+      *pins_recomputed = d.last_recomputed;
+    }
+  }
   return INSTA_OK;
 }
 

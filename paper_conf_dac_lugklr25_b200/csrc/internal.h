@@ -150,6 +150,8 @@ struct DevGraph {
   double* summary = nullptr;       // {wns, tns, nviol} on device
   // incremental
   uint32_t* dirty = nullptr;       // [n] stamp == inc_epoch: pin must be recomputed
+  int32_t* pin_level = nullptr;    // [n] level of each canonical pin
+  int32_t* lvl_range = nullptr;    // [2] {min, max} level of pending dirty marks
   unsigned long long* counters = nullptr;  // [4] recomputed pins etc.
   // host-side bookkeeping
   HostLevels host;
@@ -161,6 +163,7 @@ struct DevGraph {
   bool pending_full = true;
   float last_n_sigma = 3.0f, last_tau = 0.0f;
   int64_t last_recomputed = 0;
+  bool last_incremental = false;
 };
 
 // item tables (items.cpp)

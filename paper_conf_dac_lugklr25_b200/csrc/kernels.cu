@@ -189,6 +189,18 @@ __device__ __forceinline__ float2 arc_rf_weights(const KParams& P, int rf, int k
   return make_float2(wt[0], wt[1]);
 }
 
+// State read outside a propagation pass (parity stripped, no waiting).
+__device__ __forceinline__ Gath load_state_plain(const PinState* p) {
+  const double2 m = __ldcg(reinterpret_cast<const double2*>(p));
+  const double2 v = __ldcg(reinterpret_cast<const double2*>(p) + 1);
+  Gath g;
+  g.mu0 = strip((unsigned long long)__double_as_longlong(m.x));
+  g.mu1 = strip((unsigned long long)__double_as_longlong(m.y));
+  g.v0 = strip((unsigned long long)__double_as_longlong(v.x));
+  g.v1 = strip((unsigned long long)__double_as_longlong(v.y));
+  return g;
+}
+
 // --------------------------------------------------------------------------
 // Level-synchronous item loop.  Each CTA walks its item list in
 // level order.  Thread 0 stages item t+1's CSR slice with TMA bulk copies
@@ -611,18 +623,6 @@ __global__ void __launch_bounds__(kThreads, 1) bwd_kernel(KParams P) {
   }
 }
 
-// State read outside a propagation pass (parity stripped, no waiting).
-__device__ __forceinline__ Gath load_state_plain(const PinState* p) {
-  const double2 m = __ldcg(reinterpret_cast<const double2*>(p));
-  const double2 v = __ldcg(reinterpret_cast<const double2*>(p) + 1);
-  Gath g;
-  g.mu0 = strip((unsigned long long)__double_as_longlong(m.x));
-  g.mu1 = strip((unsigned long long)__double_as_longlong(m.y));
-  g.v0 = strip((unsigned long long)__double_as_longlong(v.x));
-  g.v1 = strip((unsigned long long)__double_as_longlong(v.y));
-  return g;
-}
-
 // Endpoint seeds: dL/dA_ep[rf*] = -dL/dslack (slack = RAT - A); TNS: dL/dslack
 // = 1 where slack < 0.
 __global__ void seed_kernel(int num_ep, const int32_t* __restrict__ ep_pin,
@@ -738,12 +738,134 @@ __global__ void arrivals_kernel(int n, const PinState* __restrict__ state,
 __global__ void update_arcs_kernel(int64_t n, const int32_t* __restrict__ ids,
                                    const float2* __restrict__ mean,
                                    const float2* __restrict__ sigma,
-                                   const int32_t* __restrict__ arc_pos, float4* fin_ms) {
+                                   const int32_t* __restrict__ arc_pos, float4* fin_ms,
+                                   const int32_t* __restrict__ arc_sink, const int32_t* __restrict__ pin_level,
+                                   uint32_t* dirty, uint32_t stamp, int32_t* lvl_range) {
   const int64_t k = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
   if (k >= n) return;
   const int q = arc_pos[ids[k]];
   const float2 m = mean[k], s = sigma[k];
   fin_ms[q] = make_float4(m.x, m.y, s.x, s.y);
+  if (dirty) {   // incremental: the sink must be recomputed in the next pass
+    const int i = arc_sink[ids[k]];
+    dirty[i] = stamp;
+    atomicMin(lvl_range, pin_level[i]);
+    atomicMax(lvl_range + 1, pin_level[i]);
+  }
+}
+
+// --------------------------------------------------------------------------
+// Incremental forward ("re-annotate ... then
+// re-propagate").  Level-synchronous persistent kernel over the same items:
+// level l starts when every CTA has published level l-1 (fence.acq_rel + red /
+// ld.acquire counters), so all dirty marks that target level l are visible.
+// A pin is recomputed only if marked dirty; it is recomputed with the same
+// device function as the full forward, so its result equals the full pass bit
+// for bit.  If the new (mu, var) differ from the old ones, every fanout sink
+// is marked (full fanout CSR) and the deepest marked level is raised; the pass
+// stops as soon as the next level is deeper than any mark (cone exhausted).
+// Records keep the parity of the last full pass.
+// --------------------------------------------------------------------------
+struct IncParams {
+  KParams P;
+  const int32_t* __restrict__ fanout_ptr;
+  const int32_t* __restrict__ fout_sink;
+  const int32_t* __restrict__ pin_level;
+  uint32_t* dirty;
+  uint32_t stamp;
+  int32_t* lvl_range;        // {min dirty level, max dirty level}
+  uint32_t* done;            // [L] zeroed per pass; target = grid
+  unsigned long long* counters;  // [0] pins recomputed, [1] pins changed
+};
+
+__device__ __forceinline__ void inc_wait(const IncParams& Q, int l) {
+  if (threadIdx.x == 0) {
+    while (ld_acquire(Q.done + l) != uint32_t(Q.P.grid)) __nanosleep(32);
+  }
+  __syncthreads();
+}
+
+template <bool kLSE>
+__global__ void __launch_bounds__(kThreads, 1) inc_kernel(IncParams Q) {
+  const KParams& P = Q.P;
+  const int c = blockIdx.x, tid = threadIdx.x;
+  __shared__ int s_exit;
+  __shared__ unsigned long long s_cnt[2];
+  const int lmin = __ldcg(Q.lvl_range);
+  if (tid == 0) s_cnt[0] = s_cnt[1] = 0ull;
+  for (int k = P.step_begin; k < P.step_end; ++k) {
+    const int4 A = __ldg(P.item_a + size_t(k) * P.grid + c);
+    const int4 B = __ldg(P.item_b + size_t(k) * P.grid + c);
+    const int l = B.x;
+    if (l < lmin) continue;   // below the shallowest mark: nothing to do, nothing to publish
+    if (l > lmin) inc_wait(Q, l - 1);
+    if (tid == 0) s_exit = l > ld_acquire(reinterpret_cast<const uint32_t*>(Q.lvl_range + 1)) ? 1 : 0;
+    __syncthreads();
+    if (s_exit) break;
+    for (int i = A.x + tid; i < A.y; i += kThreads) {
+      if (__ldcg(Q.dirty + i) != Q.stamp) continue;
+      const int b0 = __ldg(P.fanin_ptr + i), nf = __ldg(P.fanin_ptr + i + 1) - b0;
+      const Gath old = load_state_plain(P.state + i);
+      double mu0, mu1, v0, v1;
+      if (l == 0) {
+        const float4 v = __ldg(P.src_ms + i);
+        mu0 = double(v.x);
+        mu1 = double(v.y);
+        v0 = double(v.z) * double(v.z);
+        v1 = double(v.w) * double(v.w);
+      } else {
+        auto arc = [&](int kk, int32_t& w, float4& ms, Raw& rr) {
+          w = __ldg(P.fin_src + b0 + kk);
+          ms = __ldg(P.fin_ms + b0 + kk);
+          rr = ld_state_raw(P, w & kSrcMask);
+        };
+        const RfOut R = pin_rf<kLSE>(P, 0, nf, arc);
+        const RfOut F = pin_rf<kLSE>(P, 1, nf, arc);
+        if (!kLSE) {
+          P.win[i] = R.win | (F.win << 16);
+        } else {
+          for (int kk = 0; kk < nf; ++kk) {
+            const float2 wr = arc_rf_weights(P, 0, kk, R, arc);
+            const float2 wf = arc_rf_weights(P, 1, kk, F, arc);
+            P.wts[b0 + kk] = make_float4(wr.x, wr.y, wf.x, wf.y);
+          }
+        }
+        mu0 = R.mu;
+        mu1 = F.mu;
+        v0 = R.var;
+        v1 = F.var;
+      }
+      atomicAdd(&s_cnt[0], 1ull);
+      // compare with the stored (parity-stripped) value after the same truncation
+      const double n0 = strip((unsigned long long)__double_as_longlong(mu0));
+      const double n1 = strip((unsigned long long)__double_as_longlong(mu1));
+      const double w0 = strip((unsigned long long)__double_as_longlong(v0));
+      const double w1 = strip((unsigned long long)__double_as_longlong(v1));
+      if (__double_as_longlong(n0) != __double_as_longlong(old.mu0) ||
+          __double_as_longlong(n1) != __double_as_longlong(old.mu1) ||
+          __double_as_longlong(w0) != __double_as_longlong(old.v0) ||
+          __double_as_longlong(w1) != __double_as_longlong(old.v1)) {
+        store_state(P, i, mu0, mu1, v0, v1);
+        atomicAdd(&s_cnt[1], 1ull);
+        int deepest = -1;
+        for (int r = __ldg(Q.fanout_ptr + i); r < __ldg(Q.fanout_ptr + i + 1); ++r) {
+          const int sink = __ldg(Q.fout_sink + r);
+          Q.dirty[sink] = Q.stamp;
+          deepest = max(deepest, __ldg(Q.pin_level + sink));
+        }
+        if (deepest >= 0) atomicMax(Q.lvl_range + 1, deepest);
+      }
+    }
+    __syncthreads();
+    if ((B.y & kItemLast) && tid == 0) {
+      asm volatile("fence.acq_rel.gpu;\n\tred.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(Q.done + l) : "memory");
+    }
+  }
+  __syncthreads();
+  if (tid == 0) {
+    atomicAdd(Q.counters, s_cnt[0]);
+    atomicAdd(Q.counters + 1, s_cnt[1]);
+  }
 }
 
 // --------------------------------------------------------------------------
@@ -878,6 +1000,12 @@ int launch_forward(DevGraph& g, float n_sigma, float tau, int schedule, void* st
   P.tau = tau;
   P.inv_tau = tau > 0.f ? 1.0 / double(tau) : 0.0;
   const bool lse = tau > 0.f;
+  {   // a full pass supersedes pending incremental marks
+    ++g.inc_epoch;
+    const int32_t init[2] = {0x7fffffff, -1};
+    cudaError_t e = cudaMemcpyAsync(g.lvl_range, init, sizeof init, cudaMemcpyHostToDevice, st);
+    if (e != cudaSuccess) return int(e);
+  }
   if (g.n > 0) {
     P.mode = schedule == 0 ? 2 : 0;   // dataflow persistent / one launch per level
     P.par = (++g.pass_fwd) & 1u;
@@ -924,18 +1052,53 @@ int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float*
 
 int launch_update_arcs(DevGraph& g, int64_t n, const int32_t* ids, const float* mean,
                        const float* sigma, int incremental, void* stream) {
-  (void)incremental;
   if (n <= 0) return 0;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   const int blocks = int((n + 255) / 256);
   update_arcs_kernel<<<blocks, 256, 0, st>>>(n, ids, reinterpret_cast<const float2*>(mean),
                                              reinterpret_cast<const float2*>(sigma), g.arc_pos,
-                                             g.fin_ms);
+                                             g.fin_ms, g.arc_sink, g.pin_level,
+                                             incremental ? g.dirty : nullptr, g.inc_epoch + 1, g.lvl_range);
   return int(cudaGetLastError());
 }
 
+// Incremental pass over the dirty cone, then slack/TNS.  Requires the previous
+// forward to have used the same (n_sigma, tau).
 int launch_forward_incremental(DevGraph& g, float n_sigma, float tau, void* stream) {
-  return launch_forward(g, n_sigma, tau, 0, stream);
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  IncParams Q{};
+  Q.P = make_params(g, false);
+  Q.P.n_sigma = n_sigma;
+  Q.P.tau = tau;
+  Q.P.inv_tau = tau > 0.f ? 1.0 / double(tau) : 0.0;
+  Q.P.mode = 1;
+  Q.P.par = g.pass_fwd & 1u;   // keep the parity of the last full pass
+  Q.P.step_begin = 0;
+  Q.P.step_end = g.fwd_items.num_steps;
+  Q.fanout_ptr = g.fanout_ptr;
+  Q.fout_sink = g.fout_sink;
+  Q.pin_level = g.pin_level;
+  Q.dirty = g.dirty;
+  Q.stamp = ++g.inc_epoch;
+  Q.lvl_range = g.lvl_range;
+  Q.done = g.done_fwd;
+  Q.counters = g.counters;
+  cudaError_t e = cudaMemsetAsync(g.done_fwd, 0, sizeof(uint32_t) * size_t(std::max(g.num_levels, 1)), st);
+  if (e == cudaSuccess) e = cudaMemsetAsync(g.counters, 0, sizeof(unsigned long long) * 2, st);
+  if (e != cudaSuccess) return int(e);
+  if (g.n > 0) {
+    void* args[] = {&Q};
+    e = cudaLaunchCooperativeKernel(tau > 0.f ? (const void*)inc_kernel<true> : (const void*)inc_kernel<false>,
+                                    dim3(g.grid), dim3(kThreads), args, 0, st);
+    if (e != cudaSuccess) return int(e);
+  }
+  // reset the level range for the next round of marks: {INT_MAX, -1}
+  const int32_t init[2] = {0x7fffffff, -1};
+  e = cudaMemcpyAsync(g.lvl_range, init, sizeof init, cudaMemcpyHostToDevice, st);
+  if (e != cudaSuccess) return int(e);
+  g.last_n_sigma = n_sigma;
+  g.last_tau = tau;
+  return launch_slack(g, stream);
 }
 
 int launch_arrivals(DevGraph& g, float* A, float* mean, float* sigma, void* stream) {
