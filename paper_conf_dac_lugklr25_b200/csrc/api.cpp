@@ -54,7 +54,7 @@ void free_graph(insta::DevGraph& d) {
                   d.rf_star,   d.partials,  d.ticket,    d.summary,    d.dirty,     d.counters,
                   d.fin_flags, d.ep_of_pin, d.b_state,   d.b_win,      d.b_wts,     d.b_g,
                   d.b_heavy,   d.b_sc,      d.b_ov_ptr,  d.b_ov_pos,   d.b_ov_ms,   d.b_slack,
-                  d.b_rf,      d.b_partials, d.b_ticket,  d.pin_level,  d.lvl_range};
+                  d.b_rf,      d.b_partials, d.b_ticket,  d.pin_level,  d.lvl_range, d.max_sink_level};
   for (void* p : ptrs)
     if (p) cudaFree(p);
 }
@@ -223,6 +223,10 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   std::vector<int32_t> pin_level(nN);
   for (int32_t k = 0; k < n; ++k) pin_level[k] = h.level[h.order[k]];
   const int32_t lvl_init[2] = {0x7fffffff, -1};
+  std::vector<int32_t> max_sink_level(nN, -1);
+  for (int32_t k = 0; k < n; ++k)
+    for (int32_t r = h.fanout_ptr[k]; r < h.fanout_ptr[k + 1]; ++r)
+      max_sink_level[k] = std::max(max_sink_level[k], pin_level[fout_sink[r]]);
   std::vector<int32_t> ep_of_pin(nN, -1);
   for (int32_t k = 0; k < d.num_ep; ++k) ep_of_pin[ep_pin[k]] = k;
   d.h_arc_pos = arc_pos;
@@ -259,6 +263,7 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   UP(d.ep_of_pin, ep_of_pin.data(), nN);
   UP(d.pin_level, pin_level.data(), nN);
   UP(d.lvl_range, lvl_init, 2);
+  UP(d.max_sink_level, max_sink_level.data(), nN);
   UP(d.fwd_a, d.fwd_items.a.data(), d.fwd_items.a.size());
   UP(d.fwd_b, d.fwd_items.b.data(), d.fwd_items.b.size());
   UP(d.bwd_a, d.bwd_items.a.data(), d.bwd_items.a.size());

@@ -132,68 +132,17 @@ __device__ __forceinline__ void bfwd_prefetch(const BParams& P, BFwdStage* st, u
   }
 }
 
-// Merge of (pin, rf) for scenario lane s over nf arcs; arc(k, w, ms_s, raw).
-struct RfOutB {
-  double mu, var, best;
-  float sum;
-  int win;
-};
-
+// Merge of (pin, rf) for scenario lane s: the same device function as the
+// single-scenario kernels (device_common.cuh merge_rf), hence bit-identical.
 template <bool kLSE, class ArcFn>
-__device__ __forceinline__ RfOutB pin_rf_b(const BParams& P, double ns, int rf, int nf, ArcFn&& arc) {
-  Merge m;
-  merge_init(m);
-  for (int k = 0; k < nf; ++k) {
-    int32_t w;
-    float4 ms;
-    Raw r;
-    arc(k, w, ms, r);
-    const Gath st = unpack(r);
-    const int u = int(uint32_t(w) >> kUnateShift);
-    const int s0 = src_tr(rf, u, 0);
-    merge_max(m, make_cand(st, ms, rf, s0, ns), k, s0);
-    if (u == 2) merge_max(m, make_cand(st, ms, rf, rf ^ 1, ns), k, rf ^ 1);
-  }
-  RfOutB o;
-  o.best = m.best;
-  o.var = m.var;
-  o.win = m.k | (m.s << 15);
-  o.sum = 0.f;
-  o.mu = m.mu;
-  if (kLSE) {
-    float sum = 0.f;
-    for (int k = 0; k < nf; ++k) {
-      int32_t w;
-      float4 ms;
-      Raw r;
-      arc(k, w, ms, r);
-      const Gath st = unpack(r);
-      const int u = int(uint32_t(w) >> kUnateShift);
-      sum += lse_term(make_cand(st, ms, rf, src_tr(rf, u, 0), ns), m, P.inv_tau);
-      if (u == 2) sum += lse_term(make_cand(st, ms, rf, rf ^ 1, ns), m, P.inv_tau);
-    }
-    o.sum = sum;
-    o.mu = (m.best + double(P.tau) * double(logf(sum))) - ns * double(m.sig);
-  }
-  return o;
+__device__ __forceinline__ RfOut pin_rf_b(const BParams& P, double ns, int rf, int nf, ArcFn&& arc) {
+  return merge_rf<kLSE>(ns, double(P.tau), P.inv_tau, rf, nf, arc);
 }
 
 template <class ArcFn>
-__device__ __forceinline__ float2 arc_rf_weights_b(const BParams& P, double ns, int rf, int k, const RfOutB& o,
+__device__ __forceinline__ float2 arc_rf_weights_b(const BParams& P, double ns, int rf, int k, const RfOut& o,
                                                    ArcFn&& arc) {
-  int32_t w;
-  float4 ms;
-  Raw r;
-  arc(k, w, ms, r);
-  const Gath st = unpack(r);
-  const int u = int(uint32_t(w) >> kUnateShift);
-  float wt[2] = {0.f, 0.f};
-  const int s0 = src_tr(rf, u, 0);
-  Merge m;
-  m.best = o.best;
-  wt[s0] = lse_term(make_cand(st, ms, rf, s0, ns), m, P.inv_tau) / o.sum;
-  if (u == 2) wt[rf ^ 1] = lse_term(make_cand(st, ms, rf, rf ^ 1, ns), m, P.inv_tau) / o.sum;
-  return make_float2(wt[0], wt[1]);
+  return arc_weights(ns, P.inv_tau, rf, k, o, arc);
 }
 
 constexpr int kRegArcsB = 4;
@@ -284,8 +233,8 @@ __global__ void __launch_bounds__(kThreads, 1) fwdb_kernel(BParams P) {
               awaitb(P, w & kSrcMask, s, r);
             }
           };
-          const RfOutB R = pin_rf_b<kLSE>(P, ns, 0, nf, arc);
-          const RfOutB F = pin_rf_b<kLSE>(P, ns, 1, nf, arc);
+          const RfOut R = pin_rf_b<kLSE>(P, ns, 0, nf, arc);
+          const RfOut F = pin_rf_b<kLSE>(P, ns, 1, nf, arc);
           storeb(P, i, s, R.mu, F.mu, R.var, F.var);
           if (!kLSE) {
             P.bwin[size_t(i) * kLanes + s] = R.win | (F.win << 16);

@@ -9,6 +9,8 @@
 
 namespace insta {
 
+constexpr int kUnateShiftC = 30;   // fin_src bits 30..31: unateness (internal.h kUnateShift)
+
 // --------------------------------------------------------------------------
 // PTX helpers: memory model, mbarrier, TMA bulk copy
 // --------------------------------------------------------------------------
@@ -91,7 +93,13 @@ __device__ __forceinline__ Window window(int64_t a, int64_t b, int esz) {
   return w;
 }
 
-__device__ __forceinline__ float sigma_of(double var) { return sqrtf(float(var)); }
+// sigma = sqrt(var) for the corner arrival: the hardware square root
+// (sqrt.approx.f32, ~1 ulp; deterministic) of the fp32-rounded variance.
+__device__ __forceinline__ float sigma_of(double var) {
+  float r;
+  asm("sqrt.approx.f32 %0, %1;" : "=f"(r) : "f"(float(var)));
+  return r;
+}
 
 // source transitions of an arc for sink transition rf: POS {rf}; NEG {~rf}
 // (Alg 1 l.8); NON (rf, ~rf) (reading R3).
@@ -177,6 +185,109 @@ __device__ __forceinline__ void merge_max(Merge& m, const Cand& c, int k, int s)
 // Eq 6 weight of a candidate given its merge (LSE)
 __device__ __forceinline__ float lse_term(const Cand& c, const Merge& m, double tau) {
   return expf(float((c.A - m.best) * tau));   // tau: the inverse temperature 1/tau
+}
+
+// Merge of one (pin, rf) over its candidates in canonical order (fanin row,
+// then s = rf before ~rf): Alg 1 / Alg 2 with K = 1 (first arg-max, strict
+// ">") or Eq 4 (LSE with M = the arg-max).  Only corner arrivals are compared;
+// the winner's distribution is re-evaluated once (bit-identical to its scan
+// value).  arc(k, w, ms, raw) yields arc k's source word, (scenario) arc record
+// and gathered source words.  Shared by the single-scenario, incremental and
+// batched kernels.
+struct RfOut {
+  double mu, var, best;
+  float sum, sig;
+  int win;   // arg-max: k | s << 15
+};
+
+// exp((A - M) / tau) for the LSE normalizer and Eq 6 weights: fp32 exponent
+// (hardware ex2, deterministic), argument formed in fp64.
+__device__ __forceinline__ float lse_w(double A, double best, double inv_tau) {
+  return __expf(float((A - best) * inv_tau));
+}
+
+// LSE arrival (Eq 4): M + tau * log(sum)
+__device__ __forceinline__ double lse_arrival(double best, double tau, float sum) {
+  return best + tau * double(__logf(sum));
+}
+
+template <bool kLSE, class ArcFn>
+__device__ __forceinline__ RfOut merge_rf(double ns, double tau, double inv_tau, int rf, int nf, ArcFn&& arc) {
+  double best = 0.0;
+  int bk = -1, bs = 0;
+  for (int k = 0; k < nf; ++k) {
+    int32_t w;
+    float4 ms;
+    Raw r;
+    arc(k, w, ms, r);
+    const Gath st = unpack(r);
+    const int u = int(uint32_t(w) >> kUnateShiftC);
+    const int s0 = src_tr(rf, u, 0);
+    const double a0 = make_cand(st, ms, rf, s0, ns).A;
+    if (bk < 0 || a0 > best) {   // Alg 2 l.4: replace only if strictly greater
+      best = a0;
+      bk = k;
+      bs = s0;
+    }
+    if (u == 2) {
+      const double a1 = make_cand(st, ms, rf, rf ^ 1, ns).A;
+      if (a1 > best) {
+        best = a1;
+        bk = k;
+        bs = rf ^ 1;
+      }
+    }
+  }
+  RfOut o;
+  {
+    int32_t w;
+    float4 ms;
+    Raw r;
+    arc(bk, w, ms, r);
+    const Cand c = make_cand(unpack(r), ms, rf, bs, ns);   // the winner (Alg 1 l.15)
+    o.mu = c.mu;
+    o.var = c.var;
+    o.sig = c.sig;
+  }
+  o.best = best;
+  o.win = bk | (bs << 15);
+  o.sum = 0.f;
+  if (kLSE) {
+    // Eq 4: A_i = M + tau * log(sum_c exp((A_c - M) / tau)); reading R1:
+    // sigma_i = sigma of the arg-max, mu_i = A_i - n_sigma * sigma_i.
+    float sum = 0.f;
+    for (int k = 0; k < nf; ++k) {
+      int32_t w;
+      float4 ms;
+      Raw r;
+      arc(k, w, ms, r);
+      const Gath st = unpack(r);
+      const int u = int(uint32_t(w) >> kUnateShiftC);
+      sum += lse_w(make_cand(st, ms, rf, src_tr(rf, u, 0), ns).A, best, inv_tau);
+      if (u == 2) sum += lse_w(make_cand(st, ms, rf, rf ^ 1, ns).A, best, inv_tau);
+    }
+    o.sum = sum;
+    o.mu = lse_arrival(best, tau, sum) - ns * double(o.sig);
+  }
+  return o;
+}
+
+// Eq 6 weights {w[rf][s=R], w[rf][s=F]} of arc k's candidates for transition rf
+template <class ArcFn>
+__device__ __forceinline__ float2 arc_weights(double ns, double inv_tau, int rf, int k, const RfOut& o,
+                                              ArcFn&& arc) {
+  int32_t w;
+  float4 ms;
+  Raw r;
+  arc(k, w, ms, r);
+  const Gath st = unpack(r);
+  const int u = int(uint32_t(w) >> kUnateShiftC);
+  float wt[2] = {0.f, 0.f};
+  const int s0 = src_tr(rf, u, 0);
+  const float inv_sum = 1.f / o.sum;
+  wt[s0] = lse_w(make_cand(st, ms, rf, s0, ns).A, o.best, inv_tau) * inv_sum;
+  if (u == 2) wt[rf ^ 1] = lse_w(make_cand(st, ms, rf, rf ^ 1, ns).A, o.best, inv_tau) * inv_sum;
+  return make_float2(wt[0], wt[1]);
 }
 
 }  // namespace insta

@@ -42,7 +42,7 @@ constexpr int kHeavyFanout = 256;
 // (per item; two stages are double-buffered)
 constexpr int kThreads = 1024;
 constexpr int kFwdPins = 2048, kFwdArcs = 2048;                     // forward item caps
-constexpr int kBwdPins = 1024, kBwdFanout = 2048, kBwdArcs = 2048;  // backward item caps
+constexpr int kBwdPins = 2048, kBwdFanout = 2048, kBwdArcs = 2048;  // backward item caps
 static_assert(kHeavyFanout <= kBwdFanout, "a light pin's fanout row must fit one item");
 
 struct alignas(32) PinState {
@@ -151,6 +151,7 @@ struct DevGraph {
   // incremental
   uint32_t* dirty = nullptr;       // [n] stamp == inc_epoch: pin must be recomputed
   int32_t* pin_level = nullptr;    // [n] level of each canonical pin
+  int32_t* max_sink_level = nullptr;  // [n] deepest level among the pin's fanout sinks, -1 if none
   int32_t* lvl_range = nullptr;    // [2] {min, max} level of pending dirty marks
   unsigned long long* counters = nullptr;  // [4] recomputed pins etc.
   // host-side bookkeeping

@@ -119,74 +119,14 @@ __device__ __forceinline__ void store_state(const KParams& P, int i, double m0, 
                : "memory");
 }
 
-// Merge of one (pin, rf) (Alg 1 / Alg 2 with K = 1, or Eq 4) over its
-// candidates in canonical order: fanin row, then s = rf before ~rf.
-// arc(k, w, ms, raw) yields arc k's record and gathered source words.
-struct RfOut {
-  double mu, var, best;
-  float sum;
-  int win;   // arg-max: k | s << 15
-};
-
 template <bool kLSE, class ArcFn>
 __device__ __forceinline__ RfOut pin_rf(const KParams& P, int rf, int nf, ArcFn&& arc) {
-  const double ns = double(P.n_sigma);
-  Merge m;
-  merge_init(m);
-  for (int k = 0; k < nf; ++k) {
-    int32_t w;
-    float4 ms;
-    Raw r;
-    arc(k, w, ms, r);
-    const Gath st = unpack(r);
-    const int u = int(uint32_t(w) >> kUnateShift);
-    const int s0 = src_tr(rf, u, 0);
-    merge_max(m, make_cand(st, ms, rf, s0, ns), k, s0);
-    if (u == 2) merge_max(m, make_cand(st, ms, rf, rf ^ 1, ns), k, rf ^ 1);
-  }
-  RfOut o;
-  o.best = m.best;
-  o.var = m.var;
-  o.win = m.k | (m.s << 15);
-  o.sum = 0.f;
-  o.mu = m.mu;   // hard: Alg 1 l.15 / Alg 2 l.6 (the winner's distribution)
-  if (kLSE) {
-    // Eq 4: A_i = M + tau * log(sum_c exp((A_c - M) / tau)); reading R1:
-    // sigma_i = sigma of the arg-max, mu_i = A_i - n_sigma * sigma_i.
-    float sum = 0.f;
-    for (int k = 0; k < nf; ++k) {
-      int32_t w;
-      float4 ms;
-      Raw r;
-      arc(k, w, ms, r);
-      const Gath st = unpack(r);
-      const int u = int(uint32_t(w) >> kUnateShift);
-      sum += lse_term(make_cand(st, ms, rf, src_tr(rf, u, 0), ns), m, P.inv_tau);
-      if (u == 2) sum += lse_term(make_cand(st, ms, rf, rf ^ 1, ns), m, P.inv_tau);
-    }
-    o.sum = sum;
-    o.mu = (m.best + double(P.tau) * double(logf(sum))) - ns * double(m.sig);
-  }
-  return o;
+  return merge_rf<kLSE>(double(P.n_sigma), double(P.tau), P.inv_tau, rf, nf, arc);
 }
 
-// Eq 6 weights {w[rf][s=R], w[rf][s=F]} of arc k's candidates for transition rf
 template <class ArcFn>
 __device__ __forceinline__ float2 arc_rf_weights(const KParams& P, int rf, int k, const RfOut& o, ArcFn&& arc) {
-  const double ns = double(P.n_sigma);
-  int32_t w;
-  float4 ms;
-  Raw r;
-  arc(k, w, ms, r);
-  const Gath st = unpack(r);
-  const int u = int(uint32_t(w) >> kUnateShift);
-  float wt[2] = {0.f, 0.f};
-  const int s0 = src_tr(rf, u, 0);
-  Merge m;
-  m.best = o.best;
-  wt[s0] = lse_term(make_cand(st, ms, rf, s0, ns), m, P.inv_tau) / o.sum;
-  if (u == 2) wt[rf ^ 1] = lse_term(make_cand(st, ms, rf, rf ^ 1, ns), m, P.inv_tau) / o.sum;
-  return make_float2(wt[0], wt[1]);
+  return arc_weights(double(P.n_sigma), P.inv_tau, rf, k, o, arc);
 }
 
 // State read outside a propagation pass (parity stripped, no waiting).
@@ -221,7 +161,9 @@ struct FwdStage {
   int32_t src[kFwdArcs + 8];
   float4 ms[kFwdArcs];
 };
-constexpr size_t kFwdSmem = 2 * sizeof(FwdStage) + sizeof(Raw) * kFwdArcs;
+// per arc: gathered source record + corner arrivals of its candidates
+// {A[rf=R][s0], A[rf=F][s0], A[R][s1], A[F][s1]} (s1 only for non-unate arcs)
+constexpr size_t kFwdSmem = 2 * sizeof(FwdStage) + (sizeof(Raw) + sizeof(double4)) * kFwdArcs;
 
 __device__ __forceinline__ bool fwd_staged(const int4& A, const int4& B) {
   return A.y > A.x && B.x > 0 && !(B.y & kItemDirect);
@@ -283,6 +225,79 @@ __device__ __forceinline__ void fwd_pin_pair(const KParams& P, int i, int rf, in
   }
 }
 
+// Merge of one (pin, rf) from precomputed candidate corners (same candidate
+// order, comparisons and LSE sum as merge_rf, hence bit-identical to it).
+template <bool kLSE>
+__device__ __forceinline__ RfOut merge_rf_pre(const KParams& P, int rf, int nf, const int32_t* sw,
+                                              const float4* sm, const Raw* sg, const double4* ca) {
+  const double ns = double(P.n_sigma);
+  double best = 0.0;
+  int bk = -1, bs = 0;
+  for (int k = 0; k < nf; ++k) {
+    const int u = int(uint32_t(sw[k]) >> kUnateShift);
+    const double4 c = ca[k];
+    const double a0 = rf ? c.y : c.x;
+    if (bk < 0 || a0 > best) {   // Alg 2 l.4: replace only if strictly greater
+      best = a0;
+      bk = k;
+      bs = src_tr(rf, u, 0);
+    }
+    if (u == 2) {
+      const double a1 = rf ? c.w : c.z;
+      if (a1 > best) {
+        best = a1;
+        bk = k;
+        bs = rf ^ 1;
+      }
+    }
+  }
+  RfOut o;
+  const Cand cw = make_cand(unpack(sg[bk]), sm[bk], rf, bs, ns);   // the winner (Alg 1 l.15)
+  o.mu = cw.mu;
+  o.var = cw.var;
+  o.sig = cw.sig;
+  o.best = best;
+  o.win = bk | (bs << 15);
+  o.sum = 0.f;
+  if (kLSE) {
+    float sum = 0.f;
+    for (int k = 0; k < nf; ++k) {
+      const int u = int(uint32_t(sw[k]) >> kUnateShift);
+      const double4 c = ca[k];
+      sum += lse_w(rf ? c.y : c.x, best, P.inv_tau);
+      if (u == 2) sum += lse_w(rf ? c.w : c.z, best, P.inv_tau);
+    }
+    o.sum = sum;
+    o.mu = lse_arrival(best, double(P.tau), sum) - ns * double(o.sig);
+  }
+  return o;
+}
+
+template <bool kLSE>
+__device__ __forceinline__ void fwd_pin_pre(const KParams& P, int i, int nf, int q0, const int32_t* sw,
+                                            const float4* sm, const Raw* sg, const double4* ca) {
+  const RfOut R = merge_rf_pre<kLSE>(P, 0, nf, sw, sm, sg, ca);
+  const RfOut F = merge_rf_pre<kLSE>(P, 1, nf, sw, sm, sg, ca);
+  store_state(P, i, R.mu, F.mu, R.var, F.var);
+  if (!kLSE) {
+    P.win[i] = R.win | (F.win << 16);
+  } else {
+    for (int k = 0; k < nf; ++k) {
+      const int u = int(uint32_t(sw[k]) >> kUnateShift);
+      const double4 c = ca[k];
+      float wt[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
+      const float invR = 1.f / R.sum, invF = 1.f / F.sum;   // as arc_weights
+      wt[0][src_tr(0, u, 0)] = lse_w(c.x, R.best, P.inv_tau) * invR;
+      wt[1][src_tr(1, u, 0)] = lse_w(c.y, F.best, P.inv_tau) * invF;
+      if (u == 2) {
+        wt[0][1] = lse_w(c.z, R.best, P.inv_tau) * invR;
+        wt[1][0] = lse_w(c.w, F.best, P.inv_tau) * invF;
+      }
+      P.wts[q0 + k] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
+    }
+  }
+}
+
 __device__ __forceinline__ void trace_stamp(const KParams& P, int c, int nsteps, int t, int slot) {
   if (P.trace && threadIdx.x == 0) P.trace[(size_t(c) * nsteps + t) * 4 + slot] = gtimer();
 }
@@ -292,6 +307,7 @@ __global__ void __launch_bounds__(kThreads, 1) fwd_kernel(KParams P) {
   extern __shared__ __align__(128) unsigned char smem[];
   FwdStage* stage = reinterpret_cast<FwdStage*>(smem);
   Raw* gath = reinterpret_cast<Raw*>(smem + 2 * sizeof(FwdStage));
+  double4* candA = reinterpret_cast<double4*>(smem + 2 * sizeof(FwdStage) + sizeof(Raw) * kFwdArcs);
   __shared__ __align__(8) uint64_t full[2];
   const int c = blockIdx.x;
   const int tid = threadIdx.x;
@@ -336,26 +352,32 @@ __global__ void __launch_bounds__(kThreads, 1) fwd_kernel(KParams P) {
                        : "memory");
         }
         asm volatile("cp.async.wait_all;" ::: "memory");
+        const double ns = double(P.n_sigma);
         for (int a = tid; a < na; a += kThreads) {
           Raw r = gath[a];
+          const int32_t w = S.src[so + a];
           if (P.mode == 2 && !raw_ready(r, P.par)) {
-            const int j = S.src[so + a] & kSrcMask;
-            await_raw(P, j, r);
+            await_raw(P, w & kSrcMask, r);
             gath[a] = r;
           }
+          // arc-parallel candidate corners (Eq 1-3), both sink transitions
+          const Gath st = unpack(r);
+          const float4 ms = S.ms[a];
+          const int u = int(uint32_t(w) >> kUnateShift);
+          double4 ca;
+          ca.x = make_cand(st, ms, 0, src_tr(0, u, 0), ns).A;
+          ca.y = make_cand(st, ms, 1, src_tr(1, u, 0), ns).A;
+          ca.z = u == 2 ? make_cand(st, ms, 0, 1, ns).A : 0.0;
+          ca.w = u == 2 ? make_cand(st, ms, 1, 0, ns).A : 0.0;
+          candA[a] = ca;
         }
         __syncthreads();
         trace_stamp(P, c, nsteps, t, 1);
-        // (2) compute: work unit = (pin, rf), a lane pair per pin
-        for (int un = tid; un < 2 * (A.y - A.x); un += kThreads) {
-          const int p = un >> 1;
+        // (2) compute: one thread per pin (both rf), merging the precomputed corners
+        for (int p = tid; p < A.y - A.x; p += kThreads) {
           const int b0 = S.ptr[po + p] - A.z;
           const int nf = S.ptr[po + p + 1] - A.z - b0;
-          fwd_pin_pair<kLSE>(P, A.x + p, un & 1, nf, A.z + b0, [&](int kk, int32_t& w, float4& ms, Raw& rr) {
-            w = S.src[so + b0 + kk];
-            ms = S.ms[b0 + kk];
-            rr = gath[b0 + kk];
-          });
+          fwd_pin_pre<kLSE>(P, A.x + p, nf, A.z + b0, &S.src[so + b0], &S.ms[b0], &gath[b0], &candA[b0]);
         }
       } else {
         for (int i = A.x + tid; i < A.y; i += kThreads) {
@@ -370,6 +392,7 @@ __global__ void __launch_bounds__(kThreads, 1) fwd_kernel(KParams P) {
         }
       }
     }
+    trace_stamp(P, c, nsteps, t, 3);   // thread 0's own work done (debug trace)
     __syncthreads();   // stage[buf] and gath are free for reuse
     trace_stamp(P, c, nsteps, t, 2);
   }
@@ -378,25 +401,25 @@ __global__ void __launch_bounds__(kThreads, 1) fwd_kernel(KParams P) {
 // --------------------------------------------------------------------------
 // Backward kernel
 // --------------------------------------------------------------------------
+template <bool kLSE>
 struct BwdStage {
   int32_t lptr[kBwdPins + 8];   // light fanout row pointers
   int32_t lfo[kBwdFanout + 8];  // fanin position of each light fanout entry
   int32_t fptr[kBwdPins + 8];   // fanin row pointers
   int32_t src[kBwdArcs + 8];    // fin_src
   int32_t arc[kBwdArcs + 8];    // caller arc ids
-  int32_t win[kBwdPins + 8];    // hard-mode winners
   int32_t hslot[kBwdPins + 8];  // heavy accumulator slot per pin (-1: light)
   float2 seed[kBwdPins + 8];
-  float4 wts[kBwdArcs];         // LSE weights
+  int32_t win[kLSE ? 8 : kBwdPins + 8];   // hard-mode winners
+  float4 wts[kLSE ? kBwdArcs : 1];        // LSE weights
 };
-constexpr size_t kBwdSmem = 2 * sizeof(BwdStage) + sizeof(float2) * kBwdFanout;
 
 __device__ __forceinline__ bool bwd_staged(const int4& A, const int4& B) {
   return A.y > A.x && !(B.w & kItemDirect);
 }
 
 template <bool kLSE>
-__device__ __forceinline__ void bwd_prefetch(const KParams& P, BwdStage* st, uint64_t* full, int step,
+__device__ __forceinline__ void bwd_prefetch(const KParams& P, BwdStage<kLSE>* st, uint64_t* full, int step,
                                              int c) {
   const int4 A = __ldg(P.item_a + size_t(step) * P.grid + c);   // {pin_lo, pin_hi, lfo_lo, lfo_hi}
   const int4 B = __ldg(P.item_b + size_t(step) * P.grid + c);   // {arc_lo, arc_hi, level, flags}
@@ -435,11 +458,61 @@ __device__ __forceinline__ void bwd_prefetch(const KParams& P, BwdStage* st, uin
 constexpr double kFixH = 16777216.0;                    // 2^24
 constexpr long long kCountUnit = 1ll << 44;
 
-__device__ __forceinline__ void heavy_add(const KParams& P, int32_t srcw, float gx, float gy) {
+// CTA-local combining of heavy-driver contributions: a small open-addressed
+// table in shared memory (slot -> two int64 words in the same count-folded
+// fixed-point format).  Contributions of one item are combined here and
+// flushed with one global atomic per (slot, word) at the end of the item, so a
+// 20k-sink driver receives O(#CTAs) instead of O(#sinks) contended atomics.
+// Integer addition is associative, so the result is unchanged (deterministic).
+constexpr int kHeavyTab = 512;
+struct HeavyTab {
+  int32_t key[kHeavyTab];
+  unsigned long long acc[kHeavyTab][2];
+};
+
+__device__ __forceinline__ void heavy_add(const KParams& P, HeavyTab* tab, int32_t srcw, float gx, float gy) {
   if (!((srcw >> kHeavyBit) & 1)) return;
   const int slot = __ldg(P.heavy_slot + (srcw & kSrcMask));
-  atomicAdd(P.heavy_acc + 2 * slot, (unsigned long long)(kCountUnit + __double2ll_rn(double(gx) * kFixH)));
-  atomicAdd(P.heavy_acc + 2 * slot + 1, (unsigned long long)(kCountUnit + __double2ll_rn(double(gy) * kFixH)));
+  const unsigned long long vx = (unsigned long long)(kCountUnit + __double2ll_rn(double(gx) * kFixH));
+  const unsigned long long vy = (unsigned long long)(kCountUnit + __double2ll_rn(double(gy) * kFixH));
+  if (tab) {
+    int h = int((uint32_t(slot) * 2654435761u) >> 23) & (kHeavyTab - 1);
+    for (int probe = 0; probe < 8; ++probe, h = (h + 1) & (kHeavyTab - 1)) {
+      const int prev = atomicCAS(&tab->key[h], -1, slot);
+      if (prev == -1 || prev == slot) {
+        atomicAdd(&tab->acc[h][0], vx);
+        atomicAdd(&tab->acc[h][1], vy);
+        return;
+      }
+    }
+  }
+  atomicAdd(P.heavy_acc + 2 * slot, vx);   // table full (or no table): direct
+  atomicAdd(P.heavy_acc + 2 * slot + 1, vy);
+}
+
+template <bool kLSE>
+constexpr size_t bwd_smem() { return 2 * sizeof(BwdStage<kLSE>) + sizeof(float2) * kBwdFanout + sizeof(HeavyTab); }
+
+__device__ __forceinline__ void heavy_tab_clear(HeavyTab* tab) {
+  for (int h = threadIdx.x; h < kHeavyTab; h += blockDim.x) {
+    tab->key[h] = -1;
+    tab->acc[h][0] = 0ull;
+    tab->acc[h][1] = 0ull;
+  }
+}
+
+// after a barrier: flush and clear
+__device__ __forceinline__ void heavy_tab_flush(const KParams& P, HeavyTab* tab) {
+  for (int h = threadIdx.x; h < kHeavyTab; h += blockDim.x) {
+    const int slot = tab->key[h];
+    if (slot >= 0) {
+      atomicAdd(P.heavy_acc + 2 * slot, tab->acc[h][0]);
+      atomicAdd(P.heavy_acc + 2 * slot + 1, tab->acc[h][1]);
+      tab->key[h] = -1;
+      tab->acc[h][0] = 0ull;
+      tab->acc[h][1] = 0ull;
+    }
+  }
 }
 
 __device__ __forceinline__ long long heavy_count(long long acc) { return (acc + (kCountUnit >> 1)) >> 44; }
@@ -463,8 +536,8 @@ __device__ __forceinline__ float2 heavy_take(const KParams& P, int slot) {
 // per arc, g = adjoint to the source's {R, F} and dL/d(arc mean) (Eq 6 chain;
 // hard mode: one-hot at the recorded arg-max).
 template <bool kLSE, class ArcFn>
-__device__ __forceinline__ void bwd_sink(const KParams& P, int nf, int q0, float2 ab, int32_t win,
-                                         ArcFn&& arc) {
+__device__ __forceinline__ void bwd_sink(const KParams& P, HeavyTab* tab, int nf, int q0, float2 ab,
+                                         int32_t win, ArcFn&& arc) {
   const float abr[2] = {ab.x, ab.y};
   for (int k = 0; k < nf; ++k) {
     int32_t srcw, arcid;
@@ -496,7 +569,7 @@ __device__ __forceinline__ void bwd_sink(const KParams& P, int nf, int q0, float
     st2_f32(P.g + q0 + k, with_parf(gs[0], P.par), with_parf(gs[1], P.par));
     if (gm[0] != 0.f || gm[1] != 0.f)
       reinterpret_cast<float2*>(P.d_mean)[arcid] = make_float2(gm[0], gm[1]);
-    heavy_add(P, srcw, gs[0], gs[1]);
+    heavy_add(P, tab, srcw, gs[0], gs[1]);
   }
 }
 
@@ -520,8 +593,9 @@ __device__ __forceinline__ float2 load_g(const KParams& P, int q) {
 template <bool kLSE>
 __global__ void __launch_bounds__(kThreads, 1) bwd_kernel(KParams P) {
   extern __shared__ __align__(128) unsigned char smem[];
-  BwdStage* stage = reinterpret_cast<BwdStage*>(smem);
-  float2* gg = reinterpret_cast<float2*>(smem + 2 * sizeof(BwdStage));
+  BwdStage<kLSE>* stage = reinterpret_cast<BwdStage<kLSE>*>(smem);
+  float2* gg = reinterpret_cast<float2*>(smem + 2 * sizeof(BwdStage<kLSE>));
+  HeavyTab* htab = reinterpret_cast<HeavyTab*>(smem + 2 * sizeof(BwdStage<kLSE>) + sizeof(float2) * kBwdFanout);
   __shared__ __align__(8) uint64_t full[2];
   const int c = blockIdx.x;
   const int tid = threadIdx.x;
@@ -530,6 +604,7 @@ __global__ void __launch_bounds__(kThreads, 1) bwd_kernel(KParams P) {
     mbar_init1(&full[1]);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
+  heavy_tab_clear(htab);
   __syncthreads();
   uint32_t phase[2] = {0u, 0u};
   const int nsteps = P.step_end - P.step_begin;
@@ -547,7 +622,7 @@ __global__ void __launch_bounds__(kThreads, 1) bwd_kernel(KParams P) {
       if (!(B.w & kItemDirect)) {
         mbar_wait(&full[buf], phase[buf]);
         phase[buf] ^= 1u;
-        const BwdStage& S = stage[buf];
+        const BwdStage<kLSE>& S = stage[buf];
         const int lo = A.x & 3, fo = A.z & 3, ao = B.x & 3, so = A.x & 1;
         const int nfo = A.w - A.z;
         // (1) gather the sinks' per-arc adjoints of every light fanout entry:
@@ -584,7 +659,7 @@ __global__ void __launch_bounds__(kThreads, 1) bwd_kernel(KParams P) {
             if (P.d_src) reinterpret_cast<float2*>(P.d_src)[__ldg(P.order + i)] = ab;
           } else {
             const int b0 = S.fptr[lo + p] - B.x, b1 = S.fptr[lo + p + 1] - B.x;
-            bwd_sink<kLSE>(P, b1 - b0, B.x + b0, ab, kLSE ? 0 : S.win[lo + p],
+            bwd_sink<kLSE>(P, htab, b1 - b0, B.x + b0, ab, kLSE ? 0 : S.win[lo + p],
                            [&](int kk, int32_t& srcw, int32_t& arcid, float4& w4) {
                              srcw = S.src[ao + b0 + kk];
                              arcid = S.arc[ao + b0 + kk];
@@ -608,7 +683,7 @@ __global__ void __launch_bounds__(kThreads, 1) bwd_kernel(KParams P) {
             if (P.d_src) reinterpret_cast<float2*>(P.d_src)[__ldg(P.order + i)] = ab;
           } else {
             const int b0 = __ldg(P.fanin_ptr + i), b1 = __ldg(P.fanin_ptr + i + 1);
-            bwd_sink<kLSE>(P, b1 - b0, b0, ab, kLSE ? 0 : P.win[i],
+            bwd_sink<kLSE>(P, htab, b1 - b0, b0, ab, kLSE ? 0 : P.win[i],
                            [&](int kk, int32_t& srcw, int32_t& arcid, float4& w4) {
                              srcw = __ldg(P.fin_src + b0 + kk);
                              arcid = __ldg(P.fin_arc + b0 + kk);
@@ -619,6 +694,7 @@ __global__ void __launch_bounds__(kThreads, 1) bwd_kernel(KParams P) {
       }
     }
     __syncthreads();
+    heavy_tab_flush(P, htab);
     trace_stamp(P, c, nsteps, t, 2);
   }
 }
@@ -771,6 +847,7 @@ struct IncParams {
   const int32_t* __restrict__ fanout_ptr;
   const int32_t* __restrict__ fout_sink;
   const int32_t* __restrict__ pin_level;
+  const int32_t* __restrict__ max_sink_level;   // deepest level among a pin's fanout sinks (-1: none)
   uint32_t* dirty;
   uint32_t stamp;
   int32_t* lvl_range;        // {min dirty level, max dirty level}
@@ -814,10 +891,36 @@ __global__ void __launch_bounds__(kThreads, 1) inc_kernel(IncParams Q) {
         v0 = double(v.z) * double(v.z);
         v1 = double(v.w) * double(v.w);
       } else {
+        // topology and source states of the first 4 arcs are loaded together
+        constexpr int kR = 4;
+        int32_t wv[kR];
+        float4 mv[kR];
+        Raw rv[kR];
+#pragma unroll
+        for (int kk = 0; kk < kR; ++kk) {
+          if (kk < nf) {
+            wv[kk] = __ldg(P.fin_src + b0 + kk);
+            mv[kk] = __ldg(P.fin_ms + b0 + kk);
+          }
+        }
+#pragma unroll
+        for (int kk = 0; kk < kR; ++kk)
+          if (kk < nf) rv[kk] = ld_state_raw(P, wv[kk] & kSrcMask);
         auto arc = [&](int kk, int32_t& w, float4& ms, Raw& rr) {
-          w = __ldg(P.fin_src + b0 + kk);
-          ms = __ldg(P.fin_ms + b0 + kk);
-          rr = ld_state_raw(P, w & kSrcMask);
+          if (kk < kR) {
+#pragma unroll
+            for (int x = 0; x < kR; ++x) {
+              if (x == kk) {
+                w = wv[x];
+                ms = mv[x];
+                rr = rv[x];
+              }
+            }
+          } else {
+            w = __ldg(P.fin_src + b0 + kk);
+            ms = __ldg(P.fin_ms + b0 + kk);
+            rr = ld_state_raw(P, w & kSrcMask);
+          }
         };
         const RfOut R = pin_rf<kLSE>(P, 0, nf, arc);
         const RfOut F = pin_rf<kLSE>(P, 1, nf, arc);
@@ -847,12 +950,9 @@ __global__ void __launch_bounds__(kThreads, 1) inc_kernel(IncParams Q) {
           __double_as_longlong(w1) != __double_as_longlong(old.v1)) {
         store_state(P, i, mu0, mu1, v0, v1);
         atomicAdd(&s_cnt[1], 1ull);
-        int deepest = -1;
-        for (int r = __ldg(Q.fanout_ptr + i); r < __ldg(Q.fanout_ptr + i + 1); ++r) {
-          const int sink = __ldg(Q.fout_sink + r);
-          Q.dirty[sink] = Q.stamp;
-          deepest = max(deepest, __ldg(Q.pin_level + sink));
-        }
+        for (int r = __ldg(Q.fanout_ptr + i); r < __ldg(Q.fanout_ptr + i + 1); ++r)
+          Q.dirty[__ldg(Q.fout_sink + r)] = Q.stamp;
+        const int deepest = __ldg(Q.max_sink_level + i);
         if (deepest >= 0) atomicMax(Q.lvl_range + 1, deepest);
       }
     }
@@ -913,17 +1013,17 @@ int query_grid(int device, int* grid) {
   if (!coop) return int(cudaErrorNotSupported);
   int err = set_smem(fwd_kernel<false>, kFwdSmem);
   if (!err) err = set_smem(fwd_kernel<true>, kFwdSmem);
-  if (!err) err = set_smem(bwd_kernel<false>, kBwdSmem);
-  if (!err) err = set_smem(bwd_kernel<true>, kBwdSmem);
+  if (!err) err = set_smem(bwd_kernel<false>, bwd_smem<false>());
+  if (!err) err = set_smem(bwd_kernel<true>, bwd_smem<true>());
   if (err) return err;
   int occ = 1 << 30, b = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<false>, kThreads, kFwdSmem);
   occ = std::min(occ, b);
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<true>, kThreads, kFwdSmem);
   occ = std::min(occ, b);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bwd_kernel<false>, kThreads, kBwdSmem);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bwd_kernel<false>, kThreads, bwd_smem<false>());
   occ = std::min(occ, b);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bwd_kernel<true>, kThreads, kBwdSmem);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bwd_kernel<true>, kThreads, bwd_smem<true>());
   occ = std::min(occ, b);
   if (occ <= 0) return int(cudaErrorLaunchOutOfResources);
   *grid = occ * sms;
@@ -1046,7 +1146,8 @@ int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float*
   const bool lse = g.last_tau > 0.f;
   P.mode = g.bwd_schedule == 0 ? 2 : 0;
   P.par = (++g.pass_bwd) & 1u;
-  return launch_items(lse ? (const void*)bwd_kernel<true> : (const void*)bwd_kernel<false>, kBwdSmem,
+  return launch_items(lse ? (const void*)bwd_kernel<true> : (const void*)bwd_kernel<false>,
+                      lse ? bwd_smem<true>() : bwd_smem<false>(),
                       P, g.bwd_items, true, st);
 }
 
@@ -1078,6 +1179,7 @@ int launch_forward_incremental(DevGraph& g, float n_sigma, float tau, void* stre
   Q.fanout_ptr = g.fanout_ptr;
   Q.fout_sink = g.fout_sink;
   Q.pin_level = g.pin_level;
+  Q.max_sink_level = g.max_sink_level;
   Q.dirty = g.dirty;
   Q.stamp = ++g.inc_epoch;
   Q.lvl_range = g.lvl_range;

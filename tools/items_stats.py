@@ -1,4 +1,5 @@
 """Replicates csrc/items.cpp on the host to report item/round counts per config."""
+import os
 import sys
 import numpy as np
 sys.path.insert(0, '.')
@@ -41,7 +42,7 @@ for l in range(lv["num_levels"]):
     wf = np.concatenate([[0], np.cumsum(1 + f)])
     wb = np.concatenate([[0], np.cumsum(1 + f + o)])
     rf = rounds(wf, None, pc, np.zeros_like(pc), G, (2048, 2560, 1 << 30))
-    rb = rounds(wb, None, pc, oc, G, (1024, 2048, 2048))
+    rb = rounds(wb, None, pc, oc, G, tuple(int(x) for x in os.environ.get("BWD_CAPS", "1024,2048,2048").split(",")))
     tf += rf; tb += rb
     widths.append((b - a, int(pc[-1]), rf, rb))
 print("levels", lv["num_levels"], "fwd steps", tf, "bwd steps", tb)

@@ -28,19 +28,25 @@ off2line = {}
 for l in lines[start + 1:]:
     if l.strip().startswith(".section") or (l.strip().endswith(":") and l.strip().startswith(".text.")):
         break
-    m = re.search(r'//## File ".*?", line (\d+)', l)
+    m = re.search(r'//## File "(.*?)", line (\d+)', l)
     if m:
-        cur = int(m.group(1))
+        cur = (m.group(1), int(m.group(2)))
         continue
     m = re.match(r"\s*/\*([0-9a-f]{4,})\*/", l)
     if m and cur is not None:
         off2line[int(m.group(1), 16)] = cur
 by_line = collections.Counter()
 for off, n in samples.items():
-    by_line[off2line.get(off, -1)] += n
+    by_line[off2line.get(off, ("?", -1))] += n
 tot = sum(by_line.values())
-src = open(sys.argv[5] if len(sys.argv) > 5 else "paper_conf_dac_lugklr25_b200/csrc/kernels.cu").read().split("\n")
+srcs = {}
 top = int(sys.argv[4]) if len(sys.argv) > 4 else 25
-for line, n in by_line.most_common(top):
+for (f, line), n in by_line.most_common(top):
+    if f not in srcs:
+        try:
+            srcs[f] = open(f).read().split("\n")
+        except OSError:
+            srcs[f] = []
+    src = srcs[f]
     text = src[line - 1].strip() if 0 < line <= len(src) else "?"
-    print(f"{100 * n / tot:5.1f}%  L{line:5d}  {text[:100]}")
+    print(f"{100 * n / tot:5.1f}%  {f.split('/')[-1]}:{line:<5d} {text[:100]}")
