@@ -868,6 +868,9 @@ __global__ void __launch_bounds__(kThreads, 1) inc_kernel(IncParams Q) {
   const int c = blockIdx.x, tid = threadIdx.x;
   __shared__ int s_exit;
   __shared__ unsigned long long s_cnt[2];
+  constexpr int kWideMarks = 128;
+  __shared__ int s_wide[kWideMarks];
+  __shared__ int s_nwide;
   const int lmin = __ldcg(Q.lvl_range);
   if (tid == 0) s_cnt[0] = s_cnt[1] = 0ull;
   for (int k = P.step_begin; k < P.step_end; ++k) {
@@ -876,7 +879,10 @@ __global__ void __launch_bounds__(kThreads, 1) inc_kernel(IncParams Q) {
     const int l = B.x;
     if (l < lmin) continue;   // below the shallowest mark: nothing to do, nothing to publish
     if (l > lmin) inc_wait(Q, l - 1);
-    if (tid == 0) s_exit = l > ld_acquire(reinterpret_cast<const uint32_t*>(Q.lvl_range + 1)) ? 1 : 0;
+    if (tid == 0) {
+      s_exit = l > ld_acquire(reinterpret_cast<const uint32_t*>(Q.lvl_range + 1)) ? 1 : 0;
+      s_nwide = 0;
+    }
     __syncthreads();
     if (s_exit) break;
     for (int i = A.x + tid; i < A.y; i += kThreads) {
@@ -950,11 +956,28 @@ __global__ void __launch_bounds__(kThreads, 1) inc_kernel(IncParams Q) {
           __double_as_longlong(w1) != __double_as_longlong(old.v1)) {
         store_state(P, i, mu0, mu1, v0, v1);
         atomicAdd(&s_cnt[1], 1ull);
-        for (int r = __ldg(Q.fanout_ptr + i); r < __ldg(Q.fanout_ptr + i + 1); ++r)
-          Q.dirty[__ldg(Q.fout_sink + r)] = Q.stamp;
+        const int r0 = __ldg(Q.fanout_ptr + i), r1 = __ldg(Q.fanout_ptr + i + 1);
+        bool deferred = false;
+        if (r1 - r0 > 32) {   // wide fanout: marked cooperatively after the item
+          const int slot = atomicAdd(&s_nwide, 1);
+          if (slot < kWideMarks) {
+            s_wide[slot] = i;
+            deferred = true;
+          }
+        }
+        if (!deferred)
+          for (int r = r0; r < r1; ++r) Q.dirty[__ldg(Q.fout_sink + r)] = Q.stamp;
         const int deepest = __ldg(Q.max_sink_level + i);
         if (deepest >= 0) atomicMax(Q.lvl_range + 1, deepest);
       }
+    }
+    __syncthreads();
+    // cooperative marking of the wide fanouts of changed pins
+    const int nw = min(s_nwide, kWideMarks);
+    for (int w = 0; w < nw; ++w) {
+      const int pin = s_wide[w];
+      for (int r = __ldg(Q.fanout_ptr + pin) + tid; r < __ldg(Q.fanout_ptr + pin + 1); r += kThreads)
+        Q.dirty[__ldg(Q.fout_sink + r)] = Q.stamp;
     }
     __syncthreads();
     if ((B.y & kItemLast) && tid == 0) {
