@@ -41,7 +41,7 @@ constexpr int kHeavyFanout = 256;
 // CTA shape (one 1024-thread CTA per SM) and shared-memory stage capacities
 // (per item; two stages are double-buffered)
 constexpr int kThreads = 1024;
-constexpr int kFwdPins = 2048, kFwdArcs = 2048;                     // forward item caps
+constexpr int kFwdPins = 1024, kFwdArcs = 1024;                     // forward item caps
 constexpr int kBwdPins = 2048, kBwdFanout = 2048, kBwdArcs = 2048;  // backward item caps
 static_assert(kHeavyFanout <= kBwdFanout, "a light pin's fanout row must fit one item");
 

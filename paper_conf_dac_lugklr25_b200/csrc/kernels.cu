@@ -163,7 +163,6 @@ struct FwdStage {
 };
 // per arc: gathered source record + corner arrivals of its candidates
 // {A[rf=R][s0], A[rf=F][s0], A[R][s1], A[F][s1]} (s1 only for non-unate arcs)
-constexpr size_t kFwdSmem = 2 * sizeof(FwdStage) + (sizeof(Raw) + sizeof(double4)) * kFwdArcs;
 
 __device__ __forceinline__ bool fwd_staged(const int4& A, const int4& B) {
   return A.y > A.x && B.x > 0 && !(B.y & kItemDirect);
@@ -302,85 +301,139 @@ __device__ __forceinline__ void trace_stamp(const KParams& P, int c, int nsteps,
   if (P.trace && threadIdx.x == 0) P.trace[(size_t(c) * nsteps + t) * 4 + slot] = gtimer();
 }
 
+// Forward persistent kernel.  Warp 0 (lane 0) is the producer: it streams
+// items into two shared-memory stages with TMA bulk copies (full[s]: mbarrier
+// with complete_tx) and re-fills a stage once every worker warp has released
+// it (empty[s]).  Warps 1..31 are independent workers: each takes 32 pins of
+// the item at a time, gathers its pins' source records with cp.async
+// (LDGSTS) into shared memory, re-polls stale words (parity dataflow),
+// computes the candidate corners arc-parallel within the warp, then merges
+// one pin per lane and stores -- only __syncwarp between the phases, so no
+// CTA-wide barrier sits on the level-to-level dependency chain.
+__device__ __forceinline__ void mbar_arrive1(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+constexpr int kWorkerWarps = kThreads / 32 - 1;
+constexpr int kWorkers = kWorkerWarps * 32;
+constexpr size_t kFwdSmemV6 = 2 * sizeof(FwdStage) + 2 * (sizeof(Raw) + sizeof(double4)) * kFwdArcs;
+
 template <bool kLSE>
 __global__ void __launch_bounds__(kThreads, 1) fwd_kernel(KParams P) {
   extern __shared__ __align__(128) unsigned char smem[];
   FwdStage* stage = reinterpret_cast<FwdStage*>(smem);
-  Raw* gath = reinterpret_cast<Raw*>(smem + 2 * sizeof(FwdStage));
-  double4* candA = reinterpret_cast<double4*>(smem + 2 * sizeof(FwdStage) + sizeof(Raw) * kFwdArcs);
-  __shared__ __align__(8) uint64_t full[2];
-  const int c = blockIdx.x;
-  const int tid = threadIdx.x;
+  Raw* gath_all = reinterpret_cast<Raw*>(smem + 2 * sizeof(FwdStage));
+  double4* cand_all = reinterpret_cast<double4*>(smem + 2 * sizeof(FwdStage) + 2 * sizeof(Raw) * kFwdArcs);
+  __shared__ __align__(8) uint64_t full[2], empty[2];
+  const int c = blockIdx.x, tid = threadIdx.x;
+  const int warp = tid >> 5, lane = tid & 31;
   if (tid == 0) {
-    mbar_init1(&full[0]);
-    mbar_init1(&full[1]);
+    for (int x = 0; x < 2; ++x) {
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&full[x])) : "memory");
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(&empty[x])), "r"(kWorkerWarps)
+                   : "memory");
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
-  uint32_t phase[2] = {0u, 0u};
   const int nsteps = P.step_end - P.step_begin;
-  if (tid == 0 && nsteps > 0) fwd_prefetch(P, &stage[0], &full[0], P.step_begin, c);
+  if (warp == 0) {   // producer
+    if (lane == 0) {
+      for (int t = 0; t < nsteps; ++t) {
+        const int s = t & 1;
+        if (t >= 2) mbar_wait(&empty[s], uint32_t(((t >> 1) - 1) & 1));
+        const int k = P.step_begin + t;
+        const int4 A = __ldg(P.item_a + size_t(k) * P.grid + c);
+        const int4 B = __ldg(P.item_b + size_t(k) * P.grid + c);
+        if (fwd_staged(A, B)) fwd_prefetch(P, &stage[s], &full[s], k, c);
+        else mbar_arrive1(&full[s]);
+      }
+    }
+    return;
+  }
+  const int ww = warp - 1, wt = tid - 32;
+  const double ns = double(P.n_sigma);
   for (int t = 0; t < nsteps; ++t) {
-    const int buf = t & 1;
+    const int s = t & 1;
     const int k = P.step_begin + t;
     const int4 A = __ldg(P.item_a + size_t(k) * P.grid + c);   // {pin_lo, pin_hi, arc_lo, arc_hi}
     const int4 B = __ldg(P.item_b + size_t(k) * P.grid + c);   // {level, flags}
-    if (tid == 0 && t + 1 < nsteps) fwd_prefetch(P, &stage[buf ^ 1], &full[buf ^ 1], k + 1, c);
-    trace_stamp(P, c, nsteps, t, 0);
-    if (A.y > A.x) {
+    mbar_wait(&full[s], uint32_t((t >> 1) & 1));
+    if (P.trace && wt == 0) P.trace[(size_t(c) * nsteps + t) * 4 + 0] = gtimer();
+    const int np = A.y - A.x;
+    if (np > 0) {
       if (B.x == 0) {
         // startpoints: clock arrival distribution, mean and variance per rf
-        for (int i = A.x + tid; i < A.y; i += kThreads) {
+        for (int i = A.x + wt; i < A.y; i += kWorkers) {
           const float4 v = __ldg(P.src_ms + i);
           store_state(P, i, double(v.x), double(v.y), double(v.z) * double(v.z), double(v.w) * double(v.w));
         }
       } else if (!(B.y & kItemDirect)) {
-        mbar_wait(&full[buf], phase[buf]);
-        phase[buf] ^= 1u;
-        const FwdStage& S = stage[buf];
+        const FwdStage& S = stage[s];
+        Raw* gath = gath_all + s * kFwdArcs;
+        double4* candA = cand_all + s * kFwdArcs;
         const int po = A.x & 3, so = A.z & 3;
-        const int na = A.w - A.z;
-        // (1) gathers: asynchronous global->shared copies (LDGSTS, through L2)
-        // of every source record of this thread, then complete them: re-poll
-        // only records whose words do not all carry this pass's parity.
-        for (int a = tid; a < na; a += kThreads) {
-          const PinState* src = P.state + (S.src[so + a] & kSrcMask);
-          const uint32_t d = smem_u32(gath + a);
-          asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n\t"
-                       "cp.async.cg.shared.global [%2], [%3], 16;" ::"r"(d),
-                       "l"(src), "r"(d + 16u), "l"(reinterpret_cast<const char*>(src) + 16)
-                       : "memory");
-        }
-        asm volatile("cp.async.wait_all;" ::: "memory");
-        const double ns = double(P.n_sigma);
-        for (int a = tid; a < na; a += kThreads) {
-          Raw r = gath[a];
-          const int32_t w = S.src[so + a];
-          if (P.mode == 2 && !raw_ready(r, P.par)) {
-            await_raw(P, w & kSrcMask, r);
-            gath[a] = r;
+        for (int p0 = ww * 32; p0 < np; p0 += kWorkers) {
+          const int a_lo = S.ptr[po + p0] - A.z;
+          const int a_hi = S.ptr[po + min(p0 + 32, np)] - A.z;
+          if (a_hi - a_lo == min(32, np - p0)) {
+            // every pin of this round has fanin 1 (net sinks): one register
+            // gather per lane, no shared-memory staging, no warp sync.  Same
+            // merge function as the general path (nf = 1), hence bit-identical.
+            if (p0 + lane < np) {
+              const int a = a_lo + lane;
+              const int32_t w = S.src[so + a];
+              const float4 ms = S.ms[a];
+              Raw r = ld_state_raw(P, w & kSrcMask);
+              await_raw(P, w & kSrcMask, r);
+              fwd_pin<kLSE>(P, A.x + p0 + lane, 1, A.z + a, [&](int, int32_t& w_, float4& ms_, Raw& r_) {
+                w_ = w;
+                ms_ = ms;
+                r_ = r;
+              });
+            }
+            continue;
           }
-          // arc-parallel candidate corners (Eq 1-3), both sink transitions
-          const Gath st = unpack(r);
-          const float4 ms = S.ms[a];
-          const int u = int(uint32_t(w) >> kUnateShift);
-          double4 ca;
-          ca.x = make_cand(st, ms, 0, src_tr(0, u, 0), ns).A;
-          ca.y = make_cand(st, ms, 1, src_tr(1, u, 0), ns).A;
-          ca.z = u == 2 ? make_cand(st, ms, 0, 1, ns).A : 0.0;
-          ca.w = u == 2 ? make_cand(st, ms, 1, 0, ns).A : 0.0;
-          candA[a] = ca;
-        }
-        __syncthreads();
-        trace_stamp(P, c, nsteps, t, 1);
-        // (2) compute: one thread per pin (both rf), merging the precomputed corners
-        for (int p = tid; p < A.y - A.x; p += kThreads) {
-          const int b0 = S.ptr[po + p] - A.z;
-          const int nf = S.ptr[po + p + 1] - A.z - b0;
-          fwd_pin_pre<kLSE>(P, A.x + p, nf, A.z + b0, &S.src[so + b0], &S.ms[b0], &gath[b0], &candA[b0]);
+          // (1) gathers of this warp's arcs: cp.async through L2, then re-poll stale words
+          for (int a = a_lo + lane; a < a_hi; a += 32) {
+            const PinState* src = P.state + (S.src[so + a] & kSrcMask);
+            const uint32_t d = smem_u32(gath + a);
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n\t"
+                         "cp.async.cg.shared.global [%2], [%3], 16;" ::"r"(d),
+                         "l"(src), "r"(d + 16u), "l"(reinterpret_cast<const char*>(src) + 16)
+                         : "memory");
+          }
+          asm volatile("cp.async.wait_all;" ::: "memory");
+          // (2) arc-parallel candidate corners (Eq 1-3), both sink transitions
+          for (int a = a_lo + lane; a < a_hi; a += 32) {
+            Raw r = gath[a];
+            const int32_t w = S.src[so + a];
+            if (P.mode == 2 && !raw_ready(r, P.par)) {
+              await_raw(P, w & kSrcMask, r);
+              gath[a] = r;
+            }
+            const Gath st = unpack(r);
+            const float4 ms = S.ms[a];
+            const int u = int(uint32_t(w) >> kUnateShift);
+            double4 ca;
+            ca.x = make_cand(st, ms, 0, src_tr(0, u, 0), ns).A;
+            ca.y = make_cand(st, ms, 1, src_tr(1, u, 0), ns).A;
+            ca.z = u == 2 ? make_cand(st, ms, 0, 1, ns).A : 0.0;
+            ca.w = u == 2 ? make_cand(st, ms, 1, 0, ns).A : 0.0;
+            candA[a] = ca;
+          }
+          __syncwarp();
+          // (3) one pin per lane: merge the precomputed corners, store
+          const int p = p0 + lane;
+          if (p < np) {
+            const int b0 = S.ptr[po + p] - A.z;
+            const int nf = S.ptr[po + p + 1] - A.z - b0;
+            fwd_pin_pre<kLSE>(P, A.x + p, nf, A.z + b0, &S.src[so + b0], &S.ms[b0], &gath[b0], &candA[b0]);
+          }
+          __syncwarp();
         }
       } else {
-        for (int i = A.x + tid; i < A.y; i += kThreads) {
+        for (int i = A.x + wt; i < A.y; i += kWorkers) {
           const int b0 = __ldg(P.fanin_ptr + i);
           const int nf = __ldg(P.fanin_ptr + i + 1) - b0;
           fwd_pin<kLSE>(P, i, nf, b0, [&](int kk, int32_t& w, float4& ms, Raw& rr) {
@@ -392,9 +445,9 @@ __global__ void __launch_bounds__(kThreads, 1) fwd_kernel(KParams P) {
         }
       }
     }
-    trace_stamp(P, c, nsteps, t, 3);   // thread 0's own work done (debug trace)
-    __syncthreads();   // stage[buf] and gath are free for reuse
-    trace_stamp(P, c, nsteps, t, 2);
+    __syncwarp();
+    if (P.trace && wt == 0) P.trace[(size_t(c) * nsteps + t) * 4 + 2] = gtimer();
+    if (lane == 0) mbar_arrive1(&empty[s]);
   }
 }
 
@@ -1034,15 +1087,15 @@ int query_grid(int device, int* grid) {
   if (e != cudaSuccess) return int(e);
   cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, device);
   if (!coop) return int(cudaErrorNotSupported);
-  int err = set_smem(fwd_kernel<false>, kFwdSmem);
-  if (!err) err = set_smem(fwd_kernel<true>, kFwdSmem);
+  int err = set_smem(fwd_kernel<false>, kFwdSmemV6);
+  if (!err) err = set_smem(fwd_kernel<true>, kFwdSmemV6);
   if (!err) err = set_smem(bwd_kernel<false>, bwd_smem<false>());
   if (!err) err = set_smem(bwd_kernel<true>, bwd_smem<true>());
   if (err) return err;
   int occ = 1 << 30, b = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<false>, kThreads, kFwdSmem);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<false>, kThreads, kFwdSmemV6);
   occ = std::min(occ, b);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<true>, kThreads, kFwdSmem);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<true>, kThreads, kFwdSmemV6);
   occ = std::min(occ, b);
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bwd_kernel<false>, kThreads, bwd_smem<false>());
   occ = std::min(occ, b);
@@ -1133,7 +1186,7 @@ int launch_forward(DevGraph& g, float n_sigma, float tau, int schedule, void* st
     P.mode = schedule == 0 ? 2 : 0;   // dataflow persistent / one launch per level
     P.par = (++g.pass_fwd) & 1u;
     int err = launch_items(lse ? (const void*)fwd_kernel<true> : (const void*)fwd_kernel<false>,
-                           kFwdSmem, P, g.fwd_items, false, st);
+                           kFwdSmemV6, P, g.fwd_items, false, st);
     if (err) return err;
   }
   g.last_n_sigma = n_sigma;

@@ -41,6 +41,9 @@ for name in ("fwd_trace.bin", "bwd_trace.bin"):
     t0 = t[:, 0, 0].min()
     s0, s1, s2 = (t[..., i] - t0 for i in range(3))   # item start, gathers done, item done
     has_g = t[..., 1] > 0
+    if not has_g.any():   # kernels that stamp only start/end (warp-independent forward)
+        s1 = s0
+        has_g = t[..., 2] > 0
     print(f"== {name}: grid={t.shape[0]} steps={t.shape[1]} total={s2.max()/1e3:.1f} us")
     gather = np.where(has_g, s1 - s0, 0)
     comp = np.where(has_g, s2 - s1, 0)
