@@ -314,16 +314,159 @@ __device__ __forceinline__ void mbar_arrive1(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
-constexpr int kWorkerWarps = kThreads / 32 - 1;
+#ifndef INSTA_FWD_THREADS
+#define INSTA_FWD_THREADS 768
+#endif
+constexpr int kFwdThreads = INSTA_FWD_THREADS;   // forward CTA: 1 producer warp + workers
+constexpr int kWorkerWarps = kFwdThreads / 32 - 1;
 constexpr int kWorkers = kWorkerWarps * 32;
-constexpr size_t kFwdSmemV6 = 2 * sizeof(FwdStage) + 2 * (sizeof(Raw) + sizeof(double4)) * kFwdArcs;
+constexpr size_t kFwdSmemV6 = 2 * sizeof(FwdStage) + 2 * sizeof(Raw) * kFwdArcs;
+constexpr int kFastPins = ((kFwdPins + kWorkerWarps - 1) / kWorkerWarps + 31) / 32;   // fanin-1 pins per lane
+
+// One round of the forward: pins [q, q + cnt) of the item whose arcs
+// [base, base + na), na <= 32, sit one per lane.  Each lane forms its arc's
+// candidate corners (Eq 1-3) for both sink transitions; a segmented first
+// arg-max across the pin's lanes (tree of shuffles: the upper half replaces
+// the lower only if strictly greater, so ties keep the lower arc -- Alg 2
+// l.4) leaves the merge in the pin's first lane, which stores the record.
+// LSE (Eq 4, 6): the normalizer is accumulated by the first lane in the
+// canonical order of merge_rf (arc by arc, s = rf then ~rf), every lane then
+// writes its arc's weights.  Same make_cand / lse_w / lse_arrival
+// arithmetic as merge_rf, hence bit-identical to the other paths.
+struct Best {
+  double A, mu, var;
+  float sig;
+  int idx;   // k | s << 15
+};
+
+__device__ __forceinline__ Best shfl_down_best(const Best& b, int d) {
+  Best o;
+  o.A = __shfl_down_sync(0xffffffffu, b.A, d);
+  o.mu = __shfl_down_sync(0xffffffffu, b.mu, d);
+  o.var = __shfl_down_sync(0xffffffffu, b.var, d);
+  o.sig = __shfl_down_sync(0xffffffffu, b.sig, d);
+  o.idx = __shfl_down_sync(0xffffffffu, b.idx, d);
+  return o;
+}
+
+// Round layout (shared-memory topology only, so it is formed before the
+// gathers land): pins [q, q + cnt) with their arcs [base, base + na) one per
+// lane; heads = bit of each pin's first arc.
+struct Round {
+  int q, cnt, base, na, seg, seg_end;
+  uint32_t heads;
+  int32_t w;   // this lane's arc source word
+  float4 ms;   // this lane's arc (mean, sigma) per rf
+};
+
+// cnt == 0: pin q alone has more than 32 arcs
+__device__ __forceinline__ Round round_at(const FwdStage& S, const int4& A, int po, int so, int q, int q1,
+                                          int lane) {
+  Round R;
+  R.q = q;
+  R.base = S.ptr[po + q] - A.z;
+  const int e = q + lane < q1 ? S.ptr[po + q + lane + 1] - A.z - R.base : 1 << 30;
+  R.cnt = __popc(__ballot_sync(0xffffffffu, e <= 32));
+  R.na = __shfl_sync(0xffffffffu, e, R.cnt > 0 ? R.cnt - 1 : 0);
+  const int hb = __shfl_up_sync(0xffffffffu, e, 1);
+  const uint32_t head_bit = lane < R.cnt ? 1u << (lane == 0 ? 0 : hb) : 0u;
+  R.heads = __reduce_or_sync(0xffffffffu, head_bit);
+  const uint32_t below = R.heads & (0xffffffffu >> (31 - lane));
+  R.seg = 31 - __clz(below);   // first lane of my pin
+  const uint32_t above = lane == 31 ? 0u : R.heads & (0xfffffffeu << lane);
+  R.seg_end = above ? __ffs(above) - 1 : R.na;
+  if (R.cnt > 0 && lane < R.na) {
+    R.w = S.src[so + R.base + lane];
+    R.ms = S.ms[R.base + lane];
+  }
+  return R;
+}
 
 template <bool kLSE>
-__global__ void __launch_bounds__(kThreads, 1) fwd_kernel(KParams P) {
+__device__ __forceinline__ void fwd_round(const KParams& P, const Raw* gath, const int4& A, const Round& R,
+                                          int lane) {
+  const double ns = double(P.n_sigma);
+  const int q = R.q, base = R.base, seg = R.seg, seg_end = R.seg_end;
+  const uint32_t heads = R.heads;
+  const bool act = lane < R.na;
+  const int k = lane - seg;
+  Best b[2];
+  double A0[2] = {0.0, 0.0}, A1[2] = {0.0, 0.0};
+  int u = 0;
+  if (act) {
+    u = int(uint32_t(R.w) >> kUnateShift);
+    const float4 ms = R.ms;
+    const Gath st = unpack(gath[base + lane]);
+#pragma unroll
+    for (int rf = 0; rf < 2; ++rf) {
+      const int s0 = src_tr(rf, u, 0);
+      const Cand c0 = make_cand(st, ms, rf, s0, ns);
+      A0[rf] = c0.A;
+      b[rf] = Best{c0.A, c0.mu, c0.var, c0.sig, k | (s0 << 15)};
+      if (u == 2) {
+        const Cand c1 = make_cand(st, ms, rf, rf ^ 1, ns);
+        A1[rf] = c1.A;
+        if (c1.A > c0.A) b[rf] = Best{c1.A, c1.mu, c1.var, c1.sig, k | ((rf ^ 1) << 15)};
+      }
+    }
+  } else {
+    b[0] = b[1] = Best{0.0, 0.0, 0.0, 0.f, 0};
+  }
+  const int maxlen = __reduce_max_sync(0xffffffffu, act ? seg_end - seg : 0);
+  for (int d = 1; d < maxlen; d <<= 1) {
+#pragma unroll
+    for (int rf = 0; rf < 2; ++rf) {
+      const Best o = shfl_down_best(b[rf], d);
+      if ((k & (2 * d - 1)) == 0 && lane + d < seg_end && o.A > b[rf].A) b[rf] = o;
+    }
+  }
+  const int i = A.x + q + __popc(heads & ((1u << lane) - 1u));   // my pin (valid in head lanes)
+  if (!kLSE) {
+    if (act && k == 0) {
+      store_state(P, i, b[0].mu, b[1].mu, b[0].var, b[1].var);
+      P.win[i] = b[0].idx | (b[1].idx << 16);
+    }
+  } else {
+    const int src_lane = act ? seg : lane;
+    float w0[2], w1[2], inv[2];
+#pragma unroll
+    for (int rf = 0; rf < 2; ++rf) {
+      const double best = __shfl_sync(0xffffffffu, b[rf].A, src_lane);   // M of my pin
+      w0[rf] = act ? lse_w(A0[rf], best, P.inv_tau) : 0.f;
+      w1[rf] = act && u == 2 ? lse_w(A1[rf], best, P.inv_tau) : 0.f;
+      // normalizer in merge_rf's order, accumulated by the pin's first lane
+      float acc = 0.f;
+      for (int j = 0; j < maxlen; ++j) {
+        const float v0 = __shfl_down_sync(0xffffffffu, w0[rf], j);
+        const float v1 = __shfl_down_sync(0xffffffffu, w1[rf], j);
+        if (j < seg_end - lane) {
+          acc += v0;
+          acc += v1;   // 0 for non-NON arcs: exact no-op on a non-negative sum
+        }
+      }
+      if (act && k == 0) {
+        b[rf].mu = lse_arrival(b[rf].A, double(P.tau), acc) - ns * double(b[rf].sig);   // Eq 4, reading R1
+      }
+      inv[rf] = 1.f / __shfl_sync(0xffffffffu, acc, src_lane);   // as merge_rf_pre / arc_weights
+    }
+    if (act && k == 0) store_state(P, i, b[0].mu, b[1].mu, b[0].var, b[1].var);
+    if (act) {
+      float wt[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
+#pragma unroll
+      for (int rf = 0; rf < 2; ++rf) {
+        wt[rf][src_tr(rf, u, 0)] = w0[rf] * inv[rf];
+        if (u == 2) wt[rf][rf ^ 1] = w1[rf] * inv[rf];
+      }
+      P.wts[A.z + base + lane] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
+    }
+  }
+}
+
+template <bool kLSE>
+__global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
   extern __shared__ __align__(128) unsigned char smem[];
   FwdStage* stage = reinterpret_cast<FwdStage*>(smem);
   Raw* gath_all = reinterpret_cast<Raw*>(smem + 2 * sizeof(FwdStage));
-  double4* cand_all = reinterpret_cast<double4*>(smem + 2 * sizeof(FwdStage) + 2 * sizeof(Raw) * kFwdArcs);
   __shared__ __align__(8) uint64_t full[2], empty[2];
   const int c = blockIdx.x, tid = threadIdx.x;
   const int warp = tid >> 5, lane = tid & 31;
@@ -371,30 +514,39 @@ __global__ void __launch_bounds__(kThreads, 1) fwd_kernel(KParams P) {
       } else if (!(B.y & kItemDirect)) {
         const FwdStage& S = stage[s];
         Raw* gath = gath_all + s * kFwdArcs;
-        double4* candA = cand_all + s * kFwdArcs;
         const int po = A.x & 3, so = A.z & 3;
-        for (int p0 = ww * 32; p0 < np; p0 += kWorkers) {
-          const int a_lo = S.ptr[po + p0] - A.z;
-          const int a_hi = S.ptr[po + min(p0 + 32, np)] - A.z;
-          if (a_hi - a_lo == min(32, np - p0)) {
-            // every pin of this round has fanin 1 (net sinks): one register
-            // gather per lane, no shared-memory staging, no warp sync.  Same
-            // merge function as the general path (nf = 1), hence bit-identical.
-            if (p0 + lane < np) {
-              const int a = a_lo + lane;
+        // this warp's contiguous share of the item's pins
+        const int q0 = ww * np / kWorkerWarps, q1 = (ww + 1) * np / kWorkerWarps;
+        const int a_lo = S.ptr[po + q0] - A.z, a_hi = S.ptr[po + q1] - A.z;
+        if (q1 > q0 && a_hi - a_lo == q1 - q0) {
+          // every pin has fanin 1 (net sinks): register gathers, all issued
+          // before any is awaited; same merge function (nf = 1) as below
+          Raw r[kFastPins];
+#pragma unroll
+          for (int x = 0; x < kFastPins; ++x) {
+            const int p = q0 + lane + 32 * x;
+            if (p < q1) r[x] = ld_state_raw(P, S.src[so + p - q0 + a_lo] & kSrcMask);
+          }
+#pragma unroll
+          for (int x = 0; x < kFastPins; ++x) {
+            const int p = q0 + lane + 32 * x;
+            if (p < q1) {
+              const int a = a_lo + p - q0;
               const int32_t w = S.src[so + a];
               const float4 ms = S.ms[a];
-              Raw r = ld_state_raw(P, w & kSrcMask);
-              await_raw(P, w & kSrcMask, r);
-              fwd_pin<kLSE>(P, A.x + p0 + lane, 1, A.z + a, [&](int, int32_t& w_, float4& ms_, Raw& r_) {
+              await_raw(P, w & kSrcMask, r[x]);
+              const Raw rx = r[x];
+              fwd_pin<kLSE>(P, A.x + p, 1, A.z + a, [&](int, int32_t& w_, float4& ms_, Raw& r_) {
                 w_ = w;
                 ms_ = ms;
-                r_ = r;
+                r_ = rx;
               });
             }
-            continue;
           }
-          // (1) gathers of this warp's arcs: cp.async through L2, then re-poll stale words
+        } else if (q1 > q0) {
+          Round R = round_at(S, A, po, so, q0, q1, lane);
+          // (1) gathers of all this warp's arcs: cp.async through L2, then
+          // re-poll the stale ones (producer not done yet)
           for (int a = a_lo + lane; a < a_hi; a += 32) {
             const PinState* src = P.state + (S.src[so + a] & kSrcMask);
             const uint32_t d = smem_u32(gath + a);
@@ -404,33 +556,40 @@ __global__ void __launch_bounds__(kThreads, 1) fwd_kernel(KParams P) {
                          : "memory");
           }
           asm volatile("cp.async.wait_all;" ::: "memory");
-          // (2) arc-parallel candidate corners (Eq 1-3), both sink transitions
-          for (int a = a_lo + lane; a < a_hi; a += 32) {
-            Raw r = gath[a];
-            const int32_t w = S.src[so + a];
-            if (P.mode == 2 && !raw_ready(r, P.par)) {
-              await_raw(P, w & kSrcMask, r);
-              gath[a] = r;
+          if (P.trace && wt == 0) P.trace[(size_t(c) * nsteps + t) * 4 + 1] = gtimer();
+          if (P.mode == 2) {
+            for (int a = a_lo + lane; a < a_hi; a += 32) {
+              Raw r = gath[a];
+              if (!raw_ready(r, P.par)) {
+                await_raw(P, S.src[so + a] & kSrcMask, r);
+                gath[a] = r;
+              }
             }
-            const Gath st = unpack(r);
-            const float4 ms = S.ms[a];
-            const int u = int(uint32_t(w) >> kUnateShift);
-            double4 ca;
-            ca.x = make_cand(st, ms, 0, src_tr(0, u, 0), ns).A;
-            ca.y = make_cand(st, ms, 1, src_tr(1, u, 0), ns).A;
-            ca.z = u == 2 ? make_cand(st, ms, 0, 1, ns).A : 0.0;
-            ca.w = u == 2 ? make_cand(st, ms, 1, 0, ns).A : 0.0;
-            candA[a] = ca;
           }
           __syncwarp();
-          // (3) one pin per lane: merge the precomputed corners, store
-          const int p = p0 + lane;
-          if (p < np) {
-            const int b0 = S.ptr[po + p] - A.z;
-            const int nf = S.ptr[po + p + 1] - A.z - b0;
-            fwd_pin_pre<kLSE>(P, A.x + p, nf, A.z + b0, &S.src[so + b0], &S.ms[b0], &gath[b0], &candA[b0]);
+          if (P.trace && wt == 0) P.trace[(size_t(c) * nsteps + t) * 4 + 3] = gtimer();
+          // (2) rounds of consecutive pins holding <= 32 arcs: one arc per
+          // lane, segmented arg-max across the lanes of each pin
+          while (R.q < q1) {
+            if (R.cnt == 0) {   // pin q alone has more than 32 arcs: one lane, serial merge
+              const int q = R.q, base = R.base;
+              if (lane == 0) {
+                const int nf = S.ptr[po + q + 1] - A.z - base;
+                fwd_pin<kLSE>(P, A.x + q, nf, A.z + base, [&](int kk, int32_t& w_, float4& ms_, Raw& r_) {
+                  w_ = S.src[so + base + kk];
+                  ms_ = S.ms[base + kk];
+                  r_ = gath[base + kk];
+                });
+              }
+              __syncwarp();
+              R = round_at(S, A, po, so, q + 1, q1, lane);
+              continue;
+            }
+            fwd_round<kLSE>(P, gath, A, R, lane);
+            const int qn = R.q + R.cnt;
+            if (qn < q1) R = round_at(S, A, po, so, qn, q1, lane);
+            else break;
           }
-          __syncwarp();
         }
       } else {
         for (int i = A.x + wt; i < A.y; i += kWorkers) {
@@ -1093,9 +1252,9 @@ int query_grid(int device, int* grid) {
   if (!err) err = set_smem(bwd_kernel<true>, bwd_smem<true>());
   if (err) return err;
   int occ = 1 << 30, b = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<false>, kThreads, kFwdSmemV6);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<false>, kFwdThreads, kFwdSmemV6);
   occ = std::min(occ, b);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<true>, kThreads, kFwdSmemV6);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<true>, kFwdThreads, kFwdSmemV6);
   occ = std::min(occ, b);
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bwd_kernel<false>, kThreads, bwd_smem<false>());
   occ = std::min(occ, b);
@@ -1131,7 +1290,7 @@ static int dump_trace(const char* name, unsigned long long* d, int grid, int ste
 
 // mode 2 (dataflow): one cooperative launch over all items; mode 0: one launch
 // per level (kernel boundaries order the levels).
-static int launch_items(const void* fn, size_t smem, KParams& P, const ItemTable& T, bool bwd,
+static int launch_items(const void* fn, int threads, size_t smem, KParams& P, const ItemTable& T, bool bwd,
                         cudaStream_t st) {
   P.trace = nullptr;
   if (P.mode != 0) {
@@ -1143,7 +1302,7 @@ static int launch_items(const void* fn, size_t smem, KParams& P, const ItemTable
       cudaMemsetAsync(P.trace, 0, size_t(P.grid) * T.num_steps * 32, st);
     }
     void* args[] = {&P};
-    int err = int(cudaLaunchCooperativeKernel(fn, dim3(P.grid), dim3(kThreads), args, smem, st));
+    int err = int(cudaLaunchCooperativeKernel(fn, dim3(P.grid), dim3(threads), args, smem, st));
     if (!err && tracing) err = dump_trace(bwd ? "bwd_trace.bin" : "fwd_trace.bin", P.trace, P.grid, T.num_steps, st);
     return err;
   }
@@ -1153,7 +1312,7 @@ static int launch_items(const void* fn, size_t smem, KParams& P, const ItemTable
     P.step_begin = T.level_step0[l];
     P.step_end = T.level_step0[l] + T.level_steps[l];
     void* args[] = {&P};
-    int err = int(cudaLaunchKernel(fn, dim3(P.grid), dim3(kThreads), args, smem, st));
+    int err = int(cudaLaunchKernel(fn, dim3(P.grid), dim3(threads), args, smem, st));
     if (err) return err;
   }
   return 0;
@@ -1185,7 +1344,7 @@ int launch_forward(DevGraph& g, float n_sigma, float tau, int schedule, void* st
   if (g.n > 0) {
     P.mode = schedule == 0 ? 2 : 0;   // dataflow persistent / one launch per level
     P.par = (++g.pass_fwd) & 1u;
-    int err = launch_items(lse ? (const void*)fwd_kernel<true> : (const void*)fwd_kernel<false>,
+    int err = launch_items(lse ? (const void*)fwd_kernel<true> : (const void*)fwd_kernel<false>, kFwdThreads,
                            kFwdSmemV6, P, g.fwd_items, false, st);
     if (err) return err;
   }
@@ -1222,7 +1381,7 @@ int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float*
   const bool lse = g.last_tau > 0.f;
   P.mode = g.bwd_schedule == 0 ? 2 : 0;
   P.par = (++g.pass_bwd) & 1u;
-  return launch_items(lse ? (const void*)bwd_kernel<true> : (const void*)bwd_kernel<false>,
+  return launch_items(lse ? (const void*)bwd_kernel<true> : (const void*)bwd_kernel<false>, kThreads,
                       lse ? bwd_smem<true>() : bwd_smem<false>(),
                       P, g.bwd_items, true, st);
 }

@@ -1,6 +1,6 @@
 """Per-step item timing spread on a layered graph (debug; run on the GPU box).
 
-usage: W=65536 FANIN=1 python tools/chain_trace.py
+usage: W=65536 FANIN=1 python tools/chain_trace.py   (NO_TRACE=1: just run, e.g. under ncu)
 For each step: spread of item start/end times across CTAs relative to the
 previous step's last end -- separates dependency jitter from item work.
 """
@@ -38,6 +38,8 @@ G = insta.Graph(layered(W, L, F))
 for _ in range(3):
     G.forward(3.0, 0.0, sync=False)
 torch.cuda.synchronize()
+if os.environ.get("NO_TRACE"):   # plain runs only (for ncu captures)
+    sys.exit(0)
 os.environ["INSTA_TRACE_DIR"] = out
 G.forward(3.0, 0.0, sync=False)
 torch.cuda.synchronize()
@@ -47,6 +49,7 @@ grid, steps, k = np.frombuffer(raw[:12], np.int32)
 t = np.frombuffer(raw[12:], np.uint64).reshape(grid, steps, k).astype(np.int64)
 t0 = t[:, 0, 0].min()
 st, en = t[..., 0] - t0, t[..., 2] - t0
+g1, g3 = t[..., 1] - t0, t[..., 3] - t0   # warp 0: gathers landed, corners computed (staged rounds)
 print(f"W={W} fanin={F} levels={L} grid={grid} steps={steps} total={en.max()/1e3:.1f} us")
 prev = 0
 for s in range(steps):
@@ -58,5 +61,10 @@ for s in range(steps):
     q = lambda x, p: np.percentile(x, p) / 1e3
     print(f"step {s:3d}: start rel prev-end [min {(a.min()-prev)/1e3:6.2f} med {(np.median(a)-prev)/1e3:6.2f}]"
           f" end rel prev-end [min {(b.min()-prev)/1e3:6.2f} med {(np.median(b)-prev)/1e3:6.2f} p90 {(np.percentile(b,90)-prev)/1e3:6.2f} max {(b.max()-prev)/1e3:6.2f}]"
-          f" dur med {np.median(b-a)/1e3:5.2f}")
+          f" dur med {np.median(b-a)/1e3:5.2f}", end="")
+    m = (t[:, s, 1] > 0) & (t[:, s, 3] > 0) & ok
+    if m.any():
+        print(f" | w0: landed {np.median(g1[m, s]-prev)/1e3:5.2f} polled+corners {np.median(g3[m, s]-prev)/1e3:5.2f}"
+              f" end {np.median(en[m, s]-prev)/1e3:5.2f}", end="")
+    print()
     prev = b.max()
