@@ -315,9 +315,13 @@ __device__ __forceinline__ void mbar_arrive1(uint64_t* bar) {
 }
 
 #ifndef INSTA_FWD_THREADS
-#define INSTA_FWD_THREADS 768
+#define INSTA_FWD_THREADS 512
 #endif
-constexpr int kFwdThreads = INSTA_FWD_THREADS;   // forward CTA: 1 producer warp + workers
+constexpr int kFwdThreads = INSTA_FWD_THREADS;
+#ifndef INSTA_ROUNDS
+#define INSTA_ROUNDS 1
+#endif
+constexpr int kRoundsPerPass = INSTA_ROUNDS;   // independent rounds interleaved per warp   // forward CTA: 1 producer warp + workers
 constexpr int kWorkerWarps = kFwdThreads / 32 - 1;
 constexpr int kWorkers = kWorkerWarps * 32;
 constexpr size_t kFwdSmemV6 = 2 * sizeof(FwdStage) + 2 * sizeof(Raw) * kFwdArcs;
@@ -382,82 +386,92 @@ __device__ __forceinline__ Round round_at(const FwdStage& S, const int4& A, int 
   return R;
 }
 
-template <bool kLSE>
-__device__ __forceinline__ void fwd_round(const KParams& P, const Raw* gath, const int4& A, const Round& R,
-                                          int lane) {
+// NR independent rounds per warp at once (their dependent chains interleave).
+template <bool kLSE, int NR>
+__device__ __forceinline__ void fwd_rounds(const KParams& P, const Raw* gath, const int4& A, const Round* R,
+                                           int lane) {
   const double ns = double(P.n_sigma);
-  const int q = R.q, base = R.base, seg = R.seg, seg_end = R.seg_end;
-  const uint32_t heads = R.heads;
-  const bool act = lane < R.na;
-  const int k = lane - seg;
-  Best b[2];
-  double A0[2] = {0.0, 0.0}, A1[2] = {0.0, 0.0};
-  int u = 0;
-  if (act) {
-    u = int(uint32_t(R.w) >> kUnateShift);
-    const float4 ms = R.ms;
-    const Gath st = unpack(gath[base + lane]);
+  Best b[NR][2];
+  double A0[NR][2], A1[NR][2];
+  int u[NR], k[NR];
+  bool act[NR];
+  int maxlen = 0;
 #pragma unroll
-    for (int rf = 0; rf < 2; ++rf) {
-      const int s0 = src_tr(rf, u, 0);
-      const Cand c0 = make_cand(st, ms, rf, s0, ns);
-      A0[rf] = c0.A;
-      b[rf] = Best{c0.A, c0.mu, c0.var, c0.sig, k | (s0 << 15)};
-      if (u == 2) {
-        const Cand c1 = make_cand(st, ms, rf, rf ^ 1, ns);
-        A1[rf] = c1.A;
-        if (c1.A > c0.A) b[rf] = Best{c1.A, c1.mu, c1.var, c1.sig, k | ((rf ^ 1) << 15)};
-      }
-    }
-  } else {
-    b[0] = b[1] = Best{0.0, 0.0, 0.0, 0.f, 0};
-  }
-  const int maxlen = __reduce_max_sync(0xffffffffu, act ? seg_end - seg : 0);
-  for (int d = 1; d < maxlen; d <<= 1) {
-#pragma unroll
-    for (int rf = 0; rf < 2; ++rf) {
-      const Best o = shfl_down_best(b[rf], d);
-      if ((k & (2 * d - 1)) == 0 && lane + d < seg_end && o.A > b[rf].A) b[rf] = o;
-    }
-  }
-  const int i = A.x + q + __popc(heads & ((1u << lane) - 1u));   // my pin (valid in head lanes)
-  if (!kLSE) {
-    if (act && k == 0) {
-      store_state(P, i, b[0].mu, b[1].mu, b[0].var, b[1].var);
-      P.win[i] = b[0].idx | (b[1].idx << 16);
-    }
-  } else {
-    const int src_lane = act ? seg : lane;
-    float w0[2], w1[2], inv[2];
-#pragma unroll
-    for (int rf = 0; rf < 2; ++rf) {
-      const double best = __shfl_sync(0xffffffffu, b[rf].A, src_lane);   // M of my pin
-      w0[rf] = act ? lse_w(A0[rf], best, P.inv_tau) : 0.f;
-      w1[rf] = act && u == 2 ? lse_w(A1[rf], best, P.inv_tau) : 0.f;
-      // normalizer in merge_rf's order, accumulated by the pin's first lane
-      float acc = 0.f;
-      for (int j = 0; j < maxlen; ++j) {
-        const float v0 = __shfl_down_sync(0xffffffffu, w0[rf], j);
-        const float v1 = __shfl_down_sync(0xffffffffu, w1[rf], j);
-        if (j < seg_end - lane) {
-          acc += v0;
-          acc += v1;   // 0 for non-NON arcs: exact no-op on a non-negative sum
-        }
-      }
-      if (act && k == 0) {
-        b[rf].mu = lse_arrival(b[rf].A, double(P.tau), acc) - ns * double(b[rf].sig);   // Eq 4, reading R1
-      }
-      inv[rf] = 1.f / __shfl_sync(0xffffffffu, acc, src_lane);   // as merge_rf_pre / arc_weights
-    }
-    if (act && k == 0) store_state(P, i, b[0].mu, b[1].mu, b[0].var, b[1].var);
-    if (act) {
-      float wt[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
+  for (int r = 0; r < NR; ++r) {
+    act[r] = lane < R[r].na;
+    k[r] = lane - R[r].seg;
+    u[r] = 0;
+    A0[r][0] = A0[r][1] = A1[r][0] = A1[r][1] = 0.0;
+    b[r][0] = b[r][1] = Best{0.0, 0.0, 0.0, 0.f, 0};
+    if (act[r]) {
+      u[r] = int(uint32_t(R[r].w) >> kUnateShift);
+      const Gath st = unpack(gath[R[r].base + lane]);
 #pragma unroll
       for (int rf = 0; rf < 2; ++rf) {
-        wt[rf][src_tr(rf, u, 0)] = w0[rf] * inv[rf];
-        if (u == 2) wt[rf][rf ^ 1] = w1[rf] * inv[rf];
+        const int s0 = src_tr(rf, u[r], 0);
+        const Cand c0 = make_cand(st, R[r].ms, rf, s0, ns);
+        A0[r][rf] = c0.A;
+        b[r][rf] = Best{c0.A, c0.mu, c0.var, c0.sig, k[r] | (s0 << 15)};
+        if (u[r] == 2) {
+          const Cand c1 = make_cand(st, R[r].ms, rf, rf ^ 1, ns);
+          A1[r][rf] = c1.A;
+          if (c1.A > c0.A) b[r][rf] = Best{c1.A, c1.mu, c1.var, c1.sig, k[r] | ((rf ^ 1) << 15)};
+        }
       }
-      P.wts[A.z + base + lane] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
+    }
+    maxlen = max(maxlen, act[r] ? R[r].seg_end - R[r].seg : 0);
+  }
+  maxlen = __reduce_max_sync(0xffffffffu, maxlen);
+  for (int d = 1; d < maxlen; d <<= 1) {
+#pragma unroll
+    for (int r = 0; r < NR; ++r) {
+#pragma unroll
+      for (int rf = 0; rf < 2; ++rf) {
+        const Best o = shfl_down_best(b[r][rf], d);
+        if ((k[r] & (2 * d - 1)) == 0 && lane + d < R[r].seg_end && o.A > b[r][rf].A) b[r][rf] = o;
+      }
+    }
+  }
+#pragma unroll
+  for (int r = 0; r < NR; ++r) {
+    const int i = A.x + R[r].q + __popc(R[r].heads & ((1u << lane) - 1u));   // my pin (head lanes)
+    if (!kLSE) {
+      if (act[r] && k[r] == 0) {
+        store_state(P, i, b[r][0].mu, b[r][1].mu, b[r][0].var, b[r][1].var);
+        P.win[i] = b[r][0].idx | (b[r][1].idx << 16);
+      }
+    } else {
+      const int src_lane = act[r] ? R[r].seg : lane;
+      float w0[2], w1[2], inv[2];
+#pragma unroll
+      for (int rf = 0; rf < 2; ++rf) {
+        const double best = __shfl_sync(0xffffffffu, b[r][rf].A, src_lane);   // M of my pin
+        w0[rf] = act[r] ? lse_w(A0[r][rf], best, P.inv_tau) : 0.f;
+        w1[rf] = act[r] && u[r] == 2 ? lse_w(A1[r][rf], best, P.inv_tau) : 0.f;
+        // normalizer in merge_rf's order, accumulated by the pin's first lane
+        float acc = 0.f;
+        for (int j = 0; j < maxlen; ++j) {
+          const float v0 = __shfl_down_sync(0xffffffffu, w0[rf], j);
+          const float v1 = __shfl_down_sync(0xffffffffu, w1[rf], j);
+          if (j < R[r].seg_end - lane) {
+            acc += v0;
+            acc += v1;   // 0 for non-NON arcs: exact no-op on a non-negative sum
+          }
+        }
+        if (act[r] && k[r] == 0)
+          b[r][rf].mu = lse_arrival(b[r][rf].A, double(P.tau), acc) - ns * double(b[r][rf].sig);   // Eq 4, R1
+        inv[rf] = 1.f / __shfl_sync(0xffffffffu, acc, src_lane);   // as merge_rf_pre / arc_weights
+      }
+      if (act[r] && k[r] == 0) store_state(P, i, b[r][0].mu, b[r][1].mu, b[r][0].var, b[r][1].var);
+      if (act[r]) {
+        float wt[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
+#pragma unroll
+        for (int rf = 0; rf < 2; ++rf) {
+          wt[rf][src_tr(rf, u[r], 0)] = w0[rf] * inv[rf];
+          if (u[r] == 2) wt[rf][rf ^ 1] = w1[rf] * inv[rf];
+        }
+        P.wts[A.z + R[r].base + lane] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
+      }
     }
   }
 }
@@ -585,8 +599,19 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
               R = round_at(S, A, po, so, q + 1, q1, lane);
               continue;
             }
-            fwd_round<kLSE>(P, gath, A, R, lane);
-            const int qn = R.q + R.cnt;
+            Round RR[kRoundsPerPass];
+            RR[0] = R;
+            int qn = R.q + R.cnt;
+#pragma unroll
+            for (int r = 1; r < kRoundsPerPass; ++r) {
+              RR[r] = round_at(S, A, po, so, min(qn, q1), q1, lane);
+              if (qn >= q1 || RR[r].cnt == 0) {
+                RR[r].na = 0;   // inactive slot
+                RR[r].cnt = 0;
+              }
+              qn += RR[r].cnt;
+            }
+            fwd_rounds<kLSE, kRoundsPerPass>(P, gath, A, RR, lane);
             if (qn < q1) R = round_at(S, A, po, so, qn, q1, lane);
             else break;
           }

@@ -35,16 +35,21 @@ F = int(os.environ.get("FANIN", "1"))
 L = int(os.environ.get("LEVELS", "40"))
 out = os.environ.get("OUT", "gpurun_out")
 G = insta.Graph(layered(W, L, F))
+BWD = bool(os.environ.get("BWD"))
 for _ in range(3):
     G.forward(3.0, 0.0, sync=False)
+    if BWD:
+        G.backward()
 torch.cuda.synchronize()
 if os.environ.get("NO_TRACE"):   # plain runs only (for ncu captures)
     sys.exit(0)
 os.environ["INSTA_TRACE_DIR"] = out
 G.forward(3.0, 0.0, sync=False)
+if BWD:
+    G.backward()
 torch.cuda.synchronize()
 del os.environ["INSTA_TRACE_DIR"]
-raw = open(os.path.join(out, "fwd_trace.bin"), "rb").read()
+raw = open(os.path.join(out, "bwd_trace.bin" if BWD else "fwd_trace.bin"), "rb").read()
 grid, steps, k = np.frombuffer(raw[:12], np.int32)
 t = np.frombuffer(raw[12:], np.uint64).reshape(grid, steps, k).astype(np.int64)
 t0 = t[:, 0, 0].min()
@@ -62,9 +67,9 @@ for s in range(steps):
     print(f"step {s:3d}: start rel prev-end [min {(a.min()-prev)/1e3:6.2f} med {(np.median(a)-prev)/1e3:6.2f}]"
           f" end rel prev-end [min {(b.min()-prev)/1e3:6.2f} med {(np.median(b)-prev)/1e3:6.2f} p90 {(np.percentile(b,90)-prev)/1e3:6.2f} max {(b.max()-prev)/1e3:6.2f}]"
           f" dur med {np.median(b-a)/1e3:5.2f}", end="")
-    m = (t[:, s, 1] > 0) & (t[:, s, 3] > 0) & ok
+    m = (t[:, s, 1] > 0) & ok
     if m.any():
-        print(f" | w0: landed {np.median(g1[m, s]-prev)/1e3:5.2f} polled+corners {np.median(g3[m, s]-prev)/1e3:5.2f}"
+        print(f" | w0: landed {np.median(g1[m, s]-prev)/1e3:5.2f} polled+corners {np.median(np.maximum(g3[m, s], 0)-prev)/1e3:5.2f}"
               f" end {np.median(en[m, s]-prev)/1e3:5.2f}", end="")
     print()
     prev = b.max()

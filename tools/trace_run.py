@@ -60,3 +60,35 @@ for name in ("fwd_trace.bin", "bwd_trace.bin"):
         print(f"  step {k:4d}: start[min {start_min[k]/1e3:8.1f}] end[max {end_max[k]/1e3:8.1f}] inc {inc[k]/1e3:6.2f}"
               f" | gather med {np.median(gk)/1e3 if gk.size else 0:5.2f} max {gk.max()/1e3 if gk.size else 0:5.2f}"
               f" | compute med {np.median(ck)/1e3 if ck.size else 0:5.2f} max {ck.max()/1e3 if ck.size else 0:5.2f}")
+
+# per-level view of the forward: step increments next to the level sizes
+if os.environ.get("LEVELS_VIEW"):
+    lv = insta.levelize(g.num_pins, g.arc_from, g.arc_to)
+    level = np.asarray(lv["level"])
+    sizes = np.bincount(level)
+    print("level sizes (pins):", " ".join(str(x) for x in sizes))
+    t = load("fwd_trace.bin")
+    t0 = t[:, 0, 0].min()
+    end_max = (t[..., 2] - t0).max(axis=0)
+    inc = np.diff(np.concatenate([[0], end_max]))
+    print("fwd step increments (us):", " ".join(f"{x/1e3:.1f}" for x in inc))
+
+# per-step spread of item completion (relative to the previous step's last end)
+if os.environ.get("SPREAD"):
+    for name in ("fwd_trace.bin", "bwd_trace.bin"):
+        t = load(name)
+        t0 = t[:, 0, 0].min()
+        st, en = t[..., 0] - t0, t[..., 2] - t0
+        prev = 0
+        print("==", name)
+        lo, hi = (int(x) for x in os.environ["SPREAD"].split(":"))
+        for s in range(t.shape[1]):
+            a, b = st[:, s], en[:, s]
+            ok = b > 0
+            a, b = a[ok], b[ok]
+            if a.size and lo <= s < hi:
+                print(f"step {s:3d}: n={a.size:3d} start rel [min {(a.min()-prev)/1e3:6.2f} med {(np.median(a)-prev)/1e3:6.2f}]"
+                      f" end rel [min {(b.min()-prev)/1e3:6.2f} med {(np.median(b)-prev)/1e3:6.2f} p90 {(np.percentile(b,90)-prev)/1e3:6.2f} max {(b.max()-prev)/1e3:6.2f}]"
+                      f" dur med {np.median(b-a)/1e3:5.2f}")
+            if a.size:
+                prev = b.max()
