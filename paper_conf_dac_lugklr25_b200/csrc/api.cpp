@@ -49,7 +49,7 @@ void free_graph(insta::DevGraph& d) {
                   d.lfo,       d.fanout_ptr, d.fout_sink, d.heavy_slot, d.heavy_acc, d.arc_pos,
                   d.heavy_cnt, d.heavy_fo,
                   d.arc_sink,  d.order,     d.src_ms,    d.ep_pin,     d.ep_rat,    d.arc_class,
-                  d.fwd_a,     d.fwd_b,     d.bwd_a,     d.bwd_b,      d.done_fwd,  d.done_bwd,
+                  d.fwd_a,     d.fwd_b,     d.bfwd_a,    d.bfwd_b,     d.bwd_a,     d.bwd_b,      d.done_fwd,  d.done_bwd,
                   d.state,     d.win,       d.wts,       d.g,          d.seed,      d.slack,
                   d.rf_star,   d.partials,  d.ticket,    d.summary,    d.dirty,     d.counters,
                   d.fin_flags, d.ep_of_pin, d.b_state,   d.b_win,      d.b_wts,     d.b_g,
@@ -266,6 +266,8 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   UP(d.max_sink_level, max_sink_level.data(), nN);
   UP(d.fwd_a, d.fwd_items.a.data(), d.fwd_items.a.size());
   UP(d.fwd_b, d.fwd_items.b.data(), d.fwd_items.b.size());
+  UP(d.bfwd_a, d.bfwd_items.a.data(), d.bfwd_items.a.size());
+  UP(d.bfwd_b, d.bfwd_items.b.data(), d.bfwd_items.b.size());
   UP(d.bwd_a, d.bwd_items.a.data(), d.bwd_items.a.size());
   UP(d.bwd_b, d.bwd_items.b.data(), d.bwd_items.b.size());
   ZERO(d.done_fwd, std::max(d.num_levels, 1));

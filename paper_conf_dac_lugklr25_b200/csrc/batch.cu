@@ -103,10 +103,10 @@ __device__ __forceinline__ void storeb(const BParams& P, int i, int s, double m0
 
 // ---------------------------------------------------------------- forward
 struct BFwdStage {
-  int32_t ptr[kFwdPins + 8];
-  int32_t src[kFwdArcs + 8];
-  uint8_t flags[kFwdArcs + 32];
-  float4 ms[kFwdArcs];
+  int32_t ptr[kBFwdPins + 8];
+  int32_t src[kBFwdArcs + 8];
+  uint8_t flags[kBFwdArcs + 32];
+  float4 ms[kBFwdArcs];
 };
 constexpr size_t kBFwdSmem = 2 * sizeof(BFwdStage);
 
@@ -558,8 +558,8 @@ static BParams make_bparams(DevGraph& g, bool bwd) {
   P.n = g.n;
   P.num_levels = g.num_levels;
   P.grid = g.grid;
-  P.item_a = bwd ? g.bwd_a : g.fwd_a;
-  P.item_b = bwd ? g.bwd_b : g.fwd_b;
+  P.item_a = bwd ? g.bwd_a : g.bfwd_a;
+  P.item_b = bwd ? g.bwd_b : g.bfwd_b;
   P.fanin_ptr = g.fanin_ptr;
   P.fin_src = g.fin_src;
   P.fin_ms = g.fin_ms;
@@ -620,7 +620,7 @@ int launch_forward_batch(DevGraph& g, int nb, const float* sc_host /*[3][32]*/, 
   P.inv_tau = lse ? 1.0 / double(tau) : 0.0;
   P.par = (++g.pass_bfwd) & 1u;
   P.step_begin = 0;
-  P.step_end = g.fwd_items.num_steps;
+  P.step_end = g.bfwd_items.num_steps;
   if (g.n > 0) {
     void* args[] = {&P};
     e = cudaLaunchCooperativeKernel(lse ? (const void*)fwdb_kernel<true> : (const void*)fwdb_kernel<false>,

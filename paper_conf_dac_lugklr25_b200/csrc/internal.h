@@ -42,6 +42,7 @@ constexpr int kHeavyFanout = 256;
 // (per item; two stages are double-buffered)
 constexpr int kThreads = 1024;
 constexpr int kFwdPins = 1024, kFwdArcs = 1024;                     // forward item caps
+constexpr int kBFwdPins = 2048, kBFwdArcs = 2048;                  // batched forward item caps
 constexpr int kBwdPins = 2048, kBwdFanout = 2048, kBwdArcs = 2048;  // backward item caps
 static_assert(kHeavyFanout <= kBwdFanout, "a light pin's fanout row must fit one item");
 
@@ -132,9 +133,11 @@ struct DevGraph {
   // item tables
   int4* fwd_a = nullptr;
   int4* fwd_b = nullptr;
+  int4* bfwd_a = nullptr;
+  int4* bfwd_b = nullptr;
   int4* bwd_a = nullptr;
   int4* bwd_b = nullptr;
-  ItemTable fwd_items, bwd_items;
+  ItemTable fwd_items, bwd_items, bfwd_items;   // bfwd: batched forward (larger caps)
   uint32_t* done_fwd = nullptr;    // [L] level completion counters (forward)
   uint32_t* done_bwd = nullptr;    // [L] level completion counters (backward)
   // state

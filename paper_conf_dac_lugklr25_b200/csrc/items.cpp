@@ -40,13 +40,14 @@ void build_items(DevGraph& d, const std::vector<int32_t>& lfo_ptr) {
   const HostLevels& h = d.host;
   const int G = d.grid;
   const int L = h.num_levels;
-  for (int pass = 0; pass < 2; ++pass) {
+  for (int pass = 0; pass < 3; ++pass) {   // forward, backward, batched forward
     const bool bwd = pass == 1;
-    ItemTable& T = bwd ? d.bwd_items : d.fwd_items;
+    ItemTable& T = pass == 0 ? d.fwd_items : (bwd ? d.bwd_items : d.bfwd_items);
     T = ItemTable();
     T.level_step0.assign(size_t(L), 0);
     T.level_steps.assign(size_t(L), 0);
-    const Caps caps = bwd ? Caps{kBwdPins, kBwdArcs, kBwdFanout} : Caps{kFwdPins, kFwdArcs, 1 << 30};
+    const Caps caps = bwd ? Caps{kBwdPins, kBwdArcs, kBwdFanout}
+                          : (pass == 0 ? Caps{kFwdPins, kFwdArcs, 1 << 30} : Caps{kBFwdPins, kBFwdArcs, 1 << 30});
     std::vector<int64_t> prefix;
     std::vector<int32_t> cuts;
     for (int li = 0; li < L; ++li) {
