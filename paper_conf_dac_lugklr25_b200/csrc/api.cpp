@@ -4,6 +4,8 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -54,7 +56,11 @@ void free_graph(insta::DevGraph& d) {
                   d.rf_star,   d.partials,  d.ticket,    d.summary,    d.dirty,     d.counters,
                   d.fin_flags, d.ep_of_pin, d.b_state,   d.b_win,      d.b_wts,     d.b_g,
                   d.b_heavy,   d.b_sc,      d.b_ov_ptr,  d.b_ov_pos,   d.b_ov_ms,   d.b_slack,
-                  d.b_rf,      d.b_partials, d.b_ticket,  d.pin_level,  d.lvl_range, d.max_sink_level};
+                  d.b_rf,      d.b_partials, d.b_ticket,  d.pin_level,  d.lvl_range, d.max_sink_level,
+                  d.hd_pin,    d.hd_ptr,    d.hd_q0,     d.ext_w,      d.ext_ms,    d.ext_f,
+                  d.ext_fms,   d.ext_fq,    d.arc_xpos,  d.fwdf_a,     d.fwdf_b,    d.hd_hslot,
+                  d.hlfo_ptr,  d.hlfo,      d.ext_qpos,  d.ext_bw,     d.ext_arc,   d.ext_farc,
+                  d.ep_head,   d.hseed,     d.bwdf_a,    d.bwdf_b};
   for (void* p : ptrs)
     if (p) cudaFree(p);
 }
@@ -230,11 +236,22 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   std::vector<int32_t> ep_of_pin(nN, -1);
   for (int32_t k = 0; k < d.num_ep; ++k) ep_of_pin[ep_pin[k]] = k;
   d.h_arc_pos = arc_pos;
+  insta::FoldHost fold;
+  insta::build_fold(h, fin_src, fin_ms, ep_of_pin, lfo_ptr, lfo, heavy_slot, &fold);
+  d.num_heads = int32_t(fold.hd_pin.size());
+  d.num_slevels = int32_t(fold.slevel_ptr.size()) - 1;
+  d.num_ext = int64_t(fold.ext_w.size());
 
   // ---- device: grid, items, upload ------------------------------------------------
   cudaError_t e = cudaSetDevice(d.device);
   if (e == cudaSuccess) e = static_cast<cudaError_t>(insta::query_grid(d.device, &d.grid));
   if (e == cudaSuccess) insta::build_items(d, lfo_ptr);
+  if (e == cudaSuccess) insta::build_fold_items(d, fold);
+  if (getenv("INSTA_DEBUG"))
+    fprintf(stderr, "[insta] pins %d arcs %lld levels %d | folded %lld heads %d super-levels %d | steps: fwd %d "
+            "folded fwd %d bwd %d folded bwd %d batched fwd %d\n", n, (long long)E, h.num_levels,
+            (long long)(n - d.num_heads), d.num_heads, d.num_slevels, d.fwd_items.num_steps,
+            d.fwdf_items.num_steps, d.bwd_items.num_steps, d.bwdf_items.num_steps, d.bfwd_items.num_steps);
 #define UP(dst, src, cnt)                       \
   if (e == cudaSuccess) e = upload(&(dst), (src), size_t(cnt));
 #define ZERO(dst, cnt) \
@@ -270,6 +287,28 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   UP(d.bfwd_b, d.bfwd_items.b.data(), d.bfwd_items.b.size());
   UP(d.bwd_a, d.bwd_items.a.data(), d.bwd_items.a.size());
   UP(d.bwd_b, d.bwd_items.b.data(), d.bwd_items.b.size());
+  UP(d.hd_pin, fold.hd_pin.data(), fold.hd_pin.size());
+  UP(d.hd_ptr, fold.hd_ptr.data(), fold.hd_ptr.size());
+  UP(d.hd_q0, fold.hd_q0.data(), fold.hd_q0.size());
+  UP(d.ext_w, fold.ext_w.data(), fold.ext_w.size());
+  UP(d.ext_ms, fold.ext_ms.data(), fold.ext_ms.size());
+  UP(d.ext_f, fold.ext_f.data(), fold.ext_f.size());
+  UP(d.ext_fms, fold.ext_fms.data(), fold.ext_fms.size());
+  UP(d.ext_fq, fold.ext_fq.data(), fold.ext_fq.size());
+  UP(d.arc_xpos, fold.arc_xpos.data(), fold.arc_xpos.size());
+  UP(d.fwdf_a, d.fwdf_items.a.data(), d.fwdf_items.a.size());
+  UP(d.fwdf_b, d.fwdf_items.b.data(), d.fwdf_items.b.size());
+  UP(d.hd_hslot, fold.hd_hslot.data(), fold.hd_hslot.size());
+  UP(d.hlfo_ptr, fold.hlfo_ptr.data(), fold.hlfo_ptr.size());
+  UP(d.hlfo, fold.hlfo.data(), fold.hlfo.size());
+  UP(d.ext_qpos, fold.ext_qpos.data(), fold.ext_qpos.size());
+  UP(d.ext_bw, fold.ext_bw.data(), fold.ext_bw.size());
+  UP(d.ext_arc, fold.ext_arc.data(), fold.ext_arc.size());
+  UP(d.ext_farc, fold.ext_farc.data(), fold.ext_farc.size());
+  UP(d.ep_head, fold.ep_head.data(), fold.ep_head.size());
+  ZERO(d.hseed, fold.hd_pin.size());
+  UP(d.bwdf_a, d.bwdf_items.a.data(), d.bwdf_items.a.size());
+  UP(d.bwdf_b, d.bwdf_items.b.data(), d.bwdf_items.b.size());
   ZERO(d.done_fwd, std::max(d.num_levels, 1));
   ZERO(d.done_bwd, std::max(d.num_levels, 1));
   ZERO(d.state, nN);

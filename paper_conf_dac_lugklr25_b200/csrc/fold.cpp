@@ -1,0 +1,126 @@
+// fold.cpp -- host construction of the stage-folded schedule of the persistent
+// forward (DESIGN.md §4 "stage folding").
+//
+// A pin p with exactly one fanin arc e' = (j -> p) and exactly one fanout arc
+// e = (p -> q) that is not an endpoint -- in a netlist, a cell input pin -- is
+// "folded": its arrival (a merge of the candidates of e' alone, Alg 1 with one
+// fanin) is computed inside the item of its sink q, in registers, right before
+// q's candidates over e are formed.  p is still written to the state arrays, so
+// every consumer of the per-pin state (slack, backward, incremental pass,
+// arrivals) sees exactly what the per-level schedule writes; the arithmetic per
+// pin is the same device code, so the results are bit-identical.  What changes
+// is the dependency depth: q waits for j, not for p, so a (net arc, cell arc)
+// pair costs one level-to-level step instead of two (162 -> ~82 steps at C4).
+//
+// Rule (canonical order): p is folded iff indeg(p) = 1, outdeg(p) = 1, p is
+// not an endpoint, and the source j of its fanin arc is not folded.  Then the
+// sink q of p is never folded either (its fanin source p is), so folding never
+// nests.  Every other pin is a "head".  Heads are scheduled by super-level:
+// slevel = 0 for indeg-0 pins, else 1 + max over its fanin arcs (p -> q) of
+// slevel(p) (p a head) or slevel(j) (p folded, j its source); heads are
+// ordered by (slevel, canonical position), so the startpoints keep positions
+// 0..num_src-1.
+#include <algorithm>
+
+#include <vector_functions.h>
+
+#include "internal.h"
+
+namespace insta {
+
+void build_fold(const HostLevels& h, const std::vector<int32_t>& fin_src, const std::vector<float4>& fin_ms,
+                const std::vector<int32_t>& ep_of_pin, const std::vector<int32_t>& lfo_ptr,
+                const std::vector<int32_t>& lfo, const std::vector<int32_t>& heavy_slot, FoldHost* out) {
+  FoldHost& f = *out;
+  f = FoldHost();
+  const int32_t n = h.n;
+  const auto& fp = h.fanin_ptr;
+  const auto& op = h.fanout_ptr;
+  f.folded.assign(size_t(n), 0);
+  for (int32_t p = 0; p < n; ++p) {
+    if (fp[p + 1] - fp[p] != 1 || op[p + 1] - op[p] != 1 || ep_of_pin[p] >= 0) continue;
+    const int32_t j = fin_src[fp[p]] & kSrcMask;
+    if (!f.folded[j]) f.folded[p] = 1;
+  }
+  // super-levels of heads (canonical order is topological)
+  std::vector<int32_t> sl(size_t(n), 0);
+  int32_t max_sl = 0;
+  for (int32_t q = 0; q < n; ++q) {
+    if (f.folded[q] || fp[q + 1] == fp[q]) continue;
+    int32_t s = 0;
+    for (int32_t x = fp[q]; x < fp[q + 1]; ++x) {
+      int32_t p = fin_src[x] & kSrcMask;
+      if (f.folded[p]) p = fin_src[fp[p]] & kSrcMask;
+      s = std::max(s, sl[p] + 1);
+    }
+    sl[q] = s;
+    max_sl = std::max(max_sl, s);
+  }
+  const int32_t SL = n > 0 ? max_sl + 1 : 0;
+  f.slevel_ptr.assign(size_t(SL) + 1, 0);
+  for (int32_t q = 0; q < n; ++q)
+    if (!f.folded[q]) ++f.slevel_ptr[sl[q] + 1];
+  for (int32_t s = 0; s < SL; ++s) f.slevel_ptr[s + 1] += f.slevel_ptr[s];
+  const int32_t H = SL > 0 ? f.slevel_ptr[SL] : 0;
+  f.hd_pin.assign(size_t(H), 0);
+  {
+    std::vector<int32_t> fill(f.slevel_ptr.begin(), f.slevel_ptr.end() - (SL > 0 ? 1 : 0));
+    for (int32_t q = 0; q < n; ++q)
+      if (!f.folded[q]) f.hd_pin[fill[sl[q]]++] = q;
+  }
+  // entries: one per fanin arc of a head, in fanin row order
+  f.hd_ptr.assign(size_t(H) + 1, 0);
+  f.hd_q0.assign(size_t(H), 0);
+  f.hd_nfold.assign(size_t(H), 0);
+  const int64_t X = h.e - std::count(f.folded.begin(), f.folded.end(), uint8_t(1));
+  f.ext_w.assign(size_t(X), 0);
+  f.ext_f.assign(size_t(X), 0);
+  f.ext_fq.assign(size_t(X), -1);
+  f.ext_ms.assign(size_t(X), make_float4(0.f, 0.f, 0.f, 0.f));
+  f.ext_fms.assign(size_t(X), make_float4(0.f, 0.f, 0.f, 0.f));
+  f.arc_xpos.assign(size_t(h.e), -1);
+  f.ext_qpos.assign(size_t(X), 0);
+  f.ext_bw.assign(size_t(X), 0);
+  f.ext_arc.assign(size_t(X), 0);
+  f.ext_farc.assign(size_t(X), -1);
+  f.hd_hslot.assign(size_t(H), -1);
+  f.hlfo_ptr.assign(size_t(H) + 1, 0);
+  f.hlfo.clear();
+  f.ep_head.assign(size_t(std::count_if(ep_of_pin.begin(), ep_of_pin.end(), [](int32_t v) { return v >= 0; })), -1);
+  int64_t x = 0;
+  for (int32_t hh = 0; hh < H; ++hh) {
+    const int32_t q = f.hd_pin[hh];
+    f.hd_q0[hh] = fp[q];
+    f.hd_hslot[hh] = heavy_slot[q];
+    if (ep_of_pin[q] >= 0) f.ep_head[ep_of_pin[q]] = hh;
+    for (int32_t r = lfo_ptr[q]; r < lfo_ptr[q + 1]; ++r) f.hlfo.push_back(lfo[r]);
+    f.hlfo_ptr[hh + 1] = int32_t(f.hlfo.size());
+    for (int32_t y = fp[q]; y < fp[q + 1]; ++y, ++x) {
+      const int32_t p = fin_src[y] & kSrcMask;
+      const int32_t u = int32_t(uint32_t(fin_src[y]) >> kUnateShift);
+      f.ext_ms[x] = fin_ms[y];
+      f.arc_xpos[h.fanin_arc[y]] = int32_t(2 * x);
+      f.ext_qpos[x] = y;
+      f.ext_arc[x] = h.fanin_arc[y];
+      f.ext_bw[x] = fin_src[y];
+      if (f.folded[p]) {
+        const int32_t y2 = fp[p];
+        const int32_t j = fin_src[y2] & kSrcMask;
+        const int32_t u2 = int32_t(uint32_t(fin_src[y2]) >> kUnateShift);
+        f.ext_w[x] = j | (1 << kFoldBit) | int32_t(uint32_t(u) << kUnateShift);
+        f.ext_f[x] = p | int32_t(uint32_t(u2) << kUnateShift);
+        f.ext_fq[x] = y2;
+        f.ext_fms[x] = fin_ms[y2];
+        f.arc_xpos[h.fanin_arc[y2]] = int32_t(2 * x + 1);
+        f.ext_farc[x] = h.fanin_arc[y2];
+        f.ext_bw[x] = fin_src[y2];
+        ++f.hd_nfold[hh];
+      } else {
+        f.ext_w[x] = p | int32_t(uint32_t(u) << kUnateShift);
+      }
+    }
+    f.hd_ptr[hh + 1] = int32_t(x);
+  }
+}
+
+}  // namespace insta

@@ -37,6 +37,9 @@ constexpr int kHeavyBit = 29;
 constexpr int32_t kSrcMask = (1 << kHeavyBit) - 1;
 constexpr int32_t kMaxPins = (1 << 29) - 1;
 constexpr int kHeavyFanout = 256;
+// ext_w word of the stage-folded schedule (fold.cpp): bit 29 "entry goes
+// through a folded pin" (the heavy bit is not needed by the forward)
+constexpr int kFoldBit = 29;
 
 // CTA shape (one 1024-thread CTA per SM) and shared-memory stage capacities
 // (per item; two stages are double-buffered)
@@ -73,6 +76,35 @@ struct HostLevels {
 // Returns INSTA_OK / INSTA_E_CYCLE / INSTA_E_ARG.
 insta_status levelize_host(int32_t n, int64_t e, const int32_t* from, const int32_t* to,
                            HostLevels* out, std::string* err);
+
+// Stage-folded forward schedule (fold.cpp).  "Heads" are the pins that are
+// not folded, in (super-level, canonical) order; entry x of head h is the
+// fanin arc e = (p -> q) of q = hd_pin[h] at row position x - hd_ptr[h]; when
+// p is folded the entry also carries p's single fanin arc e' = (j -> p) and
+// its source word names j.
+struct FoldHost {
+  std::vector<uint8_t> folded;      // [n] canonical
+  std::vector<int32_t> slevel_ptr;  // [SL+1] head ranges per super-level
+  std::vector<int32_t> hd_pin;      // [H] canonical pin of each head
+  std::vector<int32_t> hd_ptr;      // [H+1] entry rows
+  std::vector<int32_t> hd_q0;       // [H] fanin position of the head's first fanin arc
+  std::vector<int32_t> hd_nfold;    // [H] folded entries (work estimate)
+  std::vector<int32_t> ext_w;       // [X] source (j if folded, else p) | fold << 29 | unate(e) << 30
+  std::vector<float4> ext_ms;       // [X] record of e
+  std::vector<int32_t> ext_f;       // [X] folded pin p | unate(e') << 30 (folded entries)
+  std::vector<float4> ext_fms;      // [X] record of e'
+  std::vector<int32_t> ext_fq;      // [X] fanin position of e' (-1 if not folded)
+  std::vector<int32_t> arc_xpos;    // [E] caller arc -> 2x (as e) or 2x+1 (as e')
+  // backward (reverse super-level order over the same heads)
+  std::vector<int32_t> hd_hslot;    // [H] heavy accumulator slot of the head (-1: light)
+  std::vector<int32_t> hlfo_ptr;    // [H+1] light fanout rows of the heads
+  std::vector<int32_t> hlfo;        // fanin positions (adjoint words) of those rows
+  std::vector<int32_t> ext_qpos;    // [X] fanin position of e
+  std::vector<int32_t> ext_bw;      // [X] fin_src word of the arc whose adjoint the entry writes (e, or e' if folded)
+  std::vector<int32_t> ext_arc;     // [X] caller id of e
+  std::vector<int32_t> ext_farc;    // [X] caller id of e' (-1 if not folded)
+  std::vector<int32_t> ep_head;     // [P] head index of each endpoint (endpoints are never folded)
+};
 
 // Item table: step s of CTA c is entry s * G + c.
 //  forward:  a = {pin_lo, pin_hi, arc_lo, arc_hi}, b = {level, flags, 0, 0}
@@ -138,6 +170,34 @@ struct DevGraph {
   int4* bwd_a = nullptr;
   int4* bwd_b = nullptr;
   ItemTable fwd_items, bwd_items, bfwd_items;   // bfwd: batched forward (larger caps)
+  // stage-folded forward (fold.cpp)
+  int32_t num_heads = 0, num_slevels = 0;
+  int64_t num_ext = 0;
+  int32_t* hd_pin = nullptr;
+  int32_t* hd_ptr = nullptr;
+  int32_t* hd_q0 = nullptr;
+  int32_t* ext_w = nullptr;
+  float4* ext_ms = nullptr;
+  int32_t* ext_f = nullptr;
+  float4* ext_fms = nullptr;
+  int32_t* ext_fq = nullptr;
+  int32_t* arc_xpos = nullptr;
+  int4* fwdf_a = nullptr;
+  int4* fwdf_b = nullptr;
+  ItemTable fwdf_items;
+  // stage-folded backward
+  int32_t* hd_hslot = nullptr;
+  int32_t* hlfo_ptr = nullptr;
+  int32_t* hlfo = nullptr;
+  int32_t* ext_qpos = nullptr;
+  int32_t* ext_bw = nullptr;
+  int32_t* ext_arc = nullptr;
+  int32_t* ext_farc = nullptr;
+  int32_t* ep_head = nullptr;
+  float2* hseed = nullptr;         // [H] endpoint seeds in head order
+  int4* bwdf_a = nullptr;
+  int4* bwdf_b = nullptr;
+  ItemTable bwdf_items;
   uint32_t* done_fwd = nullptr;    // [L] level completion counters (forward)
   uint32_t* done_bwd = nullptr;    // [L] level completion counters (backward)
   // state
@@ -172,6 +232,11 @@ struct DevGraph {
 
 // item tables (items.cpp)
 void build_items(DevGraph& d, const std::vector<int32_t>& lfo_ptr);
+// stage folding (fold.cpp) and its item table (items.cpp)
+void build_fold(const HostLevels& h, const std::vector<int32_t>& fin_src, const std::vector<float4>& fin_ms,
+                const std::vector<int32_t>& ep_of_pin, const std::vector<int32_t>& lfo_ptr,
+                const std::vector<int32_t>& lfo, const std::vector<int32_t>& heavy_slot, FoldHost* out);
+void build_fold_items(DevGraph& d, const FoldHost& f);
 
 }  // namespace insta
 

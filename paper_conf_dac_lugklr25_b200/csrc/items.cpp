@@ -34,69 +34,108 @@ void quantile_cuts(const std::vector<int64_t>& prefix /* over [lo, hi], prefix[0
   for (int64_t j = 1; j <= n; ++j) (*cuts)[j] = std::max((*cuts)[j], (*cuts)[j - 1]);
 }
 
+// Cut every level (unit ranges [lptr[l], lptr[l+1]) of a level-ordered unit
+// array, forward or reverse level order) into rounds x G balanced chunks.
+// work(u): work of unit u; over(a, b): chunk [a, b) exceeds the stage caps;
+// emit(T, l, a, b, flags): append the item.
+template <class Work, class Over, class Emit>
+void cut_levels(ItemTable& T, int G, const std::vector<int32_t>& lptr, bool reverse, Work&& work, Over&& over,
+                Emit&& emit) {
+  const int L = int(lptr.size()) - 1;
+  T = ItemTable();
+  T.level_step0.assign(size_t(std::max(L, 0)), 0);
+  T.level_steps.assign(size_t(std::max(L, 0)), 0);
+  std::vector<int64_t> prefix;
+  std::vector<int32_t> cuts;
+  for (int li = 0; li < L; ++li) {
+    const int l = reverse ? (L - 1 - li) : li;
+    const int32_t lo = lptr[l], hi = lptr[l + 1];
+    prefix.assign(size_t(hi - lo) + 1, 0);
+    for (int32_t p = lo; p < hi; ++p) prefix[p - lo + 1] = prefix[p - lo] + work(p);
+    int64_t m = 1;
+    for (;;) {
+      quantile_cuts(prefix, lo, m * G, &cuts);
+      bool ok = true;
+      for (int64_t j = 0; j < m * G && ok; ++j) {
+        const int32_t a = cuts[j], b = cuts[j + 1];
+        if (b - a <= 1) continue;   // single units are always accepted (direct if too big)
+        if (over(a, b)) ok = false;
+      }
+      if (ok || m * G >= int64_t(hi - lo)) break;
+      m *= 2;
+    }
+    // with m*G >= units every chunk holds <= 1 unit, so the loop above terminates
+    T.level_step0[l] = T.num_steps;
+    T.level_steps[l] = int32_t(m);
+    for (int64_t r = 0; r < m; ++r) {
+      for (int c = 0; c < G; ++c) {
+        const int64_t j = r * G + c;
+        const int32_t a = cuts[j], b = cuts[j + 1];
+        int flags = (r == m - 1) ? kItemLast : 0;
+        if (b - a > 0 && over(a, b)) flags |= kItemDirect;
+        emit(T, l, a, b, flags);
+      }
+      ++T.num_steps;
+    }
+  }
+}
+
 }  // namespace
 
 void build_items(DevGraph& d, const std::vector<int32_t>& lfo_ptr) {
   const HostLevels& h = d.host;
   const int G = d.grid;
-  const int L = h.num_levels;
-  for (int pass = 0; pass < 3; ++pass) {   // forward, backward, batched forward
-    const bool bwd = pass == 1;
-    ItemTable& T = pass == 0 ? d.fwd_items : (bwd ? d.bwd_items : d.bfwd_items);
-    T = ItemTable();
-    T.level_step0.assign(size_t(L), 0);
-    T.level_steps.assign(size_t(L), 0);
-    const Caps caps = bwd ? Caps{kBwdPins, kBwdArcs, kBwdFanout}
-                          : (pass == 0 ? Caps{kFwdPins, kFwdArcs, 1 << 30} : Caps{kBFwdPins, kBFwdArcs, 1 << 30});
-    std::vector<int64_t> prefix;
-    std::vector<int32_t> cuts;
-    for (int li = 0; li < L; ++li) {
-      const int l = bwd ? (L - 1 - li) : li;
-      const int32_t lo = h.level_ptr[l], hi = h.level_ptr[l + 1];
-      prefix.assign(size_t(hi - lo) + 1, 0);
-      for (int32_t p = lo; p < hi; ++p) {
-        int64_t w = 1 + (h.fanin_ptr[p + 1] - h.fanin_ptr[p]);
-        if (bwd) w += lfo_ptr[p + 1] - lfo_ptr[p];
-        prefix[p - lo + 1] = prefix[p - lo] + w;
-      }
-      int64_t m = 1;
-      for (;;) {
-        quantile_cuts(prefix, lo, m * G, &cuts);
-        bool ok = true;
-        for (int64_t j = 0; j < m * G && ok; ++j) {
-          const int32_t a = cuts[j], b = cuts[j + 1];
-          if (b - a <= 1) continue;   // single pins are always accepted (direct if too big)
-          const int64_t arcs = h.fanin_ptr[b] - h.fanin_ptr[a];
-          const int64_t fo = bwd ? int64_t(lfo_ptr[b] - lfo_ptr[a]) : 0;
-          if (b - a > caps.pins || arcs > caps.arcs || fo > caps.fanout) ok = false;
-        }
-        if (ok || m * G >= int64_t(hi - lo)) break;
-        m *= 2;
-      }
-      // with m*G >= pins every chunk holds <= 1 pin, so the loop above terminates
-      T.level_step0[l] = T.num_steps;
-      T.level_steps[l] = int32_t(m);
-      for (int64_t r = 0; r < m; ++r) {
-        for (int c = 0; c < G; ++c) {
-          const int64_t j = r * G + c;
-          const int32_t a = cuts[j], b = cuts[j + 1];
-          const int32_t alo = h.fanin_ptr[a], ahi = h.fanin_ptr[b];
-          const int64_t arcs = ahi - alo;
-          const int64_t fo = bwd ? int64_t(lfo_ptr[b] - lfo_ptr[a]) : 0;
-          int flags = (r == m - 1) ? kItemLast : 0;
-          if (b - a > caps.pins || arcs > caps.arcs || fo > caps.fanout) flags |= kItemDirect;
-          if (!bwd) {
-            T.a.push_back(make_int4(a, b, alo, ahi));
-            T.b.push_back(make_int4(l, flags, 0, 0));
-          } else {
-            T.a.push_back(make_int4(a, b, lfo_ptr[a], lfo_ptr[b]));
-            T.b.push_back(make_int4(alo, ahi, l, flags));
-          }
-        }
-        ++T.num_steps;
-      }
-    }
+  const auto& fp = h.fanin_ptr;
+  // forward and batched forward: work = 1 + fanin arcs
+  for (int pass = 0; pass < 2; ++pass) {
+    const Caps caps = pass == 0 ? Caps{kFwdPins, kFwdArcs, 0} : Caps{kBFwdPins, kBFwdArcs, 0};
+    cut_levels(
+        pass == 0 ? d.fwd_items : d.bfwd_items, G, h.level_ptr, false,
+        [&](int32_t p) { return int64_t(1) + (fp[p + 1] - fp[p]); },
+        [&](int32_t a, int32_t b) { return b - a > caps.pins || fp[b] - fp[a] > caps.arcs; },
+        [&](ItemTable& T, int l, int32_t a, int32_t b, int flags) {
+          T.a.push_back(make_int4(a, b, fp[a], fp[b]));
+          T.b.push_back(make_int4(l, flags, 0, 0));
+        });
   }
+  // backward: work = 1 + fanin arcs + light fanout entries, reverse level order
+  cut_levels(
+      d.bwd_items, G, h.level_ptr, true,
+      [&](int32_t p) { return int64_t(1) + (fp[p + 1] - fp[p]) + (lfo_ptr[p + 1] - lfo_ptr[p]); },
+      [&](int32_t a, int32_t b) {
+        return b - a > kBwdPins || fp[b] - fp[a] > kBwdArcs || lfo_ptr[b] - lfo_ptr[a] > kBwdFanout;
+      },
+      [&](ItemTable& T, int l, int32_t a, int32_t b, int flags) {
+        T.a.push_back(make_int4(a, b, lfo_ptr[a], lfo_ptr[b]));
+        T.b.push_back(make_int4(fp[a], fp[b], l, flags));
+      });
+}
+
+void build_fold_items(DevGraph& d, const FoldHost& f) {
+  const int G = d.grid;
+  const auto& hp = f.hd_ptr;
+  // folded forward: work of a head = 1 + entries + folded entries
+  cut_levels(
+      d.fwdf_items, G, f.slevel_ptr, false,
+      [&](int32_t h) { return int64_t(1) + (hp[h + 1] - hp[h]) + f.hd_nfold[h]; },
+      [&](int32_t a, int32_t b) { return b - a > kFwdPins || hp[b] - hp[a] > kFwdArcs; },
+      [&](ItemTable& T, int l, int32_t a, int32_t b, int flags) {
+        T.a.push_back(make_int4(a, b, hp[a], hp[b]));
+        T.b.push_back(make_int4(l, flags, 0, 0));
+      });
+  // folded backward: reverse super-level order; work = 1 + entries + folded
+  // entries + light fanout entries
+  const auto& lp = f.hlfo_ptr;
+  cut_levels(
+      d.bwdf_items, G, f.slevel_ptr, true,
+      [&](int32_t h) { return int64_t(1) + (hp[h + 1] - hp[h]) + f.hd_nfold[h] + (lp[h + 1] - lp[h]); },
+      [&](int32_t a, int32_t b) {
+        return b - a > kBwdPins || hp[b] - hp[a] > kBwdArcs || lp[b] - lp[a] > kBwdFanout;
+      },
+      [&](ItemTable& T, int l, int32_t a, int32_t b, int flags) {
+        T.a.push_back(make_int4(a, b, lp[a], lp[b]));
+        T.b.push_back(make_int4(hp[a], hp[b], l, flags));
+      });
 }
 
 }  // namespace insta

@@ -61,6 +61,20 @@ struct KParams {
   const int32_t* __restrict__ heavy_slot;
   const float4* __restrict__ src_ms;
   const int32_t* __restrict__ order;
+  // stage-folded forward (fold.cpp): canonical pin / first fanin position of
+  // each head, folded pin word and record of e', fanin position of e'
+  const int32_t* __restrict__ hd_pin;
+  const int32_t* __restrict__ hd_q0;
+  const int32_t* __restrict__ ext_f;
+  const float4* __restrict__ ext_fms;
+  const int32_t* __restrict__ ext_fq;
+  // stage-folded backward
+  const int32_t* __restrict__ hd_hslot;
+  const int32_t* __restrict__ ext_qpos;
+  const int32_t* __restrict__ ext_bw;
+  const int32_t* __restrict__ ext_arc;
+  const int32_t* __restrict__ ext_farc;
+  const float2* hseed;
   PinState* state;
   int32_t* win;
   float4* wts;
@@ -160,6 +174,12 @@ struct FwdStage {
   int32_t ptr[kFwdPins + 8];
   int32_t src[kFwdArcs + 8];
   float4 ms[kFwdArcs];
+  // stage-folded schedule only
+  int32_t pin[kFwdPins + 8];   // canonical pin of each head
+  int32_t q0[kFwdPins + 8];    // fanin position of each head's first arc
+  int32_t f[kFwdArcs + 8];     // folded pin | unate(e') << 30
+  int32_t fq[kFwdArcs + 8];    // fanin position of e'
+  float4 fms[kFwdArcs];        // record of e'
 };
 // per arc: gathered source record + corner arrivals of its candidates
 // {A[rf=R][s0], A[rf=F][s0], A[R][s1], A[F][s1]} (s1 only for non-unate arcs)
@@ -169,6 +189,7 @@ __device__ __forceinline__ bool fwd_staged(const int4& A, const int4& B) {
 }
 
 // thread 0: issue the bulk copies staging item `step` into `st`
+template <bool kFold>
 __device__ __forceinline__ void fwd_prefetch(const KParams& P, FwdStage* st, uint64_t* full, int step,
                                              int c) {
   const int4 A = __ldg(P.item_a + size_t(step) * P.grid + c);
@@ -177,19 +198,35 @@ __device__ __forceinline__ void fwd_prefetch(const KParams& P, FwdStage* st, uin
   const Window wp = window(A.x, A.y + 1, 4);
   const Window ws = window(A.z, A.w, 4);
   const uint32_t bms = uint32_t(A.w - A.z) * 16u;
+  const Window wh = window(A.x, A.y, 4);
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-  mbar_expect_tx(full, wp.bytes + ws.bytes + bms);
+  mbar_expect_tx(full, wp.bytes + ws.bytes + bms + (kFold ? 2 * wh.bytes + 2 * ws.bytes + bms : 0u));
   bulk_g2s(st->ptr, P.fanin_ptr + wp.start, wp.bytes, full);
   if (ws.bytes) bulk_g2s(st->src, P.fin_src + ws.start, ws.bytes, full);
   if (bms) bulk_g2s(st->ms, P.fin_ms + A.z, bms, full);
+  if (kFold) {
+    bulk_g2s(st->pin, P.hd_pin + wh.start, wh.bytes, full);
+    bulk_g2s(st->q0, P.hd_q0 + wh.start, wh.bytes, full);
+    if (ws.bytes) {
+      bulk_g2s(st->f, P.ext_f + ws.start, ws.bytes, full);
+      bulk_g2s(st->fq, P.ext_fq + ws.start, ws.bytes, full);
+    }
+    if (bms) bulk_g2s(st->fms, P.ext_fms + A.z, bms, full);
+  }
 }
 
-// Forward of one non-source pin by one thread (both rf).
+// Forward of one non-source pin by one thread (both rf).  Returns the words
+// it stored (parity included), which is exactly what a consumer would load.
 template <bool kLSE, class ArcFn>
-__device__ __forceinline__ void fwd_pin(const KParams& P, int i, int nf, int q0, ArcFn&& arc) {
+__device__ __forceinline__ Raw fwd_pin(const KParams& P, int i, int nf, int q0, ArcFn&& arc) {
   const RfOut R = pin_rf<kLSE>(P, 0, nf, arc);
   const RfOut F = pin_rf<kLSE>(P, 1, nf, arc);
   store_state(P, i, R.mu, F.mu, R.var, F.var);
+  Raw o;
+  o.a = (unsigned long long)__double_as_longlong(with_par(R.mu, P.par));
+  o.b = (unsigned long long)__double_as_longlong(with_par(F.mu, P.par));
+  o.c = (unsigned long long)__double_as_longlong(with_par(R.var, P.par));
+  o.d = (unsigned long long)__double_as_longlong(with_par(F.var, P.par));
   if (!kLSE) {
     P.win[i] = R.win | (F.win << 16);
   } else {
@@ -199,102 +236,80 @@ __device__ __forceinline__ void fwd_pin(const KParams& P, int i, int nf, int q0,
       P.wts[q0 + k] = make_float4(wr.x, wr.y, wf.x, wf.y);
     }
   }
-}
-
-// Forward of one pin by a lane pair: the even lane computes rf = R, the odd
-// lane rf = F (halving the dependent arithmetic per thread); the even lane
-// writes the record.  Same functions as fwd_pin, hence bit-identical.
-template <bool kLSE, class ArcFn>
-__device__ __forceinline__ void fwd_pin_pair(const KParams& P, int i, int rf, int nf, int q0, ArcFn&& arc) {
-  const unsigned pair = 3u << ((threadIdx.x & 31) & ~1);
-  const RfOut o = pin_rf<kLSE>(P, rf, nf, arc);
-  const double mu_o = __shfl_xor_sync(pair, o.mu, 1);
-  const double var_o = __shfl_xor_sync(pair, o.var, 1);
-  const int win_o = __shfl_xor_sync(pair, o.win, 1);
-  if (rf == 0) {
-    store_state(P, i, o.mu, mu_o, o.var, var_o);
-    if (!kLSE) P.win[i] = o.win | (win_o << 16);
-  }
-  if (kLSE) {
-    for (int k = 0; k < nf; ++k) {
-      const float2 w = arc_rf_weights(P, rf, k, o, arc);
-      const float wx = __shfl_xor_sync(pair, w.x, 1), wy = __shfl_xor_sync(pair, w.y, 1);
-      if (rf == 0) P.wts[q0 + k] = make_float4(w.x, w.y, wx, wy);
-    }
-  }
-}
-
-// Merge of one (pin, rf) from precomputed candidate corners (same candidate
-// order, comparisons and LSE sum as merge_rf, hence bit-identical to it).
-template <bool kLSE>
-__device__ __forceinline__ RfOut merge_rf_pre(const KParams& P, int rf, int nf, const int32_t* sw,
-                                              const float4* sm, const Raw* sg, const double4* ca) {
-  const double ns = double(P.n_sigma);
-  double best = 0.0;
-  int bk = -1, bs = 0;
-  for (int k = 0; k < nf; ++k) {
-    const int u = int(uint32_t(sw[k]) >> kUnateShift);
-    const double4 c = ca[k];
-    const double a0 = rf ? c.y : c.x;
-    if (bk < 0 || a0 > best) {   // Alg 2 l.4: replace only if strictly greater
-      best = a0;
-      bk = k;
-      bs = src_tr(rf, u, 0);
-    }
-    if (u == 2) {
-      const double a1 = rf ? c.w : c.z;
-      if (a1 > best) {
-        best = a1;
-        bk = k;
-        bs = rf ^ 1;
-      }
-    }
-  }
-  RfOut o;
-  const Cand cw = make_cand(unpack(sg[bk]), sm[bk], rf, bs, ns);   // the winner (Alg 1 l.15)
-  o.mu = cw.mu;
-  o.var = cw.var;
-  o.sig = cw.sig;
-  o.best = best;
-  o.win = bk | (bs << 15);
-  o.sum = 0.f;
-  if (kLSE) {
-    float sum = 0.f;
-    for (int k = 0; k < nf; ++k) {
-      const int u = int(uint32_t(sw[k]) >> kUnateShift);
-      const double4 c = ca[k];
-      sum += lse_w(rf ? c.y : c.x, best, P.inv_tau);
-      if (u == 2) sum += lse_w(rf ? c.w : c.z, best, P.inv_tau);
-    }
-    o.sum = sum;
-    o.mu = lse_arrival(best, double(P.tau), sum) - ns * double(o.sig);
-  }
   return o;
 }
 
+// Forward of a pin with exactly one fanin arc (w: its source word with the
+// unateness bits, ms: its record, rj: the source's words).  The same operation
+// sequence as merge_rf with nf = 1 -- scan (a0, then a1 for a non-unate arc,
+// strict ">"), winner, LSE sum 0 + w0 (+ w1), Eq 4 arrival, Eq 6 weights --
+// with each candidate evaluated once; hard mode with a unate arc has a single
+// candidate, so its corner (and square root) is not needed.  Bit-identical to
+// fwd_pin(nf = 1).  Returns the stored words.
 template <bool kLSE>
-__device__ __forceinline__ void fwd_pin_pre(const KParams& P, int i, int nf, int q0, const int32_t* sw,
-                                            const float4* sm, const Raw* sg, const double4* ca) {
-  const RfOut R = merge_rf_pre<kLSE>(P, 0, nf, sw, sm, sg, ca);
-  const RfOut F = merge_rf_pre<kLSE>(P, 1, nf, sw, sm, sg, ca);
-  store_state(P, i, R.mu, F.mu, R.var, F.var);
-  if (!kLSE) {
-    P.win[i] = R.win | (F.win << 16);
-  } else {
-    for (int k = 0; k < nf; ++k) {
-      const int u = int(uint32_t(sw[k]) >> kUnateShift);
-      const double4 c = ca[k];
-      float wt[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
-      const float invR = 1.f / R.sum, invF = 1.f / F.sum;   // as arc_weights
-      wt[0][src_tr(0, u, 0)] = lse_w(c.x, R.best, P.inv_tau) * invR;
-      wt[1][src_tr(1, u, 0)] = lse_w(c.y, F.best, P.inv_tau) * invF;
-      if (u == 2) {
-        wt[0][1] = lse_w(c.z, R.best, P.inv_tau) * invR;
-        wt[1][0] = lse_w(c.w, F.best, P.inv_tau) * invF;
+__device__ __forceinline__ Raw fwd_pin1(const KParams& P, int i, int q0, int32_t w, const float4& ms, const Raw& rj) {
+  const Gath st = unpack(rj);
+  const int u = int(uint32_t(w) >> kUnateShift);
+  const double ns = double(P.n_sigma);
+  double mu[2], var[2];
+  int win[2];
+  float wt[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
+#pragma unroll
+  for (int rf = 0; rf < 2; ++rf) {
+    const int s0 = src_tr(rf, u, 0);
+    if (!kLSE && u != 2) {
+      const double se = double(rf ? ms.w : ms.z);
+      mu[rf] = (s0 ? st.mu1 : st.mu0) + double(rf ? ms.y : ms.x);   // = make_cand(...).mu
+      var[rf] = (s0 ? st.v1 : st.v0) + se * se;                       // = make_cand(...).var
+      win[rf] = s0 << 15;
+      continue;
+    }
+    const Cand c0 = make_cand(st, ms, rf, s0, ns);
+    Cand cb = c0;
+    int bs = s0;
+    Cand c1 = c0;
+    if (u == 2) {
+      c1 = make_cand(st, ms, rf, rf ^ 1, ns);
+      if (c1.A > c0.A) {
+        cb = c1;
+        bs = rf ^ 1;
       }
-      P.wts[q0 + k] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
+    }
+    mu[rf] = cb.mu;
+    var[rf] = cb.var;
+    win[rf] = bs << 15;
+    if (kLSE) {
+      float sum = 0.f;
+      const float w0 = lse_w(c0.A, cb.A, P.inv_tau);
+      sum += w0;
+      float w1 = 0.f;
+      if (u == 2) {
+        w1 = lse_w(c1.A, cb.A, P.inv_tau);
+        sum += w1;
+      }
+      mu[rf] = lse_arrival(cb.A, double(P.tau), sum) - ns * double(cb.sig);
+      const float inv_sum = 1.f / sum;
+      wt[rf][s0] = w0 * inv_sum;
+      if (u == 2) wt[rf][rf ^ 1] = w1 * inv_sum;
     }
   }
+  store_state(P, i, mu[0], mu[1], var[0], var[1]);
+  if (!kLSE) P.win[i] = win[0] | (win[1] << 16);
+  else P.wts[q0] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
+  Raw o;
+  o.a = (unsigned long long)__double_as_longlong(with_par(mu[0], P.par));
+  o.b = (unsigned long long)__double_as_longlong(with_par(mu[1], P.par));
+  o.c = (unsigned long long)__double_as_longlong(with_par(var[0], P.par));
+  o.d = (unsigned long long)__double_as_longlong(with_par(var[1], P.par));
+  return o;
+}
+
+// Folded pin p (stage folding, fold.cpp): its single fanin arc e' = (j -> p)
+// with source words rj.  Returns p's stored words, which replace j's in the
+// gather buffer of p's sink.
+template <bool kLSE>
+__device__ __forceinline__ Raw fold_pin(const KParams& P, int32_t fw, const float4& fms, int fq, const Raw& rj) {
+  return fwd_pin1<kLSE>(P, fw & kSrcMask, fq, fw, fms, rj);
 }
 
 __device__ __forceinline__ void trace_stamp(const KParams& P, int c, int nsteps, int t, int slot) {
@@ -337,22 +352,6 @@ constexpr int kFastPins = ((kFwdPins + kWorkerWarps - 1) / kWorkerWarps + 31) / 
 // canonical order of merge_rf (arc by arc, s = rf then ~rf), every lane then
 // writes its arc's weights.  Same make_cand / lse_w / lse_arrival
 // arithmetic as merge_rf, hence bit-identical to the other paths.
-struct Best {
-  double A, mu, var;
-  float sig;
-  int idx;   // k | s << 15
-};
-
-__device__ __forceinline__ Best shfl_down_best(const Best& b, int d) {
-  Best o;
-  o.A = __shfl_down_sync(0xffffffffu, b.A, d);
-  o.mu = __shfl_down_sync(0xffffffffu, b.mu, d);
-  o.var = __shfl_down_sync(0xffffffffu, b.var, d);
-  o.sig = __shfl_down_sync(0xffffffffu, b.sig, d);
-  o.idx = __shfl_down_sync(0xffffffffu, b.idx, d);
-  return o;
-}
-
 // Round layout (shared-memory topology only, so it is formed before the
 // gathers land): pins [q, q + cnt) with their arcs [base, base + na) one per
 // lane; heads = bit of each pin's first arc.
@@ -387,11 +386,17 @@ __device__ __forceinline__ Round round_at(const FwdStage& S, const int4& A, int 
 }
 
 // NR independent rounds per warp at once (their dependent chains interleave).
-template <bool kLSE, int NR>
-__device__ __forceinline__ void fwd_rounds(const KParams& P, const Raw* gath, const int4& A, const Round* R,
-                                           int lane) {
+// The segmented arg-max moves only (corner A, candidate index) through the
+// shuffle tree; the head lane then fetches the winner's (mu, var, sigma) from
+// the winning lane, which kept its own best candidate per rf.
+template <bool kLSE, bool kFold, int NR>
+__device__ __forceinline__ void fwd_rounds(const KParams& P, const Raw* gath, const int4& A, const FwdStage& S,
+                                           int po, const Round* R, int lane) {
   const double ns = double(P.n_sigma);
-  Best b[NR][2];
+  double bA[NR][2];                  // reduced corner
+  int bi[NR][2];                     // reduced candidate index k | s << 15
+  double om[NR][2], ov[NR][2];       // this lane's best candidate (mu, var) per rf
+  float osg[NR][2];                  // and its sigma
   double A0[NR][2], A1[NR][2];
   int u[NR], k[NR];
   bool act[NR];
@@ -401,8 +406,12 @@ __device__ __forceinline__ void fwd_rounds(const KParams& P, const Raw* gath, co
     act[r] = lane < R[r].na;
     k[r] = lane - R[r].seg;
     u[r] = 0;
-    A0[r][0] = A0[r][1] = A1[r][0] = A1[r][1] = 0.0;
-    b[r][0] = b[r][1] = Best{0.0, 0.0, 0.0, 0.f, 0};
+#pragma unroll
+    for (int rf = 0; rf < 2; ++rf) {
+      A0[r][rf] = A1[r][rf] = bA[r][rf] = om[r][rf] = ov[r][rf] = 0.0;
+      osg[r][rf] = 0.f;
+      bi[r][rf] = 0;
+    }
     if (act[r]) {
       u[r] = int(uint32_t(R[r].w) >> kUnateShift);
       const Gath st = unpack(gath[R[r].base + lane]);
@@ -411,11 +420,21 @@ __device__ __forceinline__ void fwd_rounds(const KParams& P, const Raw* gath, co
         const int s0 = src_tr(rf, u[r], 0);
         const Cand c0 = make_cand(st, R[r].ms, rf, s0, ns);
         A0[r][rf] = c0.A;
-        b[r][rf] = Best{c0.A, c0.mu, c0.var, c0.sig, k[r] | (s0 << 15)};
+        bA[r][rf] = c0.A;
+        bi[r][rf] = k[r] | (s0 << 15);
+        om[r][rf] = c0.mu;
+        ov[r][rf] = c0.var;
+        osg[r][rf] = c0.sig;
         if (u[r] == 2) {
           const Cand c1 = make_cand(st, R[r].ms, rf, rf ^ 1, ns);
           A1[r][rf] = c1.A;
-          if (c1.A > c0.A) b[r][rf] = Best{c1.A, c1.mu, c1.var, c1.sig, k[r] | ((rf ^ 1) << 15)};
+          if (c1.A > c0.A) {   // strict: s = rf wins ties (merge_rf order)
+            bA[r][rf] = c1.A;
+            bi[r][rf] = k[r] | ((rf ^ 1) << 15);
+            om[r][rf] = c1.mu;
+            ov[r][rf] = c1.var;
+            osg[r][rf] = c1.sig;
+          }
         }
       }
     }
@@ -427,25 +446,41 @@ __device__ __forceinline__ void fwd_rounds(const KParams& P, const Raw* gath, co
     for (int r = 0; r < NR; ++r) {
 #pragma unroll
       for (int rf = 0; rf < 2; ++rf) {
-        const Best o = shfl_down_best(b[r][rf], d);
-        if ((k[r] & (2 * d - 1)) == 0 && lane + d < R[r].seg_end && o.A > b[r][rf].A) b[r][rf] = o;
+        const double oA = __shfl_down_sync(0xffffffffu, bA[r][rf], d);
+        const int oi = __shfl_down_sync(0xffffffffu, bi[r][rf], d);
+        // the upper half replaces the lower only if strictly greater (Alg 2 l.4)
+        if ((k[r] & (2 * d - 1)) == 0 && lane + d < R[r].seg_end && oA > bA[r][rf]) {
+          bA[r][rf] = oA;
+          bi[r][rf] = oi;
+        }
       }
     }
   }
 #pragma unroll
   for (int r = 0; r < NR; ++r) {
-    const int i = A.x + R[r].q + __popc(R[r].heads & ((1u << lane) - 1u));   // my pin (head lanes)
+    const bool head = act[r] && k[r] == 0;
+    const int hq = R[r].q + __popc(R[r].heads & ((1u << lane) - 1u));   // my pin within the item (head lanes)
+    const int i = kFold ? S.pin[po + min(hq, A.y - A.x - 1)] : A.x + hq;
+    double wm[2], wv[2];
+    float wsg[2];
+#pragma unroll
+    for (int rf = 0; rf < 2; ++rf) {   // the winner's distribution, from the winning lane
+      const int src = head ? R[r].seg + (bi[r][rf] & 0x7fff) : lane;
+      wm[rf] = __shfl_sync(0xffffffffu, om[r][rf], src);
+      wv[rf] = __shfl_sync(0xffffffffu, ov[r][rf], src);
+      wsg[rf] = kLSE ? __shfl_sync(0xffffffffu, osg[r][rf], src) : 0.f;
+    }
     if (!kLSE) {
-      if (act[r] && k[r] == 0) {
-        store_state(P, i, b[r][0].mu, b[r][1].mu, b[r][0].var, b[r][1].var);
-        P.win[i] = b[r][0].idx | (b[r][1].idx << 16);
+      if (head) {
+        store_state(P, i, wm[0], wm[1], wv[0], wv[1]);
+        P.win[i] = bi[r][0] | (bi[r][1] << 16);
       }
     } else {
       const int src_lane = act[r] ? R[r].seg : lane;
       float w0[2], w1[2], inv[2];
 #pragma unroll
       for (int rf = 0; rf < 2; ++rf) {
-        const double best = __shfl_sync(0xffffffffu, b[r][rf].A, src_lane);   // M of my pin
+        const double best = __shfl_sync(0xffffffffu, bA[r][rf], src_lane);   // M of my pin
         w0[rf] = act[r] ? lse_w(A0[r][rf], best, P.inv_tau) : 0.f;
         w1[rf] = act[r] && u[r] == 2 ? lse_w(A1[r][rf], best, P.inv_tau) : 0.f;
         // normalizer in merge_rf's order, accumulated by the pin's first lane
@@ -458,11 +493,10 @@ __device__ __forceinline__ void fwd_rounds(const KParams& P, const Raw* gath, co
             acc += v1;   // 0 for non-NON arcs: exact no-op on a non-negative sum
           }
         }
-        if (act[r] && k[r] == 0)
-          b[r][rf].mu = lse_arrival(b[r][rf].A, double(P.tau), acc) - ns * double(b[r][rf].sig);   // Eq 4, R1
-        inv[rf] = 1.f / __shfl_sync(0xffffffffu, acc, src_lane);   // as merge_rf_pre / arc_weights
+        if (head) wm[rf] = lse_arrival(bA[r][rf], double(P.tau), acc) - ns * double(wsg[rf]);   // Eq 4, R1
+        inv[rf] = 1.f / __shfl_sync(0xffffffffu, acc, src_lane);   // as arc_weights
       }
-      if (act[r] && k[r] == 0) store_state(P, i, b[r][0].mu, b[r][1].mu, b[r][0].var, b[r][1].var);
+      if (head) store_state(P, i, wm[0], wm[1], wv[0], wv[1]);
       if (act[r]) {
         float wt[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
 #pragma unroll
@@ -470,13 +504,19 @@ __device__ __forceinline__ void fwd_rounds(const KParams& P, const Raw* gath, co
           wt[rf][src_tr(rf, u[r], 0)] = w0[rf] * inv[rf];
           if (u[r] == 2) wt[rf][rf ^ 1] = w1[rf] * inv[rf];
         }
-        P.wts[A.z + R[r].base + lane] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
+        // fanin position of my arc: row start of my pin + k
+        const int qpos = kFold ? S.q0[po + R[r].q + __popc(R[r].heads & ((2u << lane) - 1u)) - 1] + k[r]
+                               : A.z + R[r].base + lane;
+        P.wts[qpos] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
       }
     }
   }
 }
 
-template <bool kLSE>
+// kFold: the stage-folded schedule (fold.cpp): items are head ranges, entries
+// through a folded pin first compute that pin from the gathered source words
+// (fold_pin) and continue with its words in place of the source's.
+template <bool kLSE, bool kFold>
 __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
   extern __shared__ __align__(128) unsigned char smem[];
   FwdStage* stage = reinterpret_cast<FwdStage*>(smem);
@@ -502,7 +542,7 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
         const int k = P.step_begin + t;
         const int4 A = __ldg(P.item_a + size_t(k) * P.grid + c);
         const int4 B = __ldg(P.item_b + size_t(k) * P.grid + c);
-        if (fwd_staged(A, B)) fwd_prefetch(P, &stage[s], &full[s], k, c);
+        if (fwd_staged(A, B)) fwd_prefetch<kFold>(P, &stage[s], &full[s], k, c);
         else mbar_arrive1(&full[s]);
       }
     }
@@ -549,12 +589,8 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
               const int32_t w = S.src[so + a];
               const float4 ms = S.ms[a];
               await_raw(P, w & kSrcMask, r[x]);
-              const Raw rx = r[x];
-              fwd_pin<kLSE>(P, A.x + p, 1, A.z + a, [&](int, int32_t& w_, float4& ms_, Raw& r_) {
-                w_ = w;
-                ms_ = ms;
-                r_ = rx;
-              });
+              if (kFold && ((w >> kFoldBit) & 1)) r[x] = fold_pin<kLSE>(P, S.f[so + a], S.fms[a], S.fq[so + a], r[x]);
+              fwd_pin1<kLSE>(P, kFold ? S.pin[po + p] : A.x + p, kFold ? S.q0[po + p] : A.z + a, w, ms, r[x]);
             }
           }
         } else if (q1 > q0) {
@@ -580,6 +616,11 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
               }
             }
           }
+          if (kFold) {   // entries through folded pins: compute the folded pin first
+            for (int a = a_lo + lane; a < a_hi; a += 32) {
+              if ((S.src[so + a] >> kFoldBit) & 1) gath[a] = fold_pin<kLSE>(P, S.f[so + a], S.fms[a], S.fq[so + a], gath[a]);
+            }
+          }
           __syncwarp();
           if (P.trace && wt == 0) P.trace[(size_t(c) * nsteps + t) * 4 + 3] = gtimer();
           // (2) rounds of consecutive pins holding <= 32 arcs: one arc per
@@ -589,7 +630,8 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
               const int q = R.q, base = R.base;
               if (lane == 0) {
                 const int nf = S.ptr[po + q + 1] - A.z - base;
-                fwd_pin<kLSE>(P, A.x + q, nf, A.z + base, [&](int kk, int32_t& w_, float4& ms_, Raw& r_) {
+                fwd_pin<kLSE>(P, kFold ? S.pin[po + q] : A.x + q, nf, kFold ? S.q0[po + q] : A.z + base,
+                              [&](int kk, int32_t& w_, float4& ms_, Raw& r_) {
                   w_ = S.src[so + base + kk];
                   ms_ = S.ms[base + kk];
                   r_ = gath[base + kk];
@@ -611,21 +653,25 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
               }
               qn += RR[r].cnt;
             }
-            fwd_rounds<kLSE, kRoundsPerPass>(P, gath, A, RR, lane);
+            fwd_rounds<kLSE, kFold, kRoundsPerPass>(P, gath, A, S, po, RR, lane);
             if (qn < q1) R = round_at(S, A, po, so, qn, q1, lane);
             else break;
           }
         }
       } else {
-        for (int i = A.x + wt; i < A.y; i += kWorkers) {
-          const int b0 = __ldg(P.fanin_ptr + i);
-          const int nf = __ldg(P.fanin_ptr + i + 1) - b0;
-          fwd_pin<kLSE>(P, i, nf, b0, [&](int kk, int32_t& w, float4& ms, Raw& rr) {
-            w = __ldg(P.fin_src + b0 + kk);
-            ms = __ldg(P.fin_ms + b0 + kk);
-            rr = ld_state_raw(P, w & kSrcMask);
-            await_raw(P, w & kSrcMask, rr);
-          });
+        for (int h = A.x + wt; h < A.y; h += kWorkers) {
+          const int b0 = __ldg(P.fanin_ptr + h);
+          const int nf = __ldg(P.fanin_ptr + h + 1) - b0;
+          fwd_pin<kLSE>(P, kFold ? __ldg(P.hd_pin + h) : h, nf, kFold ? __ldg(P.hd_q0 + h) : b0,
+                        [&](int kk, int32_t& w, float4& ms, Raw& rr) {
+                          w = __ldg(P.fin_src + b0 + kk);
+                          ms = __ldg(P.fin_ms + b0 + kk);
+                          rr = ld_state_raw(P, w & kSrcMask);
+                          await_raw(P, w & kSrcMask, rr);
+                          if (kFold && ((w >> kFoldBit) & 1))   // recomputed per call: same words
+                            rr = fold_pin<kLSE>(P, __ldg(P.ext_f + b0 + kk), __ldg(P.ext_fms + b0 + kk),
+                                                __ldg(P.ext_fq + b0 + kk), rr);
+                        });
         }
       }
     }
@@ -936,16 +982,279 @@ __global__ void __launch_bounds__(kThreads, 1) bwd_kernel(KParams P) {
   }
 }
 
+// --------------------------------------------------------------------------
+// Stage-folded backward (fold.cpp): items are head ranges in reverse
+// super-level order.  Per item:
+//  (1) fanout-entry threads gather the per-arc adjoint words of the heads'
+//      light fanout rows (cp.async, re-poll stale parity), while entry threads
+//      already load their entry's topology and Eq 6 weights into registers;
+//  (2) head threads form each head's adjoint (seed + pulled sum + heavy
+//      accumulator, the same expression as bwd_kernel) and hand it (and, hard
+//      mode, the arg-max selection) to the head's entries in shared memory;
+//  (3) entry threads apply the sink side (Eq 6 chain) of arc e = (p -> q);
+//      when p is folded they continue through p: its adjoint is exactly what
+//      p's own pull would have produced from the word just formed (0 + ((0 +
+//      g) + 0)), then the sink side of e' = (j -> p).  Same arithmetic as the
+//      per-level schedule, hence bit-identical to it.
+// --------------------------------------------------------------------------
+struct BwdfStage {
+  int32_t lptr[kBwdPins + 8];   // light fanout rows of the heads
+  int32_t lfo[kBwdFanout + 8];  // adjoint word positions of those rows
+  int32_t hptr[kBwdPins + 8];   // entry rows of the heads
+};
+constexpr int kEntPerThread = kBwdArcs / kThreads;
+constexpr int kHeadsPerThread = kBwdPins / kThreads;
+constexpr size_t kBwdfSmem = 2 * sizeof(BwdfStage) + sizeof(float2) * kBwdFanout + sizeof(float2) * kBwdArcs +
+                             sizeof(int32_t) * kBwdArcs + sizeof(HeavyTab);
+
+template <bool kLSE>
+__device__ __forceinline__ void bwdf_prefetch(const KParams& P, BwdfStage* st, uint64_t* full, int step, int c) {
+  const int4 A = __ldg(P.item_a + size_t(step) * P.grid + c);   // {h_lo, h_hi, lfo_lo, lfo_hi}
+  const int4 B = __ldg(P.item_b + size_t(step) * P.grid + c);   // {x_lo, x_hi, slevel, flags}
+  if (!bwd_staged(A, B)) return;
+  const Window wl = window(A.x, A.y + 1, 4);   // lfo_ptr and hd_ptr: same head window
+  const Window wf = window(A.z, A.w, 4);
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  mbar_expect_tx(full, 2 * wl.bytes + wf.bytes);
+  bulk_g2s(st->lptr, P.lfo_ptr + wl.start, wl.bytes, full);
+  bulk_g2s(st->hptr, P.fanin_ptr + wl.start, wl.bytes, full);
+  if (wf.bytes) bulk_g2s(st->lfo, P.lfo + wf.start, wf.bytes, full);
+}
+
+// Eq 6 sink side of one arc with sink adjoint ab: weights w[rf][s] (hard: the
+// selection bits sel, bit rf*2+s; LSE: w4).  Writes dL/d(arc mean) and returns
+// the adjoint to the source's {R, F} (as bwd_sink).
+template <bool kLSE>
+__device__ __forceinline__ float2 sink_arc(const KParams& P, float2 ab, int sel, float4 w4, int32_t arcid) {
+  const float abr[2] = {ab.x, ab.y};
+  float w[2][2];
+  if (kLSE) {
+    w[0][0] = w4.x;
+    w[0][1] = w4.y;
+    w[1][0] = w4.z;
+    w[1][1] = w4.w;
+  } else {
+#pragma unroll
+    for (int rf = 0; rf < 2; ++rf) {
+      w[rf][0] = ((sel >> (2 * rf)) & 1) ? 1.f : 0.f;
+      w[rf][1] = ((sel >> (2 * rf + 1)) & 1) ? 1.f : 0.f;
+    }
+  }
+  float gm[2], gs[2] = {0.f, 0.f};
+#pragma unroll
+  for (int rf = 0; rf < 2; ++rf) {
+    const float a0 = w[rf][0] * abr[rf], a1 = w[rf][1] * abr[rf];
+    gm[rf] = a0 + a1;
+    gs[0] += a0;
+    gs[1] += a1;
+  }
+  if (gm[0] != 0.f || gm[1] != 0.f) reinterpret_cast<float2*>(P.d_mean)[arcid] = make_float2(gm[0], gm[1]);
+  return make_float2(gs[0], gs[1]);
+}
+
+// hard-mode selection bits of fanin arc k from a pin's arg-max word
+__device__ __forceinline__ int win_sel(int32_t win, int k) {
+  int sel = 0;
+#pragma unroll
+  for (int rf = 0; rf < 2; ++rf) {
+    const int wv = (win >> (16 * rf)) & 0xffff;
+    if ((wv & 0x7fff) == k) sel |= 1 << (2 * rf + (wv >> 15));
+  }
+  return sel;
+}
+
+struct EntryIn {
+  int32_t qpos, bw, arc, farc, fq, fsel;
+  float4 w, fw;
+};
+
+template <bool kLSE>
+__device__ __forceinline__ EntryIn load_entry(const KParams& P, int x) {
+  EntryIn e;
+  e.qpos = __ldg(P.ext_qpos + x);
+  e.bw = __ldg(P.ext_bw + x);
+  e.arc = __ldg(P.ext_arc + x);
+  e.farc = __ldg(P.ext_farc + x);
+  e.fq = __ldg(P.ext_fq + x);
+  e.fsel = 0;
+  e.w = e.fw = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (kLSE) {
+    e.w = __ldcg(P.wts + e.qpos);
+    if (e.farc >= 0) e.fw = __ldcg(P.wts + e.fq);
+  } else if (e.farc >= 0) {
+    e.fsel = win_sel(__ldcg(P.win + (__ldg(P.ext_f + x) & kSrcMask)), 0);   // folded pin: one fanin arc
+  }
+  return e;
+}
+
+// sink side of entry e (and of its folded pin), given the head's adjoint ab
+template <bool kLSE>
+__device__ __forceinline__ void bwdf_entry(const KParams& P, HeavyTab* tab, const EntryIn& e, float2 ab, int sel) {
+  const float2 gs = sink_arc<kLSE>(P, ab, sel, e.w, e.arc);
+  if (e.farc < 0) {   // source p is a head: publish the per-arc adjoint for its pull
+    st2_f32(P.g + e.qpos, with_parf(gs.x, P.par), with_parf(gs.y, P.par));
+    heavy_add(P, tab, e.bw, gs.x, gs.y);
+  } else {            // folded p: its adjoint as its own pull would form it, then arc e'
+    const float gx = with_parf(gs.x, P.par), gy = with_parf(gs.y, P.par);
+    float sx = 0.f, sy = 0.f;
+    sx += stripf(__float_as_uint(gx));
+    sy += stripf(__float_as_uint(gy));
+    const float2 abp = make_float2(0.f + (sx + 0.f), 0.f + (sy + 0.f));
+    const float2 g2 = sink_arc<kLSE>(P, abp, e.fsel, e.fw, e.farc);
+    st2_f32(P.g + e.fq, with_parf(g2.x, P.par), with_parf(g2.y, P.par));
+    heavy_add(P, tab, e.bw, g2.x, g2.y);
+  }
+}
+
+template <bool kLSE>
+__global__ void __launch_bounds__(kThreads, 1) bwdf_kernel(KParams P) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  BwdfStage* stage = reinterpret_cast<BwdfStage*>(smem);
+  float2* gg = reinterpret_cast<float2*>(smem + 2 * sizeof(BwdfStage));
+  float2* eab = gg + kBwdFanout;                                    // per entry: head adjoint
+  int32_t* esel = reinterpret_cast<int32_t*>(eab + kBwdArcs);       // per entry: hard-mode selection
+  HeavyTab* htab = reinterpret_cast<HeavyTab*>(esel + kBwdArcs);
+  __shared__ __align__(8) uint64_t full[2];
+  const int c = blockIdx.x;
+  const int tid = threadIdx.x;
+  if (tid == 0) {
+    mbar_init1(&full[0]);
+    mbar_init1(&full[1]);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  heavy_tab_clear(htab);
+  __syncthreads();
+  uint32_t phase[2] = {0u, 0u};
+  const int nsteps = P.step_end - P.step_begin;
+  if (tid == 0 && nsteps > 0) bwdf_prefetch<kLSE>(P, &stage[0], &full[0], P.step_begin, c);
+  for (int t = 0; t < nsteps; ++t) {
+    const int buf = t & 1;
+    const int k = P.step_begin + t;
+    const int4 A = __ldg(P.item_a + size_t(k) * P.grid + c);   // {h_lo, h_hi, lfo_lo, lfo_hi}
+    const int4 B = __ldg(P.item_b + size_t(k) * P.grid + c);   // {x_lo, x_hi, slevel, flags}
+    if (tid == 0 && t + 1 < nsteps) bwdf_prefetch<kLSE>(P, &stage[buf ^ 1], &full[buf ^ 1], k + 1, c);
+    trace_stamp(P, c, nsteps, t, 0);
+    const int np = A.y - A.x;
+    if (np > 0 && !(B.w & kItemDirect)) {
+      // entry and head inputs: independent of the dependency chain, issued first
+      EntryIn ein[kEntPerThread];
+#pragma unroll
+      for (int j = 0; j < kEntPerThread; ++j) {
+        const int x = B.x + tid + j * kThreads;
+        if (x < B.y) ein[j] = load_entry<kLSE>(P, x);
+      }
+      int32_t hpin[kHeadsPerThread], hslot[kHeadsPerThread], hwin[kHeadsPerThread];
+      float2 hsd[kHeadsPerThread];
+#pragma unroll
+      for (int j = 0; j < kHeadsPerThread; ++j) {
+        const int h = A.x + tid + j * kThreads;
+        if (h < A.y) {
+          hpin[j] = __ldg(P.hd_pin + h);
+          hslot[j] = __ldg(P.hd_hslot + h);
+          hsd[j] = __ldcg(P.hseed + h);
+          hwin[j] = kLSE ? 0 : __ldcg(P.win + hpin[j]);
+        }
+      }
+      mbar_wait(&full[buf], phase[buf]);
+      phase[buf] ^= 1u;
+      const BwdfStage& S = stage[buf];
+      const int lo = A.x & 3, fo = A.z & 3;
+      const int nfo = A.w - A.z;
+      // (1) gather the sinks' per-arc adjoints of every light fanout entry
+      for (int e = tid; e < nfo; e += kThreads)
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(gg + e)), "l"(P.g + S.lfo[fo + e])
+                     : "memory");
+      asm volatile("cp.async.wait_all;" ::: "memory");
+      for (int e = tid; e < nfo; e += kThreads) {
+        uint32_t a = __float_as_uint(gg[e].x), b = __float_as_uint(gg[e].y);
+        if (P.mode == 2 && (((a & 1u) != P.par) || ((b & 1u) != P.par))) {
+          const int q = S.lfo[fo + e];
+          ld2_u32(P.g + q, a, b);
+          await_g(P, q, a, b);
+        }
+        gg[e] = make_float2(stripf(a), stripf(b));
+      }
+      __syncthreads();
+      trace_stamp(P, c, nsteps, t, 1);
+      // (2) heads: adjoint = seed + (pull + heavy accumulator)
+#pragma unroll
+      for (int j = 0; j < kHeadsPerThread; ++j) {
+        const int p = tid + j * kThreads;
+        if (p < np) {
+          const int r0 = S.lptr[lo + p] - A.z, r1 = S.lptr[lo + p + 1] - A.z;
+          float sx = 0.f, sy = 0.f;
+          for (int r = r0; r < r1; ++r) {
+            sx += gg[r].x;
+            sy += gg[r].y;
+          }
+          const float2 h = heavy_take(P, hslot[j]);
+          const float2 ab = make_float2(hsd[j].x + (sx + h.x), hsd[j].y + (sy + h.y));
+          if (B.z == 0) {
+            if (P.d_src) reinterpret_cast<float2*>(P.d_src)[__ldg(P.order + hpin[j])] = ab;
+          } else {
+            const int x0 = S.hptr[lo + p], x1 = S.hptr[lo + p + 1];
+            for (int x = x0; x < x1; ++x) {
+              eab[x - B.x] = ab;
+              if (!kLSE) esel[x - B.x] = win_sel(hwin[j], x - x0);
+            }
+          }
+        }
+      }
+      __syncthreads();
+      // (3) entries: sink side of e (and of the folded pin behind it)
+      if (B.z > 0) {
+#pragma unroll
+        for (int j = 0; j < kEntPerThread; ++j) {
+          const int xr = tid + j * kThreads;
+          if (B.x + xr < B.y) bwdf_entry<kLSE>(P, htab, ein[j], eab[xr], kLSE ? 0 : esel[xr]);
+        }
+      }
+    } else if (np > 0) {
+      // direct: one head with more entries than the item caps
+      __shared__ float2 s_ab;
+      __shared__ int32_t s_win;
+      if (tid == 0) {
+        const int h = A.x;
+        const int q = __ldg(P.hd_pin + h);
+        float sx = 0.f, sy = 0.f;
+        for (int r = __ldg(P.lfo_ptr + h); r < __ldg(P.lfo_ptr + h + 1); ++r) {
+          const float2 v = load_g(P, __ldg(P.lfo + r));
+          sx += v.x;
+          sy += v.y;
+        }
+        const float2 hv = heavy_take(P, __ldg(P.hd_hslot + h));
+        const float2 sd = __ldcg(P.hseed + h);
+        s_ab = make_float2(sd.x + (sx + hv.x), sd.y + (sy + hv.y));
+        s_win = kLSE ? 0 : __ldcg(P.win + q);
+        if (B.z == 0 && P.d_src) reinterpret_cast<float2*>(P.d_src)[__ldg(P.order + q)] = s_ab;
+      }
+      __syncthreads();
+      if (B.z > 0) {
+        for (int x = B.x + tid; x < B.y; x += kThreads) {
+          const EntryIn e = load_entry<kLSE>(P, x);
+          bwdf_entry<kLSE>(P, htab, e, s_ab, kLSE ? 0 : win_sel(s_win, x - B.x));
+        }
+      }
+    }
+    __syncthreads();
+    heavy_tab_flush(P, htab);
+    trace_stamp(P, c, nsteps, t, 2);
+  }
+}
+
 // Endpoint seeds: dL/dA_ep[rf*] = -dL/dslack (slack = RAT - A); TNS: dL/dslack
 // = 1 where slack < 0.
-__global__ void seed_kernel(int num_ep, const int32_t* __restrict__ ep_pin,
+// Written in canonical order (per-level schedule) and in head order (folded).
+__global__ void seed_kernel(int num_ep, const int32_t* __restrict__ ep_pin, const int32_t* __restrict__ ep_head,
                             const float* __restrict__ slack, const uint8_t* __restrict__ rf_star,
-                            const float* __restrict__ ep_seed, float2* seed) {
+                            const float* __restrict__ ep_seed, float2* seed, float2* hseed) {
   const int k = blockIdx.x * blockDim.x + threadIdx.x;
   if (k >= num_ep) return;
   const float d = ep_seed ? ep_seed[k] : (slack[k] < 0.f ? 1.f : 0.f);
   const float v = d == 0.f ? 0.f : -d;
-  seed[ep_pin[k]] = rf_star[k] ? make_float2(0.f, v) : make_float2(v, 0.f);
+  const float2 sd = rf_star[k] ? make_float2(0.f, v) : make_float2(v, 0.f);
+  seed[ep_pin[k]] = sd;
+  hseed[ep_head[k]] = sd;
 }
 
 // --------------------------------------------------------------------------
@@ -1052,6 +1361,7 @@ __global__ void update_arcs_kernel(int64_t n, const int32_t* __restrict__ ids,
                                    const float2* __restrict__ mean,
                                    const float2* __restrict__ sigma,
                                    const int32_t* __restrict__ arc_pos, float4* fin_ms,
+                                   const int32_t* __restrict__ arc_xpos, float4* ext_ms, float4* ext_fms,
                                    const int32_t* __restrict__ arc_sink, const int32_t* __restrict__ pin_level,
                                    uint32_t* dirty, uint32_t stamp, int32_t* lvl_range) {
   const int64_t k = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
@@ -1059,6 +1369,8 @@ __global__ void update_arcs_kernel(int64_t n, const int32_t* __restrict__ ids,
   const int q = arc_pos[ids[k]];
   const float2 m = mean[k], s = sigma[k];
   fin_ms[q] = make_float4(m.x, m.y, s.x, s.y);
+  const int x = arc_xpos[ids[k]];   // the stage-folded schedule's copy of the record
+  ((x & 1) ? ext_fms : ext_ms)[x >> 1] = make_float4(m.x, m.y, s.x, s.y);
   if (dirty) {   // incremental: the sink must be recomputed in the next pass
     const int i = arc_sink[ids[k]];
     dirty[i] = stamp;
@@ -1247,6 +1559,17 @@ static KParams make_params(DevGraph& g, bool bwd) {
   P.heavy_slot = g.heavy_slot;
   P.src_ms = g.src_ms;
   P.order = g.order;
+  P.hd_pin = g.hd_pin;
+  P.hd_q0 = g.hd_q0;
+  P.ext_f = g.ext_f;
+  P.ext_fms = g.ext_fms;
+  P.ext_fq = g.ext_fq;
+  P.hd_hslot = g.hd_hslot;
+  P.ext_qpos = g.ext_qpos;
+  P.ext_bw = g.ext_bw;
+  P.ext_arc = g.ext_arc;
+  P.ext_farc = g.ext_farc;
+  P.hseed = g.hseed;
   P.state = g.state;
   P.win = g.win;
   P.wts = g.wts;
@@ -1271,19 +1594,27 @@ int query_grid(int device, int* grid) {
   if (e != cudaSuccess) return int(e);
   cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, device);
   if (!coop) return int(cudaErrorNotSupported);
-  int err = set_smem(fwd_kernel<false>, kFwdSmemV6);
-  if (!err) err = set_smem(fwd_kernel<true>, kFwdSmemV6);
+  int err = set_smem(fwd_kernel<false, false>, kFwdSmemV6);
+  if (!err) err = set_smem(fwd_kernel<true, false>, kFwdSmemV6);
+  if (!err) err = set_smem(fwd_kernel<false, true>, kFwdSmemV6);
+  if (!err) err = set_smem(fwd_kernel<true, true>, kFwdSmemV6);
   if (!err) err = set_smem(bwd_kernel<false>, bwd_smem<false>());
   if (!err) err = set_smem(bwd_kernel<true>, bwd_smem<true>());
+  if (!err) err = set_smem(bwdf_kernel<false>, kBwdfSmem);
+  if (!err) err = set_smem(bwdf_kernel<true>, kBwdfSmem);
   if (err) return err;
   int occ = 1 << 30, b = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<false>, kFwdThreads, kFwdSmemV6);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<false, true>, kFwdThreads, kFwdSmemV6);
   occ = std::min(occ, b);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<true>, kFwdThreads, kFwdSmemV6);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<true, true>, kFwdThreads, kFwdSmemV6);
   occ = std::min(occ, b);
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bwd_kernel<false>, kThreads, bwd_smem<false>());
   occ = std::min(occ, b);
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bwd_kernel<true>, kThreads, bwd_smem<true>());
+  occ = std::min(occ, b);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bwdf_kernel<false>, kThreads, kBwdfSmem);
+  occ = std::min(occ, b);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bwdf_kernel<true>, kThreads, kBwdfSmem);
   occ = std::min(occ, b);
   if (occ <= 0) return int(cudaErrorLaunchOutOfResources);
   *grid = occ * sms;
@@ -1369,8 +1700,19 @@ int launch_forward(DevGraph& g, float n_sigma, float tau, int schedule, void* st
   if (g.n > 0) {
     P.mode = schedule == 0 ? 2 : 0;   // dataflow persistent / one launch per level
     P.par = (++g.pass_fwd) & 1u;
-    int err = launch_items(lse ? (const void*)fwd_kernel<true> : (const void*)fwd_kernel<false>, kFwdThreads,
-                           kFwdSmemV6, P, g.fwd_items, false, st);
+    int err;
+    if (schedule == 0) {   // stage-folded persistent pass (fold.cpp)
+      P.item_a = g.fwdf_a;
+      P.item_b = g.fwdf_b;
+      P.fanin_ptr = g.hd_ptr;
+      P.fin_src = g.ext_w;
+      P.fin_ms = g.ext_ms;
+      err = launch_items(lse ? (const void*)fwd_kernel<true, true> : (const void*)fwd_kernel<false, true>,
+                         kFwdThreads, kFwdSmemV6, P, g.fwdf_items, false, st);
+    } else {   // the paper's launch structure: one launch per timing level
+      err = launch_items(lse ? (const void*)fwd_kernel<true, false> : (const void*)fwd_kernel<false, false>,
+                         kFwdThreads, kFwdSmemV6, P, g.fwd_items, false, st);
+    }
     if (err) return err;
   }
   g.last_n_sigma = n_sigma;
@@ -1391,8 +1733,8 @@ int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float*
     if (e != cudaSuccess) return int(e);
   }
   if (g.num_ep > 0) {
-    seed_kernel<<<(g.num_ep + 255) / 256, 256, 0, st>>>(g.num_ep, g.ep_pin, g.slack, g.rf_star,
-                                                        ep_seed, g.seed);
+    seed_kernel<<<(g.num_ep + 255) / 256, 256, 0, st>>>(g.num_ep, g.ep_pin, g.ep_head, g.slack, g.rf_star,
+                                                        ep_seed, g.seed, g.hseed);
     int err = int(cudaGetLastError());
     if (err) return err;
   }
@@ -1406,6 +1748,15 @@ int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float*
   const bool lse = g.last_tau > 0.f;
   P.mode = g.bwd_schedule == 0 ? 2 : 0;
   P.par = (++g.pass_bwd) & 1u;
+  if (g.bwd_schedule == 0) {   // stage-folded persistent pass (fold.cpp)
+    P.item_a = g.bwdf_a;
+    P.item_b = g.bwdf_b;
+    P.lfo_ptr = g.hlfo_ptr;
+    P.lfo = g.hlfo;
+    P.fanin_ptr = g.hd_ptr;
+    return launch_items(lse ? (const void*)bwdf_kernel<true> : (const void*)bwdf_kernel<false>, kThreads,
+                        kBwdfSmem, P, g.bwdf_items, true, st);
+  }
   return launch_items(lse ? (const void*)bwd_kernel<true> : (const void*)bwd_kernel<false>, kThreads,
                       lse ? bwd_smem<true>() : bwd_smem<false>(),
                       P, g.bwd_items, true, st);
@@ -1418,7 +1769,7 @@ int launch_update_arcs(DevGraph& g, int64_t n, const int32_t* ids, const float* 
   const int blocks = int((n + 255) / 256);
   update_arcs_kernel<<<blocks, 256, 0, st>>>(n, ids, reinterpret_cast<const float2*>(mean),
                                              reinterpret_cast<const float2*>(sigma), g.arc_pos,
-                                             g.fin_ms, g.arc_sink, g.pin_level,
+                                             g.fin_ms, g.arc_xpos, g.ext_ms, g.ext_fms, g.arc_sink, g.pin_level,
                                              incremental ? g.dirty : nullptr, g.inc_epoch + 1, g.lvl_range);
   return int(cudaGetLastError());
 }

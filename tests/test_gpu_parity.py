@@ -279,3 +279,82 @@ def test_c4_full_size_parity():
     b = oracle.backward(g, NS, 0.0)
     assert not ((d != b["d_mean"]) & ~at).any()
     G.close()
+
+
+def _fold_shapes(seed=3):
+    """Graph shapes that exercise the stage-folded forward (fold.cpp): a
+    fanin-1/fanout-1 chain (folds alternate), cells whose inputs are all
+    folded with 3, 40 (> 32 arcs: single-lane merge) and 1500 (> the item
+    cap: direct path) inputs, non-unate arcs on both sides of a folded pin,
+    a folded pin driven by a heavy (> 256 sinks) driver, and an endpoint with
+    fanout 1 (never folded)."""
+    rng = np.random.default_rng(seed)
+    af, at, un = [], [], []
+    n = [0]
+
+    def pin():
+        n[0] += 1
+        return n[0] - 1
+
+    def arc(a, b, u):
+        af.append(a)
+        at.append(b)
+        un.append(u)
+
+    srcs = [pin() for _ in range(8)]
+    eps = []
+    # chain
+    x = srcs[0]
+    for k in range(20):
+        y = pin()
+        arc(x, y, int(rng.integers(0, 3)))
+        x = y
+    eps.append(x)
+    # heavy driver with 300 sinks, each feeding a 3-input cell
+    drv = pin()
+    arc(srcs[1], drv, 0)
+    sinks = [pin() for _ in range(300)]
+    for s_ in sinks:
+        arc(drv, s_, 0)
+    for c in range(100):
+        out = pin()
+        for s_ in sinks[3 * c:3 * c + 3]:
+            arc(s_, out, int(rng.integers(0, 3)))
+        eps.append(out)
+    # wide cells: inputs are net sinks of random earlier drivers
+    for width in (40, 1500):
+        out = pin()
+        for k in range(width):
+            ip = pin()
+            arc(int(rng.choice(srcs)), ip, int(rng.integers(0, 3)))
+            arc(ip, out, int(rng.integers(0, 3)))
+        eps.append(out)
+    # an endpoint with one fanin and one fanout: not folded
+    e1 = pin()
+    arc(srcs[2], e1, 1)
+    e2 = pin()
+    arc(e1, e2, 2)
+    eps += [e1, e2]
+    N, E = n[0], len(af)
+    return types.SimpleNamespace(
+        num_pins=N, arc_from=np.array(af, np.int32), arc_to=np.array(at, np.int32),
+        arc_unate=np.array(un, np.uint8), arc_class=np.zeros(E, np.uint8),
+        arc_mean=rng.uniform(1, 10, (E, 2)).astype(np.float32),
+        arc_sigma=rng.uniform(0, 1, (E, 2)).astype(np.float32),
+        src_mean=rng.uniform(0, 5, (N, 2)).astype(np.float32), src_sigma=rng.uniform(0, 1, (N, 2)).astype(np.float32),
+        ep_pin=np.array(eps, np.int32), ep_rat=np.full((len(eps), 2), 40.0, np.float32))
+
+
+@pytest.mark.parametrize("tau", [0.0, 1.0])
+def test_stage_folded_shapes(tau):
+    g = _fold_shapes()
+    a = run_gpu(g, tau, 0, want_src=True)
+    c = run_gpu(g, tau, 1, want_src=True)
+    assert np.array_equal(a.A, c.A) and np.array_equal(a.mu, c.mu) and np.array_equal(a.sigma, c.sigma)
+    assert np.array_equal(a.d_mean, c.d_mean) and np.array_equal(a.d_src, c.d_src)
+    f, s, b = run_oracle(g, tau)
+    ft, at = oracle.tie_taint(g, NS, eps=1e-4, margin=0.05)
+    assert not tol_ok(a.A, f["A"], ft if tau == 0 else None).any()
+    mask = at if tau == 0 else np.zeros_like(at)
+    err = np.abs(a.d_mean - b["d_mean"])
+    assert ((err <= 1e-3 * np.maximum(np.abs(b["d_mean"]), 1)) | mask).all()

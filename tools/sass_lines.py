@@ -9,7 +9,8 @@ import sys
 
 rows = list(csv.reader(open(sys.argv[1])))
 hdr = rows[1]
-ai, ni, si = hdr.index("Address"), hdr.index("Warp Stall Sampling (All Samples)"), hdr.index("Source")
+import os
+ai, ni, si = hdr.index("Address"), hdr.index(os.environ.get("COL", "Warp Stall Sampling (All Samples)")), hdr.index("Source")
 data = [r for r in rows[2:] if len(r) == len(hdr)]
 base = min(int(r[ai], 16) for r in data)
 samples = collections.Counter()
