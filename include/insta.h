@@ -146,10 +146,14 @@ insta_status insta_arrivals(insta_graph* g, float* A, float* mean, float* sigma,
  * in reverse level order.  ep_seed: DEVICE float[num_endpoints] dL/dslack, or
  * NULL for L = TNS (seed 1 where slack < 0).  d_arc_mean: DEVICE
  * float[num_arcs][2] in caller arc order, overwritten (required).
- * d_arc_sigma must be NULL in this version.  d_src: DEVICE float[num_pins][2]
- * dL/d(src_mean) in caller pin order (0 at non-source pins), or NULL.
- * Uses the tau/n_sigma of the last forward.  INSTA_E_STATE if the last
- * forward is stale. */
+ * d_arc_sigma: DEVICE float[num_arcs][2] dL/d(arc sigma), overwritten, or NULL.
+ * The sigma channel (the corner A = mu + n_sigma*sigma of
+ * Eq 3 carries sigma through sqrt(sigma_j^2 + sigma_e^2) of Eq 2, and the
+ * merged pin keeps the arg-max candidate's sigma, reading R1) runs
+ * a separate per-level pass; d_arc_mean is bit-identical either way.
+ * d_src: DEVICE float[num_pins][2] dL/d(src_mean) in caller pin order (0 at
+ * non-source pins), or NULL.  Uses the tau/n_sigma of the last forward.
+ * INSTA_E_STATE if the last forward is stale. */
 insta_status insta_backward(insta_graph* g, const float* ep_seed, float* d_arc_mean,
                             float* d_arc_sigma, float* d_src, void* cuda_stream);
 

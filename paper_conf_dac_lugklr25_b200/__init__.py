@@ -155,17 +155,21 @@ class Graph:
         check(self.lib.insta_arrivals(self._h, _dptr(A), _dptr(m), _dptr(s), self._st(stream)), "insta_arrivals")
         return A, m, s
 
-    def backward(self, ep_seed=None, want_src: bool = False, out=None, stream=None):
-        """insta_backward: dL/d(arc mean) float32[E,2] (caller arc order); L = TNS if ep_seed is None."""
+    def backward(self, ep_seed=None, want_src: bool = False, out=None, stream=None, want_sigma: bool = False):
+        """insta_backward: dL/d(arc mean) float32[E,2] (caller arc order); L = TNS if ep_seed is None.
+        want_sigma: also dL/d(arc sigma) float32[E,2]; want_src: dL/d(src mean) float32[N,2].
+        Returns d_mean, or a tuple (d_mean[, d_sigma][, d_src])."""
         t = self._torch
         d_mean = out if out is not None else t.empty((self.num_arcs, 2), dtype=t.float32, device=self.device)
+        d_sig = t.empty((self.num_arcs, 2), dtype=t.float32, device=self.device) if want_sigma else None
         d_src = t.empty((self.num_pins, 2), dtype=t.float32, device=self.device) if want_src else None
         seed = None
         if ep_seed is not None:
             seed = t.as_tensor(ep_seed, dtype=t.float32, device=self.device).contiguous()
-        check(self.lib.insta_backward(self._h, _dptr(seed), _dptr(d_mean), None, _dptr(d_src), self._st(stream)),
-              "insta_backward")
-        return (d_mean, d_src) if want_src else d_mean
+        check(self.lib.insta_backward(self._h, _dptr(seed), _dptr(d_mean), _dptr(d_sig), _dptr(d_src),
+                                      self._st(stream)), "insta_backward")
+        outs = (d_mean,) + ((d_sig,) if want_sigma else ()) + ((d_src,) if want_src else ())
+        return outs if len(outs) > 1 else d_mean
 
     def update_arcs(self, arc_ids, mean, sigma, incremental: bool = True, stream=None):
         """insta_update_arcs: re-annotate arcs (device or host arrays; copied to the device)."""

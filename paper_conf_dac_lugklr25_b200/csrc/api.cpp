@@ -60,7 +60,7 @@ void free_graph(insta::DevGraph& d) {
                   d.hd_pin,    d.hd_ptr,    d.hd_q0,     d.ext_w,      d.ext_ms,    d.ext_f,
                   d.ext_fms,   d.ext_fq,    d.arc_xpos,  d.fwdf_a,     d.fwdf_b,    d.hd_hslot,
                   d.hlfo_ptr,  d.hlfo,      d.ext_qpos,  d.ext_bw,     d.ext_arc,   d.ext_farc,
-                  d.ep_head,   d.hseed,     d.bwdf_a,    d.bwdf_b};
+                  d.ep_head,   d.hseed,     d.bwdf_a,    d.bwdf_b,    d.g4,        d.hacc4};
   for (void* p : ptrs)
     if (p) cudaFree(p);
 }
@@ -435,12 +435,11 @@ insta_status insta_arrivals(insta_graph* g, float* A, float* mean, float* sigma,
 insta_status insta_backward(insta_graph* g, const float* ep_seed, float* d_arc_mean,
                             float* d_arc_sigma, float* d_src, void* cuda_stream) {
   if (!g) return fail(INSTA_E_ARG, "backward: NULL graph");
-  if (d_arc_sigma) return fail(INSTA_E_ARG, "backward: d_arc_sigma is not supported (pass NULL)");
   insta::DevGraph& d = g->d;
   if (!d_arc_mean && d.e > 0) return fail(INSTA_E_ARG, "backward: d_arc_mean is required");
   if (!d.fwd_valid) return fail(INSTA_E_STATE, "backward: no valid forward (call insta_forward)");
   cudaSetDevice(d.device);
-  int err = insta::launch_backward(d, ep_seed, d_arc_mean, d_src, cuda_stream);
+  int err = insta::launch_backward(d, ep_seed, d_arc_mean, d_arc_sigma, d_src, cuda_stream);
   if (err) return cuda_fail(err, "backward");
   return INSTA_OK;
 }

@@ -195,6 +195,9 @@ struct DevGraph {
   int32_t* ext_farc = nullptr;
   int32_t* ep_head = nullptr;
   float2* hseed = nullptr;         // [H] endpoint seeds in head order
+  // sigma-channel backward scratch (allocated on first use)
+  void* g4 = nullptr;              // [e] float4 per fanin position
+  long long* hacc4 = nullptr;      // [num_heavy][4] fixed-point adjoints
   int4* bwdf_a = nullptr;
   int4* bwdf_b = nullptr;
   ItemTable bwdf_items;
@@ -250,7 +253,7 @@ int query_grid(int device, int* grid);
 int launch_forward(DevGraph& g, float n_sigma, float tau, int schedule, void* stream);
 int launch_forward_incremental(DevGraph& g, float n_sigma, float tau, void* stream);
 int launch_slack(DevGraph& g, void* stream);
-int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float* d_src,
+int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float* d_arc_sigma, float* d_src,
                     void* stream);
 int launch_update_arcs(DevGraph& g, int64_t n, const int32_t* ids, const float* mean,
                        const float* sigma, int incremental, void* stream);

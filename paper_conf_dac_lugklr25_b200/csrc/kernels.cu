@@ -1244,6 +1244,130 @@ __global__ void __launch_bounds__(kThreads, 1) bwdf_kernel(KParams P) {
 
 // Endpoint seeds: dL/dA_ep[rf*] = -dL/dslack (slack = RAT - A); TNS: dL/dslack
 // = 1 where slack < 0.
+// --------------------------------------------------------------------------
+// Backward with the sigma channel (insta_backward with d_arc_sigma; SURVEY
+// §8(c) O7).  The adjoint of every pin is the pair (Abar, Sbar) w.r.t. its
+// corner arrival A and its sigma.  Per candidate c = (arc e = j -> i, s) of
+// (i, rf), with Eq 6 weight w_c and arg-max c*:
+//   Abar_c = w_c Abar_i[rf]                      -> dL/d(arc mean)[rf], Abar_j[s]
+//   Sbar_c = n_sigma Abar_c + [c = c*] Sbar_i[rf] (reading R1: sigma_i = sigma_c*)
+//   dL/d(arc sigma)[rf] += Sbar_c sigma_e[rf] / sigma_c
+//   Sbar_j[s] += -n_sigma Abar_c + Sbar_c sigma_j[s] / sigma_c   (0/0 := 0)
+// since A_c = (A_j - n_sigma sigma_j) + mu_e + n_sigma sigma_c and
+// sigma_c = sqrt(sigma_j^2 + sigma_e^2) (Eq 1-3).  The candidates, the arg-max
+// and the weights are recomputed from the stored states with the forward's
+// functions (merge_rf / make_cand), so the mean channel is bit-identical to
+// the main backward.  One launch per level (reverse order; kernel boundaries
+// order the levels), one thread per pin; each fanin arc publishes its
+// adjoint to the source as a float4 {Abar_R, Abar_F, Sbar_R, Sbar_F}; heavy
+// drivers accumulate int64 fixed point (order-independent, deterministic).
+// --------------------------------------------------------------------------
+struct SigParams {
+  int32_t lo, hi, level;
+  float4* g4;                 // [E] per fanin position
+  long long* hacc4;           // [num_heavy][4]
+  float* d_sigma;             // [E][2] caller arc order
+};
+
+template <bool kLSE>
+__global__ void __launch_bounds__(256) bwds_kernel(KParams P, SigParams Q) {
+  const int i = Q.lo + blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= Q.hi) return;
+  const double ns = double(P.n_sigma);
+  float ax = 0.f, ay = 0.f, bx = 0.f, by = 0.f;
+  for (int r = __ldg(P.lfo_ptr + i); r < __ldg(P.lfo_ptr + i + 1); ++r) {
+    const float4 v = Q.g4[__ldg(P.lfo + r)];
+    ax += v.x;
+    ay += v.y;
+    bx += v.z;
+    by += v.w;
+  }
+  float2 h = make_float2(0.f, 0.f), hs = make_float2(0.f, 0.f);
+  const int slot = __ldg(P.heavy_slot + i);
+  if (slot >= 0) {
+    long long* acc = Q.hacc4 + 4 * size_t(slot);
+    h = make_float2(float(double(acc[0]) / kFixH), float(double(acc[1]) / kFixH));
+    hs = make_float2(float(double(acc[2]) / kFixH), float(double(acc[3]) / kFixH));
+    acc[0] = acc[1] = acc[2] = acc[3] = 0;
+  }
+  const float2 sd = P.seed[i];
+  const float abr[2] = {sd.x + (ax + h.x), sd.y + (ay + h.y)};   // as bwd_kernel
+  const float sbr[2] = {bx + hs.x, by + hs.y};
+  if (Q.level == 0) {
+    if (P.d_src) reinterpret_cast<float2*>(P.d_src)[__ldg(P.order + i)] = make_float2(abr[0], abr[1]);
+    return;
+  }
+  const int b0 = __ldg(P.fanin_ptr + i), nf = __ldg(P.fanin_ptr + i + 1) - b0;
+  auto arc = [&](int kk, int32_t& w, float4& ms, Raw& rr) {
+    w = __ldg(P.fin_src + b0 + kk);
+    ms = __ldg(P.fin_ms + b0 + kk);
+    const PinState* sp = P.state + (w & kSrcMask);
+    const double2 m = __ldcg(reinterpret_cast<const double2*>(sp));
+    const double2 v = __ldcg(reinterpret_cast<const double2*>(sp) + 1);
+    rr.a = (unsigned long long)__double_as_longlong(m.x);
+    rr.b = (unsigned long long)__double_as_longlong(m.y);
+    rr.c = (unsigned long long)__double_as_longlong(v.x);
+    rr.d = (unsigned long long)__double_as_longlong(v.y);
+  };
+  const RfOut o[2] = {merge_rf<kLSE>(ns, double(P.tau), P.inv_tau, 0, nf, arc),
+                      merge_rf<kLSE>(ns, double(P.tau), P.inv_tau, 1, nf, arc)};
+  for (int k = 0; k < nf; ++k) {
+    int32_t w;
+    float4 ms;
+    Raw rr;
+    arc(k, w, ms, rr);
+    const Gath st = unpack(rr);
+    const int u = int(uint32_t(w) >> kUnateShift);
+    float gm[2], gs[2] = {0.f, 0.f}, dsg[2] = {0.f, 0.f}, gsig[2] = {0.f, 0.f};
+    const float sig_j[2] = {sigma_of(st.v0), sigma_of(st.v1)};
+#pragma unroll
+    for (int rf = 0; rf < 2; ++rf) {
+      // weights w[rf][s] exactly as the forward stores them (hard: one-hot arg-max)
+      float wt[2] = {0.f, 0.f};
+      bool star[2] = {false, false};
+      const int bk = o[rf].win & 0x7fff, bs = (o[rf].win >> 15) & 1;
+      if (bk == k) star[bs] = true;
+      if (kLSE) {
+        const float2 wv = arc_weights(ns, P.inv_tau, rf, k, o[rf], arc);
+        wt[0] = wv.x;
+        wt[1] = wv.y;
+      } else {
+        wt[0] = star[0] ? 1.f : 0.f;
+        wt[1] = star[1] ? 1.f : 0.f;
+      }
+      const float a0 = wt[0] * abr[rf], a1 = wt[1] * abr[rf];
+      gm[rf] = a0 + a1;
+      gs[0] += a0;
+      gs[1] += a1;
+      const float se = rf ? ms.w : ms.z;
+#pragma unroll
+      for (int s2 = 0; s2 < 2; ++s2) {
+        const bool cand = s2 == src_tr(rf, u, 0) || (u == 2 && s2 == (rf ^ 1));
+        if (!cand) continue;
+        const Cand c = make_cand(st, ms, rf, s2, ns);
+        const float ac = s2 ? a1 : a0;
+        const float sb = float(ns) * ac + (star[s2] ? sbr[rf] : 0.f);
+        const float inv = c.sig > 0.f ? 1.f / c.sig : 0.f;
+        dsg[rf] += sb * se * inv;
+        gsig[s2] += -float(ns) * ac + sb * sig_j[s2] * inv;
+      }
+    }
+    const int32_t arcid = __ldg(P.fin_arc + b0 + k);
+    if (gm[0] != 0.f || gm[1] != 0.f) reinterpret_cast<float2*>(P.d_mean)[arcid] = make_float2(gm[0], gm[1]);
+    reinterpret_cast<float2*>(Q.d_sigma)[arcid] = make_float2(dsg[0], dsg[1]);
+    if ((w >> kHeavyBit) & 1) {
+      long long* acc = Q.hacc4 + 4 * size_t(__ldg(P.heavy_slot + (w & kSrcMask)));
+      atomicAdd(reinterpret_cast<unsigned long long*>(acc + 0), (unsigned long long)__double2ll_rn(double(gs[0]) * kFixH));
+      atomicAdd(reinterpret_cast<unsigned long long*>(acc + 1), (unsigned long long)__double2ll_rn(double(gs[1]) * kFixH));
+      atomicAdd(reinterpret_cast<unsigned long long*>(acc + 2), (unsigned long long)__double2ll_rn(double(gsig[0]) * kFixH));
+      atomicAdd(reinterpret_cast<unsigned long long*>(acc + 3), (unsigned long long)__double2ll_rn(double(gsig[1]) * kFixH));
+    } else {
+      // the mean channel carries the main backward's parity-bit truncation (LSB cleared)
+      Q.g4[b0 + k] = make_float4(stripf(__float_as_uint(gs[0])), stripf(__float_as_uint(gs[1])), gsig[0], gsig[1]);
+    }
+  }
+}
+
 // Written in canonical order (per-level schedule) and in head order (folded).
 __global__ void seed_kernel(int num_ep, const int32_t* __restrict__ ep_pin, const int32_t* __restrict__ ep_head,
                             const float* __restrict__ slack, const uint8_t* __restrict__ rf_star,
@@ -1720,12 +1844,13 @@ int launch_forward(DevGraph& g, float n_sigma, float tau, int schedule, void* st
   return launch_slack(g, stream);
 }
 
-int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float* d_src,
+int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float* d_arc_sigma, float* d_src,
                     void* stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   cudaError_t e = cudaSuccess;
   if (g.e > 0) {
     e = cudaMemsetAsync(d_arc_mean, 0, sizeof(float) * 2 * size_t(g.e), st);
+    if (e == cudaSuccess && d_arc_sigma) e = cudaMemsetAsync(d_arc_sigma, 0, sizeof(float) * 2 * size_t(g.e), st);
     if (e != cudaSuccess) return int(e);
   }
   if (d_src) {
@@ -1739,6 +1864,36 @@ int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float*
     if (err) return err;
   }
   if (g.n == 0) return 0;
+  if (d_arc_sigma) {   // sigma channel: per-level launches of bwds_kernel (canonical order)
+    if (!g.g4) {
+      e = cudaMalloc(&g.g4, sizeof(float4) * std::max<size_t>(size_t(g.e), 1));
+      if (e == cudaSuccess) e = cudaMalloc(&g.hacc4, sizeof(long long) * 4 * size_t(std::max(g.num_heavy, 1)));
+      if (e == cudaSuccess) e = cudaMemset(g.hacc4, 0, sizeof(long long) * 4 * size_t(std::max(g.num_heavy, 1)));
+      if (e != cudaSuccess) return int(e);
+    }
+    KParams P = make_params(g, true);
+    P.n_sigma = g.last_n_sigma;
+    P.tau = g.last_tau;
+    P.inv_tau = g.last_tau > 0.f ? 1.0 / double(g.last_tau) : 0.0;
+    P.d_mean = d_arc_mean;
+    P.d_src = d_src;
+    SigParams Q{};
+    Q.g4 = reinterpret_cast<float4*>(g.g4);
+    Q.hacc4 = g.hacc4;
+    Q.d_sigma = d_arc_sigma;
+    for (int l = g.num_levels - 1; l >= 0; --l) {
+      Q.level = l;
+      Q.lo = g.host.level_ptr[l];
+      Q.hi = g.host.level_ptr[l + 1];
+      const int blocks = (Q.hi - Q.lo + 255) / 256;
+      if (blocks == 0) continue;
+      if (g.last_tau > 0.f) bwds_kernel<true><<<blocks, 256, 0, st>>>(P, Q);
+      else bwds_kernel<false><<<blocks, 256, 0, st>>>(P, Q);
+      const int err = int(cudaGetLastError());
+      if (err) return err;
+    }
+    return 0;
+  }
   KParams P = make_params(g, true);
   P.n_sigma = g.last_n_sigma;
   P.tau = g.last_tau;

@@ -358,3 +358,71 @@ def test_stage_folded_shapes(tau):
     mask = at if tau == 0 else np.zeros_like(at)
     err = np.abs(a.d_mean - b["d_mean"])
     assert ((err <= 1e-3 * np.maximum(np.abs(b["d_mean"]), 1)) | mask).all()
+
+
+def _sigma_case(g, tau):
+    G = insta.Graph(g)
+    G.forward(NS, tau)
+    d0, dsrc0 = (x.cpu().numpy() for x in G.backward(want_src=True))
+    d1, ds, dsrc1 = (x.cpu().numpy() for x in G.backward(want_src=True, want_sigma=True))
+    G.close()
+    # the sigma pass reproduces the mean channel bit for bit
+    assert np.array_equal(d0, d1) and np.array_equal(dsrc0, dsrc1)
+    b = oracle.backward(g, NS, tau)
+    mask = oracle.tie_taint(g, NS, eps=1e-4, margin=0.05)[1] if tau == 0 else np.zeros(ds.shape, bool)
+    err = np.abs(ds - b["d_sigma"])
+    bad = (err > 1e-3 * np.maximum(np.abs(b["d_sigma"]), 1)) & ~mask
+    assert not bad.any(), (err[bad].max(), int(bad.sum()))
+    assert mask.mean() < 0.01
+    return ds, b["d_sigma"]
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C2"])
+@pytest.mark.parametrize("tau", [0.0, 1.0])
+def test_sigma_gradient_parity(cfg, tau):
+    """dTNS/d(arc sigma) (reading R1) vs the fp64 oracle."""
+    ds, ref = _sigma_case(synth.generate(cfg), tau)
+    assert np.count_nonzero(ref) > 0
+
+
+@pytest.mark.parametrize("tau", [0.0, 1.0])
+def test_sigma_gradient_shapes(tau):
+    """Heavy driver (fixed-point accumulation of both channels), wide non-unate
+    fanin, folded-pin shapes and the appendix example (sigma at a zero-sigma arc)."""
+    _sigma_case(_star(3000), tau)
+    _sigma_case(_fold_shapes(), tau)
+    for seed in range(4):
+        _sigma_case(bf.tiny_dag(seed, n_pins=9), tau)
+
+
+@pytest.mark.parametrize("mode", ["hard", "lse_tau1"])
+def test_appendix_a_gpu(mode):
+    """The hand-worked example (tests/golden/appendix_a.json):
+    arrivals, slack, dTNS/dmean and dTNS/dsigma from the GPU path."""
+    import json
+    import os
+    d = json.load(open(os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden", "appendix_a.json")))
+    g = types.SimpleNamespace(
+        num_pins=d["num_pins"], arc_from=np.array(d["arc_from"], np.int32), arc_to=np.array(d["arc_to"], np.int32),
+        arc_unate=np.array(d["arc_unate"], np.uint8), arc_class=None,
+        arc_mean=np.array(d["arc_mean"], np.float32), arc_sigma=np.array(d["arc_sigma"], np.float32),
+        src_mean=np.array(d["src_mean"], np.float32), src_sigma=np.array(d["src_sigma"], np.float32),
+        ep_pin=np.array(d["ep_pin"], np.int32), ep_rat=np.array(d["ep_rat"], np.float32))
+    h = d[mode]
+    tau = h.get("tau", 0.0)
+    G = insta.Graph(g)
+    G.forward(d["n_sigma"], tau)
+    A = G.arrivals()[0].cpu().numpy()
+    for name, pin in (("A_y", 2), ("A_z", 3), ("A_w", 4)):
+        assert np.allclose(A[pin], h[name], atol=1e-3)
+    dm, ds = (x.cpu().numpy() for x in G.backward(want_sigma=True))
+    G.close()
+    want_m = np.zeros((5, 2))
+    want_s = np.zeros((5, 2))
+    for k, v in h["d_mean_nonzero"].items():
+        e, r = map(int, k.split(","))
+        want_m[e, r] = v
+    for k, v in h["d_sigma_nonzero"].items():
+        e, r = map(int, k.split(","))
+        want_s[e, r] = v
+    assert np.allclose(dm, want_m, atol=1e-3) and np.allclose(ds, want_s, atol=1e-3)

@@ -50,6 +50,14 @@ for name in ("fwd_trace.bin", "bwd_trace.bin"):
     print("  per item: gather phase median %.2f us (p99 %.2f), compute phase median %.2f us (p99 %.2f)" % (
         np.median(gather[has_g]) / 1e3, np.percentile(gather[has_g], 99) / 1e3,
         np.median(comp[has_g]) / 1e3, np.percentile(comp[has_g], 99) / 1e3))
+    s3 = t[..., 3] - t0
+    has3 = has_g & (t[..., 3] > 0)
+    if has3.any():   # forward: slot 3 = stale words re-polled and folded pins computed
+        poll = np.where(has3, s3 - s1, 0)
+        rnd = np.where(has3, s2 - s3, 0)
+        print("  forward split: poll+fold median %.2f us (p90 %.2f), rounds median %.2f us (p90 %.2f)" % (
+            np.median(poll[has3]) / 1e3, np.percentile(poll[has3], 90) / 1e3,
+            np.median(rnd[has3]) / 1e3, np.percentile(rnd[has3], 90) / 1e3))
     end_max = s2.max(axis=0)
     start_min = s0.min(axis=0)
     inc = np.diff(np.concatenate([[0], end_max]))
