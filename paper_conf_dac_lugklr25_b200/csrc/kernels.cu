@@ -1001,6 +1001,9 @@ struct BwdfStage {
   int32_t lptr[kBwdPins + 8];   // light fanout rows of the heads
   int32_t lfo[kBwdFanout + 8];  // adjoint word positions of those rows
   int32_t hptr[kBwdPins + 8];   // entry rows of the heads
+  int32_t pin[kBwdPins + 8];    // canonical pin of each head (arg-max / source gathers)
+  int32_t qpos[kBwdArcs + 8];   // fanin position of each entry's arc e (weights, adjoint word)
+  int32_t f[kBwdArcs + 8];      // folded pin word of each entry (arg-max gather)
 };
 constexpr int kEntPerThread = kBwdArcs / kThreads;
 constexpr int kHeadsPerThread = kBwdPins / kThreads;
@@ -1014,11 +1017,18 @@ __device__ __forceinline__ void bwdf_prefetch(const KParams& P, BwdfStage* st, u
   if (!bwd_staged(A, B)) return;
   const Window wl = window(A.x, A.y + 1, 4);   // lfo_ptr and hd_ptr: same head window
   const Window wf = window(A.z, A.w, 4);
+  const Window wh = window(A.x, A.y, 4);
+  const Window wx = window(B.x, B.y, 4);
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-  mbar_expect_tx(full, 2 * wl.bytes + wf.bytes);
+  mbar_expect_tx(full, 2 * wl.bytes + wf.bytes + wh.bytes + (kLSE ? 1 : 2) * wx.bytes);
   bulk_g2s(st->lptr, P.lfo_ptr + wl.start, wl.bytes, full);
   bulk_g2s(st->hptr, P.fanin_ptr + wl.start, wl.bytes, full);
   if (wf.bytes) bulk_g2s(st->lfo, P.lfo + wf.start, wf.bytes, full);
+  bulk_g2s(st->pin, P.hd_pin + wh.start, wh.bytes, full);
+  if (wx.bytes) {
+    bulk_g2s(st->qpos, P.ext_qpos + wx.start, wx.bytes, full);
+    if (!kLSE) bulk_g2s(st->f, P.ext_f + wx.start, wx.bytes, full);
+  }
 }
 
 // Eq 6 sink side of one arc with sink adjoint ab: weights w[rf][s] (hard: the
@@ -1068,10 +1078,11 @@ struct EntryIn {
   float4 w, fw;
 };
 
+// qpos and f: from the staged item (S != nullptr) or global
 template <bool kLSE>
-__device__ __forceinline__ EntryIn load_entry(const KParams& P, int x) {
+__device__ __forceinline__ EntryIn load_entry(const KParams& P, int x, int32_t qpos, int32_t f) {
   EntryIn e;
-  e.qpos = __ldg(P.ext_qpos + x);
+  e.qpos = qpos;
   e.bw = __ldg(P.ext_bw + x);
   e.arc = __ldg(P.ext_arc + x);
   e.farc = __ldg(P.ext_farc + x);
@@ -1082,7 +1093,7 @@ __device__ __forceinline__ EntryIn load_entry(const KParams& P, int x) {
     e.w = __ldcg(P.wts + e.qpos);
     if (e.farc >= 0) e.fw = __ldcg(P.wts + e.fq);
   } else if (e.farc >= 0) {
-    e.fsel = win_sel(__ldcg(P.win + (__ldg(P.ext_f + x) & kSrcMask)), 0);   // folded pin: one fanin arc
+    e.fsel = win_sel(__ldcg(P.win + (f & kSrcMask)), 0);   // folded pin: one fanin arc
   }
   return e;
 }
@@ -1136,12 +1147,16 @@ __global__ void __launch_bounds__(kThreads, 1) bwdf_kernel(KParams P) {
     trace_stamp(P, c, nsteps, t, 0);
     const int np = A.y - A.x;
     if (np > 0 && !(B.w & kItemDirect)) {
+      mbar_wait(&full[buf], phase[buf]);
+      phase[buf] ^= 1u;
+      const BwdfStage& S = stage[buf];
+      const int lo = A.x & 3, fo = A.z & 3, xo = B.x & 3;
       // entry and head inputs: independent of the dependency chain, issued first
       EntryIn ein[kEntPerThread];
 #pragma unroll
       for (int j = 0; j < kEntPerThread; ++j) {
-        const int x = B.x + tid + j * kThreads;
-        if (x < B.y) ein[j] = load_entry<kLSE>(P, x);
+        const int xr = tid + j * kThreads;
+        if (B.x + xr < B.y) ein[j] = load_entry<kLSE>(P, B.x + xr, S.qpos[xo + xr], kLSE ? 0 : S.f[xo + xr]);
       }
       int32_t hpin[kHeadsPerThread], hslot[kHeadsPerThread], hwin[kHeadsPerThread];
       float2 hsd[kHeadsPerThread];
@@ -1149,16 +1164,12 @@ __global__ void __launch_bounds__(kThreads, 1) bwdf_kernel(KParams P) {
       for (int j = 0; j < kHeadsPerThread; ++j) {
         const int h = A.x + tid + j * kThreads;
         if (h < A.y) {
-          hpin[j] = __ldg(P.hd_pin + h);
+          hpin[j] = S.pin[lo + tid + j * kThreads];
           hslot[j] = __ldg(P.hd_hslot + h);
           hsd[j] = __ldcg(P.hseed + h);
           hwin[j] = kLSE ? 0 : __ldcg(P.win + hpin[j]);
         }
       }
-      mbar_wait(&full[buf], phase[buf]);
-      phase[buf] ^= 1u;
-      const BwdfStage& S = stage[buf];
-      const int lo = A.x & 3, fo = A.z & 3;
       const int nfo = A.w - A.z;
       // (1) gather the sinks' per-arc adjoints of every light fanout entry
       for (int e = tid; e < nfo; e += kThreads)
@@ -1231,7 +1242,7 @@ __global__ void __launch_bounds__(kThreads, 1) bwdf_kernel(KParams P) {
       __syncthreads();
       if (B.z > 0) {
         for (int x = B.x + tid; x < B.y; x += kThreads) {
-          const EntryIn e = load_entry<kLSE>(P, x);
+          const EntryIn e = load_entry<kLSE>(P, x, __ldg(P.ext_qpos + x), kLSE ? 0 : __ldg(P.ext_f + x));
           bwdf_entry<kLSE>(P, htab, e, s_ab, kLSE ? 0 : win_sel(s_win, x - B.x));
         }
       }
