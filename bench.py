@@ -126,6 +126,37 @@ def bwd_bytes(N, E, E_light, P, nnz_arcs, lse):
             + 8 * nnz_arcs)               # nonzero d_mean scatter
 
 
+def fwd_bytes_folded(sc, N, E, n_src, P, lse):
+    """insta_forward, stage-folded persistent schedule: per head a row pointer
+    and its pin (+ first fanin position in LSE mode); per entry a source word, the record of its
+    arc and ONE source-state gather; a folded pin adds its word and the record of its fanin arc;
+    every pin's state is written once."""
+    H, X, F = sc["num_heads"], sc["num_entries"], sc["num_folded"]
+    return (8 * H + (4 * H if lse else 0)     # head row pointer + pin (+ first fanin position)
+            + 20 * X                          # per entry: source word 4 + record of e 16
+            + 24 * X                          # per entry: source-state gather
+            + F * (20 + (4 if lse else 0))    # folded pin: word 4 + record of e' 16 (+ fanin position)
+            + 24 * N                          # state write (every pin, folded ones included)
+            + 16 * n_src
+            + (16 * E if lse else 4 * (N - n_src))   # Eq 6 weights per arc (LSE) / arg-max per pin (hard)
+            + 41 * P)
+
+
+def bwd_bytes_folded(sc, N, E, E_light, P, nnz_arcs, lse):
+    """insta_backward, stage-folded schedule: per head 24 B (light-fanout and entry row pointers,
+    pin, heavy slot, seed) + its arg-max (hard); per entry 20 B (fanin position, source word,
+    arc ids of e and e', position of e') + the folded pin word (hard); Eq 6 weights of every arc
+    (LSE) or the folded pins' arg-max (hard); one adjoint word written per entry."""
+    H, X, F = sc["num_heads"], sc["num_entries"], sc["num_folded"]
+    return (8 * E + 25 * P                    # d_mean zero fill; seeds (canonical + head order)
+            + (24 if lse else 28) * H
+            + (20 if lse else 24) * X
+            + (16 * E if lse else 4 * F)
+            + 12 * E_light                    # pull: fanout entry 4 + per-arc adjoint gather 8
+            + 8 * X                           # per-arc adjoint write
+            + 8 * nnz_arcs)                   # nonzero d_mean scatter
+
+
 def cpu_oracle_sample(cfg_name, sample_pins, tau):
     """fp64 CPU oracle (single thread) fwd + slack + bwd on a bounded sample of the workload:
     the same generator recipe (depth, fanout law, endpoint fraction) at `sample_pins` pins."""
@@ -253,8 +284,13 @@ def main():
     fo = np.bincount(g.arc_from, minlength=N)
     E_light = int(fo[fo <= HEAVY_FANOUT].sum())
     lse = args.tau > 0
-    fb = fwd_bytes(N, E, n_src, P, lse)
-    bb = bwd_bytes(N, E, E_light, P, nnz_arcs, lse)
+    sched = G.schedule()
+    if args.schedule == 0:   # stage-folded persistent passes
+        fb = fwd_bytes_folded(sched, N, E, n_src, P, lse)
+        bb = bwd_bytes_folded(sched, N, E, E_light, P, nnz_arcs, lse)
+    else:                    # one launch per level
+        fb = fwd_bytes(N, E, n_src, P, lse)
+        bb = bwd_bytes(N, E, E_light, P, nnz_arcs, lse)
     peak, peak_kind = _peaks()
     fwd_gbs = fb / (fwd_ms * 1e-3) / 1e9
     bwd_gbs = bb / (bwd_ms * 1e-3) / 1e9
@@ -357,7 +393,8 @@ def main():
             "config": {"workload": f"{cfg.name}: synthetic 3nm-shaped timing graph, {N} pins, {E} arcs, "
                                    f"{P} endpoints, {G.num_levels} levels",
                        "pins": N, "arcs": E, "endpoints": P, "levels": G.num_levels, "tau": args.tau,
-                       "n_sigma": 3.0, "schedule": ["persistent", "per-level"][args.schedule],
+                       "n_sigma": 3.0, "schedule": ["persistent, stage-folded", "per-level"][args.schedule],
+                       "super_levels": sched["num_super_levels"], "folded_pins": sched["num_folded"],
                        "parallelism": f"replicas x{world}", "l2": "working set > 126 MB L2 (no flush needed)",
                        "tns": s.tns, "wns": s.wns, "violations": s.num_violations},
             "fwd_ms": fwd_ms, "bwd_ms": bwd_ms, "fwd_bwd_ms": ms_step,

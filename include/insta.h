@@ -121,6 +121,20 @@ insta_status insta_graph_export(const insta_graph* g, int32_t* level_of_pin, int
 insta_status insta_graph_sizes(const insta_graph* g, int32_t* num_pins, int64_t* num_arcs,
                                int32_t* num_endpoints, int32_t* num_levels);
 
+/* Schedule of the persistent passes (host; DESIGN.md §4 "stage folding"):
+ * pins with one fanin and one fanout arc that are not endpoints are computed
+ * inside their sink's work item, so the dependent depth is num_super_levels
+ * instead of num_levels.  Reported for byte models and diagnostics. */
+typedef struct {
+  int32_t num_heads;          /* pins with their own work item (not folded) */
+  int32_t num_super_levels;   /* dependent steps of the folded schedule */
+  int64_t num_entries;        /* fanin arcs of heads (= num_arcs - num_folded) */
+  int64_t num_folded;         /* folded pins */
+  int64_t num_light_fanout;   /* fanout entries pulled without atomics */
+  int32_t fwd_steps, bwd_steps;   /* persistent item steps per pass */
+} insta_schedule;
+insta_status insta_graph_schedule(const insta_graph* g, insta_schedule* out);
+
 /* Forward: statistical arrival propagation (Eq 1-3, Alg 1 with K = 1, or
  * Eq 4) over all levels, then endpoint slack = RAT - A, min over rf (ties ->
  * R), and WNS/TNS.  o may be NULL (defaults n_sigma 3, tau 0, schedule 0).

@@ -100,6 +100,12 @@ class Graph:
         check(self.lib.insta_graph_sizes(self._h, None, None, None, ctypes.byref(nl)), "insta_graph_sizes")
         self.num_levels = int(nl.value)
 
+    def schedule(self) -> dict:
+        """insta_graph_schedule: the stage-folded schedule of the persistent passes."""
+        sc = _capi.insta_schedule()
+        check(self.lib.insta_graph_schedule(self._h, ctypes.byref(sc)), "insta_graph_schedule")
+        return {name: int(getattr(sc, name)) for name, _ in sc._fields_}
+
     # ------------------------------------------------------------------ lifetime
     def close(self):
         if getattr(self, "_h", None):

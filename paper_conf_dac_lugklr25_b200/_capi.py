@@ -48,6 +48,12 @@ class insta_scenario(ctypes.Structure):
                 ("n_delta", ctypes.c_int32), ("delta_arc", c_vp), ("delta_mean", c_vp), ("delta_sigma", c_vp)]
 
 
+class insta_schedule(ctypes.Structure):
+    _fields_ = [("num_heads", ctypes.c_int32), ("num_super_levels", ctypes.c_int32),
+                ("num_entries", ctypes.c_int64), ("num_folded", ctypes.c_int64),
+                ("num_light_fanout", ctypes.c_int64), ("fwd_steps", ctypes.c_int32), ("bwd_steps", ctypes.c_int32)]
+
+
 # name -> (restype, argtypes); every symbol declared in include/insta.h
 SIGNATURES = {
     "insta_levelize": (ctypes.c_int, [ctypes.c_int32, ctypes.c_int64, c_vp, c_vp, c_vp, c_vp, c_vp, c_vp,
@@ -56,6 +62,7 @@ SIGNATURES = {
     "insta_graph_destroy": (None, [c_vp]),
     "insta_graph_export": (ctypes.c_int, [c_vp, c_vp, c_vp, c_vp, c_vp, c_vp, c_vp]),
     "insta_graph_sizes": (ctypes.c_int, [c_vp, c_vp, c_vp, c_vp, c_vp]),
+    "insta_graph_schedule": (ctypes.c_int, [c_vp, ctypes.POINTER(insta_schedule)]),
     "insta_forward": (ctypes.c_int, [c_vp, ctypes.POINTER(insta_opts), c_vp, ctypes.POINTER(insta_summary)]),
     "insta_slack": (ctypes.c_int, [c_vp, c_vp, c_vp, c_vp, ctypes.POINTER(insta_summary)]),
     "insta_arrivals": (ctypes.c_int, [c_vp, c_vp, c_vp, c_vp, c_vp]),

@@ -60,7 +60,8 @@ void free_graph(insta::DevGraph& d) {
                   d.hd_pin,    d.hd_ptr,    d.hd_q0,     d.ext_w,      d.ext_ms,    d.ext_f,
                   d.ext_fms,   d.ext_fq,    d.arc_xpos,  d.fwdf_a,     d.fwdf_b,    d.hd_hslot,
                   d.hlfo_ptr,  d.hlfo,      d.ext_qpos,  d.ext_bw,     d.ext_arc,   d.ext_farc,
-                  d.ep_head,   d.hseed,     d.bwdf_a,    d.bwdf_b,    d.g4,        d.hacc4};
+                  d.ep_head,   d.hseed,     d.bwdf_a,    d.bwdf_b,    d.g4,        d.hacc4,
+                  d.ext_flags, d.bfwdf_a,   d.bfwdf_b,   d.b_ov_key};
   for (void* p : ptrs)
     if (p) cudaFree(p);
 }
@@ -241,6 +242,11 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   d.num_heads = int32_t(fold.hd_pin.size());
   d.num_slevels = int32_t(fold.slevel_ptr.size()) - 1;
   d.num_ext = int64_t(fold.ext_w.size());
+  d.h_arc_xpos = fold.arc_xpos;
+  std::vector<uint8_t> ext_flags(fold.ext_w.size(), 0);
+  for (size_t x = 0; x < ext_flags.size(); ++x)
+    ext_flags[x] = uint8_t((arc_class[fold.ext_arc[x]] ? 1 : 0) |
+                           (fold.ext_farc[x] >= 0 && arc_class[fold.ext_farc[x]] ? 4 : 0));
 
   // ---- device: grid, items, upload ------------------------------------------------
   cudaError_t e = cudaSetDevice(d.device);
@@ -308,6 +314,9 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   UP(d.ep_head, fold.ep_head.data(), fold.ep_head.size());
   ZERO(d.hseed, fold.hd_pin.size());
   UP(d.bwdf_a, d.bwdf_items.a.data(), d.bwdf_items.a.size());
+  UP(d.ext_flags, ext_flags.data(), ext_flags.size());
+  UP(d.bfwdf_a, d.bfwdf_items.a.data(), d.bfwdf_items.a.size());
+  UP(d.bfwdf_b, d.bfwdf_items.b.data(), d.bfwdf_items.b.size());
   UP(d.bwdf_b, d.bwdf_items.b.data(), d.bwdf_items.b.size());
   ZERO(d.done_fwd, std::max(d.num_levels, 1));
   ZERO(d.done_bwd, std::max(d.num_levels, 1));
@@ -364,6 +373,19 @@ insta_status insta_graph_sizes(const insta_graph* g, int32_t* num_pins, int64_t*
   if (num_arcs) *num_arcs = g->d.e;
   if (num_endpoints) *num_endpoints = g->d.num_ep;
   if (num_levels) *num_levels = g->d.num_levels;
+  return INSTA_OK;
+}
+
+insta_status insta_graph_schedule(const insta_graph* g, insta_schedule* out) {
+  if (!g || !out) return fail(INSTA_E_ARG, "graph_schedule: NULL argument");
+  const insta::DevGraph& d = g->d;
+  out->num_heads = d.num_heads;
+  out->num_super_levels = d.num_slevels;
+  out->num_entries = d.num_ext;
+  out->num_folded = int64_t(d.n) - d.num_heads;
+  out->num_light_fanout = d.e_light;
+  out->fwd_steps = d.fwdf_items.num_steps;
+  out->bwd_steps = d.bwdf_items.num_steps;
   return INSTA_OK;
 }
 
@@ -493,7 +515,7 @@ insta_status insta_forward_batch(insta_graph* g, int32_t num_scenarios, const in
   for (int32_t b0 = 0; b0 < num_scenarios; b0 += kL) {
     const int nb = std::min(kL, num_scenarios - b0);
     float par[3 * kL];
-    std::vector<int32_t> ov_ptr(kL + 1, 0), ov_pos;
+    std::vector<int32_t> ov_ptr(kL + 1, 0), ov_pos, ov_key;
     std::vector<float4> ov_ms;
     for (int s = 0; s < kL; ++s) {
       const insta_scenario* x = s < nb ? &sc[b0 + s] : nullptr;
@@ -503,13 +525,14 @@ insta_status insta_forward_batch(insta_graph* g, int32_t num_scenarios, const in
       if (x) {
         for (int32_t k = 0; k < x->n_delta; ++k) {
           ov_pos.push_back(d.h_arc_pos[x->delta_arc[k]]);
+          ov_key.push_back(d.h_arc_xpos[x->delta_arc[k]]);
           ov_ms.push_back(make_float4(x->delta_mean[2 * k], x->delta_mean[2 * k + 1], x->delta_sigma[2 * k],
                                       x->delta_sigma[2 * k + 1]));
         }
       }
       ov_ptr[s + 1] = int32_t(ov_pos.size());
     }
-    int err = insta::launch_forward_batch(d, nb, par, ov_ptr, ov_pos, ov_ms, tau, summaries + 3 * size_t(b0),
+    int err = insta::launch_forward_batch(d, nb, par, ov_ptr, ov_pos, ov_key, ov_ms, tau, summaries + 3 * size_t(b0),
                                           d_arc_mean_sum, cuda_stream);
     if (err) return cuda_fail(err, "forward_batch");
   }

@@ -52,9 +52,16 @@ struct BParams {
   const int32_t* __restrict__ heavy_fo;
   const int32_t* __restrict__ ep_of_pin;
   const float4* __restrict__ src_ms;
+  // stage-folded forward (fold.cpp): head pins and first fanin positions,
+  // folded pin word / fanin position / record of e' per entry
+  const int32_t* __restrict__ hd_pin;
+  const int32_t* __restrict__ hd_q0;
+  const int32_t* __restrict__ ext_f;
+  const int32_t* __restrict__ ext_fq;
+  const float4* __restrict__ ext_fms;
   const float* __restrict__ sc;            // [3][32]: n_sigma, derate_cell, derate_net
   const int32_t* __restrict__ ov_ptr;      // [33] overrides of scenario s: [ov_ptr[s], ov_ptr[s+1])
-  const int32_t* __restrict__ ov_pos;      // fanin positions, ascending within a scenario
+  const int32_t* __restrict__ ov_pos;      // arc keys: fanin positions (backward) / entry keys 2x, 2x+1 (forward)
   const float4* __restrict__ ov_ms;        // override arc records
   PinState* bstate;                        // [n][32]
   int32_t* bwin;                           // [n][32]
@@ -102,11 +109,20 @@ __device__ __forceinline__ void storeb(const BParams& P, int i, int s, double m0
 }
 
 // ---------------------------------------------------------------- forward
+// Stage-folded schedule (fold.cpp, as kernels.cu fwd_kernel<., true>): items
+// are head ranges per super-level; an entry through a folded pin p first
+// computes p for the lane's scenario from the gathered source words (merge1,
+// the nf = 1 merge) and stores it, then continues with p's words.  Arc keys
+// for the sparse overrides: 2x for the entry's arc e, 2x + 1 for e'.
 struct BFwdStage {
-  int32_t ptr[kBFwdPins + 8];
-  int32_t src[kBFwdArcs + 8];
-  uint8_t flags[kBFwdArcs + 32];
-  float4 ms[kBFwdArcs];
+  int32_t ptr[kBFwdPins + 8];     // entry rows of the heads
+  int32_t pin[kBFwdPins + 8];     // canonical pin of each head
+  int32_t src[kBFwdArcs + 8];     // entry source word (fold bit 29)
+  int32_t f[kBFwdArcs + 8];       // folded pin | unate(e') << 30
+  int32_t fq[kBFwdArcs + 8];      // fanin position of e'
+  uint8_t flags[kBFwdArcs + 32];  // bit 0/1: e cell / overridden, bit 2/3: e'
+  float4 ms[kBFwdArcs];           // record of e
+  float4 fms[kBFwdArcs];          // record of e'
 };
 constexpr size_t kBFwdSmem = 2 * sizeof(BFwdStage);
 
@@ -119,16 +135,21 @@ __device__ __forceinline__ void bfwd_prefetch(const BParams& P, BFwdStage* st, u
   const int4 B = __ldg(P.item_b + size_t(step) * P.grid + c);
   if (!bfwd_staged(A, B)) return;
   const Window wp = window(A.x, A.y + 1, 4);
+  const Window wh = window(A.x, A.y, 4);
   const Window ws = window(A.z, A.w, 4);
   const Window wf = window(A.z, A.w, 1);
   const uint32_t bms = uint32_t(A.w - A.z) * 16u;
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-  mbar_expect_tx(full, wp.bytes + ws.bytes + wf.bytes + bms);
+  mbar_expect_tx(full, wp.bytes + wh.bytes + (ws.bytes ? 3 * ws.bytes + wf.bytes + 2 * bms : 0u));
   bulk_g2s(st->ptr, P.fanin_ptr + wp.start, wp.bytes, full);
+  bulk_g2s(st->pin, P.hd_pin + wh.start, wh.bytes, full);
   if (ws.bytes) {
     bulk_g2s(st->src, P.fin_src + ws.start, ws.bytes, full);
+    bulk_g2s(st->f, P.ext_f + ws.start, ws.bytes, full);
+    bulk_g2s(st->fq, P.ext_fq + ws.start, ws.bytes, full);
     bulk_g2s(st->flags, P.fin_flags + wf.start, wf.bytes, full);
     bulk_g2s(st->ms, P.fin_ms + A.z, bms, full);
+    bulk_g2s(st->fms, P.ext_fms + A.z, bms, full);
   }
 }
 
@@ -146,6 +167,20 @@ __device__ __forceinline__ float2 arc_rf_weights_b(const BParams& P, double ns, 
 }
 
 constexpr int kRegArcsB = 4;
+
+// folded pin p behind entry x for scenario lane s (merge1 = the nf = 1 merge)
+template <bool kLSE>
+__device__ __forceinline__ Raw foldb(const BParams& P, int32_t fw, int32_t fq, float4 fm, uint32_t fl, int x, int s,
+                                  double ns, float dcell, float dnet, Raw rj) {
+  const float4 ms = scen_arc(P, fm, fl >> 2, 2 * x + 1, s, dcell, dnet);
+  Merge1 m;
+  merge1<kLSE>(unpack(rj), int(uint32_t(fw) >> kUnateShift), ms, ns, double(P.tau), P.inv_tau, m);
+  const int pp = fw & kSrcMask;
+  storeb(P, pp, s, m.mu[0], m.mu[1], m.var[0], m.var[1]);
+  if (!kLSE) P.bwin[size_t(pp) * kLanes + s] = m.win;
+  else P.bwts[size_t(fq) * kLanes + s] = m.wt;
+  return m.stored(P.par);
+}
 
 template <bool kLSE>
 __global__ void __launch_bounds__(kThreads, 1) fwdb_kernel(BParams P) {
@@ -172,7 +207,7 @@ __global__ void __launch_bounds__(kThreads, 1) fwdb_kernel(BParams P) {
     const int4 B = __ldg(P.item_b + size_t(k) * P.grid + c);
     if (tid == 0 && t + 1 < nsteps) bfwd_prefetch(P, &stage[buf ^ 1], &full[buf ^ 1], k + 1, c);
     if (A.y > A.x) {
-      if (B.x == 0) {
+      if (B.x == 0) {   // startpoints: heads 0..num_src-1 are canonical pins 0..num_src-1
         for (int i = A.x + warp; i < A.y; i += kThreads / 32) {
           if (!lane_on) continue;
           const float4 v = __ldg(P.src_ms + i);
@@ -187,50 +222,84 @@ __global__ void __launch_bounds__(kThreads, 1) fwdb_kernel(BParams P) {
         const BFwdStage& S = stage[buf];
         const int po = A.x & 3, so = A.z & 3, fo = A.z & 15;
         for (int p = warp; p < A.y - A.x && lane_on; p += kThreads / 32) {
-          const int i = A.x + p;
-          int b0, nf;
+          const int h = A.x + p;
+          int b0, nf, i;
           if (staged) {
             b0 = S.ptr[po + p] - A.z;
             nf = S.ptr[po + p + 1] - A.z - b0;
+            i = S.pin[po + p];
           } else {
-            b0 = __ldg(P.fanin_ptr + i) - A.z;
-            nf = __ldg(P.fanin_ptr + i + 1) - A.z - b0;
+            b0 = __ldg(P.fanin_ptr + h) - A.z;
+            nf = __ldg(P.fanin_ptr + h + 1) - A.z - b0;
+            i = __ldg(P.hd_pin + h);
           }
+          // entry kk: source word, flags, record of e (and of e' and the folded pin)
+          auto ent = [&](int kk, int32_t& w, uint32_t& fl, float4& m0) {
+            if (staged) {
+              w = S.src[so + b0 + kk];
+              fl = S.flags[fo + b0 + kk];
+              m0 = S.ms[b0 + kk];
+            } else {
+              const int x = A.z + b0 + kk;
+              w = __ldg(P.fin_src + x);
+              fl = __ldg(P.fin_flags + x);
+              m0 = __ldg(P.fin_ms + x);
+            }
+          };
+          // folded pin behind entry kk: computed for this scenario from the source words
+          auto fold = [&](int kk, uint32_t fl, const Raw& rj) -> Raw {
+            const int x = A.z + b0 + kk;
+            if (staged) return foldb<kLSE>(P, S.f[so + b0 + kk], S.fq[so + b0 + kk], S.fms[b0 + kk], fl, x, s, ns,
+                                           dcell, dnet, rj);
+            return foldb<kLSE>(P, __ldg(P.ext_f + x), __ldg(P.ext_fq + x), __ldg(P.ext_fms + x), fl, x, s, ns, dcell,
+                               dnet, rj);
+          };
           // gather the first kRegArcsB source entries of this scenario together
           Raw rr[kRegArcsB];
-          int32_t ww[kRegArcsB];
+          auto src_word = [&](int kk) { return staged ? S.src[so + b0 + kk] : __ldg(P.fin_src + A.z + b0 + kk); };
+#pragma unroll
+          for (int kk = 0; kk < kRegArcsB; ++kk)
+            if (kk < nf) rr[kk] = ldb_raw(P, src_word(kk) & kSrcMask, s);
 #pragma unroll
           for (int kk = 0; kk < kRegArcsB; ++kk) {
             if (kk < nf) {
-              ww[kk] = staged ? S.src[so + b0 + kk] : __ldg(P.fin_src + A.z + b0 + kk);
-              rr[kk] = ldb_raw(P, ww[kk] & kSrcMask, s);
+              int32_t w;
+              uint32_t fl;
+              float4 m0;
+              ent(kk, w, fl, m0);
+              awaitb(P, w & kSrcMask, s, rr[kk]);
+              if ((w >> kFoldBit) & 1) rr[kk] = fold(kk, fl, rr[kk]);
             }
           }
-#pragma unroll
-          for (int kk = 0; kk < kRegArcsB; ++kk)
-            if (kk < nf) awaitb(P, ww[kk] & kSrcMask, s, rr[kk]);
-          auto arc = [&](int kk, int32_t& w, float4& ms, Raw& r) {
-            const int q = A.z + b0 + kk;
-            float4 m0;
+          // entries past the register window: folded pins are computed (and stored) here once,
+          // the merge below then reads their words back like any other source
+          for (int kk = kRegArcsB; kk < nf; ++kk) {
+            int32_t w;
             uint32_t fl;
-            if (staged) {
-              w = S.src[so + b0 + kk];
-              m0 = S.ms[b0 + kk];
-              fl = S.flags[fo + b0 + kk];
-            } else {
-              w = __ldg(P.fin_src + q);
-              m0 = __ldg(P.fin_ms + q);
-              fl = __ldg(P.fin_flags + q);
+            float4 m0;
+            ent(kk, w, fl, m0);
+            if ((w >> kFoldBit) & 1) {
+              Raw r = ldb_raw(P, w & kSrcMask, s);
+              awaitb(P, w & kSrcMask, s, r);
+              fold(kk, fl, r);
             }
-            ms = scen_arc(P, m0, fl, q, s, dcell, dnet);
+          }
+          auto arc = [&](int kk, int32_t& w, float4& ms, Raw& r) {
+            uint32_t fl;
+            float4 m0;
+            ent(kk, w, fl, m0);
+            ms = scen_arc(P, m0, fl & 3u, 2 * (A.z + b0 + kk), s, dcell, dnet);
             if (kk < kRegArcsB) {
               r = rr[0];
 #pragma unroll
               for (int x = 1; x < kRegArcsB; ++x)
                 if (x == kk) r = rr[x];
             } else {
-              r = ldb_raw(P, w & kSrcMask, s);
-              awaitb(P, w & kSrcMask, s, r);
+              // folded: the pin stored above by this lane; else the source
+              const int src = ((w >> kFoldBit) & 1) ? ((staged ? S.f[so + b0 + kk] : __ldg(P.ext_f + A.z + b0 + kk)) & kSrcMask)
+                                                    : (w & kSrcMask);
+              r = ldb_raw(P, src, s);
+              awaitb(P, src, s, r);
             }
           };
           const RfOut R = pin_rf_b<kLSE>(P, ns, 0, nf, arc);
@@ -239,10 +308,11 @@ __global__ void __launch_bounds__(kThreads, 1) fwdb_kernel(BParams P) {
           if (!kLSE) {
             P.bwin[size_t(i) * kLanes + s] = R.win | (F.win << 16);
           } else {
+            const int q0 = __ldg(P.hd_q0 + h);
             for (int kk = 0; kk < nf; ++kk) {
               const float2 wr = arc_rf_weights_b(P, ns, 0, kk, R, arc);
               const float2 wf = arc_rf_weights_b(P, ns, 1, kk, F, arc);
-              P.bwts[size_t(A.z + b0 + kk) * kLanes + s] = make_float4(wr.x, wr.y, wf.x, wf.y);
+              P.bwts[size_t(q0 + kk) * kLanes + s] = make_float4(wr.x, wr.y, wf.x, wf.y);
             }
           }
         }
@@ -514,6 +584,16 @@ __global__ void set_flag_kernel(int n, const int32_t* __restrict__ pos, uint8_t*
   else flags[pos[k]] &= uint8_t(~bit);
 }
 
+// entry-space keys 2x (arc e) / 2x + 1 (arc e'): overridden bit 1 / bit 3
+__global__ void set_xflag_kernel(int n, const int32_t* __restrict__ key, uint8_t* flags, int on) {
+  const int k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k >= n) return;
+  const int x = key[k] >> 1;
+  const uint8_t bit = (key[k] & 1) ? 8 : 2;
+  if (on) flags[x] |= bit;
+  else flags[x] &= uint8_t(~bit);
+}
+
 // ---------------------------------------------------------------- host side
 template <class K>
 static int set_smem_b(K kernel, size_t bytes) {
@@ -558,12 +638,17 @@ static BParams make_bparams(DevGraph& g, bool bwd) {
   P.n = g.n;
   P.num_levels = g.num_levels;
   P.grid = g.grid;
-  P.item_a = bwd ? g.bwd_a : g.bfwd_a;
-  P.item_b = bwd ? g.bwd_b : g.bfwd_b;
-  P.fanin_ptr = g.fanin_ptr;
-  P.fin_src = g.fin_src;
-  P.fin_ms = g.fin_ms;
-  P.fin_flags = g.fin_flags;
+  P.item_a = bwd ? g.bwd_a : g.bfwdf_a;
+  P.item_b = bwd ? g.bwd_b : g.bfwdf_b;
+  P.fanin_ptr = bwd ? g.fanin_ptr : g.hd_ptr;
+  P.fin_src = bwd ? g.fin_src : g.ext_w;
+  P.fin_ms = bwd ? g.fin_ms : g.ext_ms;
+  P.fin_flags = bwd ? g.fin_flags : g.ext_flags;
+  P.hd_pin = g.hd_pin;
+  P.hd_q0 = g.hd_q0;
+  P.ext_f = g.ext_f;
+  P.ext_fq = g.ext_fq;
+  P.ext_fms = g.ext_fms;
   P.fin_arc = g.fin_arc;
   P.lfo_ptr = g.lfo_ptr;
   P.lfo = g.lfo;
@@ -573,7 +658,7 @@ static BParams make_bparams(DevGraph& g, bool bwd) {
   P.src_ms = g.src_ms;
   P.sc = g.b_sc;
   P.ov_ptr = g.b_ov_ptr;
-  P.ov_pos = g.b_ov_pos;
+  P.ov_pos = bwd ? g.b_ov_pos : g.b_ov_key;
   P.ov_ms = g.b_ov_ms;
   P.bstate = g.b_state;
   P.bwin = g.b_win;
@@ -586,8 +671,9 @@ static BParams make_bparams(DevGraph& g, bool bwd) {
 }
 
 int launch_forward_batch(DevGraph& g, int nb, const float* sc_host /*[3][32]*/, const std::vector<int32_t>& ov_ptr,
-                         const std::vector<int32_t>& ov_pos, const std::vector<float4>& ov_ms, float tau,
-                         double* summaries, float* d_mean_sum, void* stream) {
+                         const std::vector<int32_t>& ov_pos, const std::vector<int32_t>& ov_key,
+                         const std::vector<float4>& ov_ms, float tau, double* summaries, float* d_mean_sum,
+                         void* stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   const bool lse = tau > 0.f, grad = d_mean_sum != nullptr;
   int err = ensure_batch(g, lse, grad);
@@ -598,18 +684,23 @@ int launch_forward_batch(DevGraph& g, int nb, const float* sc_host /*[3][32]*/, 
   const int nov = int(ov_pos.size());
   if (e == cudaSuccess && nov > g.b_ov_cap) {
     cudaFree(g.b_ov_pos);
+    cudaFree(g.b_ov_key);
     cudaFree(g.b_ov_ms);
     g.b_ov_pos = nullptr;
+    g.b_ov_key = nullptr;
     g.b_ov_ms = nullptr;
     e = cudaMalloc(&g.b_ov_pos, sizeof(int32_t) * nov + 64);
+    if (e == cudaSuccess) e = cudaMalloc(&g.b_ov_key, sizeof(int32_t) * nov + 64);
     if (e == cudaSuccess) e = cudaMalloc(&g.b_ov_ms, sizeof(float4) * nov + 64);
     g.b_ov_cap = nov;
   }
   if (e == cudaSuccess && nov > 0) {
     e = cudaMemcpyAsync(g.b_ov_pos, ov_pos.data(), sizeof(int32_t) * nov, cudaMemcpyHostToDevice, st);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(g.b_ov_key, ov_key.data(), sizeof(int32_t) * nov, cudaMemcpyHostToDevice, st);
     if (e == cudaSuccess) e = cudaMemcpyAsync(g.b_ov_ms, ov_ms.data(), sizeof(float4) * nov, cudaMemcpyHostToDevice, st);
     if (e == cudaSuccess) {
       set_flag_kernel<<<(nov + 255) / 256, 256, 0, st>>>(nov, g.b_ov_pos, g.fin_flags, 2, 1);
+      set_xflag_kernel<<<(nov + 255) / 256, 256, 0, st>>>(nov, g.b_ov_key, g.ext_flags, 1);
       e = cudaGetLastError();
     }
   }
@@ -620,7 +711,7 @@ int launch_forward_batch(DevGraph& g, int nb, const float* sc_host /*[3][32]*/, 
   P.inv_tau = lse ? 1.0 / double(tau) : 0.0;
   P.par = (++g.pass_bfwd) & 1u;
   P.step_begin = 0;
-  P.step_end = g.bfwd_items.num_steps;
+  P.step_end = g.bfwdf_items.num_steps;
   if (g.n > 0) {
     void* args[] = {&P};
     e = cudaLaunchCooperativeKernel(lse ? (const void*)fwdb_kernel<true> : (const void*)fwdb_kernel<false>,
@@ -652,6 +743,7 @@ int launch_forward_batch(DevGraph& g, int nb, const float* sc_host /*[3][32]*/, 
   }
   if (nov > 0) {
     set_flag_kernel<<<(nov + 255) / 256, 256, 0, st>>>(nov, g.b_ov_pos, g.fin_flags, 2, 0);
+    set_xflag_kernel<<<(nov + 255) / 256, 256, 0, st>>>(nov, g.b_ov_key, g.ext_flags, 0);
     e = cudaGetLastError();
   }
   return int(e);

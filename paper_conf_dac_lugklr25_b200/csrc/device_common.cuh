@@ -272,6 +272,74 @@ __device__ __forceinline__ RfOut merge_rf(double ns, double tau, double inv_tau,
   return o;
 }
 
+// Merge of a pin with exactly one fanin arc (source words st, unateness u,
+// record ms): the same operation sequence as merge_rf with nf = 1 -- scan
+// (a0, then a1 for a non-unate arc, strict ">"), winner, LSE sum 0 + w0
+// (+ w1), Eq 4 arrival, Eq 6 weights -- with each candidate evaluated once;
+// hard mode with a unate arc has a single candidate, so its corner (and square
+// root) is not needed.  Bit-identical to merge_rf + arc_weights (nf = 1).
+struct Merge1 {
+  double mu[2], var[2];
+  int32_t win;   // arg-max word {R: s << 15, F: << 16}
+  float4 wt;     // Eq 6 weights {w[R][R], w[R][F], w[F][R], w[F][F]} (LSE)
+  __device__ __forceinline__ Raw stored(uint32_t par) const {   // the words a store with parity writes
+    Raw o;
+    o.a = (unsigned long long)__double_as_longlong(with_par(mu[0], par));
+    o.b = (unsigned long long)__double_as_longlong(with_par(mu[1], par));
+    o.c = (unsigned long long)__double_as_longlong(with_par(var[0], par));
+    o.d = (unsigned long long)__double_as_longlong(with_par(var[1], par));
+    return o;
+  }
+};
+
+template <bool kLSE>
+__device__ __forceinline__ void merge1(const Gath& st, int u, const float4& ms, double ns, double tau, double inv_tau,
+                                       Merge1& m) {
+  int win[2];
+  float wt[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
+#pragma unroll
+  for (int rf = 0; rf < 2; ++rf) {
+    const int s0 = src_tr(rf, u, 0);
+    if (!kLSE && u != 2) {
+      const double se = double(rf ? ms.w : ms.z);
+      m.mu[rf] = (s0 ? st.mu1 : st.mu0) + double(rf ? ms.y : ms.x);   // = make_cand(...).mu
+      m.var[rf] = (s0 ? st.v1 : st.v0) + se * se;                       // = make_cand(...).var
+      win[rf] = s0 << 15;
+      continue;
+    }
+    const Cand c0 = make_cand(st, ms, rf, s0, ns);
+    Cand cb = c0;
+    int bs = s0;
+    Cand c1 = c0;
+    if (u == 2) {
+      c1 = make_cand(st, ms, rf, rf ^ 1, ns);
+      if (c1.A > c0.A) {
+        cb = c1;
+        bs = rf ^ 1;
+      }
+    }
+    m.mu[rf] = cb.mu;
+    m.var[rf] = cb.var;
+    win[rf] = bs << 15;
+    if (kLSE) {
+      float sum = 0.f;
+      const float w0 = lse_w(c0.A, cb.A, inv_tau);
+      sum += w0;
+      float w1 = 0.f;
+      if (u == 2) {
+        w1 = lse_w(c1.A, cb.A, inv_tau);
+        sum += w1;
+      }
+      m.mu[rf] = lse_arrival(cb.A, tau, sum) - ns * double(cb.sig);
+      const float inv_sum = 1.f / sum;
+      wt[rf][s0] = w0 * inv_sum;
+      if (u == 2) wt[rf][rf ^ 1] = w1 * inv_sum;
+    }
+  }
+  m.win = win[0] | (win[1] << 16);
+  m.wt = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
+}
+
 // Eq 6 weights {w[rf][s=R], w[rf][s=F]} of arc k's candidates for transition rf
 template <class ArcFn>
 __device__ __forceinline__ float2 arc_weights(double ns, double inv_tau, int rf, int k, const RfOut& o,

@@ -201,6 +201,13 @@ struct DevGraph {
   int4* bwdf_a = nullptr;
   int4* bwdf_b = nullptr;
   ItemTable bwdf_items;
+  // stage-folded batched forward
+  uint8_t* ext_flags = nullptr;    // [X] bit 0 class(e) cell, bit 1 e overridden, bit 2/3 the same for e'
+  std::vector<int32_t> h_arc_xpos; // host copy of arc_xpos (batch overrides)
+  int4* bfwdf_a = nullptr;
+  int4* bfwdf_b = nullptr;
+  ItemTable bfwdf_items;
+  int32_t* b_ov_key = nullptr;     // [b_ov_cap] override keys in entry space (2x / 2x+1)
   uint32_t* done_fwd = nullptr;    // [L] level completion counters (forward)
   uint32_t* done_bwd = nullptr;    // [L] level completion counters (backward)
   // state
@@ -261,6 +268,7 @@ int launch_arrivals(DevGraph& g, float* A, float* mean, float* sigma, void* stre
 int launch_copy_slack(DevGraph& g, float* slack, uint8_t* rf, void* stream);
 // batch.cu: up to 32 scenarios in one pass; sc = [3][32] {n_sigma, derate_cell, derate_net}
 int launch_forward_batch(DevGraph& g, int nb, const float* sc_host, const std::vector<int32_t>& ov_ptr,
-                         const std::vector<int32_t>& ov_pos, const std::vector<float4>& ov_ms, float tau,
-                         double* summaries, float* d_mean_sum, void* stream);
+                         const std::vector<int32_t>& ov_pos, const std::vector<int32_t>& ov_key,
+                         const std::vector<float4>& ov_ms, float tau, double* summaries, float* d_mean_sum,
+                         void* stream);
 }  // namespace insta

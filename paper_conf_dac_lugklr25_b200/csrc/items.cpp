@@ -123,6 +123,15 @@ void build_fold_items(DevGraph& d, const FoldHost& f) {
         T.a.push_back(make_int4(a, b, hp[a], hp[b]));
         T.b.push_back(make_int4(l, flags, 0, 0));
       });
+  // folded batched forward (larger caps)
+  cut_levels(
+      d.bfwdf_items, G, f.slevel_ptr, false,
+      [&](int32_t h) { return int64_t(1) + (hp[h + 1] - hp[h]) + f.hd_nfold[h]; },
+      [&](int32_t a, int32_t b) { return b - a > kBFwdPins || hp[b] - hp[a] > kBFwdArcs; },
+      [&](ItemTable& T, int l, int32_t a, int32_t b, int flags) {
+        T.a.push_back(make_int4(a, b, hp[a], hp[b]));
+        T.b.push_back(make_int4(l, flags, 0, 0));
+      });
   // folded backward: reverse super-level order; work = 1 + entries + folded
   // entries + light fanout entries
   const auto& lp = f.hlfo_ptr;

@@ -240,68 +240,16 @@ __device__ __forceinline__ Raw fwd_pin(const KParams& P, int i, int nf, int q0, 
 }
 
 // Forward of a pin with exactly one fanin arc (w: its source word with the
-// unateness bits, ms: its record, rj: the source's words).  The same operation
-// sequence as merge_rf with nf = 1 -- scan (a0, then a1 for a non-unate arc,
-// strict ">"), winner, LSE sum 0 + w0 (+ w1), Eq 4 arrival, Eq 6 weights --
-// with each candidate evaluated once; hard mode with a unate arc has a single
-// candidate, so its corner (and square root) is not needed.  Bit-identical to
-// fwd_pin(nf = 1).  Returns the stored words.
+// unateness bits, ms: its record, rj: the source's words): merge1 (the nf = 1
+// merge_rf sequence, bit-identical to fwd_pin(nf = 1)).  Returns the stored words.
 template <bool kLSE>
 __device__ __forceinline__ Raw fwd_pin1(const KParams& P, int i, int q0, int32_t w, const float4& ms, const Raw& rj) {
-  const Gath st = unpack(rj);
-  const int u = int(uint32_t(w) >> kUnateShift);
-  const double ns = double(P.n_sigma);
-  double mu[2], var[2];
-  int win[2];
-  float wt[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
-#pragma unroll
-  for (int rf = 0; rf < 2; ++rf) {
-    const int s0 = src_tr(rf, u, 0);
-    if (!kLSE && u != 2) {
-      const double se = double(rf ? ms.w : ms.z);
-      mu[rf] = (s0 ? st.mu1 : st.mu0) + double(rf ? ms.y : ms.x);   // = make_cand(...).mu
-      var[rf] = (s0 ? st.v1 : st.v0) + se * se;                       // = make_cand(...).var
-      win[rf] = s0 << 15;
-      continue;
-    }
-    const Cand c0 = make_cand(st, ms, rf, s0, ns);
-    Cand cb = c0;
-    int bs = s0;
-    Cand c1 = c0;
-    if (u == 2) {
-      c1 = make_cand(st, ms, rf, rf ^ 1, ns);
-      if (c1.A > c0.A) {
-        cb = c1;
-        bs = rf ^ 1;
-      }
-    }
-    mu[rf] = cb.mu;
-    var[rf] = cb.var;
-    win[rf] = bs << 15;
-    if (kLSE) {
-      float sum = 0.f;
-      const float w0 = lse_w(c0.A, cb.A, P.inv_tau);
-      sum += w0;
-      float w1 = 0.f;
-      if (u == 2) {
-        w1 = lse_w(c1.A, cb.A, P.inv_tau);
-        sum += w1;
-      }
-      mu[rf] = lse_arrival(cb.A, double(P.tau), sum) - ns * double(cb.sig);
-      const float inv_sum = 1.f / sum;
-      wt[rf][s0] = w0 * inv_sum;
-      if (u == 2) wt[rf][rf ^ 1] = w1 * inv_sum;
-    }
-  }
-  store_state(P, i, mu[0], mu[1], var[0], var[1]);
-  if (!kLSE) P.win[i] = win[0] | (win[1] << 16);
-  else P.wts[q0] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
-  Raw o;
-  o.a = (unsigned long long)__double_as_longlong(with_par(mu[0], P.par));
-  o.b = (unsigned long long)__double_as_longlong(with_par(mu[1], P.par));
-  o.c = (unsigned long long)__double_as_longlong(with_par(var[0], P.par));
-  o.d = (unsigned long long)__double_as_longlong(with_par(var[1], P.par));
-  return o;
+  Merge1 m;
+  merge1<kLSE>(unpack(rj), int(uint32_t(w) >> kUnateShift), ms, double(P.n_sigma), double(P.tau), P.inv_tau, m);
+  store_state(P, i, m.mu[0], m.mu[1], m.var[0], m.var[1]);
+  if (!kLSE) P.win[i] = m.win;
+  else P.wts[q0] = m.wt;
+  return m.stored(P.par);
 }
 
 // Folded pin p (stage folding, fold.cpp): its single fanin arc e' = (j -> p)
@@ -549,7 +497,6 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
     return;
   }
   const int ww = warp - 1, wt = tid - 32;
-  const double ns = double(P.n_sigma);
   for (int t = 0; t < nsteps; ++t) {
     const int s = t & 1;
     const int k = P.step_begin + t;
