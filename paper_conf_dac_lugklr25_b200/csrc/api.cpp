@@ -61,7 +61,7 @@ void free_graph(insta::DevGraph& d) {
                   d.ext_fms,   d.ext_fq,    d.arc_xpos,  d.fwdf_a,     d.fwdf_b,    d.hd_hslot,
                   d.hlfo_ptr,  d.hlfo,      d.ext_qpos,  d.ext_bw,     d.ext_arc,   d.ext_farc,
                   d.ep_head,   d.hseed,     d.bwdf_a,    d.bwdf_b,    d.g4,        d.hacc4,
-                  d.ext_flags, d.bfwdf_a,   d.bfwdf_b,   d.b_ov_key};
+                  d.ext_flags, d.bfwdf_a,   d.bfwdf_b,   d.b_ov_key,  d.hd_eop};
   for (void* p : ptrs)
     if (p) cudaFree(p);
 }
@@ -312,6 +312,7 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   UP(d.ext_arc, fold.ext_arc.data(), fold.ext_arc.size());
   UP(d.ext_farc, fold.ext_farc.data(), fold.ext_farc.size());
   UP(d.ep_head, fold.ep_head.data(), fold.ep_head.size());
+  UP(d.hd_eop, fold.hd_eop.data(), fold.hd_eop.size());
   ZERO(d.hseed, fold.hd_pin.size());
   UP(d.bwdf_a, d.bwdf_items.a.data(), d.bwdf_items.a.size());
   UP(d.ext_flags, ext_flags.data(), ext_flags.size());

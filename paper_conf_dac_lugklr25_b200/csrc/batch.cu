@@ -36,6 +36,7 @@ constexpr long long kCountUnitB = 1ll << 44;
 
 struct BParams {
   int32_t n, num_levels, grid, step_begin, step_end, nb;
+  int32_t store_aux;   // forward: write the arg-max / Eq 6 weights (only when a backward follows)
   uint32_t par;
   float tau;
   double inv_tau;
@@ -59,6 +60,9 @@ struct BParams {
   const int32_t* __restrict__ ext_f;
   const int32_t* __restrict__ ext_fq;
   const float4* __restrict__ ext_fms;
+  const int32_t* __restrict__ ext_qpos;      // backward: fanin position of e
+  const int32_t* __restrict__ ext_farc;      // backward: caller id of e' (-1: not folded)
+  const int32_t* __restrict__ heavy_slot_pin;   // heavy slot per canonical pin (heavy adds)
   const float* __restrict__ sc;            // [3][32]: n_sigma, derate_cell, derate_net
   const int32_t* __restrict__ ov_ptr;      // [33] overrides of scenario s: [ov_ptr[s], ov_ptr[s+1])
   const int32_t* __restrict__ ov_pos;      // arc keys: fanin positions (backward) / entry keys 2x, 2x+1 (forward)
@@ -166,19 +170,27 @@ __device__ __forceinline__ float2 arc_rf_weights_b(const BParams& P, double ns, 
   return arc_weights(ns, P.inv_tau, rf, k, o, arc);
 }
 
-constexpr int kRegArcsB = 4;
+#ifndef INSTA_BREG
+#define INSTA_BREG 3
+#endif
+constexpr int kRegArcsB = INSTA_BREG;   // source words of a pin's first arcs held in registers
 
 // folded pin p behind entry x for scenario lane s (merge1 = the nf = 1 merge)
+// store: also write p's state (entries past the register window, read back by the merge)
 template <bool kLSE>
 __device__ __forceinline__ Raw foldb(const BParams& P, int32_t fw, int32_t fq, float4 fm, uint32_t fl, int x, int s,
-                                  double ns, float dcell, float dnet, Raw rj) {
+                                  double ns, float dcell, float dnet, Raw rj, bool store) {
   const float4 ms = scen_arc(P, fm, fl >> 2, 2 * x + 1, s, dcell, dnet);
   Merge1 m;
   merge1<kLSE>(unpack(rj), int(uint32_t(fw) >> kUnateShift), ms, ns, double(P.tau), P.inv_tau, m);
+  // normally no state store: a folded pin's only consumer is the head
+  // computing it here, and batched evaluations report summaries and gradients
   const int pp = fw & kSrcMask;
-  storeb(P, pp, s, m.mu[0], m.mu[1], m.var[0], m.var[1]);
-  if (!kLSE) P.bwin[size_t(pp) * kLanes + s] = m.win;
-  else P.bwts[size_t(fq) * kLanes + s] = m.wt;
+  if (store) storeb(P, pp, s, m.mu[0], m.mu[1], m.var[0], m.var[1]);
+  if (P.store_aux) {
+    if (!kLSE) P.bwin[size_t(pp) * kLanes + s] = m.win;
+    else P.bwts[size_t(fq) * kLanes + s] = m.wt;
+  }
   return m.stored(P.par);
 }
 
@@ -247,12 +259,12 @@ __global__ void __launch_bounds__(kThreads, 1) fwdb_kernel(BParams P) {
             }
           };
           // folded pin behind entry kk: computed for this scenario from the source words
-          auto fold = [&](int kk, uint32_t fl, const Raw& rj) -> Raw {
+          auto fold = [&](int kk, uint32_t fl, const Raw& rj, bool store) -> Raw {
             const int x = A.z + b0 + kk;
             if (staged) return foldb<kLSE>(P, S.f[so + b0 + kk], S.fq[so + b0 + kk], S.fms[b0 + kk], fl, x, s, ns,
-                                           dcell, dnet, rj);
+                                           dcell, dnet, rj, store);
             return foldb<kLSE>(P, __ldg(P.ext_f + x), __ldg(P.ext_fq + x), __ldg(P.ext_fms + x), fl, x, s, ns, dcell,
-                               dnet, rj);
+                               dnet, rj, store);
           };
           // gather the first kRegArcsB source entries of this scenario together
           Raw rr[kRegArcsB];
@@ -268,11 +280,11 @@ __global__ void __launch_bounds__(kThreads, 1) fwdb_kernel(BParams P) {
               float4 m0;
               ent(kk, w, fl, m0);
               awaitb(P, w & kSrcMask, s, rr[kk]);
-              if ((w >> kFoldBit) & 1) rr[kk] = fold(kk, fl, rr[kk]);
+              if ((w >> kFoldBit) & 1) rr[kk] = fold(kk, fl, rr[kk], false);
             }
           }
-          // entries past the register window: folded pins are computed (and stored) here once,
-          // the merge below then reads their words back like any other source
+          // entries past the register window: folded pins are computed and stored here once,
+          // the merge below reads their words back like any other source
           for (int kk = kRegArcsB; kk < nf; ++kk) {
             int32_t w;
             uint32_t fl;
@@ -281,7 +293,7 @@ __global__ void __launch_bounds__(kThreads, 1) fwdb_kernel(BParams P) {
             if ((w >> kFoldBit) & 1) {
               Raw r = ldb_raw(P, w & kSrcMask, s);
               awaitb(P, w & kSrcMask, s, r);
-              fold(kk, fl, r);
+              fold(kk, fl, r, true);
             }
           }
           auto arc = [&](int kk, int32_t& w, float4& ms, Raw& r) {
@@ -305,7 +317,8 @@ __global__ void __launch_bounds__(kThreads, 1) fwdb_kernel(BParams P) {
           const RfOut R = pin_rf_b<kLSE>(P, ns, 0, nf, arc);
           const RfOut F = pin_rf_b<kLSE>(P, ns, 1, nf, arc);
           storeb(P, i, s, R.mu, F.mu, R.var, F.var);
-          if (!kLSE) {
+          if (!P.store_aux) {
+          } else if (!kLSE) {
             P.bwin[size_t(i) * kLanes + s] = R.win | (F.win << 16);
           } else {
             const int q0 = __ldg(P.hd_q0 + h);
@@ -398,43 +411,64 @@ __global__ void __launch_bounds__(256) slackb_kernel(int num_ep, int nb, const i
 }
 
 // ---------------------------------------------------------------- backward
+// Stage-folded schedule (as kernels.cu bwdf_kernel): items are head ranges in
+// reverse super-level order, one warp per head, one lane per scenario.  The
+// head's adjoint is pulled from its light fanout rows (all loads of a chunk
+// issued before any is checked) + heavy accumulator + TNS seed; each entry
+// applies the Eq 6 sink side of its arc e and, through a folded pin p, of e'
+// (p's adjoint = what its own pull would form: 0 + ((0 + g) + 0), g with the
+// parity LSB cleared).  Bit-identical per scenario to the per-level schedule.
 struct BBwdStage {
-  int32_t lptr[kBwdPins + 8];
-  int32_t lfo[kBwdFanout + 8];
-  int32_t fptr[kBwdPins + 8];
-  int32_t src[kBwdArcs + 8];
-  int32_t arc[kBwdArcs + 8];
-  int32_t hslot[kBwdPins + 8];
-  int32_t eop[kBwdPins + 8];
+  int32_t lptr[kBwdPins + 8];   // light fanout rows of the heads
+  int32_t lfo[kBwdFanout + 8];  // adjoint word positions of those rows
+  int32_t fptr[kBwdPins + 8];   // entry rows of the heads
+  int32_t pin[kBwdPins + 8];    // canonical pin of each head
+  int32_t hslot[kBwdPins + 8];  // heavy accumulator slot (-1: light)
+  int32_t eop[kBwdPins + 8];    // endpoint index of the head (-1: none)
+  int32_t qpos[kBwdArcs + 8];   // fanin position of e
+  int32_t src[kBwdArcs + 8];    // fin_src word of the arc whose adjoint the entry writes
+  int32_t arc[kBwdArcs + 8];    // caller id of e
+  int32_t farc[kBwdArcs + 8];   // caller id of e' (-1: not folded)
+  int32_t fq[kBwdArcs + 8];     // fanin position of e'
+  int32_t f[kBwdArcs + 8];      // folded pin word
 };
 constexpr size_t kBBwdSmem = 2 * sizeof(BBwdStage);
 
 __device__ __forceinline__ void bbwd_prefetch(const BParams& P, BBwdStage* st, uint64_t* full, int step, int c) {
-  const int4 A = __ldg(P.item_a + size_t(step) * P.grid + c);   // {pin_lo, pin_hi, lfo_lo, lfo_hi}
-  const int4 B = __ldg(P.item_b + size_t(step) * P.grid + c);   // {arc_lo, arc_hi, level, flags}
+  const int4 A = __ldg(P.item_a + size_t(step) * P.grid + c);   // {h_lo, h_hi, lfo_lo, lfo_hi}
+  const int4 B = __ldg(P.item_b + size_t(step) * P.grid + c);   // {x_lo, x_hi, slevel, flags}
   if (!(A.y > A.x && !(B.w & kItemDirect))) return;
   const Window wl = window(A.x, A.y + 1, 4);
   const Window wf = window(A.z, A.w, 4);
   const Window wa = window(B.x, B.y, 4);
-  const Window ww = window(A.x, A.y, 4);
+  const Window wh = window(A.x, A.y, 4);
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-  mbar_expect_tx(full, 2 * wl.bytes + wf.bytes + 2 * wa.bytes + 2 * ww.bytes);
+  mbar_expect_tx(full, 2 * wl.bytes + wf.bytes + 6 * wa.bytes + 3 * wh.bytes);
   bulk_g2s(st->lptr, P.lfo_ptr + wl.start, wl.bytes, full);
   if (wf.bytes) bulk_g2s(st->lfo, P.lfo + wf.start, wf.bytes, full);
   bulk_g2s(st->fptr, P.fanin_ptr + wl.start, wl.bytes, full);
+  bulk_g2s(st->pin, P.hd_pin + wh.start, wh.bytes, full);
+  bulk_g2s(st->hslot, P.heavy_slot + wh.start, wh.bytes, full);
+  bulk_g2s(st->eop, P.ep_of_pin + wh.start, wh.bytes, full);
   if (wa.bytes) {
+    bulk_g2s(st->qpos, P.ext_qpos + wa.start, wa.bytes, full);
     bulk_g2s(st->src, P.fin_src + wa.start, wa.bytes, full);
     bulk_g2s(st->arc, P.fin_arc + wa.start, wa.bytes, full);
+    bulk_g2s(st->farc, P.ext_farc + wa.start, wa.bytes, full);
+    bulk_g2s(st->fq, P.ext_fq + wa.start, wa.bytes, full);
+    bulk_g2s(st->f, P.ext_f + wa.start, wa.bytes, full);
   }
-  bulk_g2s(st->hslot, P.heavy_slot + ww.start, ww.bytes, full);
-  bulk_g2s(st->eop, P.ep_of_pin + ww.start, ww.bytes, full);
+}
+
+__device__ __forceinline__ bool g_ready(uint32_t a, uint32_t b, uint32_t par) {
+  return ((a & 1u) == par) && ((b & 1u) == par);
 }
 
 __device__ __forceinline__ float2 loadb_g(const BParams& P, int q, int s) {
   uint32_t a, b;
   const float2* p = P.bg + size_t(q) * kLanes + s;
   ld2_u32(p, a, b);
-  while (((a & 1u) != P.par) || ((b & 1u) != P.par)) {
+  while (!g_ready(a, b, P.par)) {
     __nanosleep(20);
     ld2_u32(p, a, b);
   }
@@ -446,6 +480,63 @@ __device__ __forceinline__ float warp_sum(float v) {
   for (int d = 16; d >= 1; d >>= 1) v += __shfl_xor_sync(0xffffffffu, v, d);
   return v;
 }
+
+// Eq 6 sink side of one arc for this lane's scenario: weights from the
+// arg-max word (hard, fanin index kk) or the stored weights (LSE) at fanin
+// position q.  Returns the adjoint to the source; writes the scenario-summed
+// dL/d(arc mean) (lane 0, one warp per arc per pass: plain read-modify-write).
+template <bool kLSE>
+__device__ __forceinline__ float2 bsink(const BParams& P, bool lane_on, int s, float2 ab, int32_t win, int kk, int q,
+                                        int32_t arcid) {
+  float w[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
+  if (lane_on) {
+    if (kLSE) {
+      const float4 w4 = P.bwts[size_t(q) * kLanes + s];
+      w[0][0] = w4.x;
+      w[0][1] = w4.y;
+      w[1][0] = w4.z;
+      w[1][1] = w4.w;
+    } else {
+#pragma unroll
+      for (int rf = 0; rf < 2; ++rf) {
+        const int wv = (win >> (16 * rf)) & 0xffff;
+        const bool hit = (wv & 0x7fff) == kk;
+        w[rf][0] = (hit && (wv >> 15) == 0) ? 1.f : 0.f;
+        w[rf][1] = (hit && (wv >> 15) == 1) ? 1.f : 0.f;
+      }
+    }
+  }
+  const float abr[2] = {ab.x, ab.y};
+  float gm[2], gs[2] = {0.f, 0.f};
+#pragma unroll
+  for (int rf = 0; rf < 2; ++rf) {
+    const float a0 = w[rf][0] * abr[rf], a1 = w[rf][1] * abr[rf];
+    gm[rf] = a0 + a1;
+    gs[0] += a0;
+    gs[1] += a1;
+  }
+  // sum over scenarios of dTNS_s/d(arc mean'), fixed xor tree
+  const float t0 = warp_sum(gm[0]), t1 = warp_sum(gm[1]);
+  if (s == 0 && (t0 != 0.f || t1 != 0.f)) {
+    float2* o = reinterpret_cast<float2*>(P.d_mean_sum) + arcid;
+    const float2 prev = *o;
+    *o = make_float2(prev.x + t0, prev.y + t1);
+  }
+  return make_float2(gs[0], gs[1]);
+}
+
+// publish the adjoint of the arc at fanin position q to its source (srcw)
+__device__ __forceinline__ void bpublish(const BParams& P, int s, int q, int32_t srcw, float2 gs) {
+  st2_f32(P.bg + size_t(q) * kLanes + s, with_parf(gs.x, P.par), with_parf(gs.y, P.par));
+  if ((srcw >> kHeavyBit) & 1) {
+    const int hs = __ldg(P.heavy_slot_pin + (srcw & kSrcMask));
+    unsigned long long* acc = P.bheavy + (size_t(hs) * kLanes + s) * 2;
+    atomicAdd(acc, (unsigned long long)(kCountUnitB + __double2ll_rn(double(gs.x) * kFixB)));
+    atomicAdd(acc + 1, (unsigned long long)(kCountUnitB + __double2ll_rn(double(gs.y) * kFixB)));
+  }
+}
+
+constexpr int kPullChunk = 4;
 
 template <bool kLSE>
 __global__ void __launch_bounds__(kThreads, 1) bwdb_kernel(BParams P) {
@@ -479,19 +570,36 @@ __global__ void __launch_bounds__(kThreads, 1) bwdb_kernel(BParams P) {
       const BBwdStage& S = stage[buf];
       const int lo = A.x & 3, fo = A.z & 3, ao = B.x & 3;
       for (int p = warp; p < A.y - A.x; p += kThreads / 32) {
-        const int i = A.x + p;
-        const int r0 = (staged ? S.lptr[lo + p] : __ldg(P.lfo_ptr + i)) - (staged ? A.z : 0);
-        const int r1 = (staged ? S.lptr[lo + p + 1] : __ldg(P.lfo_ptr + i + 1)) - (staged ? A.z : 0);
-        const int slot = staged ? S.hslot[lo + p] : __ldg(P.heavy_slot + i);
-        const int ep = staged ? S.eop[lo + p] : __ldg(P.ep_of_pin + i);
+        const int h = A.x + p;
+        const int r0 = (staged ? S.lptr[lo + p] : __ldg(P.lfo_ptr + h)) - (staged ? A.z : 0);
+        const int r1 = (staged ? S.lptr[lo + p + 1] : __ldg(P.lfo_ptr + h + 1)) - (staged ? A.z : 0);
+        const int slot = staged ? S.hslot[lo + p] : __ldg(P.heavy_slot + h);
+        const int ep = staged ? S.eop[lo + p] : __ldg(P.ep_of_pin + h);
+        const int i = staged ? S.pin[lo + p] : __ldg(P.hd_pin + h);
         float ax = 0.f, ay = 0.f;
         if (lane_on) {
-          // pull (row order, fixed) + seed + heavy accumulator
-          for (int r = r0; r < r1; ++r) {
-            const int q = staged ? S.lfo[fo + r] : __ldg(P.lfo + r);
-            const float2 v = loadb_g(P, q, s);
-            ax += v.x;
-            ay += v.y;
+          // pull (row order, fixed): each chunk's loads issued before any is checked
+          for (int r = r0; r < r1; r += kPullChunk) {
+            uint32_t va[kPullChunk], vb[kPullChunk];
+            int qq[kPullChunk];
+#pragma unroll
+            for (int j = 0; j < kPullChunk; ++j) {
+              if (r + j < r1) {
+                qq[j] = staged ? S.lfo[fo + r + j] : __ldg(P.lfo + r + j);
+                ld2_u32(P.bg + size_t(qq[j]) * kLanes + s, va[j], vb[j]);
+              }
+            }
+#pragma unroll
+            for (int j = 0; j < kPullChunk; ++j) {
+              if (r + j < r1) {
+                while (!g_ready(va[j], vb[j], P.par)) {
+                  __nanosleep(20);
+                  ld2_u32(P.bg + size_t(qq[j]) * kLanes + s, va[j], vb[j]);
+                }
+                ax += stripf(va[j]);
+                ay += stripf(vb[j]);
+              }
+            }
           }
           if (slot >= 0) {
             unsigned long long* acc = P.bheavy + (size_t(slot) * kLanes + s) * 2;
@@ -519,55 +627,28 @@ __global__ void __launch_bounds__(kThreads, 1) bwdb_kernel(BParams P) {
           ay = sy + ay;
         }
         if (l == 0) continue;
-        const int b0 = staged ? S.fptr[lo + p] - B.x : __ldg(P.fanin_ptr + i) - B.x;
-        const int nf = (staged ? S.fptr[lo + p + 1] : __ldg(P.fanin_ptr + i + 1)) - B.x - b0;
+        const int b0 = staged ? S.fptr[lo + p] - B.x : __ldg(P.fanin_ptr + h) - B.x;
+        const int nf = (staged ? S.fptr[lo + p + 1] : __ldg(P.fanin_ptr + h + 1)) - B.x - b0;
         const int32_t win = (!kLSE && lane_on) ? P.bwin[size_t(i) * kLanes + s] : 0;
-        for (int kk = 0; kk < nf; ++kk) {   // warp-uniform loop (same pin in all lanes)
-          const int q = B.x + b0 + kk;
-          const int32_t srcw = staged ? S.src[ao + b0 + kk] : __ldg(P.fin_src + q);
-          const int32_t arcid = staged ? S.arc[ao + b0 + kk] : __ldg(P.fin_arc + q);
-          float w[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
-          if (lane_on) {
-            if (kLSE) {
-              const float4 w4 = P.bwts[size_t(q) * kLanes + s];
-              w[0][0] = w4.x;
-              w[0][1] = w4.y;
-              w[1][0] = w4.z;
-              w[1][1] = w4.w;
-            } else {
-#pragma unroll
-              for (int rf = 0; rf < 2; ++rf) {
-                const int wv = (win >> (16 * rf)) & 0xffff;
-                const bool hit = (wv & 0x7fff) == kk;
-                w[rf][0] = (hit && (wv >> 15) == 0) ? 1.f : 0.f;
-                w[rf][1] = (hit && (wv >> 15) == 1) ? 1.f : 0.f;
-              }
-            }
-          }
-          const float abr[2] = {ax, ay};
-          float gm[2], gs[2] = {0.f, 0.f};
-#pragma unroll
-          for (int rf = 0; rf < 2; ++rf) {
-            const float a0 = w[rf][0] * abr[rf], a1 = w[rf][1] * abr[rf];
-            gm[rf] = a0 + a1;
-            gs[0] += a0;
-            gs[1] += a1;
-          }
-          if (lane_on) {
-            st2_f32(P.bg + size_t(q) * kLanes + s, with_parf(gs[0], P.par), with_parf(gs[1], P.par));
-            if ((srcw >> kHeavyBit) & 1) {
-              const int hs = __ldg(P.heavy_slot + (srcw & kSrcMask));
-              unsigned long long* acc = P.bheavy + (size_t(hs) * kLanes + s) * 2;
-              atomicAdd(acc, (unsigned long long)(kCountUnitB + __double2ll_rn(double(gs[0]) * kFixB)));
-              atomicAdd(acc + 1, (unsigned long long)(kCountUnitB + __double2ll_rn(double(gs[1]) * kFixB)));
-            }
-          }
-          // sum over scenarios of dTNS_s/d(arc mean'), fixed xor tree
-          const float t0 = warp_sum(gm[0]), t1 = warp_sum(gm[1]);
-          if (s == 0 && (t0 != 0.f || t1 != 0.f)) {
-            float2* o = reinterpret_cast<float2*>(P.d_mean_sum) + arcid;
-            const float2 prev = *o;
-            *o = make_float2(prev.x + t0, prev.y + t1);
+        for (int kk = 0; kk < nf; ++kk) {   // warp-uniform loop (same head in all lanes)
+          const int xr = b0 + kk, x = B.x + xr;
+          const int q = staged ? S.qpos[ao + xr] : __ldg(P.ext_qpos + x);
+          const int32_t srcw = staged ? S.src[ao + xr] : __ldg(P.fin_src + x);
+          const int32_t arcid = staged ? S.arc[ao + xr] : __ldg(P.fin_arc + x);
+          const int32_t farc = staged ? S.farc[ao + xr] : __ldg(P.ext_farc + x);
+          const float2 gs = bsink<kLSE>(P, lane_on, s, make_float2(ax, ay), win, kk, q, arcid);
+          if (farc < 0) {
+            if (lane_on) bpublish(P, s, q, srcw, gs);
+          } else {   // folded pin: its adjoint as its own pull would form it, then arc e'
+            const int fq = staged ? S.fq[ao + xr] : __ldg(P.ext_fq + x);
+            const int pp = (staged ? S.f[ao + xr] : __ldg(P.ext_f + x)) & kSrcMask;
+            float px = 0.f, py = 0.f;
+            px += stripf(__float_as_uint(with_parf(gs.x, P.par)));
+            py += stripf(__float_as_uint(with_parf(gs.y, P.par)));
+            const float2 abp = make_float2(0.f + (px + 0.f), 0.f + (py + 0.f));
+            const int32_t pwin = (!kLSE && lane_on) ? P.bwin[size_t(pp) * kLanes + s] : 0;
+            const float2 g2 = bsink<kLSE>(P, lane_on, s, abp, pwin, 0, fq, farc);
+            if (lane_on) bpublish(P, s, fq, srcw, g2);
           }
         }
       }
@@ -638,23 +719,26 @@ static BParams make_bparams(DevGraph& g, bool bwd) {
   P.n = g.n;
   P.num_levels = g.num_levels;
   P.grid = g.grid;
-  P.item_a = bwd ? g.bwd_a : g.bfwdf_a;
-  P.item_b = bwd ? g.bwd_b : g.bfwdf_b;
-  P.fanin_ptr = bwd ? g.fanin_ptr : g.hd_ptr;
-  P.fin_src = bwd ? g.fin_src : g.ext_w;
-  P.fin_ms = bwd ? g.fin_ms : g.ext_ms;
+  P.item_a = bwd ? g.bwdf_a : g.bfwdf_a;
+  P.item_b = bwd ? g.bwdf_b : g.bfwdf_b;
+  P.fanin_ptr = g.hd_ptr;
+  P.fin_src = bwd ? g.ext_bw : g.ext_w;
+  P.fin_ms = g.ext_ms;
   P.fin_flags = bwd ? g.fin_flags : g.ext_flags;
+  P.ext_qpos = g.ext_qpos;
+  P.ext_farc = g.ext_farc;
   P.hd_pin = g.hd_pin;
   P.hd_q0 = g.hd_q0;
   P.ext_f = g.ext_f;
   P.ext_fq = g.ext_fq;
   P.ext_fms = g.ext_fms;
-  P.fin_arc = g.fin_arc;
-  P.lfo_ptr = g.lfo_ptr;
-  P.lfo = g.lfo;
-  P.heavy_slot = g.heavy_slot;
+  P.fin_arc = bwd ? g.ext_arc : g.fin_arc;
+  P.lfo_ptr = g.hlfo_ptr;
+  P.lfo = g.hlfo;
+  P.heavy_slot = bwd ? g.hd_hslot : g.heavy_slot;   // backward: per head (staged); heavy_add uses hslot_pin
+  P.heavy_slot_pin = g.heavy_slot;
   P.heavy_fo = g.heavy_fo;
-  P.ep_of_pin = g.ep_of_pin;
+  P.ep_of_pin = bwd ? g.hd_eop : g.ep_of_pin;
   P.src_ms = g.src_ms;
   P.sc = g.b_sc;
   P.ov_ptr = g.b_ov_ptr;
@@ -710,6 +794,7 @@ int launch_forward_batch(DevGraph& g, int nb, const float* sc_host /*[3][32]*/, 
   P.tau = tau;
   P.inv_tau = lse ? 1.0 / double(tau) : 0.0;
   P.par = (++g.pass_bfwd) & 1u;
+  P.store_aux = grad ? 1 : 0;
   P.step_begin = 0;
   P.step_end = g.bfwdf_items.num_steps;
   if (g.n > 0) {
@@ -735,7 +820,7 @@ int launch_forward_batch(DevGraph& g, int nb, const float* sc_host /*[3][32]*/, 
     Q.par = (++g.pass_bbwd) & 1u;
     Q.d_mean_sum = d_mean_sum;
     Q.step_begin = 0;
-    Q.step_end = g.bwd_items.num_steps;
+    Q.step_end = g.bwdf_items.num_steps;
     void* args[] = {&Q};
     e = cudaLaunchCooperativeKernel(lse ? (const void*)bwdb_kernel<true> : (const void*)bwdb_kernel<false>,
                                     dim3(g.grid), dim3(kThreads), args, kBBwdSmem, st);

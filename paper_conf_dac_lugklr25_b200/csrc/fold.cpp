@@ -84,6 +84,7 @@ void build_fold(const HostLevels& h, const std::vector<int32_t>& fin_src, const 
   f.ext_arc.assign(size_t(X), 0);
   f.ext_farc.assign(size_t(X), -1);
   f.hd_hslot.assign(size_t(H), -1);
+  f.hd_eop.assign(size_t(H), -1);
   f.hlfo_ptr.assign(size_t(H) + 1, 0);
   f.hlfo.clear();
   f.ep_head.assign(size_t(std::count_if(ep_of_pin.begin(), ep_of_pin.end(), [](int32_t v) { return v >= 0; })), -1);
@@ -93,6 +94,7 @@ void build_fold(const HostLevels& h, const std::vector<int32_t>& fin_src, const 
     f.hd_q0[hh] = fp[q];
     f.hd_hslot[hh] = heavy_slot[q];
     if (ep_of_pin[q] >= 0) f.ep_head[ep_of_pin[q]] = hh;
+    f.hd_eop[hh] = ep_of_pin[q];
     for (int32_t r = lfo_ptr[q]; r < lfo_ptr[q + 1]; ++r) f.hlfo.push_back(lfo[r]);
     f.hlfo_ptr[hh + 1] = int32_t(f.hlfo.size());
     for (int32_t y = fp[q]; y < fp[q + 1]; ++y, ++x) {

@@ -104,6 +104,7 @@ struct FoldHost {
   std::vector<int32_t> ext_arc;     // [X] caller id of e
   std::vector<int32_t> ext_farc;    // [X] caller id of e' (-1 if not folded)
   std::vector<int32_t> ep_head;     // [P] head index of each endpoint (endpoints are never folded)
+  std::vector<int32_t> hd_eop;      // [H] endpoint index of each head (-1: not an endpoint)
 };
 
 // Item table: step s of CTA c is entry s * G + c.
@@ -194,6 +195,7 @@ struct DevGraph {
   int32_t* ext_arc = nullptr;
   int32_t* ext_farc = nullptr;
   int32_t* ep_head = nullptr;
+  int32_t* hd_eop = nullptr;       // [H] endpoint index of each head, -1 otherwise
   float2* hseed = nullptr;         // [H] endpoint seeds in head order
   // sigma-channel backward scratch (allocated on first use)
   void* g4 = nullptr;              // [e] float4 per fanin position
