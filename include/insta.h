@@ -173,9 +173,11 @@ insta_status insta_backward(insta_graph* g, const float* ep_seed, float* d_arc_m
 
 /* Re-annotate n arcs ("re-annotate ... then re-propagate"):
  * arc_ids DEVICE int32[n] (caller ids, unique), mean/sigma DEVICE float[n][2].
- * incremental = 1: the next insta_forward re-propagates only the fanout cone
- * of the changed arcs (same per-pin arithmetic, so results are bit-identical
- * to a full forward); 0: the next forward is a full one.  Invalid ids or
+ * incremental = 1: the next insta_forward recomputes only the fanout cone of
+ * the changed arcs, stopping where a recomputed record does not change (a
+ * dataflow pass in which pins outside the cone only republish their record;
+ * same per-pin arithmetic, so results are bit-identical to a full forward);
+ * 0: the next forward is a full one.  Invalid ids or
  * values are not checked on the device (caller contract). */
 insta_status insta_update_arcs(insta_graph* g, int64_t n, const int32_t* arc_ids,
                                const float* mean, const float* sigma, int32_t incremental,
@@ -209,7 +211,9 @@ insta_status insta_forward_batch(insta_graph* g, int32_t num_scenarios, const in
                                  double* summaries, float* d_arc_mean_sum, void* cuda_stream);
 
 /* Statistics of the last forward: number of pins recomputed (== num_pins for a
- * full forward; the cone size for an incremental one).  Synchronizes. */
+ * full forward).  For an incremental one: the work-item heads recomputed in
+ * the changed cone (insta_graph_schedule; each head's folded input pins are
+ * recomputed with it).  Synchronizes. */
 insta_status insta_last_forward_stats(insta_graph* g, int64_t* pins_recomputed);
 
 /* Thread-local message for the last non-OK status ("" if none). */

@@ -48,20 +48,21 @@ cudaError_t alloc_zero(T** dst, size_t count) {
 
 void free_graph(insta::DevGraph& d) {
   void* ptrs[] = {d.level_ptr, d.fanin_ptr, d.fin_src,   d.fin_ms,     d.fin_arc,   d.lfo_ptr,
-                  d.lfo,       d.fanout_ptr, d.fout_sink, d.heavy_slot, d.heavy_acc, d.arc_pos,
+                  d.lfo,       d.heavy_slot, d.heavy_acc, d.arc_pos,
                   d.heavy_cnt, d.heavy_fo,
                   d.arc_sink,  d.order,     d.src_ms,    d.ep_pin,     d.ep_rat,    d.arc_class,
-                  d.fwd_a,     d.fwd_b,     d.bfwd_a,    d.bfwd_b,     d.bwd_a,     d.bwd_b,      d.done_fwd,  d.done_bwd,
+                  d.fwd_a,     d.fwd_b,     d.bfwd_a,    d.bfwd_b,     d.bwd_a,     d.bwd_b,
                   d.state,     d.win,       d.wts,       d.g,          d.seed,      d.slack,
-                  d.rf_star,   d.partials,  d.ticket,    d.summary,    d.dirty,     d.counters,
+                  d.rf_star,   d.partials,  d.ticket,    d.summary,    d.counters,
                   d.fin_flags, d.ep_of_pin, d.b_state,   d.b_win,      d.b_wts,     d.b_g,
                   d.b_heavy,   d.b_sc,      d.b_ov_ptr,  d.b_ov_pos,   d.b_ov_ms,   d.b_slack,
-                  d.b_rf,      d.b_partials, d.b_ticket,  d.pin_level,  d.lvl_range, d.max_sink_level,
+                  d.b_rf,      d.b_partials, d.b_ticket,
                   d.hd_pin,    d.hd_ptr,    d.hd_q0,     d.ext_w,      d.ext_ms,    d.ext_f,
                   d.ext_fms,   d.ext_fq,    d.arc_xpos,  d.fwdf_a,     d.fwdf_b,    d.hd_hslot,
                   d.hlfo_ptr,  d.hlfo,      d.ext_qpos,  d.ext_bw,     d.ext_arc,   d.ext_farc,
                   d.ep_head,   d.hseed,     d.bwdf_a,    d.bwdf_b,    d.g4,        d.hacc4,
-                  d.ext_flags, d.bfwdf_a,   d.bfwdf_b,   d.b_ov_key,  d.hd_eop};
+                  d.ext_flags, d.bfwdf_a,   d.bfwdf_b,   d.b_ov_key,  d.hd_eop,    d.dirty_h,
+                  d.arc_head};
   for (void* p : ptrs)
     if (p) cudaFree(p);
 }
@@ -164,7 +165,7 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
 
   // ---- canonical host arrays ------------------------------------------------
   const size_t nE = static_cast<size_t>(E), nN = static_cast<size_t>(n);
-  std::vector<int32_t> arc_pos(nE), arc_sink(nE), fin_src(nE), fout_sink(nE);
+  std::vector<int32_t> arc_pos(nE), arc_sink(nE), fin_src(nE);
   std::vector<float4> fin_ms(nE);
   std::vector<int32_t> heavy_slot(nN, -1);
   int32_t nheavy = 0, max_fanin = 0;
@@ -203,7 +204,6 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   for (int32_t k = 0; k < n; ++k) {
     for (int32_t r = h.fanout_ptr[k]; r < h.fanout_ptr[k + 1]; ++r) {
       const int32_t a = h.fanout_arc[r];
-      fout_sink[r] = arc_sink[a];
       if (heavy_slot[k] < 0) lfo.push_back(arc_pos[a]);
     }
     lfo_ptr[k + 1] = int32_t(lfo.size());
@@ -227,13 +227,6 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   if (desc->arc_class) std::copy(desc->arc_class, desc->arc_class + E, arc_class.begin());
   std::vector<uint8_t> fin_flags(nE, 0);
   for (int64_t q = 0; q < E; ++q) fin_flags[q] = arc_class[h.fanin_arc[q]] ? 1 : 0;
-  std::vector<int32_t> pin_level(nN);
-  for (int32_t k = 0; k < n; ++k) pin_level[k] = h.level[h.order[k]];
-  const int32_t lvl_init[2] = {0x7fffffff, -1};
-  std::vector<int32_t> max_sink_level(nN, -1);
-  for (int32_t k = 0; k < n; ++k)
-    for (int32_t r = h.fanout_ptr[k]; r < h.fanout_ptr[k + 1]; ++r)
-      max_sink_level[k] = std::max(max_sink_level[k], pin_level[fout_sink[r]]);
   std::vector<int32_t> ep_of_pin(nN, -1);
   for (int32_t k = 0; k < d.num_ep; ++k) ep_of_pin[ep_pin[k]] = k;
   d.h_arc_pos = arc_pos;
@@ -269,8 +262,6 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   UP(d.fin_arc, h.fanin_arc.data(), nE);
   UP(d.lfo_ptr, lfo_ptr.data(), lfo_ptr.size());
   UP(d.lfo, lfo.data(), lfo.size());
-  UP(d.fanout_ptr, h.fanout_ptr.data(), h.fanout_ptr.size());
-  UP(d.fout_sink, fout_sink.data(), nE);
   UP(d.heavy_slot, heavy_slot.data(), nN);
   ZERO(d.heavy_acc, 2 * std::max(nheavy, 1));
   ZERO(d.heavy_cnt, std::max(nheavy, 1));
@@ -284,9 +275,6 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   UP(d.arc_class, arc_class.data(), nE);
   UP(d.fin_flags, fin_flags.data(), nE);
   UP(d.ep_of_pin, ep_of_pin.data(), nN);
-  UP(d.pin_level, pin_level.data(), nN);
-  UP(d.lvl_range, lvl_init, 2);
-  UP(d.max_sink_level, max_sink_level.data(), nN);
   UP(d.fwd_a, d.fwd_items.a.data(), d.fwd_items.a.size());
   UP(d.fwd_b, d.fwd_items.b.data(), d.fwd_items.b.size());
   UP(d.bfwd_a, d.bfwd_items.a.data(), d.bfwd_items.a.size());
@@ -313,14 +301,14 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   UP(d.ext_farc, fold.ext_farc.data(), fold.ext_farc.size());
   UP(d.ep_head, fold.ep_head.data(), fold.ep_head.size());
   UP(d.hd_eop, fold.hd_eop.data(), fold.hd_eop.size());
+  ZERO(d.dirty_h, fold.hd_pin.size());
+  UP(d.arc_head, fold.arc_head.data(), fold.arc_head.size());
   ZERO(d.hseed, fold.hd_pin.size());
   UP(d.bwdf_a, d.bwdf_items.a.data(), d.bwdf_items.a.size());
   UP(d.ext_flags, ext_flags.data(), ext_flags.size());
   UP(d.bfwdf_a, d.bfwdf_items.a.data(), d.bfwdf_items.a.size());
   UP(d.bfwdf_b, d.bfwdf_items.b.data(), d.bfwdf_items.b.size());
   UP(d.bwdf_b, d.bwdf_items.b.data(), d.bwdf_items.b.size());
-  ZERO(d.done_fwd, std::max(d.num_levels, 1));
-  ZERO(d.done_bwd, std::max(d.num_levels, 1));
   ZERO(d.state, nN);
   ZERO(d.win, nN);
   ZERO(d.wts, nE);
@@ -331,7 +319,6 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   ZERO(d.partials, 3 * ((d.num_ep + 255) / 256 + 1));
   ZERO(d.ticket, 1);
   ZERO(d.summary, 4);
-  ZERO(d.dirty, nN);
   ZERO(d.counters, 4);
 #undef UP
 #undef ZERO

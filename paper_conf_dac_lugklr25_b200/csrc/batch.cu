@@ -108,7 +108,7 @@ __device__ __forceinline__ void storeb(const BParams& P, int i, int s, double m0
                                        double v1) {
   asm volatile("st.relaxed.gpu.global.v4.f64 [%0], {%1, %2, %3, %4};" ::"l"(P.bstate + size_t(i) * kLanes + s),
                "d"(with_par(m0, P.par)), "d"(with_par(m1, P.par)), "d"(with_par(v0, P.par)),
-               "d"(with_par(v1, P.par))
+               "d"(with_tag(v1, P.par, 0u))
                : "memory");
 }
 
@@ -360,7 +360,7 @@ __global__ void __launch_bounds__(256) slackb_kernel(int num_ep, int nb, const i
     const double aR = strip((unsigned long long)__double_as_longlong(m.x)) +
                       ns * double(sigma_of(strip((unsigned long long)__double_as_longlong(v.x))));
     const double aF = strip((unsigned long long)__double_as_longlong(m.y)) +
-                      ns * double(sigma_of(strip((unsigned long long)__double_as_longlong(v.y))));
+                      ns * double(sigma_of(strip2((unsigned long long)__double_as_longlong(v.y))));
     const double sR = double(rat.x) - aR, sF = double(rat.y) - aF;
     const bool fall = sF < sR;
     const double sl = fall ? sF : sR;

@@ -29,6 +29,14 @@ __device__ __forceinline__ double with_par(double x, uint32_t par) {
   return __longlong_as_double((__double_as_longlong(x) & ~1ll) | (long long)par);
 }
 __device__ __forceinline__ double strip(unsigned long long b) { return __longlong_as_double((long long)(b & ~1ull)); }
+// The var_F word (last word) of a pin record also carries, in bit 1, the
+// "record changed in this pass" flag of the incremental pass; its value is used
+// with both low bits cleared (identically in every kernel).
+__device__ __forceinline__ double with_tag(double x, uint32_t par, uint32_t chg) {
+  return __longlong_as_double((__double_as_longlong(x) & ~3ll) | (long long)(par | (chg << 1)));
+}
+__device__ __forceinline__ double strip2(unsigned long long b) { return __longlong_as_double((long long)(b & ~3ull)); }
+__device__ __forceinline__ uint32_t tag_changed(unsigned long long d) { return uint32_t(d >> 1) & 1u; }
 __device__ __forceinline__ float with_parf(float x, uint32_t par) {
   return __uint_as_float((__float_as_uint(x) & ~1u) | par);
 }
@@ -139,7 +147,7 @@ __device__ __forceinline__ Gath unpack(const Raw& r) {
   g.mu0 = strip(r.a);
   g.mu1 = strip(r.b);
   g.v0 = strip(r.c);
-  g.v1 = strip(r.d);
+  g.v1 = strip2(r.d);
   return g;
 }
 
@@ -287,7 +295,7 @@ struct Merge1 {
     o.a = (unsigned long long)__double_as_longlong(with_par(mu[0], par));
     o.b = (unsigned long long)__double_as_longlong(with_par(mu[1], par));
     o.c = (unsigned long long)__double_as_longlong(with_par(var[0], par));
-    o.d = (unsigned long long)__double_as_longlong(with_par(var[1], par));
+    o.d = (unsigned long long)__double_as_longlong(with_tag(var[1], par, 0u));
     return o;
   }
 };

@@ -123,6 +123,14 @@ void build_fold(const HostLevels& h, const std::vector<int32_t>& fin_src, const 
     }
     f.hd_ptr[hh + 1] = int32_t(x);
   }
+  // incremental pass: the head whose item evaluates each arc
+  f.arc_head.assign(size_t(h.e), -1);
+  for (int32_t hh = 0; hh < H; ++hh) {
+    for (int32_t y = f.hd_ptr[hh]; y < f.hd_ptr[hh + 1]; ++y) {
+      f.arc_head[f.ext_arc[y]] = hh;
+      if (f.ext_farc[y] >= 0) f.arc_head[f.ext_farc[y]] = hh;
+    }
+  }
 }
 
 }  // namespace insta

@@ -105,6 +105,8 @@ struct FoldHost {
   std::vector<int32_t> ext_farc;    // [X] caller id of e' (-1 if not folded)
   std::vector<int32_t> ep_head;     // [P] head index of each endpoint (endpoints are never folded)
   std::vector<int32_t> hd_eop;      // [H] endpoint index of each head (-1: not an endpoint)
+  // incremental pass
+  std::vector<int32_t> arc_head;    // [E] caller arc -> head whose item evaluates the arc
 };
 
 // Item table: step s of CTA c is entry s * G + c.
@@ -130,8 +132,6 @@ struct DevGraph {
   int32_t* fin_arc = nullptr;      // [e] caller arc id
   int32_t* lfo_ptr = nullptr;      // [n+1] light fanout rows (heavy drivers' rows empty)
   int32_t* lfo = nullptr;          // [e_light] fanin position of each light fanout entry
-  int32_t* fanout_ptr = nullptr;   // [n+1] full fanout rows (incremental marking)
-  int32_t* fout_sink = nullptr;    // [e] canonical sink of each full fanout entry
   int32_t* heavy_slot = nullptr;   // [n] accumulator slot of heavy drivers, -1 otherwise
   unsigned long long* heavy_acc = nullptr;  // [num_heavy][2] fixed-point adjoints
   uint32_t* heavy_cnt = nullptr;   // [num_heavy] sink arcs that have contributed this pass
@@ -196,6 +196,8 @@ struct DevGraph {
   int32_t* ext_farc = nullptr;
   int32_t* ep_head = nullptr;
   int32_t* hd_eop = nullptr;       // [H] endpoint index of each head, -1 otherwise
+  uint32_t* dirty_h = nullptr;     // [H] incremental: stamp == inc epoch -> recompute
+  int32_t* arc_head = nullptr;     // [E] caller arc -> head
   float2* hseed = nullptr;         // [H] endpoint seeds in head order
   // sigma-channel backward scratch (allocated on first use)
   void* g4 = nullptr;              // [e] float4 per fanin position
@@ -210,8 +212,6 @@ struct DevGraph {
   int4* bfwdf_b = nullptr;
   ItemTable bfwdf_items;
   int32_t* b_ov_key = nullptr;     // [b_ov_cap] override keys in entry space (2x / 2x+1)
-  uint32_t* done_fwd = nullptr;    // [L] level completion counters (forward)
-  uint32_t* done_bwd = nullptr;    // [L] level completion counters (backward)
   // state
   PinState* state = nullptr;       // [n]
   int32_t* win = nullptr;          // [n] hard-mode winners {R: k | s<<15, F: << 16}
@@ -224,10 +224,6 @@ struct DevGraph {
   uint32_t* ticket = nullptr;      // last-block ticket
   double* summary = nullptr;       // {wns, tns, nviol} on device
   // incremental
-  uint32_t* dirty = nullptr;       // [n] stamp == inc_epoch: pin must be recomputed
-  int32_t* pin_level = nullptr;    // [n] level of each canonical pin
-  int32_t* max_sink_level = nullptr;  // [n] deepest level among the pin's fanout sinks, -1 if none
-  int32_t* lvl_range = nullptr;    // [2] {min, max} level of pending dirty marks
   unsigned long long* counters = nullptr;  // [4] recomputed pins etc.
   // host-side bookkeeping
   HostLevels host;

@@ -75,6 +75,10 @@ struct KParams {
   const int32_t* __restrict__ ext_arc;
   const int32_t* __restrict__ ext_farc;
   const float2* hseed;
+  // incremental dataflow pass on the folded schedule
+  const uint32_t* dirty_h;                   // [H] stamp == `stamp`: head must be recomputed
+  uint32_t stamp;
+  unsigned long long* counters;              // [0] heads recomputed
   PinState* state;
   int32_t* win;
   float4* wts;
@@ -126,10 +130,10 @@ __device__ __forceinline__ Gath load_state(const KParams& P, int j) {
 }
 
 __device__ __forceinline__ void store_state(const KParams& P, int i, double m0, double m1, double v0,
-                                            double v1) {
+                                            double v1, uint32_t chg = 0u) {
   asm volatile("st.relaxed.gpu.global.v4.f64 [%0], {%1, %2, %3, %4};" ::"l"(P.state + i),
                "d"(with_par(m0, P.par)), "d"(with_par(m1, P.par)), "d"(with_par(v0, P.par)),
-               "d"(with_par(v1, P.par))
+               "d"(with_tag(v1, P.par, chg))
                : "memory");
 }
 
@@ -151,7 +155,7 @@ __device__ __forceinline__ Gath load_state_plain(const PinState* p) {
   g.mu0 = strip((unsigned long long)__double_as_longlong(m.x));
   g.mu1 = strip((unsigned long long)__double_as_longlong(m.y));
   g.v0 = strip((unsigned long long)__double_as_longlong(v.x));
-  g.v1 = strip((unsigned long long)__double_as_longlong(v.y));
+  g.v1 = strip2((unsigned long long)__double_as_longlong(v.y));
   return g;
 }
 
@@ -226,7 +230,7 @@ __device__ __forceinline__ Raw fwd_pin(const KParams& P, int i, int nf, int q0, 
   o.a = (unsigned long long)__double_as_longlong(with_par(R.mu, P.par));
   o.b = (unsigned long long)__double_as_longlong(with_par(F.mu, P.par));
   o.c = (unsigned long long)__double_as_longlong(with_par(R.var, P.par));
-  o.d = (unsigned long long)__double_as_longlong(with_par(F.var, P.par));
+  o.d = (unsigned long long)__double_as_longlong(with_tag(F.var, P.par, 0u));
   if (!kLSE) {
     P.win[i] = R.win | (F.win << 16);
   } else {
@@ -281,13 +285,12 @@ __device__ __forceinline__ void mbar_arrive1(uint64_t* bar) {
 #define INSTA_FWD_THREADS 512
 #endif
 constexpr int kFwdThreads = INSTA_FWD_THREADS;
-#ifndef INSTA_ROUNDS
-#define INSTA_ROUNDS 1
-#endif
-constexpr int kRoundsPerPass = INSTA_ROUNDS;   // independent rounds interleaved per warp   // forward CTA: 1 producer warp + workers
 constexpr int kWorkerWarps = kFwdThreads / 32 - 1;
 constexpr int kWorkers = kWorkerWarps * 32;
-constexpr size_t kFwdSmemV6 = 2 * sizeof(FwdStage) + 2 * sizeof(Raw) * kFwdArcs;
+constexpr int kHeadsPerWarp = (kFwdPins + kWorkerWarps - 1) / kWorkerWarps;   // max heads in a warp's share
+constexpr int kStampWords = (kHeadsPerWarp + 31) / 32;
+// stages + gather buffers + (incremental) previous records of each warp's heads
+constexpr size_t kFwdSmemV6 = 2 * sizeof(FwdStage) + 2 * sizeof(Raw) * kFwdArcs + sizeof(Raw) * kWorkerWarps * kHeadsPerWarp;
 constexpr int kFastPins = ((kFwdPins + kWorkerWarps - 1) / kWorkerWarps + 31) / 32;   // fanin-1 pins per lane
 
 // One round of the forward: pins [q, q + cnt) of the item whose arcs
@@ -333,142 +336,170 @@ __device__ __forceinline__ Round round_at(const FwdStage& S, const int4& A, int 
   return R;
 }
 
-// NR independent rounds per warp at once (their dependent chains interleave).
-// The segmented arg-max moves only (corner A, candidate index) through the
-// shuffle tree; the head lane then fetches the winner's (mu, var, sigma) from
-// the winning lane, which kept its own best candidate per rf.
-template <bool kLSE, bool kFold, int NR>
-__device__ __forceinline__ void fwd_rounds(const KParams& P, const Raw* gath, const int4& A, const FwdStage& S,
-                                           int po, const Round* R, int lane) {
+// Incremental pass (kInc).  A head is recomputed iff it is stamped dirty
+// (insta_update_arcs changed an arc it evaluates) or the record of one of its
+// entries' sources carries the "changed" tag (bit 1 of its var_F word) of
+// this pass; otherwise it republishes its previous record with this pass's
+// parity and the tag cleared.  A recomputed head tags its record when it
+// differs from the previous one.  No marks, counters or fences: the tag
+// travels inside the record the consumer waits for anyway.
+__device__ __forceinline__ bool record_changed(const Raw& o, double m0, double m1, double v0, double v1) {
+  return strip(o.a) != strip((unsigned long long)__double_as_longlong(m0)) ||
+         strip(o.b) != strip((unsigned long long)__double_as_longlong(m1)) ||
+         strip(o.c) != strip((unsigned long long)__double_as_longlong(v0)) ||
+         strip2(o.d) != strip2((unsigned long long)__double_as_longlong(v1));
+}
+
+__device__ __forceinline__ void republish(const KParams& P, int i, const Raw& o) {
+  store_state(P, i, strip(o.a), strip(o.b), strip(o.c), strip2(o.d), 0u);
+}
+
+template <bool kLSE, class ArcFn>
+__device__ __forceinline__ void fwd_pin_inc(const KParams& P, int i, int nf, int q0, const Raw& old, ArcFn&& arc) {
+  const RfOut R = pin_rf<kLSE>(P, 0, nf, arc);
+  const RfOut F = pin_rf<kLSE>(P, 1, nf, arc);
+  if (kLSE) {
+    for (int k = 0; k < nf; ++k) {
+      const float2 wr = arc_rf_weights(P, 0, k, R, arc);
+      const float2 wf = arc_rf_weights(P, 1, k, F, arc);
+      P.wts[q0 + k] = make_float4(wr.x, wr.y, wf.x, wf.y);
+    }
+  }
+  store_state(P, i, R.mu, F.mu, R.var, F.var, record_changed(old, R.mu, F.mu, R.var, F.var) ? 1u : 0u);
+  if (!kLSE) P.win[i] = R.win | (F.win << 16);
+}
+
+// One round.  The segmented arg-max moves only (corner A, candidate index)
+// through the shuffle tree; the head lane then fetches the winner's (mu, var,
+// sigma) from the winning lane, which kept its own best candidate per rf.
+// kInc: folded pins are computed in the round (the incremental pass has no
+// pre-pass); `hdirty` / `hold`: the head lane's dirty flag and previous record
+// (a recomputed head tags its record if it differs from the previous one).
+template <bool kLSE, bool kFold, bool kInc>
+__device__ __forceinline__ void fwd_round(const KParams& P, const Raw* gath, const int4& A, const FwdStage& S,
+                                          int po, int so, const Round& R, int lane, bool hdirty = false,
+                                          const Raw* hold = nullptr) {
   const double ns = double(P.n_sigma);
-  double bA[NR][2];                  // reduced corner
-  int bi[NR][2];                     // reduced candidate index k | s << 15
-  double om[NR][2], ov[NR][2];       // this lane's best candidate (mu, var) per rf
-  float osg[NR][2];                  // and its sigma
-  double A0[NR][2], A1[NR][2];
-  int u[NR], k[NR];
-  bool act[NR];
-  int maxlen = 0;
-#pragma unroll
-  for (int r = 0; r < NR; ++r) {
-    act[r] = lane < R[r].na;
-    k[r] = lane - R[r].seg;
-    u[r] = 0;
+  double bA[2] = {0.0, 0.0}, om[2] = {0.0, 0.0}, ov[2] = {0.0, 0.0}, A0[2] = {0.0, 0.0}, A1[2] = {0.0, 0.0};
+  float osg[2] = {0.f, 0.f};
+  int bi[2] = {0, 0};
+  const bool act = lane < R.na;
+  const int k = lane - R.seg;
+  int u = 0;
+  if (act) {
+    u = int(uint32_t(R.w) >> kUnateShift);
+    Raw rs = gath[R.base + lane];
+    if (kInc && ((R.w >> kFoldBit) & 1))
+      rs = fold_pin<kLSE>(P, S.f[so + R.base + lane], S.fms[R.base + lane], S.fq[so + R.base + lane], rs);
+    const Gath st = unpack(rs);
 #pragma unroll
     for (int rf = 0; rf < 2; ++rf) {
-      A0[r][rf] = A1[r][rf] = bA[r][rf] = om[r][rf] = ov[r][rf] = 0.0;
-      osg[r][rf] = 0.f;
-      bi[r][rf] = 0;
-    }
-    if (act[r]) {
-      u[r] = int(uint32_t(R[r].w) >> kUnateShift);
-      const Gath st = unpack(gath[R[r].base + lane]);
-#pragma unroll
-      for (int rf = 0; rf < 2; ++rf) {
-        const int s0 = src_tr(rf, u[r], 0);
-        const Cand c0 = make_cand(st, R[r].ms, rf, s0, ns);
-        A0[r][rf] = c0.A;
-        bA[r][rf] = c0.A;
-        bi[r][rf] = k[r] | (s0 << 15);
-        om[r][rf] = c0.mu;
-        ov[r][rf] = c0.var;
-        osg[r][rf] = c0.sig;
-        if (u[r] == 2) {
-          const Cand c1 = make_cand(st, R[r].ms, rf, rf ^ 1, ns);
-          A1[r][rf] = c1.A;
-          if (c1.A > c0.A) {   // strict: s = rf wins ties (merge_rf order)
-            bA[r][rf] = c1.A;
-            bi[r][rf] = k[r] | ((rf ^ 1) << 15);
-            om[r][rf] = c1.mu;
-            ov[r][rf] = c1.var;
-            osg[r][rf] = c1.sig;
-          }
+      const int s0 = src_tr(rf, u, 0);
+      const Cand c0 = make_cand(st, R.ms, rf, s0, ns);
+      A0[rf] = c0.A;
+      bA[rf] = c0.A;
+      bi[rf] = k | (s0 << 15);
+      om[rf] = c0.mu;
+      ov[rf] = c0.var;
+      osg[rf] = c0.sig;
+      if (u == 2) {
+        const Cand c1 = make_cand(st, R.ms, rf, rf ^ 1, ns);
+        A1[rf] = c1.A;
+        if (c1.A > c0.A) {   // strict: s = rf wins ties (merge_rf order)
+          bA[rf] = c1.A;
+          bi[rf] = k | ((rf ^ 1) << 15);
+          om[rf] = c1.mu;
+          ov[rf] = c1.var;
+          osg[rf] = c1.sig;
         }
       }
     }
-    maxlen = max(maxlen, act[r] ? R[r].seg_end - R[r].seg : 0);
   }
-  maxlen = __reduce_max_sync(0xffffffffu, maxlen);
+  const int maxlen = __reduce_max_sync(0xffffffffu, act ? R.seg_end - R.seg : 0);
   for (int d = 1; d < maxlen; d <<= 1) {
 #pragma unroll
-    for (int r = 0; r < NR; ++r) {
-#pragma unroll
-      for (int rf = 0; rf < 2; ++rf) {
-        const double oA = __shfl_down_sync(0xffffffffu, bA[r][rf], d);
-        const int oi = __shfl_down_sync(0xffffffffu, bi[r][rf], d);
-        // the upper half replaces the lower only if strictly greater (Alg 2 l.4)
-        if ((k[r] & (2 * d - 1)) == 0 && lane + d < R[r].seg_end && oA > bA[r][rf]) {
-          bA[r][rf] = oA;
-          bi[r][rf] = oi;
-        }
+    for (int rf = 0; rf < 2; ++rf) {
+      const double oA = __shfl_down_sync(0xffffffffu, bA[rf], d);
+      const int oi = __shfl_down_sync(0xffffffffu, bi[rf], d);
+      // the upper half replaces the lower only if strictly greater (Alg 2 l.4)
+      if ((k & (2 * d - 1)) == 0 && lane + d < R.seg_end && oA > bA[rf]) {
+        bA[rf] = oA;
+        bi[rf] = oi;
       }
     }
   }
+  const bool head = act && k == 0;
+  const int hq = R.q + __popc(R.heads & ((1u << lane) - 1u));   // my pin within the item (head lanes)
+  const int i = kFold ? S.pin[po + min(hq, A.y - A.x - 1)] : A.x + hq;
+  double wm[2], wv[2];
+  float wsg[2];
 #pragma unroll
-  for (int r = 0; r < NR; ++r) {
-    const bool head = act[r] && k[r] == 0;
-    const int hq = R[r].q + __popc(R[r].heads & ((1u << lane) - 1u));   // my pin within the item (head lanes)
-    const int i = kFold ? S.pin[po + min(hq, A.y - A.x - 1)] : A.x + hq;
-    double wm[2], wv[2];
-    float wsg[2];
+  for (int rf = 0; rf < 2; ++rf) {   // the winner's distribution, from the winning lane
+    const int src = head ? R.seg + (bi[rf] & 0x7fff) : lane;
+    wm[rf] = __shfl_sync(0xffffffffu, om[rf], src);
+    wv[rf] = __shfl_sync(0xffffffffu, ov[rf], src);
+    wsg[rf] = kLSE ? __shfl_sync(0xffffffffu, osg[rf], src) : 0.f;
+  }
+  if (kLSE) {
+    const int src_lane = act ? R.seg : lane;
+    float w0[2], w1[2], inv[2];
 #pragma unroll
-    for (int rf = 0; rf < 2; ++rf) {   // the winner's distribution, from the winning lane
-      const int src = head ? R[r].seg + (bi[r][rf] & 0x7fff) : lane;
-      wm[rf] = __shfl_sync(0xffffffffu, om[r][rf], src);
-      wv[rf] = __shfl_sync(0xffffffffu, ov[r][rf], src);
-      wsg[rf] = kLSE ? __shfl_sync(0xffffffffu, osg[r][rf], src) : 0.f;
-    }
-    if (!kLSE) {
-      if (head) {
-        store_state(P, i, wm[0], wm[1], wv[0], wv[1]);
-        P.win[i] = bi[r][0] | (bi[r][1] << 16);
+    for (int rf = 0; rf < 2; ++rf) {
+      const double best = __shfl_sync(0xffffffffu, bA[rf], src_lane);   // M of my pin
+      w0[rf] = act ? lse_w(A0[rf], best, P.inv_tau) : 0.f;
+      w1[rf] = act && u == 2 ? lse_w(A1[rf], best, P.inv_tau) : 0.f;
+      // normalizer in merge_rf's order, accumulated by the pin's first lane
+      float acc = 0.f;
+      for (int j = 0; j < maxlen; ++j) {
+        const float v0 = __shfl_down_sync(0xffffffffu, w0[rf], j);
+        const float v1 = __shfl_down_sync(0xffffffffu, w1[rf], j);
+        if (j < R.seg_end - lane) {
+          acc += v0;
+          acc += v1;   // 0 for non-NON arcs: exact no-op on a non-negative sum
+        }
       }
-    } else {
-      const int src_lane = act[r] ? R[r].seg : lane;
-      float w0[2], w1[2], inv[2];
+      if (head) wm[rf] = lse_arrival(bA[rf], double(P.tau), acc) - ns * double(wsg[rf]);   // Eq 4, R1
+      inv[rf] = 1.f / __shfl_sync(0xffffffffu, acc, src_lane);   // as arc_weights
+    }
+    if (act) {
+      float wt[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
 #pragma unroll
       for (int rf = 0; rf < 2; ++rf) {
-        const double best = __shfl_sync(0xffffffffu, bA[r][rf], src_lane);   // M of my pin
-        w0[rf] = act[r] ? lse_w(A0[r][rf], best, P.inv_tau) : 0.f;
-        w1[rf] = act[r] && u[r] == 2 ? lse_w(A1[r][rf], best, P.inv_tau) : 0.f;
-        // normalizer in merge_rf's order, accumulated by the pin's first lane
-        float acc = 0.f;
-        for (int j = 0; j < maxlen; ++j) {
-          const float v0 = __shfl_down_sync(0xffffffffu, w0[rf], j);
-          const float v1 = __shfl_down_sync(0xffffffffu, w1[rf], j);
-          if (j < R[r].seg_end - lane) {
-            acc += v0;
-            acc += v1;   // 0 for non-NON arcs: exact no-op on a non-negative sum
-          }
-        }
-        if (head) wm[rf] = lse_arrival(bA[r][rf], double(P.tau), acc) - ns * double(wsg[rf]);   // Eq 4, R1
-        inv[rf] = 1.f / __shfl_sync(0xffffffffu, acc, src_lane);   // as arc_weights
+        wt[rf][src_tr(rf, u, 0)] = w0[rf] * inv[rf];
+        if (u == 2) wt[rf][rf ^ 1] = w1[rf] * inv[rf];
       }
-      if (head) store_state(P, i, wm[0], wm[1], wv[0], wv[1]);
-      if (act[r]) {
-        float wt[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
-#pragma unroll
-        for (int rf = 0; rf < 2; ++rf) {
-          wt[rf][src_tr(rf, u[r], 0)] = w0[rf] * inv[rf];
-          if (u[r] == 2) wt[rf][rf ^ 1] = w1[rf] * inv[rf];
-        }
-        // fanin position of my arc: row start of my pin + k
-        const int qpos = kFold ? S.q0[po + R[r].q + __popc(R[r].heads & ((2u << lane) - 1u)) - 1] + k[r]
-                               : A.z + R[r].base + lane;
-        P.wts[qpos] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
-      }
+      // fanin position of my arc: row start of my pin + k
+      const int qpos = kFold ? S.q0[po + R.q + __popc(R.heads & ((2u << lane) - 1u)) - 1] + k : A.z + R.base + lane;
+      P.wts[qpos] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
     }
+  }
+  if (head) {
+    const uint32_t chg = (kInc && hdirty && record_changed(*hold, wm[0], wm[1], wv[0], wv[1])) ? 1u : 0u;
+    store_state(P, i, wm[0], wm[1], wv[0], wv[1], chg);
+    if (!kLSE) P.win[i] = bi[0] | (bi[1] << 16);
   }
 }
 
 // kFold: the stage-folded schedule (fold.cpp): items are head ranges, entries
 // through a folded pin first compute that pin from the gathered source words
 // (fold_pin) and continue with its words in place of the source's.
-template <bool kLSE, bool kFold>
+// kInc (requires kFold): incremental dataflow pass.  Every
+// head waits for its sources as in a full pass; a head marked dirty (by
+// insta_update_arcs or by a changed source head) is recomputed with the same
+// code, a clean one only republishes its previous record with this pass's
+// parity.  A recomputed head whose record changed marks its consumer heads
+// before publishing.  Bit-identical to a full pass (tested).
+template <bool kInc>
+__device__ __forceinline__ void count_recomputed(const KParams& P, int n) {
+  if (kInc && n) atomicAdd(P.counters, (unsigned long long)n);
+}
+
+template <bool kLSE, bool kFold, bool kInc>
 __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
   extern __shared__ __align__(128) unsigned char smem[];
   FwdStage* stage = reinterpret_cast<FwdStage*>(smem);
   Raw* gath_all = reinterpret_cast<Raw*>(smem + 2 * sizeof(FwdStage));
+  Raw* hrec_all = gath_all + 2 * kFwdArcs;
   __shared__ __align__(8) uint64_t full[2], empty[2];
   const int c = blockIdx.x, tid = threadIdx.x;
   const int warp = tid >> 5, lane = tid & 31;
@@ -509,8 +540,12 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
       if (B.x == 0) {
         // startpoints: clock arrival distribution, mean and variance per rf
         for (int i = A.x + wt; i < A.y; i += kWorkers) {
-          const float4 v = __ldg(P.src_ms + i);
-          store_state(P, i, double(v.x), double(v.y), double(v.z) * double(v.z), double(v.w) * double(v.w));
+          if (kInc) {
+            republish(P, i, ld_state_raw(P, i));   // arc updates never change a startpoint
+          } else {
+            const float4 v = __ldg(P.src_ms + i);
+            store_state(P, i, double(v.x), double(v.y), double(v.z) * double(v.z), double(v.w) * double(v.w));
+          }
         }
       } else if (!(B.y & kItemDirect)) {
         const FwdStage& S = stage[s];
@@ -519,7 +554,7 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
         // this warp's contiguous share of the item's pins
         const int q0 = ww * np / kWorkerWarps, q1 = (ww + 1) * np / kWorkerWarps;
         const int a_lo = S.ptr[po + q0] - A.z, a_hi = S.ptr[po + q1] - A.z;
-        if (q1 > q0 && a_hi - a_lo == q1 - q0) {
+        if (!kInc && q1 > q0 && a_hi - a_lo == q1 - q0) {
           // every pin has fanin 1 (net sinks): register gathers, all issued
           // before any is awaited; same merge function (nf = 1) as below
           Raw r[kFastPins];
@@ -542,6 +577,23 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
           }
         } else if (q1 > q0) {
           Round R = round_at(S, A, po, so, q0, q1, lane);
+          Raw* hrec = hrec_all + ww * kHeadsPerWarp;
+          uint32_t stampm[kStampWords];
+          if (kInc) {   // previous records and update stamps of this warp's heads
+            for (int p = q0 + lane; p < q1; p += 32) {
+              const PinState* src = P.state + S.pin[po + p];
+              const uint32_t d = smem_u32(hrec + (p - q0));
+              asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n\t"
+                           "cp.async.cg.shared.global [%2], [%3], 16;" ::"r"(d),
+                           "l"(src), "r"(d + 16u), "l"(reinterpret_cast<const char*>(src) + 16)
+                           : "memory");
+            }
+#pragma unroll
+            for (int j = 0; j < kStampWords; ++j) {   // loads issued now, consumed after the gathers land
+              const int p = q0 + lane + 32 * j;
+              stampm[j] = p < q1 ? __ldcg(P.dirty_h + A.x + p) : 0u;
+            }
+          }
           // (1) gathers of all this warp's arcs: cp.async through L2, then
           // re-poll the stale ones (producer not done yet)
           for (int a = a_lo + lane; a < a_hi; a += 32) {
@@ -554,6 +606,11 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
           }
           asm volatile("cp.async.wait_all;" ::: "memory");
           if (P.trace && wt == 0) P.trace[(size_t(c) * nsteps + t) * 4 + 1] = gtimer();
+          if (kInc) {
+#pragma unroll
+            for (int j = 0; j < kStampWords; ++j)
+              stampm[j] = __ballot_sync(0xffffffffu, q0 + lane + 32 * j < q1 && stampm[j] == P.stamp);
+          }
           if (P.mode == 2) {
             for (int a = a_lo + lane; a < a_hi; a += 32) {
               Raw r = gath[a];
@@ -563,7 +620,7 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
               }
             }
           }
-          if (kFold) {   // entries through folded pins: compute the folded pin first
+          if (kFold && !kInc) {   // entries through folded pins: compute the folded pin first
             for (int a = a_lo + lane; a < a_hi; a += 32) {
               if ((S.src[so + a] >> kFoldBit) & 1) gath[a] = fold_pin<kLSE>(P, S.f[so + a], S.fms[a], S.fq[so + a], gath[a]);
             }
@@ -577,30 +634,58 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
               const int q = R.q, base = R.base;
               if (lane == 0) {
                 const int nf = S.ptr[po + q + 1] - A.z - base;
-                fwd_pin<kLSE>(P, kFold ? S.pin[po + q] : A.x + q, nf, kFold ? S.q0[po + q] : A.z + base,
-                              [&](int kk, int32_t& w_, float4& ms_, Raw& r_) {
+                const int i = kFold ? S.pin[po + q] : A.x + q;
+                const int qf = kFold ? S.q0[po + q] : A.z + base;
+                auto arc = [&](int kk, int32_t& w_, float4& ms_, Raw& r_) {
                   w_ = S.src[so + base + kk];
                   ms_ = S.ms[base + kk];
                   r_ = gath[base + kk];
-                });
+                };
+                if (!kInc) {
+                  fwd_pin<kLSE>(P, i, nf, qf, arc);
+                } else {
+                  const int hr = q - q0;
+                  bool dirty = (stampm[min(hr >> 5, kStampWords - 1)] >> (hr & 31)) & 1u;
+                  for (int kk = 0; kk < nf; ++kk) dirty |= tag_changed(gath[base + kk].d) != 0u;
+                  if (!dirty) {
+                    republish(P, i, hrec[hr]);
+                  } else {
+                    count_recomputed<kInc>(P, 1);
+                    for (int kk = 0; kk < nf; ++kk)   // folded pins first (the incremental pass has no pre-pass)
+                      if ((S.src[so + base + kk] >> kFoldBit) & 1)
+                        gath[base + kk] = fold_pin<kLSE>(P, S.f[so + base + kk], S.fms[base + kk], S.fq[so + base + kk],
+                                                         gath[base + kk]);
+                    fwd_pin_inc<kLSE>(P, i, nf, qf, hrec[hr], arc);
+                  }
+                }
               }
               __syncwarp();
               R = round_at(S, A, po, so, q + 1, q1, lane);
               continue;
             }
-            Round RR[kRoundsPerPass];
-            RR[0] = R;
-            int qn = R.q + R.cnt;
+            if (kInc) {
+              // a head is dirty if stamped or if any of its entries' sources changed
+              const bool act = lane < R.na;
+              const uint32_t cb = __ballot_sync(0xffffffffu, act && tag_changed(gath[R.base + lane].d) != 0u);
+              const bool head = act && lane == R.seg;
+              const int hr = R.q + __popc(R.heads & ((1u << lane) - 1u)) - q0;   // head lanes
+              const uint32_t seg = (R.seg_end >= 32 ? 0xffffffffu : ((1u << R.seg_end) - 1u)) & ~((1u << lane) - 1u);
+              uint32_t sw = 0u;
 #pragma unroll
-            for (int r = 1; r < kRoundsPerPass; ++r) {
-              RR[r] = round_at(S, A, po, so, min(qn, q1), q1, lane);
-              if (qn >= q1 || RR[r].cnt == 0) {
-                RR[r].na = 0;   // inactive slot
-                RR[r].cnt = 0;
+              for (int j = 0; j < kStampWords; ++j)
+                if ((hr >> 5) == j) sw = stampm[j];
+              const bool dirty = head && ((((sw >> (hr & 31)) & 1u) != 0u) || (cb & seg) != 0u);
+              const uint32_t dm = __ballot_sync(0xffffffffu, dirty);
+              if (dm == 0) {   // no dirty head in this round: republish
+                if (lane < R.cnt) republish(P, S.pin[po + R.q + lane], hrec[R.q + lane - q0]);
+              } else {
+                if (lane == 0) count_recomputed<kInc>(P, __popc(dm));
+                fwd_round<kLSE, kFold, true>(P, gath, A, S, po, so, R, lane, dirty, hrec + (head ? hr : 0));
               }
-              qn += RR[r].cnt;
+            } else {
+              fwd_round<kLSE, kFold, false>(P, gath, A, S, po, so, R, lane);
             }
-            fwd_rounds<kLSE, kFold, kRoundsPerPass>(P, gath, A, S, po, RR, lane);
+            const int qn = R.q + R.cnt;
             if (qn < q1) R = round_at(S, A, po, so, qn, q1, lane);
             else break;
           }
@@ -609,16 +694,34 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
         for (int h = A.x + wt; h < A.y; h += kWorkers) {
           const int b0 = __ldg(P.fanin_ptr + h);
           const int nf = __ldg(P.fanin_ptr + h + 1) - b0;
-          fwd_pin<kLSE>(P, kFold ? __ldg(P.hd_pin + h) : h, nf, kFold ? __ldg(P.hd_q0 + h) : b0,
-                        [&](int kk, int32_t& w, float4& ms, Raw& rr) {
-                          w = __ldg(P.fin_src + b0 + kk);
-                          ms = __ldg(P.fin_ms + b0 + kk);
-                          rr = ld_state_raw(P, w & kSrcMask);
-                          await_raw(P, w & kSrcMask, rr);
-                          if (kFold && ((w >> kFoldBit) & 1))   // recomputed per call: same words
-                            rr = fold_pin<kLSE>(P, __ldg(P.ext_f + b0 + kk), __ldg(P.ext_fms + b0 + kk),
-                                                __ldg(P.ext_fq + b0 + kk), rr);
-                        });
+          const int i = kFold ? __ldg(P.hd_pin + h) : h;
+          const int qf = kFold ? __ldg(P.hd_q0 + h) : b0;
+          auto arc = [&](int kk, int32_t& w, float4& ms, Raw& rr) {
+            w = __ldg(P.fin_src + b0 + kk);
+            ms = __ldg(P.fin_ms + b0 + kk);
+            rr = ld_state_raw(P, w & kSrcMask);
+            await_raw(P, w & kSrcMask, rr);
+            if (kFold && ((w >> kFoldBit) & 1))   // recomputed per call: same words
+              rr = fold_pin<kLSE>(P, __ldg(P.ext_f + b0 + kk), __ldg(P.ext_fms + b0 + kk), __ldg(P.ext_fq + b0 + kk), rr);
+          };
+          if (!kInc) {
+            fwd_pin<kLSE>(P, i, nf, qf, arc);
+          } else {
+            const Raw old = ld_state_raw(P, i);
+            bool dirty = __ldcg(P.dirty_h + h) == P.stamp;
+            for (int kk = 0; kk < nf; ++kk) {   // wait for every source; any changed one dirties the head
+              const int32_t w = __ldg(P.fin_src + b0 + kk);
+              Raw rr = ld_state_raw(P, w & kSrcMask);
+              await_raw(P, w & kSrcMask, rr);
+              dirty |= tag_changed(rr.d) != 0u;
+            }
+            if (!dirty) {
+              republish(P, i, old);
+            } else {
+              count_recomputed<kInc>(P, 1);
+              fwd_pin_inc<kLSE>(P, i, nf, qf, old, arc);
+            }
+          }
         }
       }
     }
@@ -1444,8 +1547,7 @@ __global__ void update_arcs_kernel(int64_t n, const int32_t* __restrict__ ids,
                                    const float2* __restrict__ sigma,
                                    const int32_t* __restrict__ arc_pos, float4* fin_ms,
                                    const int32_t* __restrict__ arc_xpos, float4* ext_ms, float4* ext_fms,
-                                   const int32_t* __restrict__ arc_sink, const int32_t* __restrict__ pin_level,
-                                   uint32_t* dirty, uint32_t stamp, int32_t* lvl_range) {
+                                   const int32_t* __restrict__ arc_head, uint32_t* dirty_h, uint32_t stamp) {
   const int64_t k = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
   if (k >= n) return;
   const int q = arc_pos[ids[k]];
@@ -1453,173 +1555,7 @@ __global__ void update_arcs_kernel(int64_t n, const int32_t* __restrict__ ids,
   fin_ms[q] = make_float4(m.x, m.y, s.x, s.y);
   const int x = arc_xpos[ids[k]];   // the stage-folded schedule's copy of the record
   ((x & 1) ? ext_fms : ext_ms)[x >> 1] = make_float4(m.x, m.y, s.x, s.y);
-  if (dirty) {   // incremental: the sink must be recomputed in the next pass
-    const int i = arc_sink[ids[k]];
-    dirty[i] = stamp;
-    atomicMin(lvl_range, pin_level[i]);
-    atomicMax(lvl_range + 1, pin_level[i]);
-  }
-}
-
-// --------------------------------------------------------------------------
-// Incremental forward ("re-annotate ... then
-// re-propagate").  Level-synchronous persistent kernel over the same items:
-// level l starts when every CTA has published level l-1 (fence.acq_rel + red /
-// ld.acquire counters), so all dirty marks that target level l are visible.
-// A pin is recomputed only if marked dirty; it is recomputed with the same
-// device function as the full forward, so its result equals the full pass bit
-// for bit.  If the new (mu, var) differ from the old ones, every fanout sink
-// is marked (full fanout CSR) and the deepest marked level is raised; the pass
-// stops as soon as the next level is deeper than any mark (cone exhausted).
-// Records keep the parity of the last full pass.
-// --------------------------------------------------------------------------
-struct IncParams {
-  KParams P;
-  const int32_t* __restrict__ fanout_ptr;
-  const int32_t* __restrict__ fout_sink;
-  const int32_t* __restrict__ pin_level;
-  const int32_t* __restrict__ max_sink_level;   // deepest level among a pin's fanout sinks (-1: none)
-  uint32_t* dirty;
-  uint32_t stamp;
-  int32_t* lvl_range;        // {min dirty level, max dirty level}
-  uint32_t* done;            // [L] zeroed per pass; target = grid
-  unsigned long long* counters;  // [0] pins recomputed, [1] pins changed
-};
-
-__device__ __forceinline__ void inc_wait(const IncParams& Q, int l) {
-  if (threadIdx.x == 0) {
-    while (ld_acquire(Q.done + l) != uint32_t(Q.P.grid)) __nanosleep(32);
-  }
-  __syncthreads();
-}
-
-template <bool kLSE>
-__global__ void __launch_bounds__(kThreads, 1) inc_kernel(IncParams Q) {
-  const KParams& P = Q.P;
-  const int c = blockIdx.x, tid = threadIdx.x;
-  __shared__ int s_exit;
-  __shared__ unsigned long long s_cnt[2];
-  constexpr int kWideMarks = 128;
-  __shared__ int s_wide[kWideMarks];
-  __shared__ int s_nwide;
-  const int lmin = __ldcg(Q.lvl_range);
-  if (tid == 0) s_cnt[0] = s_cnt[1] = 0ull;
-  for (int k = P.step_begin; k < P.step_end; ++k) {
-    const int4 A = __ldg(P.item_a + size_t(k) * P.grid + c);
-    const int4 B = __ldg(P.item_b + size_t(k) * P.grid + c);
-    const int l = B.x;
-    if (l < lmin) continue;   // below the shallowest mark: nothing to do, nothing to publish
-    if (l > lmin) inc_wait(Q, l - 1);
-    if (tid == 0) {
-      s_exit = l > ld_acquire(reinterpret_cast<const uint32_t*>(Q.lvl_range + 1)) ? 1 : 0;
-      s_nwide = 0;
-    }
-    __syncthreads();
-    if (s_exit) break;
-    for (int i = A.x + tid; i < A.y; i += kThreads) {
-      if (__ldcg(Q.dirty + i) != Q.stamp) continue;
-      const int b0 = __ldg(P.fanin_ptr + i), nf = __ldg(P.fanin_ptr + i + 1) - b0;
-      const Gath old = load_state_plain(P.state + i);
-      double mu0, mu1, v0, v1;
-      if (l == 0) {
-        const float4 v = __ldg(P.src_ms + i);
-        mu0 = double(v.x);
-        mu1 = double(v.y);
-        v0 = double(v.z) * double(v.z);
-        v1 = double(v.w) * double(v.w);
-      } else {
-        // topology and source states of the first 4 arcs are loaded together
-        constexpr int kR = 4;
-        int32_t wv[kR];
-        float4 mv[kR];
-        Raw rv[kR];
-#pragma unroll
-        for (int kk = 0; kk < kR; ++kk) {
-          if (kk < nf) {
-            wv[kk] = __ldg(P.fin_src + b0 + kk);
-            mv[kk] = __ldg(P.fin_ms + b0 + kk);
-          }
-        }
-#pragma unroll
-        for (int kk = 0; kk < kR; ++kk)
-          if (kk < nf) rv[kk] = ld_state_raw(P, wv[kk] & kSrcMask);
-        auto arc = [&](int kk, int32_t& w, float4& ms, Raw& rr) {
-          if (kk < kR) {
-#pragma unroll
-            for (int x = 0; x < kR; ++x) {
-              if (x == kk) {
-                w = wv[x];
-                ms = mv[x];
-                rr = rv[x];
-              }
-            }
-          } else {
-            w = __ldg(P.fin_src + b0 + kk);
-            ms = __ldg(P.fin_ms + b0 + kk);
-            rr = ld_state_raw(P, w & kSrcMask);
-          }
-        };
-        const RfOut R = pin_rf<kLSE>(P, 0, nf, arc);
-        const RfOut F = pin_rf<kLSE>(P, 1, nf, arc);
-        if (!kLSE) {
-          P.win[i] = R.win | (F.win << 16);
-        } else {
-          for (int kk = 0; kk < nf; ++kk) {
-            const float2 wr = arc_rf_weights(P, 0, kk, R, arc);
-            const float2 wf = arc_rf_weights(P, 1, kk, F, arc);
-            P.wts[b0 + kk] = make_float4(wr.x, wr.y, wf.x, wf.y);
-          }
-        }
-        mu0 = R.mu;
-        mu1 = F.mu;
-        v0 = R.var;
-        v1 = F.var;
-      }
-      atomicAdd(&s_cnt[0], 1ull);
-      // compare with the stored (parity-stripped) value after the same truncation
-      const double n0 = strip((unsigned long long)__double_as_longlong(mu0));
-      const double n1 = strip((unsigned long long)__double_as_longlong(mu1));
-      const double w0 = strip((unsigned long long)__double_as_longlong(v0));
-      const double w1 = strip((unsigned long long)__double_as_longlong(v1));
-      if (__double_as_longlong(n0) != __double_as_longlong(old.mu0) ||
-          __double_as_longlong(n1) != __double_as_longlong(old.mu1) ||
-          __double_as_longlong(w0) != __double_as_longlong(old.v0) ||
-          __double_as_longlong(w1) != __double_as_longlong(old.v1)) {
-        store_state(P, i, mu0, mu1, v0, v1);
-        atomicAdd(&s_cnt[1], 1ull);
-        const int r0 = __ldg(Q.fanout_ptr + i), r1 = __ldg(Q.fanout_ptr + i + 1);
-        bool deferred = false;
-        if (r1 - r0 > 32) {   // wide fanout: marked cooperatively after the item
-          const int slot = atomicAdd(&s_nwide, 1);
-          if (slot < kWideMarks) {
-            s_wide[slot] = i;
-            deferred = true;
-          }
-        }
-        if (!deferred)
-          for (int r = r0; r < r1; ++r) Q.dirty[__ldg(Q.fout_sink + r)] = Q.stamp;
-        const int deepest = __ldg(Q.max_sink_level + i);
-        if (deepest >= 0) atomicMax(Q.lvl_range + 1, deepest);
-      }
-    }
-    __syncthreads();
-    // cooperative marking of the wide fanouts of changed pins
-    const int nw = min(s_nwide, kWideMarks);
-    for (int w = 0; w < nw; ++w) {
-      const int pin = s_wide[w];
-      for (int r = __ldg(Q.fanout_ptr + pin) + tid; r < __ldg(Q.fanout_ptr + pin + 1); r += kThreads)
-        Q.dirty[__ldg(Q.fout_sink + r)] = Q.stamp;
-    }
-    __syncthreads();
-    if ((B.y & kItemLast) && tid == 0) {
-      asm volatile("fence.acq_rel.gpu;\n\tred.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(Q.done + l) : "memory");
-    }
-  }
-  __syncthreads();
-  if (tid == 0) {
-    atomicAdd(Q.counters, s_cnt[0]);
-    atomicAdd(Q.counters + 1, s_cnt[1]);
-  }
+  if (dirty_h) dirty_h[arc_head[ids[k]]] = stamp;   // incremental: the head evaluating the arc recomputes
 }
 
 // --------------------------------------------------------------------------
@@ -1652,6 +1588,8 @@ static KParams make_params(DevGraph& g, bool bwd) {
   P.ext_arc = g.ext_arc;
   P.ext_farc = g.ext_farc;
   P.hseed = g.hseed;
+  P.dirty_h = g.dirty_h;
+  P.counters = g.counters;
   P.state = g.state;
   P.win = g.win;
   P.wts = g.wts;
@@ -1676,19 +1614,23 @@ int query_grid(int device, int* grid) {
   if (e != cudaSuccess) return int(e);
   cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, device);
   if (!coop) return int(cudaErrorNotSupported);
-  int err = set_smem(fwd_kernel<false, false>, kFwdSmemV6);
-  if (!err) err = set_smem(fwd_kernel<true, false>, kFwdSmemV6);
-  if (!err) err = set_smem(fwd_kernel<false, true>, kFwdSmemV6);
-  if (!err) err = set_smem(fwd_kernel<true, true>, kFwdSmemV6);
+  int err = set_smem(fwd_kernel<false, false, false>, kFwdSmemV6);
+  if (!err) err = set_smem(fwd_kernel<true, false, false>, kFwdSmemV6);
+  if (!err) err = set_smem(fwd_kernel<false, true, false>, kFwdSmemV6);
+  if (!err) err = set_smem(fwd_kernel<true, true, false>, kFwdSmemV6);
+  if (!err) err = set_smem(fwd_kernel<false, true, true>, kFwdSmemV6);
+  if (!err) err = set_smem(fwd_kernel<true, true, true>, kFwdSmemV6);
   if (!err) err = set_smem(bwd_kernel<false>, bwd_smem<false>());
   if (!err) err = set_smem(bwd_kernel<true>, bwd_smem<true>());
   if (!err) err = set_smem(bwdf_kernel<false>, kBwdfSmem);
   if (!err) err = set_smem(bwdf_kernel<true>, kBwdfSmem);
   if (err) return err;
   int occ = 1 << 30, b = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<false, true>, kFwdThreads, kFwdSmemV6);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<false, true, false>, kFwdThreads, kFwdSmemV6);
   occ = std::min(occ, b);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<true, true>, kFwdThreads, kFwdSmemV6);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<true, true, false>, kFwdThreads, kFwdSmemV6);
+  occ = std::min(occ, b);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fwd_kernel<true, true, true>, kFwdThreads, kFwdSmemV6);
   occ = std::min(occ, b);
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bwd_kernel<false>, kThreads, bwd_smem<false>());
   occ = std::min(occ, b);
@@ -1773,12 +1715,7 @@ int launch_forward(DevGraph& g, float n_sigma, float tau, int schedule, void* st
   P.tau = tau;
   P.inv_tau = tau > 0.f ? 1.0 / double(tau) : 0.0;
   const bool lse = tau > 0.f;
-  {   // a full pass supersedes pending incremental marks
-    ++g.inc_epoch;
-    const int32_t init[2] = {0x7fffffff, -1};
-    cudaError_t e = cudaMemcpyAsync(g.lvl_range, init, sizeof init, cudaMemcpyHostToDevice, st);
-    if (e != cudaSuccess) return int(e);
-  }
+  ++g.inc_epoch;   // a full pass supersedes pending incremental marks
   if (g.n > 0) {
     P.mode = schedule == 0 ? 2 : 0;   // dataflow persistent / one launch per level
     P.par = (++g.pass_fwd) & 1u;
@@ -1789,10 +1726,10 @@ int launch_forward(DevGraph& g, float n_sigma, float tau, int schedule, void* st
       P.fanin_ptr = g.hd_ptr;
       P.fin_src = g.ext_w;
       P.fin_ms = g.ext_ms;
-      err = launch_items(lse ? (const void*)fwd_kernel<true, true> : (const void*)fwd_kernel<false, true>,
+      err = launch_items(lse ? (const void*)fwd_kernel<true, true, false> : (const void*)fwd_kernel<false, true, false>,
                          kFwdThreads, kFwdSmemV6, P, g.fwdf_items, false, st);
     } else {   // the paper's launch structure: one launch per timing level
-      err = launch_items(lse ? (const void*)fwd_kernel<true, false> : (const void*)fwd_kernel<false, false>,
+      err = launch_items(lse ? (const void*)fwd_kernel<true, false, false> : (const void*)fwd_kernel<false, false, false>,
                          kFwdThreads, kFwdSmemV6, P, g.fwd_items, false, st);
     }
     if (err) return err;
@@ -1882,46 +1819,35 @@ int launch_update_arcs(DevGraph& g, int64_t n, const int32_t* ids, const float* 
   const int blocks = int((n + 255) / 256);
   update_arcs_kernel<<<blocks, 256, 0, st>>>(n, ids, reinterpret_cast<const float2*>(mean),
                                              reinterpret_cast<const float2*>(sigma), g.arc_pos,
-                                             g.fin_ms, g.arc_xpos, g.ext_ms, g.ext_fms, g.arc_sink, g.pin_level,
-                                             incremental ? g.dirty : nullptr, g.inc_epoch + 1, g.lvl_range);
+                                             g.fin_ms, g.arc_xpos, g.ext_ms, g.ext_fms, g.arc_head,
+                                             incremental ? g.dirty_h : nullptr, g.inc_epoch + 1);
   return int(cudaGetLastError());
 }
 
-// Incremental pass over the dirty cone, then slack/TNS.  Requires the previous
-// forward to have used the same (n_sigma, tau).
+// Incremental pass over the dirty cone (dataflow, stage-folded schedule), then
+// slack/TNS.  Requires the previous forward to have used the same (n_sigma, tau).
 int launch_forward_incremental(DevGraph& g, float n_sigma, float tau, void* stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  IncParams Q{};
-  Q.P = make_params(g, false);
-  Q.P.n_sigma = n_sigma;
-  Q.P.tau = tau;
-  Q.P.inv_tau = tau > 0.f ? 1.0 / double(tau) : 0.0;
-  Q.P.mode = 1;
-  Q.P.par = g.pass_fwd & 1u;   // keep the parity of the last full pass
-  Q.P.step_begin = 0;
-  Q.P.step_end = g.fwd_items.num_steps;
-  Q.fanout_ptr = g.fanout_ptr;
-  Q.fout_sink = g.fout_sink;
-  Q.pin_level = g.pin_level;
-  Q.max_sink_level = g.max_sink_level;
-  Q.dirty = g.dirty;
-  Q.stamp = ++g.inc_epoch;
-  Q.lvl_range = g.lvl_range;
-  Q.done = g.done_fwd;
-  Q.counters = g.counters;
-  cudaError_t e = cudaMemsetAsync(g.done_fwd, 0, sizeof(uint32_t) * size_t(std::max(g.num_levels, 1)), st);
-  if (e == cudaSuccess) e = cudaMemsetAsync(g.counters, 0, sizeof(unsigned long long) * 2, st);
+  KParams P = make_params(g, false);
+  P.n_sigma = n_sigma;
+  P.tau = tau;
+  P.inv_tau = tau > 0.f ? 1.0 / double(tau) : 0.0;
+  P.mode = 2;
+  P.par = (++g.pass_fwd) & 1u;
+  P.stamp = ++g.inc_epoch;
+  P.item_a = g.fwdf_a;
+  P.item_b = g.fwdf_b;
+  P.fanin_ptr = g.hd_ptr;
+  P.fin_src = g.ext_w;
+  P.fin_ms = g.ext_ms;
+  cudaError_t e = cudaMemsetAsync(g.counters, 0, sizeof(unsigned long long) * 2, st);
   if (e != cudaSuccess) return int(e);
   if (g.n > 0) {
-    void* args[] = {&Q};
-    e = cudaLaunchCooperativeKernel(tau > 0.f ? (const void*)inc_kernel<true> : (const void*)inc_kernel<false>,
-                                    dim3(g.grid), dim3(kThreads), args, 0, st);
-    if (e != cudaSuccess) return int(e);
+    const int err = launch_items(tau > 0.f ? (const void*)fwd_kernel<true, true, true>
+                                           : (const void*)fwd_kernel<false, true, true>,
+                                 kFwdThreads, kFwdSmemV6, P, g.fwdf_items, false, st);
+    if (err) return err;
   }
-  // reset the level range for the next round of marks: {INT_MAX, -1}
-  const int32_t init[2] = {0x7fffffff, -1};
-  e = cudaMemcpyAsync(g.lvl_range, init, sizeof init, cudaMemcpyHostToDevice, st);
-  if (e != cudaSuccess) return int(e);
   g.last_n_sigma = n_sigma;
   g.last_tau = tau;
   return launch_slack(g, stream);

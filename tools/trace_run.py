@@ -23,6 +23,10 @@ for _ in range(3):
     G.forward(3.0, tau, sync=False)
     G.backward()
 torch.cuda.synchronize()
+if os.environ.get("INC"):   # trace an incremental forward after a 1 % sizing step
+    ids, m, s_ = synth.sizing_step(g, 0, frac=0.01)
+    G.update_arcs(ids, m, s_, incremental=True)
+    torch.cuda.synchronize()
 os.environ["INSTA_TRACE_DIR"] = out
 G.forward(3.0, tau, sync=False)
 G.backward()
