@@ -62,7 +62,7 @@ void free_graph(insta::DevGraph& d) {
                   d.hlfo_ptr,  d.hlfo,      d.ext_qpos,  d.ext_bw,     d.ext_arc,   d.ext_farc,
                   d.ep_head,   d.hseed,     d.bwdf_a,    d.bwdf_b,    d.g4,        d.hacc4,
                   d.ext_flags, d.bfwdf_a,   d.bfwdf_b,   d.b_ov_key,  d.hd_eop,    d.dirty_h,
-                  d.arc_head};
+                  d.arc_head,  d.ext_h};
   for (void* p : ptrs)
     if (p) cudaFree(p);
 }
@@ -299,6 +299,7 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   UP(d.ext_bw, fold.ext_bw.data(), fold.ext_bw.size());
   UP(d.ext_arc, fold.ext_arc.data(), fold.ext_arc.size());
   UP(d.ext_farc, fold.ext_farc.data(), fold.ext_farc.size());
+  UP(d.ext_h, fold.ext_h.data(), fold.ext_h.size());
   UP(d.ep_head, fold.ep_head.data(), fold.ep_head.size());
   UP(d.hd_eop, fold.hd_eop.data(), fold.hd_eop.size());
   ZERO(d.dirty_h, fold.hd_pin.size());

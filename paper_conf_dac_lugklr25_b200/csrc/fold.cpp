@@ -83,6 +83,7 @@ void build_fold(const HostLevels& h, const std::vector<int32_t>& fin_src, const 
   f.ext_bw.assign(size_t(X), 0);
   f.ext_arc.assign(size_t(X), 0);
   f.ext_farc.assign(size_t(X), -1);
+  f.ext_h.assign(size_t(X), 0);
   f.hd_hslot.assign(size_t(H), -1);
   f.hd_eop.assign(size_t(H), -1);
   f.hlfo_ptr.assign(size_t(H) + 1, 0);
@@ -103,6 +104,7 @@ void build_fold(const HostLevels& h, const std::vector<int32_t>& fin_src, const 
       f.ext_ms[x] = fin_ms[y];
       f.arc_xpos[h.fanin_arc[y]] = int32_t(2 * x);
       f.ext_qpos[x] = y;
+      f.ext_h[x] = hh;
       f.ext_arc[x] = h.fanin_arc[y];
       f.ext_bw[x] = fin_src[y];
       if (f.folded[p]) {

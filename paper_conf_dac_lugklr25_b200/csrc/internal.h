@@ -103,6 +103,7 @@ struct FoldHost {
   std::vector<int32_t> ext_bw;      // [X] fin_src word of the arc whose adjoint the entry writes (e, or e' if folded)
   std::vector<int32_t> ext_arc;     // [X] caller id of e
   std::vector<int32_t> ext_farc;    // [X] caller id of e' (-1 if not folded)
+  std::vector<int32_t> ext_h;       // [X] head of each entry
   std::vector<int32_t> ep_head;     // [P] head index of each endpoint (endpoints are never folded)
   std::vector<int32_t> hd_eop;      // [H] endpoint index of each head (-1: not an endpoint)
   // incremental pass
@@ -194,6 +195,7 @@ struct DevGraph {
   int32_t* ext_bw = nullptr;
   int32_t* ext_arc = nullptr;
   int32_t* ext_farc = nullptr;
+  int32_t* ext_h = nullptr;
   int32_t* ep_head = nullptr;
   int32_t* hd_eop = nullptr;       // [H] endpoint index of each head, -1 otherwise
   uint32_t* dirty_h = nullptr;     // [H] incremental: stamp == inc epoch -> recompute

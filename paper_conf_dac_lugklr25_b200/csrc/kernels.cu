@@ -74,6 +74,7 @@ struct KParams {
   const int32_t* __restrict__ ext_bw;
   const int32_t* __restrict__ ext_arc;
   const int32_t* __restrict__ ext_farc;
+  const int32_t* __restrict__ ext_h;
   const float2* hseed;
   // incremental dataflow pass on the folded schedule
   const uint32_t* dirty_h;                   // [H] stamp == `stamp`: head must be recomputed
@@ -850,6 +851,21 @@ __device__ __forceinline__ void heavy_tab_flush(const KParams& P, HeavyTab* tab)
 
 __device__ __forceinline__ long long heavy_count(long long acc) { return (acc + (kCountUnit >> 1)) >> 44; }
 
+// read-only variant: the accumulators are zeroed before the pass, so every
+// entry of a heavy head can read the completed sum
+__device__ __forceinline__ float2 heavy_read(const KParams& P, int slot) {
+  if (slot < 0) return make_float2(0.f, 0.f);
+  const long long target = __ldg(P.heavy_fo + slot);
+  unsigned long long x, y;
+  ld2_u64(P.heavy_acc + 2 * slot, x, y);
+  while (heavy_count((long long)x) != target || heavy_count((long long)y) != target) {
+    __nanosleep(32);
+    ld2_u64(P.heavy_acc + 2 * slot, x, y);
+  }
+  const long long vx = (long long)x - target * kCountUnit, vy = (long long)y - target * kCountUnit;
+  return make_float2(float(double(vx) / kFixH), float(double(vy) / kFixH));
+}
+
 __device__ __forceinline__ float2 heavy_take(const KParams& P, int slot) {
   if (slot < 0) return make_float2(0.f, 0.f);
   // wait until every sink arc has arrived in both words, then decode and reset
@@ -1054,11 +1070,11 @@ struct BwdfStage {
   int32_t pin[kBwdPins + 8];    // canonical pin of each head (arg-max / source gathers)
   int32_t qpos[kBwdArcs + 8];   // fanin position of each entry's arc e (weights, adjoint word)
   int32_t f[kBwdArcs + 8];      // folded pin word of each entry (arg-max gather)
+  int32_t eh[kBwdArcs + 8];     // head of each entry
 };
 constexpr int kEntPerThread = kBwdArcs / kThreads;
 constexpr int kHeadsPerThread = kBwdPins / kThreads;
-constexpr size_t kBwdfSmem = 2 * sizeof(BwdfStage) + sizeof(float2) * kBwdFanout + sizeof(float2) * kBwdArcs +
-                             sizeof(int32_t) * kBwdArcs + sizeof(HeavyTab);
+constexpr size_t kBwdfSmem = 2 * sizeof(BwdfStage) + sizeof(float2) * kBwdFanout + sizeof(HeavyTab);
 
 template <bool kLSE>
 __device__ __forceinline__ void bwdf_prefetch(const KParams& P, BwdfStage* st, uint64_t* full, int step, int c) {
@@ -1070,7 +1086,7 @@ __device__ __forceinline__ void bwdf_prefetch(const KParams& P, BwdfStage* st, u
   const Window wh = window(A.x, A.y, 4);
   const Window wx = window(B.x, B.y, 4);
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-  mbar_expect_tx(full, 2 * wl.bytes + wf.bytes + wh.bytes + (kLSE ? 1 : 2) * wx.bytes);
+  mbar_expect_tx(full, 2 * wl.bytes + wf.bytes + wh.bytes + (kLSE ? 2 : 3) * wx.bytes);
   bulk_g2s(st->lptr, P.lfo_ptr + wl.start, wl.bytes, full);
   bulk_g2s(st->hptr, P.fanin_ptr + wl.start, wl.bytes, full);
   if (wf.bytes) bulk_g2s(st->lfo, P.lfo + wf.start, wf.bytes, full);
@@ -1078,6 +1094,7 @@ __device__ __forceinline__ void bwdf_prefetch(const KParams& P, BwdfStage* st, u
   if (wx.bytes) {
     bulk_g2s(st->qpos, P.ext_qpos + wx.start, wx.bytes, full);
     if (!kLSE) bulk_g2s(st->f, P.ext_f + wx.start, wx.bytes, full);
+    bulk_g2s(st->eh, P.ext_h + wx.start, wx.bytes, full);
   }
 }
 
@@ -1172,9 +1189,7 @@ __global__ void __launch_bounds__(kThreads, 1) bwdf_kernel(KParams P) {
   extern __shared__ __align__(128) unsigned char smem[];
   BwdfStage* stage = reinterpret_cast<BwdfStage*>(smem);
   float2* gg = reinterpret_cast<float2*>(smem + 2 * sizeof(BwdfStage));
-  float2* eab = gg + kBwdFanout;                                    // per entry: head adjoint
-  int32_t* esel = reinterpret_cast<int32_t*>(eab + kBwdArcs);       // per entry: hard-mode selection
-  HeavyTab* htab = reinterpret_cast<HeavyTab*>(esel + kBwdArcs);
+  HeavyTab* htab = reinterpret_cast<HeavyTab*>(gg + kBwdFanout);
   __shared__ __align__(8) uint64_t full[2];
   const int c = blockIdx.x;
   const int tid = threadIdx.x;
@@ -1201,23 +1216,21 @@ __global__ void __launch_bounds__(kThreads, 1) bwdf_kernel(KParams P) {
       phase[buf] ^= 1u;
       const BwdfStage& S = stage[buf];
       const int lo = A.x & 3, fo = A.z & 3, xo = B.x & 3;
-      // entry and head inputs: independent of the dependency chain, issued first
+      // entry inputs (with their head's seed, heavy slot and arg-max): independent
+      // of the dependency chain, issued first
       EntryIn ein[kEntPerThread];
+      int32_t ehr[kEntPerThread], eslot[kEntPerThread], ewin[kEntPerThread];
+      float2 esd[kEntPerThread];
 #pragma unroll
       for (int j = 0; j < kEntPerThread; ++j) {
         const int xr = tid + j * kThreads;
-        if (B.x + xr < B.y) ein[j] = load_entry<kLSE>(P, B.x + xr, S.qpos[xo + xr], kLSE ? 0 : S.f[xo + xr]);
-      }
-      int32_t hpin[kHeadsPerThread], hslot[kHeadsPerThread], hwin[kHeadsPerThread];
-      float2 hsd[kHeadsPerThread];
-#pragma unroll
-      for (int j = 0; j < kHeadsPerThread; ++j) {
-        const int h = A.x + tid + j * kThreads;
-        if (h < A.y) {
-          hpin[j] = S.pin[lo + tid + j * kThreads];
-          hslot[j] = __ldg(P.hd_hslot + h);
-          hsd[j] = __ldcg(P.hseed + h);
-          hwin[j] = kLSE ? 0 : __ldcg(P.win + hpin[j]);
+        if (B.x + xr < B.y) {
+          ein[j] = load_entry<kLSE>(P, B.x + xr, S.qpos[xo + xr], kLSE ? 0 : S.f[xo + xr]);
+          const int h = S.eh[xo + xr];
+          ehr[j] = h - A.x;
+          eslot[j] = __ldg(P.hd_hslot + h);
+          esd[j] = __ldcg(P.hseed + h);
+          ewin[j] = kLSE ? 0 : __ldcg(P.win + S.pin[lo + ehr[j]]);
         }
       }
       const int nfo = A.w - A.z;
@@ -1237,37 +1250,39 @@ __global__ void __launch_bounds__(kThreads, 1) bwdf_kernel(KParams P) {
       }
       __syncthreads();
       trace_stamp(P, c, nsteps, t, 1);
-      // (2) heads: adjoint = seed + (pull + heavy accumulator)
-#pragma unroll
-      for (int j = 0; j < kHeadsPerThread; ++j) {
-        const int p = tid + j * kThreads;
-        if (p < np) {
+      if (B.z == 0) {   // startpoints: dL/d(source mean)
+        for (int p = tid; p < np; p += kThreads) {
           const int r0 = S.lptr[lo + p] - A.z, r1 = S.lptr[lo + p + 1] - A.z;
           float sx = 0.f, sy = 0.f;
           for (int r = r0; r < r1; ++r) {
             sx += gg[r].x;
             sy += gg[r].y;
           }
-          const float2 h = heavy_take(P, hslot[j]);
-          const float2 ab = make_float2(hsd[j].x + (sx + h.x), hsd[j].y + (sy + h.y));
-          if (B.z == 0) {
-            if (P.d_src) reinterpret_cast<float2*>(P.d_src)[__ldg(P.order + hpin[j])] = ab;
-          } else {
-            const int x0 = S.hptr[lo + p], x1 = S.hptr[lo + p + 1];
-            for (int x = x0; x < x1; ++x) {
-              eab[x - B.x] = ab;
-              if (!kLSE) esel[x - B.x] = win_sel(hwin[j], x - x0);
-            }
-          }
+          const float2 h = heavy_read(P, __ldg(P.hd_hslot + A.x + p));
+          const float2 sd = __ldcg(P.hseed + A.x + p);
+          if (P.d_src)
+            reinterpret_cast<float2*>(P.d_src)[__ldg(P.order + S.pin[lo + p])] =
+                make_float2(sd.x + (sx + h.x), sd.y + (sy + h.y));
         }
-      }
-      __syncthreads();
-      // (3) entries: sink side of e (and of the folded pin behind it)
-      if (B.z > 0) {
+      } else {
+        // (2) entries: the head's adjoint (seed + (pull + heavy), the same
+        // expression as the per-level schedule; computed by each entry of the
+        // head) and the sink side of e (and of the folded pin behind it)
 #pragma unroll
         for (int j = 0; j < kEntPerThread; ++j) {
           const int xr = tid + j * kThreads;
-          if (B.x + xr < B.y) bwdf_entry<kLSE>(P, htab, ein[j], eab[xr], kLSE ? 0 : esel[xr]);
+          if (B.x + xr < B.y) {
+            const int p = ehr[j];
+            const int r0 = S.lptr[lo + p] - A.z, r1 = S.lptr[lo + p + 1] - A.z;
+            float sx = 0.f, sy = 0.f;
+            for (int r = r0; r < r1; ++r) {
+              sx += gg[r].x;
+              sy += gg[r].y;
+            }
+            const float2 h = heavy_read(P, eslot[j]);
+            const float2 ab = make_float2(esd[j].x + (sx + h.x), esd[j].y + (sy + h.y));
+            bwdf_entry<kLSE>(P, htab, ein[j], ab, kLSE ? 0 : win_sel(ewin[j], B.x + xr - S.hptr[lo + p]));
+          }
         }
       }
     } else if (np > 0) {
@@ -1283,7 +1298,7 @@ __global__ void __launch_bounds__(kThreads, 1) bwdf_kernel(KParams P) {
           sx += v.x;
           sy += v.y;
         }
-        const float2 hv = heavy_take(P, __ldg(P.hd_hslot + h));
+        const float2 hv = heavy_read(P, __ldg(P.hd_hslot + h));
         const float2 sd = __ldcg(P.hseed + h);
         s_ab = make_float2(sd.x + (sx + hv.x), sd.y + (sy + hv.y));
         s_win = kLSE ? 0 : __ldcg(P.win + q);
@@ -1587,6 +1602,7 @@ static KParams make_params(DevGraph& g, bool bwd) {
   P.ext_bw = g.ext_bw;
   P.ext_arc = g.ext_arc;
   P.ext_farc = g.ext_farc;
+  P.ext_h = g.ext_h;
   P.hseed = g.hseed;
   P.dirty_h = g.dirty_h;
   P.counters = g.counters;
@@ -1799,6 +1815,9 @@ int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float*
   P.mode = g.bwd_schedule == 0 ? 2 : 0;
   P.par = (++g.pass_bwd) & 1u;
   if (g.bwd_schedule == 0) {   // stage-folded persistent pass (fold.cpp)
+    // heavy accumulators start from zero (bwdf reads them without resetting)
+    e = cudaMemsetAsync(g.heavy_acc, 0, sizeof(unsigned long long) * 2 * size_t(std::max(g.num_heavy, 1)), st);
+    if (e != cudaSuccess) return int(e);
     P.item_a = g.bwdf_a;
     P.item_b = g.bwdf_b;
     P.lfo_ptr = g.hlfo_ptr;
