@@ -329,7 +329,13 @@ __device__ __forceinline__ void merge1(const Gath& st, int u, const float4& ms, 
     m.mu[rf] = cb.mu;
     m.var[rf] = cb.var;
     win[rf] = bs << 15;
-    if (kLSE) {
+    if (kLSE && u != 2) {
+      // one candidate: w0 = exp(0) = 1 and the normalizer is 0 + 1 = 1 exactly,
+      // ln(1) = 0, 1 / 1 = 1: the Eq 4 arrival is A_c itself and the Eq 6
+      // weight is 1 (the same values the general sequence below produces)
+      m.mu[rf] = (cb.A + 0.0) - ns * double(cb.sig);
+      wt[rf][s0] = 1.f;
+    } else if (kLSE) {
       float sum = 0.f;
       const float w0 = lse_w(c0.A, cb.A, inv_tau);
       sum += w0;
