@@ -170,3 +170,37 @@ def validate(g, n_sigma=3.0, tau=0.0) -> int:
     L = lib()
     L.orc_validate.argtypes = [ctypes.c_void_p, ctypes.c_double, ctypes.c_double]
     return int(L.orc_validate(ctypes.byref(og.c), float(n_sigma), float(tau)))
+
+
+def topk_forward(g, n_sigma=3.0, K=4):
+    """NEXT 1, Alg 1 + Alg 2: Top-K unique-startpoint queues.
+    Returns dict(A, mu, sigma [N,2,K] float64, sp [N,2,K] int32 caller ids, -1 = empty)."""
+    og = _og(g)
+    N = og.N
+    A = np.zeros((N, 2, K)); mu = np.zeros((N, 2, K)); sig = np.zeros((N, 2, K))
+    sp = np.zeros((N, 2, K), np.int32)
+    L = lib()
+    L.orc_topk_forward.argtypes = [ctypes.c_void_p, ctypes.c_double, ctypes.c_int32] + [ctypes.c_void_p] * 4
+    _check(L.orc_topk_forward(ctypes.byref(og.c), float(n_sigma), int(K), _p(A), _p(mu), _p(sig), _p(sp)))
+    return dict(A=A, mu=mu, sigma=sig, sp=sp)
+
+
+def topk_slack(g, q, rat_table=None):
+    """CPPR slack over Top-K queues q (from topk_forward).  rat_table = (ptr [P+1], sp [M], rat [M,2]) or None.
+    Returns dict(slack, rf_star, k_star, sp_star [P], wns, tns, num_viol)."""
+    og = _og(g)
+    K = int(q["A"].shape[2])
+    A = np.ascontiguousarray(q["A"], np.float64)
+    sp = np.ascontiguousarray(q["sp"], np.int32)
+    rp = rs = rv = None
+    if rat_table is not None:
+        rp = np.ascontiguousarray(rat_table[0], np.int32)
+        rs = np.ascontiguousarray(rat_table[1], np.int32)
+        rv = np.ascontiguousarray(np.asarray(rat_table[2], np.float64).reshape(-1, 2))
+    s = np.zeros(og.P); r = np.zeros(og.P, np.uint8); ks = np.zeros(og.P, np.int32); ss = np.zeros(og.P, np.int32)
+    wns = ctypes.c_double(); tns = ctypes.c_double(); nv = ctypes.c_int32()
+    L = lib()
+    L.orc_topk_slack.argtypes = [ctypes.c_void_p, ctypes.c_int32] + [ctypes.c_void_p] * 12
+    _check(L.orc_topk_slack(ctypes.byref(og.c), K, _p(A), _p(sp), _p(rp), _p(rs), _p(rv), _p(s), _p(r), _p(ks),
+                            _p(ss), ctypes.byref(wns), ctypes.byref(tns), ctypes.byref(nv)))
+    return dict(slack=s, rf_star=r, k_star=ks, sp_star=ss, wns=wns.value, tns=tns.value, num_viol=nv.value)

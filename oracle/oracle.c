@@ -493,3 +493,145 @@ int orc_tie_taint(const orc_graph* g, double n_sigma, double eps, double margin,
   topo_free(&t);
   return 0;
 }
+
+/* ------------------------------------------------------------------------- */
+/* NEXT 1: Top-K statistical arrival propagation with unique   */
+/* startpoints (Alg 1 + Alg 2) and CPPR-aware slack         */
+/* (endpoint required times "associated with respective startpoints").*/
+/*                                                                           */
+/* Per pin and sink transition rf a queue of K entries {A, mu, sig, SP},      */
+/* descending in A; an empty entry has A = -inf and SP = -1 (reading R13).    */
+/* Startpoints: entry 0 = the clock arrival distribution with SP = the pin    */
+/* itself (caller id).  Other pins, Alg 1 l.7: for k = 0..K-1 (outer), for    */
+/* each fanin arc in row order (inner), for s in S(rf, u) (reading R3), the   */
+/* parent's entry k of transition s -- if it exists -- gives a candidate      */
+/* (Eq 1-3, l.9-16) that is offered to the queue by Alg 2 (l.17).             */
+/* ------------------------------------------------------------------------- */
+typedef struct { double A, mu, sig; int32_t sp; } tk_ent;
+
+/* Alg 2: in-place update of one queue (q[0..K-1], descending in A). */
+static void alg2_update(tk_ent* q, int K, tk_ent nw) {
+  /* Step 1 (l.2-8): is SP_new already in the queue? */
+  for (int j = 0; j < K; ++j) {
+    if (q[j].sp == nw.sp) {
+      if (nw.A > q[j].A) {                       /* l.4: replace only if strictly greater */
+        q[j] = nw;                               /* l.5-6 */
+        /* reading R13: the in-place update can break descending order;
+         * re-bubble the entry up past strictly smaller entries */
+        while (j > 0 && q[j].A > q[j - 1].A) { tk_ent x = q[j]; q[j] = q[j - 1]; q[j - 1] = x; --j; }
+      }
+      return;                                    /* l.8: exit once SP_new is found */
+    }
+  }
+  /* Step 2 (l.9-): SP_new not found -- insert before the first smaller entry,
+   * shifting the rest down; the last entry falls off ("checks whether
+   * A_new exceeds the smallest arrival time ... inserted in the appropriate
+   * position to maintain descending order") */
+  for (int j = 0; j < K; ++j) {
+    if (nw.A > q[j].A) {
+      for (int m = K - 1; m > j; --m) q[m] = q[m - 1];
+      q[j] = nw;
+      return;
+    }
+  }
+}
+
+int orc_topk_forward(const orc_graph* g, double n_sigma, int32_t K, double* A, double* mu,
+                     double* sig, int32_t* sp) {
+  int st = orc_validate(g, n_sigma, 0.0);
+  if (st) return st;
+  if (K < 1) return 1;
+  topo_t t;
+  st = topo_build(g->num_pins, g->num_arcs, g->arc_from, g->arc_to, &t);
+  if (st) return st;
+  int32_t N = g->num_pins;
+  tk_ent* Q = malloc(sizeof(tk_ent) * ((size_t)N * 2 * K + 1));  /* [N][2][K], caller-indexed */
+  const tk_ent empty = {-INFINITY, 0.0, 0.0, -1};
+  for (int32_t k = 0; k < N; ++k) {
+    int32_t i = t.order[k];
+    for (int rf = 0; rf < 2; ++rf) {
+      tk_ent* q = Q + ((size_t)i * 2 + rf) * K;
+      for (int m = 0; m < K; ++m) q[m] = empty;
+      if (t.fanin_ptr[k] == t.fanin_ptr[k + 1]) {
+        /* startpoint: clock arrival, corner via Eq 3; SP = this pin */
+        q[0].mu = g->src_mean ? g->src_mean[2 * (int64_t)i + rf] : 0.0;
+        q[0].sig = g->src_sigma ? g->src_sigma[2 * (int64_t)i + rf] : 0.0;
+        q[0].A = q[0].mu + n_sigma * q[0].sig;
+        q[0].sp = i;
+        continue;
+      }
+      for (int kk = 0; kk < K; ++kk) {                              /* Alg 1 l.7: k outer */
+        for (int32_t r = t.fanin_ptr[k]; r < t.fanin_ptr[k + 1]; ++r) { /* parents, row order */
+          int32_t e = t.fanin_arc[r];
+          int32_t j = g->arc_from[e];
+          int ss[2];
+          int ns = sources_of(rf, g->arc_unate[e], ss);             /* Alg 1 l.8, reading R3 */
+          for (int a = 0; a < ns; ++a) {
+            const tk_ent* p = Q + ((size_t)j * 2 + ss[a]) * K + kk;
+            if (p->sp < 0) continue;                                /* no k-th arrival at the parent */
+            double arc_mean = g->arc_mean[2 * (int64_t)e + rf];
+            double arc_std = g->arc_sigma[2 * (int64_t)e + rf];
+            tk_ent c;
+            c.mu = p->mu + arc_mean;                                /* l.12, Eq 1 */
+            c.sig = sqrt(p->sig * p->sig + arc_std * arc_std);      /* l.13, Eq 2 */
+            c.A = c.mu + n_sigma * c.sig;                           /* l.14, Eq 3 */
+            c.sp = p->sp;                                           /* l.16 */
+            alg2_update(q, K, c);                                   /* l.17 */
+          }
+        }
+      }
+    }
+  }
+  for (size_t x = 0; x < (size_t)N * 2 * K; ++x) {
+    if (A) A[x] = Q[x].A;
+    if (mu) mu[x] = Q[x].mu;
+    if (sig) sig[x] = Q[x].sig;
+    if (sp) sp[x] = Q[x].sp;
+  }
+  free(Q);
+  topo_free(&t);
+  return 0;
+}
+
+/* CPPR slack: endpoint required times are associated with
+ * startpoints.  rat_ptr[P+1] / rat_sp[] / rat_val[][2]: per endpoint, a list of
+ * (startpoint caller id, RAT{R,F}); a startpoint not in its endpoint's list
+ * takes the endpoint's default ep_rat.  slack = min over rf (R first) and over
+ * the K queue entries (in queue order) of RAT(ep, SP_k)[rf] - A_k[rf]; the
+ * first minimum wins ties.  WNS / TNS / violations as in orc_slack.
+ * Outputs: slack[P], rf_star[P], k_star[P], sp_star[P] (caller id). */
+int orc_topk_slack(const orc_graph* g, int32_t K, const double* A, const int32_t* sp,
+                   const int32_t* rat_ptr, const int32_t* rat_sp, const double* rat_val,
+                   double* slack, uint8_t* rf_star, int32_t* k_star, int32_t* sp_star,
+                   double* wns, double* tns, int32_t* num_viol) {
+  double w = 0.0, tt = 0.0;
+  int32_t nv = 0;
+  for (int32_t e = 0; e < g->num_endpoints; ++e) {
+    int32_t p = g->ep_pin[e];
+    double best = INFINITY;
+    int br = 0, bk = 0;
+    int32_t bsp = -1;
+    for (int rf = 0; rf < 2; ++rf) {
+      for (int k = 0; k < K; ++k) {
+        size_t x = ((size_t)p * 2 + rf) * K + k;
+        if (sp[x] < 0) continue;
+        double rat = g->ep_rat[2 * e + rf];
+        if (rat_ptr)
+          for (int32_t m = rat_ptr[e]; m < rat_ptr[e + 1]; ++m)
+            if (rat_sp[m] == sp[x]) { rat = rat_val[2 * (int64_t)m + rf]; break; }
+        double s = rat - A[x];
+        if (s < best) { best = s; br = rf; bk = k; bsp = sp[x]; }
+      }
+    }
+    if (slack) slack[e] = best;
+    if (rf_star) rf_star[e] = (uint8_t)br;
+    if (k_star) k_star[e] = bk;
+    if (sp_star) sp_star[e] = bsp;
+    if (best < 0) { tt += best; ++nv; }
+    if (best < w) w = best;
+  }
+  if (wns) *wns = w;
+  if (tns) *tns = tt;
+  if (num_viol) *num_viol = nv;
+  return 0;
+}

@@ -75,6 +75,20 @@ int orc_backward(const orc_graph* g, double n_sigma, double tau,
 int orc_tie_taint(const orc_graph* g, double n_sigma, double eps, double margin,
                   uint8_t* fwd_taint, uint8_t* arc_taint);
 
+/* NEXT 1: Top-K unique-startpoint propagation (Alg 1 + Alg 2).
+ * Outputs [N][2][K] caller-indexed, each queue descending in A; empty entries
+ * have A = -inf and sp = -1.  sp = caller id of the startpoint pin. */
+int orc_topk_forward(const orc_graph* g, double n_sigma, int32_t K, double* A, double* mu,
+                     double* sig, int32_t* sp);
+
+/* CPPR slack over the Top-K queues: per endpoint e the list
+ * rat_ptr[e]..rat_ptr[e+1] of (rat_sp, rat_val{R,F}) overrides the default
+ * ep_rat for those startpoints.  rat_ptr may be NULL (no overrides). */
+int orc_topk_slack(const orc_graph* g, int32_t K, const double* A, const int32_t* sp,
+                   const int32_t* rat_ptr, const int32_t* rat_sp, const double* rat_val,
+                   double* slack, uint8_t* rf_star, int32_t* k_star, int32_t* sp_star,
+                   double* wns, double* tns, int32_t* num_viol);
+
 #ifdef __cplusplus
 }
 #endif

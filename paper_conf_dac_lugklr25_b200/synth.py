@@ -365,3 +365,40 @@ def ocv_scenario(s: int, seed: int = 505):
     """OCV scenario s (C5 scenarios 0..511): (n_sigma, derate_cell, derate_net)."""
     rng = np.random.default_rng([seed, s])
     return float(rng.uniform(2.5, 3.5)), float(rng.uniform(0.95, 1.10)), float(rng.uniform(0.95, 1.10))
+
+
+# ---------------------------------------------------------------------------
+# CPPR required-time table (SURVEY §8(f) NEXT 1; P:L62 "SP/EP attributes (e.g.
+# clock arrival times, minimum required times)", P:L119 endpoint required times
+# "associated with respective startpoints").  Structural input, no arithmetic
+# of the method: for each endpoint, `per_ep` random backward walks over fanin
+# arcs reach startpoints of its cone; each distinct one gets a clock-
+# reconvergence credit U(2, 25) ps added to the endpoint's default required
+# time (the common clock path removes pessimism, so RAT(ep, sp) >= RAT(ep)).
+# ---------------------------------------------------------------------------
+def cppr_rat_table(g, per_ep: int = 8, seed: int = 4242, dyadic: bool = False):
+    """Returns (ptr int32[P+1], sp int32[M] caller pin ids ascending per endpoint, rat float32[M,2])."""
+    rng = np.random.default_rng(seed)
+    N, P = int(g.num_pins), int(np.asarray(g.ep_pin).shape[0])
+    to = np.asarray(g.arc_to, np.int64)
+    order = np.argsort(to, kind="stable")
+    ptr = np.zeros(N + 1, np.int64)
+    np.add.at(ptr, to + 1, 1)
+    ptr = np.cumsum(ptr)
+    src_of = np.asarray(g.arc_from, np.int64)[order]
+    cur = np.repeat(np.asarray(g.ep_pin, np.int64), per_ep)
+    while True:
+        deg = ptr[cur + 1] - ptr[cur]
+        live = deg > 0
+        if not live.any():
+            break
+        pick = ptr[cur[live]] + (rng.random(int(live.sum())) * deg[live]).astype(np.int64)
+        cur[live] = src_of[pick]
+    pairs = np.unique(np.stack([np.repeat(np.arange(P), per_ep), cur], 1), axis=0)   # sorted (ep, sp)
+    cnt = np.bincount(pairs[:, 0], minlength=P)
+    rptr = np.concatenate([[0], np.cumsum(cnt)]).astype(np.int32)
+    credit = rng.uniform(2.0, 25.0, pairs.shape[0])
+    if dyadic:
+        credit = np.round(credit * 64) / 64
+    rat = np.asarray(g.ep_rat, np.float64).reshape(P, 2)[pairs[:, 0]] + credit[:, None]
+    return rptr, pairs[:, 1].astype(np.int32), rat.astype(np.float32)
