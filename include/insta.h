@@ -210,6 +210,53 @@ typedef struct {
 insta_status insta_forward_batch(insta_graph* g, int32_t num_scenarios, const insta_scenario* sc, float tau,
                                  double* summaries, float* d_arc_mean_sum, void* cuda_stream);
 
+/* ---- Top-K unique-startpoint propagation with CPPR ----
+ *
+ * The paper's CPPR handling: every pin keeps, per transition rf, a
+ * queue of the K largest statistical arrivals that come from DISTINCT
+ * startpoints (Alg 1 l.1-18; Alg 2), and endpoint slack is
+ * taken against required times "associated with respective startpoints"
+ * (P:L109, L119).  Queue semantics (readings R13, R17): candidates
+ * are offered in Alg 1's order (k outer, fanin arcs in caller-arc-id order,
+ * s = rf before ~rf for non-unate arcs); Alg 2 replaces a queued startpoint's
+ * entry only if strictly greater (then re-sorts) and inserts a new startpoint
+ * only if strictly greater than the smallest entry; an empty slot has SP = -1.
+ * K = 1 is the K = 1 hard merge of insta_forward (tau = 0). */
+
+/* Per-(endpoint, startpoint) required times.  rat_ptr: HOST [num_endpoints+1]
+ * row offsets (rat_ptr[0] = 0, non-decreasing); rat_sp: HOST [M] caller ids of
+ * startpoint pins (indegree 0), unique within a row; rat: HOST [M][2] {R, F}
+ * required times, M = rat_ptr[num_endpoints].  A startpoint missing from its
+ * endpoint's row takes the endpoint's default ep_rat.  rat_ptr = NULL clears
+ * the table.  Copied; synchronous.  E_ARG: malformed rows, a non-startpoint
+ * pin, a duplicate, non-finite values. */
+insta_status insta_set_cppr_rat(insta_graph* g, const int32_t* rat_ptr, const int32_t* rat_sp, const float* rat);
+
+/* Top-K forward (Alg 1 + Alg 2) over all levels with the graph's current arc
+ * delays; 1 <= K <= 32, n_sigma as in Eq 3.  Device state: K * 40 bytes per
+ * pin (fp64 mean and variance + int32 startpoint per slot and rf).  Enqueued on
+ * cuda_stream.  E_ARG: K or n_sigma out of range. */
+insta_status insta_topk_forward(insta_graph* g, int32_t K, float n_sigma, void* cuda_stream);
+
+/* CPPR endpoint slack over the Top-K queues: slack(ep) = min over rf (R
+ * first) and queue slots k (in order) of RAT(ep, SP_k)[rf] - A_k[rf]; the
+ * first minimum wins ties.  WNS / TNS / num_violations as in insta_slack
+ * (fixed-order fp64 sums).  slack: DEVICE float[num_endpoints] or NULL;
+ * sp_star: DEVICE int32[num_endpoints] caller id of the critical startpoint
+ * or NULL; out: summary (synchronizes) or NULL.  E_STATE without a valid
+ * insta_topk_forward (insta_update_arcs invalidates it). */
+insta_status insta_topk_slack(insta_graph* g, float* slack, int32_t* sp_star, void* cuda_stream, insta_summary* out);
+
+/* The (rf, slot) of each endpoint's critical entry from the last
+ * insta_topk_slack: rf_star DEVICE uint8[num_endpoints], k_star DEVICE
+ * int32[num_endpoints] (either may be NULL).  E_STATE before insta_topk_slack. */
+insta_status insta_topk_critical(insta_graph* g, uint8_t* rf_star, int32_t* k_star, void* cuda_stream);
+
+/* Export of the queues in caller pin order, DEVICE arrays [num_pins][2][K]
+ * (any may be NULL): A corner arrival (-inf for an empty slot), mean, sigma,
+ * sp = caller id of the startpoint (-1 for an empty slot). */
+insta_status insta_topk_queues(insta_graph* g, float* A, float* mean, float* sigma, int32_t* sp, void* cuda_stream);
+
 /* Statistics of the last forward: number of pins recomputed (== num_pins for a
  * full forward).  For an incremental one: the work-item heads recomputed in
  * the changed cone (insta_graph_schedule; each head's folded input pins are

@@ -186,6 +186,51 @@ class Graph:
         check(self.lib.insta_update_arcs(self._h, int(ids.numel()), _dptr(ids), _dptr(m), _dptr(s),
                                          int(bool(incremental)), self._st(stream)), "insta_update_arcs")
 
+    # ------------------------------------------------------------------ Top-K / CPPR
+    def set_cppr_rat(self, rat_ptr=None, rat_sp=None, rat=None):
+        """insta_set_cppr_rat: per-(endpoint, startpoint) required times (host arrays; None clears)."""
+        if rat_ptr is None:
+            check(self.lib.insta_set_cppr_rat(self._h, None, None, None), "insta_set_cppr_rat")
+            return
+        rp = _np(rat_ptr, np.int32)
+        rs = _np(rat_sp, np.int32)
+        rv = _np(rat, np.float32, (-1, 2))
+        check(self.lib.insta_set_cppr_rat(self._h, _ptr(rp), _ptr(rs), _ptr(rv)), "insta_set_cppr_rat")
+
+    def topk_forward(self, K: int, n_sigma: float = 3.0, stream=None):
+        """insta_topk_forward: Top-K unique-startpoint queues (Alg 1 + Alg 2)."""
+        self.topk_K = int(K)
+        check(self.lib.insta_topk_forward(self._h, int(K), float(n_sigma), self._st(stream)), "insta_topk_forward")
+
+    def topk_slack(self, stream=None, sync: bool = True):
+        """insta_topk_slack: CPPR slack.  Returns (Summary or None, slack float32[P], sp_star int32[P])."""
+        t = self._torch
+        s = t.empty(self.num_endpoints, dtype=t.float32, device=self.device)
+        sp = t.empty(self.num_endpoints, dtype=t.int32, device=self.device)
+        out = _capi.insta_summary() if sync else None
+        check(self.lib.insta_topk_slack(self._h, _dptr(s), _dptr(sp), self._st(stream),
+                                        ctypes.byref(out) if out is not None else None), "insta_topk_slack")
+        summ = None if out is None else Summary(out.wns, out.tns, out.num_violations, out.num_levels)
+        return summ, s, sp
+
+    def topk_critical(self, stream=None):
+        """insta_topk_critical: (rf_star uint8[P], k_star int32[P]) of the last topk_slack."""
+        t = self._torch
+        r = t.empty(self.num_endpoints, dtype=t.uint8, device=self.device)
+        k = t.empty(self.num_endpoints, dtype=t.int32, device=self.device)
+        check(self.lib.insta_topk_critical(self._h, _dptr(r), _dptr(k), self._st(stream)), "insta_topk_critical")
+        return r, k
+
+    def topk_queues(self, stream=None):
+        """insta_topk_queues: dict(A, mean, sigma float32[N,2,K], sp int32[N,2,K]) in caller pin order."""
+        t = self._torch
+        K = self.topk_K
+        A, m, s = (t.empty((self.num_pins, 2, K), dtype=t.float32, device=self.device) for _ in range(3))
+        sp = t.empty((self.num_pins, 2, K), dtype=t.int32, device=self.device)
+        check(self.lib.insta_topk_queues(self._h, _dptr(A), _dptr(m), _dptr(s), _dptr(sp), self._st(stream)),
+              "insta_topk_queues")
+        return dict(A=A, mean=m, sigma=s, sp=sp)
+
     def forward_batch(self, scenarios, tau: float = 0.0, want_grad: bool = False, summaries=None, d_mean_sum=None,
                       stream=None):
         """insta_forward_batch: evaluate independent scenarios (dicts with n_sigma, derate_cell, derate_net and

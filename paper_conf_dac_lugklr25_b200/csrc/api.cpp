@@ -55,16 +55,20 @@ void free_graph(insta::DevGraph& d) {
                   d.state,     d.win,       d.wts,       d.g,          d.seed,      d.slack,
                   d.rf_star,   d.partials,  d.ticket,    d.summary,    d.counters,
                   d.fin_flags, d.ep_of_pin, d.b_state,   d.b_win,      d.b_wts,     d.b_g,
-                  d.b_heavy,   d.b_sc,      d.b_ov_ptr,  d.b_ov_pos,   d.b_ov_ms,   d.b_slack,
+                  d.b_heavy,   d.b_stage,   d.b_slack,
                   d.b_rf,      d.b_partials, d.b_ticket,
                   d.hd_pin,    d.hd_ptr,    d.hd_q0,     d.ext_w,      d.ext_ms,    d.ext_f,
                   d.ext_fms,   d.ext_fq,    d.arc_xpos,  d.fwdf_a,     d.fwdf_b,    d.hd_hslot,
                   d.hlfo_ptr,  d.hlfo,      d.ext_qpos,  d.ext_bw,     d.ext_arc,   d.ext_farc,
                   d.ep_head,   d.hseed,     d.bwdf_a,    d.bwdf_b,    d.g4,        d.hacc4,
-                  d.ext_flags, d.bfwdf_a,   d.bfwdf_b,   d.b_ov_key,  d.hd_eop,    d.dirty_h,
-                  d.arc_head,  d.ext_h};
+                  d.ext_flags, d.bfwdf_a,   d.bfwdf_b,   d.hd_eop,    d.dirty_h,
+                  d.arc_head,  d.ext_h,     d.tk_q,      d.tk_sp,      d.tk_slack,  d.tk_star,
+                  d.tk_summary, d.rat_ptr,  d.rat_sp,    d.rat_val};
   for (void* p : ptrs)
     if (p) cudaFree(p);
+  if (d.b_stage_h) cudaFreeHost(d.b_stage_h);
+  if (d.b_stage_copied) cudaEventDestroy(static_cast<cudaEvent_t>(d.b_stage_copied));
+  if (d.b_stage_done) cudaEventDestroy(static_cast<cudaEvent_t>(d.b_stage_done));
 }
 
 bool finite2(const float* a, int64_t n, bool nonneg) {
@@ -467,6 +471,7 @@ insta_status insta_update_arcs(insta_graph* g, int64_t n, const int32_t* arc_ids
   int err = insta::launch_update_arcs(d, n, arc_ids, mean, sigma, incremental, cuda_stream);
   if (err) return cuda_fail(err, "update_arcs");
   d.fwd_valid = false;
+  d.tk_valid = false;
   if (incremental && !d.pending_full) d.pending_incremental = true;
   else d.pending_full = true;
   return INSTA_OK;
@@ -500,31 +505,167 @@ insta_status insta_forward_batch(insta_graph* g, int32_t num_scenarios, const in
     cudaError_t e = cudaMemsetAsync(d_arc_mean_sum, 0, sizeof(float) * 2 * size_t(d.e), st);
     if (e != cudaSuccess) return cuda_fail(int(e), "forward_batch");
   }
+  // Pack every micro-batch of 32 scenarios: [3][32] parameters, [33] override ranges, then the
+  // override fanin positions, entry keys and records of all micro-batches (one H2D copy).
   constexpr int kL = 32;
-  for (int32_t b0 = 0; b0 < num_scenarios; b0 += kL) {
-    const int nb = std::min(kL, num_scenarios - b0);
-    float par[3 * kL];
-    std::vector<int32_t> ov_ptr(kL + 1, 0), ov_pos, ov_key;
-    std::vector<float4> ov_ms;
+  const int nm = (num_scenarios + kL - 1) / kL;
+  int64_t nov_all = 0;
+  for (int32_t s = 0; s < num_scenarios; ++s) nov_all += sc[s].n_delta;
+  const size_t head = size_t(nm) * (3 * kL + kL + 1) * 4;
+  const size_t o_pos = (head + 15) & ~size_t(15);
+  const size_t o_key = o_pos + ((size_t(nov_all) * 4 + 15) & ~size_t(15));
+  const size_t o_ms = o_key + ((size_t(nov_all) * 4 + 15) & ~size_t(15));
+  const size_t bytes = o_ms + size_t(nov_all) * 16;
+  std::vector<char> buf(bytes);
+  int64_t nov = 0;
+  std::vector<int> nov_of(nm), first_of(nm);
+  for (int m = 0; m < nm; ++m) {
+    float* par = reinterpret_cast<float*>(buf.data() + size_t(m) * (4 * kL + 1) * 4);
+    int32_t* ovp = reinterpret_cast<int32_t*>(par + 3 * kL);
+    first_of[m] = int(nov);
+    ovp[0] = 0;
     for (int s = 0; s < kL; ++s) {
-      const insta_scenario* x = s < nb ? &sc[b0 + s] : nullptr;
+      const int b = m * kL + s;
+      const insta_scenario* x = b < num_scenarios ? &sc[b] : nullptr;
       par[s] = x ? x->n_sigma : 0.f;
       par[kL + s] = x ? x->derate_cell : 1.f;
       par[2 * kL + s] = x ? x->derate_net : 1.f;
-      if (x) {
-        for (int32_t k = 0; k < x->n_delta; ++k) {
-          ov_pos.push_back(d.h_arc_pos[x->delta_arc[k]]);
-          ov_key.push_back(d.h_arc_xpos[x->delta_arc[k]]);
-          ov_ms.push_back(make_float4(x->delta_mean[2 * k], x->delta_mean[2 * k + 1], x->delta_sigma[2 * k],
-                                      x->delta_sigma[2 * k + 1]));
-        }
+      for (int32_t k = 0; x && k < x->n_delta; ++k, ++nov) {
+        reinterpret_cast<int32_t*>(buf.data() + o_pos)[nov] = d.h_arc_pos[x->delta_arc[k]];
+        reinterpret_cast<int32_t*>(buf.data() + o_key)[nov] = d.h_arc_xpos[x->delta_arc[k]];
+        reinterpret_cast<float4*>(buf.data() + o_ms)[nov] =
+            make_float4(x->delta_mean[2 * k], x->delta_mean[2 * k + 1], x->delta_sigma[2 * k], x->delta_sigma[2 * k + 1]);
       }
-      ov_ptr[s + 1] = int32_t(ov_pos.size());
+      ovp[s + 1] = int32_t(nov - first_of[m]);
     }
-    int err = insta::launch_forward_batch(d, nb, par, ov_ptr, ov_pos, ov_key, ov_ms, tau, summaries + 3 * size_t(b0),
-                                          d_arc_mean_sum, cuda_stream);
+    nov_of[m] = int(nov - first_of[m]);
+  }
+  int err = insta::batch_stage(d, buf.data(), bytes, cuda_stream);
+  if (err) return cuda_fail(err, "forward_batch");
+  for (int m = 0; m < nm; ++m) {
+    const char* dev = d.b_stage;
+    insta::BatchSlice b;
+    b.nb = std::min(kL, num_scenarios - m * kL);
+    b.nov = nov_of[m];
+    b.sc = reinterpret_cast<const float*>(dev + size_t(m) * (4 * kL + 1) * 4);
+    b.ov_ptr = reinterpret_cast<const int32_t*>(b.sc + 3 * kL);
+    b.ov_pos = reinterpret_cast<const int32_t*>(dev + o_pos) + first_of[m];
+    b.ov_key = reinterpret_cast<const int32_t*>(dev + o_key) + first_of[m];
+    b.ov_ms = reinterpret_cast<const float4*>(dev + o_ms) + first_of[m];
+    err = insta::launch_forward_batch(d, b, tau, summaries + 3 * size_t(m) * kL, d_arc_mean_sum, cuda_stream);
     if (err) return cuda_fail(err, "forward_batch");
   }
+  err = insta::batch_stage_release(d, cuda_stream);
+  if (err) return cuda_fail(err, "forward_batch");
+  return INSTA_OK;
+}
+
+// ---------------------------------------------------------------------------
+// Top-K unique-startpoint propagation and CPPR slack
+// ---------------------------------------------------------------------------
+insta_status insta_set_cppr_rat(insta_graph* g, const int32_t* rat_ptr, const int32_t* rat_sp, const float* rat) {
+  if (!g) return fail(INSTA_E_ARG, "set_cppr_rat: NULL graph");
+  insta::DevGraph& d = g->d;
+  cudaSetDevice(d.device);
+  if (d.rat_ptr) cudaFree(d.rat_ptr);
+  if (d.rat_sp) cudaFree(d.rat_sp);
+  if (d.rat_val) cudaFree(d.rat_val);
+  d.rat_ptr = nullptr;
+  d.rat_sp = nullptr;
+  d.rat_val = nullptr;
+  d.tk_slack_done = false;
+  if (!rat_ptr) return INSTA_OK;   // table cleared: every startpoint takes the default RAT
+  const int32_t P = d.num_ep;
+  if (rat_ptr[0] != 0) return fail(INSTA_E_ARG, "set_cppr_rat: rat_ptr[0] must be 0");
+  for (int32_t e = 0; e < P; ++e)
+    if (rat_ptr[e + 1] < rat_ptr[e]) return fail(INSTA_E_ARG, "set_cppr_rat: rat_ptr must be non-decreasing");
+  const int32_t M = rat_ptr[P];
+  if (M > 0 && (!rat_sp || !rat)) return fail(INSTA_E_ARG, "set_cppr_rat: NULL table");
+  std::vector<std::pair<int32_t, int32_t>> row;
+  std::vector<int32_t> sp(size_t(std::max(M, 1)));
+  std::vector<float2> val(size_t(std::max(M, 1)));
+  for (int32_t e = 0; e < P; ++e) {
+    row.clear();
+    for (int32_t m = rat_ptr[e]; m < rat_ptr[e + 1]; ++m) {
+      const int32_t p = rat_sp[m];
+      if (p < 0 || p >= d.n) return fail(INSTA_E_ARG, "set_cppr_rat: startpoint id out of range");
+      const int32_t c = d.host.pos[p];
+      if (c >= d.num_src) return fail(INSTA_E_ARG, "set_cppr_rat: pin is not a startpoint (has fanin)");
+      if (!std::isfinite(rat[2 * size_t(m)]) || !std::isfinite(rat[2 * size_t(m) + 1]))
+        return fail(INSTA_E_ARG, "set_cppr_rat: non-finite required time");
+      row.emplace_back(c, m);
+    }
+    std::sort(row.begin(), row.end());
+    for (size_t k = 0; k < row.size(); ++k) {
+      if (k && row[k].first == row[k - 1].first) return fail(INSTA_E_ARG, "set_cppr_rat: duplicate startpoint in a row");
+      sp[rat_ptr[e] + k] = row[k].first;
+      val[rat_ptr[e] + k] = make_float2(rat[2 * size_t(row[k].second)], rat[2 * size_t(row[k].second) + 1]);
+    }
+  }
+  cudaError_t e = cudaMalloc(&d.rat_ptr, sizeof(int32_t) * (size_t(P) + 1));
+  if (e == cudaSuccess) e = cudaMalloc(&d.rat_sp, sizeof(int32_t) * sp.size());
+  if (e == cudaSuccess) e = cudaMalloc(&d.rat_val, sizeof(float2) * val.size());
+  if (e == cudaSuccess) e = cudaMemcpy(d.rat_ptr, rat_ptr, sizeof(int32_t) * (size_t(P) + 1), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(d.rat_sp, sp.data(), sizeof(int32_t) * sp.size(), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(d.rat_val, val.data(), sizeof(float2) * val.size(), cudaMemcpyHostToDevice);
+  if (e != cudaSuccess) return cuda_fail(int(e), "set_cppr_rat");
+  return INSTA_OK;
+}
+
+insta_status insta_topk_forward(insta_graph* g, int32_t K, float n_sigma, void* cuda_stream) {
+  if (!g) return fail(INSTA_E_ARG, "topk_forward: NULL graph");
+  if (K < 1 || K > 32) return fail(INSTA_E_ARG, "topk_forward: K must be in [1, 32]");
+  if (!std::isfinite(n_sigma) || n_sigma < 0.f) return fail(INSTA_E_ARG, "topk_forward: n_sigma must be >= 0");
+  insta::DevGraph& d = g->d;
+  cudaSetDevice(d.device);
+  int err = insta::launch_topk_forward(d, K, n_sigma, cuda_stream);
+  if (err) return cuda_fail(err, "topk_forward");
+  d.tk_ns = n_sigma;
+  d.tk_valid = true;
+  d.tk_slack_done = false;
+  return INSTA_OK;
+}
+
+insta_status insta_topk_slack(insta_graph* g, float* slack, int32_t* sp_star, void* cuda_stream, insta_summary* out) {
+  if (!g) return fail(INSTA_E_ARG, "topk_slack: NULL graph");
+  insta::DevGraph& d = g->d;
+  if (!d.tk_valid) return fail(INSTA_E_STATE, "topk_slack: no valid Top-K forward (call insta_topk_forward)");
+  cudaSetDevice(d.device);
+  int err = insta::launch_topk_slack(d, d.tk_ns, cuda_stream);
+  if (!err && (slack || sp_star)) err = insta::launch_topk_export_slack(d, slack, sp_star, nullptr, nullptr, cuda_stream);
+  if (err) return cuda_fail(err, "topk_slack");
+  d.tk_slack_done = true;
+  if (out) {
+    double s[3];
+    cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    cudaError_t e = cudaMemcpyAsync(s, d.tk_summary, sizeof s, cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) return cuda_fail(int(e), "topk_slack");
+    out->wns = s[0];
+    out->tns = s[1];
+    out->num_violations = int32_t(s[2]);
+    out->num_levels = d.num_levels;
+  }
+  return INSTA_OK;
+}
+
+insta_status insta_topk_critical(insta_graph* g, uint8_t* rf_star, int32_t* k_star, void* cuda_stream) {
+  if (!g) return fail(INSTA_E_ARG, "topk_critical: NULL graph");
+  insta::DevGraph& d = g->d;
+  if (!d.tk_valid || !d.tk_slack_done) return fail(INSTA_E_STATE, "topk_critical: call insta_topk_slack first");
+  cudaSetDevice(d.device);
+  int err = insta::launch_topk_export_slack(d, nullptr, nullptr, rf_star, k_star, cuda_stream);
+  if (err) return cuda_fail(err, "topk_critical");
+  return INSTA_OK;
+}
+
+insta_status insta_topk_queues(insta_graph* g, float* A, float* mean, float* sigma, int32_t* sp, void* cuda_stream) {
+  if (!g) return fail(INSTA_E_ARG, "topk_queues: NULL graph");
+  insta::DevGraph& d = g->d;
+  if (!d.tk_valid) return fail(INSTA_E_STATE, "topk_queues: no valid Top-K forward (call insta_topk_forward)");
+  cudaSetDevice(d.device);
+  int err = insta::launch_topk_export(d, A, mean, sigma, sp, cuda_stream);
+  if (err) return cuda_fail(err, "topk_queues");
   return INSTA_OK;
 }
 

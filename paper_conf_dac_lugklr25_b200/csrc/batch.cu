@@ -22,6 +22,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstring>
 #include <cstdint>
 #include <vector>
 
@@ -691,16 +692,20 @@ static int ensure_batch(DevGraph& g, bool lse, bool grad) {
     if (err) return err;
     attrs = true;
   }
-  auto alloc = [](void** p, size_t bytes) -> int {
+  // cudaMemset runs on the legacy default stream, which the caller's (torch,
+  // non-blocking) stream does not wait for: synchronize once after any
+  // allocation so the first pass never sees the buffers before they are zeroed
+  // (the parity dataflow would otherwise wait on words the memset overwrites).
+  bool fresh = false;
+  auto alloc = [&fresh](void** p, size_t bytes) -> int {
     if (*p) return 0;
     cudaError_t e = cudaMalloc(p, bytes + 64);
     if (e != cudaSuccess) return int(e);
+    fresh = true;
     return int(cudaMemset(*p, 0, bytes + 64));
   };
   const size_t n = size_t(std::max(g.n, 1)), e = size_t(std::max<int64_t>(g.e, 1));
   int err = alloc(reinterpret_cast<void**>(&g.b_state), n * kLanes * sizeof(PinState));
-  if (!err) err = alloc(reinterpret_cast<void**>(&g.b_sc), 3 * kLanes * sizeof(float));
-  if (!err) err = alloc(reinterpret_cast<void**>(&g.b_ov_ptr), (kLanes + 1) * sizeof(int32_t));
   if (!err) err = alloc(reinterpret_cast<void**>(&g.b_slack), size_t(std::max(g.num_ep, 1)) * kLanes * sizeof(float));
   if (!err) err = alloc(reinterpret_cast<void**>(&g.b_rf), size_t(std::max(g.num_ep, 1)) * kLanes);
   if (!err) err = alloc(reinterpret_cast<void**>(&g.b_partials),
@@ -711,6 +716,7 @@ static int ensure_batch(DevGraph& g, bool lse, bool grad) {
   if (!err && grad) err = alloc(reinterpret_cast<void**>(&g.b_g), e * kLanes * sizeof(float2));
   if (!err && grad) err = alloc(reinterpret_cast<void**>(&g.b_heavy),
                                 size_t(std::max(g.num_heavy, 1)) * kLanes * 2 * sizeof(unsigned long long));
+  if (!err && fresh) err = int(cudaDeviceSynchronize());
   return err;
 }
 
@@ -740,10 +746,6 @@ static BParams make_bparams(DevGraph& g, bool bwd) {
   P.heavy_fo = g.heavy_fo;
   P.ep_of_pin = bwd ? g.hd_eop : g.ep_of_pin;
   P.src_ms = g.src_ms;
-  P.sc = g.b_sc;
-  P.ov_ptr = g.b_ov_ptr;
-  P.ov_pos = bwd ? g.b_ov_pos : g.b_ov_key;
-  P.ov_ms = g.b_ov_ms;
   P.bstate = g.b_state;
   P.bwin = g.b_win;
   P.bwts = g.b_wts;
@@ -754,42 +756,59 @@ static BParams make_bparams(DevGraph& g, bool bwd) {
   return P;
 }
 
-int launch_forward_batch(DevGraph& g, int nb, const float* sc_host /*[3][32]*/, const std::vector<int32_t>& ov_ptr,
-                         const std::vector<int32_t>& ov_pos, const std::vector<int32_t>& ov_key,
-                         const std::vector<float4>& ov_ms, float tau, double* summaries, float* d_mean_sum,
+int batch_stage(DevGraph& g, const void* host, size_t bytes, void* stream) {
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  cudaError_t e = cudaSuccess;
+  if (!g.b_stage_copied) e = cudaEventCreateWithFlags(reinterpret_cast<cudaEvent_t*>(&g.b_stage_copied), cudaEventDisableTiming);
+  if (e == cudaSuccess && !g.b_stage_done)
+    e = cudaEventCreateWithFlags(reinterpret_cast<cudaEvent_t*>(&g.b_stage_done), cudaEventDisableTiming);
+  if (e != cudaSuccess) return int(e);
+  // the previous call's kernels may still read the device copy (possibly on another stream), and
+  // its H2D copy may still read the pinned buffer
+  e = cudaStreamWaitEvent(st, static_cast<cudaEvent_t>(g.b_stage_done), 0);
+  if (e == cudaSuccess) e = cudaEventSynchronize(static_cast<cudaEvent_t>(g.b_stage_copied));
+  if (e == cudaSuccess && bytes > g.b_stage_cap) {
+    e = cudaStreamSynchronize(st);
+    if (e == cudaSuccess && g.b_stage) e = cudaFree(g.b_stage);
+    if (e == cudaSuccess && g.b_stage_h) e = cudaFreeHost(g.b_stage_h);
+    g.b_stage = nullptr;
+    g.b_stage_h = nullptr;
+    g.b_stage_cap = 0;
+    const size_t cap = std::max<size_t>(bytes + bytes / 2, 1 << 16);
+    if (e == cudaSuccess) e = cudaMalloc(&g.b_stage, cap);
+    if (e == cudaSuccess) e = cudaMallocHost(&g.b_stage_h, cap);
+    if (e == cudaSuccess) g.b_stage_cap = cap;
+  }
+  if (e != cudaSuccess) return int(e);
+  std::memcpy(g.b_stage_h, host, bytes);
+  e = cudaMemcpyAsync(g.b_stage, g.b_stage_h, bytes, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) e = cudaEventRecord(static_cast<cudaEvent_t>(g.b_stage_copied), st);
+  return int(e);
+}
+
+int batch_stage_release(DevGraph& g, void* stream) {
+  return int(cudaEventRecord(static_cast<cudaEvent_t>(g.b_stage_done), static_cast<cudaStream_t>(stream)));
+}
+
+int launch_forward_batch(DevGraph& g, const BatchSlice& bs, float tau, double* summaries, float* d_mean_sum,
                          void* stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   const bool lse = tau > 0.f, grad = d_mean_sum != nullptr;
+  const int nb = bs.nb, nov = bs.nov;
   int err = ensure_batch(g, lse, grad);
   if (err) return err;
-  cudaError_t e = cudaMemcpyAsync(g.b_sc, sc_host, 3 * kLanes * sizeof(float), cudaMemcpyHostToDevice, st);
-  if (e == cudaSuccess)
-    e = cudaMemcpyAsync(g.b_ov_ptr, ov_ptr.data(), (kLanes + 1) * sizeof(int32_t), cudaMemcpyHostToDevice, st);
-  const int nov = int(ov_pos.size());
-  if (e == cudaSuccess && nov > g.b_ov_cap) {
-    cudaFree(g.b_ov_pos);
-    cudaFree(g.b_ov_key);
-    cudaFree(g.b_ov_ms);
-    g.b_ov_pos = nullptr;
-    g.b_ov_key = nullptr;
-    g.b_ov_ms = nullptr;
-    e = cudaMalloc(&g.b_ov_pos, sizeof(int32_t) * nov + 64);
-    if (e == cudaSuccess) e = cudaMalloc(&g.b_ov_key, sizeof(int32_t) * nov + 64);
-    if (e == cudaSuccess) e = cudaMalloc(&g.b_ov_ms, sizeof(float4) * nov + 64);
-    g.b_ov_cap = nov;
-  }
-  if (e == cudaSuccess && nov > 0) {
-    e = cudaMemcpyAsync(g.b_ov_pos, ov_pos.data(), sizeof(int32_t) * nov, cudaMemcpyHostToDevice, st);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(g.b_ov_key, ov_key.data(), sizeof(int32_t) * nov, cudaMemcpyHostToDevice, st);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(g.b_ov_ms, ov_ms.data(), sizeof(float4) * nov, cudaMemcpyHostToDevice, st);
-    if (e == cudaSuccess) {
-      set_flag_kernel<<<(nov + 255) / 256, 256, 0, st>>>(nov, g.b_ov_pos, g.fin_flags, 2, 1);
-      set_xflag_kernel<<<(nov + 255) / 256, 256, 0, st>>>(nov, g.b_ov_key, g.ext_flags, 1);
-      e = cudaGetLastError();
-    }
+  cudaError_t e = cudaSuccess;
+  if (nov > 0) {
+    set_flag_kernel<<<(nov + 255) / 256, 256, 0, st>>>(nov, bs.ov_pos, g.fin_flags, 2, 1);
+    set_xflag_kernel<<<(nov + 255) / 256, 256, 0, st>>>(nov, bs.ov_key, g.ext_flags, 1);
+    e = cudaGetLastError();
   }
   if (e != cudaSuccess) return int(e);
   BParams P = make_bparams(g, false);
+  P.sc = bs.sc;
+  P.ov_ptr = bs.ov_ptr;
+  P.ov_pos = bs.ov_key;
+  P.ov_ms = bs.ov_ms;
   P.nb = nb;
   P.tau = tau;
   P.inv_tau = lse ? 1.0 / double(tau) : 0.0;
@@ -805,7 +824,7 @@ int launch_forward_batch(DevGraph& g, int nb, const float* sc_host /*[3][32]*/, 
   }
   if (g.num_ep > 0) {
     const int blocks = (g.num_ep + kSlackEps * 64 - 1) / (kSlackEps * 64);
-    slackb_kernel<<<blocks, 256, 0, st>>>(g.num_ep, nb, g.ep_pin, g.ep_rat, g.b_state, g.b_sc, g.b_slack, g.b_rf,
+    slackb_kernel<<<blocks, 256, 0, st>>>(g.num_ep, nb, g.ep_pin, g.ep_rat, g.b_state, bs.sc, g.b_slack, g.b_rf,
                                           g.b_partials, g.b_ticket, summaries);
     e = cudaGetLastError();
   } else {
@@ -814,6 +833,10 @@ int launch_forward_batch(DevGraph& g, int nb, const float* sc_host /*[3][32]*/, 
   if (e != cudaSuccess) return int(e);
   if (grad && g.n > 0) {
     BParams Q = make_bparams(g, true);
+    Q.sc = bs.sc;
+    Q.ov_ptr = bs.ov_ptr;
+    Q.ov_pos = bs.ov_pos;
+    Q.ov_ms = bs.ov_ms;
     Q.nb = nb;
     Q.tau = tau;
     Q.inv_tau = P.inv_tau;
@@ -827,8 +850,8 @@ int launch_forward_batch(DevGraph& g, int nb, const float* sc_host /*[3][32]*/, 
     if (e != cudaSuccess) return int(e);
   }
   if (nov > 0) {
-    set_flag_kernel<<<(nov + 255) / 256, 256, 0, st>>>(nov, g.b_ov_pos, g.fin_flags, 2, 0);
-    set_xflag_kernel<<<(nov + 255) / 256, 256, 0, st>>>(nov, g.b_ov_key, g.ext_flags, 0);
+    set_flag_kernel<<<(nov + 255) / 256, 256, 0, st>>>(nov, bs.ov_pos, g.fin_flags, 2, 0);
+    set_xflag_kernel<<<(nov + 255) / 256, 256, 0, st>>>(nov, bs.ov_key, g.ext_flags, 0);
     e = cudaGetLastError();
   }
   return int(e);

@@ -154,11 +154,13 @@ struct DevGraph {
   float4* b_wts = nullptr;
   float2* b_g = nullptr;
   unsigned long long* b_heavy = nullptr;
-  float* b_sc = nullptr;
-  int32_t* b_ov_ptr = nullptr;
-  int32_t* b_ov_pos = nullptr;
-  float4* b_ov_ms = nullptr;
-  int32_t b_ov_cap = 0;
+  // per-call scenario staging (insta_forward_batch): every micro-batch's parameters and override lists
+  // packed in one pinned host buffer, moved with one H2D copy (batch_stage)
+  char* b_stage = nullptr;         // device [b_stage_cap]
+  void* b_stage_h = nullptr;       // pinned host [b_stage_cap]
+  size_t b_stage_cap = 0;
+  void* b_stage_copied = nullptr;  // cudaEvent_t: the last H2D copy out of b_stage_h finished
+  void* b_stage_done = nullptr;    // cudaEvent_t: the last kernel reading b_stage finished
   float* b_slack = nullptr;
   uint8_t* b_rf = nullptr;
   double* b_partials = nullptr;
@@ -213,7 +215,20 @@ struct DevGraph {
   int4* bfwdf_a = nullptr;
   int4* bfwdf_b = nullptr;
   ItemTable bfwdf_items;
-  int32_t* b_ov_key = nullptr;     // [b_ov_cap] override keys in entry space (2x / 2x+1)
+  // Top-K unique-startpoint propagation (topk.cu)
+  int32_t tk_K = 0;                // queue length the buffers are sized for
+  float tk_ns = 3.f;               // N_sigma of the last insta_topk_forward
+  bool tk_valid = false;           // queues match the current arcs
+  bool tk_slack_done = false;      // tk_slack / tk_star hold the slack of the current queues
+  double2* tk_q = nullptr;         // [n][2][K] {mu, var} per queue slot (canonical pins)
+  int32_t* tk_sp = nullptr;        // [n][2][K] canonical startpoint, -1 = empty slot
+  double* tk_slack = nullptr;      // [P] CPPR slack (fp64)
+  int32_t* tk_star = nullptr;      // [2][P] critical startpoint | rf << 30, slot k
+  double* tk_summary = nullptr;    // {wns, tns, violations}
+  // CPPR required times per (endpoint, startpoint) (insta_set_cppr_rat)
+  int32_t* rat_ptr = nullptr;      // [P+1] or NULL (no table)
+  int32_t* rat_sp = nullptr;       // [M] canonical startpoints, ascending within a row
+  float2* rat_val = nullptr;       // [M] RAT {R, F}
   // state
   PinState* state = nullptr;       // [n]
   int32_t* win = nullptr;          // [n] hard-mode winners {R: k | s<<15, F: << 16}
@@ -266,9 +281,26 @@ int launch_update_arcs(DevGraph& g, int64_t n, const int32_t* ids, const float* 
                        const float* sigma, int incremental, void* stream);
 int launch_arrivals(DevGraph& g, float* A, float* mean, float* sigma, void* stream);
 int launch_copy_slack(DevGraph& g, float* slack, uint8_t* rf, void* stream);
-// batch.cu: up to 32 scenarios in one pass; sc = [3][32] {n_sigma, derate_cell, derate_net}
-int launch_forward_batch(DevGraph& g, int nb, const float* sc_host, const std::vector<int32_t>& ov_ptr,
-                         const std::vector<int32_t>& ov_pos, const std::vector<int32_t>& ov_key,
-                         const std::vector<float4>& ov_ms, float tau, double* summaries, float* d_mean_sum,
+// batch.cu: one micro-batch of up to 32 scenarios in one pass.  All pointers are device pointers into
+// the staging buffer: sc = [3][32] {n_sigma, derate_cell, derate_net}, ov_ptr = [33] per-scenario
+// override ranges, ov_pos / ov_key / ov_ms = [nov] override fanin positions, entry keys, records.
+struct BatchSlice {
+  int nb, nov;
+  const float* sc;
+  const int32_t* ov_ptr;
+  const int32_t* ov_pos;
+  const int32_t* ov_key;
+  const float4* ov_ms;
+};
+int launch_forward_batch(DevGraph& g, const BatchSlice& b, float tau, double* summaries, float* d_mean_sum,
                          void* stream);
+int launch_topk_forward(DevGraph& g, int K, float n_sigma, void* stream);
+int launch_topk_slack(DevGraph& g, float n_sigma, void* stream);
+int launch_topk_export(DevGraph& g, float* A, float* mean, float* sigma, int32_t* sp, void* stream);
+int launch_topk_export_slack(DevGraph& g, float* slack, int32_t* sp_star, uint8_t* rf_star, int32_t* k_star,
+                             void* stream);
+// copy `bytes` of packed host data to g.b_stage (pinned bounce buffer, one async H2D copy)
+int batch_stage(DevGraph& g, const void* host, size_t bytes, void* stream);
+// record that every kernel reading g.b_stage has been enqueued on `stream`
+int batch_stage_release(DevGraph& g, void* stream);
 }  // namespace insta

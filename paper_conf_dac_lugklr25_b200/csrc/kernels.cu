@@ -1780,6 +1780,7 @@ int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float*
       e = cudaMalloc(&g.g4, sizeof(float4) * std::max<size_t>(size_t(g.e), 1));
       if (e == cudaSuccess) e = cudaMalloc(&g.hacc4, sizeof(long long) * 4 * size_t(std::max(g.num_heavy, 1)));
       if (e == cudaSuccess) e = cudaMemset(g.hacc4, 0, sizeof(long long) * 4 * size_t(std::max(g.num_heavy, 1)));
+      if (e == cudaSuccess) e = cudaDeviceSynchronize();   // legacy-stream memset vs the caller's stream
       if (e != cudaSuccess) return int(e);
     }
     KParams P = make_params(g, true);
