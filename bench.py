@@ -157,6 +157,16 @@ def bwd_bytes_folded(sc, N, E, E_light, P, nnz_arcs, lse):
             + 8 * nnz_arcs)                   # nonzero d_mean scatter
 
 
+def topk_bytes(g, K):
+    """insta_topk_forward: per non-source pin a row pointer; per arc its source word and
+    record (20 B); per (arc, sink rf, source transition) the parent's K queue slots ({mu, var} 16 B +
+    startpoint 4 B); every (pin, rf) writes its K slots."""
+    N, E = int(g.num_pins), int(g.num_arcs)
+    n_src = int(np.count_nonzero(np.bincount(g.arc_to, minlength=N) == 0))
+    n_non = int(np.count_nonzero(g.arc_unate == 2))
+    return 4 * (N - n_src) + 20 * E + (2 * E + 2 * n_non) * K * 20 + 2 * N * K * 20
+
+
 def cpu_oracle_sample(cfg_name, sample_pins, tau):
     """fp64 CPU oracle (single thread) fwd + slack + bwd on a bounded sample of the workload:
     the same generator recipe (depth, fanout law, endpoint fraction) at `sample_pins` pins."""
@@ -210,6 +220,7 @@ def main():
     ap.add_argument("--ref-sample-pins", type=int, default=1_500_000)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--batch-scenarios", type=int, default=1024, help="C5 batched evaluations (0 = skip)")
+    ap.add_argument("--topk", type=int, default=32, help="Top-K CPPR propagation K (0 = skip)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -351,8 +362,8 @@ def main():
 
         dd = torch.distributed if world > 1 else None
         with torch.cuda.stream(stream):
-            ev(scs[:32], True)                      # warm-up (allocates the batch buffers)
-            ev(scs[n_ocv:n_ocv + 32], False)
+            # warm-up: one untimed pass of the same calls (allocates the batch and staging buffers)
+            idist.evaluate_sharded(ev, scs, n_ocv, E, rank, world, dev, dd)
             stream.synchronize()
             if world > 1:
                 torch.distributed.barrier()
@@ -374,6 +385,36 @@ def main():
                    "collectives": "all_gather(per-scenario summaries) + all_reduce(SUM, gradient sum)" if world > 1
                    else "none (1 rank)",
                    "tns_min": float(sa[:, 1].min()), "tns_max": float(sa[:, 1].max())}
+
+    # ---------------- Top-K unique-startpoint propagation + CPPR slack -------------
+    topk = None
+    if args.topk > 0:
+        G.set_cppr_rat(*synth.cppr_rat_table(g))
+        K = args.topk
+        with torch.cuda.stream(stream):
+            for _ in range(2):
+                G.topk_forward(K, 3.0, stream=stream)
+                G.topk_slack(stream=stream, sync=False)
+            stream.synchronize()
+            nk = max(1, min(args.steps, 5))
+            t0, t1, t2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+            t0.record(stream)
+            for _ in range(nk):
+                G.topk_forward(K, 3.0, stream=stream)
+            t1.record(stream)
+            for _ in range(nk):
+                G.topk_slack(stream=stream, sync=False)
+            t2.record(stream)
+            stream.synchronize()
+            ts, _, _ = G.topk_slack(stream=stream)
+        tf, tsl = t0.elapsed_time(t1) / nk, t1.elapsed_time(t2) / nk
+        tk_bytes = topk_bytes(g, K)
+        topk = {"workload": f"{cfg.name}, Top-K = {K} unique-startpoint queues (Alg 1 + Alg 2) + CPPR slack against "
+                            f"a per-(endpoint, startpoint) RAT table", "K": K, "fwd_ms": tf, "slack_ms": tsl,
+                "pins_per_s": N / ((tf + tsl) * 1e-3), "alg_bytes": tk_bytes, "gbs": tk_bytes / (tf * 1e-3) / 1e9,
+                "tns": ts.tns, "wns": ts.wns, "violations": ts.num_violations,
+                "paper_context": "PAPER.md Table I (L184-193): block-1 (15M pins) at TopK=32 in 0.39 s on 1x A100 "
+                                 "(incl. its own slack); other hardware, other design"}
 
     cpu = None
     if rank == 0 and not args.no_cpu_baseline:
@@ -404,7 +445,7 @@ def main():
                          "frac": ach / peak, "peak_kind": peak_kind, "traffic": traffic,
                          "fwd_gbs": fwd_gbs, "bwd_gbs": bwd_gbs, "fwd_alg_bytes": fb, "bwd_alg_bytes": bb},
             "cpu_baseline": cpu, "e2e": e2e, "clocks": clk, "gpu_launches": launches_per_step * args.steps,
-            "batched": batched,
+            "batched": batched, "topk": topk,
             "paper_context": "PAPER.md L9/L37: full-graph propagation < 0.1 s on a 15M-pin 3nm design, 1x A100 "
                              "(forward only, Top-K not stated); not the same metric",
         }

@@ -63,7 +63,7 @@ void free_graph(insta::DevGraph& d) {
                   d.ep_head,   d.hseed,     d.bwdf_a,    d.bwdf_b,    d.g4,        d.hacc4,
                   d.ext_flags, d.bfwdf_a,   d.bfwdf_b,   d.hd_eop,    d.dirty_h,
                   d.arc_head,  d.ext_h,     d.tk_q,      d.tk_sp,      d.tk_slack,  d.tk_star,
-                  d.tk_summary, d.rat_ptr,  d.rat_sp,    d.rat_val};
+                  d.tk_summary, d.rat_ptr,  d.rat_sp,    d.rat_val,   d.tk_list};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   if (d.b_stage_h) cudaFreeHost(d.b_stage_h);
@@ -668,6 +668,9 @@ insta_status insta_topk_queues(insta_graph* g, float* A, float* mean, float* sig
   if (err) return cuda_fail(err, "topk_queues");
   return INSTA_OK;
 }
+
+// debug builds (-DTK_STATS): merge batches of the Top-K kernel by survivor count (33 counters)
+int insta_debug_topk_stats(unsigned long long* out) { return insta::topk_stats(out); }
 
 insta_status insta_last_forward_stats(insta_graph* g, int64_t* pins_recomputed) {
   if (!g) return fail(INSTA_E_ARG, "stats: NULL graph");

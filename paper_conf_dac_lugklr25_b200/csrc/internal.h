@@ -222,6 +222,8 @@ struct DevGraph {
   bool tk_slack_done = false;      // tk_slack / tk_star hold the slack of the current queues
   double2* tk_q = nullptr;         // [n][2][K] {mu, var} per queue slot (canonical pins)
   int32_t* tk_sp = nullptr;        // [n][2][K] canonical startpoint, -1 = empty slot
+  int32_t* tk_list = nullptr;      // [n - num_src] per level: single-arc pins, then merging pins
+  std::vector<int32_t> tk_one_ptr, tk_multi_ptr;   // [L+1] offsets of the two parts per level
   double* tk_slack = nullptr;      // [P] CPPR slack (fp64)
   int32_t* tk_star = nullptr;      // [2][P] critical startpoint | rf << 30, slot k
   double* tk_summary = nullptr;    // {wns, tns, violations}
@@ -296,6 +298,7 @@ int launch_forward_batch(DevGraph& g, const BatchSlice& b, float tau, double* su
                          void* stream);
 int launch_topk_forward(DevGraph& g, int K, float n_sigma, void* stream);
 int launch_topk_slack(DevGraph& g, float n_sigma, void* stream);
+int topk_stats(unsigned long long* out);
 int launch_topk_export(DevGraph& g, float* A, float* mean, float* sigma, int32_t* sp, void* stream);
 int launch_topk_export_slack(DevGraph& g, float* slack, int32_t* sp_star, uint8_t* rf_star, int32_t* k_star,
                              void* stream);

@@ -35,10 +35,20 @@
 #include "device_common.cuh"
 #include "internal.h"
 
+// resident blocks per SM the level kernel is compiled for (register budget)
+#ifndef TK_MINB
+#define TK_MINB 4
+#endif
+
 namespace insta {
+
+#ifdef TK_STATS
+__device__ unsigned long long tk_stats[33];   // merge batches by survivor count (debug builds)
+#endif
 
 struct TkParams {
   int32_t lo, hi, K;
+  const int32_t* __restrict__ list;   // canonical pins of this launch: list[lo..hi)
   double ns;
   const int32_t* __restrict__ fanin_ptr;
   const int32_t* __restrict__ fin_src;
@@ -68,108 +78,288 @@ __global__ void tk_src_kernel(int n_src, int K, const float4* __restrict__ src_m
   }
 }
 
+// A queue slot or a candidate: corner arrival A, key position t, distribution, startpoint.
+struct TkEnt {
+  double A, mu, var;
+  int t, sp;
+};
+
+__device__ __forceinline__ TkEnt tk_empty() { return TkEnt{-INFINITY, 0.0, 0.0, INT_MAX, -1}; }
+
+__device__ __forceinline__ TkEnt shfl_ent(unsigned gm, const TkEnt& e, int src) {
+  TkEnt o;
+  o.A = __shfl_sync(gm, e.A, src);
+  o.mu = __shfl_sync(gm, e.mu, src);
+  o.var = __shfl_sync(gm, e.var, src);
+  o.t = __shfl_sync(gm, e.t, src);
+  o.sp = __shfl_sync(gm, e.sp, src);
+  return o;
+}
+
 template <int G>
-__global__ void __launch_bounds__(256) tk_level_kernel(TkParams P) {
+struct Log2 {
+  static constexpr int v = G <= 1 ? 0 : 1 + Log2<(G > 1 ? G / 2 : 1)>::v;
+};
+template <>
+struct Log2<1> {
+  static constexpr int v = 0;
+};
+
+// Bitonic sort of (A, t) keys over the G lanes of a group, descending; idx
+// follows its key (the lane that held it before the sort).
+template <int G>
+__device__ __forceinline__ void bitonic_desc(unsigned gm, int gl, double& sA, int& st, int& idx) {
+#pragma unroll
+  for (int k = 2; k <= G; k <<= 1) {
+#pragma unroll
+    for (int jj = k >> 1; jj > 0; jj >>= 1) {
+      const double oA = __shfl_xor_sync(gm, sA, jj, G);
+      const int ot = __shfl_xor_sync(gm, st, jj, G), oi = __shfl_xor_sync(gm, idx, jj, G);
+      const bool want_max = ((gl & jj) == 0) == ((gl & k) == 0);
+      if (want_max ? key_gt(oA, ot, sA, st) : key_gt(sA, st, oA, ot)) {
+        sA = oA;
+        st = ot;
+        idx = oi;
+      }
+    }
+  }
+}
+
+// parent slot loads of one batch (fanin arc held by lane `src`, source
+// transition index si); the {mu, var} load does not wait for the startpoint
+// word (empty slots hold zeros)
+__device__ __forceinline__ void tk_issue(const TkParams& P, unsigned gm, int src, int32_t wl, int rf, int si, int K,
+                                         int gl, bool slot, int& csp, double2& pv) {
+  const int32_t w = __shfl_sync(gm, wl, src);
+  const size_t ps = (size_t(w & kSrcMask) * 2 + src_tr(rf, int(uint32_t(w) >> kUnateShift), si)) * K + gl;
+  csp = slot ? __ldg(P.qsp + ps) : -1;
+  pv = slot ? __ldg(P.q + ps) : make_double2(0.0, 0.0);
+}
+
+template <int G>
+__global__ void __launch_bounds__(256, TK_MINB) tk_level_kernel(TkParams P) {
+  // per-group scatter area of the bulk merge (one slot per thread of the block)
+  __shared__ double smA[256], smMu[256], smVar[256];
+  __shared__ int smT[256], smSp[256];
   const int lane = threadIdx.x & 31;
-  const int gl = lane & (G - 1), gbase = lane & ~(G - 1);
+  const int gl = lane & (G - 1), gbase = lane & ~(G - 1), tbase = threadIdx.x & ~(G - 1);
   const unsigned gm = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << gbase);
   const long long grp = (blockIdx.x * (long long)blockDim.x + threadIdx.x) / G;
   if (grp >= 2LL * (P.hi - P.lo)) return;   // uniform within a group
-  const int i = P.lo + int(grp >> 1), rf = int(grp & 1), K = P.K;
+  const int i = __ldg(P.list + P.lo + int(grp >> 1)), rf = int(grp & 1), K = P.K;
   const bool slot = gl < K;
   const int last = gbase + K - 1;
-  double qA = -INFINITY, qmu = 0.0, qvar = 0.0;
-  int qsp = -1, qt = INT_MAX;
+  TkEnt q = tk_empty();
+  bool first = true;
   const int b0 = __ldg(P.fanin_ptr + i), b1 = __ldg(P.fanin_ptr + i + 1), nf = b1 - b0;
-  for (int a = b0; a < b1; ++a) {
-    const int32_t w = __ldg(P.fin_src + a);
-    const int j = w & kSrcMask, u = int(uint32_t(w) >> kUnateShift);
-    const float4 ms = __ldg(P.fin_ms + a);
-    const double am = double(rf ? ms.y : ms.x), se = double(rf ? ms.w : ms.z);
-    for (int si = 0; si < n_src_tr(u); ++si) {
-      const size_t ps = (size_t(j) * 2 + src_tr(rf, u, si)) * K + gl;
-      const int csp = slot ? __ldg(P.qsp + ps) : -1;
-      double cA = -INFINITY, cmu = 0.0, cvar = 0.0;
-      const int ct = (gl * nf + (a - b0)) * 2 + si;   // Alg 1 order: k outer, arcs, s
-      if (csp >= 0) {
-        const double2 pv = __ldg(P.q + ps);
-        cmu = pv.x + am;                               // Eq 1 (l.12)
-        cvar = pv.y + se * se;                         // Eq 2 (l.13)
-        cA = cmu + P.ns * double(sigma_of(cvar));      // Eq 3 (l.14)
-      }
-      if (a == b0 && si == 0) {
-        // first batch into an empty queue: one parent's queue has unique
-        // startpoints, so Alg 2 reduces to ordering the candidates by key --
-        // a bitonic sort over the group (skipped when already in order)
-        const double nA = __shfl_down_sync(gm, cA, 1, G);
-        const int nt = __shfl_down_sync(gm, ct, 1, G);
-        const bool bad = gl + 1 < G && key_gt(nA, nt, cA, ct);
-        int idx = gl;
-        if (__ballot_sync(gm, bad) & gm) {
-          double sA = cA;
-          int st = csp >= 0 ? ct : INT_MAX;
-#pragma unroll
-          for (int k = 2; k <= G; k <<= 1) {
-#pragma unroll
-            for (int jj = k >> 1; jj > 0; jj >>= 1) {
-              const double oA = __shfl_xor_sync(gm, sA, jj, G);
-              const int ot = __shfl_xor_sync(gm, st, jj, G), oi = __shfl_xor_sync(gm, idx, jj, G);
-              const bool want_max = ((gl & jj) == 0) == ((gl & k) == 0);
-              if (want_max ? key_gt(oA, ot, sA, st) : key_gt(sA, st, oA, ot)) {
-                sA = oA;
-                st = ot;
-                idx = oi;
-              }
+  for (int c0 = b0; c0 < b1; c0 += G) {
+    // the row's topology, one fanin arc per lane (rows longer than G in chunks)
+    const int cn = min(G, b1 - c0);
+    int32_t wl = 0;
+    float4 msl = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (gl < cn) {
+      wl = __ldg(P.fin_src + c0 + gl);
+      msl = __ldg(P.fin_ms + c0 + gl);
+    }
+    // parent slot loads run one batch ahead of the merge; the {mu, var} load
+    // does not wait for the startpoint word (empty slots hold zeros)
+    int csp_n;
+    double2 pv_n;
+    tk_issue(P, gm, gbase + 0, wl, rf, 0, K, gl, slot, csp_n, pv_n);
+    for (int x = 0; x < cn; ++x) {
+      const int32_t w = __shfl_sync(gm, wl, gbase + x);
+      const int u = int(uint32_t(w) >> kUnateShift);
+      const float am_f = __shfl_sync(gm, rf ? msl.y : msl.x, gbase + x);
+      const float se_f = __shfl_sync(gm, rf ? msl.w : msl.z, gbase + x);
+      const double am = double(am_f), se = double(se_f);
+      for (int si = 0; si < n_src_tr(u); ++si) {
+        const int csp = csp_n;
+        const double2 pv = pv_n;
+        {
+          int nx = x, nsi = si + 1;
+          if (nsi >= n_src_tr(u)) {
+            nx = x + 1;
+            nsi = 0;
+          }
+          if (nx < cn) tk_issue(P, gm, gbase + nx, wl, rf, nsi, K, gl, slot, csp_n, pv_n);
+        }
+        TkEnt c;
+        c.sp = csp;
+        c.t = (gl * nf + (c0 + x - b0)) * 2 + si;   // Alg 1 order: k outer, arcs, s
+        c.mu = pv.x + am;                            // Eq 1 (l.12)
+        c.var = pv.y + se * se;                      // Eq 2 (l.13)
+        c.A = csp >= 0 ? c.mu + P.ns * double(sigma_of(c.var)) : -INFINITY;   // Eq 3 (l.14)
+        if (first) {
+          // first batch into an empty queue: one parent's queue has unique
+          // startpoints, so Alg 2 reduces to ordering the candidates by key
+          first = false;
+          const double nA = __shfl_down_sync(gm, c.A, 1, G);
+          const int nt = __shfl_down_sync(gm, c.t, 1, G);
+          int idx = gl;
+          if (__ballot_sync(gm, gl + 1 < G && key_gt(nA, nt, c.A, c.t)) & gm) {
+            double sA = c.A;
+            int st = csp >= 0 ? c.t : INT_MAX;
+            bitonic_desc<G>(gm, gl, sA, st, idx);
+          }
+          q = shfl_ent(gm, c, gbase + idx);
+          if (q.sp < 0) q = tk_empty();
+          continue;
+        }
+        // one ballot prunes every candidate below the queue's last slot: it can
+        // neither enter nor beat its startpoint's entry
+        const double mA = __shfl_sync(gm, q.A, last);
+        const int mt = __shfl_sync(gm, q.t, last);
+        const bool surv = csp >= 0 && key_gt(c.A, c.t, mA, mt);
+        unsigned m = __ballot_sync(gm, surv) & gm;
+#ifdef TK_STATS
+        if (gl == 0) atomicAdd(&tk_stats[min(__popc(m), 32)], 1ull);
+#endif
+        if (__popc(m) <= 2) {
+          while (m) {   // Alg 2, one survivor at a time
+            const int src = __ffs(m) - 1;
+            m &= m - 1;
+            const TkEnt n = shfl_ent(gm, c, src);
+            const unsigned fm = __ballot_sync(gm, slot && q.sp == n.sp) & gm;
+            int f;
+            if (fm) {                                      // Step 1: the startpoint is queued
+              f = __ffs(fm) - 1;
+              if (!key_gt(n.A, n.t, __shfl_sync(gm, q.A, f), __shfl_sync(gm, q.t, f))) continue;
+              f -= gbase;
+            } else {                                       // Step 2: a new startpoint
+              if (!key_gt(n.A, n.t, __shfl_sync(gm, q.A, last), __shfl_sync(gm, q.t, last))) continue;
+              f = K - 1;                                   // the last entry falls off
             }
+            const int p = __popc(__ballot_sync(gm, slot && key_gt(q.A, q.t, n.A, n.t)) & gm);
+            TkEnt up;
+            up.A = __shfl_up_sync(gm, q.A, 1, G);
+            up.mu = __shfl_up_sync(gm, q.mu, 1, G);
+            up.var = __shfl_up_sync(gm, q.var, 1, G);
+            up.t = __shfl_up_sync(gm, q.t, 1, G);
+            up.sp = __shfl_up_sync(gm, q.sp, 1, G);
+            if (gl > p && gl <= f) q = up;
+            else if (gl == p) q = n;
+          }
+          continue;
+        }
+        // bulk merge of many survivors: (1) match each survivor's startpoint
+        // in the queue; a matched one replaces its entry only if its key is
+        // larger, else it is dropped; (2) sort the kept candidates; (3) rank
+        // every alive queue entry and kept candidate in the union by binary
+        // search in the other sorted list; (4) scatter the top K through
+        // shared memory.
+        int f = -1;
+        for (int r = 0; r < K; ++r)
+          if (__shfl_sync(gm, q.sp, gbase + r) == csp) f = r;
+        const double fA = __shfl_sync(gm, q.A, gbase + max(f, 0));
+        const int ft = __shfl_sync(gm, q.t, gbase + max(f, 0));
+        bool keep = surv;
+        unsigned deadbit = 0u;
+        if (surv && f >= 0) {
+          if (key_gt(c.A, c.t, fA, ft)) deadbit = 1u << f;
+          else keep = false;
+        }
+        const unsigned dead = __reduce_or_sync(gm, deadbit);
+        double sA = keep ? c.A : -INFINITY;
+        int st = keep ? c.t : INT_MAX, idx = gl;
+        bitonic_desc<G>(gm, gl, sA, st, idx);
+        const int nC = __popc(__ballot_sync(gm, keep) & gm);
+        const unsigned qv = (__ballot_sync(gm, slot && q.sp >= 0) & gm) >> gbase;
+        const int nQ = __popc(qv);
+        int lo = 0, hi = nC;   // kept candidates ahead of my queue entry
+#pragma unroll
+        for (int it = 0; it <= Log2<G>::v; ++it) {
+          const int mid = (lo + hi) >> 1;
+          const double xA = __shfl_sync(gm, sA, gbase + min(mid, G - 1));
+          const int xt = __shfl_sync(gm, st, gbase + min(mid, G - 1));
+          if (lo < hi) {
+            if (key_gt(xA, xt, q.A, q.t)) lo = mid + 1;
+            else hi = mid;
           }
         }
-        qA = __shfl_sync(gm, cA, gbase + idx);
-        qmu = __shfl_sync(gm, cmu, gbase + idx);
-        qvar = __shfl_sync(gm, cvar, gbase + idx);
-        qsp = __shfl_sync(gm, csp, gbase + idx);
-        qt = __shfl_sync(gm, ct, gbase + idx);
-        if (qsp < 0) {
-          qA = -INFINITY;
-          qt = INT_MAX;
+        const int rankQ = __popc(qv & ~dead & ((1u << gl) - 1u)) + lo;
+        int lo2 = 0, hi2 = nQ;   // queue entries ahead of my sorted candidate
+#pragma unroll
+        for (int it = 0; it <= Log2<G>::v; ++it) {
+          const int mid = (lo2 + hi2) >> 1;
+          const double xA = __shfl_sync(gm, q.A, gbase + min(mid, G - 1));
+          const int xt = __shfl_sync(gm, q.t, gbase + min(mid, G - 1));
+          if (lo2 < hi2) {
+            if (key_gt(xA, xt, sA, st)) lo2 = mid + 1;
+            else hi2 = mid;
+          }
         }
-        continue;
-      }
-      // one ballot prunes everything below the queue's last slot
-      const double mA = __shfl_sync(gm, qA, last);
-      const int mt = __shfl_sync(gm, qt, last);
-      unsigned m = __ballot_sync(gm, csp >= 0 && key_gt(cA, ct, mA, mt)) & gm;
-      while (m) {                                      // Alg 2 for each survivor
-        const int src = __ffs(m) - 1;
-        m &= m - 1;
-        const double nA = __shfl_sync(gm, cA, src), nmu = __shfl_sync(gm, cmu, src),
-                     nvar = __shfl_sync(gm, cvar, src);
-        const int nt = __shfl_sync(gm, ct, src), nsp = __shfl_sync(gm, csp, src);
-        const unsigned fm = __ballot_sync(gm, slot && qsp == nsp) & gm;
-        int f;
-        if (fm) {                                      // Step 1: the startpoint is queued
-          f = __ffs(fm) - 1;
-          if (!key_gt(nA, nt, __shfl_sync(gm, qA, f), __shfl_sync(gm, qt, f))) continue;
-          f -= gbase;
-        } else {                                       // Step 2: new startpoint
-          if (!key_gt(nA, nt, __shfl_sync(gm, qA, last), __shfl_sync(gm, qt, last))) continue;
-          f = K - 1;                                   // the last entry falls off
+        const int rankC = gl + lo2 - __popc(lo2 >= 32 ? dead : dead & ((1u << lo2) - 1u));
+        const TkEnt gc = shfl_ent(gm, c, gbase + idx);
+        __syncwarp(gm);
+        if (slot && q.sp >= 0 && !((dead >> gl) & 1u) && rankQ < K) {
+          smA[tbase + rankQ] = q.A;
+          smMu[tbase + rankQ] = q.mu;
+          smVar[tbase + rankQ] = q.var;
+          smT[tbase + rankQ] = q.t;
+          smSp[tbase + rankQ] = q.sp;
         }
-        const int p = __popc(__ballot_sync(gm, slot && key_gt(qA, qt, nA, nt)) & gm);
-        const double uA = __shfl_up_sync(gm, qA, 1, G), umu = __shfl_up_sync(gm, qmu, 1, G),
-                     uvar = __shfl_up_sync(gm, qvar, 1, G);
-        const int usp = __shfl_up_sync(gm, qsp, 1, G), ut = __shfl_up_sync(gm, qt, 1, G);
-        if (gl > p && gl <= f) {
-          qA = uA; qmu = umu; qvar = uvar; qsp = usp; qt = ut;
-        } else if (gl == p) {
-          qA = nA; qmu = nmu; qvar = nvar; qsp = nsp; qt = nt;
+        if (gl < nC && rankC < K) {
+          smA[tbase + rankC] = gc.A;
+          smMu[tbase + rankC] = gc.mu;
+          smVar[tbase + rankC] = gc.var;
+          smT[tbase + rankC] = gc.t;
+          smSp[tbase + rankC] = gc.sp;
         }
+        __syncwarp(gm);
+        if (gl < min(K, nQ - __popc(dead) + nC)) {
+          q.A = smA[tbase + gl];
+          q.mu = smMu[tbase + gl];
+          q.var = smVar[tbase + gl];
+          q.t = smT[tbase + gl];
+          q.sp = smSp[tbase + gl];
+        } else {
+          q = tk_empty();
+        }
+        __syncwarp(gm);
       }
     }
   }
   if (slot) {
     const size_t o = (size_t(i) * 2 + rf) * K + gl;
-    P.q[o] = make_double2(qmu, qvar);
-    P.qsp[o] = qsp;
+    P.q[o] = make_double2(q.mu, q.var);
+    P.qsp[o] = q.sp;
+  }
+}
+
+// Pins with exactly one fanin arc that is not non-unate (net sinks, the
+// inputs of one-input cells): one batch from one parent, whose startpoints
+// are unique, so Alg 2 reduces to ordering the K candidates by key.  A lean
+// kernel (no merge state) that runs at full occupancy.
+template <int G>
+__global__ void __launch_bounds__(256, 8) tk_one_kernel(TkParams P) {
+  const int lane = threadIdx.x & 31;
+  const int gl = lane & (G - 1), gbase = lane & ~(G - 1);
+  const unsigned gm = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << gbase);
+  const long long grp = (blockIdx.x * (long long)blockDim.x + threadIdx.x) / G;
+  if (grp >= 2LL * (P.hi - P.lo)) return;
+  const int i = __ldg(P.list + P.lo + int(grp >> 1)), rf = int(grp & 1), K = P.K;
+  const bool slot = gl < K;
+  const int a = __ldg(P.fanin_ptr + i);
+  const int32_t w = __ldg(P.fin_src + a);
+  const float4 ms = __ldg(P.fin_ms + a);
+  const size_t ps = (size_t(w & kSrcMask) * 2 + src_tr(rf, int(uint32_t(w) >> kUnateShift), 0)) * K + gl;
+  const int csp = slot ? __ldg(P.qsp + ps) : -1;
+  const double2 pv = slot ? __ldg(P.q + ps) : make_double2(0.0, 0.0);
+  const double se = double(rf ? ms.w : ms.z);
+  const double mu = pv.x + double(rf ? ms.y : ms.x);   // Eq 1
+  const double var = pv.y + se * se;                   // Eq 2
+  double A = csp >= 0 ? mu + P.ns * double(sigma_of(var)) : -INFINITY;   // Eq 3
+  int t = csp >= 0 ? gl * 2 : INT_MAX;                 // single arc: t = 2k
+  const double nA = __shfl_down_sync(gm, A, 1, G);
+  const int nt = __shfl_down_sync(gm, t, 1, G);
+  int idx = gl;
+  if (__ballot_sync(gm, gl + 1 < G && key_gt(nA, nt, A, t)) & gm) bitonic_desc<G>(gm, gl, A, t, idx);
+  const double omu = __shfl_sync(gm, mu, gbase + idx), ovar = __shfl_sync(gm, var, gbase + idx);
+  const int osp = __shfl_sync(gm, csp, gbase + idx);
+  if (slot) {
+    const size_t o = (size_t(i) * 2 + rf) * K + gl;
+    P.q[o] = osp >= 0 ? make_double2(omu, ovar) : make_double2(0.0, 0.0);
+    P.qsp[o] = osp;
   }
 }
 
@@ -299,6 +489,35 @@ static int pow2_group(int K) {
 }
 
 int ensure_topk(DevGraph& g, int K) {
+  if (!g.tk_list && g.n > 0) {
+    // per level: single-arc (not non-unate) pins first, then the merging ones
+    std::vector<int32_t> fsrc(size_t(std::max<int64_t>(g.e, 1)));
+    if (g.e > 0) {
+      cudaError_t e = cudaMemcpy(fsrc.data(), g.fin_src, sizeof(int32_t) * size_t(g.e), cudaMemcpyDeviceToHost);
+      if (e != cudaSuccess) return int(e);
+    }
+    const std::vector<int32_t>& lp = g.host.level_ptr;
+    const std::vector<int32_t>& fp = g.host.fanin_ptr;
+    std::vector<int32_t> list;
+    list.reserve(size_t(g.n));
+    g.tk_one_ptr.assign(size_t(g.num_levels) + 1, 0);
+    g.tk_multi_ptr.assign(size_t(g.num_levels) + 1, 0);
+    for (int l = 0; l < g.num_levels; ++l) {
+      g.tk_one_ptr[l] = int32_t(list.size());
+      if (l > 0)
+        for (int p = lp[l]; p < lp[l + 1]; ++p)
+          if (fp[p + 1] - fp[p] == 1 && (uint32_t(fsrc[fp[p]]) >> kUnateShift) != 2u) list.push_back(p);
+      g.tk_multi_ptr[l] = int32_t(list.size());
+      if (l > 0)
+        for (int p = lp[l]; p < lp[l + 1]; ++p)
+          if (!(fp[p + 1] - fp[p] == 1 && (uint32_t(fsrc[fp[p]]) >> kUnateShift) != 2u)) list.push_back(p);
+    }
+    g.tk_one_ptr[g.num_levels] = g.tk_multi_ptr[g.num_levels] = int32_t(list.size());
+    cudaError_t e = cudaMalloc(&g.tk_list, sizeof(int32_t) * std::max<size_t>(list.size(), 1));
+    if (e == cudaSuccess && !list.empty())
+      e = cudaMemcpy(g.tk_list, list.data(), sizeof(int32_t) * list.size(), cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) return int(e);
+  }
   if (g.tk_K == K && g.tk_q) return 0;
   if (g.tk_q) cudaFree(g.tk_q);
   if (g.tk_sp) cudaFree(g.tk_sp);
@@ -316,6 +535,26 @@ int ensure_topk(DevGraph& g, int K) {
   return 0;
 }
 
+template <int G>
+static void launch_one(unsigned blocks, cudaStream_t st, const TkParams& P) {
+  tk_one_kernel<G><<<blocks, 256, 0, st>>>(P);
+}
+template <int G>
+static void launch_multi(unsigned blocks, cudaStream_t st, const TkParams& P) {
+  tk_level_kernel<G><<<blocks, 256, 0, st>>>(P);
+}
+
+static void launch_g(bool one, int G, unsigned blocks, cudaStream_t st, const TkParams& P) {
+  switch (G) {
+    case 1: one ? launch_one<1>(blocks, st, P) : launch_multi<1>(blocks, st, P); break;
+    case 2: one ? launch_one<2>(blocks, st, P) : launch_multi<2>(blocks, st, P); break;
+    case 4: one ? launch_one<4>(blocks, st, P) : launch_multi<4>(blocks, st, P); break;
+    case 8: one ? launch_one<8>(blocks, st, P) : launch_multi<8>(blocks, st, P); break;
+    case 16: one ? launch_one<16>(blocks, st, P) : launch_multi<16>(blocks, st, P); break;
+    default: one ? launch_one<32>(blocks, st, P) : launch_multi<32>(blocks, st, P); break;
+  }
+}
+
 int launch_topk_forward(DevGraph& g, int K, float n_sigma, void* stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   int err = ensure_topk(g, K);
@@ -326,28 +565,32 @@ int launch_topk_forward(DevGraph& g, int K, float n_sigma, void* stream) {
   TkParams P;
   P.K = K;
   P.ns = double(n_sigma);
+  P.list = g.tk_list;
   P.fanin_ptr = g.fanin_ptr;
   P.fin_src = g.fin_src;
   P.fin_ms = g.fin_ms;
   P.q = g.tk_q;
   P.qsp = g.tk_sp;
   const int G = pow2_group(K);
-  const std::vector<int32_t>& lp = g.host.level_ptr;
   for (int l = 1; l < g.num_levels; ++l) {
-    P.lo = lp[l];
-    P.hi = lp[l + 1];
-    const long long threads = 2LL * (P.hi - P.lo) * G;
-    const unsigned blocks = unsigned((threads + 255) / 256);
-    switch (G) {
-      case 1: tk_level_kernel<1><<<blocks, 256, 0, st>>>(P); break;
-      case 2: tk_level_kernel<2><<<blocks, 256, 0, st>>>(P); break;
-      case 4: tk_level_kernel<4><<<blocks, 256, 0, st>>>(P); break;
-      case 8: tk_level_kernel<8><<<blocks, 256, 0, st>>>(P); break;
-      case 16: tk_level_kernel<16><<<blocks, 256, 0, st>>>(P); break;
-      default: tk_level_kernel<32><<<blocks, 256, 0, st>>>(P); break;
+    for (int part = 0; part < 2; ++part) {   // single-arc pins, then merging pins (independent)
+      P.lo = part == 0 ? g.tk_one_ptr[l] : g.tk_multi_ptr[l];
+      P.hi = part == 0 ? g.tk_multi_ptr[l] : g.tk_one_ptr[l + 1];
+      if (P.hi <= P.lo) continue;
+      const long long threads = 2LL * (P.hi - P.lo) * G;
+      launch_g(part == 0, G, unsigned((threads + 255) / 256), st, P);
     }
   }
   return int(cudaGetLastError());
+}
+
+int topk_stats(unsigned long long* out) {
+#ifdef TK_STATS
+  return int(cudaMemcpyFromSymbol(out, tk_stats, sizeof(unsigned long long) * 33));
+#else
+  (void)out;
+  return -1;
+#endif
 }
 
 int launch_topk_slack(DevGraph& g, float n_sigma, void* stream) {

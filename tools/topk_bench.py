@@ -6,7 +6,7 @@ import json
 import os
 import sys
 
-ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+ROOT = os.environ.get("INSTA_ROOT") or os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
 import numpy as np  # noqa: E402
@@ -43,5 +43,6 @@ for K in Ks:
     s_ms = ev[1].elapsed_time(ev[2]) / n
     out.append(dict(config=cfg, K=K, fwd_ms=f_ms, slack_ms=s_ms, tns=summ.tns, wns=summ.wns,
                     nviol=summ.num_violations, pins=g.num_pins, arcs=g.num_arcs))
+    out[-1]["variant"] = os.environ.get("VARIANT", "")
     print(json.dumps(out[-1]), flush=True)
 G.close()
