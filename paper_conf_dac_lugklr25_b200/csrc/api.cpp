@@ -67,6 +67,9 @@ void free_graph(insta::DevGraph& d) {
   for (void* p : ptrs)
     if (p) cudaFree(p);
   if (d.b_stage_h) cudaFreeHost(d.b_stage_h);
+  for (void* ev : d.tk_ev)
+    if (ev) cudaEventDestroy(static_cast<cudaEvent_t>(ev));
+  if (d.tk_side) cudaStreamDestroy(static_cast<cudaStream_t>(d.tk_side));
   if (d.b_stage_copied) cudaEventDestroy(static_cast<cudaEvent_t>(d.b_stage_copied));
   if (d.b_stage_done) cudaEventDestroy(static_cast<cudaEvent_t>(d.b_stage_done));
 }

@@ -224,6 +224,8 @@ struct DevGraph {
   int32_t* tk_sp = nullptr;        // [n][2][K] canonical startpoint, -1 = empty slot
   int32_t* tk_list = nullptr;      // [n - num_src] per level: single-arc pins, then merging pins
   std::vector<int32_t> tk_one_ptr, tk_multi_ptr;   // [L+1] offsets of the two parts per level
+  void* tk_side = nullptr;         // cudaStream_t for the single-arc part of each level
+  void* tk_ev[2] = {nullptr, nullptr};   // cudaEvent_t join events
   double* tk_slack = nullptr;      // [P] CPPR slack (fp64)
   int32_t* tk_star = nullptr;      // [2][P] critical startpoint | rf << 30, slot k
   double* tk_summary = nullptr;    // {wns, tns, violations}

@@ -248,8 +248,29 @@ __global__ void __launch_bounds__(256, TK_MINB) tk_level_kernel(TkParams P) {
         // search in the other sorted list; (4) scatter the top K through
         // shared memory.
         int f = -1;
-        for (int r = 0; r < K; ++r)
-          if (__shfl_sync(gm, q.sp, gbase + r) == csp) f = r;
+        const int ssp = surv ? csp : -1;
+        if (G >= 4) {
+          // __match_any over half-groups: lanes [0, H) carry queue slots,
+          // lanes [H, G) survivors' startpoints; four calls cover all pairs
+          constexpr int H = G / 2;
+#pragma unroll
+          for (int qh = 0; qh < 2; ++qh) {
+#pragma unroll
+            for (int ch = 0; ch < 2; ++ch) {
+              const int qs = __shfl_sync(gm, q.sp, gbase + qh * H + (gl & (H - 1)));
+              const int cs = __shfl_sync(gm, ssp, gbase + ch * H + (gl & (H - 1)));
+              const unsigned v = gl < H ? (qs >= 0 ? unsigned(qs) : 0x40000000u | gl)
+                                        : (cs >= 0 ? unsigned(cs) : 0x60000000u | gl);
+              const unsigned qb = (__match_any_sync(gm, v) >> gbase) & ((1u << H) - 1u);
+              const int fq = qb ? qh * H + __ffs(qb) - 1 : -1;
+              const int r = __shfl_sync(gm, fq, gbase + H + (gl & (H - 1)));
+              if ((gl >> Log2<H>::v) == ch && r >= 0) f = r;
+            }
+          }
+        } else {
+          for (int r = 0; r < K; ++r)
+            if (__shfl_sync(gm, q.sp, gbase + r) == ssp && ssp >= 0) f = r;
+        }
         const double fA = __shfl_sync(gm, q.A, gbase + max(f, 0));
         const int ft = __shfl_sync(gm, q.t, gbase + max(f, 0));
         bool keep = surv;
@@ -259,10 +280,22 @@ __global__ void __launch_bounds__(256, TK_MINB) tk_level_kernel(TkParams P) {
           else keep = false;
         }
         const unsigned dead = __reduce_or_sync(gm, deadbit);
-        double sA = keep ? c.A : -INFINITY;
-        int st = keep ? c.t : INT_MAX, idx = gl;
-        bitonic_desc<G>(gm, gl, sA, st, idx);
-        const int nC = __popc(__ballot_sync(gm, keep) & gm);
+        // kept candidates compacted in lane order (a parent's queue order is
+        // mostly preserved by Eq 1-3), then sorted only if out of order
+        const unsigned km = (__ballot_sync(gm, keep) & gm) >> gbase;
+        const int nC = __popc(km);
+        int idx = gl < nC ? int(__fns(km, 0, gl + 1)) : gl;
+        double sA = __shfl_sync(gm, c.A, gbase + idx);
+        int st = __shfl_sync(gm, c.t, gbase + idx);
+        if (gl >= nC) {
+          sA = -INFINITY;
+          st = INT_MAX;
+        }
+        {
+          const double nA = __shfl_down_sync(gm, sA, 1, G);
+          const int nt = __shfl_down_sync(gm, st, 1, G);
+          if (__ballot_sync(gm, gl + 1 < nC && key_gt(nA, nt, sA, st)) & gm) bitonic_desc<G>(gm, gl, sA, st, idx);
+        }
         const unsigned qv = (__ballot_sync(gm, slot && q.sp >= 0) & gm) >> gbase;
         const int nQ = __popc(qv);
         int lo = 0, hi = nC;   // kept candidates ahead of my queue entry
@@ -518,6 +551,15 @@ int ensure_topk(DevGraph& g, int K) {
       e = cudaMemcpy(g.tk_list, list.data(), sizeof(int32_t) * list.size(), cudaMemcpyHostToDevice);
     if (e != cudaSuccess) return int(e);
   }
+  if (!g.tk_side) {
+    cudaStream_t s2;
+    cudaError_t e = cudaStreamCreateWithFlags(&s2, cudaStreamNonBlocking);
+    if (e != cudaSuccess) return int(e);
+    g.tk_side = s2;
+    cudaEvent_t* ev = reinterpret_cast<cudaEvent_t*>(g.tk_ev);
+    for (int k = 0; k < 2 && e == cudaSuccess; ++k) e = cudaEventCreateWithFlags(&ev[k], cudaEventDisableTiming);
+    if (e != cudaSuccess) return int(e);
+  }
   if (g.tk_K == K && g.tk_q) return 0;
   if (g.tk_q) cudaFree(g.tk_q);
   if (g.tk_sp) cudaFree(g.tk_sp);
@@ -572,15 +614,33 @@ int launch_topk_forward(DevGraph& g, int K, float n_sigma, void* stream) {
   P.q = g.tk_q;
   P.qsp = g.tk_sp;
   const int G = pow2_group(K);
-  for (int l = 1; l < g.num_levels; ++l) {
-    for (int part = 0; part < 2; ++part) {   // single-arc pins, then merging pins (independent)
-      P.lo = part == 0 ? g.tk_one_ptr[l] : g.tk_multi_ptr[l];
-      P.hi = part == 0 ? g.tk_multi_ptr[l] : g.tk_one_ptr[l + 1];
-      if (P.hi <= P.lo) continue;
-      const long long threads = 2LL * (P.hi - P.lo) * G;
-      launch_g(part == 0, G, unsigned((threads + 255) / 256), st, P);
+  // The two parts of a level are independent: the bandwidth-bound single-arc
+  // kernel runs on a side stream next to the ALU-bound merging kernel on the
+  // caller's stream; each waits for both parts of the previous level.
+  cudaStream_t s2 = static_cast<cudaStream_t>(g.tk_side);
+  cudaEvent_t* ev = reinterpret_cast<cudaEvent_t*>(g.tk_ev);
+  cudaError_t e = cudaEventRecord(ev[0], st);   // sources written
+  if (e == cudaSuccess) e = cudaStreamWaitEvent(s2, ev[0], 0);
+  for (int l = 1; l < g.num_levels && e == cudaSuccess; ++l) {
+    const bool has_one = g.tk_multi_ptr[l] > g.tk_one_ptr[l];
+    const bool has_multi = g.tk_one_ptr[l + 1] > g.tk_multi_ptr[l];
+    if (has_one) {
+      P.lo = g.tk_one_ptr[l];
+      P.hi = g.tk_multi_ptr[l];
+      launch_g(true, G, unsigned((2LL * (P.hi - P.lo) * G + 255) / 256), s2, P);
+      e = cudaEventRecord(ev[1], s2);
     }
+    if (has_multi) {
+      P.lo = g.tk_multi_ptr[l];
+      P.hi = g.tk_one_ptr[l + 1];
+      launch_g(false, G, unsigned((2LL * (P.hi - P.lo) * G + 255) / 256), st, P);
+    }
+    // join: the caller's stream waits for the side part; the side stream for the caller's
+    if (e == cudaSuccess && has_one) e = cudaStreamWaitEvent(st, ev[1], 0);
+    if (e == cudaSuccess && has_multi) e = cudaEventRecord(ev[0], st);
+    if (e == cudaSuccess && has_multi) e = cudaStreamWaitEvent(s2, ev[0], 0);
   }
+  if (e != cudaSuccess) return int(e);
   return int(cudaGetLastError());
 }
 
