@@ -204,3 +204,27 @@ def topk_slack(g, q, rat_table=None):
     _check(L.orc_topk_slack(ctypes.byref(og.c), K, _p(A), _p(sp), _p(rp), _p(rs), _p(rv), _p(s), _p(r), _p(ks),
                             _p(ss), ctypes.byref(wns), ctypes.byref(tns), ctypes.byref(nv)))
     return dict(slack=s, rf_star=r, k_star=ks, sp_star=ss, wns=wns.value, tns=tns.value, num_viol=nv.value)
+
+
+def clark_forward(g, n_sigma=3.0):
+    """NEXT 2: Clark moment-matching merge.  Returns dict(A, mu, sigma [N,2])."""
+    og = _og(g)
+    N = og.N
+    A = np.zeros((N, 2)); mu = np.zeros((N, 2)); sig = np.zeros((N, 2))
+    L = lib()
+    L.orc_clark_forward.argtypes = [ctypes.c_void_p, ctypes.c_double] + [ctypes.c_void_p] * 3
+    _check(L.orc_clark_forward(ctypes.byref(og.c), float(n_sigma), _p(A), _p(mu), _p(sig)))
+    return dict(A=A, mu=mu, sigma=sig)
+
+
+def clark_backward(g, n_sigma=3.0, dslack=None):
+    """Backward of the Clark path.  Returns dict(d_mean, d_sigma [E,2], d_src_mean, d_src_sigma [N,2])."""
+    og = _og(g)
+    E, N = og.E, og.N
+    dm = np.zeros((E, 2)); ds = np.zeros((E, 2)); dsm = np.zeros((N, 2)); dss = np.zeros((N, 2))
+    if dslack is not None:
+        dslack = np.ascontiguousarray(dslack, np.float64)
+    L = lib()
+    L.orc_clark_backward.argtypes = [ctypes.c_void_p, ctypes.c_double] + [ctypes.c_void_p] * 5
+    _check(L.orc_clark_backward(ctypes.byref(og.c), float(n_sigma), _p(dslack), _p(dm), _p(ds), _p(dsm), _p(dss)))
+    return dict(d_mean=dm, d_sigma=ds, d_src_mean=dsm, d_src_sigma=dss)

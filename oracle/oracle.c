@@ -635,3 +635,212 @@ int orc_topk_slack(const orc_graph* g, int32_t K, const double* A, const int32_t
   if (num_viol) *num_viol = nv;
   return 0;
 }
+
+/* ------------------------------------------------------------------------- */
+/* NEXT 2: Clark moment-matching statistical max, the merge    */
+/* the north star names beside the paper's smooth max.  The state of a pin is */
+/* the Gaussian (mu, V = sigma^2) per rf; a candidate is (mu_j[s] + mean_e,   */
+/* V_j[s] + std_e^2) (Eq 1-2); the merge folds the candidates in canonical    */
+/* order (fanin row, then s = rf before ~rf) with Clark's two-input max of    */
+/* independent Gaussians (reading R20: rho = 0):                              */
+/*   a = sqrt(V1 + V2), alpha = (mu1 - mu2) / a                               */
+/*   mu  = mu1 Phi(alpha) + mu2 Phi(-alpha) + a phi(alpha)                    */
+/*   E2  = (mu1^2 + V1) Phi(alpha) + (mu2^2 + V2) Phi(-alpha)                 */
+/*         + (mu1 + mu2) a phi(alpha),      V = E2 - mu^2                     */
+/* (a = 0: the hard max, first input wins ties).  Endpoint arrival Eq 3:      */
+/* A = mu + N_sigma sqrt(V); slack / WNS / TNS as O6.                         */
+/* ------------------------------------------------------------------------- */
+static double Phi_(double x) { return 0.5 * erfc(-x / sqrt(2.0)); }
+static double phi_(double x) { return exp(-0.5 * x * x) / sqrt(2.0 * 3.14159265358979323846); }
+
+static void clark2(double m1, double v1, double m2, double v2, double* m, double* v) {
+  double a2 = v1 + v2;
+  if (!(a2 > 0.0)) {                     /* both deterministic: hard max, first wins ties */
+    if (m2 > m1) { *m = m2; *v = v2; } else { *m = m1; *v = v1; }
+    return;
+  }
+  double a = sqrt(a2), al = (m1 - m2) / a;
+  double P = Phi_(al), Q = Phi_(-al), p = phi_(al);
+  *m = m1 * P + m2 * Q + a * p;
+  double e2 = (m1 * m1 + v1) * P + (m2 * m2 + v2) * Q + (m1 + m2) * a * p;
+  *v = e2 - (*m) * (*m);
+  if (*v < 0.0) *v = 0.0;
+}
+
+/* Jacobian of clark2: d(mu, V)/d(m1, v1, m2, v2), rows J[0] = dmu, J[1] = dV */
+static void clark2_jac(double m1, double v1, double m2, double v2, double J[2][4]) {
+  double a2 = v1 + v2;
+  if (!(a2 > 0.0)) {
+    int second = m2 > m1;
+    for (int r = 0; r < 2; ++r) for (int c = 0; c < 4; ++c) J[r][c] = 0.0;
+    J[0][second ? 2 : 0] = 1.0;
+    J[1][second ? 3 : 1] = 1.0;
+    return;
+  }
+  double a = sqrt(a2), al = (m1 - m2) / a;
+  double P = Phi_(al), Q = Phi_(-al), p = phi_(al);
+  double mu = m1 * P + m2 * Q + a * p;
+  /* d mu */
+  double dm1 = P, dm2 = Q, dv = p / (2.0 * a);
+  /* d E2 (derived from the closed form; pinned by finite differences in tests) */
+  double e_m1 = 2.0 * m1 * P + a * p + (p / a) * (v1 - v2);
+  double e_m2 = 2.0 * m2 * Q + a * p - (p / a) * (v1 - v2);
+  double e_a = (m1 + m2) * p - al * p * (v1 - v2) / a;
+  double e_v1 = P + e_a / (2.0 * a), e_v2 = Q + e_a / (2.0 * a);
+  J[0][0] = dm1; J[0][1] = dv; J[0][2] = dm2; J[0][3] = dv;
+  J[1][0] = e_m1 - 2.0 * mu * dm1;
+  J[1][1] = e_v1 - 2.0 * mu * dv;
+  J[1][2] = e_m2 - 2.0 * mu * dm2;
+  J[1][3] = e_v2 - 2.0 * mu * dv;
+}
+
+typedef struct { int32_t arc, src; int s; double mu, v; } ccand_t;
+
+static int clark_candidates(const orc_graph* g, const topo_t* t, int32_t k, int rf, const double* M,
+                            const double* V, ccand_t* c) {
+  int n = 0;
+  for (int32_t q = t->fanin_ptr[k]; q < t->fanin_ptr[k + 1]; ++q) {
+    int32_t e = t->fanin_arc[q], j = g->arc_from[e];
+    int ss[2];
+    int ns = sources_of(rf, g->arc_unate[e], ss);
+    for (int a = 0; a < ns; ++a) {
+      double sd = g->arc_sigma[2 * (int64_t)e + rf];
+      c[n].arc = e; c[n].src = j; c[n].s = ss[a];
+      c[n].mu = M[2 * (int64_t)j + ss[a]] + g->arc_mean[2 * (int64_t)e + rf];   /* Eq 1 */
+      c[n].v = V[2 * (int64_t)j + ss[a]] + sd * sd;                              /* Eq 2 */
+      ++n;
+    }
+  }
+  return n;
+}
+
+static void clark_propagate(const orc_graph* g, const topo_t* t, double* M, double* V) {
+  ccand_t* c = malloc(sizeof(ccand_t) * 2 * (size_t)max_fanin(t));
+  for (int32_t k = 0; k < t->n; ++k) {
+    int32_t i = t->order[k];
+    for (int rf = 0; rf < 2; ++rf) {
+      int64_t x = 2 * (int64_t)i + rf;
+      if (t->fanin_ptr[k] == t->fanin_ptr[k + 1]) {     /* startpoint */
+        double s = g->src_sigma ? g->src_sigma[x] : 0.0;
+        M[x] = g->src_mean ? g->src_mean[x] : 0.0;
+        V[x] = s * s;
+        continue;
+      }
+      int n = clark_candidates(g, t, k, rf, M, V, c);
+      double m = c[0].mu, v = c[0].v;
+      for (int a = 1; a < n; ++a) clark2(m, v, c[a].mu, c[a].v, &m, &v);   /* fold in order */
+      M[x] = m;
+      V[x] = v;
+    }
+  }
+  free(c);
+}
+
+int orc_clark_forward(const orc_graph* g, double n_sigma, double* A, double* mu, double* sig) {
+  int st = orc_validate(g, n_sigma, 0.0);
+  if (st) return st;
+  topo_t t;
+  st = topo_build(g->num_pins, g->num_arcs, g->arc_from, g->arc_to, &t);
+  if (st) return st;
+  size_t n2 = 2 * (size_t)g->num_pins + 2;
+  double* M = malloc(n2 * sizeof(double));
+  double* V = malloc(n2 * sizeof(double));
+  clark_propagate(g, &t, M, V);
+  for (int64_t x = 0; x < 2 * (int64_t)g->num_pins; ++x) {
+    if (A) A[x] = M[x] + n_sigma * sqrt(V[x]);   /* Eq 3 */
+    if (mu) mu[x] = M[x];
+    if (sig) sig[x] = sqrt(V[x]);
+  }
+  free(M); free(V);
+  topo_free(&t);
+  return 0;
+}
+
+/* Backward of the Clark path (push style, reverse canonical order).  Seeds:
+ * slack = RAT - (mu + Ns sqrt(V)) at rf*, so dL/dmu = -seed and
+ * dL/dV = -seed Ns / (2 sqrt(V)) (0 if V = 0).  Through the fold: reverse
+ * over the prefix results r_k = clark(r_{k-1}, c_k) with clark2_jac.  A
+ * candidate passes its adjoint to the source (mu, V) and to the arc:
+ * d mean_e += mubar_c, d sigma_e += 2 std_e Vbar_c; sources: d src_mean =
+ * mubar, d src_sigma = 2 sigma_src Vbar. */
+int orc_clark_backward(const orc_graph* g, double n_sigma, const double* dslack, double* d_mean,
+                       double* d_sigma, double* d_src_mean, double* d_src_sigma) {
+  int st = orc_validate(g, n_sigma, 0.0);
+  if (st) return st;
+  topo_t t;
+  st = topo_build(g->num_pins, g->num_arcs, g->arc_from, g->arc_to, &t);
+  if (st) return st;
+  int32_t N = g->num_pins;
+  int64_t E = g->num_arcs;
+  size_t n2 = 2 * (size_t)N + 2;
+  double* M = malloc(n2 * sizeof(double));
+  double* V = malloc(n2 * sizeof(double));
+  clark_propagate(g, &t, M, V);
+  double* mb = calloc(n2, sizeof(double));
+  double* vb = calloc(n2, sizeof(double));
+  double* dm = calloc(2 * (size_t)E + 2, sizeof(double));
+  double* ds = calloc(2 * (size_t)E + 2, sizeof(double));
+  for (int32_t k = 0; k < g->num_endpoints; ++k) {
+    int32_t p = g->ep_pin[k];
+    double ar = M[2 * (int64_t)p] + n_sigma * sqrt(V[2 * (int64_t)p]);
+    double af = M[2 * (int64_t)p + 1] + n_sigma * sqrt(V[2 * (int64_t)p + 1]);
+    double sr = g->ep_rat[2 * k] - ar, sf = g->ep_rat[2 * k + 1] - af;
+    int r = (sf < sr) ? FALL : RISE;
+    double s = (r == FALL) ? sf : sr;
+    double seed = dslack ? dslack[k] : (s < 0 ? 1.0 : 0.0);
+    int64_t x = 2 * (int64_t)p + r;
+    mb[x] += -seed;
+    if (V[x] > 0.0) vb[x] += -seed * n_sigma / (2.0 * sqrt(V[x]));
+  }
+  int mf = 2 * max_fanin(&t);
+  ccand_t* c = malloc(sizeof(ccand_t) * (size_t)mf);
+  double* rm = malloc(sizeof(double) * (size_t)mf);
+  double* rv = malloc(sizeof(double) * (size_t)mf);
+  double* cmb = malloc(sizeof(double) * (size_t)mf);
+  double* cvb = malloc(sizeof(double) * (size_t)mf);
+  for (int32_t k = N - 1; k >= 0; --k) {
+    int32_t i = t.order[k];
+    if (t.fanin_ptr[k] == t.fanin_ptr[k + 1]) continue;
+    for (int rf = 0; rf < 2; ++rf) {
+      int64_t x = 2 * (int64_t)i + rf;
+      if (mb[x] == 0.0 && vb[x] == 0.0) continue;
+      int n = clark_candidates(g, &t, k, rf, M, V, c);
+      rm[0] = c[0].mu; rv[0] = c[0].v;                 /* prefix results of the fold */
+      for (int a = 1; a < n; ++a) clark2(rm[a - 1], rv[a - 1], c[a].mu, c[a].v, &rm[a], &rv[a]);
+      double um = mb[x], uv = vb[x];                   /* adjoint of r_{n-1} */
+      for (int a = n - 1; a >= 1; --a) {
+        double J[2][4];
+        clark2_jac(rm[a - 1], rv[a - 1], c[a].mu, c[a].v, J);
+        cmb[a] = um * J[0][2] + uv * J[1][2];
+        cvb[a] = um * J[0][3] + uv * J[1][3];
+        double pm = um * J[0][0] + uv * J[1][0];
+        double pv = um * J[0][1] + uv * J[1][1];
+        um = pm; uv = pv;
+      }
+      cmb[0] = um; cvb[0] = uv;
+      for (int a = 0; a < n; ++a) {
+        int64_t e = c[a].arc;
+        int64_t y = 2 * (int64_t)c[a].src + c[a].s;
+        mb[y] += cmb[a];
+        vb[y] += cvb[a];
+        dm[2 * e + rf] += cmb[a];
+        ds[2 * e + rf] += 2.0 * g->arc_sigma[2 * e + rf] * cvb[a];
+      }
+    }
+  }
+  if (d_mean) memcpy(d_mean, dm, sizeof(double) * 2 * (size_t)E);
+  if (d_sigma) memcpy(d_sigma, ds, sizeof(double) * 2 * (size_t)E);
+  for (int32_t p = 0; p < N; ++p) {
+    int is_src = (t.fanin_ptr[t.pos[p]] == t.fanin_ptr[t.pos[p] + 1]);
+    for (int rf = 0; rf < 2; ++rf) {
+      int64_t x = 2 * (int64_t)p + rf;
+      double ssd = g->src_sigma ? g->src_sigma[x] : 0.0;
+      if (d_src_mean) d_src_mean[x] = is_src ? mb[x] : 0.0;
+      if (d_src_sigma) d_src_sigma[x] = is_src ? 2.0 * ssd * vb[x] : 0.0;
+    }
+  }
+  free(c); free(rm); free(rv); free(cmb); free(cvb);
+  free(M); free(V); free(mb); free(vb); free(dm); free(ds);
+  topo_free(&t);
+  return 0;
+}

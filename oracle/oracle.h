@@ -89,6 +89,15 @@ int orc_topk_slack(const orc_graph* g, int32_t K, const double* A, const int32_t
                    double* slack, uint8_t* rf_star, int32_t* k_star, int32_t* sp_star,
                    double* wns, double* tns, int32_t* num_viol);
 
+/* NEXT 2: Clark moment-matching merge (reading R20, rho = 0), folded in
+ * candidate order.  A/mu/sig [N][2] caller-indexed (sig = sqrt(V)). */
+int orc_clark_forward(const orc_graph* g, double n_sigma, double* A, double* mu, double* sig);
+
+/* Backward of the Clark path: dL/d(arc mean), dL/d(arc sigma) [E][2],
+ * dL/d(src mean / sigma) [N][2]; dslack = NULL means L = TNS.  Any output may be NULL. */
+int orc_clark_backward(const orc_graph* g, double n_sigma, const double* dslack, double* d_mean,
+                       double* d_sigma, double* d_src_mean, double* d_src_sigma);
+
 #ifdef __cplusplus
 }
 #endif
