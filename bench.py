@@ -221,6 +221,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--batch-scenarios", type=int, default=1024, help="C5 batched evaluations (0 = skip)")
     ap.add_argument("--topk", type=int, default=32, help="Top-K CPPR propagation K (0 = skip)")
+    ap.add_argument("--clark", type=int, default=1, help="time the Clark merge path (0 = skip)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -416,6 +417,31 @@ def main():
                 "paper_context": "PAPER.md Table I (L184-193): block-1 (15M pins) at TopK=32 in 0.39 s on 1x A100 "
                                  "(incl. its own slack); other hardware, other design"}
 
+    # ---------------- Clark moment-matching merge -------------
+    clark = None
+    if args.clark:
+        with torch.cuda.stream(stream):
+            for _ in range(2):
+                G.clark_forward(3.0, sync=False, stream=stream)
+                G.clark_backward(stream=stream)
+            stream.synchronize()
+            nk = max(1, min(args.steps, 5))
+            c0, c1, c2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+            dcl = torch.empty((E, 2), dtype=torch.float32, device=dev)
+            c0.record(stream)
+            for _ in range(nk):
+                G.clark_forward(3.0, sync=False, stream=stream)
+            c1.record(stream)
+            for _ in range(nk):
+                G.lib.insta_clark_backward(G._h, None, dcl.data_ptr(), None, None, stream.cuda_stream)
+            c2.record(stream)
+            stream.synchronize()
+            cs = G.clark_forward(3.0, stream=stream)
+        cf, cb = c0.elapsed_time(c1) / nk, c1.elapsed_time(c2) / nk
+        clark = {"workload": f"{cfg.name}, Clark moment-matching max (fp64, per-level launches) + slack, and its "
+                             f"TNS backward", "fwd_ms": cf, "bwd_ms": cb, "pins_per_s": N / ((cf + cb) * 1e-3),
+                 "tns": cs.tns, "wns": cs.wns, "violations": cs.num_violations}
+
     cpu = None
     if rank == 0 and not args.no_cpu_baseline:
         try:
@@ -445,7 +471,7 @@ def main():
                          "frac": ach / peak, "peak_kind": peak_kind, "traffic": traffic,
                          "fwd_gbs": fwd_gbs, "bwd_gbs": bwd_gbs, "fwd_alg_bytes": fb, "bwd_alg_bytes": bb},
             "cpu_baseline": cpu, "e2e": e2e, "clocks": clk, "gpu_launches": launches_per_step * args.steps,
-            "batched": batched, "topk": topk,
+            "batched": batched, "topk": topk, "clark": clark,
             "paper_context": "PAPER.md L9/L37: full-graph propagation < 0.1 s on a 15M-pin 3nm design, 1x A100 "
                              "(forward only, Top-K not stated); not the same metric",
         }

@@ -257,6 +257,35 @@ insta_status insta_topk_critical(insta_graph* g, uint8_t* rf_star, int32_t* k_st
  * sp = caller id of the startpoint (-1 for an empty slot). */
 insta_status insta_topk_queues(insta_graph* g, float* A, float* mean, float* sigma, int32_t* sp, void* cuda_stream);
 
+/* ---- Clark moment-matching statistical max ----
+ *
+ * The north star's alternative to the paper's smooth max (Eq 4): a pin's
+ * arrival per rf is the Gaussian (mu, V = sigma^2); candidates (Eq 1-2) are
+ * merged by folding, in canonical candidate order (fanin arcs by caller arc
+ * id, s = rf before ~rf), Clark's exact first two moments of the max of two
+ * INDEPENDENT Gaussians (reading R20, correlation 0); endpoint
+ * arrival A = mu + n_sigma sqrt(V) (Eq 3), slack / WNS / TNS as insta_slack.
+ * fp64 state and arithmetic.  Device memory: 16 B per pin and rf + 128 B per
+ * arc (fold prefixes and candidate adjoints), allocated on first use. */
+
+/* Forward + endpoint slack; out: summary (synchronizes) or NULL. */
+insta_status insta_clark_forward(insta_graph* g, float n_sigma, void* cuda_stream, insta_summary* out);
+
+/* Results of the last insta_clark_forward, DEVICE arrays, caller order, any may
+ * be NULL: A / mean / sigma float[num_pins][2]; slack float[num_endpoints];
+ * rf_star uint8[num_endpoints].  E_STATE without a valid forward. */
+insta_status insta_clark_results(insta_graph* g, float* A, float* mean, float* sigma, float* slack, uint8_t* rf_star,
+                                 void* cuda_stream);
+
+/* Backward of the Clark path: d_arc_mean (required) / d_arc_sigma (NULL ok)
+ * DEVICE float[num_arcs][2] = dL/d(arc mean / arc sigma), d_src DEVICE
+ * float[num_pins][2] = dL/d(startpoint mean) or NULL; L = TNS if ep_seed is
+ * NULL, else sum_ep ep_seed[ep] * slack[ep] (ep_seed DEVICE float[num_endpoints]).
+ * Reverse-level pull through Clark's Jacobian, no atomics (deterministic).
+ * E_STATE without a valid insta_clark_forward (insta_update_arcs invalidates it). */
+insta_status insta_clark_backward(insta_graph* g, const float* ep_seed, float* d_arc_mean, float* d_arc_sigma,
+                                  float* d_src, void* cuda_stream);
+
 /* Statistics of the last forward: number of pins recomputed (== num_pins for a
  * full forward).  For an incremental one: the work-item heads recomputed in
  * the changed cone (insta_graph_schedule; each head's folded input pins are

@@ -231,6 +231,36 @@ class Graph:
               "insta_topk_queues")
         return dict(A=A, mean=m, sigma=s, sp=sp)
 
+    # ------------------------------------------------------------------ Clark merge
+    def clark_forward(self, n_sigma: float = 3.0, sync: bool = True, stream=None):
+        """insta_clark_forward: Clark moment-matching propagation + slack.  Returns a Summary if sync."""
+        out = _capi.insta_summary() if sync else None
+        check(self.lib.insta_clark_forward(self._h, float(n_sigma), self._st(stream),
+                                           ctypes.byref(out) if out is not None else None), "insta_clark_forward")
+        return None if out is None else Summary(out.wns, out.tns, out.num_violations, out.num_levels)
+
+    def clark_results(self, stream=None):
+        """insta_clark_results: dict(A, mean, sigma float32[N,2], slack float32[P], rf_star uint8[P])."""
+        t = self._torch
+        A, m, s = (t.empty((self.num_pins, 2), dtype=t.float32, device=self.device) for _ in range(3))
+        sl = t.empty(self.num_endpoints, dtype=t.float32, device=self.device)
+        rf = t.empty(self.num_endpoints, dtype=t.uint8, device=self.device)
+        check(self.lib.insta_clark_results(self._h, _dptr(A), _dptr(m), _dptr(s), _dptr(sl), _dptr(rf),
+                                           self._st(stream)), "insta_clark_results")
+        return dict(A=A, mean=m, sigma=s, slack=sl, rf_star=rf)
+
+    def clark_backward(self, ep_seed=None, want_sigma: bool = False, want_src: bool = False, stream=None):
+        """insta_clark_backward: d_mean float32[E,2] (+ d_sigma [E,2], + d_src [N,2]) of L = TNS or sum seed*slack."""
+        t = self._torch
+        d_mean = t.empty((self.num_arcs, 2), dtype=t.float32, device=self.device)
+        d_sig = t.empty((self.num_arcs, 2), dtype=t.float32, device=self.device) if want_sigma else None
+        d_src = t.empty((self.num_pins, 2), dtype=t.float32, device=self.device) if want_src else None
+        seed = None if ep_seed is None else t.as_tensor(ep_seed, dtype=t.float32, device=self.device).contiguous()
+        check(self.lib.insta_clark_backward(self._h, _dptr(seed), _dptr(d_mean), _dptr(d_sig), _dptr(d_src),
+                                            self._st(stream)), "insta_clark_backward")
+        outs = (d_mean,) + ((d_sig,) if want_sigma else ()) + ((d_src,) if want_src else ())
+        return outs if len(outs) > 1 else d_mean
+
     def forward_batch(self, scenarios, tau: float = 0.0, want_grad: bool = False, summaries=None, d_mean_sum=None,
                       stream=None):
         """insta_forward_batch: evaluate independent scenarios (dicts with n_sigma, derate_cell, derate_net and

@@ -76,6 +76,9 @@ SIGNATURES = {
     "insta_topk_slack": (ctypes.c_int, [c_vp, c_vp, c_vp, c_vp, ctypes.POINTER(insta_summary)]),
     "insta_topk_critical": (ctypes.c_int, [c_vp, c_vp, c_vp, c_vp]),
     "insta_topk_queues": (ctypes.c_int, [c_vp, c_vp, c_vp, c_vp, c_vp, c_vp]),
+    "insta_clark_forward": (ctypes.c_int, [c_vp, ctypes.c_float, c_vp, ctypes.POINTER(insta_summary)]),
+    "insta_clark_results": (ctypes.c_int, [c_vp, c_vp, c_vp, c_vp, c_vp, c_vp, c_vp]),
+    "insta_clark_backward": (ctypes.c_int, [c_vp, c_vp, c_vp, c_vp, c_vp, c_vp]),
     "insta_last_error": (ctypes.c_char_p, []),
     "insta_version": (ctypes.c_char_p, []),
 }

@@ -63,7 +63,9 @@ void free_graph(insta::DevGraph& d) {
                   d.ep_head,   d.hseed,     d.bwdf_a,    d.bwdf_b,    d.g4,        d.hacc4,
                   d.ext_flags, d.bfwdf_a,   d.bfwdf_b,   d.hd_eop,    d.dirty_h,
                   d.arc_head,  d.ext_h,     d.tk_q,      d.tk_sp,      d.tk_slack,  d.tk_star,
-                  d.tk_summary, d.rat_ptr,  d.rat_sp,    d.rat_val,   d.tk_list};
+                  d.tk_summary, d.rat_ptr,  d.rat_sp,    d.rat_val,   d.tk_list,
+                  d.cl_mv,     d.cl_pre,    d.cl_g,      d.cl_fo_ptr,  d.cl_fo_q,   d.cl_slack,
+                  d.cl_rf,     d.cl_summary, d.cl_hv_list, d.cl_hv_of, d.cl_hv_sum};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   if (d.b_stage_h) cudaFreeHost(d.b_stage_h);
@@ -475,6 +477,7 @@ insta_status insta_update_arcs(insta_graph* g, int64_t n, const int32_t* arc_ids
   if (err) return cuda_fail(err, "update_arcs");
   d.fwd_valid = false;
   d.tk_valid = false;
+  d.cl_valid = false;
   if (incremental && !d.pending_full) d.pending_incremental = true;
   else d.pending_full = true;
   return INSTA_OK;
@@ -669,6 +672,55 @@ insta_status insta_topk_queues(insta_graph* g, float* A, float* mean, float* sig
   cudaSetDevice(d.device);
   int err = insta::launch_topk_export(d, A, mean, sigma, sp, cuda_stream);
   if (err) return cuda_fail(err, "topk_queues");
+  return INSTA_OK;
+}
+
+// ---------------------------------------------------------------------------
+// Clark moment-matching merge
+// ---------------------------------------------------------------------------
+insta_status insta_clark_forward(insta_graph* g, float n_sigma, void* cuda_stream, insta_summary* out) {
+  if (!g) return fail(INSTA_E_ARG, "clark_forward: NULL graph");
+  if (!std::isfinite(n_sigma) || n_sigma < 0.f) return fail(INSTA_E_ARG, "clark_forward: n_sigma must be >= 0");
+  insta::DevGraph& d = g->d;
+  cudaSetDevice(d.device);
+  int err = insta::launch_clark_forward(d, n_sigma, cuda_stream);
+  if (err) return cuda_fail(err, "clark_forward");
+  d.cl_ns = n_sigma;
+  d.cl_valid = true;
+  if (out) {
+    double s[3];
+    cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    cudaError_t e = cudaMemcpyAsync(s, d.cl_summary, sizeof s, cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) return cuda_fail(int(e), "clark_forward");
+    out->wns = s[0];
+    out->tns = s[1];
+    out->num_violations = int32_t(s[2]);
+    out->num_levels = d.num_levels;
+  }
+  return INSTA_OK;
+}
+
+insta_status insta_clark_results(insta_graph* g, float* A, float* mean, float* sigma, float* slack, uint8_t* rf_star,
+                                 void* cuda_stream) {
+  if (!g) return fail(INSTA_E_ARG, "clark_results: NULL graph");
+  insta::DevGraph& d = g->d;
+  if (!d.cl_valid) return fail(INSTA_E_STATE, "clark_results: no valid insta_clark_forward");
+  cudaSetDevice(d.device);
+  int err = insta::launch_clark_export(d, A, mean, sigma, slack, rf_star, cuda_stream);
+  if (err) return cuda_fail(err, "clark_results");
+  return INSTA_OK;
+}
+
+insta_status insta_clark_backward(insta_graph* g, const float* ep_seed, float* d_arc_mean, float* d_arc_sigma,
+                                  float* d_src, void* cuda_stream) {
+  if (!g) return fail(INSTA_E_ARG, "clark_backward: NULL graph");
+  if (!d_arc_mean && g->d.e > 0) return fail(INSTA_E_ARG, "clark_backward: NULL d_arc_mean");
+  insta::DevGraph& d = g->d;
+  if (!d.cl_valid) return fail(INSTA_E_STATE, "clark_backward: no valid insta_clark_forward");
+  cudaSetDevice(d.device);
+  int err = insta::launch_clark_backward(d, ep_seed, d_arc_mean, d_arc_sigma, d_src, cuda_stream);
+  if (err) return cuda_fail(err, "clark_backward");
   return INSTA_OK;
 }
 

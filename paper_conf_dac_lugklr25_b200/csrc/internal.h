@@ -229,6 +229,21 @@ struct DevGraph {
   double* tk_slack = nullptr;      // [P] CPPR slack (fp64)
   int32_t* tk_star = nullptr;      // [2][P] critical startpoint | rf << 30, slot k
   double* tk_summary = nullptr;    // {wns, tns, violations}
+  // Clark moment-matching merge (clark.cu)
+  void* cl_mv = nullptr;           // double2 [n][2] {mu, V}
+  void* cl_pre = nullptr;          // double2 [e][2][2] fold prefix after each candidate
+  void* cl_g = nullptr;            // double2 [e][2][2] candidate adjoints {mubar, Vbar}
+  int32_t* cl_fo_ptr = nullptr;    // [n+1] full fanout rows
+  int32_t* cl_fo_q = nullptr;      // [e] fanin position of each fanout arc
+  double* cl_slack = nullptr;      // [P]
+  uint8_t* cl_rf = nullptr;        // [P]
+  double* cl_summary = nullptr;    // {wns, tns, violations}
+  float cl_ns = 3.f;
+  bool cl_valid = false;
+  int32_t* cl_hv_list = nullptr;   // wide-fanout pins grouped by level
+  int32_t* cl_hv_of = nullptr;     // [n] index into cl_hv_list, -1 = narrow
+  void* cl_hv_sum = nullptr;       // double2 [wide][2]
+  std::vector<int32_t> cl_hv_ptr;  // [L+1]
   // CPPR required times per (endpoint, startpoint) (insta_set_cppr_rat)
   int32_t* rat_ptr = nullptr;      // [P+1] or NULL (no table)
   int32_t* rat_sp = nullptr;       // [M] canonical startpoints, ascending within a row
@@ -301,6 +316,10 @@ int launch_forward_batch(DevGraph& g, const BatchSlice& b, float tau, double* su
 int launch_topk_forward(DevGraph& g, int K, float n_sigma, void* stream);
 int launch_topk_slack(DevGraph& g, float n_sigma, void* stream);
 int topk_stats(unsigned long long* out);
+int launch_clark_forward(DevGraph& g, float n_sigma, void* stream);
+int launch_clark_backward(DevGraph& g, const float* ep_seed, float* d_mean, float* d_sigma, float* d_src,
+                          void* stream);
+int launch_clark_export(DevGraph& g, float* A, float* mean, float* sigma, float* slack, uint8_t* rf, void* stream);
 int launch_topk_export(DevGraph& g, float* A, float* mean, float* sigma, int32_t* sp, void* stream);
 int launch_topk_export_slack(DevGraph& g, float* slack, int32_t* sp_star, uint8_t* rf_star, int32_t* k_star,
                              void* stream);
