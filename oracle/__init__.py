@@ -228,3 +228,16 @@ def clark_backward(g, n_sigma=3.0, dslack=None):
     L.orc_clark_backward.argtypes = [ctypes.c_void_p, ctypes.c_double] + [ctypes.c_void_p] * 5
     _check(L.orc_clark_backward(ctypes.byref(og.c), float(n_sigma), _p(dslack), _p(dm), _p(ds), _p(dsm), _p(dss)))
     return dict(d_mean=dm, d_sigma=ds, d_src_mean=dsm, d_src_sigma=dss)
+
+
+def timing_loss(g, x, y, w, lambda_rc=1.0):
+    """NEXT 4, Eq 7: returns (L, grad_x [N], grad_y [N])."""
+    og = _og(g)
+    x = np.ascontiguousarray(x, np.float64); y = np.ascontiguousarray(y, np.float64)
+    w = np.ascontiguousarray(w, np.float64)
+    gx = np.zeros(og.N); gy = np.zeros(og.N); L = ctypes.c_double()
+    lb = lib()
+    lb.orc_timing_loss.argtypes = [ctypes.c_void_p] * 4 + [ctypes.c_double] + [ctypes.c_void_p] * 3
+    _check(lb.orc_timing_loss(ctypes.byref(og.c), _p(x), _p(y), _p(w), float(lambda_rc), ctypes.byref(L), _p(gx),
+                              _p(gy)))
+    return L.value, gx, gy

@@ -844,3 +844,30 @@ int orc_clark_backward(const orc_graph* g, double n_sigma, const double* dslack,
   topo_free(&t);
   return 0;
 }
+
+/* ------------------------------------------------------------------------- */
+/* NEXT 4: INSTA-Place timing objective, Eq 7:    */
+/*   L = lambda_RC * sum_k (|x_f - x_t| + |y_f - y_t|) * w_k                  */
+/* over every arc k = (f -> t) with weight w_k (reading R21: w_k = the arc's  */
+/* timing sensitivity -dTNS/d(delay), zero for non-critical arcs), and its    */
+/* gradient w.r.t. the pin positions (subgradient sign(0) = 0).  Positions     */
+/* and weights in caller order.                                               */
+/* ------------------------------------------------------------------------- */
+static double sgn(double d) { return d > 0.0 ? 1.0 : (d < 0.0 ? -1.0 : 0.0); }
+
+int orc_timing_loss(const orc_graph* g, const double* x, const double* y, const double* w, double lambda_rc,
+                    double* loss, double* gx, double* gy) {
+  if (!g || !x || !y || !w) return 1;
+  double L = 0.0;
+  if (gx) memset(gx, 0, sizeof(double) * (size_t)g->num_pins);
+  if (gy) memset(gy, 0, sizeof(double) * (size_t)g->num_pins);
+  for (int64_t k = 0; k < g->num_arcs; ++k) {
+    int32_t f = g->arc_from[k], t = g->arc_to[k];
+    double dx = x[f] - x[t], dy = y[f] - y[t];
+    L += (fabs(dx) + fabs(dy)) * w[k];
+    if (gx) { gx[f] += lambda_rc * w[k] * sgn(dx); gx[t] -= lambda_rc * w[k] * sgn(dx); }
+    if (gy) { gy[f] += lambda_rc * w[k] * sgn(dy); gy[t] -= lambda_rc * w[k] * sgn(dy); }
+  }
+  if (loss) *loss = lambda_rc * L;
+  return 0;
+}

@@ -98,6 +98,10 @@ int orc_clark_forward(const orc_graph* g, double n_sigma, double* A, double* mu,
 int orc_clark_backward(const orc_graph* g, double n_sigma, const double* dslack, double* d_mean,
                        double* d_sigma, double* d_src_mean, double* d_src_sigma);
 
+/* NEXT 4: Eq 7 timing objective and its gradient w.r.t. pin x/y (caller order). */
+int orc_timing_loss(const orc_graph* g, const double* x, const double* y, const double* w, double lambda_rc,
+                    double* loss, double* gx, double* gy);
+
 #ifdef __cplusplus
 }
 #endif
