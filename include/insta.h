@@ -286,6 +286,45 @@ insta_status insta_clark_results(insta_graph* g, float* A, float* mean, float* s
 insta_status insta_clark_backward(insta_graph* g, const float* ep_seed, float* d_arc_mean, float* d_arc_sigma,
                                   float* d_src, void* cuda_stream);
 
+/* ---- INSTA-Size device steps ----
+ *
+ * Stage gradient of every cell arc (arc_class 1): "the gradient sum of a cell
+ * arc and its driving net arc" (R22: the driving net arc is
+ * the single fanin arc of the cell arc's input pin when that pin has exactly
+ * one fanin arc and it is a net arc), summed over both transitions; 0 for net
+ * arcs.  d_arc_mean: DEVICE float[num_arcs][2] (e.g. insta_backward's TNS
+ * gradient); stage_grad: DEVICE float[num_arcs], caller order.  E_ARG if the
+ * graph was created without arc_class. */
+insta_status insta_stage_gradients(insta_graph* g, const float* d_arc_mean, float* stage_grad, void* cuda_stream);
+
+/* Threshold + rank ("Stages with gradients above a pre-defined
+ * threshold are prioritized by magnitude"): the caller arc ids with
+ * stage_grad < -threshold (TNS gradients are <= 0), most negative first, ties
+ * in arc id order, written to out_arcs DEVICE int32[num_arcs] (entries past the
+ * count are -1); out_count DEVICE int32[1].  Device-side select + stable radix
+ * sort (CUB). */
+insta_status insta_select_stages(insta_graph* g, const float* stage_grad, float threshold, int32_t* out_arcs,
+                                 int32_t* out_count, void* cuda_stream);
+
+/* ---- INSTA-Place timing objective (Eq 7-8) ----
+ *
+ * L = lambda_rc * sum over arcs k = (f -> t) of (|x_f - x_t| + |y_f - y_t|) * w_k
+ * (Eq 7) with per-arc weights w_k -- the paper's "timing gradients" of the
+ * critical arcs; R21: w_k = -(dTNS/dmean_R + dTNS/dmean_F) of arc k
+ * (>= 0, zero for non-critical arcs), e.g. from insta_backward -- and its
+ * gradient w.r.t. the pin positions (subgradient sign(0) = 0).  pin_x / pin_y:
+ * DEVICE float[num_pins] caller order; arc_w: DEVICE float[num_arcs] caller
+ * order; loss: DEVICE double[1] or NULL; grad_x / grad_y: DEVICE
+ * float[num_pins] or both NULL.  Deterministic (fixed-order fp64 sums, pull-
+ * style gradient, no atomics). */
+insta_status insta_timing_loss(insta_graph* g, const float* pin_x, const float* pin_y, const float* arc_w,
+                               float lambda_rc, double* loss, float* grad_x, float* grad_y, void* cuda_stream);
+
+/* Eq 8's lambda_2 = ||a||_2 / ||b||_2 for two DEVICE float[n] gradient vectors
+ * (a = the default objective's gradient, b = the timing objective's);
+ * out: DEVICE double[1] (0 if ||b|| = 0).  No graph needed. */
+insta_status insta_grad_norm_ratio(int64_t n, const float* a, const float* b, double* out, void* cuda_stream);
+
 /* Statistics of the last forward: number of pins recomputed (== num_pins for a
  * full forward).  For an incremental one: the work-item heads recomputed in
  * the changed cone (insta_graph_schedule; each head's folded input pins are

@@ -241,3 +241,15 @@ def timing_loss(g, x, y, w, lambda_rc=1.0):
     _check(lb.orc_timing_loss(ctypes.byref(og.c), _p(x), _p(y), _p(w), float(lambda_rc), ctypes.byref(L), _p(gx),
                               _p(gy)))
     return L.value, gx, gy
+
+
+def stage_gradients(g, d_mean):
+    """NEXT 3 (R22): per cell arc, the gradient sum of the cell arc and its driving net arc; 0 for net arcs."""
+    og = _og(g)
+    cls = np.ascontiguousarray(g.arc_class, np.uint8)
+    dm = np.ascontiguousarray(np.asarray(d_mean, np.float64).reshape(og.E, 2))
+    out = np.zeros(og.E)
+    L = lib()
+    L.orc_stage_gradients.argtypes = [ctypes.c_void_p] * 4
+    _check(L.orc_stage_gradients(ctypes.byref(og.c), _p(cls), _p(dm), _p(out)))
+    return out

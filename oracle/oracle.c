@@ -871,3 +871,29 @@ int orc_timing_loss(const orc_graph* g, const double* x, const double* y, const 
   if (loss) *loss = lambda_rc * L;
   return 0;
 }
+
+/* ------------------------------------------------------------------------- */
+/* NEXT 3: INSTA-Size stage gradients: "the timing    */
+/* gradient of each stage (i.e., the gradient sum of a cell arc and its       */
+/* driving net arc)".  Reading R22: the stage of a cell arc e_c = (p -> o) is  */
+/* e_c plus the single net arc into p when p has exactly one fanin arc and it  */
+/* is a net arc; stage_grad[e_c] = sum_rf d_mean[e_c][rf] + sum_rf            */
+/* d_mean[e_n][rf]; 0 for net arcs.  arc_class: 0 net, 1 cell (caller order). */
+/* ------------------------------------------------------------------------- */
+int orc_stage_gradients(const orc_graph* g, const uint8_t* arc_class, const double* d_mean, double* out) {
+  if (!g || !arc_class || !d_mean || !out) return 1;
+  int32_t N = g->num_pins;
+  int32_t* nin = calloc((size_t)N + 1, sizeof(int32_t));
+  int64_t* in_arc = malloc(sizeof(int64_t) * ((size_t)N + 1));
+  for (int32_t p = 0; p < N; ++p) in_arc[p] = -1;
+  for (int64_t e = 0; e < g->num_arcs; ++e) { nin[g->arc_to[e]]++; in_arc[g->arc_to[e]] = e; }
+  for (int64_t e = 0; e < g->num_arcs; ++e) {
+    if (arc_class[e] != 1) { out[e] = 0.0; continue; }
+    double s = d_mean[2 * e] + d_mean[2 * e + 1];
+    int32_t p = g->arc_from[e];
+    if (nin[p] == 1 && arc_class[in_arc[p]] == 0) s += d_mean[2 * in_arc[p]] + d_mean[2 * in_arc[p] + 1];
+    out[e] = s;
+  }
+  free(nin); free(in_arc);
+  return 0;
+}

@@ -102,6 +102,9 @@ int orc_clark_backward(const orc_graph* g, double n_sigma, const double* dslack,
 int orc_timing_loss(const orc_graph* g, const double* x, const double* y, const double* w, double lambda_rc,
                     double* loss, double* gx, double* gy);
 
+/* NEXT 3: INSTA-Size stage gradients (reading R22), out[E] caller order. */
+int orc_stage_gradients(const orc_graph* g, const uint8_t* arc_class, const double* d_mean, double* out);
+
 #ifdef __cplusplus
 }
 #endif

@@ -17,7 +17,7 @@ import numpy as np
 from . import _capi
 from ._capi import InstaError, check
 
-__all__ = ["Graph", "Summary", "InstaError", "levelize", "version"]
+__all__ = ["Graph", "Summary", "InstaError", "levelize", "version", "grad_norm_ratio"]
 
 
 @dataclasses.dataclass
@@ -57,6 +57,18 @@ def levelize(num_pins: int, arc_from, arc_to) -> dict:
                              _ptr(out["fanin_ptr"]), _ptr(out["fanin_arc"]), _ptr(out["fanout_ptr"]),
                              _ptr(out["fanout_arc"]), ctypes.byref(nl)), "insta_levelize")
     out["num_levels"] = int(nl.value)
+    return out
+
+
+def grad_norm_ratio(a, b, stream=None):
+    """insta_grad_norm_ratio (Eq 8): ||a|| / ||b|| of two float32 device tensors, as a float64 device scalar."""
+    import torch
+    a = a.contiguous().float()
+    b = b.contiguous().float()
+    out = torch.empty(1, dtype=torch.float64, device=a.device)
+    st = ctypes.c_void_p((stream or torch.cuda.current_stream(a.device)).cuda_stream)
+    check(_capi.load().insta_grad_norm_ratio(int(a.numel()), _dptr(a), _dptr(b), _dptr(out), st),
+          "insta_grad_norm_ratio")
     return out
 
 
@@ -260,6 +272,38 @@ class Graph:
                                             self._st(stream)), "insta_clark_backward")
         outs = (d_mean,) + ((d_sig,) if want_sigma else ()) + ((d_src,) if want_src else ())
         return outs if len(outs) > 1 else d_mean
+
+    # ------------------------------------------------------------------ INSTA-Size steps
+    def stage_gradients(self, d_mean, stream=None):
+        """insta_stage_gradients: float32[E] stage gradient per cell arc (0 for net arcs)."""
+        t = self._torch
+        dm = t.as_tensor(d_mean, dtype=t.float32, device=self.device).contiguous()
+        out = t.empty(self.num_arcs, dtype=t.float32, device=self.device)
+        check(self.lib.insta_stage_gradients(self._h, _dptr(dm), _dptr(out), self._st(stream)), "insta_stage_gradients")
+        return out
+
+    def select_stages(self, stage_grad, threshold: float = 0.0, stream=None):
+        """insta_select_stages: int32 device tensor of cell arc ids with grad < -threshold, most negative first."""
+        t = self._torch
+        arcs = t.empty(max(self.num_arcs, 1), dtype=t.int32, device=self.device)
+        cnt = t.zeros(1, dtype=t.int32, device=self.device)
+        check(self.lib.insta_select_stages(self._h, _dptr(stage_grad), float(threshold), _dptr(arcs), _dptr(cnt),
+                                           self._st(stream)), "insta_select_stages")
+        return arcs[: int(cnt.item())]
+
+    # ------------------------------------------------------------------ INSTA-Place Eq 7 (SURVEY §8(f) NEXT 4)
+    def timing_loss(self, pin_x, pin_y, arc_w, lambda_rc: float = 1.0, want_grad: bool = True, stream=None):
+        """insta_timing_loss: (L float64 device scalar, grad_x float32[N], grad_y float32[N]) of Eq 7."""
+        t = self._torch
+        x = t.as_tensor(pin_x, dtype=t.float32, device=self.device).contiguous()
+        y = t.as_tensor(pin_y, dtype=t.float32, device=self.device).contiguous()
+        w = t.as_tensor(arc_w, dtype=t.float32, device=self.device).contiguous()
+        L = t.empty(1, dtype=t.float64, device=self.device)
+        gx = t.empty(self.num_pins, dtype=t.float32, device=self.device) if want_grad else None
+        gy = t.empty(self.num_pins, dtype=t.float32, device=self.device) if want_grad else None
+        check(self.lib.insta_timing_loss(self._h, _dptr(x), _dptr(y), _dptr(w), float(lambda_rc), _dptr(L), _dptr(gx),
+                                         _dptr(gy), self._st(stream)), "insta_timing_loss")
+        return L, gx, gy
 
     def forward_batch(self, scenarios, tau: float = 0.0, want_grad: bool = False, summaries=None, d_mean_sum=None,
                       stream=None):

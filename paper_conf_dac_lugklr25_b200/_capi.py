@@ -79,6 +79,10 @@ SIGNATURES = {
     "insta_clark_forward": (ctypes.c_int, [c_vp, ctypes.c_float, c_vp, ctypes.POINTER(insta_summary)]),
     "insta_clark_results": (ctypes.c_int, [c_vp, c_vp, c_vp, c_vp, c_vp, c_vp, c_vp]),
     "insta_clark_backward": (ctypes.c_int, [c_vp, c_vp, c_vp, c_vp, c_vp, c_vp]),
+    "insta_stage_gradients": (ctypes.c_int, [c_vp, c_vp, c_vp, c_vp]),
+    "insta_select_stages": (ctypes.c_int, [c_vp, c_vp, ctypes.c_float, c_vp, c_vp, c_vp]),
+    "insta_timing_loss": (ctypes.c_int, [c_vp, c_vp, c_vp, c_vp, ctypes.c_float, c_vp, c_vp, c_vp, c_vp]),
+    "insta_grad_norm_ratio": (ctypes.c_int, [ctypes.c_int64, c_vp, c_vp, c_vp, c_vp]),
     "insta_last_error": (ctypes.c_char_p, []),
     "insta_version": (ctypes.c_char_p, []),
 }

@@ -65,7 +65,7 @@ void free_graph(insta::DevGraph& d) {
                   d.arc_head,  d.ext_h,     d.tk_q,      d.tk_sp,      d.tk_slack,  d.tk_star,
                   d.tk_summary, d.rat_ptr,  d.rat_sp,    d.rat_val,   d.tk_list,
                   d.cl_mv,     d.cl_pre,    d.cl_g,      d.cl_fo_ptr,  d.cl_fo_q,   d.cl_slack,
-                  d.cl_rf,     d.cl_summary, d.cl_hv_list, d.cl_hv_of, d.cl_hv_sum};
+                  d.cl_rf,     d.cl_summary, d.cl_hv_list, d.cl_hv_of, d.cl_hv_sum, d.tl_partials, d.sz_tmp};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   if (d.b_stage_h) cudaFreeHost(d.b_stage_h);
@@ -721,6 +721,56 @@ insta_status insta_clark_backward(insta_graph* g, const float* ep_seed, float* d
   cudaSetDevice(d.device);
   int err = insta::launch_clark_backward(d, ep_seed, d_arc_mean, d_arc_sigma, d_src, cuda_stream);
   if (err) return cuda_fail(err, "clark_backward");
+  return INSTA_OK;
+}
+
+// ---------------------------------------------------------------------------
+// INSTA-Place timing objective, Eq 7 / Eq 8
+// ---------------------------------------------------------------------------
+insta_status insta_timing_loss(insta_graph* g, const float* pin_x, const float* pin_y, const float* arc_w,
+                               float lambda_rc, double* loss, float* grad_x, float* grad_y, void* cuda_stream) {
+  if (!g) return fail(INSTA_E_ARG, "timing_loss: NULL graph");
+  insta::DevGraph& d = g->d;
+  if (d.n > 0 && (!pin_x || !pin_y)) return fail(INSTA_E_ARG, "timing_loss: NULL pin positions");
+  if (d.e > 0 && !arc_w) return fail(INSTA_E_ARG, "timing_loss: NULL arc weights");
+  if ((grad_x == nullptr) != (grad_y == nullptr)) return fail(INSTA_E_ARG, "timing_loss: grad_x and grad_y go together");
+  if (!std::isfinite(lambda_rc)) return fail(INSTA_E_ARG, "timing_loss: lambda_rc must be finite");
+  cudaSetDevice(d.device);
+  int err = insta::launch_timing_loss(d, pin_x, pin_y, arc_w, lambda_rc, loss, grad_x, grad_y, cuda_stream);
+  if (err) return cuda_fail(err, "timing_loss");
+  return INSTA_OK;
+}
+
+insta_status insta_grad_norm_ratio(int64_t n, const float* a, const float* b, double* out, void* cuda_stream) {
+  if (n < 0 || !out || (n > 0 && (!a || !b))) return fail(INSTA_E_ARG, "grad_norm_ratio: bad arguments");
+  int err = insta::launch_norm_ratio(n, a, b, out, cuda_stream);
+  if (err) return cuda_fail(err, "grad_norm_ratio");
+  return INSTA_OK;
+}
+
+// ---------------------------------------------------------------------------
+// INSTA-Size device steps
+// ---------------------------------------------------------------------------
+insta_status insta_stage_gradients(insta_graph* g, const float* d_arc_mean, float* stage_grad, void* cuda_stream) {
+  if (!g) return fail(INSTA_E_ARG, "stage_gradients: NULL graph");
+  insta::DevGraph& d = g->d;
+  if (d.e > 0 && (!d_arc_mean || !stage_grad)) return fail(INSTA_E_ARG, "stage_gradients: NULL array");
+  if (d.e > 0 && !d.arc_class) return fail(INSTA_E_ARG, "stage_gradients: the graph has no arc_class");
+  cudaSetDevice(d.device);
+  int err = insta::launch_stage_gradients(d, d_arc_mean, stage_grad, cuda_stream);
+  if (err) return cuda_fail(err, "stage_gradients");
+  return INSTA_OK;
+}
+
+insta_status insta_select_stages(insta_graph* g, const float* stage_grad, float threshold, int32_t* out_arcs,
+                                 int32_t* out_count, void* cuda_stream) {
+  if (!g) return fail(INSTA_E_ARG, "select_stages: NULL graph");
+  insta::DevGraph& d = g->d;
+  if (!out_count || (d.e > 0 && (!stage_grad || !out_arcs))) return fail(INSTA_E_ARG, "select_stages: NULL array");
+  if (!std::isfinite(threshold) || threshold < 0.f) return fail(INSTA_E_ARG, "select_stages: threshold must be >= 0");
+  cudaSetDevice(d.device);
+  int err = insta::launch_select_stages(d, stage_grad, threshold, out_arcs, out_count, cuda_stream);
+  if (err) return cuda_fail(err, "select_stages");
   return INSTA_OK;
 }
 

@@ -320,12 +320,13 @@ __global__ void cl_bwd_kernel(ClParams P) {
 // --------------------------------------------------------------------------
 // host launchers
 // --------------------------------------------------------------------------
-static int ensure_clark(DevGraph& g) {
-  if (g.cl_mv) return 0;
-  // full fanout rows with the fanin position of every fanout arc (heavy drivers included)
+// Full fanout rows (heavy drivers included) as words fanin position << 2 |
+// unateness, and the wide-fanout pins per level; shared by the Clark backward
+// and the Eq 7 gradient (place.cu).
+int ensure_fanout_words(DevGraph& g) {
+  if (g.cl_fo_q) return 0;
   const HostLevels& h = g.host;
   std::vector<int32_t> fo_q(size_t(std::max<int64_t>(g.e, 1)));
-  // fanout word: fanin position << 2 | unateness of the arc (fin_src bits 30-31)
   std::vector<int32_t> fsrc(size_t(std::max<int64_t>(g.e, 1)));
   if (g.e > 0) {
     cudaError_t e0 = cudaMemcpy(fsrc.data(), g.fin_src, sizeof(int32_t) * size_t(g.e), cudaMemcpyDeviceToHost);
@@ -348,24 +349,32 @@ static int ensure_clark(DevGraph& g) {
       }
   }
   g.cl_hv_ptr[g.num_levels] = int32_t(hv_list.size());
-  cudaError_t e = cudaMalloc(&g.cl_mv, sizeof(double2) * 2 * size_t(std::max(g.n, 1)));
-  if (e == cudaSuccess) e = cudaMalloc(&g.cl_hv_list, sizeof(int32_t) * std::max<size_t>(hv_list.size(), 1));
+  cudaError_t e = cudaMalloc(&g.cl_hv_list, sizeof(int32_t) * std::max<size_t>(hv_list.size(), 1));
   if (e == cudaSuccess) e = cudaMalloc(&g.cl_hv_of, sizeof(int32_t) * hv_of.size());
   if (e == cudaSuccess) e = cudaMalloc(&g.cl_hv_sum, sizeof(double2) * 2 * std::max<size_t>(hv_list.size(), 1));
   if (e == cudaSuccess && !hv_list.empty())
     e = cudaMemcpy(g.cl_hv_list, hv_list.data(), sizeof(int32_t) * hv_list.size(), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(g.cl_hv_of, hv_of.data(), sizeof(int32_t) * hv_of.size(), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMalloc(&g.cl_fo_ptr, sizeof(int32_t) * (size_t(g.n) + 1));
+  if (e == cudaSuccess)
+    e = cudaMemcpy(g.cl_fo_ptr, h.fanout_ptr.data(), sizeof(int32_t) * (size_t(g.n) + 1), cudaMemcpyHostToDevice);
+  int32_t* fq = nullptr;
+  if (e == cudaSuccess) e = cudaMalloc(&fq, sizeof(int32_t) * fo_q.size());
+  if (e == cudaSuccess) e = cudaMemcpy(fq, fo_q.data(), sizeof(int32_t) * fo_q.size(), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) g.cl_fo_q = fq;
+  return int(e);
+}
+
+static int ensure_clark(DevGraph& g) {
+  if (g.cl_mv) return 0;
+  int err = ensure_fanout_words(g);
+  if (err) return err;
+  cudaError_t e = cudaMalloc(&g.cl_mv, sizeof(double2) * 2 * size_t(std::max(g.n, 1)));
   if (e == cudaSuccess) e = cudaMalloc(&g.cl_pre, sizeof(double2) * 4 * size_t(std::max<int64_t>(g.e, 1)));
   if (e == cudaSuccess) e = cudaMalloc(&g.cl_g, sizeof(double2) * 4 * size_t(std::max<int64_t>(g.e, 1)));
-  if (e == cudaSuccess) e = cudaMalloc(&g.cl_fo_ptr, sizeof(int32_t) * (size_t(g.n) + 1));
-  if (e == cudaSuccess) e = cudaMalloc(&g.cl_fo_q, sizeof(int32_t) * fo_q.size());
   if (e == cudaSuccess) e = cudaMalloc(&g.cl_slack, sizeof(double) * size_t(std::max(g.num_ep, 1)));
   if (e == cudaSuccess) e = cudaMalloc(&g.cl_rf, size_t(std::max(g.num_ep, 1)));
   if (e == cudaSuccess) e = cudaMalloc(&g.cl_summary, 4 * sizeof(double));
-  if (e == cudaSuccess)
-    e = cudaMemcpy(g.cl_fo_ptr, h.fanout_ptr.data(), sizeof(int32_t) * (size_t(g.n) + 1), cudaMemcpyHostToDevice);
-  if (e == cudaSuccess)
-    e = cudaMemcpy(g.cl_fo_q, fo_q.data(), sizeof(int32_t) * fo_q.size(), cudaMemcpyHostToDevice);
   return int(e);
 }
 

@@ -244,6 +244,12 @@ struct DevGraph {
   int32_t* cl_hv_of = nullptr;     // [n] index into cl_hv_list, -1 = narrow
   void* cl_hv_sum = nullptr;       // double2 [wide][2]
   std::vector<int32_t> cl_hv_ptr;  // [L+1]
+  // INSTA-Size selection scratch (size.cu)
+  void* sz_tmp = nullptr;
+  size_t sz_cap = 0;
+  // Eq 7 timing objective (place.cu)
+  double* tl_partials = nullptr;
+  int32_t tl_cap = 0;
   // CPPR required times per (endpoint, startpoint) (insta_set_cppr_rat)
   int32_t* rat_ptr = nullptr;      // [P+1] or NULL (no table)
   int32_t* rat_sp = nullptr;       // [M] canonical startpoints, ascending within a row
@@ -319,6 +325,12 @@ int topk_stats(unsigned long long* out);
 int launch_clark_forward(DevGraph& g, float n_sigma, void* stream);
 int launch_clark_backward(DevGraph& g, const float* ep_seed, float* d_mean, float* d_sigma, float* d_src,
                           void* stream);
+int launch_timing_loss(DevGraph& g, const float* x, const float* y, const float* w, float lambda_rc, double* loss,
+                       float* gx, float* gy, void* stream);
+int launch_stage_gradients(DevGraph& g, const float* d_mean, float* out, void* stream);
+int launch_select_stages(DevGraph& g, const float* grad, float threshold, int32_t* out_arcs, int32_t* out_count,
+                         void* stream);
+int launch_norm_ratio(int64_t n, const float* a, const float* b, double* out, void* stream);
 int launch_clark_export(DevGraph& g, float* A, float* mean, float* sigma, float* slack, uint8_t* rf, void* stream);
 int launch_topk_export(DevGraph& g, float* A, float* mean, float* sigma, int32_t* sp, void* stream);
 int launch_topk_export_slack(DevGraph& g, float* slack, int32_t* sp_star, uint8_t* rf_star, int32_t* k_star,

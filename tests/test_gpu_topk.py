@@ -7,8 +7,8 @@
   identical except where the oracle's own entries are within 1e-3 ps of each
   other (fp32 sqrt vs fp64 may swap them), CPPR slack / TNS within tolerance;
 * K = 1 equals the GPU hard forward (insta_forward, tau = 0);
-* C4 at full size: queue invariants on the device (descending, unique
-  startpoints, startpoints are sources, entry 0 >= the hard arrival).
+* C4 at full size: K = 1 equals the hard forward; K = 8 queue invariants on
+  the device (descending, unique startpoints, startpoints are sources).
 """
 import types
 
@@ -160,6 +160,10 @@ def test_topk_c4_invariants():
     G = insta.Graph(g)
     G.forward(NS, 0.0)
     A_hard = G.arrivals()[0]
+    G.topk_forward(1, NS)                      # K = 1 is the hard merge at full size
+    A1 = G.topk_queues()["A"][:, :, 0]
+    assert torch.allclose(A1, A_hard, rtol=1e-6, atol=1e-4)
+    del A1
     K = 8
     G.set_cppr_rat(*synth.cppr_rat_table(g))
     G.topk_forward(K, NS)
@@ -178,7 +182,7 @@ def test_topk_c4_invariants():
     indeg = np.bincount(g.arc_to, minlength=g.num_pins)
     is_src = torch.as_tensor(indeg == 0, device=sp.device)
     assert is_src[sp[valid].long()].all()
-    # entry 0 collects at least the hard (K = 1) arrival
-    assert (A[:, :, 0] >= A_hard - 1e-4 * A_hard.abs() - 1e-3).all()
+    # (entry 0 is NOT bounded below by the hard arrival when sigma > 0: the hard state of a pin need not be
+    # its startpoint's best-key entry, and sqrt(var + std^2) can reorder them downstream)
     assert summ.num_violations > 0 and np.isfinite(summ.tns)
     G.close()
