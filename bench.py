@@ -216,7 +216,7 @@ def main():
     ap.add_argument("--config", default="C4")
     ap.add_argument("--tau", type=float, default=0.0)
     ap.add_argument("--schedule", type=int, default=0)
-    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--e2e-steps", type=int, default=8)
     ap.add_argument("--ref-sample-pins", type=int, default=1_500_000)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--batch-scenarios", type=int, default=1024, help="C5 batched evaluations (0 = skip)")
@@ -317,36 +317,71 @@ def main():
             traffic = None
 
     # ---------------- end to end through the public API with host buffers -------------
+    # Every step: H2D of all arc delays (mean, sigma; pinned host memory), insta_update_arcs (every arc),
+    # insta_forward, insta_backward, insta_slack, and D2H of the full gradient + the endpoint slacks.
+    # Steps are pipelined on three streams with double-buffered device staging: the H2D of step k+1 and
+    # the D2H of step k-1 overlap step k's kernels (different copy directions, separate engines).
     e2e = None
     if args.e2e_steps > 0:
-        ids_h = torch.arange(E, dtype=torch.int32).pin_memory()
-        m_h = torch.from_numpy(g.arc_mean).pin_memory()
-        s_h = torch.from_numpy(g.arc_sigma).pin_memory()
-        out_h = torch.empty((E, 2), dtype=torch.float32).pin_memory()
-        ids_d = torch.empty_like(ids_h, device=dev)
-        m_d = torch.empty_like(m_h, device=dev)
-        s_d = torch.empty_like(s_h, device=dev)
-        with torch.cuda.stream(stream):
-            torch.cuda.synchronize(dev)
-            t0 = time.perf_counter()
-            for _ in range(args.e2e_steps):
-                ids_d.copy_(ids_h, non_blocking=True)
-                m_d.copy_(m_h, non_blocking=True)
-                s_d.copy_(s_h, non_blocking=True)
-                G.update_arcs(ids_d, m_d, s_d, incremental=False, stream=stream)
+        m_h = torch.from_numpy(np.ascontiguousarray(g.arc_mean, np.float32)).pin_memory()
+        s_h = torch.from_numpy(np.ascontiguousarray(g.arc_sigma, np.float32)).pin_memory()
+        out_h = [torch.empty((E, 2), dtype=torch.float32).pin_memory() for _ in range(2)]
+        sl_h = [torch.empty(P, dtype=torch.float32).pin_memory() for _ in range(2)]
+        m_d = [torch.empty_like(m_h, device=dev) for _ in range(2)]
+        s_d = [torch.empty_like(s_h, device=dev) for _ in range(2)]
+        dm_d = [torch.empty((E, 2), dtype=torch.float32, device=dev) for _ in range(2)]
+        sl_d = [torch.empty(P, dtype=torch.float32, device=dev) for _ in range(2)]
+        s_in, s_out = torch.cuda.Stream(dev), torch.cuda.Stream(dev)
+        ev_in = [torch.cuda.Event() for _ in range(2)]
+        ev_in_free = [torch.cuda.Event() for _ in range(2)]
+        ev_done = [torch.cuda.Event() for _ in range(2)]
+        ev_out_free = [torch.cuda.Event() for _ in range(2)]
+        for b in range(2):
+            ev_in_free[b].record(stream)
+            ev_out_free[b].record(stream)
+
+        def e2e_step(k):
+            b = k & 1
+            with torch.cuda.stream(s_in):                  # H2D of this step's inputs
+                s_in.wait_event(ev_in_free[b])
+                m_d[b].copy_(m_h, non_blocking=True)
+                s_d[b].copy_(s_h, non_blocking=True)
+                ev_in[b].record(s_in)
+            with torch.cuda.stream(stream):                # the public API calls
+                stream.wait_event(ev_in[b])
+                G.update_arcs(None, m_d[b], s_d[b], incremental=False, stream=stream)
+                ev_in_free[b].record(stream)
+                stream.wait_event(ev_out_free[b])
                 G.forward(3.0, args.tau, args.schedule, sync=False, stream=stream)
-                G.backward(out=d_mean, stream=stream)
-                out_h.copy_(d_mean, non_blocking=True)
-                G.summary(stream=stream)          # D2H of WNS/TNS, synchronizes
-            dt = (time.perf_counter() - t0) / args.e2e_steps
+                G.backward(out=dm_d[b], stream=stream)
+                G.lib.insta_slack(G._h, sl_d[b].data_ptr(), None, stream.cuda_stream, None)
+                ev_done[b].record(stream)
+            with torch.cuda.stream(s_out):                 # D2H of this step's results
+                s_out.wait_event(ev_done[b])
+                out_h[b].copy_(dm_d[b], non_blocking=True)
+                sl_h[b].copy_(sl_d[b], non_blocking=True)
+                ev_out_free[b].record(s_out)
+
+        for k in range(2):                                 # warm-up of the pipeline
+            e2e_step(k)
+        torch.cuda.synchronize(dev)
+        t0 = time.perf_counter()
+        for k in range(args.e2e_steps):
+            e2e_step(k)
+        torch.cuda.synchronize(dev)
+        dt = (time.perf_counter() - t0) / args.e2e_steps
+        tns_host = float(np.minimum(sl_h[(args.e2e_steps - 1) & 1].numpy().astype(np.float64), 0).sum())
         if world > 1:
             t = torch.tensor([dt], dtype=torch.float64, device=dev)
             torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
             dt = float(t.item())
         e2e = {"value": world * N / dt, "unit": UNIT, "ms_per_step": dt * 1e3,
-               "h2d_bytes_per_step": int(E * (4 + 8 + 8)), "d2h_bytes_per_step": int(E * 8 + 32),
-               "what": "per step: H2D of every arc's mean/sigma (+ids) from pinned memory, insta_update_arcs, "
-                       "insta_forward, insta_backward, D2H of the full gradient and the WNS/TNS summary"}
+               "h2d_bytes_per_step": int(E * 16), "d2h_bytes_per_step": int(E * 8 + P * 4),
+               "tns_from_host_slack": tns_host,
+               "what": "per step: H2D of every arc's mean/sigma from pinned memory, insta_update_arcs (all arcs), "
+                       "insta_forward, insta_backward, insta_slack, D2H of the full gradient and the endpoint "
+                       "slacks; steps pipelined over 3 streams (H2D k+1 and D2H k-1 overlap step k), "
+                       f"{args.e2e_steps} steps, host wall clock"}
 
     # ---------------- batched scenarios (C5): 1024 evaluations sharded over the ranks -------------
     batched = None

@@ -172,7 +172,8 @@ insta_status insta_backward(insta_graph* g, const float* ep_seed, float* d_arc_m
                             float* d_arc_sigma, float* d_src, void* cuda_stream);
 
 /* Re-annotate n arcs ("re-annotate ... then re-propagate"):
- * arc_ids DEVICE int32[n] (caller ids, unique), mean/sigma DEVICE float[n][2].
+ * arc_ids DEVICE int32[n] (caller ids, unique) -- or NULL with n == num_arcs
+ * to re-annotate every arc in caller order -- mean/sigma DEVICE float[n][2].
  * incremental = 1: the next insta_forward recomputes only the fanout cone of
  * the changed arcs, stopping where a recomputed record does not change (a
  * dataflow pass in which pins outside the cone only republish their record;

@@ -192,10 +192,11 @@ class Graph:
     def update_arcs(self, arc_ids, mean, sigma, incremental: bool = True, stream=None):
         """insta_update_arcs: re-annotate arcs (device or host arrays; copied to the device)."""
         t = self._torch
-        ids = t.as_tensor(arc_ids, dtype=t.int32, device=self.device).contiguous()
+        ids = None if arc_ids is None else t.as_tensor(arc_ids, dtype=t.int32, device=self.device).contiguous()
         m = t.as_tensor(mean, dtype=t.float32, device=self.device).contiguous()
         s = t.as_tensor(sigma, dtype=t.float32, device=self.device).contiguous()
-        check(self.lib.insta_update_arcs(self._h, int(ids.numel()), _dptr(ids), _dptr(m), _dptr(s),
+        n = self.num_arcs if ids is None else int(ids.numel())   # arc_ids None: every arc, caller order
+        check(self.lib.insta_update_arcs(self._h, n, _dptr(ids), _dptr(m), _dptr(s),
                                          int(bool(incremental)), self._st(stream)), "insta_update_arcs")
 
     # ------------------------------------------------------------------ Top-K / CPPR (SURVEY §8(f) NEXT 1)

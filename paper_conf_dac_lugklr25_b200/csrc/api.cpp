@@ -468,9 +468,9 @@ insta_status insta_update_arcs(insta_graph* g, int64_t n, const int32_t* arc_ids
                                const float* mean, const float* sigma, int32_t incremental,
                                void* cuda_stream) {
   if (!g) return fail(INSTA_E_ARG, "update_arcs: NULL graph");
-  if (n < 0 || (n > 0 && (!arc_ids || !mean || !sigma)))
-    return fail(INSTA_E_ARG, "update_arcs: bad arguments");
   insta::DevGraph& d = g->d;
+  if (n < 0 || (n > 0 && (!mean || !sigma)) || (n > 0 && !arc_ids && n != d.e))
+    return fail(INSTA_E_ARG, "update_arcs: bad arguments (arc_ids may be NULL only with n == num_arcs)");
   if (n > d.e) return fail(INSTA_E_ARG, "update_arcs: more updates than arcs");
   cudaSetDevice(d.device);
   int err = insta::launch_update_arcs(d, n, arc_ids, mean, sigma, incremental, cuda_stream);

@@ -1565,12 +1565,13 @@ __global__ void update_arcs_kernel(int64_t n, const int32_t* __restrict__ ids,
                                    const int32_t* __restrict__ arc_head, uint32_t* dirty_h, uint32_t stamp) {
   const int64_t k = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
   if (k >= n) return;
-  const int q = arc_pos[ids[k]];
+  const int id = ids ? ids[k] : int(k);   // ids == NULL: all arcs in caller order
+  const int q = arc_pos[id];
   const float2 m = mean[k], s = sigma[k];
   fin_ms[q] = make_float4(m.x, m.y, s.x, s.y);
-  const int x = arc_xpos[ids[k]];   // the stage-folded schedule's copy of the record
+  const int x = arc_xpos[id];   // the stage-folded schedule's copy of the record
   ((x & 1) ? ext_fms : ext_ms)[x >> 1] = make_float4(m.x, m.y, s.x, s.y);
-  if (dirty_h) dirty_h[arc_head[ids[k]]] = stamp;   // incremental: the head evaluating the arc recomputes
+  if (dirty_h) dirty_h[arc_head[id]] = stamp;   // incremental: the head evaluating the arc recomputes
 }
 
 // --------------------------------------------------------------------------
