@@ -427,6 +427,8 @@ def main():
     if args.topk > 0:
         G.set_cppr_rat(*synth.cppr_rat_table(g))
         K = args.topk
+        torch.cuda.synchronize(dev)
+        free0 = torch.cuda.mem_get_info(dev)[0]
         with torch.cuda.stream(stream):
             for _ in range(2):
                 G.topk_forward(K, 3.0, stream=stream)
@@ -444,13 +446,14 @@ def main():
             stream.synchronize()
             ts, _, _ = G.topk_slack(stream=stream)
         tf, tsl = t0.elapsed_time(t1) / nk, t1.elapsed_time(t2) / nk
+        tk_mem = (free0 - torch.cuda.mem_get_info(dev)[0]) / 1e9   # queues + slack + lists (library cudaMalloc)
         tk_bytes = topk_bytes(g, K)
         topk = {"workload": f"{cfg.name}, Top-K = {K} unique-startpoint queues (Alg 1 + Alg 2) + CPPR slack against "
                             f"a per-(endpoint, startpoint) RAT table", "K": K, "fwd_ms": tf, "slack_ms": tsl,
                 "pins_per_s": N / ((tf + tsl) * 1e-3), "alg_bytes": tk_bytes, "gbs": tk_bytes / (tf * 1e-3) / 1e9,
-                "tns": ts.tns, "wns": ts.wns, "violations": ts.num_violations,
-                "paper_context": "PAPER.md Table I (L184-193): block-1 (15M pins) at TopK=32 in 0.39 s on 1x A100 "
-                                 "(incl. its own slack); other hardware, other design"}
+                "tns": ts.tns, "wns": ts.wns, "violations": ts.num_violations, "device_memory_gb": tk_mem,
+                "paper_context": "PAPER.md Table I (L184-193): block-1 (15M pins) at TopK=32 in 0.39 s and 21.13 GB on "
+                                 "1x A100 (incl. its own slack); other hardware, other design"}
 
     # ---------------- Clark moment-matching merge -------------
     clark = None

@@ -35,6 +35,7 @@ def test_no_arcs_endpoint_is_startpoint():
     assert G.clark_backward().numel() == 0
     L, gx, gy = G.timing_loss(np.zeros(3), np.zeros(3), np.zeros(0))
     assert float(L.item()) == 0.0 and (gx.cpu() == 0).all()
+    G.forward(3.0, 0.0)
     d = G.backward()
     assert G.select_stages(G.stage_gradients(d)).numel() == 0
     G.close()
