@@ -37,7 +37,7 @@
 
 // resident blocks per SM the level kernel is compiled for (register budget)
 #ifndef TK_MINB
-#define TK_MINB 4
+#define TK_MINB 6
 #endif
 
 namespace insta {
