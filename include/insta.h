@@ -332,6 +332,11 @@ insta_status insta_grad_norm_ratio(int64_t n, const float* a, const float* b, do
  * recomputed with it).  Synchronizes. */
 insta_status insta_last_forward_stats(insta_graph* g, int64_t* pins_recomputed);
 
+/* Debug builds only (compiled with -DTK_STATS): histogram of the Top-K merge
+ * batches by number of surviving candidates (33 counters, HOST output).
+ * Returns 0 on success, -1 in normal builds (no counters compiled in). */
+int insta_debug_topk_stats(unsigned long long* out);
+
 /* Thread-local message for the last non-OK status ("" if none). */
 const char* insta_last_error(void);
 

@@ -83,6 +83,7 @@ SIGNATURES = {
     "insta_select_stages": (ctypes.c_int, [c_vp, c_vp, ctypes.c_float, c_vp, c_vp, c_vp]),
     "insta_timing_loss": (ctypes.c_int, [c_vp, c_vp, c_vp, c_vp, ctypes.c_float, c_vp, c_vp, c_vp, c_vp]),
     "insta_grad_norm_ratio": (ctypes.c_int, [ctypes.c_int64, c_vp, c_vp, c_vp, c_vp]),
+    "insta_debug_topk_stats": (ctypes.c_int, [c_vp]),
     "insta_last_error": (ctypes.c_char_p, []),
     "insta_version": (ctypes.c_char_p, []),
 }
