@@ -315,8 +315,14 @@ __global__ void __launch_bounds__(kThreads, 1) fwdb_kernel(BParams P) {
               awaitb(P, src, s, r);
             }
           };
-          const RfOut R = pin_rf_b<kLSE>(P, ns, 0, nf, arc);
-          const RfOut F = pin_rf_b<kLSE>(P, ns, 1, nf, arc);
+          RfOut R, F;
+          if (nf <= kRegArcsB) {   // register window: unrolled merge, no run-time source selection
+            R = merge_rf_unrolled<kLSE, kRegArcsB>(ns, double(P.tau), P.inv_tau, 0, nf, arc);
+            F = merge_rf_unrolled<kLSE, kRegArcsB>(ns, double(P.tau), P.inv_tau, 1, nf, arc);
+          } else {
+            R = pin_rf_b<kLSE>(P, ns, 0, nf, arc);
+            F = pin_rf_b<kLSE>(P, ns, 1, nf, arc);
+          }
           storeb(P, i, s, R.mu, F.mu, R.var, F.var);
           if (!P.store_aux) {
           } else if (!kLSE) {

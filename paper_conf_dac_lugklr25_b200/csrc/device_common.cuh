@@ -280,6 +280,73 @@ __device__ __forceinline__ RfOut merge_rf(double ns, double tau, double inv_tau,
   return o;
 }
 
+// merge_rf for nf <= NMAX with the candidate loop unrolled (arc(k) is called
+// with compile-time k, so register-held source words need no run-time
+// selection) and the winner kept from the scan instead of re-evaluated: the
+// same operations in the same order as merge_rf, hence bit-identical.
+template <bool kLSE, int NMAX, class ArcFn>
+__device__ __forceinline__ RfOut merge_rf_unrolled(double ns, double tau, double inv_tau, int rf, int nf, ArcFn&& arc) {
+  double best = 0.0;
+  int bk = -1, bs = 0;
+  Cand win;
+  win.mu = win.var = win.A = 0.0;
+  win.sig = 0.f;
+#pragma unroll
+  for (int k = 0; k < NMAX; ++k) {
+    if (k < nf) {
+      int32_t w;
+      float4 ms;
+      Raw r;
+      arc(k, w, ms, r);
+      const Gath st = unpack(r);
+      const int u = int(uint32_t(w) >> kUnateShiftC);
+      const int s0 = src_tr(rf, u, 0);
+      const Cand c0 = make_cand(st, ms, rf, s0, ns);
+      if (bk < 0 || c0.A > best) {   // Alg 2 l.4: replace only if strictly greater
+        best = c0.A;
+        bk = k;
+        bs = s0;
+        win = c0;
+      }
+      if (u == 2) {
+        const Cand c1 = make_cand(st, ms, rf, rf ^ 1, ns);
+        if (c1.A > best) {
+          best = c1.A;
+          bk = k;
+          bs = rf ^ 1;
+          win = c1;
+        }
+      }
+    }
+  }
+  RfOut o;
+  o.mu = win.mu;
+  o.var = win.var;
+  o.sig = win.sig;
+  o.best = best;
+  o.win = bk | (bs << 15);
+  o.sum = 0.f;
+  if (kLSE) {
+    float sum = 0.f;
+#pragma unroll
+    for (int k = 0; k < NMAX; ++k) {
+      if (k < nf) {
+        int32_t w;
+        float4 ms;
+        Raw r;
+        arc(k, w, ms, r);
+        const Gath st = unpack(r);
+        const int u = int(uint32_t(w) >> kUnateShiftC);
+        sum += lse_w(make_cand(st, ms, rf, src_tr(rf, u, 0), ns).A, best, inv_tau);
+        if (u == 2) sum += lse_w(make_cand(st, ms, rf, rf ^ 1, ns).A, best, inv_tau);
+      }
+    }
+    o.sum = sum;
+    o.mu = lse_arrival(best, tau, sum) - ns * double(o.sig);
+  }
+  return o;
+}
+
 // Merge of a pin with exactly one fanin arc (source words st, unateness u,
 // record ms): the same operation sequence as merge_rf with nf = 1 -- scan
 // (a0, then a1 for a non-unate arc, strict ">"), winner, LSE sum 0 + w0
