@@ -100,7 +100,7 @@ __device__ __forceinline__ Raw ldb_raw(const BParams& P, int j, int s) {
 
 __device__ __forceinline__ void awaitb(const BParams& P, int j, int s, Raw& r) {
   while (!raw_ready(r, P.par)) {
-    __nanosleep(20);
+    INSTA_POLL_SLEEP();
     r = ldb_raw(P, j, s);
   }
 }
@@ -476,7 +476,7 @@ __device__ __forceinline__ float2 loadb_g(const BParams& P, int q, int s) {
   const float2* p = P.bg + size_t(q) * kLanes + s;
   ld2_u32(p, a, b);
   while (!g_ready(a, b, P.par)) {
-    __nanosleep(20);
+    INSTA_POLL_SLEEP();
     ld2_u32(p, a, b);
   }
   return make_float2(stripf(a), stripf(b));
@@ -600,7 +600,7 @@ __global__ void __launch_bounds__(kThreads, 1) bwdb_kernel(BParams P) {
             for (int j = 0; j < kPullChunk; ++j) {
               if (r + j < r1) {
                 while (!g_ready(va[j], vb[j], P.par)) {
-                  __nanosleep(20);
+                  INSTA_POLL_SLEEP();
                   ld2_u32(P.bg + size_t(qq[j]) * kLanes + s, va[j], vb[j]);
                 }
                 ax += stripf(va[j]);
@@ -615,7 +615,7 @@ __global__ void __launch_bounds__(kThreads, 1) bwdb_kernel(BParams P) {
             ld2_u64(acc, x, y);
             while (((long long)x + (kCountUnitB >> 1)) >> 44 != target ||
                    ((long long)y + (kCountUnitB >> 1)) >> 44 != target) {
-              __nanosleep(32);
+              INSTA_POLL_SLEEP();
               ld2_u64(acc, x, y);
             }
             asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %1};" ::"l"(acc), "l"(0ull) : "memory");

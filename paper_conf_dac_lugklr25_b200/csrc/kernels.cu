@@ -118,7 +118,7 @@ __device__ __forceinline__ Raw ld_state_raw(const KParams& P, int j) {
 __device__ __forceinline__ void await_raw(const KParams& P, int j, Raw& r) {
   if (P.mode == 2) {
     while (!raw_ready(r, P.par)) {
-      __nanosleep(20);
+      INSTA_POLL_SLEEP();
       r = ld_state_raw(P, j);
     }
   }
@@ -859,7 +859,7 @@ __device__ __forceinline__ float2 heavy_read(const KParams& P, int slot) {
   unsigned long long x, y;
   ld2_u64(P.heavy_acc + 2 * slot, x, y);
   while (heavy_count((long long)x) != target || heavy_count((long long)y) != target) {
-    __nanosleep(32);
+    INSTA_POLL_SLEEP();
     ld2_u64(P.heavy_acc + 2 * slot, x, y);
   }
   const long long vx = (long long)x - target * kCountUnit, vy = (long long)y - target * kCountUnit;
@@ -873,7 +873,7 @@ __device__ __forceinline__ float2 heavy_take(const KParams& P, int slot) {
   unsigned long long x, y;
   ld2_u64(P.heavy_acc + 2 * slot, x, y);
   while (heavy_count((long long)x) != target || heavy_count((long long)y) != target) {
-    __nanosleep(32);
+    INSTA_POLL_SLEEP();
     ld2_u64(P.heavy_acc + 2 * slot, x, y);
   }
   asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %1};" ::"l"(P.heavy_acc + 2 * slot), "l"(0ull) : "memory");
@@ -926,7 +926,7 @@ __device__ __forceinline__ void bwd_sink(const KParams& P, HeavyTab* tab, int nf
 __device__ __forceinline__ void await_g(const KParams& P, int q, uint32_t& a, uint32_t& b) {
   if (P.mode == 2) {
     while (((a & 1u) != P.par) || ((b & 1u) != P.par)) {
-      __nanosleep(20);
+      INSTA_POLL_SLEEP();
       ld2_u32(P.g + q, a, b);
     }
   }
