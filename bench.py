@@ -116,7 +116,7 @@ def fwd_bytes(N, E, n_src, P, lse):
 
 
 def bwd_bytes(N, E, E_light, P, nnz_arcs, lse):
-    """insta_backward: zero fill + seed kernel + propagation kernel."""
+    """insta_backward: prologue kernel (seeds + zero fill) + propagation kernel."""
     return (8 * E                         # d_mean zero fill
             + 17 * P                      # seeds: ep pin 4 + slack 4 + rf 1 + seed write 8
             + 24 * N                      # per pin: light-fanout ptr 4, fanin ptr 4, seed 8, heavy slot 4, + 4
@@ -505,7 +505,7 @@ def main():
             "fwd_ms": fwd_ms, "bwd_ms": bwd_ms, "fwd_bwd_ms": ms_step,
             "fwd_pins_per_s": N / (fwd_ms * 1e-3),
             "roofline": {"bound": "hbm", "kernel": "fwd_persistent(+slack)" if dom == "fwd" else
-                         "bwd_persistent(+seed,memset)", "achieved": ach, "peak": peak, "unit": "GB/s",
+                         "bwd_persistent(+prologue: seeds, zero fill)", "achieved": ach, "peak": peak, "unit": "GB/s",
                          "frac": ach / peak, "peak_kind": peak_kind, "traffic": traffic,
                          "fwd_gbs": fwd_gbs, "bwd_gbs": bwd_gbs, "fwd_alg_bytes": fb, "bwd_alg_bytes": bb},
             "cpu_baseline": cpu, "e2e": e2e, "clocks": clk, "gpu_launches": launches_per_step * args.steps,

@@ -148,6 +148,30 @@ def test_custom_endpoint_seed_and_source_gradient():
     assert np.abs(r.d_src - b["d_src_mean"]).max() <= 1e-3 * max(1.0, np.abs(b["d_src_mean"]).max())
 
 
+@pytest.mark.parametrize("tau", [0.0, 1.0])
+@pytest.mark.parametrize("schedule", [0, 1])
+def test_backward_overwrites_poisoned_outputs(tau, schedule):
+    """insta_backward fully defines its outputs (include/insta.h): outputs prefilled
+    with NaN, at an 8-byte offset (not 16-byte aligned, odd float2 count) so the
+    prologue kernel's zero fill covers its unaligned head and tail, give the
+    same gradients, bit for bit, as fresh buffers (which the other tests check
+    against the oracle)."""
+    import torch
+
+    g = synth.generate("C2")
+    G = insta.Graph(g)
+    G.forward(NS, tau, schedule)
+    ref = G.backward().cpu().numpy()
+    E = g.num_arcs
+    raw = torch.full((2 * E + 2,), float("nan"), dtype=torch.float32, device="cuda")
+    out = raw[2:].view(E, 2)   # 8-byte offset
+    d = G.backward(out=out).cpu().numpy()
+    G.close()
+    assert np.isfinite(d).all()                            # every element written (zero or gradient)
+    assert np.array_equal(d, ref)
+    assert np.isnan(raw[:2].cpu().numpy()).all()          # nothing written before the buffer
+
+
 @pytest.mark.parametrize("seed", range(6))
 @pytest.mark.parametrize("tau", [0.0, 1.0])
 def test_tiny_dags(seed, tau):
