@@ -804,9 +804,9 @@ struct HeavyTab {
   unsigned long long acc[kHeavyTab][2];
 };
 
-__device__ __forceinline__ void heavy_add(const KParams& P, HeavyTab* tab, int32_t srcw, float gx, float gy) {
-  if (!((srcw >> kHeavyBit) & 1)) return;
-  const int slot = __ldg(P.heavy_slot + (srcw & kSrcMask));
+// slot: the heavy slot of the source (< 0: not heavy)
+__device__ __forceinline__ void heavy_add_slot(const KParams& P, HeavyTab* tab, int slot, float gx, float gy) {
+  if (slot < 0) return;
   const unsigned long long vx = (unsigned long long)(kCountUnit + __double2ll_rn(double(gx) * kFixH));
   const unsigned long long vy = (unsigned long long)(kCountUnit + __double2ll_rn(double(gy) * kFixH));
   if (tab) {
@@ -822,6 +822,15 @@ __device__ __forceinline__ void heavy_add(const KParams& P, HeavyTab* tab, int32
   }
   atomicAdd(P.heavy_acc + 2 * slot, vx);   // table full (or no table): direct
   atomicAdd(P.heavy_acc + 2 * slot + 1, vy);
+}
+
+__device__ __forceinline__ int heavy_slot_of(const KParams& P, int32_t srcw) {
+  return ((srcw >> kHeavyBit) & 1) ? __ldg(P.heavy_slot + (srcw & kSrcMask)) : -1;
+}
+
+__device__ __forceinline__ void heavy_add(const KParams& P, HeavyTab* tab, int32_t srcw, float gx, float gy) {
+  if (!((srcw >> kHeavyBit) & 1)) return;
+  heavy_add_slot(P, tab, __ldg(P.heavy_slot + (srcw & kSrcMask)), gx, gy);
 }
 
 template <bool kLSE>
@@ -1144,7 +1153,7 @@ __device__ __forceinline__ int win_sel(int32_t win, int k) {
 }
 
 struct EntryIn {
-  int32_t qpos, bw, arc, farc, fq, fsel;
+  int32_t qpos, bw, arc, farc, fq, fsel, bslot;   // bslot: heavy slot of the source (-1: light)
   float4 w, fw;
 };
 
@@ -1157,6 +1166,7 @@ __device__ __forceinline__ EntryIn load_entry(const KParams& P, int x, int32_t q
   e.arc = __ldg(P.ext_arc + x);
   e.farc = __ldg(P.ext_farc + x);
   e.fq = __ldg(P.ext_fq + x);
+  e.bslot = heavy_slot_of(P, e.bw);   // loaded ahead of the dependency chain
   e.fsel = 0;
   e.w = e.fw = make_float4(0.f, 0.f, 0.f, 0.f);
   if (kLSE) {
@@ -1174,7 +1184,7 @@ __device__ __forceinline__ void bwdf_entry(const KParams& P, HeavyTab* tab, cons
   const float2 gs = sink_arc<kLSE>(P, ab, sel, e.w, e.arc);
   if (e.farc < 0) {   // source p is a head: publish the per-arc adjoint for its pull
     st2_f32(P.g + e.qpos, with_parf(gs.x, P.par), with_parf(gs.y, P.par));
-    heavy_add(P, tab, e.bw, gs.x, gs.y);
+    heavy_add_slot(P, tab, e.bslot, gs.x, gs.y);
   } else {            // folded p: its adjoint as its own pull would form it, then arc e'
     const float gx = with_parf(gs.x, P.par), gy = with_parf(gs.y, P.par);
     float sx = 0.f, sy = 0.f;
@@ -1183,7 +1193,7 @@ __device__ __forceinline__ void bwdf_entry(const KParams& P, HeavyTab* tab, cons
     const float2 abp = make_float2(0.f + (sx + 0.f), 0.f + (sy + 0.f));
     const float2 g2 = sink_arc<kLSE>(P, abp, e.fsel, e.fw, e.farc);
     st2_f32(P.g + e.fq, with_parf(g2.x, P.par), with_parf(g2.y, P.par));
-    heavy_add(P, tab, e.bw, g2.x, g2.y);
+    heavy_add_slot(P, tab, e.bslot, g2.x, g2.y);
   }
 }
 
@@ -1241,6 +1251,12 @@ __global__ void __launch_bounds__(kThreads, 1) bwdf_kernel(KParams P) {
       for (int e = tid; e < nfo; e += kThreads)
         asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(gg + e)), "l"(P.g + S.lfo[fo + e])
                      : "memory");
+      // heavy heads' accumulators complete when their sinks' words do: read
+      // them while the gathers are in flight, not after the barrier
+      float2 eh[kEntPerThread];
+#pragma unroll
+      for (int j = 0; j < kEntPerThread; ++j)
+        eh[j] = (B.z != 0 && B.x + tid + j * kThreads < B.y) ? heavy_read(P, eslot[j]) : make_float2(0.f, 0.f);
       asm volatile("cp.async.wait_all;" ::: "memory");
       for (int e = tid; e < nfo; e += kThreads) {
         uint32_t a = __float_as_uint(gg[e].x), b = __float_as_uint(gg[e].y);
@@ -1282,7 +1298,7 @@ __global__ void __launch_bounds__(kThreads, 1) bwdf_kernel(KParams P) {
               sx += gg[r].x;
               sy += gg[r].y;
             }
-            const float2 h = heavy_read(P, eslot[j]);
+            const float2 h = eh[j];
             const float2 ab = make_float2(esd[j].x + (sx + h.x), esd[j].y + (sy + h.y));
             bwdf_entry<kLSE>(P, htab, ein[j], ab, kLSE ? 0 : win_sel(ewin[j], B.x + xr - S.hptr[lo + p]));
           }
