@@ -21,7 +21,9 @@
  *                  lse, sigma==0: pinned (tau*logsumexp over all paths)
  *                  lse, sigma>0: PARITY UNPINNED w.r.t. paper intent (reading
  *                  #1: sigma of the merged arrival = sigma of the arg-max;
- *                  pinned only by limits tau->0 / sigma->0 and FD consistency)
+ *                  pinned only by limits tau->0 / sigma->0, FD consistency and
+ *                  the equal-variance layered closed form, which holds for
+ *                  any choice of the kept sigma)
  *   orc_slack      pinned (closed forms)
  *   orc_backward   pinned (central finite differences of orc_forward; path
  *                  marginals for sigma==0 LSE; integer path counts in hard mode)
