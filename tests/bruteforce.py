@@ -60,6 +60,34 @@ def tiny_dag(seed, n_pins=8, p_edge=0.35, sigma0=False, dyadic=False, unate_p=(0
         ep_pin=np.asarray(eps, np.int32), ep_rat=rat, meta={})
 
 
+def layered_equal_variance(seed, widths=(3, 3, 2, 2), s0=1.5, sa=2.0):
+    """Strictly layered DAG (every arc joins consecutive layers), one sigma s0 on every source and
+    one sigma sa on every arc and rf: every path into a layer-l pin carries variance s0^2 + l*sa^2."""
+    rng = np.random.default_rng(seed)
+    layers, n = [], 0
+    for w in widths:
+        layers.append(list(range(n, n + w)))
+        n += w
+    arcs = []
+    for l in range(1, len(layers)):
+        for b in layers[l]:
+            srcs = [a for a in layers[l - 1] if rng.random() < 0.7] or [layers[l - 1][0]]
+            arcs += [(a, b) for a in srcs]
+    E = len(arcs)
+    lvl = np.zeros(n, int)
+    for l, ps in enumerate(layers):
+        lvl[ps] = l
+    g = types.SimpleNamespace(
+        num_pins=n, arc_class=np.zeros(E, np.uint8), arc_from=np.array([a for a, _ in arcs], np.int32),
+        arc_to=np.array([b for _, b in arcs], np.int32),
+        arc_unate=rng.choice(3, size=E, p=[0.4, 0.4, 0.2]).astype(np.uint8),
+        arc_mean=rng.uniform(1.0, 9.0, size=(E, 2)).astype(np.float32).astype(np.float64), arc_sigma=np.full((E, 2), sa),
+        src_mean=np.where(lvl[:, None] == 0, rng.uniform(0.0, 3.0, size=(n, 2)), 0.0).astype(np.float32).astype(np.float64),
+        src_sigma=np.where(lvl[:, None] == 0, np.full((n, 2), s0), 0.0),
+        ep_pin=np.array(layers[-1], np.int32), ep_rat=np.full((len(layers[-1]), 2), 25.0))
+    return g, lvl
+
+
 def source_transitions(rf, u):
     if u == POS:
         return [rf]

@@ -185,6 +185,22 @@ def test_tiny_dags(seed, tau):
     assert ((err <= 1e-3 * np.maximum(np.abs(b["d_mean"]), 1)) | mask).all()
 
 
+@pytest.mark.parametrize("seed", range(4))
+@pytest.mark.parametrize("tau", [0.3, 2.0])
+def test_lse_sigma_pos_equal_variance_layered(seed, tau):
+    """LSE with sigma > 0 on the layered equal-variance DAGs of the oracle pin: the GPU matches the
+    oracle and the closed form tau*logsumexp(path means) + N_sigma*sqrt(common variance)."""
+    from scipy.special import logsumexp
+    g, lvl = bf.layered_equal_variance(seed)
+    r = run_gpu(g, tau)
+    f, s, b = run_oracle(g, tau)
+    assert not tol_ok(r.A, f["A"]).any()
+    for (i, rf), ps in bf.enumerate_paths(g).items():
+        want = tau * logsumexp(np.array([m for m, _, _ in ps]) / tau) + NS * np.sqrt(1.5 ** 2 + lvl[i] * 4.0)
+        assert abs(r.A[i][rf] - want) <= max(1e-4 * abs(want), 1e-3)
+    assert (np.abs(r.d_mean - b["d_mean"]) <= 1e-3 * np.maximum(np.abs(b["d_mean"]), 1)).all()
+
+
 def _star(n_sinks, tau_unate=2, wide=9):
     """One driver with a huge fanout (> 128, the heavy-driver path) and a wide
     (9-input) NON-unate cell: exercises the atomic accumulator and the slow fanin path."""

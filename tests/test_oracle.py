@@ -313,34 +313,6 @@ def test_lse_sigma0_gradient_is_gibbs_path_marginal(seed):
         assert np.allclose(-b["d_mean"], want, atol=1e-10)
 
 
-def _layered_equal_variance(seed, widths=(3, 3, 2, 2), s0=1.5, sa=2.0):
-    """Strictly layered DAG (every arc joins consecutive layers), one sigma s0 on every source and
-    one sigma sa on every arc and rf: every path into a layer-l pin carries variance s0^2 + l*sa^2."""
-    rng = np.random.default_rng(seed)
-    layers, n = [], 0
-    for w in widths:
-        layers.append(list(range(n, n + w)))
-        n += w
-    arcs = []
-    for l in range(1, len(layers)):
-        for b in layers[l]:
-            srcs = [a for a in layers[l - 1] if rng.random() < 0.7] or [layers[l - 1][0]]
-            arcs += [(a, b) for a in srcs]
-    E = len(arcs)
-    lvl = np.zeros(n, int)
-    for l, ps in enumerate(layers):
-        lvl[ps] = l
-    g = types.SimpleNamespace(
-        num_pins=n, arc_from=np.array([a for a, _ in arcs], np.int32),
-        arc_to=np.array([b for _, b in arcs], np.int32),
-        arc_unate=rng.choice(3, size=E, p=[0.4, 0.4, 0.2]).astype(np.uint8),
-        arc_mean=rng.uniform(1.0, 9.0, size=(E, 2)), arc_sigma=np.full((E, 2), sa),
-        src_mean=np.where(lvl[:, None] == 0, rng.uniform(0.0, 3.0, size=(n, 2)), 0.0),
-        src_sigma=np.where(lvl[:, None] == 0, np.full((n, 2), s0), 0.0),
-        ep_pin=np.array(layers[-1], np.int32), ep_rat=np.full((len(layers[-1]), 2), 25.0))
-    return g, lvl
-
-
 @pytest.mark.parametrize("seed", range(10))
 @pytest.mark.parametrize("tau", [0.3, 2.0])
 def test_lse_sigma_pos_equal_variance_closed_form(seed, tau):
@@ -350,7 +322,7 @@ def test_lse_sigma_pos_equal_variance_closed_form(seed, tau):
     Eq 1-4 bookkeeping of the sigma > 0 LSE merge independently of reading R1); dA/dmu_e is the
     softmax path marginal (Eq 6) since the sigma term is a constant offset."""
     s0, sa = 1.5, 2.0
-    g, lvl = _layered_equal_variance(seed, s0=s0, sa=sa)
+    g, lvl = bf.layered_equal_variance(seed, s0=s0, sa=sa)
     paths = bf.enumerate_paths(g)
     f = oracle.forward(g, NS, tau)
     for (i, rf), ps in paths.items():
