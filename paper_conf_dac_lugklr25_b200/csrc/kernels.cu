@@ -490,9 +490,11 @@ __device__ __forceinline__ void fwd_round(const KParams& P, const Raw* gath, con
 // code, a clean one only republishes its previous record with this pass's
 // parity.  A recomputed head whose record changed marks its consumer heads
 // before publishing.  Bit-identical to a full pass (tested).
+// Counted per thread and flushed once per warp at the end of the pass (one
+// global atomic per warp instead of one per round with a dirty head).
 template <bool kInc>
-__device__ __forceinline__ void count_recomputed(const KParams& P, int n) {
-  if (kInc && n) atomicAdd(P.counters, (unsigned long long)n);
+__device__ __forceinline__ void count_recomputed(uint32_t& cnt, int n) {
+  if (kInc) cnt += uint32_t(n);
 }
 
 template <bool kLSE, bool kFold, bool kInc>
@@ -529,6 +531,7 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
     return;
   }
   const int ww = warp - 1, wt = tid - 32;
+  uint32_t nrec = 0u;   // kInc: heads recomputed by this thread
   for (int t = 0; t < nsteps; ++t) {
     const int s = t & 1;
     const int k = P.step_begin + t;
@@ -651,7 +654,7 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
                   if (!dirty) {
                     republish(P, i, hrec[hr]);
                   } else {
-                    count_recomputed<kInc>(P, 1);
+                    count_recomputed<kInc>(nrec, 1);
                     for (int kk = 0; kk < nf; ++kk)   // folded pins first (the incremental pass has no pre-pass)
                       if ((S.src[so + base + kk] >> kFoldBit) & 1)
                         gath[base + kk] = fold_pin<kLSE>(P, S.f[so + base + kk], S.fms[base + kk], S.fq[so + base + kk],
@@ -680,7 +683,7 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
               if (dm == 0) {   // no dirty head in this round: republish
                 if (lane < R.cnt) republish(P, S.pin[po + R.q + lane], hrec[R.q + lane - q0]);
               } else {
-                if (lane == 0) count_recomputed<kInc>(P, __popc(dm));
+                if (lane == 0) count_recomputed<kInc>(nrec, __popc(dm));
                 fwd_round<kLSE, kFold, true>(P, gath, A, S, po, so, R, lane, dirty, hrec + (head ? hr : 0));
               }
             } else {
@@ -719,7 +722,7 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
             if (!dirty) {
               republish(P, i, old);
             } else {
-              count_recomputed<kInc>(P, 1);
+              count_recomputed<kInc>(nrec, 1);
               fwd_pin_inc<kLSE>(P, i, nf, qf, old, arc);
             }
           }
@@ -729,6 +732,10 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
     __syncwarp();
     if (P.trace && wt == 0) P.trace[(size_t(c) * nsteps + t) * 4 + 2] = gtimer();
     if (lane == 0) mbar_arrive1(&empty[s]);
+  }
+  if (kInc) {
+    const uint32_t n = __reduce_add_sync(0xffffffffu, nrec);
+    if (lane == 0 && n) atomicAdd(P.counters, (unsigned long long)n);
   }
 }
 
