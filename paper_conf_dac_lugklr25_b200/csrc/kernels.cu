@@ -379,18 +379,22 @@ __device__ __forceinline__ void fwd_pin_inc(const KParams& P, int i, int nf, int
 template <bool kLSE, bool kFold, bool kInc>
 __device__ __forceinline__ void fwd_round(const KParams& P, const Raw* gath, const int4& A, const FwdStage& S,
                                           int po, int so, const Round& R, int lane, bool hdirty = false,
-                                          const Raw* hold = nullptr) {
+                                          const Raw* hold = nullptr, uint32_t dm = 0u) {
   const double ns = double(P.n_sigma);
   double bA[2] = {0.0, 0.0}, om[2] = {0.0, 0.0}, ov[2] = {0.0, 0.0}, A0[2] = {0.0, 0.0}, A1[2] = {0.0, 0.0};
   float osg[2] = {0.f, 0.f};
   int bi[2] = {0, 0};
   const bool act = lane < R.na;
   const int k = lane - R.seg;
+  // kInc: lanes of clean heads skip the folded pins and all stores (the head
+  // republishes its previous record; its folded pins, arg-max and weights
+  // are those of the previous pass, unchanged since nothing it reads changed)
+  const bool mine = !kInc || ((dm >> R.seg) & 1u);
   int u = 0;
   if (act) {
     u = int(uint32_t(R.w) >> kUnateShift);
     Raw rs = gath[R.base + lane];
-    if (kInc && ((R.w >> kFoldBit) & 1))
+    if (kInc && mine && ((R.w >> kFoldBit) & 1))
       rs = fold_pin<kLSE>(P, S.f[so + R.base + lane], S.fms[R.base + lane], S.fq[so + R.base + lane], rs);
     const Gath st = unpack(rs);
 #pragma unroll
@@ -471,13 +475,17 @@ __device__ __forceinline__ void fwd_round(const KParams& P, const Raw* gath, con
       }
       // fanin position of my arc: row start of my pin + k
       const int qpos = kFold ? S.q0[po + R.q + __popc(R.heads & ((2u << lane) - 1u)) - 1] + k : A.z + R.base + lane;
-      P.wts[qpos] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
+      if (mine) P.wts[qpos] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
     }
   }
   if (head) {
-    const uint32_t chg = (kInc && hdirty && record_changed(*hold, wm[0], wm[1], wv[0], wv[1])) ? 1u : 0u;
-    store_state(P, i, wm[0], wm[1], wv[0], wv[1], chg);
-    if (!kLSE) P.win[i] = bi[0] | (bi[1] << 16);
+    if (kInc && !hdirty) {
+      republish(P, i, *hold);
+    } else {
+      const uint32_t chg = (kInc && record_changed(*hold, wm[0], wm[1], wv[0], wv[1])) ? 1u : 0u;
+      store_state(P, i, wm[0], wm[1], wv[0], wv[1], chg);
+      if (!kLSE) P.win[i] = bi[0] | (bi[1] << 16);
+    }
   }
 }
 
@@ -684,7 +692,7 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
                 if (lane < R.cnt) republish(P, S.pin[po + R.q + lane], hrec[R.q + lane - q0]);
               } else {
                 if (lane == 0) count_recomputed<kInc>(nrec, __popc(dm));
-                fwd_round<kLSE, kFold, true>(P, gath, A, S, po, so, R, lane, dirty, hrec + (head ? hr : 0));
+                fwd_round<kLSE, kFold, true>(P, gath, A, S, po, so, R, lane, dirty, hrec + (head ? hr : 0), dm);
               }
             } else {
               fwd_round<kLSE, kFold, false>(P, gath, A, S, po, so, R, lane);
