@@ -480,7 +480,7 @@ __device__ __forceinline__ void fwd_round(const KParams& P, const Raw* gath, con
   }
   if (head) {
     if (kInc && !hdirty) {
-      republish(P, i, *hold);
+      // clean head: republished before the round (fwd_kernel)
     } else {
       const uint32_t chg = (kInc && record_changed(*hold, wm[0], wm[1], wv[0], wv[1])) ? 1u : 0u;
       store_state(P, i, wm[0], wm[1], wv[0], wv[1], chg);
@@ -692,6 +692,8 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
                 if (lane < R.cnt) republish(P, S.pin[po + R.q + lane], hrec[R.q + lane - q0]);
               } else {
                 if (lane == 0) count_recomputed<kInc>(nrec, __popc(dm));
+                // clean heads publish now, not after the round: their consumers do not wait on it
+                if (head && !dirty) republish(P, kFold ? S.pin[po + q0 + hr] : A.x + q0 + hr, hrec[hr]);
                 fwd_round<kLSE, kFold, true>(P, gath, A, S, po, so, R, lane, dirty, hrec + (head ? hr : 0), dm);
               }
             } else {
