@@ -216,7 +216,7 @@ def main():
     ap.add_argument("--config", default="C4")
     ap.add_argument("--tau", type=float, default=0.0)
     ap.add_argument("--schedule", type=int, default=0)
-    ap.add_argument("--e2e-steps", type=int, default=8)
+    ap.add_argument("--e2e-steps", type=int, default=20)
     ap.add_argument("--ref-sample-pins", type=int, default=1_500_000)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--batch-scenarios", type=int, default=1024, help="C5 batched evaluations (0 = skip)")
