@@ -13,7 +13,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libinsta.so")
-SOURCES = ["kernels.cu", "batch.cu", "topk.cu", "clark.cu", "place.cu", "size.cu", "levelize.cpp", "items.cpp", "fold.cpp", "api.cpp"]
+SOURCES = ["kernels.cu", "sweep.cu", "batch.cu", "topk.cu", "clark.cu", "place.cu", "size.cu", "levelize.cpp", "items.cpp", "fold.cpp", "api.cpp"]
 HEADERS = ["internal.h", "device_common.cuh"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 NVCC_FLAGS = ["-O3", "-std=c++17", "--fmad=false", "-lineinfo", "-Xcompiler", "-fPIC",

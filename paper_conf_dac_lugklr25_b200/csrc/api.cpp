@@ -65,7 +65,9 @@ void free_graph(insta::DevGraph& d) {
                   d.arc_head,  d.ext_h,     d.tk_q,      d.tk_sp,      d.tk_slack,  d.tk_star,
                   d.tk_summary, d.rat_ptr,  d.rat_sp,    d.rat_val,   d.tk_list,
                   d.cl_mv,     d.cl_pre,    d.cl_g,      d.cl_fo_ptr,  d.cl_fo_q,   d.cl_slack,
-                  d.cl_rf,     d.cl_summary, d.cl_hv_list, d.cl_hv_of, d.cl_hv_sum, d.tl_partials, d.sz_tmp};
+                  d.cl_rf,     d.cl_summary, d.cl_hv_list, d.cl_hv_of, d.cl_hv_sum, d.tl_partials, d.sz_tmp,
+                  d.sl_ptr,    d.ext_sh,    d.hfo_ptr,   d.hfo,       d.acc_h,     d.sl_bar,    d.sl_cnt,
+                  d.hwin,      d.ew,        d.fwin,      d.efw};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   if (d.b_stage_h) cudaFreeHost(d.b_stage_h);
@@ -240,7 +242,9 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   for (int32_t k = 0; k < d.num_ep; ++k) ep_of_pin[ep_pin[k]] = k;
   d.h_arc_pos = arc_pos;
   insta::FoldHost fold;
-  insta::build_fold(h, fin_src, fin_ms, ep_of_pin, lfo_ptr, lfo, heavy_slot, &fold);
+  int sms = 148;   // the sweep's grid (one CTA per SM): heads are ordered within its per-CTA slices
+  if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, desc->device) != cudaSuccess || sms <= 0) sms = 148;
+  insta::build_fold(h, fin_src, fin_ms, ep_of_pin, lfo_ptr, lfo, heavy_slot, sms, &fold);
   d.num_heads = int32_t(fold.hd_pin.size());
   d.num_slevels = int32_t(fold.slevel_ptr.size()) - 1;
   d.num_ext = int64_t(fold.ext_w.size());
@@ -253,6 +257,8 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   // ---- device: grid, items, upload ------------------------------------------------
   cudaError_t e = cudaSetDevice(d.device);
   if (e == cudaSuccess) e = static_cast<cudaError_t>(insta::query_grid(d.device, &d.grid));
+  if (e == cudaSuccess) e = static_cast<cudaError_t>(insta::query_sl_grid(d.device, &d.sl_grid, &d.sl_grid_b));
+  d.h_sl_ptr = fold.slevel_ptr;
   if (e == cudaSuccess) insta::build_items(d, lfo_ptr);
   if (e == cudaSuccess) insta::build_fold_items(d, fold);
   if (getenv("INSTA_DEBUG"))
@@ -319,6 +325,17 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   UP(d.bfwdf_a, d.bfwdf_items.a.data(), d.bfwdf_items.a.size());
   UP(d.bfwdf_b, d.bfwdf_items.b.data(), d.bfwdf_items.b.size());
   UP(d.bwdf_b, d.bwdf_items.b.data(), d.bwdf_items.b.size());
+  UP(d.sl_ptr, fold.slevel_ptr.data(), fold.slevel_ptr.size());
+  UP(d.ext_sh, fold.ext_sh.data(), fold.ext_sh.size());
+  UP(d.hfo_ptr, fold.hfo_ptr.data(), fold.hfo_ptr.size());
+  UP(d.hfo, fold.hfo.data(), fold.hfo.size());
+  ZERO(d.acc_h, 2 * fold.hd_pin.size());
+  ZERO(d.hwin, fold.hd_pin.size());
+  ZERO(d.ew, fold.ext_w.size());
+  ZERO(d.fwin, fold.ext_w.size());
+  ZERO(d.efw, fold.ext_w.size());
+  ZERO(d.sl_bar, 64);
+  ZERO(d.sl_cnt, std::max<size_t>(fold.slevel_ptr.size(), 1));
   ZERO(d.state, nN);
   ZERO(d.win, nN);
   ZERO(d.wts, nE);
@@ -409,17 +426,56 @@ insta_status insta_forward(insta_graph* g, const insta_opts* o, void* cuda_strea
       opt.tau < 0.f)
     return fail(INSTA_E_ARG, "forward: n_sigma and tau must be finite and >= 0");
   if (opt.want_grad_sigma != 0) return fail(INSTA_E_ARG, "forward: want_grad_sigma unsupported");
-  if (opt.schedule != 0 && opt.schedule != 1) return fail(INSTA_E_ARG, "forward: bad schedule");
+  if (opt.schedule < 0 || opt.schedule > 3) return fail(INSTA_E_ARG, "forward: bad schedule");
   insta::DevGraph& d = g->d;
   cudaSetDevice(d.device);
   // incremental cone pass when only incremental updates happened since a
-  // forward with the same options (persistent schedule)
-  const bool inc = d.pending_incremental && !d.pending_full && opt.schedule == 0 &&
-                   opt.n_sigma == d.last_n_sigma && opt.tau == d.last_tau;
-  int err = inc ? insta::launch_forward_incremental(d, opt.n_sigma, opt.tau, cuda_stream)
-                : insta::launch_forward(d, opt.n_sigma, opt.tau, opt.schedule, cuda_stream);
+  // forward with the same options (schedules 0, 2 and 3)
+  // (the cone pass keeps the previous pass's records, arg-max and weights of clean heads: they
+  // must be in the layout this schedule's backward reads -- head/entry order for 0 and 3,
+  // canonical for 2)
+  const bool sweep_sched = opt.schedule == 0 || opt.schedule == 3;
+  const bool inc = d.pending_incremental && !d.pending_full && opt.schedule != 1 &&
+                   opt.n_sigma == d.last_n_sigma && opt.tau == d.last_tau &&
+                   (sweep_sched ? d.sweep_valid : d.canon_valid);
+  int err = 0;
+  if ((opt.schedule == 0 || opt.schedule == 3) && inc) {   // cone pass (sweep.cu)
+    err = insta::launch_forward_cone(d, opt.n_sigma, opt.tau, cuda_stream);
+    if (!err) {
+      d.last_n_sigma = opt.n_sigma;
+      d.last_tau = opt.tau;
+      err = insta::launch_slack(d, cuda_stream);
+    }
+  } else if (opt.schedule == 3 || (opt.schedule == 0 && d.parity_mixed)) {
+    // level-synchronous sweep forward (sweep.cu); also the default's full pass
+    // right after a cone pass, whose mixed record parity cannot order a dataflow pass
+    err = insta::launch_forward_sl(d, opt.n_sigma, opt.tau, cuda_stream);
+    if (!err) {
+      d.last_n_sigma = opt.n_sigma;
+      d.last_tau = opt.tau;
+      err = insta::launch_slack(d, cuda_stream);
+    }
+  } else if (opt.schedule == 0) {   // stage-folded dataflow forward writing the sweep backward's inputs
+    err = insta::launch_forward(d, opt.n_sigma, opt.tau, 0, cuda_stream, 1);
+  } else if (inc && !d.parity_mixed) {   // schedule 2: dataflow incremental pass over every head
+    err = insta::launch_forward_incremental(d, opt.n_sigma, opt.tau, cuda_stream);
+  } else {   // 1: one launch per level; 2: persistent dataflow (kernels.cu); both store every record
+    // (schedule 2 orders by parity: after a sweep cone pass the parity is mixed -> per-level launches once)
+    const int ks = (opt.schedule == 2 && !d.parity_mixed) ? 0 : 1;
+    err = insta::launch_forward(d, opt.n_sigma, opt.tau, ks, cuda_stream);
+    if (!err) d.parity_mixed = false;
+  }
   if (err) return cuda_fail(err, "forward");
+  if (!inc) {
+    d.sweep_valid = sweep_sched;
+    d.canon_valid = !sweep_sched;
+  } else if (sweep_sched) {
+    d.canon_valid = false;
+  } else {
+    d.sweep_valid = false;
+  }
   d.bwd_schedule = opt.schedule;
+  d.fwd_schedule = opt.schedule;
   d.fwd_valid = true;
   d.pending_full = false;
   d.pending_incremental = false;

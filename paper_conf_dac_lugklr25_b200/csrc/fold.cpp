@@ -18,8 +18,9 @@
 // nests.  Every other pin is a "head".  Heads are scheduled by super-level:
 // slevel = 0 for indeg-0 pins, else 1 + max over its fanin arcs (p -> q) of
 // slevel(p) (p a head) or slevel(j) (p folded, j its source); heads are
-// ordered by (slevel, canonical position), so the startpoints keep positions
-// 0..num_src-1.
+// ordered by slevel, then (past level 0) by shape (fanin count, folded
+// entries, non-unate arc), then canonical position, so the startpoints keep
+// positions 0..num_src-1.
 #include <algorithm>
 
 #include <vector_functions.h>
@@ -30,7 +31,7 @@ namespace insta {
 
 void build_fold(const HostLevels& h, const std::vector<int32_t>& fin_src, const std::vector<float4>& fin_ms,
                 const std::vector<int32_t>& ep_of_pin, const std::vector<int32_t>& lfo_ptr,
-                const std::vector<int32_t>& lfo, const std::vector<int32_t>& heavy_slot, FoldHost* out) {
+                const std::vector<int32_t>& lfo, const std::vector<int32_t>& heavy_slot, int grid, FoldHost* out) {
   FoldHost& f = *out;
   f = FoldHost();
   const int32_t n = h.n;
@@ -67,6 +68,38 @@ void build_fold(const HostLevels& h, const std::vector<int32_t>& fin_src, const 
     std::vector<int32_t> fill(f.slevel_ptr.begin(), f.slevel_ptr.end() - (SL > 0 ? 1 : 0));
     for (int32_t q = 0; q < n; ++q)
       if (!f.folded[q]) f.hd_pin[fill[sl[q]]++] = q;
+  }
+  // within a super-level (past the startpoints) heads are ordered by their
+  // shape -- fanin count, folded entries, a non-unate arc -- then canonical
+  // position: the heads of one level are independent, and a warp of
+  // same-shape heads runs the fanin-specialized code without divergence
+  // (sweep.cu); every schedule walks the same head order
+  {
+    std::vector<int64_t> key(size_t(n), 0);
+    for (int32_t q = 0; q < n; ++q) {
+      if (f.folded[q]) continue;
+      const int32_t nf = fp[q + 1] - fp[q];
+      int32_t nfold = 0, non = 0;
+      for (int32_t x = fp[q]; x < fp[q + 1]; ++x) {
+        const int32_t p = fin_src[x] & kSrcMask;
+        if (uint32_t(fin_src[x]) >> kUnateShift == 2) non = 1;
+        if (f.folded[p]) {
+          ++nfold;
+          if (uint32_t(fin_src[fp[p]]) >> kUnateShift == 2) non = 1;
+        }
+      }
+      key[q] = (int64_t(std::min(nf, 255)) << 40) | (int64_t(std::min(nfold, 255)) << 32) | (int64_t(non) << 31) | q;
+    }
+    // sorted within each CTA slice of the sweep (sweep.cu cta_slice: CTA c of G
+    // owns heads [lo + n c / G, lo + n (c + 1) / G) of a level): every CTA keeps
+    // the level's natural mix of shapes (balanced work), its warps get uniform ones
+    const int64_t G = std::max(grid, 1);
+    for (int32_t s = 1; s < SL; ++s) {
+      const int64_t lo = f.slevel_ptr[s], nh = f.slevel_ptr[s + 1] - lo;
+      for (int64_t c = 0; c < G; ++c)
+        std::sort(f.hd_pin.begin() + lo + nh * c / G, f.hd_pin.begin() + lo + nh * (c + 1) / G,
+                  [&](int32_t x, int32_t y) { return key[x] < key[y]; });
+    }
   }
   // entries: one per fanin arc of a head, in fanin row order
   f.hd_ptr.assign(size_t(H) + 1, 0);
@@ -124,6 +157,47 @@ void build_fold(const HostLevels& h, const std::vector<int32_t>& fin_src, const 
       }
     }
     f.hd_ptr[hh + 1] = int32_t(x);
+  }
+  // level-synchronous sweep: source head of every entry and the consumer
+  // heads of every head (the heads whose entries read its record)
+  std::vector<int32_t> head_of(size_t(n), -1);
+  for (int32_t hh = 0; hh < H; ++hh) head_of[f.hd_pin[hh]] = hh;
+  f.ext_sh.assign(size_t(X), -1);
+  std::vector<int64_t> pair_src;
+  std::vector<int32_t> pair_dst;
+  pair_src.reserve(size_t(X));
+  pair_dst.reserve(size_t(X));
+  for (int32_t hh = 0; hh < H; ++hh) {
+    for (int32_t y = f.hd_ptr[hh]; y < f.hd_ptr[hh + 1]; ++y) {
+      const int32_t sp = f.ext_w[y] & kSrcMask;
+      f.ext_sh[y] = head_of[sp];
+      pair_src.push_back(head_of[sp]);
+      pair_dst.push_back(hh);
+    }
+  }
+  f.hfo_ptr.assign(size_t(H) + 1, 0);
+  for (int64_t k : pair_src) ++f.hfo_ptr[k + 1];
+  for (int32_t hh = 0; hh < H; ++hh) f.hfo_ptr[hh + 1] += f.hfo_ptr[hh];
+  f.hfo.assign(pair_src.size(), 0);
+  {
+    std::vector<int32_t> fill(f.hfo_ptr.begin(), f.hfo_ptr.end() - 1);
+    for (size_t k = 0; k < pair_src.size(); ++k) f.hfo[fill[pair_src[k]]++] = pair_dst[k];
+  }
+  // deduplicate each row (a consumer reading the same source through several entries)
+  {
+    int32_t w = 0;
+    int32_t lo = 0;
+    for (int32_t hh = 0; hh < H; ++hh) {
+      const int32_t hi = f.hfo_ptr[hh + 1];
+      std::sort(f.hfo.begin() + lo, f.hfo.begin() + hi);
+      const int32_t start = w;
+      for (int32_t k = lo; k < hi; ++k)
+        if (k == lo || f.hfo[k] != f.hfo[k - 1]) f.hfo[w++] = f.hfo[k];
+      f.hfo_ptr[hh] = start;
+      lo = hi;
+    }
+    f.hfo_ptr[H] = w;
+    f.hfo.resize(size_t(w));
   }
   // incremental pass: the head whose item evaluates each arc
   f.arc_head.assign(size_t(h.e), -1);

@@ -108,6 +108,10 @@ struct FoldHost {
   std::vector<int32_t> hd_eop;      // [H] endpoint index of each head (-1: not an endpoint)
   // incremental pass
   std::vector<int32_t> arc_head;    // [E] caller arc -> head whose item evaluates the arc
+  // level-synchronous sweep (sweep.cu)
+  std::vector<int32_t> ext_sh;      // [X] head index of the entry's source (j if folded, else p)
+  std::vector<int32_t> hfo_ptr;     // [H+1] consumer heads of each head (cone marking), deduplicated
+  std::vector<int32_t> hfo;         // consumer head indices
 };
 
 // Item table: step s of CTA c is entry s * G + c.
@@ -203,6 +207,26 @@ struct DevGraph {
   uint32_t* dirty_h = nullptr;     // [H] incremental: stamp == inc epoch -> recompute
   int32_t* arc_head = nullptr;     // [E] caller arc -> head
   float2* hseed = nullptr;         // [H] endpoint seeds in head order
+  // level-synchronous sweep (sweep.cu; schedule 0): one persistent launch per
+  // pass, a grid barrier per super-level, one thread per head
+  int sl_grid = 0, sl_grid_b = 0; // resident CTAs of the sweep forward / backward kernels
+  std::vector<int32_t> h_sl_ptr;   // [SL+1] host copy of the super-level head ranges
+  int32_t* sl_ptr = nullptr;       // [SL+1]
+  int32_t* ext_sh = nullptr;       // [X] source head of each entry
+  int32_t* hfo_ptr = nullptr;      // [H+1] consumer heads of each head
+  int32_t* hfo = nullptr;
+  long long* acc_h = nullptr;      // [H][2] fixed-point adjoint accumulators (zero between passes)
+  int32_t* hwin = nullptr;         // [H] arg-max word per head (hard mode, head order)
+  float4* ew = nullptr;            // [X] Eq 6 weights per entry (LSE, entry order)
+  int32_t* fwin = nullptr;         // [X] arg-max word of a non-unate folded pin
+  float4* efw = nullptr;           // [X] Eq 6 weights of a non-unate folded pin's arc
+  uint32_t* sl_bar = nullptr;      // grid barrier counters [0..1] (reset by the last CTA of each launch)
+  uint32_t* sl_cnt = nullptr;      // [SL] cone pass: dirty marks per super-level
+  bool folded_valid = false;       // folded pins' records / arg-max / weights are stored (arrivals, sigma bwd)
+  bool parity_mixed = false;
+  bool sweep_valid = false;        // hwin / ew / fwin / efw describe every head (last full pass: schedule 0 or 3)
+  bool canon_valid = false;        // win / wts (canonical) describe every pin (last full pass: schedule 1 or 2)       // a cone pass left records of different passes' parity (no dataflow pass next)
+  int fwd_schedule = 0;            // schedule of the last forward
   // sigma-channel backward scratch (allocated on first use)
   void* g4 = nullptr;              // [e] float4 per fanin position
   long long* hacc4 = nullptr;      // [num_heavy][4] fixed-point adjoints
@@ -285,7 +309,7 @@ void build_items(DevGraph& d, const std::vector<int32_t>& lfo_ptr);
 // stage folding (fold.cpp) and its item table (items.cpp)
 void build_fold(const HostLevels& h, const std::vector<int32_t>& fin_src, const std::vector<float4>& fin_ms,
                 const std::vector<int32_t>& ep_of_pin, const std::vector<int32_t>& lfo_ptr,
-                const std::vector<int32_t>& lfo, const std::vector<int32_t>& heavy_slot, FoldHost* out);
+                const std::vector<int32_t>& lfo, const std::vector<int32_t>& heavy_slot, int grid, FoldHost* out);
 void build_fold_items(DevGraph& d, const FoldHost& f);
 
 }  // namespace insta
@@ -297,7 +321,7 @@ struct insta_graph {
 namespace insta {
 // kernels.cu launchers; return cudaError_t as int
 int query_grid(int device, int* grid);
-int launch_forward(DevGraph& g, float n_sigma, float tau, int schedule, void* stream);
+int launch_forward(DevGraph& g, float n_sigma, float tau, int schedule, void* stream, int sweep_out = 0);
 int launch_forward_incremental(DevGraph& g, float n_sigma, float tau, void* stream);
 int launch_slack(DevGraph& g, void* stream);
 int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float* d_arc_sigma, float* d_src,
@@ -305,6 +329,12 @@ int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float*
 int launch_update_arcs(DevGraph& g, int64_t n, const int32_t* ids, const float* mean,
                        const float* sigma, int incremental, void* stream);
 int launch_arrivals(DevGraph& g, float* A, float* mean, float* sigma, void* stream);
+// sweep.cu: level-synchronous thread-per-head passes (schedule 0)
+int query_sl_grid(int device, int* grid_fwd, int* grid_bwd);
+int launch_forward_sl(DevGraph& g, float n_sigma, float tau, void* stream);
+int launch_forward_cone(DevGraph& g, float n_sigma, float tau, void* stream);
+int launch_backward_sl(DevGraph& g, float* d_arc_mean, float* d_src, void* stream);
+int launch_fold_fill(DevGraph& g, void* stream);   // materialize folded pins after a sweep forward
 int launch_copy_slack(DevGraph& g, float* slack, uint8_t* rf, void* stream);
 // batch.cu: one micro-batch of up to 32 scenarios in one pass.  All pointers are device pointers into
 // the staging buffer: sc = [3][32] {n_sigma, derate_cell, derate_net}, ov_ptr = [33] per-scenario

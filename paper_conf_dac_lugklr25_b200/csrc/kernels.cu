@@ -27,8 +27,10 @@
 // barrier sits on the level-to-level critical path; a CTA waits for exactly
 // the words it consumes.  Heavy drivers count arrivals inside their atomic
 // accumulator words.  mode 0 is one launch per level (schedule = 1); both
-// modes run the same item code and are bit-identical.  Arithmetic: fp64 state, fp32 inputs, IEEE sqrt/div/exp/log,
-// --fmad=false: deterministic and bit-reproducible.
+// modes run the same item code and are bit-identical.  Arithmetic: fp64 mean/variance state, fp32 inputs;
+// sigma = sqrt.approx.f32 (hardware, ~1 ulp), LSE exponentials/logarithms __expf/__logf (hardware ex2/lg2
+// approximations), IEEE fp32 division; --fmad=false: deterministic and bit-reproducible (not IEEE
+// sqrt/exp/log -- the oracle comparison tolerances cover the approximations).
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -93,6 +95,15 @@ struct KParams {
   float n_sigma, tau;
   double inv_tau;                // 1 / tau (LSE exponent scale)
   unsigned long long* trace;     // optional per-(CTA, step, warp) {start, end} globaltimer (debug)
+  // schedule 0 (the default): the stage-folded dataflow forward writes what the
+  // sweep backward (sweep.cu) reads -- arg-max per head, Eq 6 weights per entry,
+  // a non-unate folded pin's arg-max / weights per entry -- and does not store
+  // the folded pins' records (materialized on demand, launch_fold_fill)
+  int32_t sweep_out;
+  int32_t* hwin;                 // [H]
+  float4* ew;                    // [X]
+  int32_t* fwin;                 // [X]
+  float4* efw;                   // [X]
 };
 
 // --------------------------------------------------------------------------
@@ -223,7 +234,8 @@ __device__ __forceinline__ void fwd_prefetch(const KParams& P, FwdStage* st, uin
 // Forward of one non-source pin by one thread (both rf).  Returns the words
 // it stored (parity included), which is exactly what a consumer would load.
 template <bool kLSE, class ArcFn>
-__device__ __forceinline__ Raw fwd_pin(const KParams& P, int i, int nf, int q0, ArcFn&& arc) {
+__device__ __forceinline__ Raw fwd_pin(const KParams& P, int i, int nf, int q0, ArcFn&& arc, int h = -1,
+                                       int x0 = 0) {
   const RfOut R = pin_rf<kLSE>(P, 0, nf, arc);
   const RfOut F = pin_rf<kLSE>(P, 1, nf, arc);
   store_state(P, i, R.mu, F.mu, R.var, F.var);
@@ -232,13 +244,16 @@ __device__ __forceinline__ Raw fwd_pin(const KParams& P, int i, int nf, int q0, 
   o.b = (unsigned long long)__double_as_longlong(with_par(F.mu, P.par));
   o.c = (unsigned long long)__double_as_longlong(with_par(R.var, P.par));
   o.d = (unsigned long long)__double_as_longlong(with_tag(F.var, P.par, 0u));
+  const bool sw = P.sweep_out && h >= 0;   // head / entry order (schedule 0)
   if (!kLSE) {
-    P.win[i] = R.win | (F.win << 16);
+    if (sw) P.hwin[h] = R.win | (F.win << 16);
+    else P.win[i] = R.win | (F.win << 16);
   } else {
     for (int k = 0; k < nf; ++k) {
       const float2 wr = arc_rf_weights(P, 0, k, R, arc);
       const float2 wf = arc_rf_weights(P, 1, k, F, arc);
-      P.wts[q0 + k] = make_float4(wr.x, wr.y, wf.x, wf.y);
+      if (sw) P.ew[x0 + k] = make_float4(wr.x, wr.y, wf.x, wf.y);
+      else P.wts[q0 + k] = make_float4(wr.x, wr.y, wf.x, wf.y);
     }
   }
   return o;
@@ -247,22 +262,38 @@ __device__ __forceinline__ Raw fwd_pin(const KParams& P, int i, int nf, int q0, 
 // Forward of a pin with exactly one fanin arc (w: its source word with the
 // unateness bits, ms: its record, rj: the source's words): merge1 (the nf = 1
 // merge_rf sequence, bit-identical to fwd_pin(nf = 1)).  Returns the stored words.
+// h >= 0: a head (index h, entry x); h == -1: a folded pin of entry x;
+// h == -2: no head/entry bookkeeping (canonical outputs).
 template <bool kLSE>
-__device__ __forceinline__ Raw fwd_pin1(const KParams& P, int i, int q0, int32_t w, const float4& ms, const Raw& rj) {
+__device__ __forceinline__ Raw fwd_pin1(const KParams& P, int i, int q0, int32_t w, const float4& ms, const Raw& rj,
+                                        int h = -2, int x = 0) {
   Merge1 m;
-  merge1<kLSE>(unpack(rj), int(uint32_t(w) >> kUnateShift), ms, double(P.n_sigma), double(P.tau), P.inv_tau, m);
+  const int u = int(uint32_t(w) >> kUnateShift);
+  merge1<kLSE>(unpack(rj), u, ms, double(P.n_sigma), double(P.tau), P.inv_tau, m);
+  if (P.sweep_out && h == -1) {   // folded pin, schedule 0: only what the sweep backward reads
+    if (u == 2) {
+      if (!kLSE) P.fwin[x] = m.win;
+      else P.efw[x] = m.wt;
+    }
+    return m.stored(P.par);
+  }
   store_state(P, i, m.mu[0], m.mu[1], m.var[0], m.var[1]);
-  if (!kLSE) P.win[i] = m.win;
-  else P.wts[q0] = m.wt;
+  if (P.sweep_out && h >= 0) {
+    if (!kLSE) P.hwin[h] = m.win;
+    else P.ew[x] = m.wt;
+  } else {
+    if (!kLSE) P.win[i] = m.win;
+    else P.wts[q0] = m.wt;
+  }
   return m.stored(P.par);
 }
 
-// Folded pin p (stage folding, fold.cpp): its single fanin arc e' = (j -> p)
-// with source words rj.  Returns p's stored words, which replace j's in the
-// gather buffer of p's sink.
+// Folded pin p (stage folding, fold.cpp) of entry x: its single fanin arc
+// e' = (j -> p) with source words rj.  Returns p's words (as stored), which
+// replace j's in the gather buffer of p's sink.
 template <bool kLSE>
-__device__ __forceinline__ Raw fold_pin(const KParams& P, int32_t fw, const float4& fms, int fq, const Raw& rj) {
-  return fwd_pin1<kLSE>(P, fw & kSrcMask, fq, fw, fms, rj);
+__device__ __forceinline__ Raw fold_pin(const KParams& P, int32_t fw, const float4& fms, int fq, const Raw& rj, int x) {
+  return fwd_pin1<kLSE>(P, fw & kSrcMask, fq, fw, fms, rj, -1, x);
 }
 
 __device__ __forceinline__ void trace_stamp(const KParams& P, int c, int nsteps, int t, int slot) {
@@ -395,7 +426,8 @@ __device__ __forceinline__ void fwd_round(const KParams& P, const Raw* gath, con
     u = int(uint32_t(R.w) >> kUnateShift);
     Raw rs = gath[R.base + lane];
     if (kInc && mine && ((R.w >> kFoldBit) & 1))
-      rs = fold_pin<kLSE>(P, S.f[so + R.base + lane], S.fms[R.base + lane], S.fq[so + R.base + lane], rs);
+      rs = fold_pin<kLSE>(P, S.f[so + R.base + lane], S.fms[R.base + lane], S.fq[so + R.base + lane], rs,
+                          A.z + R.base + lane);
     const Gath st = unpack(rs);
 #pragma unroll
     for (int rf = 0; rf < 2; ++rf) {
@@ -475,7 +507,10 @@ __device__ __forceinline__ void fwd_round(const KParams& P, const Raw* gath, con
       }
       // fanin position of my arc: row start of my pin + k
       const int qpos = kFold ? S.q0[po + R.q + __popc(R.heads & ((2u << lane) - 1u)) - 1] + k : A.z + R.base + lane;
-      if (mine) P.wts[qpos] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
+      if (mine) {
+        if (P.sweep_out) P.ew[A.z + R.base + lane] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
+        else P.wts[qpos] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
+      }
     }
   }
   if (head) {
@@ -484,7 +519,10 @@ __device__ __forceinline__ void fwd_round(const KParams& P, const Raw* gath, con
     } else {
       const uint32_t chg = (kInc && record_changed(*hold, wm[0], wm[1], wv[0], wv[1])) ? 1u : 0u;
       store_state(P, i, wm[0], wm[1], wv[0], wv[1], chg);
-      if (!kLSE) P.win[i] = bi[0] | (bi[1] << 16);
+      if (!kLSE) {
+        if (P.sweep_out) P.hwin[A.x + hq] = bi[0] | (bi[1] << 16);
+        else P.win[i] = bi[0] | (bi[1] << 16);
+      }
     }
   }
 }
@@ -583,8 +621,10 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
               const int32_t w = S.src[so + a];
               const float4 ms = S.ms[a];
               await_raw(P, w & kSrcMask, r[x]);
-              if (kFold && ((w >> kFoldBit) & 1)) r[x] = fold_pin<kLSE>(P, S.f[so + a], S.fms[a], S.fq[so + a], r[x]);
-              fwd_pin1<kLSE>(P, kFold ? S.pin[po + p] : A.x + p, kFold ? S.q0[po + p] : A.z + a, w, ms, r[x]);
+              if (kFold && ((w >> kFoldBit) & 1))
+                r[x] = fold_pin<kLSE>(P, S.f[so + a], S.fms[a], S.fq[so + a], r[x], A.z + a);
+              fwd_pin1<kLSE>(P, kFold ? S.pin[po + p] : A.x + p, kFold ? S.q0[po + p] : A.z + a, w, ms, r[x],
+                             kFold ? A.x + p : -2, A.z + a);
             }
           }
         } else if (q1 > q0) {
@@ -634,7 +674,8 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
           }
           if (kFold && !kInc) {   // entries through folded pins: compute the folded pin first
             for (int a = a_lo + lane; a < a_hi; a += 32) {
-              if ((S.src[so + a] >> kFoldBit) & 1) gath[a] = fold_pin<kLSE>(P, S.f[so + a], S.fms[a], S.fq[so + a], gath[a]);
+              if ((S.src[so + a] >> kFoldBit) & 1)
+                gath[a] = fold_pin<kLSE>(P, S.f[so + a], S.fms[a], S.fq[so + a], gath[a], A.z + a);
             }
           }
           __syncwarp();
@@ -654,7 +695,7 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
                   r_ = gath[base + kk];
                 };
                 if (!kInc) {
-                  fwd_pin<kLSE>(P, i, nf, qf, arc);
+                  fwd_pin<kLSE>(P, i, nf, qf, arc, kFold ? A.x + q : -1, A.z + base);
                 } else {
                   const int hr = q - q0;
                   bool dirty = (stampm[min(hr >> 5, kStampWords - 1)] >> (hr & 31)) & 1u;
@@ -666,7 +707,7 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
                     for (int kk = 0; kk < nf; ++kk)   // folded pins first (the incremental pass has no pre-pass)
                       if ((S.src[so + base + kk] >> kFoldBit) & 1)
                         gath[base + kk] = fold_pin<kLSE>(P, S.f[so + base + kk], S.fms[base + kk], S.fq[so + base + kk],
-                                                         gath[base + kk]);
+                                                         gath[base + kk], A.z + base + kk);
                     fwd_pin_inc<kLSE>(P, i, nf, qf, hrec[hr], arc);
                   }
                 }
@@ -716,10 +757,11 @@ __global__ void __launch_bounds__(kFwdThreads, 1) fwd_kernel(KParams P) {
             rr = ld_state_raw(P, w & kSrcMask);
             await_raw(P, w & kSrcMask, rr);
             if (kFold && ((w >> kFoldBit) & 1))   // recomputed per call: same words
-              rr = fold_pin<kLSE>(P, __ldg(P.ext_f + b0 + kk), __ldg(P.ext_fms + b0 + kk), __ldg(P.ext_fq + b0 + kk), rr);
+              rr = fold_pin<kLSE>(P, __ldg(P.ext_f + b0 + kk), __ldg(P.ext_fms + b0 + kk), __ldg(P.ext_fq + b0 + kk), rr,
+                                  b0 + kk);
           };
           if (!kInc) {
-            fwd_pin<kLSE>(P, i, nf, qf, arc);
+            fwd_pin<kLSE>(P, i, nf, qf, arc, kFold ? h : -1, b0);
           } else {
             const Raw old = ld_state_raw(P, i);
             bool dirty = __ldcg(P.dirty_h + h) == P.stamp;
@@ -1630,7 +1672,8 @@ __global__ void update_arcs_kernel(int64_t n, const int32_t* __restrict__ ids,
                                    const float2* __restrict__ sigma,
                                    const int32_t* __restrict__ arc_pos, float4* fin_ms,
                                    const int32_t* __restrict__ arc_xpos, float4* ext_ms, float4* ext_fms,
-                                   const int32_t* __restrict__ arc_head, uint32_t* dirty_h, uint32_t stamp) {
+                                   const int32_t* __restrict__ arc_head, uint32_t* dirty_h, uint32_t stamp,
+                                   const int32_t* __restrict__ sl_ptr, int num_sl, uint32_t* sl_cnt) {
   const int64_t k = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
   if (k >= n) return;
   const int id = ids ? ids[k] : int(k);   // ids == NULL: all arcs in caller order
@@ -1639,7 +1682,17 @@ __global__ void update_arcs_kernel(int64_t n, const int32_t* __restrict__ ids,
   fin_ms[q] = make_float4(m.x, m.y, s.x, s.y);
   const int x = arc_xpos[id];   // the stage-folded schedule's copy of the record
   ((x & 1) ? ext_fms : ext_ms)[x >> 1] = make_float4(m.x, m.y, s.x, s.y);
-  if (dirty_h) dirty_h[arc_head[id]] = stamp;   // incremental: the head evaluating the arc recomputes
+  if (dirty_h) {   // incremental: the head evaluating the arc recomputes
+    const int h = arc_head[id];
+    dirty_h[h] = stamp;
+    int lo = 0, hi = num_sl;   // its super-level: flagged (the cone pass skips levels without marks)
+    while (hi - lo > 1) {
+      const int mid = (lo + hi) >> 1;
+      if (sl_ptr[mid] <= h) lo = mid;
+      else hi = mid;
+    }
+    sl_cnt[lo] = 1u;
+  }
 }
 
 // --------------------------------------------------------------------------
@@ -1793,11 +1846,16 @@ int launch_slack(DevGraph& g, void* stream) {
   return int(cudaGetLastError());
 }
 
-int launch_forward(DevGraph& g, float n_sigma, float tau, int schedule, void* stream) {
+int launch_forward(DevGraph& g, float n_sigma, float tau, int schedule, void* stream, int sweep_out) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   KParams P = make_params(g, false);
   P.n_sigma = n_sigma;
   P.tau = tau;
+  P.sweep_out = schedule == 0 ? sweep_out : 0;
+  P.hwin = g.hwin;
+  P.ew = g.ew;
+  P.fwin = g.fwin;
+  P.efw = g.efw;
   P.inv_tau = tau > 0.f ? 1.0 / double(tau) : 0.0;
   const bool lse = tau > 0.f;
   ++g.inc_epoch;   // a full pass supersedes pending incremental marks
@@ -1821,6 +1879,7 @@ int launch_forward(DevGraph& g, float n_sigma, float tau, int schedule, void* st
   }
   g.last_n_sigma = n_sigma;
   g.last_tau = tau;
+  g.folded_valid = P.sweep_out == 0;
   return launch_slack(g, stream);
 }
 
@@ -1837,7 +1896,7 @@ int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float*
       if (d_arc_sigma) Z.z[1] = ZeroRange{d_arc_sigma, sizeof(float) * 2 * size_t(g.e)};
     }
     if (d_src && g.n > 0) Z.z[2] = ZeroRange{d_src, sizeof(float) * 2 * size_t(g.n)};
-    if (!d_arc_sigma && g.bwd_schedule == 0 && g.n > 0)
+    if (!d_arc_sigma && g.bwd_schedule == 2 && g.n > 0)
       Z.z[3] = ZeroRange{g.heavy_acc, sizeof(unsigned long long) * 2 * size_t(std::max(g.num_heavy, 1))};
     size_t work = size_t(g.num_ep);
     for (int r = 0; r < kPrepRanges; ++r) work = std::max(work, Z.z[r].p ? Z.z[r].bytes / 16 : size_t(0));
@@ -1851,6 +1910,8 @@ int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float*
   }
   if (g.n == 0) return 0;
   if (d_arc_sigma) {   // sigma channel: per-level launches of bwds_kernel (canonical order)
+    const int ferr = launch_fold_fill(g, stream);   // folded pins' records after a sweep forward
+    if (ferr) return ferr;
     if (!g.g4) {
       e = cudaMalloc(&g.g4, sizeof(float4) * std::max<size_t>(size_t(g.e), 1));
       if (e == cudaSuccess) e = cudaMalloc(&g.hacc4, sizeof(long long) * 4 * size_t(std::max(g.num_heavy, 1)));
@@ -1881,6 +1942,8 @@ int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float*
     }
     return 0;
   }
+  if (g.bwd_schedule == 0 || g.bwd_schedule == 3)   // sweep backward (sweep.cu)
+    return launch_backward_sl(g, d_arc_mean, d_src, stream);
   KParams P = make_params(g, true);
   P.n_sigma = g.last_n_sigma;
   P.tau = g.last_tau;
@@ -1888,9 +1951,9 @@ int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float*
   P.d_mean = d_arc_mean;
   P.d_src = d_src;
   const bool lse = g.last_tau > 0.f;
-  P.mode = g.bwd_schedule == 0 ? 2 : 0;
+  P.mode = g.bwd_schedule == 2 ? 2 : 0;
   P.par = (++g.pass_bwd) & 1u;
-  if (g.bwd_schedule == 0) {   // stage-folded persistent pass (fold.cpp); heavy_acc zeroed above
+  if (g.bwd_schedule == 2) {   // stage-folded persistent pass (fold.cpp); heavy_acc zeroed above
     P.item_a = g.bwdf_a;
     P.item_b = g.bwdf_b;
     P.lfo_ptr = g.hlfo_ptr;
@@ -1912,7 +1975,8 @@ int launch_update_arcs(DevGraph& g, int64_t n, const int32_t* ids, const float* 
   update_arcs_kernel<<<blocks, 256, 0, st>>>(n, ids, reinterpret_cast<const float2*>(mean),
                                              reinterpret_cast<const float2*>(sigma), g.arc_pos,
                                              g.fin_ms, g.arc_xpos, g.ext_ms, g.ext_fms, g.arc_head,
-                                             incremental ? g.dirty_h : nullptr, g.inc_epoch + 1);
+                                             incremental ? g.dirty_h : nullptr, g.inc_epoch + 1, g.sl_ptr,
+                                             g.num_slevels, g.sl_cnt);
   return int(cudaGetLastError());
 }
 
@@ -1942,11 +2006,14 @@ int launch_forward_incremental(DevGraph& g, float n_sigma, float tau, void* stre
   }
   g.last_n_sigma = n_sigma;
   g.last_tau = tau;
+  g.folded_valid = true;
   return launch_slack(g, stream);
 }
 
 int launch_arrivals(DevGraph& g, float* A, float* mean, float* sigma, void* stream) {
   if (g.n == 0) return 0;
+  const int ferr = launch_fold_fill(g, stream);   // folded pins' records after a sweep forward
+  if (ferr) return ferr;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   arrivals_kernel<<<(g.n + 255) / 256, 256, 0, st>>>(
       g.n, g.state, g.order, g.last_n_sigma, reinterpret_cast<float2*>(A),

@@ -76,7 +76,7 @@ def test_incremental_fallbacks_to_full():
     A0 = G.arrivals()[0].cpu().numpy()
     G.update_arcs(ids, g.arc_mean[ids], g.arc_sigma[ids], incremental=True)
     G.forward(3.0, 0.0)
-    assert G.last_forward_stats() <= 3
+    assert G.last_forward_stats() <= 3 * 5   # the 3 heads evaluating the arcs (+ their folded input pins)
     assert np.array_equal(G.arrivals()[0].cpu().numpy(), A0)
     # option change -> full pass
     G.update_arcs(ids, g.arc_mean[ids] * 1.1, g.arc_sigma[ids], incremental=True)

@@ -67,7 +67,7 @@ def test_levelization_bit_exact(cfg):
 
 
 @pytest.mark.parametrize("cfg", ["C1", "C2"])
-@pytest.mark.parametrize("schedule", [0, 1])
+@pytest.mark.parametrize("schedule", [0, 1, 2, 3])
 def test_dyadic_hard_bit_exact(cfg, schedule):
     """sigma = 0 and mu on a 2^-6 grid: fp32 sums are exact, so GPU == oracle bit for bit,
     including tie-breaking (first candidate wins)."""
@@ -126,16 +126,31 @@ def test_lse_tau_0p01_normwise_c1():
     assert rel <= 1e-3, rel
 
 
+def grads_match(x, y, tau):
+    """Gradients of two schedules: the sweep (0) accumulates adjoints in 2^-32 fixed point, the
+    others sum fp32 per-arc adjoints, so they agree bit for bit where the adjoints are integers
+    (hard mode: path counts) and to fp32 summation rounding otherwise."""
+    if tau == 0.0:
+        return np.array_equal(x, y)
+    return bool((np.abs(x - y) <= 1e-5 * np.maximum(np.abs(y), 1.0)).all())
+
+
 @pytest.mark.parametrize("tau", [0.0, 1.0])
 def test_schedules_and_reruns_bit_identical(tau):
+    """Forward results are the same bit for bit under every schedule (same merge arithmetic);
+    reruns of a schedule are bit-identical in full (deterministic accumulation)."""
     g = synth.generate("C2")
     a = run_gpu(g, tau, 0)
     c = run_gpu(g, tau, 1)
+    e = run_gpu(g, tau, 2)
+    f = run_gpu(g, tau, 3)
     d = run_gpu(g, tau, 0)
-    for x, y in ((a, c), (a, d)):
+    for x, y in ((a, c), (a, d), (a, e), (a, f)):
         assert np.array_equal(x.A, y.A) and np.array_equal(x.sigma, y.sigma)
         assert np.array_equal(x.slack, y.slack) and x.summary == y.summary
-        assert np.array_equal(x.d_mean, y.d_mean)
+    assert np.array_equal(a.d_mean, d.d_mean) and np.array_equal(a.d_mean, f.d_mean)
+    assert np.array_equal(c.d_mean, e.d_mean)
+    assert grads_match(a.d_mean, c.d_mean, tau)
 
 
 def test_custom_endpoint_seed_and_source_gradient():
@@ -149,7 +164,7 @@ def test_custom_endpoint_seed_and_source_gradient():
 
 
 @pytest.mark.parametrize("tau", [0.0, 1.0])
-@pytest.mark.parametrize("schedule", [0, 1])
+@pytest.mark.parametrize("schedule", [0, 1, 2, 3])
 def test_backward_overwrites_poisoned_outputs(tau, schedule):
     """insta_backward fully defines its outputs (include/insta.h): outputs prefilled
     with NaN, at an 8-byte offset (not 16-byte aligned, odd float2 count) so the
@@ -238,7 +253,7 @@ def test_heavy_fanout_and_wide_fanin(n_sinks, tau):
     assert (err <= 1e-3 * np.maximum(np.abs(b["d_mean"]), 1)).all(), err.max()
     assert np.abs(r.d_src - b["d_src_mean"]).max() <= 1e-3 * max(1, np.abs(b["d_src_mean"]).max())
     r1 = run_gpu(g, tau, schedule=1)
-    assert np.array_equal(r1.d_mean, r.d_mean)
+    assert grads_match(r.d_mean, r1.d_mean, tau)
 
 
 def test_degenerate_graphs():
@@ -390,8 +405,13 @@ def test_stage_folded_shapes(tau):
     g = _fold_shapes()
     a = run_gpu(g, tau, 0, want_src=True)
     c = run_gpu(g, tau, 1, want_src=True)
-    assert np.array_equal(a.A, c.A) and np.array_equal(a.mu, c.mu) and np.array_equal(a.sigma, c.sigma)
-    assert np.array_equal(a.d_mean, c.d_mean) and np.array_equal(a.d_src, c.d_src)
+    e = run_gpu(g, tau, 2, want_src=True)
+    f3 = run_gpu(g, tau, 3, want_src=True)
+    assert np.array_equal(a.d_mean, f3.d_mean) and np.array_equal(a.A, f3.A)
+    for y in (c, e):
+        assert np.array_equal(a.A, y.A) and np.array_equal(a.mu, y.mu) and np.array_equal(a.sigma, y.sigma)
+        assert grads_match(a.d_mean, y.d_mean, tau) and grads_match(a.d_src, y.d_src, tau)
+    assert np.array_equal(c.d_mean, e.d_mean) and np.array_equal(c.d_src, e.d_src)
     f, s, b = run_oracle(g, tau)
     ft, at = oracle.tie_taint(g, NS, eps=1e-4, margin=0.05)
     assert not tol_ok(a.A, f["A"], ft if tau == 0 else None).any()
@@ -406,8 +426,9 @@ def _sigma_case(g, tau):
     d0, dsrc0 = (x.cpu().numpy() for x in G.backward(want_src=True))
     d1, ds, dsrc1 = (x.cpu().numpy() for x in G.backward(want_src=True, want_sigma=True))
     G.close()
-    # the sigma pass reproduces the mean channel bit for bit
-    assert np.array_equal(d0, d1) and np.array_equal(dsrc0, dsrc1)
+    # the sigma pass reproduces the mean channel (bit for bit in hard mode; to the
+    # fp32-sum vs fixed-point accumulation rounding with tau > 0)
+    assert grads_match(d0, d1, tau) and grads_match(dsrc0, dsrc1, tau)
     b = oracle.backward(g, NS, tau)
     mask = oracle.tie_taint(g, NS, eps=1e-4, margin=0.05)[1] if tau == 0 else np.zeros(ds.shape, bool)
     err = np.abs(ds - b["d_sigma"])
