@@ -66,8 +66,8 @@ void free_graph(insta::DevGraph& d) {
                   d.tk_summary, d.rat_ptr,  d.rat_sp,    d.rat_val,   d.tk_list,
                   d.cl_mv,     d.cl_pre,    d.cl_g,      d.cl_fo_ptr,  d.cl_fo_q,   d.cl_slack,
                   d.cl_rf,     d.cl_summary, d.cl_hv_list, d.cl_hv_of, d.cl_hv_sum, d.tl_partials, d.sz_tmp,
-                  d.sl_ptr,    d.ext_sh,    d.hfo_ptr,   d.hfo,       d.acc_h,     d.sl_bar,    d.sl_cnt,
-                  d.hwin,      d.ew,        d.fwin,      d.efw};
+                  d.sl_ptr,    d.ext_sh,    d.hd_csl,    d.chg,       d.acc_h,     d.sl_bar,    d.sl_cnt,
+                  d.hwin,      d.ew,        d.fwin,      d.efw,       d.sl_slice};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   if (d.b_stage_h) cudaFreeHost(d.b_stage_h);
@@ -326,9 +326,22 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   UP(d.bfwdf_b, d.bfwdf_items.b.data(), d.bfwdf_items.b.size());
   UP(d.bwdf_b, d.bwdf_items.b.data(), d.bwdf_items.b.size());
   UP(d.sl_ptr, fold.slevel_ptr.data(), fold.slevel_ptr.size());
+  {   // per-CTA slices of the sweep (sweep.cu): CTA c owns heads [lo + n c / G, lo + n (c + 1) / G)
+    const int64_t G = std::max(d.sl_grid, 1);
+    const int32_t SLn = d.num_slevels;
+    std::vector<int4> slc(size_t(std::max<int64_t>(int64_t(SLn) * G, 1)));
+    for (int32_t sv = 0; sv < SLn; ++sv) {
+      const int64_t lo = fold.slevel_ptr[sv], nh = fold.slevel_ptr[sv + 1] - lo;
+      for (int64_t c = 0; c < G; ++c) {
+        const int32_t a = int32_t(lo + nh * c / G), b = int32_t(lo + nh * (c + 1) / G);
+        slc[size_t(sv) * G + c] = make_int4(a, b, fold.hd_ptr[a], fold.hd_ptr[b]);
+      }
+    }
+    UP(d.sl_slice, slc.data(), slc.size());
+  }
   UP(d.ext_sh, fold.ext_sh.data(), fold.ext_sh.size());
-  UP(d.hfo_ptr, fold.hfo_ptr.data(), fold.hfo_ptr.size());
-  UP(d.hfo, fold.hfo.data(), fold.hfo.size());
+  UP(d.hd_csl, fold.hd_csl.data(), fold.hd_csl.size());
+  ZERO(d.chg, nN);
   ZERO(d.acc_h, 2 * fold.hd_pin.size());
   ZERO(d.hwin, fold.hd_pin.size());
   ZERO(d.ew, fold.ext_w.size());
@@ -479,6 +492,7 @@ insta_status insta_forward(insta_graph* g, const insta_opts* o, void* cuda_strea
   d.fwd_valid = true;
   d.pending_full = false;
   d.pending_incremental = false;
+  d.pending_updates = 0;
   d.last_incremental = inc;
   d.last_recomputed = d.n;
   if (out) return read_summary(d, cuda_stream, out);
@@ -536,6 +550,7 @@ insta_status insta_update_arcs(insta_graph* g, int64_t n, const int32_t* arc_ids
   d.cl_valid = false;
   if (incremental && !d.pending_full) d.pending_incremental = true;
   else d.pending_full = true;
+  d.pending_updates += n;
   return INSTA_OK;
 }
 

@@ -110,8 +110,7 @@ struct FoldHost {
   std::vector<int32_t> arc_head;    // [E] caller arc -> head whose item evaluates the arc
   // level-synchronous sweep (sweep.cu)
   std::vector<int32_t> ext_sh;      // [X] head index of the entry's source (j if folded, else p)
-  std::vector<int32_t> hfo_ptr;     // [H+1] consumer heads of each head (cone marking), deduplicated
-  std::vector<int32_t> hfo;         // consumer head indices
+  std::vector<int32_t> hd_csl;      // [H] super-levels of each head's consumers: min | max << 16, -1: none
 };
 
 // Item table: step s of CTA c is entry s * G + c.
@@ -212,9 +211,10 @@ struct DevGraph {
   int sl_grid = 0, sl_grid_b = 0; // resident CTAs of the sweep forward / backward kernels
   std::vector<int32_t> h_sl_ptr;   // [SL+1] host copy of the super-level head ranges
   int32_t* sl_ptr = nullptr;       // [SL+1]
+  int4* sl_slice = nullptr;        // [SL][sl_grid] per-CTA slices {a, b, xa, xb} of every super-level
   int32_t* ext_sh = nullptr;       // [X] source head of each entry
-  int32_t* hfo_ptr = nullptr;      // [H+1] consumer heads of each head
-  int32_t* hfo = nullptr;
+  int32_t* hd_csl = nullptr;       // [H] consumer super-level range of each head
+  uint32_t* chg = nullptr;         // [n] cone pass: stamp of the pass that changed the pin's record
   long long* acc_h = nullptr;      // [H][2] fixed-point adjoint accumulators (zero between passes)
   int32_t* hwin = nullptr;         // [H] arg-max word per head (hard mode, head order)
   float4* ew = nullptr;            // [X] Eq 6 weights per entry (LSE, entry order)
@@ -299,6 +299,7 @@ struct DevGraph {
   bool fwd_valid = false;          // a forward ran since the last update
   bool pending_incremental = false;
   bool pending_full = true;
+  int64_t pending_updates = 0;     // arcs re-annotated (incremental) since the last forward
   float last_n_sigma = 3.0f, last_tau = 0.0f;
   int64_t last_recomputed = 0;
   bool last_incremental = false;

@@ -72,6 +72,7 @@ constexpr double kAccInv = 1.0 / 4294967296.0;
 struct SLParams {
   int32_t num_sl, num_src, num_heads;
   const int32_t* __restrict__ sl_ptr;
+  const int4* __restrict__ slice;        // [SL][grid] {a, b, xa, xb}: CTA c's heads [a, b) of a level, entries [xa, xb)
   const int32_t* __restrict__ hd_ptr;
   const int32_t* __restrict__ hd_pin;
   const int32_t* __restrict__ hd_q0;
@@ -96,8 +97,8 @@ struct SLParams {
   // cone pass
   uint32_t* dirty;                       // [H] == stamp: recompute
   uint32_t stamp;
-  const int32_t* __restrict__ hfo_ptr;
-  const int32_t* __restrict__ hfo;
+  const int32_t* __restrict__ hd_csl;     // [H] consumer super-level range (min | max << 16, -1 none)
+  uint32_t* chg;                          // [n] == stamp: the pin's record changed in this cone pass
   uint32_t* sl_cnt;                      // [SL] level marked (cleared by the pass)
   unsigned long long* counters;          // [0] pins recomputed
   // backward
@@ -182,16 +183,16 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
-// this CTA's heads of level s: [a, b)
-__device__ __forceinline__ void cta_slice(const SLParams& P, int s, int& a, int& b) {
-  const int lo = __ldg(P.sl_ptr + s), n = __ldg(P.sl_ptr + s + 1) - lo;
-  if (n < (1 << 22)) {   // n * (grid <= 512) fits 32 bits: no 64-bit division
-    a = lo + int((uint32_t(n) * blockIdx.x) / gridDim.x);
-    b = lo + int((uint32_t(n) * (blockIdx.x + 1)) / gridDim.x);
-  } else {
-    a = lo + int(int64_t(n) * blockIdx.x / gridDim.x);
-    b = lo + int(int64_t(n) * (blockIdx.x + 1) / gridDim.x);
-  }
+// this CTA's slice of level s: heads [a, b), entries [xa, xb) (host table,
+// kept in shared memory for the first kSliceCap levels: no global round trip
+// on the level-to-level chain)
+constexpr int kSliceCap = 1024;
+__device__ __forceinline__ int4 slice_of(const SLParams& P, const int4* s_slc, int s) {
+  return s < kSliceCap ? s_slc[s] : __ldg(P.slice + size_t(s) * gridDim.x + blockIdx.x);
+}
+__device__ __forceinline__ void load_slices(const SLParams& P, int4* s_slc) {
+  for (int s = threadIdx.x; s < min(P.num_sl, kSliceCap); s += blockDim.x)
+    s_slc[s] = __ldg(P.slice + size_t(s) * gridDim.x + blockIdx.x);
 }
 
 struct HeadTopo {
@@ -209,20 +210,18 @@ __device__ __forceinline__ HeadTopo load_topo(const SLParams& P, int h) {
 // forward stage: head rows and entry words of one CTA slice
 constexpr int kFRowCap = 1024, kFEntCap = 2560;
 // Per CTA: head rows and entry words of two levels (double-buffered, staged a
-// level ahead), the arc records of the current level (staged while the
-// barrier and the gathers run), and the gathered source records.
+// level ahead; the arc records are read next to the source gathers), then the
+// CTA's slice table.
 struct FStageSet {
   int32_t ptr[2][kFRowCap + 8];
   int32_t pin[2][kFRowCap + 8];
   int32_t w[2][kFEntCap + 8];
   int32_t f[2][kFEntCap + 8];
-  float4 ms[kFEntCap];    // records of e and e' (16-byte elements: staged from exactly xa)
-  float4 fms[kFEntCap];
-  Raw gath[kFEntCap];     // source record of every entry of the slice (cp.async, 32 B)
-  uint64_t full[2], rec;
+  uint64_t full[2];
   int32_t ok[2];          // the slice fit the stage (else its heads read global)
 };
-constexpr size_t kFStageBytes = sizeof(FStageSet);
+constexpr size_t kFSlcOff = (sizeof(FStageSet) + 15) & ~size_t(15);   // int4 slice table after the stage
+constexpr size_t kFStageBytes = kFSlcOff + sizeof(int4) * kSliceCap;
 
 __device__ __forceinline__ bool fwd_fits(int a, int b, int xa, int xb) {
   return b > a && b - a <= kFRowCap && xb - xa <= kFEntCap;
@@ -247,19 +246,6 @@ __device__ __forceinline__ void fwd_issue(const SLParams& P, FStageSet* S, int b
   }
 }
 
-// thread 0: stage the arc records of the slice's entries [xa, xb)
-__device__ __forceinline__ void fwd_issue_rec(const SLParams& P, FStageSet* S, int xa, int xb, bool fits) {
-  const uint32_t bms = fits ? uint32_t(xb - xa) * 16u : 0u;
-  if (!bms) {
-    mbar_arrive(&S->rec);
-    return;
-  }
-  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-  mbar_expect_tx(&S->rec, 2 * bms);
-  bulk_g2s(S->ms, P.ext_ms + xa, bms, &S->rec);
-  bulk_g2s(S->fms, P.ext_fms + xa, bms, &S->rec);
-}
-
 // Folded pin p (fold.cpp) on its single fanin arc e' = (j -> p) (word f,
 // record fms, entry x): merge1, the nf = 1 merge (bit-identical to merge_rf),
 // on j's words rj.  Returns p's words as a store would leave them (parity
@@ -282,30 +268,22 @@ __device__ __forceinline__ Raw sl_fold(const SLParams& P, int32_t f, const float
   return m.stored(P.par);
 }
 
-// cone pass: super-levels that received marks, per CTA in shared memory
+// cone pass: super-levels that may hold a dirty head, per CTA in shared memory
 // (flushed to sl_cnt once per level; levels >= kMarkBits go to global directly)
 constexpr int kMarkWords = 64;
 constexpr int kMarkBits = 32 * kMarkWords;
-constexpr int kMarkSerial = 32;   // consumer rows longer than this are marked by the whole CTA
-constexpr int kBigCap = 64;
 
-__device__ __forceinline__ int sl_of(const SLParams& P, int q) {
-  int lo = 0, hi = P.num_sl;   // last s with sl_ptr[s] <= q
-  while (hi - lo > 1) {
-    const int mid = (lo + hi) >> 1;
-    if (__ldg(P.sl_ptr + mid) <= q) lo = mid;
-    else hi = mid;
-  }
-  return lo;
-}
-
-__device__ __forceinline__ void mark_row(const SLParams& P, int r0, int r1, int off, int step, uint32_t* s_mark) {
-  for (int r = r0 + off; r < r1; r += step) {
-    const int q = __ldg(P.hfo + r);
-    P.dirty[q] = P.stamp;
-    const int sq = sl_of(P, q);
-    if (sq < kMarkBits) atomicOr(s_mark + (sq >> 5), 1u << (sq & 31));
-    else atomicOr(P.sl_cnt + sq, 1u);
+// flag levels [lo, hi]
+__device__ __forceinline__ void mark_range(const SLParams& P, uint32_t* s_mark, int lo, int hi) {
+  for (int w = lo >> 5; w <= (hi >> 5); ++w) {
+    if (w >= kMarkWords) {
+      for (int s = max(lo, 32 * w); s <= hi; ++s) atomicOr(P.sl_cnt + s, 1u);
+      return;
+    }
+    uint32_t m = 0xffffffffu;
+    if (w == (lo >> 5)) m &= 0xffffffffu << (lo & 31);
+    if (w == (hi >> 5)) m &= 0xffffffffu >> (31 - (hi & 31));
+    atomicOr(s_mark + w, m);
   }
 }
 
@@ -347,9 +325,9 @@ __device__ __forceinline__ int sl_fwd_core(const SLParams& P, const HeadTopo& t,
     }
   }
 #ifdef INSTA_SL_PHASES
-  if (ph && !ph[2]) {   // debug: the gathers and records have landed (first use)
+  if (ph && !ph[4]) {   // debug: the first head's gathers and records have landed
     const unsigned long long dep = (r[0].a | __float_as_uint(ms[NF - 1].x)) & 0ull;
-    ph[2] = gtimer() + dep;
+    ph[4] = gtimer() + dep;
   }
 #endif
 #pragma unroll
@@ -419,7 +397,7 @@ __device__ __noinline__ int sl_fwd_wide(const SLParams P, const HeadTopo t, RfOu
 // when it changed, mark the consumer heads.  Returns the pins evaluated.
 template <bool kLSE, bool kInc>
 __device__ __forceinline__ int sl_fwd_head(const SLParams& P, int h, const HeadTopo& t, const EntSrc& E,
-                                           uint32_t* s_mark, int* s_big, unsigned long long* ph = nullptr) {
+                                           uint32_t* s_mark, unsigned long long* ph = nullptr) {
   RfOut R, F;
   Raw old;
   if (kInc) old = ld_raw(P.state + t.pin);
@@ -435,16 +413,10 @@ __device__ __forceinline__ int sl_fwd_head(const SLParams& P, int h, const HeadT
   if (kInc) {
     if (rec_changed(old, R.mu, F.mu, R.var, F.var)) {
       st_state(P.state + t.pin, R.mu, F.mu, R.var, F.var, P.par);
-      // the consumers of this record recompute (their super-levels are later);
-      // long rows (high-fanout drivers) are marked by the whole CTA afterwards
-      const int r0 = __ldg(P.hfo_ptr + h), r1 = __ldg(P.hfo_ptr + h + 1);
-      if (r1 - r0 > kMarkSerial) {
-        const int slot = atomicAdd(s_big + kBigCap, 1);
-        if (slot < kBigCap) s_big[slot] = h;
-        else mark_row(P, r0, r1, 0, 1, s_mark);
-      } else {
-        mark_row(P, r0, r1, 0, 1, s_mark);
-      }
+      // its consumers (later levels) see the change through chg; their levels are flagged
+      P.chg[t.pin] = P.stamp;
+      const int32_t cs = __ldg(P.hd_csl + h);
+      if (cs != -1) mark_range(P, s_mark, cs & 0xffff, int(uint32_t(cs) >> 16));
     }
   } else {
     st_state(P.state + t.pin, R.mu, F.mu, R.var, F.var, P.par);
@@ -452,176 +424,155 @@ __device__ __forceinline__ int sl_fwd_head(const SLParams& P, int h, const HeadT
   return npins;
 }
 
-// flush the CTA's level marks (after a CTA barrier; before the grid barrier)
-__device__ __forceinline__ void mark_flush(const SLParams& P, uint32_t* s_mark) {
+
+// Cone pass (kInc): is head h dirty?  Stamped by insta_update_arcs (an arc it
+// evaluates changed) or one of its entries' source records changed in this
+// pass (chg, written by the recomputed source head before the level barrier).
+__device__ __forceinline__ bool head_dirty(const SLParams& P, int h, const int32_t* w, int nf) {
+  uint32_t c[4];   // every load in flight at once (no chain through an early exit)
+  const uint32_t d = __ldcg(P.dirty + h);
+#pragma unroll
+  for (int k = 0; k < 4; ++k) c[k] = k < nf ? __ldcg(P.chg + (w[k] & kSrcMask)) : 0u;
+  bool any = d == P.stamp;
+#pragma unroll
+  for (int k = 0; k < 4; ++k) any |= c[k] == P.stamp;
+  for (int k = 4; k < nf && !any; ++k) any = __ldcg(P.chg + (w[k] & kSrcMask)) == P.stamp;
+  return any;
+}
+
+// flush the CTA's level flags (after a CTA barrier; before the grid barrier):
+// each level's flag is stored at most once per pass by a CTA (s_pub)
+__device__ __forceinline__ void mark_flush(const SLParams& P, uint32_t* s_mark, uint32_t* s_pub) {
   for (int k = threadIdx.x; k < kMarkWords; k += blockDim.x) {
-    uint32_t m = s_mark[k];
-    if (m) {
-      s_mark[k] = 0u;
-      while (m) {
-        const int b = __ffs(m) - 1;
-        m &= m - 1;
-        const int sl = 32 * k + b;
-        if (sl < P.num_sl && __ldcg(P.sl_cnt + sl) == 0u) P.sl_cnt[sl] = 1u;
-      }
+    uint32_t m = s_mark[k] & ~s_pub[k];
+    s_mark[k] = 0u;
+    s_pub[k] |= m;
+    while (m) {
+      const int b = __ffs(m) - 1;
+      m &= m - 1;
+      const int sl = 32 * k + b;
+      if (sl < P.num_sl) P.sl_cnt[sl] = 1u;
     }
   }
 }
 
-// kMode 0: full pass; 1: cone pass (dirty heads only, no staging)
+// kMode 0: full pass.  1: cone pass over the staged slices (large updates).
+// 2: cone pass reading only the dirty heads' topology (small updates).  The
+// cone passes recompute dirty heads only and skip (without a barrier) every
+// level no head flagged: its flag is final once the levels before it are done.
 template <bool kLSE, int kMode>
 __global__ void __launch_bounds__(kSLFwdThreads, 1) fwdl_kernel(SLParams P) {
+  constexpr bool kInc = kMode != 0;
+  constexpr bool kStaged = kMode != 2;
   extern __shared__ __align__(128) unsigned char sl_smem[];
-  __shared__ uint32_t s_mark[kMarkWords];
-  __shared__ int s_big[kBigCap + 1];
+  __shared__ uint32_t s_mark[kMarkWords], s_pub[kMarkWords];
   __shared__ uint32_t s_cnt;
-  const int nthr = gridDim.x * blockDim.x;
   const int gt = blockIdx.x * blockDim.x + threadIdx.x;
+  const int nthr = gridDim.x * blockDim.x;
   const int tid = threadIdx.x;
-  uint32_t nbar = 0;
+  const int L = P.num_sl;
+  uint32_t nbar = 0, nrec = 0;
   if (P.trace && gt == 0) P.trace[0] = gtimer();
-  if (kMode == 0) {
-    FStageSet* S = reinterpret_cast<FStageSet*>(sl_smem);
-    const int L = P.num_sl;
-    int xa_c = 0, xb_c = 0;   // thread 0: entry range of this CTA's slice of the current level
-    int xa_n = 0, xb_n = 0;   // ... and of the next level
-    if (tid == 0) {
-      mbar_init(&S->full[0]);
-      mbar_init(&S->full[1]);
-      mbar_init(&S->rec);
-      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-      if (L > 1) {
-        int a, b;
-        cta_slice(P, 1, a, b);
-        xa_c = __ldg(P.hd_ptr + a);
-        xb_c = __ldg(P.hd_ptr + b);
-        fwd_issue(P, S, 1, a, b, xa_c, xb_c);
-      }
-      if (L > 2) {
-        int a, b;
-        cta_slice(P, 2, a, b);
-        xa_n = __ldg(P.hd_ptr + a);
-        xb_n = __ldg(P.hd_ptr + b);
-      }
+  for (int k = tid; k < kMarkWords; k += blockDim.x) s_mark[k] = s_pub[k] = 0u;
+  FStageSet* S = reinterpret_cast<FStageSet*>(sl_smem);
+  int4* s_slc = reinterpret_cast<int4*>(sl_smem + kFSlcOff);
+  load_slices(P, s_slc);
+  __syncthreads();
+  if (kStaged && tid == 0) {
+    mbar_init(&S->full[0]);
+    mbar_init(&S->full[1]);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    if (L > 1) {
+      const int4 c = slice_of(P, s_slc, 1);
+      fwd_issue(P, S, 1, c.x, c.y, c.z, c.w);
     }
-    for (int s = gt; s < L; s += nthr) P.sl_cnt[s] = 0u;   // a full pass supersedes pending marks
+  }
+  if (!kInc) {
+    for (int s = gt; s < L; s += nthr) P.sl_cnt[s] = 0u;   // a full pass supersedes pending flags
     // startpoints: clock arrival distribution, mean and variance per rf
     for (int i = gt; i < P.num_src; i += nthr) {
       const float4 v = __ldg(P.src_ms + i);
       st_state(P.state + i, double(v.x), double(v.y), double(v.z) * double(v.z), double(v.w) * double(v.w), P.par);
     }
-    uint32_t phase[2] = {0u, 0u}, rphase = 0u;
-    for (int s = 1; s < L; ++s) {
-      const int bf = s & 1;
-      __syncthreads();   // every thread is done with level s - 1 (rows buffer bf ^ 1, records, gathers)
-      if (tid == 0) {
-        int a, b;
-        cta_slice(P, s, a, b);
-        fwd_issue_rec(P, S, xa_c, xb_c, fwd_fits(a, b, xa_c, xb_c));   // this level's arc records
-        if (s + 1 < L) {   // rows and entry words of level s + 1
-          cta_slice(P, s + 1, a, b);
-          fwd_issue(P, S, bf ^ 1, a, b, xa_n, xb_n);
-          xa_c = xa_n;
-          xb_c = xb_n;
-          if (s + 2 < L) {
-            cta_slice(P, s + 2, a, b);
-            xa_n = __ldg(P.hd_ptr + a);
-            xb_n = __ldg(P.hd_ptr + b);
-          }
-        }
-      }
-      grid_sync(P.bar, ++nbar, P.trace);   // levels < s are complete
-      unsigned long long* ph = nullptr;
-#ifdef INSTA_SL_PHASES
-      if (P.trace && tid == 0) {   // debug: per (level, CTA) {barrier exit, stage landed, gathers landed, done}
-        ph = P.trace + 512 + size_t(L + 8) * 2 * gridDim.x + (size_t(s) * gridDim.x + blockIdx.x) * 4;
-        ph[0] = gtimer();
-      }
-#endif
-      mbar_wait(&S->full[bf], phase[bf]);
-      phase[bf] ^= 1u;
-      int a, b;
-      cta_slice(P, s, a, b);
-      const bool ok = S->ok[bf] != 0;
-      const Window wp = window(a, b + 1, 4), wh = window(a, b, 4);
-      const int xa = ok ? S->ptr[bf][wp.off] : 0;
-      const int xb = ok ? S->ptr[bf][wp.off + (b - a)] : 0;
-      const Window wx = window(xa, xb, 4);
-      if (ok) {   // gather every entry's source record into shared memory: all in flight at once
-        for (int i = tid; i < xb - xa; i += blockDim.x) {
-          const PinState* src = P.state + (S->w[bf][wx.off + i] & kSrcMask);
-          const uint32_t d = smem_u32(S->gath + i);
-          asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n\t"
-                       "cp.async.cg.shared.global [%2], [%3], 16;" ::"r"(d),
-                       "l"(src), "r"(d + 16u), "l"(reinterpret_cast<const char*>(src) + 16)
-                       : "memory");
-        }
-        asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
-      }
-      mbar_wait(&S->rec, rphase);
-      rphase ^= 1u;
-      __syncthreads();
-#ifdef INSTA_SL_PHASES
-      if (ph) ph[1] = ph[2] = gtimer();
-#endif
-#ifdef INSTA_SL_NOWORK
-      continue;
-#endif
-      for (int h = a + tid; h < b; h += blockDim.x) {
-        const int r = h - a;
-        HeadTopo t;
-        EntSrc E;   // entry words, arc records, gathered records: staged slice, or global
-        if (ok) {
-          t.x0 = S->ptr[bf][wp.off + r];
-          t.nf = S->ptr[bf][wp.off + r + 1] - t.x0;
-          t.pin = S->pin[bf][wh.off + r];
-          const int xr = wx.off + t.x0 - xa, xe = t.x0 - xa;
-          E = EntSrc{S->w[bf] + xr, S->f[bf] + xr, S->ms + xe, S->fms + xe, S->gath + xe};
-        } else {
-          t = load_topo(P, h);
-          E = EntSrc{P.ext_w + t.x0, P.ext_f + t.x0, P.ext_ms + t.x0, P.ext_fms + t.x0, nullptr};
-        }
-        (void)sl_fwd_head<kLSE, false>(P, h, t, E, s_mark, s_big, ph);
-      }
-#ifdef INSTA_SL_PHASES
-      if (ph) ph[3] = gtimer();
-#endif
+  }
+  uint32_t phase[2] = {0u, 0u};
+  bool need_bar = !kInc;   // cone: flags of level 1 come from insta_update_arcs (an earlier launch)
+  for (int s = 1; s < L; ++s) {
+    const int bf = s & 1;
+    __syncthreads();   // every thread is done with level s - 1 (rows buffer bf ^ 1)
+    if (kStaged && tid == 0 && s + 1 < L) {   // rows and entry words of level s + 1
+      const int4 c = slice_of(P, s_slc, s + 1);
+      fwd_issue(P, S, bf ^ 1, c.x, c.y, c.z, c.w);
     }
-  } else {
-    for (int k = tid; k < kMarkWords; k += blockDim.x) s_mark[k] = 0u;
-    if (tid == 0) s_big[kBigCap] = 0;
-    uint32_t nrec = 0;
-    bool need_bar = false;   // marks of level 1 come from insta_update_arcs (an earlier launch)
-    for (int s = 1; s < P.num_sl; ++s) {
-      // marks into level s come from levels < s, all complete here (the
-      // previous barrier, or no work since it); unmarked levels are skipped
-      if (need_bar) grid_sync(P.bar, ++nbar, P.trace);
+    if (need_bar) grid_sync(P.bar, ++nbar, P.trace);   // levels < s are complete
+    unsigned long long* ph = nullptr;
+#ifdef INSTA_SL_PHASES
+    if (P.trace && tid == 0) {   // debug: per (level, CTA) timestamps
+      ph = P.trace + 512 + size_t(L + 8) * 2 * gridDim.x + (size_t(s) * gridDim.x + blockIdx.x) * 8;
+      ph[0] = gtimer();
+    }
+#endif
+    bool work = true;
+    if (kInc) {   // flags of level s come from levels < s: final here
       if (tid == 0) s_cnt = __ldcg(P.sl_cnt + s);
       __syncthreads();
-      const uint32_t cnt = s_cnt;
-      need_bar = cnt != 0;
-      if (!cnt) continue;
-      const int lo = __ldg(P.sl_ptr + s), hi = __ldg(P.sl_ptr + s + 1);
-      for (int h = lo + gt; h < hi; h += nthr) {
-        if (__ldcg(P.dirty + h) != P.stamp) continue;
-        const HeadTopo t = load_topo(P, h);
-        nrec += uint32_t(sl_fwd_head<kLSE, true>(
-            P, h, t, EntSrc{P.ext_w + t.x0, P.ext_f + t.x0, P.ext_ms + t.x0, P.ext_fms + t.x0, nullptr}, s_mark,
-            s_big));
-      }
-      __syncthreads();
-      const int nbig = min(s_big[kBigCap], kBigCap);
-      for (int k = 0; k < nbig; ++k) {
-        const int hb = s_big[k];
-        mark_row(P, __ldg(P.hfo_ptr + hb), __ldg(P.hfo_ptr + hb + 1), tid, blockDim.x, s_mark);
-      }
-      __syncthreads();
-      if (tid == 0) s_big[kBigCap] = 0;
-      mark_flush(P, s_mark);
+      work = s_cnt != 0;
+      need_bar = work;
+#ifdef INSTA_SL_PHASES
+      if (ph) ph[1] = gtimer();
+#endif
     }
-    // clear the level marks for the next cone pass (every CTA has read them)
+    const int4 sc = slice_of(P, s_slc, s);
+    const int a = sc.x, b = sc.y;
+    bool ok = false;
+    if (kStaged) {
+      mbar_wait(&S->full[bf], phase[bf]);
+      phase[bf] ^= 1u;
+      ok = S->ok[bf] != 0;
+    }
+#ifdef INSTA_SL_PHASES
+    if (ph) ph[2] = gtimer();
+#endif
+    if (!work) continue;
+    const Window wp = window(a, b + 1, 4), wh = window(a, b, 4);
+    const int xa = sc.z;
+    const Window wx = window(xa, sc.w, 4);
+    for (int h = a + tid; h < b; h += blockDim.x) {
+      const int r = h - a;
+      HeadTopo t;
+      EntSrc E;   // entry words, arc records: staged slice, or global
+      if (ok) {
+        t.x0 = S->ptr[bf][wp.off + r];
+        t.nf = S->ptr[bf][wp.off + r + 1] - t.x0;
+        t.pin = S->pin[bf][wh.off + r];
+        const int xr = wx.off + t.x0 - xa;
+        E = EntSrc{S->w[bf] + xr, S->f[bf] + xr, P.ext_ms + t.x0, P.ext_fms + t.x0, nullptr};
+      } else {
+        t = load_topo(P, h);
+        E = EntSrc{P.ext_w + t.x0, P.ext_f + t.x0, P.ext_ms + t.x0, P.ext_fms + t.x0, nullptr};
+      }
+      if (kInc) {
+        if (!head_dirty(P, h, E.w, t.nf)) continue;
+        nrec += uint32_t(sl_fwd_head<kLSE, true>(P, h, t, E, s_mark, ph));
+      } else {
+        (void)sl_fwd_head<kLSE, false>(P, h, t, E, s_mark, ph);
+      }
+    }
+#ifdef INSTA_SL_PHASES
+    if (ph) ph[5] = gtimer();
+#endif
+    if (kInc) {
+      __syncthreads();
+      mark_flush(P, s_mark, s_pub);
+#ifdef INSTA_SL_PHASES
+      if (ph) ph[6] = gtimer();
+#endif
+    }
+  }
+  if (kInc) {
+    // clear the level flags for the next cone pass (every CTA has read them)
     grid_sync(P.bar, ++nbar, P.trace);
-    for (int s = gt; s < P.num_sl; s += nthr) P.sl_cnt[s] = 0u;
+    for (int s = gt; s < L; s += nthr) P.sl_cnt[s] = 0u;
     const uint32_t n = __reduce_add_sync(0xffffffffu, nrec);
     if ((tid & 31) == 0 && n) atomicAdd(P.counters, (unsigned long long)n);
   }
@@ -741,7 +692,8 @@ struct BStageSet {
   uint64_t full[2];
   int32_t ok[2];
 };
-constexpr size_t kBStageBytes = sizeof(BStageSet);
+constexpr size_t kBSlcOff = (sizeof(BStageSet) + 15) & ~size_t(15);
+constexpr size_t kBStageBytes = kBSlcOff + sizeof(int4) * kSliceCap;
 
 template <bool kLSE>
 __device__ __forceinline__ void bwd_issue(const SLParams& P, BStageSet* S, int bf, int a, int b, int xa, int xb) {
@@ -834,21 +786,16 @@ __global__ void __launch_bounds__(kSLBwdThreads, 1) bwdl_kernel(SLParams P) {
   const int L = P.num_sl;
   uint32_t nbar = 0;
   if (P.trace && blockIdx.x == 0 && tid == 0) P.trace[0] = gtimer();
-  int xa_n = 0, xb_n = 0;
+  int4* s_slc = reinterpret_cast<int4*>(sl_smem + kBSlcOff);
+  load_slices(P, s_slc);
+  __syncthreads();
   if (tid == 0) {
     mbar_init(&S->full[0]);
     mbar_init(&S->full[1]);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     if (L > 1) {
-      int a, b;
-      cta_slice(P, L - 1, a, b);
-      bwd_issue<kLSE>(P, S, (L - 1) & 1, a, b, __ldg(P.hd_ptr + a), __ldg(P.hd_ptr + b));
-    }
-    if (L > 2) {
-      int a, b;
-      cta_slice(P, L - 2, a, b);
-      xa_n = __ldg(P.hd_ptr + a);
-      xb_n = __ldg(P.hd_ptr + b);
+      const int4 c = slice_of(P, s_slc, L - 1);
+      bwd_issue<kLSE>(P, S, (L - 1) & 1, c.x, c.y, c.z, c.w);
     }
   }
   uint32_t phase[2] = {0u, 0u};
@@ -856,26 +803,20 @@ __global__ void __launch_bounds__(kSLBwdThreads, 1) bwdl_kernel(SLParams P) {
     const int bf = s & 1;
     __syncthreads();   // every thread is done with buffer bf ^ 1 (level s + 1)
     if (tid == 0 && s - 1 >= 1) {   // stage level s - 1 while level s runs
-      int a, b;
-      cta_slice(P, s - 1, a, b);
-      bwd_issue<kLSE>(P, S, bf ^ 1, a, b, xa_n, xb_n);
-      if (s - 2 >= 1) {
-        cta_slice(P, s - 2, a, b);
-        xa_n = __ldg(P.hd_ptr + a);
-        xb_n = __ldg(P.hd_ptr + b);
-      }
+      const int4 c = slice_of(P, s_slc, s - 1);
+      bwd_issue<kLSE>(P, S, bf ^ 1, c.x, c.y, c.z, c.w);
     }
     if (s < L - 1) grid_sync(P.bar, ++nbar, P.trace);   // levels > s are complete
     mbar_wait(&S->full[bf], phase[bf]);
     phase[bf] ^= 1u;
-    int a, b;
-    cta_slice(P, s, a, b);
+    const int4 sc = slice_of(P, s_slc, s);
+    const int a = sc.x, b = sc.y;
     if (b > a) {
       const BStage& T = S->st[bf];
       if (S->ok[bf]) {
         const Window wp = window(a, b + 1, 4), wh = window(a, b, 4), ws = window(a, b, 8);
-        const int xa = T.ptr[wp.off];
-        const Window wx = window(xa, T.ptr[wp.off + (b - a)], 4);
+        const int xa = sc.z;
+        const Window wx = window(xa, sc.w, 4);
         for (int h = a + tid; h < b; h += blockDim.x) {
           const int r = h - a;
           const int x0 = T.ptr[wp.off + r], nf = T.ptr[wp.off + r + 1] - x0;
@@ -928,6 +869,7 @@ static SLParams sl_params(DevGraph& g) {
   P.num_src = g.num_src;
   P.num_heads = g.num_heads;
   P.sl_ptr = g.sl_ptr;
+  P.slice = g.sl_slice;
   P.hd_ptr = g.hd_ptr;
   P.hd_pin = g.hd_pin;
   P.hd_q0 = g.hd_q0;
@@ -946,8 +888,8 @@ static SLParams sl_params(DevGraph& g) {
   P.efw = g.efw;
   P.bar = g.sl_bar;
   P.dirty = g.dirty_h;
-  P.hfo_ptr = g.hfo_ptr;
-  P.hfo = g.hfo;
+  P.hd_csl = g.hd_csl;
+  P.chg = g.chg;
   P.sl_cnt = g.sl_cnt;
   P.counters = g.counters;
   P.ext_arc = g.ext_arc;
@@ -971,14 +913,19 @@ int query_sl_grid(int device, int* grid_f, int* grid_b) {
   cudaError_t e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
   if (e == cudaSuccess) e = sl_smem_attr(fwdl_kernel<false, 0>, kFStageBytes);
   if (e == cudaSuccess) e = sl_smem_attr(fwdl_kernel<true, 0>, kFStageBytes);
+  if (e == cudaSuccess) e = sl_smem_attr(fwdl_kernel<false, 1>, kFStageBytes);
+  if (e == cudaSuccess) e = sl_smem_attr(fwdl_kernel<true, 1>, kFStageBytes);
+  if (e == cudaSuccess) e = sl_smem_attr(fwdl_kernel<false, 2>, kFStageBytes);
+  if (e == cudaSuccess) e = sl_smem_attr(fwdl_kernel<true, 2>, kFStageBytes);
   if (e == cudaSuccess) e = sl_smem_attr(bwdl_kernel<false>, kBStageBytes);
   if (e == cudaSuccess) e = sl_smem_attr(bwdl_kernel<true>, kBStageBytes);
   if (e != cudaSuccess) return int(e);
   int occ = 1 << 30, b = 0;
   const void* kf[] = {(const void*)fwdl_kernel<false, 0>, (const void*)fwdl_kernel<true, 0>,
-                      (const void*)fwdl_kernel<false, 1>, (const void*)fwdl_kernel<true, 1>};
-  const size_t sf[] = {kFStageBytes, kFStageBytes, 0, 0};
-  for (int i = 0; i < 4; ++i) {
+                      (const void*)fwdl_kernel<false, 1>, (const void*)fwdl_kernel<true, 1>,
+                      (const void*)fwdl_kernel<false, 2>, (const void*)fwdl_kernel<true, 2>};
+  const size_t sf[] = {kFStageBytes, kFStageBytes, kFStageBytes, kFStageBytes, kFStageBytes, kFStageBytes};
+  for (int i = 0; i < 6; ++i) {
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kf[i], kSLFwdThreads, sf[i]);
     if (e != cudaSuccess) return int(e);
     occ = std::min(occ, b);
@@ -1002,7 +949,7 @@ int query_sl_grid(int device, int* grid_f, int* grid_b) {
 static int launch_coop(const void* fn, int grid, int threads, size_t smem, SLParams& P, cudaStream_t st,
                        const char* name) {
   const char* dir = getenv("INSTA_SL_TRACE");
-  const size_t nt = 512 + size_t(P.num_sl + 8) * 6 * size_t(grid);
+  const size_t nt = 512 + size_t(P.num_sl + 8) * 10 * size_t(grid);
   P.trace = nullptr;
   if (dir) {
     cudaMalloc(&P.trace, nt * 8);
@@ -1056,8 +1003,12 @@ int launch_forward_cone(DevGraph& g, float n_sigma, float tau, void* stream) {
   P.stamp = ++g.inc_epoch;
   const bool lse = tau > 0.f;
   g.parity_mixed = true;   // clean heads keep the parity of the pass that last wrote them
-  const int err = launch_coop(lse ? (const void*)fwdl_kernel<true, 1> : (const void*)fwdl_kernel<false, 1>, g.sl_grid,
-                              kSLFwdThreads, 0, P, st, "cone");
+  // large update batches: stage every level's topology (latency off the chain);
+  // small ones: read only the dirty heads' topology
+  const bool staged = g.pending_updates * 1000 > g.e;
+  const void* fn = staged ? (lse ? (const void*)fwdl_kernel<true, 1> : (const void*)fwdl_kernel<false, 1>)
+                          : (lse ? (const void*)fwdl_kernel<true, 2> : (const void*)fwdl_kernel<false, 2>);
+  const int err = launch_coop(fn, g.sl_grid, kSLFwdThreads, kFStageBytes, P, st, "cone");
   g.folded_valid = false;
   return err;
 }

@@ -94,4 +94,54 @@ with torch.cuda.stream(st):
         ts.append(e0.elapsed_time(e1))
         cone.append(G.last_forward_stats() / g.num_pins)
     print("cone ms", " ".join(f"{x:.3f}" for x in ts), "pins frac", " ".join(f"{x:.3f}" for x in cone), flush=True)
+    for frac in (1e-7, 1e-5, 1e-4, 1e-3):   # small updates: 1 cell, ~1e-5 of the arcs, ...
+        ts, cone = [], []
+        for k in range(5):
+            ids, m, s = synth.sizing_step(g, 100 + k, frac=frac)
+            ids, m, s = (torch.as_tensor(x, device="cuda") for x in (ids, m, s))
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(st)
+            G.update_arcs(ids, m, s, incremental=True, stream=st)
+            G.forward(3.0, tau, sched, sync=False, stream=st)
+            e1.record(st)
+            st.synchronize()
+            ts.append(e0.elapsed_time(e1))
+            cone.append(G.last_forward_stats() / g.num_pins)
+        print(f"update frac {frac:g} ({len(ids)} arcs): ms", " ".join(f"{x:.3f}" for x in ts), "pins frac",
+              " ".join(f"{x:.4f}" for x in cone), flush=True)
+    if trace:   # one more cone pass, traced
+        ids, m, s = synth.sizing_step(g, 9, frac=0.01)
+        ids, m, s = (torch.as_tensor(x, device="cuda") for x in (ids, m, s))
+        G.update_arcs(ids, m, s, incremental=True, stream=st)
+        st.synchronize()
+        os.environ["INSTA_SL_TRACE"] = trace
+        t0 = time.perf_counter()
+        G.forward(3.0, tau, sched, sync=False, stream=st)
+        st.synchronize()
+        os.environ.pop("INSTA_SL_TRACE")
+        p = os.path.join(trace, "sl_cone.bin")
+        if os.path.exists(p):
+            raw = np.fromfile(p, np.uint64).astype(np.int64)
+            t = raw[:512]
+            t = t[t > 0]
+            grid = 148
+            Lc = (len(raw) - 512) // grid // 10 - 8
+            ph = raw[512 + (Lc + 8) * 2 * grid: 512 + (Lc + 8) * 2 * grid + Lc * grid * 8].reshape(Lc, grid, 8)
+            if (ph[:, :, 0] > 0).any():
+                out = []
+                for s_ in range(1, Lc):
+                    p8 = ph[s_].astype(np.int64)
+                    ok = p8[:, 0] > 0
+                    if not ok.any():
+                        continue
+                    p8 = p8[ok]
+                    base = p8[:, 0:1]
+                    rel = np.where(p8 > 0, (p8 - base) / 1e3, np.nan)
+                    med = np.nanmedian(rel, axis=0)
+                    mx = np.nanmax(rel, axis=0)
+                    out.append(f"{s_}:" + "/".join("-" if np.isnan(v) else f"{v:.1f}" for v in med[1:7]) +
+                               f"(max {np.nanmax(mx):.1f})")
+                print("cone phases rel. to barrier exit, median us (flag/stage/-/gath/loop/flush):", " ".join(out[:30]))
+            print("cone total us", (t[-1] - t[0]) / 1e3, "barriers", len(t) - 1, "per barrier us:",
+                  " ".join(f"{x:.1f}" for x in np.diff(t) / 1e3))
 G.close()
