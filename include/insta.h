@@ -76,13 +76,24 @@ typedef struct {
 /* Forward options.  n_sigma: the pessimism level of Eq 3 (3.0 in the
  * paper).  tau: 0 selects the paper's hard max (Alg 1/Alg 2 with Top-K = 1,
  * strict ">" P:L97); tau > 0 selects the LSE smooth max of Eq 4 with
- * Eq 6 gradients.  schedule: 0 = persistent dataflow kernel (default),
- * 1 = one launch per timing level (the paper's launch structure). */
+ * Eq 6 gradients.  schedule (all bit-identical arrivals):
+ *   0 = stage-folded persistent dataflow forward + level-synchronous sweep
+ *       backward (default);
+ *   1 = one launch per timing level (the paper's launch structure);
+ *   2 = stage-folded persistent dataflow forward and backward (round-1 kernels);
+ *   3 = level-synchronous sweep forward and backward.
+ * cone_max: after insta_update_arcs(incremental = 1), the next forward takes
+ * the cone pass (only heads whose inputs changed are
+ * recomputed) when at most this many arcs were re-annotated, else a full pass
+ * (for large batches the cone of a random update reaches every level, and the
+ * dataflow full pass is faster).  0 = default limit max(64, num_arcs / 1e5);
+ * < 0 = never. */
 typedef struct {
   float n_sigma;
   float tau;
   int32_t want_grad_sigma; /* reserved; must be 0 in this version */
   int32_t schedule;
+  int64_t cone_max;
 } insta_opts;
 
 /* Global timing metrics: WNS = min(0, min slack),

@@ -143,9 +143,10 @@ class Graph:
         return _stream(self._torch, self.device)
 
     def forward(self, n_sigma: float = 3.0, tau: float = 0.0, schedule: int = 0, sync: bool = True,
-                stream=None):
-        """insta_forward: arrivals -> endpoint slack -> WNS/TNS.  Returns a Summary if sync."""
-        opts = _capi.insta_opts(float(n_sigma), float(tau), 0, int(schedule))
+                stream=None, cone_max: int = 0):
+        """insta_forward: arrivals -> endpoint slack -> WNS/TNS.  Returns a Summary if sync.
+        cone_max: incremental policy (include/insta.h): 0 default, < 0 never, > 0 max arcs for the cone pass."""
+        opts = _capi.insta_opts(float(n_sigma), float(tau), 0, int(schedule), int(cone_max))
         out = _capi.insta_summary() if sync else None
         check(self.lib.insta_forward(self._h, ctypes.byref(opts), self._st(stream),
                                      ctypes.byref(out) if out is not None else None), "insta_forward")

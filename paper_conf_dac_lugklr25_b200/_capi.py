@@ -35,7 +35,7 @@ class insta_graph_desc(ctypes.Structure):
 
 class insta_opts(ctypes.Structure):
     _fields_ = [("n_sigma", ctypes.c_float), ("tau", ctypes.c_float),
-                ("want_grad_sigma", ctypes.c_int32), ("schedule", ctypes.c_int32)]
+                ("want_grad_sigma", ctypes.c_int32), ("schedule", ctypes.c_int32), ("cone_max", ctypes.c_int64)]
 
 
 class insta_summary(ctypes.Structure):

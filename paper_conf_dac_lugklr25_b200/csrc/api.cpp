@@ -67,7 +67,7 @@ void free_graph(insta::DevGraph& d) {
                   d.cl_mv,     d.cl_pre,    d.cl_g,      d.cl_fo_ptr,  d.cl_fo_q,   d.cl_slack,
                   d.cl_rf,     d.cl_summary, d.cl_hv_list, d.cl_hv_of, d.cl_hv_sum, d.tl_partials, d.sz_tmp,
                   d.sl_ptr,    d.ext_sh,    d.hd_csl,    d.chg,       d.acc_h,     d.sl_bar,    d.sl_cnt,
-                  d.hwin,      d.ew,        d.fwin,      d.efw,       d.sl_slice};
+                  d.hwin,      d.ew,        d.fwin,      d.efw,       d.sl_slice,  d.hfo_ptr,   d.hfo,       d.hd_hsrc};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   if (d.b_stage_h) cudaFreeHost(d.b_stage_h);
@@ -341,6 +341,9 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   }
   UP(d.ext_sh, fold.ext_sh.data(), fold.ext_sh.size());
   UP(d.hd_csl, fold.hd_csl.data(), fold.hd_csl.size());
+  UP(d.hfo_ptr, fold.hfo_ptr.data(), fold.hfo_ptr.size());
+  UP(d.hfo, fold.hfo.data(), fold.hfo.size());
+  UP(d.hd_hsrc, fold.hd_hsrc.data(), fold.hd_hsrc.size());
   ZERO(d.chg, nN);
   ZERO(d.acc_h, 2 * fold.hd_pin.size());
   ZERO(d.hwin, fold.hd_pin.size());
@@ -433,7 +436,7 @@ static insta_status read_summary(insta::DevGraph& d, void* stream, insta_summary
 insta_status insta_forward(insta_graph* g, const insta_opts* o, void* cuda_stream,
                            insta_summary* out) {
   if (!g) return fail(INSTA_E_ARG, "forward: NULL graph");
-  insta_opts opt{3.0f, 0.0f, 0, 0};
+  insta_opts opt{3.0f, 0.0f, 0, 0, 0};
   if (o) opt = *o;
   if (!std::isfinite(opt.n_sigma) || opt.n_sigma < 0.f || !std::isfinite(opt.tau) ||
       opt.tau < 0.f)
@@ -448,9 +451,10 @@ insta_status insta_forward(insta_graph* g, const insta_opts* o, void* cuda_strea
   // must be in the layout this schedule's backward reads -- head/entry order for 0 and 3,
   // canonical for 2)
   const bool sweep_sched = opt.schedule == 0 || opt.schedule == 3;
+  const int64_t cone_max = opt.cone_max != 0 ? opt.cone_max : std::max<int64_t>(64, d.e / 100000);
   const bool inc = d.pending_incremental && !d.pending_full && opt.schedule != 1 &&
                    opt.n_sigma == d.last_n_sigma && opt.tau == d.last_tau &&
-                   (sweep_sched ? d.sweep_valid : d.canon_valid);
+                   (sweep_sched ? d.sweep_valid && d.pending_updates <= cone_max : d.canon_valid);
   int err = 0;
   if ((opt.schedule == 0 || opt.schedule == 3) && inc) {   // cone pass (sweep.cu)
     err = insta::launch_forward_cone(d, opt.n_sigma, opt.tau, cuda_stream);

@@ -175,19 +175,44 @@ void build_fold(const HostLevels& h, const std::vector<int32_t>& fin_src, const 
       pair_dst.push_back(hh);
     }
   }
-  // consumer super-level range of every head (cone pass: a changed record
-  // flags the levels its consumers live in): min | max << 16, or -1 (none)
-  f.hd_csl.assign(size_t(H), -1);
+  // cone pass (sweep.cu): consumer heads of every head (deduplicated rows,
+  // marked by a changed head when short), their super-level range (flagged
+  // when the row is long), and per head whether one of its sources has a long
+  // row (such a head checks its sources' change stamps itself)
+  f.hfo_ptr.assign(size_t(H) + 1, 0);
+  for (int64_t k : pair_src) ++f.hfo_ptr[k + 1];
+  for (int32_t hh = 0; hh < H; ++hh) f.hfo_ptr[hh + 1] += f.hfo_ptr[hh];
+  f.hfo.assign(pair_src.size(), 0);
   {
-    std::vector<int32_t> cmin(size_t(H), INT32_MAX), cmax(size_t(H), -1);
-    for (size_t k = 0; k < pair_src.size(); ++k) {
-      const int64_t src = pair_src[k];
-      const int32_t cs = sl[f.hd_pin[pair_dst[k]]];
-      cmin[src] = std::min(cmin[src], cs);
-      cmax[src] = std::max(cmax[src], cs);
+    std::vector<int32_t> fill(f.hfo_ptr.begin(), f.hfo_ptr.end() - 1);
+    for (size_t k = 0; k < pair_src.size(); ++k) f.hfo[fill[pair_src[k]]++] = pair_dst[k];
+    int32_t w = 0, lo = 0;
+    for (int32_t hh = 0; hh < H; ++hh) {
+      const int32_t hi = f.hfo_ptr[hh + 1];
+      std::sort(f.hfo.begin() + lo, f.hfo.begin() + hi);
+      const int32_t start = w;
+      for (int32_t k = lo; k < hi; ++k)
+        if (k == lo || f.hfo[k] != f.hfo[k - 1]) f.hfo[w++] = f.hfo[k];
+      f.hfo_ptr[hh] = start;
+      lo = hi;
     }
-    for (int32_t hh = 0; hh < H; ++hh)
-      if (cmax[hh] >= 0) f.hd_csl[hh] = std::min(cmin[hh], 65535) | (std::min(cmax[hh], 65535) << 16);
+    f.hfo_ptr[H] = w;
+    f.hfo.resize(size_t(w));
+  }
+  f.hd_csl.assign(size_t(H), -1);
+  f.hd_hsrc.assign(size_t(H), 0);
+  for (int32_t hh = 0; hh < H; ++hh) {
+    const int32_t r0 = f.hfo_ptr[hh], r1 = f.hfo_ptr[hh + 1];
+    if (r1 == r0) continue;
+    int32_t cmin = INT32_MAX, cmax = -1;
+    for (int32_t r = r0; r < r1; ++r) {
+      const int32_t cs = sl[f.hd_pin[f.hfo[r]]];
+      cmin = std::min(cmin, cs);
+      cmax = std::max(cmax, cs);
+    }
+    f.hd_csl[hh] = std::min(cmin, 65535) | (std::min(cmax, 65535) << 16);
+    if (r1 - r0 > kConeRow)
+      for (int32_t r = r0; r < r1; ++r) f.hd_hsrc[f.hfo[r]] = 1;
   }
   // incremental pass: the head whose item evaluates each arc
   f.arc_head.assign(size_t(h.e), -1);

@@ -37,6 +37,7 @@ constexpr int kHeavyBit = 29;
 constexpr int32_t kSrcMask = (1 << kHeavyBit) - 1;
 constexpr int32_t kMaxPins = (1 << 29) - 1;
 constexpr int kHeavyFanout = 256;
+constexpr int kConeRow = 32;       // cone pass: consumer rows longer than this are not marked one by one
 // ext_w word of the stage-folded schedule (fold.cpp): bit 29 "entry goes
 // through a folded pin" (the heavy bit is not needed by the forward)
 constexpr int kFoldBit = 29;
@@ -110,7 +111,10 @@ struct FoldHost {
   std::vector<int32_t> arc_head;    // [E] caller arc -> head whose item evaluates the arc
   // level-synchronous sweep (sweep.cu)
   std::vector<int32_t> ext_sh;      // [X] head index of the entry's source (j if folded, else p)
+  std::vector<int32_t> hfo_ptr;     // [H+1] consumer heads of each head (deduplicated)
+  std::vector<int32_t> hfo;
   std::vector<int32_t> hd_csl;      // [H] super-levels of each head's consumers: min | max << 16, -1: none
+  std::vector<uint8_t> hd_hsrc;     // [H] 1: a source of the head has more than kConeRow consumers
 };
 
 // Item table: step s of CTA c is entry s * G + c.
@@ -214,6 +218,9 @@ struct DevGraph {
   int4* sl_slice = nullptr;        // [SL][sl_grid] per-CTA slices {a, b, xa, xb} of every super-level
   int32_t* ext_sh = nullptr;       // [X] source head of each entry
   int32_t* hd_csl = nullptr;       // [H] consumer super-level range of each head
+  int32_t* hfo_ptr = nullptr;      // [H+1] consumer heads of each head
+  int32_t* hfo = nullptr;
+  uint8_t* hd_hsrc = nullptr;      // [H] a source with a long consumer row
   uint32_t* chg = nullptr;         // [n] cone pass: stamp of the pass that changed the pin's record
   long long* acc_h = nullptr;      // [H][2] fixed-point adjoint accumulators (zero between passes)
   int32_t* hwin = nullptr;         // [H] arg-max word per head (hard mode, head order)

@@ -1693,7 +1693,7 @@ __global__ void update_arcs_kernel(int64_t n, const int32_t* __restrict__ ids,
     }
     // one store per (warp, level) instead of one per arc (hot words)
     const uint32_t peers = __match_any_sync(__activemask(), lo);
-    if ((threadIdx.x & 31) == __ffs(peers) - 1) sl_cnt[lo] = 1u;
+    if ((threadIdx.x & 31) == __ffs(peers) - 1) atomicOr(sl_cnt + lo, 1u);
   }
 }
 

@@ -98,6 +98,9 @@ struct SLParams {
   uint32_t* dirty;                       // [H] == stamp: recompute
   uint32_t stamp;
   const int32_t* __restrict__ hd_csl;     // [H] consumer super-level range (min | max << 16, -1 none)
+  const int32_t* __restrict__ hfo_ptr;    // [H+1] consumer heads (deduplicated rows)
+  const int32_t* __restrict__ hfo;
+  const uint8_t* __restrict__ hd_hsrc;    // [H] a source of the head has a long consumer row
   uint32_t* chg;                          // [n] == stamp: the pin's record changed in this cone pass
   uint32_t* sl_cnt;                      // [SL] level marked (cleared by the pass)
   unsigned long long* counters;          // [0] pins recomputed
@@ -221,7 +224,7 @@ struct FStageSet {
   int32_t ok[2];          // the slice fit the stage (else its heads read global)
 };
 constexpr size_t kFSlcOff = (sizeof(FStageSet) + 15) & ~size_t(15);   // int4 slice table after the stage
-constexpr size_t kFStageBytes = kFSlcOff + sizeof(int4) * kSliceCap;
+constexpr size_t kFStageBytes = kFSlcOff + sizeof(int4) * kSliceCap + sizeof(int32_t) * (kSliceCap + 4);
 
 __device__ __forceinline__ bool fwd_fits(int a, int b, int xa, int xb) {
   return b > a && b - a <= kFRowCap && xb - xa <= kFEntCap;
@@ -268,23 +271,41 @@ __device__ __forceinline__ Raw sl_fold(const SLParams& P, int32_t f, const float
   return m.stored(P.par);
 }
 
-// cone pass: super-levels that may hold a dirty head, per CTA in shared memory
-// (flushed to sl_cnt once per level; levels >= kMarkBits go to global directly)
-constexpr int kMarkWords = 64;
-constexpr int kMarkBits = 32 * kMarkWords;
+// cone pass: super-levels that may hold a dirty head, per CTA in shared
+// memory (flushed to sl_cnt once per level).  Bit 0 (s_mark): a head of the
+// level was stamped dirty; bit 1 (s_mark + kMarkWords): a source with a long
+// consumer row changed -- the level's heads with such a source check it.
+constexpr int kMarkWords = 64;   // levels >= 32 * kMarkWords are flagged in global directly
 
-// flag levels [lo, hi]
+__device__ __forceinline__ void mark_level(const SLParams& P, uint32_t* s_mark, int s, uint32_t kind) {
+  if (s < 32 * kMarkWords) atomicOr(s_mark + (kind - 1) * kMarkWords + (s >> 5), 1u << (s & 31));
+  else atomicOr(P.sl_cnt + s, kind);
+}
+
+// flag levels [lo, hi] (kind 2)
 __device__ __forceinline__ void mark_range(const SLParams& P, uint32_t* s_mark, int lo, int hi) {
   for (int w = lo >> 5; w <= (hi >> 5); ++w) {
     if (w >= kMarkWords) {
-      for (int s = max(lo, 32 * w); s <= hi; ++s) atomicOr(P.sl_cnt + s, 1u);
+      for (int s = max(lo, 32 * w); s <= hi; ++s) atomicOr(P.sl_cnt + s, 2u);
       return;
     }
     uint32_t m = 0xffffffffu;
     if (w == (lo >> 5)) m &= 0xffffffffu << (lo & 31);
     if (w == (hi >> 5)) m &= 0xffffffffu >> (31 - (hi & 31));
-    atomicOr(s_mark + w, m);
+    atomicOr(s_mark + kMarkWords + w, m);
   }
+}
+
+// super-level of head q: last s with sl_ptr[s] <= q (level table in shared memory)
+__device__ __forceinline__ int sl_of(const SLParams& P, const int32_t* s_slp, int q) {
+  int lo = 0, hi = P.num_sl;
+  while (hi - lo > 1) {
+    const int mid = (lo + hi) >> 1;
+    const int v = mid <= kSliceCap ? s_slp[mid] : __ldg(P.sl_ptr + mid);
+    if (v <= q) lo = mid;
+    else hi = mid;
+  }
+  return lo;
 }
 
 // where a head's entry words and arc records are read: its staged slice
@@ -397,7 +418,7 @@ __device__ __noinline__ int sl_fwd_wide(const SLParams P, const HeadTopo t, RfOu
 // when it changed, mark the consumer heads.  Returns the pins evaluated.
 template <bool kLSE, bool kInc>
 __device__ __forceinline__ int sl_fwd_head(const SLParams& P, int h, const HeadTopo& t, const EntSrc& E,
-                                           uint32_t* s_mark, unsigned long long* ph = nullptr) {
+                                           uint32_t* s_mark, const int32_t* s_slp, unsigned long long* ph = nullptr) {
   RfOut R, F;
   Raw old;
   if (kInc) old = ld_raw(P.state + t.pin);
@@ -413,10 +434,27 @@ __device__ __forceinline__ int sl_fwd_head(const SLParams& P, int h, const HeadT
   if (kInc) {
     if (rec_changed(old, R.mu, F.mu, R.var, F.var)) {
       st_state(P.state + t.pin, R.mu, F.mu, R.var, F.var, P.par);
-      // its consumers (later levels) see the change through chg; their levels are flagged
+      // consumers (later levels): a short row is stamped dirty one by one; a
+      // long row's consumers see the change through chg (levels flagged)
       P.chg[t.pin] = P.stamp;
-      const int32_t cs = __ldg(P.hd_csl + h);
-      if (cs != -1) mark_range(P, s_mark, cs & 0xffff, int(uint32_t(cs) >> 16));
+      const int r0 = __ldg(P.hfo_ptr + h), r1 = __ldg(P.hfo_ptr + h + 1);
+      if (r1 - r0 <= kConeRow) {
+        for (int r = r0; r < r1; r += 8) {   // the row's loads in flight together
+          int32_t q[8];
+#pragma unroll
+          for (int j = 0; j < 8; ++j) q[j] = r + j < r1 ? __ldg(P.hfo + r + j) : -1;
+#pragma unroll
+          for (int j = 0; j < 8; ++j) {
+            if (q[j] >= 0) {
+              P.dirty[q[j]] = P.stamp;
+              mark_level(P, s_mark, sl_of(P, s_slp, q[j]), 1u);
+            }
+          }
+        }
+      } else {
+        const int32_t cs = __ldg(P.hd_csl + h);
+        mark_range(P, s_mark, cs & 0xffff, int(uint32_t(cs) >> 16));
+      }
     }
   } else {
     st_state(P.state + t.pin, R.mu, F.mu, R.var, F.var, P.par);
@@ -428,12 +466,13 @@ __device__ __forceinline__ int sl_fwd_head(const SLParams& P, int h, const HeadT
 // Cone pass (kInc): is head h dirty?  Stamped by insta_update_arcs (an arc it
 // evaluates changed) or one of its entries' source records changed in this
 // pass (chg, written by the recomputed source head before the level barrier).
-__device__ __forceinline__ bool head_dirty(const SLParams& P, int h, const int32_t* w, int nf) {
-  uint32_t c[4];   // every load in flight at once (no chain through an early exit)
-  const uint32_t d = __ldcg(P.dirty + h);
+__device__ __forceinline__ bool head_dirty(const SLParams& P, int h, const int32_t* w, int nf, uint32_t lvl) {
+  if (__ldcg(P.dirty + h) == P.stamp) return true;
+  if (!(lvl & 2u) || !__ldg(P.hd_hsrc + h)) return false;
+  uint32_t c[4];   // every load in flight at once
 #pragma unroll
   for (int k = 0; k < 4; ++k) c[k] = k < nf ? __ldcg(P.chg + (w[k] & kSrcMask)) : 0u;
-  bool any = d == P.stamp;
+  bool any = false;
 #pragma unroll
   for (int k = 0; k < 4; ++k) any |= c[k] == P.stamp;
   for (int k = 4; k < nf && !any; ++k) any = __ldcg(P.chg + (w[k] & kSrcMask)) == P.stamp;
@@ -441,17 +480,19 @@ __device__ __forceinline__ bool head_dirty(const SLParams& P, int h, const int32
 }
 
 // flush the CTA's level flags (after a CTA barrier; before the grid barrier):
-// each level's flag is stored at most once per pass by a CTA (s_pub)
+// each (level, kind) flag is published at most once per pass by a CTA (s_pub)
 __device__ __forceinline__ void mark_flush(const SLParams& P, uint32_t* s_mark, uint32_t* s_pub) {
-  for (int k = threadIdx.x; k < kMarkWords; k += blockDim.x) {
+  for (int k = threadIdx.x; k < 2 * kMarkWords; k += blockDim.x) {
     uint32_t m = s_mark[k] & ~s_pub[k];
     s_mark[k] = 0u;
     s_pub[k] |= m;
+    const uint32_t kind = k < kMarkWords ? 1u : 2u;
+    const int w = k % kMarkWords;
     while (m) {
       const int b = __ffs(m) - 1;
       m &= m - 1;
-      const int sl = 32 * k + b;
-      if (sl < P.num_sl) P.sl_cnt[sl] = 1u;
+      const int sl = 32 * w + b;
+      if (sl < P.num_sl) atomicOr(P.sl_cnt + sl, kind);
     }
   }
 }
@@ -465,7 +506,7 @@ __global__ void __launch_bounds__(kSLFwdThreads, 1) fwdl_kernel(SLParams P) {
   constexpr bool kInc = kMode != 0;
   constexpr bool kStaged = kMode != 2;
   extern __shared__ __align__(128) unsigned char sl_smem[];
-  __shared__ uint32_t s_mark[kMarkWords], s_pub[kMarkWords];
+  __shared__ uint32_t s_mark[2 * kMarkWords], s_pub[2 * kMarkWords];
   __shared__ uint32_t s_cnt;
   const int gt = blockIdx.x * blockDim.x + threadIdx.x;
   const int nthr = gridDim.x * blockDim.x;
@@ -473,10 +514,12 @@ __global__ void __launch_bounds__(kSLFwdThreads, 1) fwdl_kernel(SLParams P) {
   const int L = P.num_sl;
   uint32_t nbar = 0, nrec = 0;
   if (P.trace && gt == 0) P.trace[0] = gtimer();
-  for (int k = tid; k < kMarkWords; k += blockDim.x) s_mark[k] = s_pub[k] = 0u;
+  for (int k = tid; k < 2 * kMarkWords; k += blockDim.x) s_mark[k] = s_pub[k] = 0u;
   FStageSet* S = reinterpret_cast<FStageSet*>(sl_smem);
   int4* s_slc = reinterpret_cast<int4*>(sl_smem + kFSlcOff);
+  int32_t* s_slp = reinterpret_cast<int32_t*>(s_slc + kSliceCap);   // level table (cone: level of a head)
   load_slices(P, s_slc);
+  for (int v = tid; v <= min(P.num_sl, kSliceCap); v += blockDim.x) s_slp[v] = __ldg(P.sl_ptr + v);
   __syncthreads();
   if (kStaged && tid == 0) {
     mbar_init(&S->full[0]);
@@ -497,14 +540,38 @@ __global__ void __launch_bounds__(kSLFwdThreads, 1) fwdl_kernel(SLParams P) {
   }
   uint32_t phase[2] = {0u, 0u};
   bool need_bar = !kInc;   // cone: flags of level 1 come from insta_update_arcs (an earlier launch)
+  __shared__ int s_next;
   for (int s = 1; s < L; ++s) {
+    if (kMode == 2) {
+      // unstaged cone: no staging pipeline to keep, so jump straight to the next
+      // flagged level -- every flag at or past s is final (no level ran since
+      // the last barrier); one warp scans them 32 at a time
+      if (need_bar) grid_sync(P.bar, ++nbar, P.trace);
+      need_bar = false;
+      if (tid < 32) {
+        int nx = L;
+        for (int base = s; base < L; base += 32) {
+          const uint32_t f = base + tid < L ? __ldcg(P.sl_cnt + base + tid) : 0u;
+          const uint32_t hit = __ballot_sync(0xffffffffu, f != 0u);
+          if (hit) {
+            nx = base + __ffs(hit) - 1;
+            break;
+          }
+        }
+        if (tid == 0) s_next = nx;
+      }
+      __syncthreads();
+      s = s_next;
+      __syncthreads();
+      if (s >= L) break;
+    }
     const int bf = s & 1;
     __syncthreads();   // every thread is done with level s - 1 (rows buffer bf ^ 1)
     if (kStaged && tid == 0 && s + 1 < L) {   // rows and entry words of level s + 1
       const int4 c = slice_of(P, s_slc, s + 1);
       fwd_issue(P, S, bf ^ 1, c.x, c.y, c.z, c.w);
     }
-    if (need_bar) grid_sync(P.bar, ++nbar, P.trace);   // levels < s are complete
+    if (kMode != 2 && need_bar) grid_sync(P.bar, ++nbar, P.trace);   // levels < s are complete
     unsigned long long* ph = nullptr;
 #ifdef INSTA_SL_PHASES
     if (P.trace && tid == 0) {   // debug: per (level, CTA) timestamps
@@ -513,10 +580,12 @@ __global__ void __launch_bounds__(kSLFwdThreads, 1) fwdl_kernel(SLParams P) {
     }
 #endif
     bool work = true;
+    uint32_t lvl = 0;
     if (kInc) {   // flags of level s come from levels < s: final here
       if (tid == 0) s_cnt = __ldcg(P.sl_cnt + s);
       __syncthreads();
-      work = s_cnt != 0;
+      lvl = s_cnt;
+      work = lvl != 0;
       need_bar = work;
 #ifdef INSTA_SL_PHASES
       if (ph) ph[1] = gtimer();
@@ -552,10 +621,10 @@ __global__ void __launch_bounds__(kSLFwdThreads, 1) fwdl_kernel(SLParams P) {
         E = EntSrc{P.ext_w + t.x0, P.ext_f + t.x0, P.ext_ms + t.x0, P.ext_fms + t.x0, nullptr};
       }
       if (kInc) {
-        if (!head_dirty(P, h, E.w, t.nf)) continue;
-        nrec += uint32_t(sl_fwd_head<kLSE, true>(P, h, t, E, s_mark, ph));
+        if (!head_dirty(P, h, E.w, t.nf, lvl)) continue;
+        nrec += uint32_t(sl_fwd_head<kLSE, true>(P, h, t, E, s_mark, s_slp, ph));
       } else {
-        (void)sl_fwd_head<kLSE, false>(P, h, t, E, s_mark, ph);
+        (void)sl_fwd_head<kLSE, false>(P, h, t, E, s_mark, s_slp, ph);
       }
     }
 #ifdef INSTA_SL_PHASES
@@ -889,6 +958,9 @@ static SLParams sl_params(DevGraph& g) {
   P.bar = g.sl_bar;
   P.dirty = g.dirty_h;
   P.hd_csl = g.hd_csl;
+  P.hfo_ptr = g.hfo_ptr;
+  P.hfo = g.hfo;
+  P.hd_hsrc = g.hd_hsrc;
   P.chg = g.chg;
   P.sl_cnt = g.sl_cnt;
   P.counters = g.counters;
@@ -999,10 +1071,12 @@ int launch_forward_cone(DevGraph& g, float n_sigma, float tau, void* stream) {
   P.n_sigma = n_sigma;
   P.tau = tau;
   P.inv_tau = tau > 0.f ? 1.0 / double(tau) : 0.0;
-  P.par = (++g.pass_fwd) & 1u;
+  // the cone pass is ordered by its barriers, not by parity: it rewrites the
+  // changed records with the CURRENT parity, so the records stay uniform and the
+  // next dataflow pass (new parity) can wait on them
+  P.par = g.pass_fwd & 1u;
   P.stamp = ++g.inc_epoch;
   const bool lse = tau > 0.f;
-  g.parity_mixed = true;   // clean heads keep the parity of the pass that last wrote them
   // large update batches: stage every level's topology (latency off the chain);
   // small ones: read only the dirty heads' topology
   const bool staged = g.pending_updates * 1000 > g.e;
