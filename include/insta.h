@@ -178,7 +178,13 @@ insta_status insta_arrivals(insta_graph* g, float* A, float* mean, float* sigma,
  * a separate per-level pass; d_arc_mean is bit-identical either way.
  * d_src: DEVICE float[num_pins][2] dL/d(src_mean) in caller pin order (0 at
  * non-source pins), or NULL.  Uses the tau/n_sigma of the last forward.
- * INSTA_E_STATE if the last forward is stale. */
+ * INSTA_E_STATE if the last forward is stale.  Accumulator range: every adjoint
+ * is bounded by S = sum_ep |ep_seed| (TNS: S <= num_endpoints); INSTA_E_ARG
+ * (nothing launched) unless S < 2^30 (schedules 0 and 3: 2^-32 fixed point in
+ * int64), S < 2^18 (schedules 1 and 2: heavy-driver words fold an arrival
+ * count above bit 44) or S < 2^38 (sigma channel), or if a seed is not
+ * finite.  A non-NULL ep_seed costs one device reduction and a synchronization
+ * for this check. */
 insta_status insta_backward(insta_graph* g, const float* ep_seed, float* d_arc_mean,
                             float* d_arc_sigma, float* d_src, void* cuda_stream);
 

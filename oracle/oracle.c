@@ -453,14 +453,19 @@ int orc_tie_taint(const orc_graph* g, double n_sigma, double eps, double margin,
       ft[2 * (int64_t)i + rf] = x;
     }
   }
-  /* backward taint originates at endpoints with ambiguous seeds or tainted state */
+  /* backward taint originates at endpoints whose seed (slack sign, rf*) is
+   * ambiguous: within eps of a kink, or within `margin` of one when the
+   * endpoint's state is tainted (a near tie upstream moves its arrival by less
+   * than margin).  A tainted endpoint whose seed is certain routes no uncertain
+   * adjoint: no taint (T2). */
   for (int32_t k = 0; k < g->num_endpoints; ++k) {
     int32_t p = g->ep_pin[k];
     double ar = mu[2 * (int64_t)p] + n_sigma * sig[2 * (int64_t)p];
     double af = mu[2 * (int64_t)p + 1] + n_sigma * sig[2 * (int64_t)p + 1];
     double sr = g->ep_rat[2 * k] - ar, sf = g->ep_rat[2 * k + 1] - af;
     double s = sf < sr ? sf : sr;
-    if (fabs(sr - sf) <= eps || fabs(s) <= eps || ft[2 * (int64_t)p] || ft[2 * (int64_t)p + 1]) {
+    double tol = (ft[2 * (int64_t)p] || ft[2 * (int64_t)p + 1]) ? margin : eps;
+    if (fabs(sr - sf) <= tol || fabs(s) <= tol) {
       bt[2 * (int64_t)p] = bt[2 * (int64_t)p + 1] = 1;
     }
   }

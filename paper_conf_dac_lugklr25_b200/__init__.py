@@ -142,6 +142,13 @@ class Graph:
             return ctypes.c_void_p(stream.cuda_stream)
         return _stream(self._torch, self.device)
 
+    def _dev(self, x, dtype, stream=None):
+        """A contiguous device copy of x allocated on the call's stream (the caching allocator then
+        never hands its memory to another stream while the library kernel still reads it)."""
+        t = self._torch
+        with t.cuda.stream(stream or t.cuda.current_stream(self.device)):
+            return t.as_tensor(x, dtype=dtype, device=self.device).contiguous()
+
     def forward(self, n_sigma: float = 3.0, tau: float = 0.0, schedule: int = 0, sync: bool = True,
                 stream=None, cone_max: int = 0):
         """insta_forward: arrivals -> endpoint slack -> WNS/TNS.  Returns a Summary if sync.
@@ -184,7 +191,10 @@ class Graph:
         d_src = t.empty((self.num_pins, 2), dtype=t.float32, device=self.device) if want_src else None
         seed = None
         if ep_seed is not None:
-            seed = t.as_tensor(ep_seed, dtype=t.float32, device=self.device).contiguous()
+            with t.cuda.stream(stream or t.cuda.current_stream(self.device)):   # allocated on the call's stream
+                seed = t.as_tensor(ep_seed, dtype=t.float32, device=self.device).contiguous()
+            if seed.numel() != self.num_endpoints:
+                raise ValueError(f"ep_seed: expected {self.num_endpoints} values, got {seed.numel()}")
         check(self.lib.insta_backward(self._h, _dptr(seed), _dptr(d_mean), _dptr(d_sig), _dptr(d_src),
                                       self._st(stream)), "insta_backward")
         outs = (d_mean,) + ((d_sig,) if want_sigma else ()) + ((d_src,) if want_src else ())
@@ -193,10 +203,15 @@ class Graph:
     def update_arcs(self, arc_ids, mean, sigma, incremental: bool = True, stream=None):
         """insta_update_arcs: re-annotate arcs (device or host arrays; copied to the device)."""
         t = self._torch
-        ids = None if arc_ids is None else t.as_tensor(arc_ids, dtype=t.int32, device=self.device).contiguous()
-        m = t.as_tensor(mean, dtype=t.float32, device=self.device).contiguous()
-        s = t.as_tensor(sigma, dtype=t.float32, device=self.device).contiguous()
+        # temporaries live on the stream the library call is ordered on (the caching allocator
+        # cannot hand their memory to another stream while the kernel still reads it)
+        with t.cuda.stream(stream or t.cuda.current_stream(self.device)):
+            ids = None if arc_ids is None else t.as_tensor(arc_ids, dtype=t.int32, device=self.device).contiguous()
+            m = t.as_tensor(mean, dtype=t.float32, device=self.device).contiguous()
+            s = t.as_tensor(sigma, dtype=t.float32, device=self.device).contiguous()
         n = self.num_arcs if ids is None else int(ids.numel())   # arc_ids None: every arc, caller order
+        if m.numel() != 2 * n or s.numel() != 2 * n:
+            raise ValueError(f"update_arcs: mean and sigma need {2 * n} values ([n][2]), got {m.numel()}, {s.numel()}")
         check(self.lib.insta_update_arcs(self._h, n, _dptr(ids), _dptr(m), _dptr(s),
                                          int(bool(incremental)), self._st(stream)), "insta_update_arcs")
 
@@ -269,7 +284,7 @@ class Graph:
         d_mean = t.empty((self.num_arcs, 2), dtype=t.float32, device=self.device)
         d_sig = t.empty((self.num_arcs, 2), dtype=t.float32, device=self.device) if want_sigma else None
         d_src = t.empty((self.num_pins, 2), dtype=t.float32, device=self.device) if want_src else None
-        seed = None if ep_seed is None else t.as_tensor(ep_seed, dtype=t.float32, device=self.device).contiguous()
+        seed = None if ep_seed is None else self._dev(ep_seed, t.float32, stream)
         check(self.lib.insta_clark_backward(self._h, _dptr(seed), _dptr(d_mean), _dptr(d_sig), _dptr(d_src),
                                             self._st(stream)), "insta_clark_backward")
         outs = (d_mean,) + ((d_sig,) if want_sigma else ()) + ((d_src,) if want_src else ())
@@ -279,7 +294,7 @@ class Graph:
     def stage_gradients(self, d_mean, stream=None):
         """insta_stage_gradients: float32[E] stage gradient per cell arc (0 for net arcs)."""
         t = self._torch
-        dm = t.as_tensor(d_mean, dtype=t.float32, device=self.device).contiguous()
+        dm = self._dev(d_mean, t.float32, stream)
         out = t.empty(self.num_arcs, dtype=t.float32, device=self.device)
         check(self.lib.insta_stage_gradients(self._h, _dptr(dm), _dptr(out), self._st(stream)), "insta_stage_gradients")
         return out
@@ -297,9 +312,9 @@ class Graph:
     def timing_loss(self, pin_x, pin_y, arc_w, lambda_rc: float = 1.0, want_grad: bool = True, stream=None):
         """insta_timing_loss: (L float64 device scalar, grad_x float32[N], grad_y float32[N]) of Eq 7."""
         t = self._torch
-        x = t.as_tensor(pin_x, dtype=t.float32, device=self.device).contiguous()
-        y = t.as_tensor(pin_y, dtype=t.float32, device=self.device).contiguous()
-        w = t.as_tensor(arc_w, dtype=t.float32, device=self.device).contiguous()
+        x = self._dev(pin_x, t.float32, stream)
+        y = self._dev(pin_y, t.float32, stream)
+        w = self._dev(arc_w, t.float32, stream)
         L = t.empty(1, dtype=t.float64, device=self.device)
         gx = t.empty(self.num_pins, dtype=t.float32, device=self.device) if want_grad else None
         gy = t.empty(self.num_pins, dtype=t.float32, device=self.device) if want_grad else None

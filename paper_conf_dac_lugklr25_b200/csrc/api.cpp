@@ -533,6 +533,25 @@ insta_status insta_backward(insta_graph* g, const float* ep_seed, float* d_arc_m
   if (!d_arc_mean && d.e > 0) return fail(INSTA_E_ARG, "backward: d_arc_mean is required");
   if (!d.fwd_valid) return fail(INSTA_E_STATE, "backward: no valid forward (call insta_forward)");
   cudaSetDevice(d.device);
+  // accumulator range (include/insta.h): every adjoint is bounded by sum |ep_seed|
+  // (TNS: the number of violating endpoints <= num_endpoints).  The sweep backward
+  // accumulates 2^-32 fixed point in int64; schedules 1 and 2 fold an arrival count
+  // into the words of heavy drivers (2^-24 units below bit 44); the sigma channel
+  // accumulates 2^-24 fixed point in int64.
+  const double limit = d_arc_sigma ? 0x1p38 : (d.bwd_schedule == 0 || d.bwd_schedule == 3) ? 0x1p30 : 0x1p18;
+  if (ep_seed) {
+    double sum = 0.0;
+    const int e2 = insta::seed_abs_sum(d, ep_seed, &sum, cuda_stream);
+    if (e2) return cuda_fail(e2, "backward");
+    if (!(sum < limit)) {
+      char msg[160];
+      snprintf(msg, sizeof msg, "backward: sum |ep_seed| = %g is not finite or exceeds the adjoint bound %g", sum,
+               limit);
+      return fail(INSTA_E_ARG, msg);
+    }
+  } else if (double(d.num_ep) >= limit) {
+    return fail(INSTA_E_ARG, "backward: too many endpoints for this schedule's accumulators (use schedule 0)");
+  }
   int err = insta::launch_backward(d, ep_seed, d_arc_mean, d_arc_sigma, d_src, cuda_stream);
   if (err) return cuda_fail(err, "backward");
   return INSTA_OK;
@@ -582,6 +601,8 @@ insta_status insta_forward_batch(insta_graph* g, int32_t num_scenarios, const in
   }
   cudaSetDevice(d.device);
   cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+  if (d_arc_mean_sum && d.num_ep >= (1 << 19))   // batched backward: count-folded heavy accumulators (TNS seeds)
+    return fail(INSTA_E_ARG, "forward_batch: gradients need num_endpoints < 2^19 (heavy accumulator range)");
   if (d_arc_mean_sum && d.e > 0) {
     cudaError_t e = cudaMemsetAsync(d_arc_mean_sum, 0, sizeof(float) * 2 * size_t(d.e), st);
     if (e != cudaSuccess) return cuda_fail(int(e), "forward_batch");

@@ -99,8 +99,9 @@ __device__ __forceinline__ Raw ldb_raw(const BParams& P, int j, int s) {
 }
 
 __device__ __forceinline__ void awaitb(const BParams& P, int j, int s, Raw& r) {
+  uint32_t npoll_ = 0;
   while (!raw_ready(r, P.par)) {
-    INSTA_POLL_SLEEP();
+    insta_poll_pause(npoll_);
     r = ldb_raw(P, j, s);
   }
 }
@@ -475,8 +476,9 @@ __device__ __forceinline__ float2 loadb_g(const BParams& P, int q, int s) {
   uint32_t a, b;
   const float2* p = P.bg + size_t(q) * kLanes + s;
   ld2_u32(p, a, b);
+  uint32_t npoll_ = 0;
   while (!g_ready(a, b, P.par)) {
-    INSTA_POLL_SLEEP();
+    insta_poll_pause(npoll_);
     ld2_u32(p, a, b);
   }
   return make_float2(stripf(a), stripf(b));
@@ -599,8 +601,9 @@ __global__ void __launch_bounds__(kThreads, 1) bwdb_kernel(BParams P) {
 #pragma unroll
             for (int j = 0; j < kPullChunk; ++j) {
               if (r + j < r1) {
+                uint32_t npoll_ = 0;
                 while (!g_ready(va[j], vb[j], P.par)) {
-                  INSTA_POLL_SLEEP();
+                  insta_poll_pause(npoll_);
                   ld2_u32(P.bg + size_t(qq[j]) * kLanes + s, va[j], vb[j]);
                 }
                 ax += stripf(va[j]);
@@ -613,9 +616,10 @@ __global__ void __launch_bounds__(kThreads, 1) bwdb_kernel(BParams P) {
             const long long target = __ldg(P.heavy_fo + slot);
             unsigned long long x, y;
             ld2_u64(acc, x, y);
+            uint32_t npoll_ = 0;
             while (((long long)x + (kCountUnitB >> 1)) >> 44 != target ||
                    ((long long)y + (kCountUnitB >> 1)) >> 44 != target) {
-              INSTA_POLL_SLEEP();
+              insta_poll_pause(npoll_);
               ld2_u64(acc, x, y);
             }
             asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %1};" ::"l"(acc), "l"(0ull) : "memory");
@@ -673,13 +677,21 @@ __global__ void set_flag_kernel(int n, const int32_t* __restrict__ pos, uint8_t*
 }
 
 // entry-space keys 2x (arc e) / 2x + 1 (arc e'): overridden bit 1 / bit 3
+// Override bits of entry x: bit 1 (arc e of the entry) or bit 3 (arc e' of
+// its folded pin).  Two keys of one micro-batch can hit the same byte (a cell
+// arc and the input net arc behind its folded pin), so the byte is updated
+// with a 32-bit atomic on its aligned word (a plain read-modify-write of the
+// byte could lose the other key's bit).
 __global__ void set_xflag_kernel(int n, const int32_t* __restrict__ key, uint8_t* flags, int on) {
   const int k = blockIdx.x * blockDim.x + threadIdx.x;
   if (k >= n) return;
   const int x = key[k] >> 1;
-  const uint8_t bit = (key[k] & 1) ? 8 : 2;
-  if (on) flags[x] |= bit;
-  else flags[x] &= uint8_t(~bit);
+  const uint32_t bit = (key[k] & 1) ? 8u : 2u;
+  const uintptr_t addr = reinterpret_cast<uintptr_t>(flags + x);
+  unsigned int* word = reinterpret_cast<unsigned int*>(addr & ~uintptr_t(3));
+  const uint32_t sh = uint32_t(addr & 3) * 8u;
+  if (on) atomicOr(word, bit << sh);
+  else atomicAnd(word, ~(bit << sh));
 }
 
 // ---------------------------------------------------------------- host side

@@ -21,6 +21,18 @@
 
 namespace insta {
 
+// Dataflow waits are bounded: a word that never arrives (which valid inputs
+// cannot cause; insta_backward / insta_forward_batch validate the adjoint
+// bound of the count-folded accumulators) aborts the kernel -- the launch
+// fails with an error -- instead of hanging the GPU.
+#ifndef INSTA_POLL_LIMIT
+#define INSTA_POLL_LIMIT (1u << 26)
+#endif
+__device__ __forceinline__ void insta_poll_pause(uint32_t& n) {
+  INSTA_POLL_SLEEP();
+  if (++n > INSTA_POLL_LIMIT) __trap();
+}
+
 constexpr int kUnateShiftC = 30;   // fin_src bits 30..31: unateness (internal.h kUnateShift)
 
 // --------------------------------------------------------------------------

@@ -334,6 +334,8 @@ int launch_forward_incremental(DevGraph& g, float n_sigma, float tau, void* stre
 int launch_slack(DevGraph& g, void* stream);
 int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float* d_arc_sigma, float* d_src,
                     void* stream);
+// sum |ep_seed| on the device (synchronizes)
+int seed_abs_sum(DevGraph& g, const float* seed, double* host_out, void* stream);
 int launch_update_arcs(DevGraph& g, int64_t n, const int32_t* ids, const float* mean,
                        const float* sigma, int incremental, void* stream);
 int launch_arrivals(DevGraph& g, float* A, float* mean, float* sigma, void* stream);

@@ -128,8 +128,9 @@ __device__ __forceinline__ Raw ld_state_raw(const KParams& P, int j) {
 // word carries this pass's parity.
 __device__ __forceinline__ void await_raw(const KParams& P, int j, Raw& r) {
   if (P.mode == 2) {
+    uint32_t npoll_ = 0;
     while (!raw_ready(r, P.par)) {
-      INSTA_POLL_SLEEP();
+      insta_poll_pause(npoll_);
       r = ld_state_raw(P, j);
     }
   }
@@ -926,8 +927,9 @@ __device__ __forceinline__ float2 heavy_read(const KParams& P, int slot) {
   const long long target = __ldg(P.heavy_fo + slot);
   unsigned long long x, y;
   ld2_u64(P.heavy_acc + 2 * slot, x, y);
+  uint32_t npoll_ = 0;
   while (heavy_count((long long)x) != target || heavy_count((long long)y) != target) {
-    INSTA_POLL_SLEEP();
+    insta_poll_pause(npoll_);
     ld2_u64(P.heavy_acc + 2 * slot, x, y);
   }
   const long long vx = (long long)x - target * kCountUnit, vy = (long long)y - target * kCountUnit;
@@ -940,8 +942,9 @@ __device__ __forceinline__ float2 heavy_take(const KParams& P, int slot) {
   const long long target = __ldg(P.heavy_fo + slot);
   unsigned long long x, y;
   ld2_u64(P.heavy_acc + 2 * slot, x, y);
+  uint32_t npoll_ = 0;
   while (heavy_count((long long)x) != target || heavy_count((long long)y) != target) {
-    INSTA_POLL_SLEEP();
+    insta_poll_pause(npoll_);
     ld2_u64(P.heavy_acc + 2 * slot, x, y);
   }
   asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %1};" ::"l"(P.heavy_acc + 2 * slot), "l"(0ull) : "memory");
@@ -993,8 +996,9 @@ __device__ __forceinline__ void bwd_sink(const KParams& P, HeavyTab* tab, int nf
 // Per-arc adjoint words written by a sink (fanin position q)
 __device__ __forceinline__ void await_g(const KParams& P, int q, uint32_t& a, uint32_t& b) {
   if (P.mode == 2) {
+    uint32_t npoll_ = 0;
     while (((a & 1u) != P.par) || ((b & 1u) != P.par)) {
-      INSTA_POLL_SLEEP();
+      insta_poll_pause(npoll_);
       ld2_u32(P.g + q, a, b);
     }
   }
@@ -1967,6 +1971,30 @@ int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float*
   return launch_items(lse ? (const void*)bwd_kernel<true> : (const void*)bwd_kernel<false>, kThreads,
                       lse ? bwd_smem<true>() : bwd_smem<false>(),
                       P, g.bwd_items, true, st);
+}
+
+// sum |ep_seed| (the bound on every adjoint and accumulator partial sum:
+// weights are convex, so |dL/dA_j| <= sum_ep |dL/dslack_ep|); NaN propagates
+__global__ void seed_abs_sum_kernel(int n, const float* __restrict__ seed, double* out) {
+  double v = 0.0;
+  for (int k = blockIdx.x * blockDim.x + threadIdx.x; k < n; k += gridDim.x * blockDim.x) v += fabs(double(seed[k]));
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xffffffffu, v, o);
+  if ((threadIdx.x & 31) == 0 && v != 0.0) atomicAdd(out, v);
+  if ((threadIdx.x & 31) == 0 && v != v) atomicAdd(out, v);
+}
+
+int seed_abs_sum(DevGraph& g, const float* seed, double* host_out, void* stream) {
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  *host_out = 0.0;
+  if (g.num_ep == 0) return 0;
+  cudaError_t e = cudaMemsetAsync(g.summary + 3, 0, sizeof(double), st);
+  if (e != cudaSuccess) return int(e);
+  const int blocks = std::min((g.num_ep + 255) / 256, 1184);
+  seed_abs_sum_kernel<<<blocks, 256, 0, st>>>(g.num_ep, seed, g.summary + 3);
+  e = cudaGetLastError();
+  if (e == cudaSuccess) e = cudaMemcpyAsync(host_out, g.summary + 3, sizeof(double), cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  return int(e);
 }
 
 int launch_update_arcs(DevGraph& g, int64_t n, const int32_t* ids, const float* mean,

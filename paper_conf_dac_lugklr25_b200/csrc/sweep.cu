@@ -129,10 +129,11 @@ __device__ __forceinline__ void grid_sync_ctr(uint32_t* bar, uint32_t target, un
     if (trace) trace[512 + size_t(target / gridDim.x) * gridDim.x + blockIdx.x] = gtimer();
 #ifndef INSTA_SL_NOBAR
     asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(bar) : "memory");
-    uint32_t v;
+    uint32_t v, npoll = 0;
     for (;;) {
       asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(bar) : "memory");
       if (v >= target) break;
+      if (++npoll > (1u << 26)) __trap();   // bounded: never a silent hang
     }
 #endif
     if (trace && blockIdx.x == 0) trace[target / gridDim.x] = gtimer();

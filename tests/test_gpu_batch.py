@@ -109,3 +109,27 @@ def test_batch_forward_only_and_errors():
     with pytest.raises(insta.InstaError, match="E_ARG"):
         G.forward_batch([dict(delta_arc=np.array([10 ** 8]), delta_mean=np.zeros((1, 2)), delta_sigma=np.zeros((1, 2)))])
     G.close()
+
+
+@pytest.mark.parametrize("tau", [0.0, 1.0])
+def test_batch_sizing_candidates_with_input_nets(tau):
+    """C5 sizing candidates (synth.sizing_scenario): a cell's arcs AND its input net arcs are
+    overridden in one scenario, so a cell arc and the net arc behind its folded input pin share an
+    entry (override bits 1 and 3 of one flag byte, set concurrently).  Every scenario equals
+    insta_forward on its materialized graph, and clearing the overrides restores the base."""
+    g = synth.generate("C2")
+    scs = [synth.sizing_scenario(g, s) for s in range(512, 512 + 64)]
+    assert any(len(sc["delta_arc"]) > 4 for sc in scs)
+    G = insta.Graph(g)
+    base = G.forward(3.0, tau)
+    summ, _ = G.forward_batch(scs, tau=tau)
+    summ = summ.cpu().numpy()
+    again, _ = G.forward_batch([dict(n_sigma=3.0, derate_cell=1.0, derate_net=1.0)], tau=tau)
+    assert again.cpu().numpy()[0, 1] == pytest.approx(base.tns, rel=1e-12)   # no stale override bits
+    G.close()
+    for k, sc in enumerate(scs):
+        H = insta.Graph(materialize(g, sc))
+        s = H.forward(3.0, tau)
+        H.close()
+        assert summ[k, 0] == s.wns and summ[k, 2] == s.num_violations, k
+        assert summ[k, 1] == pytest.approx(s.tns, rel=1e-12, abs=1e-9), k
