@@ -6,8 +6,10 @@ A step = one full evaluation of the hot path on the 15M-pin synthetic graph
 levels + endpoint slack + WNS/TNS) followed by insta_backward (dTNS/d(arc
 mean) for every arc).  value = pins processed per second (whole job: N ranks x
 pins / max-over-ranks step time).  With N > 1 each rank evaluates its own
-independent scenario of the same graph (weak scaling; no data-path collective,
-one all_reduce of the timing at the end).
+independent replica of the same graph (weak scaling; no data-path collective,
+one all_reduce of the timing at the end); the C5 batched leg shards 1024
+scenarios over the ranks.  `--gpus N` without torchrun re-launches itself
+with torch.distributed.run (one process per GPU).
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--tau 0] [--schedule 0]
   python bench.py --impl reference ...   # the fp64 CPU oracle on the box's host cores
@@ -104,57 +106,27 @@ class ClockSampler:
 HEAVY_FANOUT = 256   # csrc/internal.h kHeavyFanout: drivers above it use the atomic path
 
 
-def fwd_bytes(N, E, n_src, P, lse):
-    """insta_forward: propagation kernel + slack/TNS kernel."""
-    return (4 * (N - n_src) + 4           # fanin row pointers
-            + 20 * E                      # per arc: source word 4 + {mu,sigma}x{R,F} 16 (TMA-staged)
-            + 24 * E                      # per arc: source state gather {mu_R, mu_F (f64), sigma_R, sigma_F}
-            + 24 * N                      # state write
-            + 16 * n_src                  # startpoint (clock) arrival read
-            + (16 * E if lse else 4 * (N - n_src))   # Eq 6 weights per arc (LSE) / arg-max per pin (hard)
-            + 41 * P)                     # slack: ep pin 4 + RAT 8 + state 24 + slack 4 + rf 1
+def survey_bytes(N, E, P, lse):
+    """SURVEY.md §8(d) algorithmic bytes (fp32 16 B state, 20 B arc record; the roofline's model):
+    forward 20 B/pin + 36 B/arc (+8 B/arc Eq 6 weights in LSE) + 32 B/endpoint;
+    backward (mean channel, stored weights) 12 B/pin + 28 B/arc + 12 B/endpoint."""
+    fwd = 20 * N + (44 if lse else 36) * E + 32 * P
+    bwd = 12 * N + 28 * E + 12 * P
+    return fwd, bwd
 
 
-def bwd_bytes(N, E, E_light, P, nnz_arcs, lse):
-    """insta_backward: prologue kernel (seeds + zero fill) + propagation kernel."""
-    return (8 * E                         # d_mean zero fill
-            + 17 * P                      # seeds: ep pin 4 + slack 4 + rf 1 + seed write 8
-            + 24 * N                      # per pin: light-fanout ptr 4, fanin ptr 4, seed 8, heavy slot 4, + 4
-            + (16 * E if lse else 0)      # Eq 6 weights (LSE); the hard arg-max is in the 24 B/pin above
-            + 12 * E_light                # pull: fanout entry 4 + per-arc adjoint gather 8
-            + 16 * E                      # per arc: source word 4 + arc id 4 + per-arc adjoint write 8
-            + 8 * nnz_arcs)               # nonzero d_mean scatter
-
-
-def fwd_bytes_folded(sc, N, E, n_src, P, lse):
-    """insta_forward, stage-folded persistent schedule: per head a row pointer
-    and its pin (+ first fanin position in LSE mode); per entry a source word, the record of its
-    arc and ONE source-state gather; a folded pin adds its word and the record of its fanin arc;
-    every pin's state is written once."""
+def sched0_bytes(sc, N, E, n_src, P, nnz_arcs, lse):
+    """Bytes the default schedule's kernels move (this layout): forward (stage-folded
+    dataflow kernel, folded pins kept in registers) 8 B/head (row, pin) + per entry 20 B (source
+    word, record of e) + a 32 B source-record gather + 20 B/folded pin (word, record of e') + a 32 B
+    record store per head + arg-max 4 B/head (hard) or Eq 6 weights 16 B/entry (LSE) + 16 B/startpoint
+    + 41 B/endpoint (slack); backward (sweep) 8 B/arc zero fill + 25 B/endpoint seeds + per head
+    52 B (row 4, seed 8, arg-max 4, accumulator read + clear 32; LSE: no arg-max) + per entry 20 B
+    topology (+16 B weights in LSE) + 16 B share pushed + 8 B per nonzero gradient."""
     H, X, F = sc["num_heads"], sc["num_entries"], sc["num_folded"]
-    return (8 * H + (4 * H if lse else 0)     # head row pointer + pin (+ first fanin position)
-            + 20 * X                          # per entry: source word 4 + record of e 16
-            + 24 * X                          # per entry: source-state gather
-            + F * (20 + (4 if lse else 0))    # folded pin: word 4 + record of e' 16 (+ fanin position)
-            + 24 * N                          # state write (every pin, folded ones included)
-            + 16 * n_src
-            + (16 * E if lse else 4 * (N - n_src))   # Eq 6 weights per arc (LSE) / arg-max per pin (hard)
-            + 41 * P)
-
-
-def bwd_bytes_folded(sc, N, E, E_light, P, nnz_arcs, lse):
-    """insta_backward, stage-folded schedule: per head 24 B (light-fanout and entry row pointers,
-    pin, heavy slot, seed) + its arg-max (hard); per entry 20 B (fanin position, source word,
-    arc ids of e and e', position of e') + the folded pin word (hard); Eq 6 weights of every arc
-    (LSE) or the folded pins' arg-max (hard); one adjoint word written per entry."""
-    H, X, F = sc["num_heads"], sc["num_entries"], sc["num_folded"]
-    return (8 * E + 25 * P                    # d_mean zero fill; seeds (canonical + head order)
-            + (24 if lse else 28) * H
-            + (20 if lse else 24) * X
-            + (16 * E if lse else 4 * F)
-            + 12 * E_light                    # pull: fanout entry 4 + per-arc adjoint gather 8
-            + 8 * X                           # per-arc adjoint write
-            + 8 * nnz_arcs)                   # nonzero d_mean scatter
+    fwd = (8 * H + 20 * X + 32 * X + 20 * F + 32 * H + (16 * X if lse else 4 * H) + 16 * n_src + 41 * P)
+    bwd = (8 * E + 25 * P + (48 if lse else 52) * H + (36 if lse else 20) * X + 16 * X + 8 * nnz_arcs)
+    return fwd, bwd
 
 
 def topk_bytes(g, K):
@@ -167,18 +139,34 @@ def topk_bytes(g, K):
     return 4 * (N - n_src) + 20 * E + (2 * E + 2 * n_non) * K * 20 + 2 * N * K * 20
 
 
-def cpu_oracle_sample(cfg_name, sample_pins, tau):
-    """fp64 CPU oracle (single thread) fwd + slack + bwd on a bounded sample of the workload:
-    the same generator recipe (depth, fanout law, endpoint fraction) at `sample_pins` pins."""
+def cpu_oracle_sample(cfg_name, sample_pins, tau, omp=False, g=None):
+    """fp64 CPU oracle fwd + slack + bwd on the workload (or a bounded sample of it: the same generator
+    recipe -- depth, fanout law, endpoint fraction -- at `sample_pins` pins).  omp: the OpenMP
+    level-parallel build of the same oracle on every host core."""
     import oracle  # test infrastructure: allowed in the cpu_baseline / reference leg only
-    g = synth.generate(cfg_name, pins=sample_pins)
+    if g is None:
+        g = synth.generate(cfg_name, pins=sample_pins)
     og = oracle.OGraph(g)
     t0 = time.perf_counter()
-    f = oracle.forward(og, 3.0, tau)
+    f = oracle.forward(og, 3.0, tau, omp=omp)
     oracle.slack(og, f["A"])
-    oracle.backward(og, 3.0, tau)
+    oracle.backward(og, 3.0, tau, omp=omp)
     dt = time.perf_counter() - t0
     return g.num_pins, dt
+
+
+def host_info():
+    cores = len(os.sched_getaffinity(0))
+    model = None
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            if line.startswith("Model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except Exception:
+        pass
+    return cores, model
 
 
 def run_reference(args, rank, world):
@@ -194,17 +182,38 @@ def run_reference(args, rank, world):
             times.append(dt)
     T = float(np.sum(times))
     val = npins * len(times) / T
+    cores, model = host_info()
     line = {
         "impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * T / len(times),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": f"{cfg.name} recipe, oracle sample of {npins} pins (full workload {cfg.pins} pins)",
                    "tau": args.tau, "n_sigma": 3.0},
-        "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle",
-                         "sample": f"{npins}-pin graph from the {cfg.name} generator recipe, fwd+slack+bwd"},
+        "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle", "cpu_model": model,
+                         "host_cores": cores,
+                         "sample": f"{npins}-pin graph from the {cfg.name} generator recipe, fwd+slack+bwd, 1 thread"},
         "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
+
+
+def timed_passes(G, stream, dev, steps, tau, schedule, d_mean, flush=None):
+    """CUDA-event time of insta_forward and insta_backward over `steps` passes on `stream`;
+    flush: a callable run before each pass outside the timed events (cold L2)."""
+    import torch
+    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(steps)]
+    for k in range(steps):
+        if flush is not None:
+            flush()
+        ev[k][0].record(stream)
+        G.forward(3.0, tau, schedule, sync=False, stream=stream)
+        ev[k][1].record(stream)
+        G.backward(out=d_mean, stream=stream)
+        ev[k][2].record(stream)
+    torch.cuda.synchronize(dev)
+    f = [ev[k][0].elapsed_time(ev[k][1]) for k in range(steps)]
+    b = [ev[k][1].elapsed_time(ev[k][2]) for k in range(steps)]
+    return float(np.mean(f)), float(np.mean(b)), float(np.median(f)), float(np.median(b))
 
 
 def main():
@@ -219,13 +228,27 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=20)
     ap.add_argument("--ref-sample-pins", type=int, default=1_500_000)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-full", type=int, default=1, help="cpu_baseline on the full workload (else the sample)")
     ap.add_argument("--batch-scenarios", type=int, default=1024, help="C5 batched evaluations (0 = skip)")
     ap.add_argument("--topk", type=int, default=32, help="Top-K CPPR propagation K (0 = skip)")
     ap.add_argument("--clark", type=int, default=1, help="time the Clark merge path (0 = skip)")
+    ap.add_argument("--lse", type=int, default=1, help="time the LSE (tau = 1 ps) fwd+bwd leg (0 = skip)")
+    ap.add_argument("--cold", type=int, default=1, help="time fwd+bwd with L2 flushed before every pass (0 = skip)")
     ap.add_argument("--incremental", type=int, default=1,
-                    help="time the incremental re-annotation + cone forward (a7) on 1%% sizing steps (0 = skip)")
+                    help="time incremental re-annotation (a7): C4 small updates, C3 1%% steps (0 = skip)")
+    ap.add_argument("--c3-steps", type=int, default=100)
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
+
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        # one process per GPU: re-launch under torch.distributed.run (rank 0 prints the line)
+        import socket
+        with socket.socket() as so:
+            so.bind(("127.0.0.1", 0))
+            port = so.getsockname()[1]
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+        sys.exit(subprocess.call(cmd))
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -251,14 +274,14 @@ def main():
     n_src = int(np.count_nonzero(np.bincount(g.arc_to, minlength=N) == 0))
     stream = torch.cuda.Stream(dev)
     d_mean = torch.empty((E, 2), dtype=torch.float32, device=dev)
+    sched = G.schedule()
+    peak, peak_kind = _peaks()
 
-    def step():
-        G.forward(3.0, args.tau, args.schedule, sync=False, stream=stream)
-        G.backward(out=d_mean, stream=stream)
-
+    # ---------------- the headline: C4 hard mode fwd+bwd, K timed passes -------------
     with torch.cuda.stream(stream):
         for _ in range(args.warmup):
-            step()
+            G.forward(3.0, args.tau, args.schedule, sync=False, stream=stream)
+            G.backward(out=d_mean, stream=stream)
         stream.synchronize()
         s = G.summary(stream=stream)
         K = args.steps
@@ -292,31 +315,68 @@ def main():
     ms_step = total_ms / args.steps
     value = world * N / (ms_step * 1e-3)
 
-    # byte model inputs: nonzero gradient arcs and light (pulled) fanout entries
+    # roofline: SURVEY §8(d) algorithmic bytes over the event-timed call; the dominant kernel
+    lse = args.tau > 0
     dm = d_mean.cpu().numpy()
     nnz_arcs = int(np.count_nonzero((dm != 0).any(axis=1)))
-    fo = np.bincount(g.arc_from, minlength=N)
-    E_light = int(fo[fo <= HEAVY_FANOUT].sum())
-    lse = args.tau > 0
-    sched = G.schedule()
-    if args.schedule == 0:   # stage-folded persistent passes
-        fb = fwd_bytes_folded(sched, N, E, n_src, P, lse)
-        bb = bwd_bytes_folded(sched, N, E, E_light, P, nnz_arcs, lse)
-    else:                    # one launch per level
-        fb = fwd_bytes(N, E, n_src, P, lse)
-        bb = bwd_bytes(N, E, E_light, P, nnz_arcs, lse)
-    peak, peak_kind = _peaks()
-    fwd_gbs = fb / (fwd_ms * 1e-3) / 1e9
-    bwd_gbs = bb / (bwd_ms * 1e-3) / 1e9
+    sfb, sbb = survey_bytes(N, E, P, lse)
+    kfb, kbb = sched0_bytes(sched, N, E, n_src, P, nnz_arcs, lse)
+    fwd_gbs, bwd_gbs = sfb / (fwd_ms * 1e-3) / 1e9, sbb / (bwd_ms * 1e-3) / 1e9
     dom = "fwd" if fwd_ms >= bwd_ms else "bwd"
     ach = fwd_gbs if dom == "fwd" else bwd_gbs
     traffic = None
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp):
         try:
-            traffic = json.load(open(tp)).get(f"{args.config}_{dom}_tau{args.tau:g}")
+            traffic = json.load(open(tp)).get(f"{args.config}_{dom}_tau{args.tau:g}_s{args.schedule}")
         except Exception:
             traffic = None
+    roofline = {
+        "bound": "hbm", "kernel": ("fwd_kernel<stage-folded dataflow> + slack_kernel (insta_forward)" if dom == "fwd"
+                                   else "bwd_prep_kernel + bwdl_kernel<sweep> (insta_backward)"),
+        "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak, "peak_kind": peak_kind,
+        "traffic": traffic, "traffic_source": "profiles/traffic.json: ncu --set full dram__bytes_read.sum + "
+                                              "dram__bytes_write.sum per launch, round 2",
+        "byte_model": "SURVEY.md 8(d): fwd 20 B/pin + 36 B/arc + 32 B/endpoint (+8 B/arc LSE), "
+                      "bwd 12 B/pin + 28 B/arc + 12 B/endpoint",
+        "fwd_alg_bytes": sfb, "bwd_alg_bytes": sbb, "fwd_gbs": fwd_gbs, "bwd_gbs": bwd_gbs,
+        "fwd_bwd_gbs": (sfb + sbb) / ((fwd_ms + bwd_ms) * 1e-3) / 1e9,
+        "fwd_bwd_frac": (sfb + sbb) / ((fwd_ms + bwd_ms) * 1e-3) / 1e9 / peak,
+        "kernel_layout_bytes": {"fwd": kfb, "bwd": kbb, "fwd_gbs": kfb / (fwd_ms * 1e-3) / 1e9,
+                                "bwd_gbs": kbb / (bwd_ms * 1e-3) / 1e9,
+                                "what": "bytes the default schedule's kernels move (bench.sched0_bytes, DESIGN.md §6)"},
+    }
+
+    # ---------------- LSE (tau = 1 ps): the differentiable mode (Eq 4, Eq 6) -------------
+    lse_leg = None
+    if args.lse and world == 1:
+        with torch.cuda.stream(stream):
+            for _ in range(3):
+                G.forward(3.0, 1.0, args.schedule, sync=False, stream=stream)
+                G.backward(out=d_mean, stream=stream)
+            lf, lb, _, _ = timed_passes(G, stream, dev, max(5, min(args.steps, 10)), 1.0, args.schedule, d_mean)
+            ls = G.summary(stream=stream)
+        lfb, lbb = survey_bytes(N, E, P, True)
+        lse_leg = {"tau": 1.0, "fwd_ms": lf, "bwd_ms": lb, "fwd_bwd_ms": lf + lb, "pins_per_s": N / ((lf + lb) * 1e-3),
+                   "fwd_gbs": lfb / (lf * 1e-3) / 1e9, "bwd_gbs": lbb / (lb * 1e-3) / 1e9,
+                   "fwd_frac": lfb / (lf * 1e-3) / 1e9 / peak, "bwd_frac": lbb / (lb * 1e-3) / 1e9 / peak,
+                   "fwd_bwd_frac": (lfb + lbb) / ((lf + lb) * 1e-3) / 1e9 / peak, "tns": ls.tns, "wns": ls.wns}
+
+    # ---------------- cold L2: a 512 MB write before every pass -------------
+    cold = None
+    if args.cold and world == 1:
+        junk = torch.empty(128 * 1024 * 1024, dtype=torch.float32, device=dev)
+
+        def flush():
+            junk.zero_()   # on the current stream (the pass's stream, below)
+
+        with torch.cuda.stream(stream):
+            cf, cb, cfm, cbm = timed_passes(G, stream, dev, max(5, min(args.steps, 10)), args.tau, args.schedule,
+                                            d_mean, flush)
+        del junk
+        cold = {"what": "512 MB buffer written before every pass (L2 = 126 MB), events around the pass only",
+                "fwd_ms": cf, "bwd_ms": cb, "fwd_bwd_ms": cf + cb,
+                "fwd_bwd_frac": (sfb + sbb) / ((cf + cb) * 1e-3) / 1e9 / peak}
 
     # ---------------- end to end through the public API with host buffers -------------
     # Every step: H2D of all arc delays (mean, sigma; pinned host memory), insta_update_arcs (every arc),
@@ -385,6 +445,47 @@ def main():
                        "slacks; steps pipelined over 3 streams (H2D k+1 and D2H k-1 overlap step k), "
                        f"{args.e2e_steps} steps, host wall clock"}
 
+    # ---------------- end to end, incremental (the sizing loop's step): 1 % re-annotation -------------
+    # Per step: H2D of the step's updated arcs (ids, mean, sigma from pinned memory), insta_update_arcs
+    # (incremental), insta_forward with the summary read back (synchronous: the host decides the next
+    # step on TNS), insta_backward into device memory (consumed on the device by insta_stage_gradients),
+    # D2H of the endpoint slacks.  Host wall clock.  Runs on a copy of the annotation: restored after.
+    e2e_inc = None
+    if args.e2e_steps > 0 and world == 1:
+        upd = [synth.sizing_step(g, 9000 + k, frac=0.01) for k in range(args.e2e_steps + 2)]
+        pinned = [tuple(torch.from_numpy(np.ascontiguousarray(x)).pin_memory() for x in u) for u in upd]
+        sl_h = torch.empty(P, dtype=torch.float32).pin_memory()
+        sl_d = torch.empty(P, dtype=torch.float32, device=dev)
+        h2d = 0
+        with torch.cuda.stream(stream):
+            G.forward(3.0, args.tau, args.schedule, stream=stream)
+            for k, (ih, mh, sh) in enumerate(pinned):
+                if k == 2:
+                    torch.cuda.synchronize(dev)
+                    t0 = time.perf_counter()
+                ids = ih.to(dev, non_blocking=True)
+                m = mh.to(dev, non_blocking=True)
+                sg = sh.to(dev, non_blocking=True)
+                if k >= 2:
+                    h2d += ih.numel() * 4 + mh.numel() * 4 + sh.numel() * 4
+                G.update_arcs(ids, m, sg, incremental=True, stream=stream)
+                summ_k = G.forward(3.0, args.tau, args.schedule, stream=stream)
+                G.backward(out=d_mean, stream=stream)
+                G.lib.insta_slack(G._h, sl_d.data_ptr(), None, stream.cuda_stream, None)
+                sl_h.copy_(sl_d, non_blocking=True)
+            stream.synchronize()
+            dt = (time.perf_counter() - t0) / args.e2e_steps
+            # restore the original annotation for the legs that follow
+            G.update_arcs(None, torch.as_tensor(g.arc_mean, device=dev), torch.as_tensor(g.arc_sigma, device=dev),
+                          incremental=False, stream=stream)
+            G.forward(3.0, args.tau, args.schedule, stream=stream)
+        e2e_inc = {"value": N / dt, "unit": UNIT, "ms_per_step": dt * 1e3,
+                   "h2d_bytes_per_step": int(h2d / args.e2e_steps), "d2h_bytes_per_step": int(P * 4 + 24),
+                   "tns_last": summ_k.tns,
+                   "what": "per step: H2D of a 1 % sizing update (synth.sizing_step: ids, mean, sigma), "
+                           "insta_update_arcs(incremental), insta_forward + summary read (sync), insta_backward "
+                           "(gradient stays on the device), D2H of the endpoint slacks; host wall clock"}
+
     # ---------------- batched scenarios (C5): 1024 evaluations sharded over the ranks -------------
     batched = None
     if args.batch_scenarios > 0:
@@ -426,7 +527,7 @@ def main():
 
     # ---------------- Top-K unique-startpoint propagation + CPPR slack -------------
     topk = None
-    if args.topk > 0:
+    if args.topk > 0 and world == 1:
         G.set_cppr_rat(*synth.cppr_rat_table(g))
         K = args.topk
         torch.cuda.synchronize(dev)
@@ -459,7 +560,7 @@ def main():
 
     # ---------------- Clark moment-matching merge -------------
     clark = None
-    if args.clark:
+    if args.clark and world == 1:
         with torch.cuda.stream(stream):
             for _ in range(2):
                 G.clark_forward(3.0, sync=False, stream=stream)
@@ -482,61 +583,95 @@ def main():
                              f"TNS backward", "fwd_ms": cf, "bwd_ms": cb, "pins_per_s": N / ((cf + cb) * 1e-3),
                  "tns": cs.tns, "wns": cs.wns, "violations": cs.num_violations}
 
-    # ---------------- incremental re-annotation: 1 % sizing steps -------------
-    # Runs last: it changes the graph's arcs.  Each step: insta_update_arcs of ~1 % of the arcs (device
-    # buffers) + insta_forward; incremental = cone dataflow pass, full = the same update then a full pass.
-    incremental = None
-    if args.incremental:
-        upd = [tuple(torch.as_tensor(x, device=dev) for x in synth.sizing_step(g, k, frac=0.01)) for k in range(6)]
-        res = {}
+    # ---------------- incremental re-annotation -------------
+    # Runs last: it changes the graph's arcs.  Each step: insta_update_arcs (device buffers, incremental)
+    # + insta_forward, CUDA events around both.  C4: small sizing updates (1 cell, ~1e-5, ~1e-4 of the arcs)
+    # take the cone pass (default policy, include/insta.h cone_max), against update + full pass.  C3
+    # (BASELINE configs[2]): 100 steps of 1 % sizing updates, default policy (a full pass: the cone of a
+    # random 1 % update reaches every level) and the cone pass forced, against update + full pass.
+    def inc_series(GG, gg, fracs_steps, modes, seed0):
+        out = {}
         with torch.cuda.stream(stream):
-            G.forward(3.0, args.tau, 0, stream=stream)   # a full pass first: the cone pass starts from its records
-            for mode in ("incremental", "full"):
-                ts, cone = [], []
-                for ids, m, sg in upd:
-                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                    e0.record(stream)
-                    G.update_arcs(ids, m, sg, incremental=(mode == "incremental"), stream=stream)
-                    G.forward(3.0, args.tau, 0, sync=False, stream=stream)
-                    e1.record(stream)
-                    stream.synchronize()
-                    ts.append(e0.elapsed_time(e1))
-                    cone.append(G.last_forward_stats() / N)
-                res[mode] = (float(np.median(ts[1:])), float(np.median(cone[1:])))
-        incremental = {"workload": f"{cfg.name}, 1 % of arcs re-annotated per step (synth.sizing_step: random cells, "
-                                   f"~{len(upd[0][0])} arcs), insta_update_arcs + insta_forward, median of steps 1-5",
-                       "incremental_ms": res["incremental"][0], "recomputed_frac": res["incremental"][1],
-                       "full_ms": res["full"][0]}
+            GG.forward(3.0, 0.0, 0, stream=stream)
+            for frac, nst in fracs_steps:
+                upd = [tuple(torch.as_tensor(x, device=dev) for x in synth.sizing_step(gg, seed0 + k, frac=frac))
+                       for k in range(nst)]
+                row = {"frac": frac, "arcs_per_step": int(np.mean([len(u[0]) for u in upd])), "steps": nst}
+                for mode, cmax in modes:
+                    ts, cone = [], []
+                    for ids, m, sg in upd:
+                        a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                        a0.record(stream)
+                        GG.update_arcs(ids, m, sg, incremental=(mode != "full"), stream=stream)
+                        GG.forward(3.0, 0.0, 0, sync=False, stream=stream, cone_max=cmax)
+                        a1.record(stream)
+                        stream.synchronize()
+                        ts.append(a0.elapsed_time(a1))
+                        cone.append(GG.last_forward_stats() / gg.num_pins)
+                    row[mode] = {"ms_median": float(np.median(ts[1:] if len(ts) > 1 else ts)),
+                                 "ms_mean": float(np.mean(ts)), "pins_recomputed_frac": float(np.median(cone))}
+                out[f"{frac:g}"] = row
+        return out
+
+    incremental = None
+    if args.incremental and world == 1:
+        big = 10 ** 12
+        c4 = inc_series(G, g, [(1e-7, 20), (1e-5, 20), (1e-4, 10)], [("incremental", 0), ("full", 0)], 7000)
+        incremental = {"C4_small_updates": c4,
+                       "what": "per step: insta_update_arcs + insta_forward (CUDA events); incremental = default "
+                               "policy (cone pass for <= max(64, E/1e5) updated arcs), full = the same updates "
+                               "then a full pass"}
+        try:
+            g3 = synth.generate("C3")
+            G3 = insta.Graph(g3, device=local)
+            c3 = inc_series(G3, g3, [(0.01, args.c3_steps)],
+                            [("incremental", 0), ("cone_forced", big), ("full", 0)], 3030)
+            G3.close()
+            row = c3["0.01"]
+            incremental["C3_1pct_steps"] = row
+            incremental["C3_speedup_vs_full"] = {m: row["full"]["ms_median"] / row[m]["ms_median"]
+                                                 for m in ("incremental", "cone_forced")}
+        except Exception as ex:  # pragma: no cover
+            incremental["C3_1pct_steps"] = f"failed: {ex}"
 
     cpu = None
-    if rank == 0 and not args.no_cpu_baseline:
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cores, model = host_info()
         try:
-            npins, dt = cpu_oracle_sample(args.config, args.ref_sample_pins, args.tau)
-            cpu = {"value": npins / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
-                   "sample": f"{npins}-pin graph from the {cfg.name} generator recipe, fp64 fwd+slack+bwd, 1 run"}
+            gg = g if args.cpu_full else None
+            npins, dt = cpu_oracle_sample(args.config, args.ref_sample_pins, args.tau, omp=False, g=gg)
+            npo, dto = cpu_oracle_sample(args.config, args.ref_sample_pins, args.tau, omp=True, g=gg)
+            what = "the full workload" if args.cpu_full else f"a {npins}-pin sample of the {cfg.name} recipe"
+            cpu = {"value": npins / dt, "unit": UNIT, "cores": 1, "kind": "oracle", "cpu_model": model,
+                   "host_cores": cores,
+                   "sample": f"{what} ({npins} pins), fp64 fwd+slack+bwd, 1 run, 1 thread",
+                   "all_cores": {"value": npo / dto, "unit": UNIT, "cores": cores,
+                                 "what": "OpenMP level-parallel build of the same oracle (pins of a level in "
+                                         "parallel), all cores in the affinity mask, 1 run"}}
         except Exception as ex:  # pragma: no cover
             cpu = {"value": None, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": f"failed: {ex}"}
 
-    launches_per_step = 4 if args.schedule == 0 else 2 * G.num_levels + 2
+    launches_per_step = 4 if args.schedule in (0, 2, 3) else 2 * G.num_levels + 2
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
-            "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": f"{cfg.name}: synthetic 3nm-shaped timing graph, {N} pins, {E} arcs, "
                                    f"{P} endpoints, {G.num_levels} levels",
                        "pins": N, "arcs": E, "endpoints": P, "levels": G.num_levels, "tau": args.tau,
-                       "n_sigma": 3.0, "schedule": ["persistent, stage-folded", "per-level"][args.schedule],
+                       "n_sigma": 3.0, "schedule": {0: "dataflow forward + sweep backward", 1: "per-level",
+                                                    2: "dataflow forward + dataflow backward",
+                                                    3: "sweep forward + sweep backward"}[args.schedule],
                        "super_levels": sched["num_super_levels"], "folded_pins": sched["num_folded"],
-                       "parallelism": f"replicas x{world}", "l2": "working set > 126 MB L2 (no flush needed)",
-                       "tns": s.tns, "wns": s.wns, "violations": s.num_violations},
+                       "parallelism": f"replicas x{world}",
+                       "l2": "working set > 126 MB L2 (no flush between passes; the `cold` leg flushes)",
+                       "tns": s.tns, "wns": s.wns, "violations": s.num_violations,
+                       "precision": "fp32 inputs, fp64 mean/variance state, fp32 sqrt/exp, fp64 TNS"},
             "fwd_ms": fwd_ms, "bwd_ms": bwd_ms, "fwd_bwd_ms": ms_step,
             "fwd_pins_per_s": N / (fwd_ms * 1e-3),
-            "roofline": {"bound": "hbm", "kernel": "fwd_persistent(+slack)" if dom == "fwd" else
-                         "bwd_persistent(+prologue: seeds, zero fill)", "achieved": ach, "peak": peak, "unit": "GB/s",
-                         "frac": ach / peak, "peak_kind": peak_kind, "traffic": traffic,
-                         "fwd_gbs": fwd_gbs, "bwd_gbs": bwd_gbs, "fwd_alg_bytes": fb, "bwd_alg_bytes": bb},
-            "cpu_baseline": cpu, "e2e": e2e, "clocks": clk, "gpu_launches": launches_per_step * args.steps,
+            "roofline": roofline, "lse": lse_leg, "cold": cold,
+            "cpu_baseline": cpu, "e2e": e2e, "e2e_incremental": e2e_inc, "clocks": clk, "gpu_launches": launches_per_step * args.steps,
             "batched": batched, "topk": topk, "clark": clark, "incremental": incremental,
             "paper_context": "PAPER.md L9/L37: full-graph propagation < 0.1 s on a 15M-pin 3nm design, 1x A100 "
                              "(forward only, Top-K not stated); not the same metric",

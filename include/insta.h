@@ -228,6 +228,21 @@ typedef struct {
 insta_status insta_forward_batch(insta_graph* g, int32_t num_scenarios, const insta_scenario* sc, float tau,
                                  double* summaries, float* d_arc_mean_sum, void* cuda_stream);
 
+/* One-cell what-if evaluation through the cone pass (SURVEY §8(f) C5 sizing
+ * candidates, P:L156 INSTA-Size: "estimate the timing of each candidate"):
+ * candidate i re-annotates arcs arc_ids[cand_ptr[i] .. cand_ptr[i+1]) (caller
+ * ids, DEVICE int32) with mean / sigma (DEVICE float[..][2]); its summary
+ * {wns, tns, num_violations} goes to summaries[i] (DEVICE double[n][3]).  Each
+ * candidate is applied, evaluated with the cone pass (recomputing only what
+ * its arcs reach), and reverted with a second cone pass, so the summary equals
+ * insta_forward on the candidate's materialized graph bit for bit, and the
+ * graph is back to its base state on return.  cand_ptr: HOST int32[n + 1],
+ * ascending.  Needs a current forward of schedule 0 or 3 (E_STATE otherwise;
+ * uses its n_sigma / tau).  Asynchronous on cuda_stream. */
+insta_status insta_eval_candidates(insta_graph* g, int32_t num_candidates, const int32_t* cand_ptr,
+                                   const int32_t* arc_ids, const float* mean, const float* sigma, double* summaries,
+                                   void* cuda_stream);
+
 /* ---- Top-K unique-startpoint propagation with CPPR ----
  *
  * The paper's CPPR handling: every pin keeps, per transition rf, a

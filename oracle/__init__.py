@@ -17,19 +17,29 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _LIB = os.path.join(_HERE, "liboracle.so")
+_LIB_OMP = os.path.join(_HERE, "liboracle_omp.so")   # all-core build (bench cpu_baseline only)
 _lib = None
+_lib_omp = None
 
 
 def build(force: bool = False) -> str:
     src = os.path.join(_HERE, "oracle.c")
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(src):
-        subprocess.check_call(["gcc", "-O2", "-std=c11", "-ffp-contract=off", "-fPIC", "-shared",
-                               "-Wall", "-o", _LIB, src, "-lm"])
+    for out, extra in ((_LIB, []), (_LIB_OMP, ["-fopenmp"])):
+        if force or not os.path.exists(out) or os.path.getmtime(out) < os.path.getmtime(src):
+            subprocess.check_call(["gcc", "-O2", "-std=c11", "-ffp-contract=off", "-fPIC", "-shared",
+                                   "-Wall", *extra, "-o", out, src, "-lm"])
     return _LIB
 
 
-def lib():
-    global _lib
+def lib(omp: bool = False):
+    """The serial oracle, or (omp=True) the OpenMP level-parallel build of the same source: forward
+    identical, backward equal to rounding (atomic pushes), used only to time the all-core baseline."""
+    global _lib, _lib_omp
+    if omp:
+        if _lib_omp is None:
+            build()
+            _lib_omp = ctypes.CDLL(_LIB_OMP)
+        return _lib_omp
     if _lib is None:
         build()
         _lib = ctypes.CDLL(_LIB)
@@ -113,13 +123,13 @@ def levelize(num_pins, arc_from, arc_to):
     return out
 
 
-def forward(g, n_sigma=3.0, tau=0.0):
+def forward(g, n_sigma=3.0, tau=0.0, omp=False):
     """Returns dict(A, sigma, mu [N,2], win_arc, win_s [N,2], gap [N,2])."""
     og = _og(g)
     N = og.N
     A = np.zeros((N, 2)); sig = np.zeros((N, 2)); mu = np.zeros((N, 2))
     wa = np.zeros((N, 2), np.int32); ws = np.zeros((N, 2), np.int8); gap = np.zeros((N, 2))
-    L = lib()
+    L = lib(omp)
     L.orc_forward.argtypes = [ctypes.c_void_p, ctypes.c_double, ctypes.c_double] + [ctypes.c_void_p] * 6
     _check(L.orc_forward(ctypes.byref(og.c), float(n_sigma), float(tau), _p(A), _p(sig), _p(mu),
                          _p(wa), _p(ws), _p(gap)))
@@ -139,7 +149,7 @@ def slack(g, A):
     return dict(slack=s, rf_star=r, wns=wns.value, tns=tns.value, num_viol=nv.value)
 
 
-def backward(g, n_sigma=3.0, tau=0.0, dslack=None):
+def backward(g, n_sigma=3.0, tau=0.0, dslack=None, omp=False):
     """Returns dict(d_mean, d_sigma [E,2], d_src_mean, d_src_sigma, abar [N,2])."""
     og = _og(g)
     E, N = og.E, og.N
@@ -147,7 +157,7 @@ def backward(g, n_sigma=3.0, tau=0.0, dslack=None):
     dsm = np.zeros((N, 2)); dss = np.zeros((N, 2)); ab = np.zeros((N, 2))
     if dslack is not None:
         dslack = np.ascontiguousarray(dslack, np.float64)
-    L = lib()
+    L = lib(omp)
     L.orc_backward.argtypes = [ctypes.c_void_p, ctypes.c_double, ctypes.c_double] + [ctypes.c_void_p] * 6
     _check(L.orc_backward(ctypes.byref(og.c), float(n_sigma), float(tau), _p(dslack), _p(dm), _p(ds),
                           _p(dsm), _p(dss), _p(ab)))

@@ -83,11 +83,13 @@ typedef struct {
   int32_t *level, *order, *pos;         /* pos[p] = canonical position of pin p */
   int32_t *fanin_ptr, *fanin_arc;       /* over canonical positions            */
   int32_t *fanout_ptr, *fanout_arc;
+  int32_t *level_ptr;                   /* [num_levels + 1] canonical range of each level */
 } topo_t;
 
 static void topo_free(topo_t* t) {
   free(t->level); free(t->order); free(t->pos);
   free(t->fanin_ptr); free(t->fanin_arc); free(t->fanout_ptr); free(t->fanout_arc);
+  free(t->level_ptr);
   memset(t, 0, sizeof *t);
 }
 
@@ -135,6 +137,8 @@ static int topo_build(int32_t n, int64_t E, const int32_t* from, const int32_t* 
   int32_t* cnt = calloc((size_t)L + 1, sizeof(int32_t));
   for (int32_t p = 0; p < n; ++p) cnt[t->level[p] + 1]++;
   for (int32_t l = 0; l < L; ++l) cnt[l + 1] += cnt[l];
+  t->level_ptr = calloc((size_t)L + 2, sizeof(int32_t));
+  for (int32_t l = 0; l <= L; ++l) t->level_ptr[l] = cnt[l];
   for (int32_t p = 0; p < n; ++p) { int32_t k = cnt[t->level[p]]++; t->order[k] = p; t->pos[p] = k; }
   free(cnt);
 
@@ -227,49 +231,69 @@ static int max_fanin(const topo_t* t) {
   return m;
 }
 
-/* O3 + O4 + O5 over the whole graph; mu/sig are the per-pin state (Eq 1-2). */
-static void propagate(const orc_graph* g, const topo_t* t, double n_sigma, double tau,
-                      double* mu, double* sig, int32_t* win_arc, int8_t* win_s, double* gap) {
-  cand_t* c = malloc(sizeof(cand_t) * 2 * (size_t)max_fanin(t));
-  for (int32_t k = 0; k < t->n; ++k) {
-    int32_t i = t->order[k];
-    if (t->fanin_ptr[k] == t->fanin_ptr[k + 1]) {
-      /* O3: startpoint -- clock arrival distribution, corner via Eq 3 */
-      for (int rf = 0; rf < 2; ++rf) {
-        mu[2 * (int64_t)i + rf] = g->src_mean ? g->src_mean[2 * (int64_t)i + rf] : 0.0;
-        sig[2 * (int64_t)i + rf] = g->src_sigma ? g->src_sigma[2 * (int64_t)i + rf] : 0.0;
-        if (win_arc) win_arc[2 * (int64_t)i + rf] = -1;
-        if (win_s) win_s[2 * (int64_t)i + rf] = -1;
-        if (gap) gap[2 * (int64_t)i + rf] = INFINITY;
-      }
-      continue;
-    }
+/* O3 + O4 + O5 for the pin at canonical position k; mu/sig are the per-pin
+ * state (Eq 1-2); c: candidate scratch. */
+static void propagate_pin(const orc_graph* g, const topo_t* t, int32_t k, double n_sigma, double tau,
+                          double* mu, double* sig, int32_t* win_arc, int8_t* win_s, double* gap, cand_t* c) {
+  int32_t i = t->order[k];
+  if (t->fanin_ptr[k] == t->fanin_ptr[k + 1]) {
+    /* O3: startpoint -- clock arrival distribution, corner via Eq 3 */
     for (int rf = 0; rf < 2; ++rf) {
-      int n = candidates(g, t, k, rf, n_sigma, mu, sig, c);
-      int b = first_argmax(c, n);
-      if (tau == 0.0) {
-        /* hard: Alg 1 + Alg 2 with K = 1 -- keep the distribution of the max */
-        mu[2 * (int64_t)i + rf] = c[b].mu;
-        sig[2 * (int64_t)i + rf] = c[b].sig;
-      } else {
-        /* LSE (Eq 4): A_i = M + tau * log(sum exp((A_c - M)/tau)), M = max.
-         * Reading #1: sigma_i = sigma of the arg-max; mu_i = A_i - N_sigma*sigma_i. */
-        double M = c[b].A, sum = 0.0;
-        for (int a = 0; a < n; ++a) sum += exp((c[a].A - M) / tau);
-        double A_i = M + tau * log(sum);
-        sig[2 * (int64_t)i + rf] = c[b].sig;
-        mu[2 * (int64_t)i + rf] = A_i - n_sigma * c[b].sig;
-      }
-      if (win_arc) win_arc[2 * (int64_t)i + rf] = c[b].arc;
-      if (win_s) win_s[2 * (int64_t)i + rf] = (int8_t)c[b].s;
-      if (gap) {
-        double second = -INFINITY;
-        for (int a = 0; a < n; ++a) if (a != b && c[a].A > second) second = c[a].A;
-        gap[2 * (int64_t)i + rf] = (n > 1) ? c[b].A - second : INFINITY;
-      }
+      mu[2 * (int64_t)i + rf] = g->src_mean ? g->src_mean[2 * (int64_t)i + rf] : 0.0;
+      sig[2 * (int64_t)i + rf] = g->src_sigma ? g->src_sigma[2 * (int64_t)i + rf] : 0.0;
+      if (win_arc) win_arc[2 * (int64_t)i + rf] = -1;
+      if (win_s) win_s[2 * (int64_t)i + rf] = -1;
+      if (gap) gap[2 * (int64_t)i + rf] = INFINITY;
+    }
+    return;
+  }
+  for (int rf = 0; rf < 2; ++rf) {
+    int n = candidates(g, t, k, rf, n_sigma, mu, sig, c);
+    int b = first_argmax(c, n);
+    if (tau == 0.0) {
+      /* hard: Alg 1 + Alg 2 with K = 1 -- keep the distribution of the max */
+      mu[2 * (int64_t)i + rf] = c[b].mu;
+      sig[2 * (int64_t)i + rf] = c[b].sig;
+    } else {
+      /* LSE (Eq 4): A_i = M + tau * log(sum exp((A_c - M)/tau)), M = max.
+       * Reading #1: sigma_i = sigma of the arg-max; mu_i = A_i - N_sigma*sigma_i. */
+      double M = c[b].A, sum = 0.0;
+      for (int a = 0; a < n; ++a) sum += exp((c[a].A - M) / tau);
+      double A_i = M + tau * log(sum);
+      sig[2 * (int64_t)i + rf] = c[b].sig;
+      mu[2 * (int64_t)i + rf] = A_i - n_sigma * c[b].sig;
+    }
+    if (win_arc) win_arc[2 * (int64_t)i + rf] = c[b].arc;
+    if (win_s) win_s[2 * (int64_t)i + rf] = (int8_t)c[b].s;
+    if (gap) {
+      double second = -INFINITY;
+      for (int a = 0; a < n; ++a) if (a != b && c[a].A > second) second = c[a].A;
+      gap[2 * (int64_t)i + rf] = (n > 1) ? c[b].A - second : INFINITY;
     }
   }
+}
+
+/* Over the whole graph in canonical order.  The OpenMP build (liboracle_omp,
+ * the bench's all-core CPU baseline) runs the pins of one level in parallel:
+ * they only read earlier levels, so the result is the same. */
+static void propagate(const orc_graph* g, const topo_t* t, double n_sigma, double tau,
+                      double* mu, double* sig, int32_t* win_arc, int8_t* win_s, double* gap) {
+#ifdef _OPENMP
+  for (int32_t l = 0; l < t->num_levels; ++l) {
+#pragma omp parallel
+    {
+      cand_t* c = malloc(sizeof(cand_t) * 2 * (size_t)max_fanin(t));
+#pragma omp for schedule(static)
+      for (int32_t k = t->level_ptr[l]; k < t->level_ptr[l + 1]; ++k)
+        propagate_pin(g, t, k, n_sigma, tau, mu, sig, win_arc, win_s, gap, c);
+      free(c);
+    }
+  }
+#else
+  cand_t* c = malloc(sizeof(cand_t) * 2 * (size_t)max_fanin(t));
+  for (int32_t k = 0; k < t->n; ++k) propagate_pin(g, t, k, n_sigma, tau, mu, sig, win_arc, win_s, gap, c);
   free(c);
+#endif
 }
 
 int orc_forward(const orc_graph* g, double n_sigma, double tau, double* A,
@@ -333,6 +357,47 @@ int orc_slack(const orc_graph* g, const double* A, double* slack,
 /*   sbar_j[s] += sbar_c*sig_j[s]/sig_c, dsigma_e[rf] += sbar_c*sig_e/sig_c   */
 /*   (0/0 := 0).                                                              */
 /* ------------------------------------------------------------------------- */
+#ifdef _OPENMP
+#define ORC_PUSH(x, v) do { double v_ = (v); _Pragma("omp atomic") (x) += v_; } while (0)
+#else
+#define ORC_PUSH(x, v) ((x) += (v))
+#endif
+static void backward_pin(const orc_graph* g, const topo_t* t, int32_t k, double n_sigma, double tau,
+                         const double* mu, const double* sig, double* mbar, double* sbar, double* dm, double* ds,
+                         cand_t* c, double* w) {
+  int32_t i = t->order[k];
+  if (t->fanin_ptr[k] == t->fanin_ptr[k + 1]) return;
+  for (int rf = 0; rf < 2; ++rf) {
+    double mb = mbar[2 * (int64_t)i + rf], sb = sbar[2 * (int64_t)i + rf];
+    if (mb == 0.0 && sb == 0.0) continue;
+    int n = candidates(g, t, k, rf, n_sigma, mu, sig, c);
+    int b = first_argmax(c, n);
+    if (tau == 0.0) {
+      for (int a = 0; a < n; ++a) w[a] = (a == b) ? 1.0 : 0.0;
+    } else {
+      double M = c[b].A, sum = 0.0;
+      for (int a = 0; a < n; ++a) sum += exp((c[a].A - M) / tau);
+      for (int a = 0; a < n; ++a) w[a] = exp((c[a].A - M) / tau) / sum;   /* Eq 6 */
+    }
+    for (int a = 0; a < n; ++a) {
+      double Abar_c = w[a] * mb;
+      double mbar_c = Abar_c;
+      double sbar_c = n_sigma * Abar_c + ((a == b) ? (sb - n_sigma * mb) : 0.0);
+      int64_t e = c[a].arc;
+      int32_t j = c[a].src;
+      int s = c[a].s;
+      double sig_j = sig[2 * (int64_t)j + s];
+      double sig_e = g->arc_sigma[2 * e + rf];
+      ORC_PUSH(mbar[2 * (int64_t)j + s], mbar_c);
+      dm[2 * e + rf] += mbar_c;   /* arc e has one sink: written by this pin only */
+      if (c[a].sig > 0.0) {
+        ORC_PUSH(sbar[2 * (int64_t)j + s], sbar_c * sig_j / c[a].sig);
+        ds[2 * e + rf] += sbar_c * sig_e / c[a].sig;
+      }
+    }
+  }
+}
+
 int orc_backward(const orc_graph* g, double n_sigma, double tau,
                  const double* dslack, double* d_mean, double* d_sigma,
                  double* d_src_mean, double* d_src_sigma, double* abar) {
@@ -365,42 +430,26 @@ int orc_backward(const orc_graph* g, double n_sigma, double tau,
     sbar[2 * (int64_t)p + r] += -n_sigma * seed;
   }
 
-  cand_t* c = malloc(sizeof(cand_t) * 2 * (size_t)max_fanin(&t));
-  double* w = malloc(sizeof(double) * 2 * (size_t)max_fanin(&t));
-  for (int32_t k = N - 1; k >= 0; --k) {
-    int32_t i = t.order[k];
-    if (t.fanin_ptr[k] == t.fanin_ptr[k + 1]) continue;
-    for (int rf = 0; rf < 2; ++rf) {
-      double mb = mbar[2 * (int64_t)i + rf], sb = sbar[2 * (int64_t)i + rf];
-      if (mb == 0.0 && sb == 0.0) continue;
-      int n = candidates(g, &t, k, rf, n_sigma, mu, sig, c);
-      int b = first_argmax(c, n);
-      if (tau == 0.0) {
-        for (int a = 0; a < n; ++a) w[a] = (a == b) ? 1.0 : 0.0;
-      } else {
-        double M = c[b].A, sum = 0.0;
-        for (int a = 0; a < n; ++a) sum += exp((c[a].A - M) / tau);
-        for (int a = 0; a < n; ++a) w[a] = exp((c[a].A - M) / tau) / sum;   /* Eq 6 */
-      }
-      for (int a = 0; a < n; ++a) {
-        double Abar_c = w[a] * mb;
-        double mbar_c = Abar_c;
-        double sbar_c = n_sigma * Abar_c + ((a == b) ? (sb - n_sigma * mb) : 0.0);
-        int64_t e = c[a].arc;
-        int32_t j = c[a].src;
-        int s = c[a].s;
-        double sig_j = sig[2 * (int64_t)j + s];
-        double sig_e = g->arc_sigma[2 * e + rf];
-        mbar[2 * (int64_t)j + s] += mbar_c;
-        dm[2 * e + rf] += mbar_c;
-        if (c[a].sig > 0.0) {
-          sbar[2 * (int64_t)j + s] += sbar_c * sig_j / c[a].sig;
-          ds[2 * e + rf] += sbar_c * sig_e / c[a].sig;
-        }
-      }
+#ifdef _OPENMP
+  /* all-core build: the pins of a level in parallel, pushes as atomic adds (the
+   * summation order of a source's adjoint varies: equal to rounding) */
+  for (int32_t l = t.num_levels - 1; l >= 0; --l) {
+#pragma omp parallel
+    {
+      cand_t* c = malloc(sizeof(cand_t) * 2 * (size_t)max_fanin(&t));
+      double* w = malloc(sizeof(double) * 2 * (size_t)max_fanin(&t));
+#pragma omp for schedule(static)
+      for (int32_t k = t.level_ptr[l]; k < t.level_ptr[l + 1]; ++k)
+        backward_pin(g, &t, k, n_sigma, tau, mu, sig, mbar, sbar, dm, ds, c, w);
+      free(c); free(w);
     }
   }
+#else
+  cand_t* c = malloc(sizeof(cand_t) * 2 * (size_t)max_fanin(&t));
+  double* w = malloc(sizeof(double) * 2 * (size_t)max_fanin(&t));
+  for (int32_t k = N - 1; k >= 0; --k) backward_pin(g, &t, k, n_sigma, tau, mu, sig, mbar, sbar, dm, ds, c, w);
   free(c); free(w);
+#endif
 
   if (d_mean) memcpy(d_mean, dm, sizeof(double) * 2 * (size_t)E);
   if (d_sigma) memcpy(d_sigma, ds, sizeof(double) * 2 * (size_t)E);

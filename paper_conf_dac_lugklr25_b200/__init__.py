@@ -353,6 +353,26 @@ class Graph:
               "insta_forward_batch")
         return summ, dsum
 
+    def eval_candidates(self, candidates, stream=None, summaries=None):
+        """insta_eval_candidates: what-if summaries of sparse re-annotations (dicts with delta_arc /
+        delta_mean / delta_sigma host arrays, e.g. synth.sizing_scenario), each applied, evaluated with the
+        cone pass and reverted.  Returns float64[n, 3] {wns, tns, num_violations} device tensor."""
+        t = self._torch
+        n = len(candidates)
+        ptr = np.zeros(n + 1, np.int32)
+        for k, c in enumerate(candidates):
+            ptr[k + 1] = ptr[k] + len(c["delta_arc"])
+        ids = np.concatenate([np.asarray(c["delta_arc"], np.int32) for c in candidates]) if n else np.zeros(0, np.int32)
+        m = np.concatenate([np.asarray(c["delta_mean"], np.float32).reshape(-1, 2) for c in candidates]) if n else \
+            np.zeros((0, 2), np.float32)
+        sg = np.concatenate([np.asarray(c["delta_sigma"], np.float32).reshape(-1, 2) for c in candidates]) if n else \
+            np.zeros((0, 2), np.float32)
+        di, dm, ds = (self._dev(x, dt, stream) for x, dt in ((ids, t.int32), (m, t.float32), (sg, t.float32)))
+        out = summaries if summaries is not None else t.empty((n, 3), dtype=t.float64, device=self.device)
+        check(self.lib.insta_eval_candidates(self._h, n, _ptr(ptr), _dptr(di), _dptr(dm), _dptr(ds), _dptr(out),
+                                             self._st(stream)), "insta_eval_candidates")
+        return out
+
     def last_forward_stats(self) -> int:
         v = ctypes.c_int64()
         check(self.lib.insta_last_forward_stats(self._h, ctypes.byref(v)), "insta_last_forward_stats")

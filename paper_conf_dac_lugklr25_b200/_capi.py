@@ -71,6 +71,7 @@ SIGNATURES = {
     "insta_last_forward_stats": (ctypes.c_int, [c_vp, c_vp]),
     "insta_forward_batch": (ctypes.c_int, [c_vp, ctypes.c_int32, ctypes.POINTER(insta_scenario), ctypes.c_float,
                                            c_vp, c_vp, c_vp]),
+    "insta_eval_candidates": (ctypes.c_int, [c_vp, ctypes.c_int32, c_vp, c_vp, c_vp, c_vp, c_vp, c_vp]),
     "insta_set_cppr_rat": (ctypes.c_int, [c_vp, c_vp, c_vp, c_vp]),
     "insta_topk_forward": (ctypes.c_int, [c_vp, ctypes.c_int32, ctypes.c_float, c_vp]),
     "insta_topk_slack": (ctypes.c_int, [c_vp, c_vp, c_vp, c_vp, ctypes.POINTER(insta_summary)]),

@@ -67,7 +67,8 @@ void free_graph(insta::DevGraph& d) {
                   d.cl_mv,     d.cl_pre,    d.cl_g,      d.cl_fo_ptr,  d.cl_fo_q,   d.cl_slack,
                   d.cl_rf,     d.cl_summary, d.cl_hv_list, d.cl_hv_of, d.cl_hv_sum, d.tl_partials, d.sz_tmp,
                   d.sl_ptr,    d.ext_sh,    d.hd_csl,    d.chg,       d.acc_h,     d.sl_bar,    d.sl_cnt,
-                  d.hwin,      d.ew,        d.fwin,      d.efw,       d.sl_slice,  d.hfo_ptr,   d.hfo,       d.hd_hsrc};
+                  d.hwin,      d.ew,        d.fwin,      d.efw,       d.sl_slice,  d.hfo_ptr,   d.hfo,       d.hd_hsrc,
+                  d.cand_old};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   if (d.b_stage_h) cudaFreeHost(d.b_stage_h);
@@ -574,6 +575,64 @@ insta_status insta_update_arcs(insta_graph* g, int64_t n, const int32_t* arc_ids
   if (incremental && !d.pending_full) d.pending_incremental = true;
   else d.pending_full = true;
   d.pending_updates += n;
+  return INSTA_OK;
+}
+
+insta_status insta_eval_candidates(insta_graph* g, int32_t num_candidates, const int32_t* cand_ptr,
+                                   const int32_t* arc_ids, const float* mean, const float* sigma, double* summaries,
+                                   void* cuda_stream) {
+  if (!g) return fail(INSTA_E_ARG, "eval_candidates: NULL graph");
+  insta::DevGraph& d = g->d;
+  if (num_candidates < 0 || (num_candidates > 0 && (!cand_ptr || !summaries)))
+    return fail(INSTA_E_ARG, "eval_candidates: bad arguments");
+  if (!d.fwd_valid || d.pending_full || d.pending_incremental || !d.sweep_valid)
+    return fail(INSTA_E_STATE, "eval_candidates: needs a current schedule-0/3 forward (call insta_forward)");
+  int32_t maxn = 0;
+  for (int32_t i = 0; i < num_candidates; ++i) {
+    const int32_t n = cand_ptr[i + 1] - cand_ptr[i];
+    if (n < 0 || cand_ptr[i] < 0) return fail(INSTA_E_ARG, "eval_candidates: cand_ptr not ascending");
+    maxn = std::max(maxn, n);
+  }
+  if (maxn > 0 && (!arc_ids || !mean || !sigma)) return fail(INSTA_E_ARG, "eval_candidates: NULL arc arrays");
+  cudaSetDevice(d.device);
+  cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+  if (maxn > d.cand_cap) {
+    if (d.cand_old) cudaFree(d.cand_old);
+    d.cand_old = nullptr;
+    d.cand_cap = 0;
+    cudaError_t e = cudaMalloc(reinterpret_cast<void**>(&d.cand_old), sizeof(float) * 4 * size_t(maxn));
+    if (e != cudaSuccess) return cuda_fail(int(e), "eval_candidates");
+    d.cand_cap = maxn;
+  }
+  const float n_sigma = d.last_n_sigma, tau = d.last_tau;
+  float* old_m = d.cand_old;
+  float* old_s = d.cand_old + 2 * size_t(std::max(maxn, 1));
+  for (int32_t i = 0; i < num_candidates; ++i) {
+    const int32_t off = cand_ptr[i], n = cand_ptr[i + 1] - off;
+    int err = 0;
+    if (n > 0) {
+      // apply: save the current records, re-annotate, cone pass, slack; revert: the saved records, cone pass
+      err = insta::launch_gather_arcs(d, n, arc_ids + off, old_m, old_s, st);
+      if (!err) err = insta::launch_update_arcs(d, n, arc_ids + off, mean + 2 * size_t(off), sigma + 2 * size_t(off), 1, st);
+      if (!err) err = insta::launch_forward_cone(d, n_sigma, tau, st);
+    }
+    if (!err) err = insta::launch_slack(d, st);
+    if (!err) err = int(cudaMemcpyAsync(summaries + 3 * size_t(i), d.summary, sizeof(double) * 3,
+                                        cudaMemcpyDeviceToDevice, st));
+    if (!err && n > 0) {
+      err = insta::launch_update_arcs(d, n, arc_ids + off, old_m, old_s, 1, st);
+      if (!err) err = insta::launch_forward_cone(d, n_sigma, tau, st);
+    }
+    if (err) {
+      d.fwd_valid = false;
+      d.pending_full = true;
+      return cuda_fail(err, "eval_candidates");
+    }
+  }
+  // every candidate reverted: the base state, bit for bit; its slack/summary are restored too
+  int err = insta::launch_slack(d, st);
+  if (err) return cuda_fail(err, "eval_candidates");
+  d.pending_updates = 0;
   return INSTA_OK;
 }
 

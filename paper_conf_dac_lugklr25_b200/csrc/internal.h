@@ -275,6 +275,9 @@ struct DevGraph {
   int32_t* cl_hv_of = nullptr;     // [n] index into cl_hv_list, -1 = narrow
   void* cl_hv_sum = nullptr;       // double2 [wide][2]
   std::vector<int32_t> cl_hv_ptr;  // [L+1]
+  // insta_eval_candidates: previous records of a candidate's arcs
+  float* cand_old = nullptr;       // [cand_cap][4] {mean R, F, sigma R, F}
+  int32_t cand_cap = 0;
   // INSTA-Size selection scratch (size.cu)
   void* sz_tmp = nullptr;
   size_t sz_cap = 0;
@@ -334,6 +337,7 @@ int launch_forward_incremental(DevGraph& g, float n_sigma, float tau, void* stre
 int launch_slack(DevGraph& g, void* stream);
 int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float* d_arc_sigma, float* d_src,
                     void* stream);
+int launch_gather_arcs(DevGraph& g, int n, const int32_t* ids, float* mean, float* sigma, void* stream);
 // sum |ep_seed| on the device (synchronizes)
 int seed_abs_sum(DevGraph& g, const float* seed, double* host_out, void* stream);
 int launch_update_arcs(DevGraph& g, int64_t n, const int32_t* ids, const float* mean,

@@ -1973,6 +1973,23 @@ int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float*
                       P, g.bwd_items, true, st);
 }
 
+// current (mean, sigma) of arcs ids[0..n) (caller ids) from the fanin-order records
+__global__ void gather_arcs_kernel(int n, const int32_t* __restrict__ ids, const int32_t* __restrict__ arc_pos,
+                                   const float4* __restrict__ fin_ms, float2* mean, float2* sigma) {
+  const int k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k >= n) return;
+  const float4 r = fin_ms[arc_pos[ids[k]]];
+  mean[k] = make_float2(r.x, r.y);
+  sigma[k] = make_float2(r.z, r.w);
+}
+
+int launch_gather_arcs(DevGraph& g, int n, const int32_t* ids, float* mean, float* sigma, void* stream) {
+  if (n <= 0) return 0;
+  gather_arcs_kernel<<<(n + 255) / 256, 256, 0, static_cast<cudaStream_t>(stream)>>>(
+      n, ids, g.arc_pos, g.fin_ms, reinterpret_cast<float2*>(mean), reinterpret_cast<float2*>(sigma));
+  return int(cudaGetLastError());
+}
+
 // sum |ep_seed| (the bound on every adjoint and accumulator partial sum:
 // weights are convex, so |dL/dA_j| <= sum_ep |dL/dslack_ep|); NaN propagates
 __global__ void seed_abs_sum_kernel(int n, const float* __restrict__ seed, double* out) {

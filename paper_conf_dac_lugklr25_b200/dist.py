@@ -37,6 +37,9 @@ def evaluate_sharded(evaluate, scenarios, n_grad: int, num_arcs: int, rank: int,
         s_g, d_g = evaluate([scenarios[s] for s in g_idx], True)
         summ[: len(g_idx)] = s_g
         grad += d_g
+    # the gradient sum is final once the gradient scenarios are done: its
+    # all_reduce runs (on NCCL's stream) while the forward-only scenarios compute
+    work = dist.all_reduce(grad, op=dist.ReduceOp.SUM, async_op=True) if world > 1 else None
     if f_idx:
         s_f, _ = evaluate([scenarios[s] for s in f_idx], False)
         summ[len(g_idx): len(g_idx) + len(f_idx)] = s_f
@@ -44,7 +47,7 @@ def evaluate_sharded(evaluate, scenarios, n_grad: int, num_arcs: int, rank: int,
         parts = [torch.empty_like(summ) for _ in range(world)]
         dist.all_gather(parts, summ)
         allsum = torch.cat(parts)
-        dist.all_reduce(grad, op=dist.ReduceOp.SUM)
+        work.wait()
         summ = allsum[:n]
     else:
         summ = summ[:n]

@@ -133,3 +133,25 @@ def test_batch_sizing_candidates_with_input_nets(tau):
         H.close()
         assert summ[k, 0] == s.wns and summ[k, 2] == s.num_violations, k
         assert summ[k, 1] == pytest.approx(s.tns, rel=1e-12, abs=1e-9), k
+
+
+@pytest.mark.parametrize("tau", [0.0, 1.0])
+def test_eval_candidates_cone(tau):
+    """insta_eval_candidates (C5 sizing candidates through the cone pass): every candidate's summary equals
+    insta_forward on its materialized graph bit for bit, and the graph returns to its base state."""
+    g = synth.generate("C2")
+    scs = [synth.sizing_scenario(g, s) for s in range(512, 512 + 24)]
+    G = insta.Graph(g)
+    base = G.forward(3.0, tau)
+    A0 = G.arrivals()[0].cpu().numpy()
+    d0 = G.backward().cpu().numpy()
+    summ = G.eval_candidates(scs).cpu().numpy()
+    assert np.array_equal(G.arrivals()[0].cpu().numpy(), A0)
+    assert np.array_equal(G.backward().cpu().numpy(), d0)
+    assert G.summary().tns == base.tns
+    G.close()
+    for k, sc in enumerate(scs):
+        H = insta.Graph(materialize(g, sc))
+        s = H.forward(3.0, tau)
+        H.close()
+        assert summ[k, 0] == s.wns and summ[k, 1] == s.tns and summ[k, 2] == s.num_violations, k

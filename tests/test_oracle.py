@@ -386,3 +386,17 @@ def test_validation_rejects_bad_inputs():
     dup = types.SimpleNamespace(**{**vars(g), "ep_pin": np.array([0, 0], np.int32),
                                    "ep_rat": np.zeros((2, 2))})
     assert oracle.validate(dup) == 1
+
+
+def test_openmp_build_matches_serial():
+    """The all-core oracle build (OpenMP, pins of a level in parallel; bench cpu_baseline) computes the
+    same forward bit for bit and the same backward to rounding (atomic pushes reorder sums)."""
+    from paper_conf_dac_lugklr25_b200 import synth
+    g = synth.generate("C1")
+    for tau in (0.0, 1.0):
+        a = oracle.forward(g, 3.0, tau)
+        b = oracle.forward(g, 3.0, tau, omp=True)
+        assert np.array_equal(a["A"], b["A"]) and np.array_equal(a["win_arc"], b["win_arc"])
+        da = oracle.backward(g, 3.0, tau)["d_mean"]
+        db = oracle.backward(g, 3.0, tau, omp=True)["d_mean"]
+        assert np.allclose(da, db, rtol=1e-12, atol=1e-12)
