@@ -65,6 +65,8 @@ def grad_norm_ratio(a, b, stream=None):
     import torch
     a = a.contiguous().float()
     b = b.contiguous().float()
+    if a.numel() != b.numel():   # the ABI reads n elements of both
+        raise ValueError(f"grad_norm_ratio: a has {a.numel()} elements, b has {b.numel()}")
     out = torch.empty(1, dtype=torch.float64, device=a.device)
     st = ctypes.c_void_p((stream or torch.cuda.current_stream(a.device)).cuda_stream)
     check(_capi.load().insta_grad_norm_ratio(int(a.numel()), _dptr(a), _dptr(b), _dptr(out), st),

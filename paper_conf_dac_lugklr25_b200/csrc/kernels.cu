@@ -1576,52 +1576,67 @@ __global__ void __launch_bounds__(256) bwd_prep_kernel(int num_ep, const int32_t
 // fp64 with a fixed reduction tree (block partials, then the last block).
 // --------------------------------------------------------------------------
 constexpr int kRedThreads = 256;
+constexpr int kRedBlocksPerSM = 4;   // grid: a fixed multiple of the SM count (fixed summation order)
+
+// warp reduction in a fixed order (deterministic): sum / min of fp64
+__device__ __forceinline__ double warp_sum(double v) {
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xffffffffu, v, o);
+  return v;
+}
+__device__ __forceinline__ double warp_min(double v) {
+  for (int o = 16; o > 0; o >>= 1) v = fmin(v, __shfl_down_sync(0xffffffffu, v, o));
+  return v;
+}
 
 __global__ void __launch_bounds__(kRedThreads)
 slack_kernel(int num_ep, const int32_t* __restrict__ ep_pin, const float2* __restrict__ ep_rat,
              const PinState* __restrict__ state, float n_sigma, float* slack, uint8_t* rf_star,
              double* partials, uint32_t* ticket, double* summary) {
-  __shared__ double s_tns[kRedThreads];
-  __shared__ double s_wns[kRedThreads];
-  __shared__ double s_nv[kRedThreads];
+  __shared__ double s_red[3][kRedThreads / 32];
   __shared__ bool s_last;
-  const int k = blockIdx.x * kRedThreads + threadIdx.x;
   double tns = 0.0, wns = 0.0, nv = 0.0;
-  if (k < num_ep) {
+  const double ns = double(n_sigma);
+  // grid-stride: every endpoint's state gathered with the others in flight, summed in index order per thread
+  for (int k = blockIdx.x * kRedThreads + threadIdx.x; k < num_ep; k += gridDim.x * kRedThreads) {
     const Gath st = load_state_plain(state + ep_pin[k]);
     const float2 rat = ep_rat[k];
-    const double ns = double(n_sigma);
     const double sR = double(rat.x) - (st.mu0 + ns * double(sigma_of(st.v0)));   // Eq 3 corner
     const double sF = double(rat.y) - (st.mu1 + ns * double(sigma_of(st.v1)));
     const bool fall = sF < sR;
-    const double s = fall ? sF : sR;
-    slack[k] = float(s);
+    const double sv = fall ? sF : sR;
+    slack[k] = float(sv);
     rf_star[k] = fall ? 1 : 0;
-    if (s < 0.0) {
-      tns = s;
-      nv = 1.0;
-      wns = s;
+    if (sv < 0.0) {
+      tns += sv;
+      nv += 1.0;
+      wns = fmin(wns, sv);
     }
   }
-  s_tns[threadIdx.x] = tns;
-  s_wns[threadIdx.x] = wns;
-  s_nv[threadIdx.x] = nv;
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  tns = warp_sum(tns);
+  wns = warp_min(wns);
+  nv = warp_sum(nv);
+  if (lane == 0) {
+    s_red[0][w] = tns;
+    s_red[1][w] = wns;
+    s_red[2][w] = nv;
+  }
   __syncthreads();
-  for (int w = kRedThreads / 2; w > 0; w >>= 1) {
-    if (threadIdx.x < w) {
-      s_tns[threadIdx.x] += s_tns[threadIdx.x + w];
-      s_wns[threadIdx.x] = fmin(s_wns[threadIdx.x], s_wns[threadIdx.x + w]);
-      s_nv[threadIdx.x] += s_nv[threadIdx.x + w];
+  if (w == 0) {
+    tns = lane < kRedThreads / 32 ? s_red[0][lane] : 0.0;
+    wns = lane < kRedThreads / 32 ? s_red[1][lane] : 0.0;
+    nv = lane < kRedThreads / 32 ? s_red[2][lane] : 0.0;
+    tns = warp_sum(tns);
+    wns = warp_min(wns);
+    nv = warp_sum(nv);
+    if (lane == 0) {
+      partials[3 * blockIdx.x + 0] = tns;
+      partials[3 * blockIdx.x + 1] = wns;
+      partials[3 * blockIdx.x + 2] = nv;
+      __threadfence();
+      const uint32_t prev = atomicAdd(ticket, 1u);
+      s_last = prev == gridDim.x - 1;
     }
-    __syncthreads();
-  }
-  if (threadIdx.x == 0) {
-    partials[3 * blockIdx.x + 0] = s_tns[0];
-    partials[3 * blockIdx.x + 1] = s_wns[0];
-    partials[3 * blockIdx.x + 2] = s_nv[0];
-    __threadfence();
-    const uint32_t prev = atomicAdd(ticket, 1u);
-    s_last = prev == gridDim.x - 1;
   }
   __syncthreads();
   if (!s_last) return;
@@ -1634,22 +1649,27 @@ slack_kernel(int num_ep, const int32_t* __restrict__ ep_pin, const float2* __res
     wns = fmin(wns, __ldcg(partials + 3 * b + 1));
     nv += __ldcg(partials + 3 * b + 2);
   }
-  s_tns[threadIdx.x] = tns;
-  s_wns[threadIdx.x] = wns;
-  s_nv[threadIdx.x] = nv;
-  __syncthreads();
-  for (int w = kRedThreads / 2; w > 0; w >>= 1) {
-    if (threadIdx.x < w) {
-      s_tns[threadIdx.x] += s_tns[threadIdx.x + w];
-      s_wns[threadIdx.x] = fmin(s_wns[threadIdx.x], s_wns[threadIdx.x + w]);
-      s_nv[threadIdx.x] += s_nv[threadIdx.x + w];
-    }
-    __syncthreads();
+  tns = warp_sum(tns);
+  wns = warp_min(wns);
+  nv = warp_sum(nv);
+  if (lane == 0) {
+    s_red[0][w] = tns;
+    s_red[1][w] = wns;
+    s_red[2][w] = nv;
   }
+  __syncthreads();
   if (threadIdx.x == 0) {
-    summary[0] = s_wns[0];
-    summary[1] = s_tns[0];
-    summary[2] = s_nv[0];
+    tns = 0.0;
+    wns = 0.0;
+    nv = 0.0;
+    for (int k = 0; k < kRedThreads / 32; ++k) {
+      tns += s_red[0][k];
+      wns = fmin(wns, s_red[1][k]);
+      nv += s_red[2][k];
+    }
+    summary[0] = wns;
+    summary[1] = tns;
+    summary[2] = nv;
     *ticket = 0u;
   }
 }
@@ -1845,7 +1865,8 @@ static int launch_items(const void* fn, int threads, size_t smem, KParams& P, co
 int launch_slack(DevGraph& g, void* stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   if (g.num_ep == 0) return int(cudaMemsetAsync(g.summary, 0, sizeof(double) * 3, st));
-  const int blocks = (g.num_ep + kRedThreads - 1) / kRedThreads;
+  const int sms = g.sl_grid > 0 ? g.sl_grid : 148;
+  const int blocks = std::max(1, std::min((g.num_ep + kRedThreads - 1) / kRedThreads, kRedBlocksPerSM * sms));
   slack_kernel<<<blocks, kRedThreads, 0, st>>>(g.num_ep, g.ep_pin, g.ep_rat, g.state,
                                               g.last_n_sigma, g.slack, g.rf_star, g.partials,
                                               g.ticket, g.summary);

@@ -34,7 +34,7 @@ def test_timing_loss_parity(cfg):
     assert Lg == pytest.approx(Lo, rel=1e-9)
     assert np.allclose(gx, ox, rtol=1e-6, atol=1e-9)
     assert np.allclose(gy, oy, rtol=1e-6, atol=1e-9)
-    a = torch.as_tensor(rng.normal(size=4 * g.num_pins).astype(np.float32), device="cuda")
+    a = torch.as_tensor(rng.normal(size=2 * g.num_pins).astype(np.float32), device="cuda")   # as long as b
     b = torch.as_tensor(np.concatenate([gx, gy]), device="cuda")
     r = float(insta.grad_norm_ratio(a, b).item())
     assert r == pytest.approx(np.linalg.norm(a.cpu().numpy().astype(np.float64)) /
@@ -60,3 +60,9 @@ def test_timing_loss_heavy_fanout_and_determinism():
     wide = fo > 32
     assert wide.any()
     assert np.allclose(r1[1][wide], ox[wide], rtol=1e-6, atol=1e-6)
+
+
+def test_grad_norm_ratio_rejects_mismatched_lengths():
+    import torch
+    with pytest.raises(ValueError):
+        insta.grad_norm_ratio(torch.ones(10, device="cuda"), torch.ones(12, device="cuda"))
