@@ -195,6 +195,17 @@ def topk_forward(g, n_sigma=3.0, K=4):
     return dict(A=A, mu=mu, sigma=sig, sp=sp)
 
 
+def topk_taint(g, n_sigma=3.0, K=4, eps=1e-3):
+    """Test support: [N,2] bool, queue rows whose startpoint SET may differ on another correct
+    implementation (boundary near tie within eps, or an uncertain parent entry that can reach the row)."""
+    og = _og(g)
+    t = np.zeros((og.N, 2), np.uint8)
+    L = lib()
+    L.orc_topk_taint.argtypes = [ctypes.c_void_p, ctypes.c_double, ctypes.c_int32, ctypes.c_double, ctypes.c_void_p]
+    _check(L.orc_topk_taint(ctypes.byref(og.c), float(n_sigma), int(K), float(eps), _p(t)))
+    return t.astype(bool)
+
+
 def topk_slack(g, q, rat_table=None):
     """CPPR slack over Top-K queues q (from topk_forward).  rat_table = (ptr [P+1], sp [M], rat [M,2]) or None.
     Returns dict(slack, rf_star, k_star, sp_star [P], wns, tns, num_viol)."""

@@ -692,6 +692,102 @@ int orc_topk_slack(const orc_graph* g, int32_t K, const double* A, const int32_t
   return 0;
 }
 
+/* Test support (T9): which Top-K queue rows may legitimately hold a
+ * different startpoint SET on another correct implementation.  By Alg 2
+ * a queue ends as the K largest per-startpoint maxima of its candidates, so its
+ * set is ambiguous only where (a) the K-th and (K+1)-th per-startpoint maxima are
+ * within eps (a near tie at the eviction boundary), or (b) a parent row's set is
+ * ambiguous and one of its uncertain entries could reach this queue.  A tainted
+ * row carries hi = an upper bound on the arrival of any entry whose membership is
+ * uncertain; through arc e an uncertain parent entry A = mu + n sigma moves to
+ * A' = A + mean_e + n (sqrt(sigma^2 + std_e^2) - sigma) <= A + mean_e + n std_e
+ * (Eq 1-3), so it can enter a full queue only if hi_p + mean_e + n std_e reaches
+ * the K-th kept arrival minus eps; a queue that is not full takes any candidate.
+ * Output: taint[N][2] (caller ids).  Order ties inside a row (two kept entries
+ * within eps) are not flagged here: they reorder, not change, the set. */
+typedef struct { double A; int32_t sp; } tk_cand;
+static int cmp_cand_sp(const void* a, const void* b) {
+  const tk_cand *x = a, *y = b;
+  if (x->sp != y->sp) return x->sp < y->sp ? -1 : 1;
+  return (x->A > y->A) ? -1 : (x->A < y->A);
+}
+static int cmp_cand_desc(const void* a, const void* b) {
+  const tk_cand *x = a, *y = b;
+  return (x->A > y->A) ? -1 : (x->A < y->A);
+}
+
+int orc_topk_taint(const orc_graph* g, double n_sigma, int32_t K, double eps, uint8_t* taint) {
+  int st = orc_validate(g, n_sigma, 0.0);
+  if (st) return st;
+  if (K < 1) return 1;
+  int32_t N = g->num_pins;
+  size_t nq = (size_t)N * 2 * K;
+  double* mu = malloc(sizeof(double) * (nq + 1));
+  double* sig = malloc(sizeof(double) * (nq + 1));
+  int32_t* sp = malloc(sizeof(int32_t) * (nq + 1));
+  st = orc_topk_forward(g, n_sigma, K, NULL, mu, sig, sp);
+  if (st) { free(mu); free(sig); free(sp); return st; }
+  topo_t t;
+  st = topo_build(g->num_pins, g->num_arcs, g->arc_from, g->arc_to, &t);
+  if (st) { free(mu); free(sig); free(sp); return st; }
+  uint8_t* tn = calloc(2 * (size_t)N + 2, 1);
+  double* hi = malloc(sizeof(double) * (2 * (size_t)N + 2));
+  int32_t maxfi = max_fanin(&t);
+  tk_cand* c = malloc(sizeof(tk_cand) * ((size_t)maxfi * 2 * K + 1));
+  for (int32_t k = 0; k < N; ++k) {
+    int32_t i = t.order[k];
+    if (t.fanin_ptr[k] == t.fanin_ptr[k + 1]) continue;        /* startpoint: one certain entry */
+    for (int rf = 0; rf < 2; ++rf) {
+      int n = 0;
+      double U = -INFINITY;                                      /* bound on uncertain candidates */
+      int any_parent = 0;
+      for (int32_t r = t.fanin_ptr[k]; r < t.fanin_ptr[k + 1]; ++r) {
+        int32_t e = t.fanin_arc[r];
+        int32_t j = g->arc_from[e];
+        int ss[2];
+        int ns = sources_of(rf, g->arc_unate[e], ss);
+        double am = g->arc_mean[2 * (int64_t)e + rf], as = g->arc_sigma[2 * (int64_t)e + rf];
+        for (int a = 0; a < ns; ++a) {
+          size_t row = (size_t)j * 2 + ss[a];
+          for (int m = 0; m < K; ++m) {
+            size_t x = row * K + m;
+            if (sp[x] < 0) continue;
+            c[n].A = mu[x] + am + n_sigma * sqrt(sig[x] * sig[x] + as * as);   /* Eq 1-3 */
+            c[n].sp = sp[x];
+            ++n;
+          }
+          if (tn[row]) {
+            any_parent = 1;
+            double u = hi[row] + am + n_sigma * as;
+            if (u > U) U = u;
+          }
+        }
+      }
+      /* per-startpoint maxima, descending */
+      qsort(c, (size_t)n, sizeof(tk_cand), cmp_cand_sp);
+      int nu = 0;
+      for (int a = 0; a < n; ++a)
+        if (a == 0 || c[a].sp != c[a - 1].sp) c[nu++] = c[a];
+      qsort(c, (size_t)nu, sizeof(tk_cand), cmp_cand_desc);
+      int64_t q = 2 * (int64_t)i + rf;
+      double h = -INFINITY;
+      int x = 0;
+      if (nu > K && c[K - 1].A - c[K].A <= eps) { x = 1; h = c[K - 1].A + eps; }     /* (a) */
+      if (any_parent && (nu < K || U >= c[K - 1].A - eps)) {                        /* (b) */
+        x = 1;
+        double b = (nu >= K && c[K - 1].A + eps > U) ? c[K - 1].A + eps : U + eps;
+        if (b > h) h = b;
+      }
+      tn[q] = (uint8_t)x;
+      hi[q] = h;
+    }
+  }
+  if (taint) memcpy(taint, tn, 2 * (size_t)N);
+  free(c); free(hi); free(tn); free(mu); free(sig); free(sp);
+  topo_free(&t);
+  return 0;
+}
+
 /* ------------------------------------------------------------------------- */
 /* NEXT 2: Clark moment-matching statistical max, the merge    */
 /* the north star names beside the paper's smooth max.  The state of a pin is */

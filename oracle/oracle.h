@@ -88,6 +88,9 @@ int orc_topk_slack(const orc_graph* g, int32_t K, const double* A, const int32_t
                    const int32_t* rat_ptr, const int32_t* rat_sp, const double* rat_val,
                    double* slack, uint8_t* rf_star, int32_t* k_star, int32_t* sp_star,
                    double* wns, double* tns, int32_t* num_viol);
+/* Test support: Top-K queue rows whose startpoint set is legitimately ambiguous
+ * (near tie at the eviction boundary, propagated); taint[N][2]. */
+int orc_topk_taint(const orc_graph* g, double n_sigma, int32_t K, double eps, uint8_t* taint);
 
 /* NEXT 2: Clark moment-matching merge (reading R20, rho = 0), folded in
  * candidate order.  A/mu/sig [N][2] caller-indexed (sig = sqrt(V)). */

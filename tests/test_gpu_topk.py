@@ -3,9 +3,11 @@
 * dyadic mode (mu on a 2^-6 grid, sigma = 0): queues (A, startpoint, order) and
   CPPR slack bit-exact, ties included -- this checks that the kernel's (A, t)
   key merge reproduces the literal sequential Alg 2 of the oracle;
-* sigma > 0: every queue's A within max(1e-4 |A|, 1e-3 ps), startpoint lists
-  identical except where the oracle's own entries are within 1e-3 ps of each
-  other (fp32 sqrt vs fp64 may swap them), CPPR slack / TNS within tolerance;
+* sigma > 0: every queue's A within max(1e-4 |A|, 1e-3 ps); startpoint SETS
+  identical except in rows the oracle's propagated eviction-boundary near-tie
+  taint flags (oracle.topk_taint, T9); startpoint ORDER identical
+  except where the oracle's own entries are within 1e-3 ps of each other (fp32
+  sqrt vs fp64 may swap them); CPPR slack / TNS within tolerance;
 * K = 1 equals the GPU hard forward (insta_forward, tau = 0);
 * C4 at full size: K = 1 equals the hard forward; K = 8 queue invariants on
   the device (descending, unique startpoints, startpoints are sources).
@@ -95,9 +97,15 @@ def test_topk_sigma_parity(cfg, K):
     ref = oq["A"][valid]
     err = np.abs(gq.q["A"][valid].astype(np.float64) - ref)
     assert (err <= np.maximum(1e-4 * np.abs(ref), 1e-3)).all(), err.max()
+    # startpoint SETS equal except in rows the oracle's propagated boundary-tie taint flags
+    # (orc_topk_taint, pinned by tests/test_topk_taint_oracle.py); order equal except at a local near tie
+    set_same = (np.sort(gq.q["sp"], axis=2) == np.sort(oq["sp"], axis=2)).all(axis=2)
+    taint = oracle.topk_taint(g, NS, K, eps=1e-3)
+    assert (set_same | taint).all(), np.argwhere(~(set_same | taint))[:8]
+    assert taint.mean() < 0.05, taint.mean()   # C2, K = 16: 2.6 %
     rows_same = (gq.q["sp"] == oq["sp"]).all(axis=2)
     tie = _near_tie_rows(oq)
-    assert (rows_same | tie).mean() >= 0.999, (~(rows_same | tie)).sum()
+    assert (rows_same | tie | ~set_same).all(), (~(rows_same | tie | ~set_same)).sum()
     serr = np.abs(gq.slack.astype(np.float64) - os_["slack"])
     assert (serr <= np.maximum(1e-4 * np.abs(os_["slack"]), 1e-3)).all(), serr.max()
     assert abs(gq.summary.tns - os_["tns"]) <= 1e-6 * abs(os_["tns"]) + 1e-3
