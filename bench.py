@@ -494,13 +494,22 @@ def main():
         n_ocv = nsc // 2
         scs = synth.c5_scenarios(g, n=nsc, n_ocv=n_ocv)
 
+        def is_sizing(sc):
+            return sc.get("delta_arc") is not None and sc["n_sigma"] == 3.0 and sc["derate_cell"] == 1.0 \
+                and sc["derate_net"] == 1.0
+
         def ev(sub, want_grad):
+            # OCV scenarios (and anything with derates): the batched kernels, 32 per pass; sizing candidates
+            # (one cell's arcs re-annotated): the cone pass per candidate (insta_eval_candidates)
             with torch.cuda.stream(stream):
+                if not want_grad and all(is_sizing(sc) for sc in sub):
+                    return G.eval_candidates(sub, stream=stream), None
                 summ, dsum = G.forward_batch(sub, tau=args.tau, want_grad=want_grad, stream=stream)
             return summ, dsum
 
         dd = torch.distributed if world > 1 else None
         with torch.cuda.stream(stream):
+            G.forward(3.0, args.tau, 0, stream=stream)   # the base state the candidates are evaluated against
             # warm-up: one untimed pass of the same calls (allocates the batch and staging buffers)
             idist.evaluate_sharded(ev, scs, n_ocv, E, rank, world, dev, dd)
             stream.synchronize()
@@ -517,8 +526,24 @@ def main():
             torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
             bms = float(t.item())
         sa = summ_all.cpu().numpy()
+        split = None
+        if world == 1:   # the two halves timed separately (and the sizing half on the batched kernels too)
+            with torch.cuda.stream(stream):
+                t0, t1, t2, t3 = (torch.cuda.Event(enable_timing=True) for _ in range(4))
+                t0.record(stream)
+                ev(scs[:n_ocv], True)
+                t1.record(stream)
+                ev(scs[n_ocv:], False)
+                t2.record(stream)
+                G.forward_batch(scs[n_ocv:], tau=args.tau, want_grad=False, stream=stream)
+                t3.record(stream)
+                torch.cuda.synchronize(dev)
+            split = {"ocv_fwd_bwd_ms": t0.elapsed_time(t1), "sizing_cone_ms": t1.elapsed_time(t2),
+                     "sizing_batched_kernels_ms": t2.elapsed_time(t3),
+                     "sizing_evals_per_s_cone": (nsc - n_ocv) / (t1.elapsed_time(t2) * 1e-3)}
         batched = {"workload": f"C5: {nsc} scenarios on the {cfg.name} graph ({n_ocv} OCV fwd+bwd with TNS-gradient "
-                               f"sum, {nsc - n_ocv} sizing candidates fwd), 32 scenarios per pass",
+                               f"sum, 32 scenarios per batched pass; {nsc - n_ocv} one-cell sizing candidates through "
+                               f"the cone pass, insta_eval_candidates)", "split": split,
                    "evals": nsc, "ms": bms, "evals_per_s": nsc / (bms * 1e-3),
                    "pins_per_s": nsc * N / (bms * 1e-3), "n_gpus": world,
                    "collectives": "all_gather(per-scenario summaries) + all_reduce(SUM, gradient sum)" if world > 1
