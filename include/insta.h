@@ -234,11 +234,16 @@ insta_status insta_forward_batch(insta_graph* g, int32_t num_scenarios, const in
  * ids, DEVICE int32) with mean / sigma (DEVICE float[..][2]); its summary
  * {wns, tns, num_violations} goes to summaries[i] (DEVICE double[n][3]).  Each
  * candidate is applied, evaluated with the cone pass (recomputing only what
- * its arcs reach), and reverted with a second cone pass, so the summary equals
- * insta_forward on the candidate's materialized graph bit for bit, and the
- * graph is back to its base state on return.  cand_ptr: HOST int32[n + 1],
- * ascending.  Needs a current forward of schedule 0 or 3 (E_STATE otherwise;
- * uses its n_sigma / tau).  Asynchronous on cuda_stream. */
+ * its arcs reach; the endpoint slack only of the blocks it reached), and
+ * reverted with a second cone pass, so the summary equals insta_forward on the
+ * candidate's materialized graph bit for bit, and the graph (arrivals, slack,
+ * summary) is back to its base state on return.  All candidates run inside one
+ * persistent cooperative launch (grid barriers between the steps).  cand_ptr:
+ * HOST int32[n + 1], ascending, cand_ptr[0] = 0.  Arc ids must lie in
+ * [0, num_arcs) (device array: not checked here; the Python binding checks);
+ * an arc listed twice in one candidate must carry the same record (else which
+ * one applies is unspecified).  Needs a current forward of schedule 0 or 3
+ * (E_STATE otherwise; uses its n_sigma / tau).  Asynchronous on cuda_stream. */
 insta_status insta_eval_candidates(insta_graph* g, int32_t num_candidates, const int32_t* cand_ptr,
                                    const int32_t* arc_ids, const float* mean, const float* sigma, double* summaries,
                                    void* cuda_stream);
@@ -266,9 +271,11 @@ insta_status insta_eval_candidates(insta_graph* g, int32_t num_candidates, const
 insta_status insta_set_cppr_rat(insta_graph* g, const int32_t* rat_ptr, const int32_t* rat_sp, const float* rat);
 
 /* Top-K forward (Alg 1 + Alg 2) over all levels with the graph's current arc
- * delays; 1 <= K <= 32, n_sigma as in Eq 3.  Device state: K * 40 bytes per
- * pin (fp64 mean and variance + int32 startpoint per slot and rf).  Enqueued on
- * cuda_stream.  E_ARG: K or n_sigma out of range. */
+ * delays; 1 <= K <= 128 (the paper's CPPR study uses K = 128), n_sigma
+ * as in Eq 3.  Device state: K * 40 bytes per pin (fp64 mean and variance +
+ * int32 startpoint per slot and rf; C4 at K = 128: 77 GB).  Enqueued on
+ * cuda_stream.  E_ARG: K or n_sigma out of range; E_CUDA (out of memory) when
+ * the queues do not fit. */
 insta_status insta_topk_forward(insta_graph* g, int32_t K, float n_sigma, void* cuda_stream);
 
 /* CPPR endpoint slack over the Top-K queues: slack(ep) = min over rf (R

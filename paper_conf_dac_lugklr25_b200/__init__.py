@@ -359,6 +359,20 @@ class Graph:
         """insta_eval_candidates: what-if summaries of sparse re-annotations (dicts with delta_arc /
         delta_mean / delta_sigma host arrays, e.g. synth.sizing_scenario), each applied, evaluated with the
         cone pass and reverted.  Returns float64[n, 3] {wns, tns, num_violations} device tensor."""
+        return self.eval_packed(self.pack_candidates(candidates, stream), stream=stream, summaries=summaries)
+
+    def eval_packed(self, packed, stream=None, summaries=None):
+        """insta_eval_candidates on candidates already packed by pack_candidates (no host work per call)."""
+        t = self._torch
+        ptr, di, dm, ds = packed
+        n = len(ptr) - 1
+        out = summaries if summaries is not None else t.empty((n, 3), dtype=t.float64, device=self.device)
+        check(self.lib.insta_eval_candidates(self._h, n, _ptr(ptr), _dptr(di), _dptr(dm), _dptr(ds), _dptr(out),
+                                             self._st(stream)), "insta_eval_candidates")
+        return out
+
+    def pack_candidates(self, candidates, stream=None):
+        """(cand_ptr host int32[n + 1], arc ids, mean, sigma device tensors) for eval_packed."""
         t = self._torch
         n = len(candidates)
         ptr = np.zeros(n + 1, np.int32)
@@ -369,11 +383,12 @@ class Graph:
             np.zeros((0, 2), np.float32)
         sg = np.concatenate([np.asarray(c["delta_sigma"], np.float32).reshape(-1, 2) for c in candidates]) if n else \
             np.zeros((0, 2), np.float32)
+        if len(ids) and (int(ids.min()) < 0 or int(ids.max()) >= self.num_arcs):   # the ABI reads them unchecked
+            raise ValueError(f"eval_candidates: arc ids must be in [0, {self.num_arcs})")
+        if len(m) != len(ids) or len(sg) != len(ids):
+            raise ValueError("eval_candidates: delta_mean / delta_sigma need one [2] row per delta_arc")
         di, dm, ds = (self._dev(x, dt, stream) for x, dt in ((ids, t.int32), (m, t.float32), (sg, t.float32)))
-        out = summaries if summaries is not None else t.empty((n, 3), dtype=t.float64, device=self.device)
-        check(self.lib.insta_eval_candidates(self._h, n, _ptr(ptr), _dptr(di), _dptr(dm), _dptr(ds), _dptr(out),
-                                             self._st(stream)), "insta_eval_candidates")
-        return out
+        return ptr, di, dm, ds
 
     def last_forward_stats(self) -> int:
         v = ctypes.c_int64()

@@ -68,7 +68,7 @@ void free_graph(insta::DevGraph& d) {
                   d.cl_rf,     d.cl_summary, d.cl_hv_list, d.cl_hv_of, d.cl_hv_sum, d.tl_partials, d.sz_tmp,
                   d.sl_ptr,    d.ext_sh,    d.hd_csl,    d.chg,       d.acc_h,     d.sl_bar,    d.sl_cnt,
                   d.hwin,      d.ew,        d.fwin,      d.efw,       d.sl_slice,  d.hfo_ptr,   d.hfo,       d.hd_hsrc,
-                  d.cand_old};
+                  d.cand_old,  d.ep_blk,    d.cand_ptr_d, d.pl_ptr,    d.pl_ent,    d.pl_arc,    d.pl_wide};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   if (d.b_stage_h) cudaFreeHost(d.b_stage_h);
@@ -361,6 +361,7 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   ZERO(d.slack, d.num_ep);
   ZERO(d.rf_star, d.num_ep);
   ZERO(d.partials, 3 * ((d.num_ep + 255) / 256 + 1));
+  ZERO(d.ep_blk, ((d.num_ep + 255) / 256 + 1) / 32 + 1);
   ZERO(d.ticket, 1);
   ZERO(d.summary, 4);
   ZERO(d.counters, 4);
@@ -462,7 +463,7 @@ insta_status insta_forward(insta_graph* g, const insta_opts* o, void* cuda_strea
     if (!err) {
       d.last_n_sigma = opt.n_sigma;
       d.last_tau = opt.tau;
-      err = insta::launch_slack(d, cuda_stream);
+      err = insta::launch_slack_delta(d, cuda_stream);   // only the slack blocks the cone reached
     }
   } else if (opt.schedule == 3 || (opt.schedule == 0 && d.parity_mixed)) {
     // level-synchronous sweep forward (sweep.cu); also the default's full pass
@@ -595,43 +596,21 @@ insta_status insta_eval_candidates(insta_graph* g, int32_t num_candidates, const
   }
   if (maxn > 0 && (!arc_ids || !mean || !sigma)) return fail(INSTA_E_ARG, "eval_candidates: NULL arc arrays");
   cudaSetDevice(d.device);
-  cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
-  if (maxn > d.cand_cap) {
-    if (d.cand_old) cudaFree(d.cand_old);
-    d.cand_old = nullptr;
-    d.cand_cap = 0;
-    cudaError_t e = cudaMalloc(reinterpret_cast<void**>(&d.cand_old), sizeof(float) * 4 * size_t(maxn));
-    if (e != cudaSuccess) return cuda_fail(int(e), "eval_candidates");
-    d.cand_cap = maxn;
+  if (num_candidates == 0) return INSTA_OK;
+  if (cand_ptr[0] != 0) return fail(INSTA_E_ARG, "eval_candidates: cand_ptr[0] must be 0");
+  if (!d.slack_valid) {   // the base slack blocks the kernel updates in place
+    const int err = insta::launch_slack(d, cuda_stream);
+    if (err) return cuda_fail(err, "eval_candidates");
   }
-  const float n_sigma = d.last_n_sigma, tau = d.last_tau;
-  float* old_m = d.cand_old;
-  float* old_s = d.cand_old + 2 * size_t(std::max(maxn, 1));
-  for (int32_t i = 0; i < num_candidates; ++i) {
-    const int32_t off = cand_ptr[i], n = cand_ptr[i + 1] - off;
-    int err = 0;
-    if (n > 0) {
-      // apply: save the current records, re-annotate, cone pass, slack; revert: the saved records, cone pass
-      err = insta::launch_gather_arcs(d, n, arc_ids + off, old_m, old_s, st);
-      if (!err) err = insta::launch_update_arcs(d, n, arc_ids + off, mean + 2 * size_t(off), sigma + 2 * size_t(off), 1, st);
-      if (!err) err = insta::launch_forward_cone(d, n_sigma, tau, st);
-    }
-    if (!err) err = insta::launch_slack(d, st);
-    if (!err) err = int(cudaMemcpyAsync(summaries + 3 * size_t(i), d.summary, sizeof(double) * 3,
-                                        cudaMemcpyDeviceToDevice, st));
-    if (!err && n > 0) {
-      err = insta::launch_update_arcs(d, n, arc_ids + off, old_m, old_s, 1, st);
-      if (!err) err = insta::launch_forward_cone(d, n_sigma, tau, st);
-    }
-    if (err) {
-      d.fwd_valid = false;
-      d.pending_full = true;
-      return cuda_fail(err, "eval_candidates");
-    }
+  // every candidate applied, evaluated and reverted inside one persistent launch (sweep.cu
+  // eval_kernel); on return the graph, its slack and summary are the base state bit for bit
+  const int err = insta::launch_eval_candidates(d, num_candidates, cand_ptr, arc_ids, mean, sigma, summaries,
+                                                cuda_stream);
+  if (err) {
+    d.fwd_valid = false;
+    d.pending_full = true;
+    return cuda_fail(err, "eval_candidates");
   }
-  // every candidate reverted: the base state, bit for bit; its slack/summary are restored too
-  int err = insta::launch_slack(d, st);
-  if (err) return cuda_fail(err, "eval_candidates");
   d.pending_updates = 0;
   return INSTA_OK;
 }
@@ -775,7 +754,7 @@ insta_status insta_set_cppr_rat(insta_graph* g, const int32_t* rat_ptr, const in
 
 insta_status insta_topk_forward(insta_graph* g, int32_t K, float n_sigma, void* cuda_stream) {
   if (!g) return fail(INSTA_E_ARG, "topk_forward: NULL graph");
-  if (K < 1 || K > 32) return fail(INSTA_E_ARG, "topk_forward: K must be in [1, 32]");
+  if (K < 1 || K > 128) return fail(INSTA_E_ARG, "topk_forward: K must be in [1, 128]");
   if (!std::isfinite(n_sigma) || n_sigma < 0.f) return fail(INSTA_E_ARG, "topk_forward: n_sigma must be >= 0");
   insta::DevGraph& d = g->d;
   cudaSetDevice(d.device);

@@ -284,6 +284,11 @@ struct DevGraph {
   // Eq 7 timing objective (place.cu)
   double* tl_partials = nullptr;
   int32_t tl_cap = 0;
+  int32_t* pl_ptr = nullptr;       // [n+1] incident arcs of each caller pin (fanout then fanin)
+  int32_t* pl_ent = nullptr;       // [2e] other end (caller pin) | 1 << 31 if the pin is the arc's sink
+  int32_t* pl_arc = nullptr;       // [2e] caller arc id
+  int32_t* pl_wide = nullptr;      // caller pins with more than kPlWide incident arcs
+  int32_t num_pl_wide = -1;        // -1: not built
   // CPPR required times per (endpoint, startpoint) (insta_set_cppr_rat)
   int32_t* rat_ptr = nullptr;      // [P+1] or NULL (no table)
   int32_t* rat_sp = nullptr;       // [M] canonical startpoints, ascending within a row
@@ -299,6 +304,10 @@ struct DevGraph {
   double* partials = nullptr;      // slack reduction partials
   uint32_t* ticket = nullptr;      // last-block ticket
   double* summary = nullptr;       // {wns, tns, nviol} on device
+  uint32_t* ep_blk = nullptr;      // slack blocks holding an endpoint a cone pass changed (bitmask)
+  bool slack_valid = false;        // partials hold the slack blocks of the current state
+  int32_t* cand_ptr_d = nullptr;   // insta_eval_candidates: device copy of cand_ptr
+  int32_t cand_ptr_cap = 0;
   // incremental
   unsigned long long* counters = nullptr;  // [4] recomputed pins etc.
   // host-side bookkeeping
@@ -347,6 +356,9 @@ int launch_arrivals(DevGraph& g, float* A, float* mean, float* sigma, void* stre
 int query_sl_grid(int device, int* grid_fwd, int* grid_bwd);
 int launch_forward_sl(DevGraph& g, float n_sigma, float tau, void* stream);
 int launch_forward_cone(DevGraph& g, float n_sigma, float tau, void* stream);
+int launch_eval_candidates(DevGraph& g, int num, const int32_t* cand_ptr, const int32_t* arc_ids, const float* mean,
+                           const float* sigma, double* out, void* stream);
+int launch_slack_delta(DevGraph& g, void* stream);
 int launch_backward_sl(DevGraph& g, float* d_arc_mean, float* d_src, void* stream);
 int launch_fold_fill(DevGraph& g, void* stream);   // materialize folded pins after a sweep forward
 int launch_copy_slack(DevGraph& g, float* slack, uint8_t* rf, void* stream);

@@ -43,6 +43,7 @@
 
 #include "device_common.cuh"
 #include "internal.h"
+#include "slack_common.cuh"
 
 namespace insta {
 
@@ -161,16 +162,6 @@ __device__ __forceinline__ float2 arc_rf_weights(const KParams& P, int rf, int k
 }
 
 // State read outside a propagation pass (parity stripped, no waiting).
-__device__ __forceinline__ Gath load_state_plain(const PinState* p) {
-  const double2 m = __ldcg(reinterpret_cast<const double2*>(p));
-  const double2 v = __ldcg(reinterpret_cast<const double2*>(p) + 1);
-  Gath g;
-  g.mu0 = strip((unsigned long long)__double_as_longlong(m.x));
-  g.mu1 = strip((unsigned long long)__double_as_longlong(m.y));
-  g.v0 = strip((unsigned long long)__double_as_longlong(v.x));
-  g.v1 = strip2((unsigned long long)__double_as_longlong(v.y));
-  return g;
-}
 
 // --------------------------------------------------------------------------
 // Level-synchronous item loop.  Each CTA walks its item list in
@@ -1575,103 +1566,50 @@ __global__ void __launch_bounds__(256) bwd_prep_kernel(int num_ep, const int32_t
 // Endpoint slack + WNS/TNS: slack = RAT - A, min over rf, tie -> R; TNS in
 // fp64 with a fixed reduction tree (block partials, then the last block).
 // --------------------------------------------------------------------------
-constexpr int kRedThreads = 256;
-constexpr int kRedBlocksPerSM = 4;   // grid: a fixed multiple of the SM count (fixed summation order)
-
-// warp reduction in a fixed order (deterministic): sum / min of fp64
-__device__ __forceinline__ double warp_sum(double v) {
-  for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xffffffffu, v, o);
-  return v;
-}
-__device__ __forceinline__ double warp_min(double v) {
-  for (int o = 16; o > 0; o >>= 1) v = fmin(v, __shfl_down_sync(0xffffffffu, v, o));
-  return v;
-}
-
 __global__ void __launch_bounds__(kRedThreads)
 slack_kernel(int num_ep, const int32_t* __restrict__ ep_pin, const float2* __restrict__ ep_rat,
              const PinState* __restrict__ state, float n_sigma, float* slack, uint8_t* rf_star,
              double* partials, uint32_t* ticket, double* summary) {
-  __shared__ double s_red[3][kRedThreads / 32];
+  __shared__ SlackRed sr;
   __shared__ bool s_last;
-  double tns = 0.0, wns = 0.0, nv = 0.0;
-  const double ns = double(n_sigma);
   // grid-stride: every endpoint's state gathered with the others in flight, summed in index order per thread
-  for (int k = blockIdx.x * kRedThreads + threadIdx.x; k < num_ep; k += gridDim.x * kRedThreads) {
-    const Gath st = load_state_plain(state + ep_pin[k]);
-    const float2 rat = ep_rat[k];
-    const double sR = double(rat.x) - (st.mu0 + ns * double(sigma_of(st.v0)));   // Eq 3 corner
-    const double sF = double(rat.y) - (st.mu1 + ns * double(sigma_of(st.v1)));
-    const bool fall = sF < sR;
-    const double sv = fall ? sF : sR;
-    slack[k] = float(sv);
-    rf_star[k] = fall ? 1 : 0;
-    if (sv < 0.0) {
-      tns += sv;
-      nv += 1.0;
-      wns = fmin(wns, sv);
-    }
-  }
-  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  tns = warp_sum(tns);
-  wns = warp_min(wns);
-  nv = warp_sum(nv);
-  if (lane == 0) {
-    s_red[0][w] = tns;
-    s_red[1][w] = wns;
-    s_red[2][w] = nv;
-  }
-  __syncthreads();
-  if (w == 0) {
-    tns = lane < kRedThreads / 32 ? s_red[0][lane] : 0.0;
-    wns = lane < kRedThreads / 32 ? s_red[1][lane] : 0.0;
-    nv = lane < kRedThreads / 32 ? s_red[2][lane] : 0.0;
-    tns = warp_sum(tns);
-    wns = warp_min(wns);
-    nv = warp_sum(nv);
-    if (lane == 0) {
-      partials[3 * blockIdx.x + 0] = tns;
-      partials[3 * blockIdx.x + 1] = wns;
-      partials[3 * blockIdx.x + 2] = nv;
-      __threadfence();
-      const uint32_t prev = atomicAdd(ticket, 1u);
-      s_last = prev == gridDim.x - 1;
-    }
+  slack_block(blockIdx.x, gridDim.x, num_ep, ep_pin, ep_rat, state, double(n_sigma), slack, rf_star, partials, sr);
+  if (threadIdx.x == 0) {
+    __threadfence();
+    const uint32_t prev = atomicAdd(ticket, 1u);
+    s_last = prev == gridDim.x - 1;
   }
   __syncthreads();
   if (!s_last) return;
   __threadfence();
-  tns = 0.0;
-  wns = 0.0;
-  nv = 0.0;
-  for (int b = threadIdx.x; b < int(gridDim.x); b += kRedThreads) {
-    tns += __ldcg(partials + 3 * b + 0);
-    wns = fmin(wns, __ldcg(partials + 3 * b + 1));
-    nv += __ldcg(partials + 3 * b + 2);
-  }
-  tns = warp_sum(tns);
-  wns = warp_min(wns);
-  nv = warp_sum(nv);
-  if (lane == 0) {
-    s_red[0][w] = tns;
-    s_red[1][w] = wns;
-    s_red[2][w] = nv;
+  slack_final(gridDim.x, partials, summary, sr);
+  if (threadIdx.x == 0) *ticket = 0u;
+}
+
+// After a cone pass: recompute only the slack blocks holding a changed endpoint
+// (flagged in ep_blk), then the final reduction -- the same arithmetic as
+// slack_kernel on the other blocks' stored partials, so the summary is bit-
+// identical to a full slack pass.  The last block clears the flags.
+__global__ void __launch_bounds__(kRedThreads)
+slack_delta_kernel(int num_ep, const int32_t* __restrict__ ep_pin, const float2* __restrict__ ep_rat,
+                   const PinState* __restrict__ state, float n_sigma, float* slack, uint8_t* rf_star,
+                   double* partials, uint32_t* ticket, double* summary, uint32_t* ep_blk) {
+  __shared__ SlackRed sr;
+  __shared__ bool s_last;
+  const int b = blockIdx.x;
+  if ((__ldcg(ep_blk + (b >> 5)) >> (b & 31)) & 1u)
+    slack_block(b, gridDim.x, num_ep, ep_pin, ep_rat, state, double(n_sigma), slack, rf_star, partials, sr);
+  if (threadIdx.x == 0) {
+    __threadfence();
+    const uint32_t prev = atomicAdd(ticket, 1u);
+    s_last = prev == gridDim.x - 1;
   }
   __syncthreads();
-  if (threadIdx.x == 0) {
-    tns = 0.0;
-    wns = 0.0;
-    nv = 0.0;
-    for (int k = 0; k < kRedThreads / 32; ++k) {
-      tns += s_red[0][k];
-      wns = fmin(wns, s_red[1][k]);
-      nv += s_red[2][k];
-    }
-    summary[0] = wns;
-    summary[1] = tns;
-    summary[2] = nv;
-    *ticket = 0u;
-  }
+  if (!s_last) return;
+  __threadfence();
+  slack_final(gridDim.x, partials, summary, sr);
+  for (int w = threadIdx.x; w < int((gridDim.x + 31) / 32); w += blockDim.x) ep_blk[w] = 0u;
+  if (threadIdx.x == 0) *ticket = 0u;
 }
 
 // --------------------------------------------------------------------------
@@ -1865,11 +1803,22 @@ static int launch_items(const void* fn, int threads, size_t smem, KParams& P, co
 int launch_slack(DevGraph& g, void* stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   if (g.num_ep == 0) return int(cudaMemsetAsync(g.summary, 0, sizeof(double) * 3, st));
-  const int sms = g.sl_grid > 0 ? g.sl_grid : 148;
-  const int blocks = std::max(1, std::min((g.num_ep + kRedThreads - 1) / kRedThreads, kRedBlocksPerSM * sms));
+  const int blocks = slack_blocks(g.num_ep, g.sl_grid > 0 ? g.sl_grid : 148);
   slack_kernel<<<blocks, kRedThreads, 0, st>>>(g.num_ep, g.ep_pin, g.ep_rat, g.state,
                                               g.last_n_sigma, g.slack, g.rf_star, g.partials,
                                               g.ticket, g.summary);
+  const int err = int(cudaGetLastError());
+  g.slack_valid = err == 0;
+  return err;
+}
+
+int launch_slack_delta(DevGraph& g, void* stream) {
+  if (!g.slack_valid) return launch_slack(g, stream);
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (g.num_ep == 0) return int(cudaMemsetAsync(g.summary, 0, sizeof(double) * 3, st));
+  const int blocks = slack_blocks(g.num_ep, g.sl_grid > 0 ? g.sl_grid : 148);
+  slack_delta_kernel<<<blocks, kRedThreads, 0, st>>>(g.num_ep, g.ep_pin, g.ep_rat, g.state, g.last_n_sigma, g.slack,
+                                                    g.rf_star, g.partials, g.ticket, g.summary, g.ep_blk);
   return int(cudaGetLastError());
 }
 

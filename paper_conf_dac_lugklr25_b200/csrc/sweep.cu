@@ -54,6 +54,7 @@
 
 #include "device_common.cuh"
 #include "internal.h"
+#include "slack_common.cuh"
 
 namespace insta {
 
@@ -115,6 +116,29 @@ struct SLParams {
   float* d_mean;
   float* d_src;
   unsigned long long* trace;             // debug (INSTA_SL_TRACE)
+  // endpoint slack (cone passes: the slack blocks holding a changed endpoint are flagged)
+  const int32_t* __restrict__ hd_eop;    // [H] endpoint index of the head, -1 none
+  uint32_t* ep_blk;                      // [ceil(slack_nb / 32)] flagged slack blocks, or nullptr
+  int32_t slack_nb, num_ep;
+  const int32_t* __restrict__ ep_pin;
+  const float2* __restrict__ ep_rat;
+  float* slack;
+  uint8_t* rf_star;
+  double* partials;
+  // candidate evaluation (eval_kernel): arc record arrays and the candidates
+  const int32_t* __restrict__ arc_pos;
+  const int32_t* __restrict__ arc_xpos;
+  const int32_t* __restrict__ arc_head;
+  float4* fin_ms;
+  float4* ext_ms_w;
+  float4* ext_fms_w;
+  const int32_t* __restrict__ cand_ptr;  // [n + 1] (device copy)
+  const int32_t* __restrict__ cand_arc;
+  const float2* __restrict__ cand_m;
+  const float2* __restrict__ cand_s;
+  float4* cand_old;                      // [arcs of all candidates] saved records
+  double* cand_out;                      // [n][3]
+  int32_t num_cand;
 };
 
 // --------------------------------------------------------------------------
@@ -419,7 +443,8 @@ __device__ __noinline__ int sl_fwd_wide(const SLParams P, const HeadTopo t, RfOu
 // when it changed, mark the consumer heads.  Returns the pins evaluated.
 template <bool kLSE, bool kInc>
 __device__ __forceinline__ int sl_fwd_head(const SLParams& P, int h, const HeadTopo& t, const EntSrc& E,
-                                           uint32_t* s_mark, const int32_t* s_slp, unsigned long long* ph = nullptr) {
+                                           uint32_t* s_mark, const int32_t* s_slp, uint32_t stamp,
+                                           unsigned long long* ph = nullptr) {
   RfOut R, F;
   Raw old;
   if (kInc) old = ld_raw(P.state + t.pin);
@@ -437,7 +462,14 @@ __device__ __forceinline__ int sl_fwd_head(const SLParams& P, int h, const HeadT
       st_state(P.state + t.pin, R.mu, F.mu, R.var, F.var, P.par);
       // consumers (later levels): a short row is stamped dirty one by one; a
       // long row's consumers see the change through chg (levels flagged)
-      P.chg[t.pin] = P.stamp;
+      P.chg[t.pin] = stamp;
+      if (P.ep_blk) {   // an endpoint: its slack block is recomputed after the pass
+        const int k = __ldg(P.hd_eop + h);
+        if (k >= 0) {
+          const int b = (k / kRedThreads) % P.slack_nb;
+          atomicOr(P.ep_blk + (b >> 5), 1u << (b & 31));
+        }
+      }
       const int r0 = __ldg(P.hfo_ptr + h), r1 = __ldg(P.hfo_ptr + h + 1);
       if (r1 - r0 <= kConeRow) {
         for (int r = r0; r < r1; r += 8) {   // the row's loads in flight together
@@ -447,7 +479,7 @@ __device__ __forceinline__ int sl_fwd_head(const SLParams& P, int h, const HeadT
 #pragma unroll
           for (int j = 0; j < 8; ++j) {
             if (q[j] >= 0) {
-              P.dirty[q[j]] = P.stamp;
+              P.dirty[q[j]] = stamp;
               mark_level(P, s_mark, sl_of(P, s_slp, q[j]), 1u);
             }
           }
@@ -467,16 +499,17 @@ __device__ __forceinline__ int sl_fwd_head(const SLParams& P, int h, const HeadT
 // Cone pass (kInc): is head h dirty?  Stamped by insta_update_arcs (an arc it
 // evaluates changed) or one of its entries' source records changed in this
 // pass (chg, written by the recomputed source head before the level barrier).
-__device__ __forceinline__ bool head_dirty(const SLParams& P, int h, const int32_t* w, int nf, uint32_t lvl) {
-  if (__ldcg(P.dirty + h) == P.stamp) return true;
+__device__ __forceinline__ bool head_dirty(const SLParams& P, int h, const int32_t* w, int nf, uint32_t lvl,
+                                           uint32_t stamp) {
+  if (__ldcg(P.dirty + h) == stamp) return true;
   if (!(lvl & 2u) || !__ldg(P.hd_hsrc + h)) return false;
   uint32_t c[4];   // every load in flight at once
 #pragma unroll
   for (int k = 0; k < 4; ++k) c[k] = k < nf ? __ldcg(P.chg + (w[k] & kSrcMask)) : 0u;
   bool any = false;
 #pragma unroll
-  for (int k = 0; k < 4; ++k) any |= c[k] == P.stamp;
-  for (int k = 4; k < nf && !any; ++k) any = __ldcg(P.chg + (w[k] & kSrcMask)) == P.stamp;
+  for (int k = 0; k < 4; ++k) any |= c[k] == stamp;
+  for (int k = 4; k < nf && !any; ++k) any = __ldcg(P.chg + (w[k] & kSrcMask)) == stamp;
   return any;
 }
 
@@ -498,6 +531,59 @@ __device__ __forceinline__ void mark_flush(const SLParams& P, uint32_t* s_mark, 
   }
 }
 
+// Shared memory of a cone pass that reads topology from global (small cone).
+struct ConeSm {
+  uint32_t mark[2 * kMarkWords];
+  uint32_t pub[2 * kMarkWords];
+  uint32_t cnt;
+  int32_t next;
+};
+
+// Unstaged cone pass over levels 1 .. L-1 (flags in P.sl_cnt, dirty stamps ==
+// stamp): jumps from flagged level to flagged level -- every flag at or past
+// the current level is final (the levels before it are done) -- with one grid
+// barrier per level that recomputed something.  The caller has zeroed
+// cs.pub, and barriers the grid before and after.
+template <bool kLSE>
+__device__ __forceinline__ void cone_levels(const SLParams& P, uint32_t stamp, ConeSm& cs, const int4* s_slc,
+                                            const int32_t* s_slp, uint32_t& nbar, uint32_t& nrec) {
+  const int tid = threadIdx.x, L = P.num_sl;
+  bool need_bar = false;
+  for (int s = 1; s < L; ++s) {
+    if (need_bar) grid_sync(P.bar, ++nbar, P.trace);
+    need_bar = false;
+    if (tid < 32) {   // one warp scans the flags 32 at a time
+      int nx = L;
+      for (int base = s; base < L; base += 32) {
+        const uint32_t f = base + tid < L ? __ldcg(P.sl_cnt + base + tid) : 0u;
+        const uint32_t hit = __ballot_sync(0xffffffffu, f != 0u);
+        if (hit) {
+          nx = base + __ffs(hit) - 1;
+          const uint32_t fv = __shfl_sync(0xffffffffu, f, __ffs(hit) - 1);
+          if (tid == 0) cs.cnt = fv;
+          break;
+        }
+      }
+      if (tid == 0) cs.next = nx;
+    }
+    __syncthreads();
+    s = cs.next;
+    const uint32_t lvl = cs.cnt;
+    __syncthreads();
+    if (s >= L) break;
+    need_bar = true;
+    const int4 sc = slice_of(P, s_slc, s);
+    for (int h = sc.x + tid; h < sc.y; h += blockDim.x) {
+      const HeadTopo t = load_topo(P, h);
+      const EntSrc E{P.ext_w + t.x0, P.ext_f + t.x0, P.ext_ms + t.x0, P.ext_fms + t.x0, nullptr};
+      if (!head_dirty(P, h, E.w, t.nf, lvl, stamp)) continue;
+      nrec += uint32_t(sl_fwd_head<kLSE, true>(P, h, t, E, cs.mark, s_slp, stamp));
+    }
+    __syncthreads();
+    mark_flush(P, cs.mark, cs.pub);
+  }
+}
+
 // kMode 0: full pass.  1: cone pass over the staged slices (large updates).
 // 2: cone pass reading only the dirty heads' topology (small updates).  The
 // cone passes recompute dirty heads only and skip (without a barrier) every
@@ -505,138 +591,113 @@ __device__ __forceinline__ void mark_flush(const SLParams& P, uint32_t* s_mark, 
 template <bool kLSE, int kMode>
 __global__ void __launch_bounds__(kSLFwdThreads, 1) fwdl_kernel(SLParams P) {
   constexpr bool kInc = kMode != 0;
-  constexpr bool kStaged = kMode != 2;
   extern __shared__ __align__(128) unsigned char sl_smem[];
-  __shared__ uint32_t s_mark[2 * kMarkWords], s_pub[2 * kMarkWords];
-  __shared__ uint32_t s_cnt;
+  __shared__ ConeSm cs;
   const int gt = blockIdx.x * blockDim.x + threadIdx.x;
   const int nthr = gridDim.x * blockDim.x;
   const int tid = threadIdx.x;
   const int L = P.num_sl;
   uint32_t nbar = 0, nrec = 0;
   if (P.trace && gt == 0) P.trace[0] = gtimer();
-  for (int k = tid; k < 2 * kMarkWords; k += blockDim.x) s_mark[k] = s_pub[k] = 0u;
+  for (int k = tid; k < 2 * kMarkWords; k += blockDim.x) cs.mark[k] = cs.pub[k] = 0u;
   FStageSet* S = reinterpret_cast<FStageSet*>(sl_smem);
   int4* s_slc = reinterpret_cast<int4*>(sl_smem + kFSlcOff);
   int32_t* s_slp = reinterpret_cast<int32_t*>(s_slc + kSliceCap);   // level table (cone: level of a head)
   load_slices(P, s_slc);
   for (int v = tid; v <= min(P.num_sl, kSliceCap); v += blockDim.x) s_slp[v] = __ldg(P.sl_ptr + v);
   __syncthreads();
-  if (kStaged && tid == 0) {
-    mbar_init(&S->full[0]);
-    mbar_init(&S->full[1]);
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    if (L > 1) {
-      const int4 c = slice_of(P, s_slc, 1);
-      fwd_issue(P, S, 1, c.x, c.y, c.z, c.w);
-    }
-  }
-  if (!kInc) {
-    for (int s = gt; s < L; s += nthr) P.sl_cnt[s] = 0u;   // a full pass supersedes pending flags
-    // startpoints: clock arrival distribution, mean and variance per rf
-    for (int i = gt; i < P.num_src; i += nthr) {
-      const float4 v = __ldg(P.src_ms + i);
-      st_state(P.state + i, double(v.x), double(v.y), double(v.z) * double(v.z), double(v.w) * double(v.w), P.par);
-    }
-  }
-  uint32_t phase[2] = {0u, 0u};
-  bool need_bar = !kInc;   // cone: flags of level 1 come from insta_update_arcs (an earlier launch)
-  __shared__ int s_next;
-  for (int s = 1; s < L; ++s) {
-    if (kMode == 2) {
-      // unstaged cone: no staging pipeline to keep, so jump straight to the next
-      // flagged level -- every flag at or past s is final (no level ran since
-      // the last barrier); one warp scans them 32 at a time
-      if (need_bar) grid_sync(P.bar, ++nbar, P.trace);
-      need_bar = false;
-      if (tid < 32) {
-        int nx = L;
-        for (int base = s; base < L; base += 32) {
-          const uint32_t f = base + tid < L ? __ldcg(P.sl_cnt + base + tid) : 0u;
-          const uint32_t hit = __ballot_sync(0xffffffffu, f != 0u);
-          if (hit) {
-            nx = base + __ffs(hit) - 1;
-            break;
-          }
-        }
-        if (tid == 0) s_next = nx;
+  if constexpr (kMode == 2) {
+    cone_levels<kLSE>(P, P.stamp, cs, s_slc, s_slp, nbar, nrec);
+  } else {
+    if (tid == 0) {
+      mbar_init(&S->full[0]);
+      mbar_init(&S->full[1]);
+      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+      if (L > 1) {
+        const int4 c = slice_of(P, s_slc, 1);
+        fwd_issue(P, S, 1, c.x, c.y, c.z, c.w);
       }
-      __syncthreads();
-      s = s_next;
-      __syncthreads();
-      if (s >= L) break;
     }
-    const int bf = s & 1;
-    __syncthreads();   // every thread is done with level s - 1 (rows buffer bf ^ 1)
-    if (kStaged && tid == 0 && s + 1 < L) {   // rows and entry words of level s + 1
-      const int4 c = slice_of(P, s_slc, s + 1);
-      fwd_issue(P, S, bf ^ 1, c.x, c.y, c.z, c.w);
+    if (!kInc) {
+      for (int s = gt; s < L; s += nthr) P.sl_cnt[s] = 0u;   // a full pass supersedes pending flags
+      // startpoints: clock arrival distribution, mean and variance per rf
+      for (int i = gt; i < P.num_src; i += nthr) {
+        const float4 v = __ldg(P.src_ms + i);
+        st_state(P.state + i, double(v.x), double(v.y), double(v.z) * double(v.z), double(v.w) * double(v.w), P.par);
+      }
     }
-    if (kMode != 2 && need_bar) grid_sync(P.bar, ++nbar, P.trace);   // levels < s are complete
-    unsigned long long* ph = nullptr;
+    uint32_t phase[2] = {0u, 0u};
+    bool need_bar = !kInc;   // cone: flags of level 1 come from insta_update_arcs (an earlier launch)
+    for (int s = 1; s < L; ++s) {
+      const int bf = s & 1;
+      __syncthreads();   // every thread is done with level s - 1 (rows buffer bf ^ 1)
+      if (tid == 0 && s + 1 < L) {   // rows and entry words of level s + 1
+        const int4 c = slice_of(P, s_slc, s + 1);
+        fwd_issue(P, S, bf ^ 1, c.x, c.y, c.z, c.w);
+      }
+      if (need_bar) grid_sync(P.bar, ++nbar, P.trace);   // levels < s are complete
+      unsigned long long* ph = nullptr;
 #ifdef INSTA_SL_PHASES
-    if (P.trace && tid == 0) {   // debug: per (level, CTA) timestamps
-      ph = P.trace + 512 + size_t(L + 8) * 2 * gridDim.x + (size_t(s) * gridDim.x + blockIdx.x) * 8;
-      ph[0] = gtimer();
-    }
+      if (P.trace && tid == 0) {   // debug: per (level, CTA) timestamps
+        ph = P.trace + 512 + size_t(L + 8) * 2 * gridDim.x + (size_t(s) * gridDim.x + blockIdx.x) * 8;
+        ph[0] = gtimer();
+      }
 #endif
-    bool work = true;
-    uint32_t lvl = 0;
-    if (kInc) {   // flags of level s come from levels < s: final here
-      if (tid == 0) s_cnt = __ldcg(P.sl_cnt + s);
-      __syncthreads();
-      lvl = s_cnt;
-      work = lvl != 0;
-      need_bar = work;
+      bool work = true;
+      uint32_t lvl = 0;
+      if (kInc) {   // flags of level s come from levels < s: final here
+        if (tid == 0) cs.cnt = __ldcg(P.sl_cnt + s);
+        __syncthreads();
+        lvl = cs.cnt;
+        work = lvl != 0;
+        need_bar = work;
 #ifdef INSTA_SL_PHASES
-      if (ph) ph[1] = gtimer();
+        if (ph) ph[1] = gtimer();
 #endif
-    }
-    const int4 sc = slice_of(P, s_slc, s);
-    const int a = sc.x, b = sc.y;
-    bool ok = false;
-    if (kStaged) {
+      }
+      const int4 sc = slice_of(P, s_slc, s);
+      const int a = sc.x, b = sc.y;
       mbar_wait(&S->full[bf], phase[bf]);
       phase[bf] ^= 1u;
-      ok = S->ok[bf] != 0;
-    }
+      const bool ok = S->ok[bf] != 0;
 #ifdef INSTA_SL_PHASES
-    if (ph) ph[2] = gtimer();
+      if (ph) ph[2] = gtimer();
 #endif
-    if (!work) continue;
-    const Window wp = window(a, b + 1, 4), wh = window(a, b, 4);
-    const int xa = sc.z;
-    const Window wx = window(xa, sc.w, 4);
-    for (int h = a + tid; h < b; h += blockDim.x) {
-      const int r = h - a;
-      HeadTopo t;
-      EntSrc E;   // entry words, arc records: staged slice, or global
-      if (ok) {
-        t.x0 = S->ptr[bf][wp.off + r];
-        t.nf = S->ptr[bf][wp.off + r + 1] - t.x0;
-        t.pin = S->pin[bf][wh.off + r];
-        const int xr = wx.off + t.x0 - xa;
-        E = EntSrc{S->w[bf] + xr, S->f[bf] + xr, P.ext_ms + t.x0, P.ext_fms + t.x0, nullptr};
-      } else {
-        t = load_topo(P, h);
-        E = EntSrc{P.ext_w + t.x0, P.ext_f + t.x0, P.ext_ms + t.x0, P.ext_fms + t.x0, nullptr};
+      if (!work) continue;
+      const Window wp = window(a, b + 1, 4), wh = window(a, b, 4);
+      const int xa = sc.z;
+      const Window wx = window(xa, sc.w, 4);
+      for (int h = a + tid; h < b; h += blockDim.x) {
+        const int r = h - a;
+        HeadTopo t;
+        EntSrc E;   // entry words, arc records: staged slice, or global
+        if (ok) {
+          t.x0 = S->ptr[bf][wp.off + r];
+          t.nf = S->ptr[bf][wp.off + r + 1] - t.x0;
+          t.pin = S->pin[bf][wh.off + r];
+          const int xr = wx.off + t.x0 - xa;
+          E = EntSrc{S->w[bf] + xr, S->f[bf] + xr, P.ext_ms + t.x0, P.ext_fms + t.x0, nullptr};
+        } else {
+          t = load_topo(P, h);
+          E = EntSrc{P.ext_w + t.x0, P.ext_f + t.x0, P.ext_ms + t.x0, P.ext_fms + t.x0, nullptr};
+        }
+        if (kInc) {
+          if (!head_dirty(P, h, E.w, t.nf, lvl, P.stamp)) continue;
+          nrec += uint32_t(sl_fwd_head<kLSE, true>(P, h, t, E, cs.mark, s_slp, P.stamp, ph));
+        } else {
+          (void)sl_fwd_head<kLSE, false>(P, h, t, E, cs.mark, s_slp, P.stamp, ph);
+        }
       }
+#ifdef INSTA_SL_PHASES
+      if (ph) ph[5] = gtimer();
+#endif
       if (kInc) {
-        if (!head_dirty(P, h, E.w, t.nf, lvl)) continue;
-        nrec += uint32_t(sl_fwd_head<kLSE, true>(P, h, t, E, s_mark, s_slp, ph));
-      } else {
-        (void)sl_fwd_head<kLSE, false>(P, h, t, E, s_mark, s_slp, ph);
+        __syncthreads();
+        mark_flush(P, cs.mark, cs.pub);
+#ifdef INSTA_SL_PHASES
+        if (ph) ph[6] = gtimer();
+#endif
       }
-    }
-#ifdef INSTA_SL_PHASES
-    if (ph) ph[5] = gtimer();
-#endif
-    if (kInc) {
-      __syncthreads();
-      mark_flush(P, s_mark, s_pub);
-#ifdef INSTA_SL_PHASES
-      if (ph) ph[6] = gtimer();
-#endif
     }
   }
   if (kInc) {
@@ -646,6 +707,103 @@ __global__ void __launch_bounds__(kSLFwdThreads, 1) fwdl_kernel(SLParams P) {
     const uint32_t n = __reduce_add_sync(0xffffffffu, nrec);
     if ((tid & 31) == 0 && n) atomicAdd(P.counters, (unsigned long long)n);
   }
+  grid_exit(P.bar);
+}
+
+// --------------------------------------------------------------------------
+// One-cell what-if candidates (insta_eval_candidates; SURVEY §8(f) C5
+// INSTA-Size "estimate the timing of each candidate"), all in ONE persistent
+// launch.  Per candidate i (stamps 2i / 2i + 1 past the graph's epoch):
+//   A  save the records of its arcs                          | barrier
+//   B  write its records, stamp the heads evaluating them     | barrier
+//   C  cone pass (levels flagged, one barrier per level)      | barrier
+//   D  clear the level flags; recompute the flagged slack blocks' partials
+//      (slack_common.cuh: the same per-block arithmetic as slack_kernel)  | barrier
+//   E  CTA 0: the final slack reduction -> cand_out[i]; every CTA: write the
+//      saved records back, stamp                              | barrier
+//   F  cone pass again (reverts every record)                 | barrier
+//   G  clear the level flags; recompute the flagged blocks again (base
+//      partials, slack and rf* restored bit for bit); then A of i + 1.
+// The flagged-block set is cleared in B of the next candidate (read in D, G).
+// --------------------------------------------------------------------------
+template <bool kLSE>
+__device__ __forceinline__ void eval_apply(const SLParams& P, int i, bool revert, uint32_t stamp) {
+  const int a0 = __ldg(P.cand_ptr + i), a1 = __ldg(P.cand_ptr + i + 1);
+  for (int k = a0 + blockIdx.x * blockDim.x + threadIdx.x; k < a1; k += gridDim.x * blockDim.x) {
+    const int id = __ldg(P.cand_arc + k);
+    float4 r;
+    if (revert) {
+      r = P.cand_old[k];
+    } else {
+      const float2 m = __ldg(P.cand_m + k), sg = __ldg(P.cand_s + k);
+      r = make_float4(m.x, m.y, sg.x, sg.y);
+    }
+    P.fin_ms[__ldg(P.arc_pos + id)] = r;
+    const int x = __ldg(P.arc_xpos + id);   // the stage-folded schedule's copy of the record
+    ((x & 1) ? P.ext_fms_w : P.ext_ms_w)[x >> 1] = r;
+    const int h = __ldg(P.arc_head + id);
+    P.dirty[h] = stamp;
+    int lo = 0, hi = P.num_sl;   // its super-level is flagged
+    while (hi - lo > 1) {
+      const int mid = (lo + hi) >> 1;
+      if (__ldg(P.sl_ptr + mid) <= h) lo = mid;
+      else hi = mid;
+    }
+    atomicOr(P.sl_cnt + lo, 1u);
+  }
+}
+
+__device__ __forceinline__ void eval_save(const SLParams& P, int i) {
+  const int a0 = __ldg(P.cand_ptr + i), a1 = __ldg(P.cand_ptr + i + 1);
+  for (int k = a0 + blockIdx.x * blockDim.x + threadIdx.x; k < a1; k += gridDim.x * blockDim.x)
+    P.cand_old[k] = __ldcg(P.fin_ms + __ldg(P.arc_pos + __ldg(P.cand_arc + k)));
+}
+
+// flagged slack blocks of this CTA (b = blockIdx.x, blockIdx.x + grid, ...)
+__device__ __forceinline__ void eval_slack_blocks(const SLParams& P, SlackRed& sr) {
+  for (int b = blockIdx.x; b < P.slack_nb; b += gridDim.x) {
+    if (!((__ldcg(P.ep_blk + (b >> 5)) >> (b & 31)) & 1u)) continue;
+    slack_block(b, P.slack_nb, P.num_ep, P.ep_pin, P.ep_rat, P.state, double(P.n_sigma), P.slack, P.rf_star,
+                P.partials, sr);
+  }
+}
+
+template <bool kLSE>
+__global__ void __launch_bounds__(kSLFwdThreads, 1) eval_kernel(SLParams P) {
+  extern __shared__ __align__(128) unsigned char sl_smem[];
+  __shared__ ConeSm cs;
+  __shared__ SlackRed sr;
+  int4* s_slc = reinterpret_cast<int4*>(sl_smem);
+  int32_t* s_slp = reinterpret_cast<int32_t*>(s_slc + kSliceCap);
+  const int tid = threadIdx.x, gt = blockIdx.x * blockDim.x + tid, nthr = gridDim.x * blockDim.x;
+  const int L = P.num_sl, nw = (P.slack_nb + 31) / 32;
+  load_slices(P, s_slc);
+  for (int v = tid; v <= min(P.num_sl, kSliceCap); v += blockDim.x) s_slp[v] = __ldg(P.sl_ptr + v);
+  uint32_t nbar = 0, nrec = 0;
+  if (P.num_cand > 0) eval_save(P, 0);
+  for (int i = 0; i < P.num_cand; ++i) {
+    grid_sync(P.bar, ++nbar, P.trace);                                          // A done
+    for (int w = gt; w < nw; w += nthr) P.ep_blk[w] = 0u;                      // read in D, G of i - 1
+    for (int k = tid; k < 2 * kMarkWords; k += blockDim.x) cs.mark[k] = cs.pub[k] = 0u;
+    eval_apply<kLSE>(P, i, false, P.stamp + 2 * i);
+    grid_sync(P.bar, ++nbar, P.trace);                                          // B done
+    cone_levels<kLSE>(P, P.stamp + 2 * i, cs, s_slc, s_slp, nbar, nrec);
+    grid_sync(P.bar, ++nbar, P.trace);                                          // C done
+    for (int s = gt; s < L; s += nthr) P.sl_cnt[s] = 0u;
+    eval_slack_blocks(P, sr);
+    grid_sync(P.bar, ++nbar, P.trace);                                          // D done
+    if (blockIdx.x == 0) slack_final(P.slack_nb, P.partials, P.cand_out + 3 * size_t(i), sr);
+    for (int k = tid; k < 2 * kMarkWords; k += blockDim.x) cs.mark[k] = cs.pub[k] = 0u;
+    eval_apply<kLSE>(P, i, true, P.stamp + 2 * i + 1);
+    grid_sync(P.bar, ++nbar, P.trace);                                          // E done
+    cone_levels<kLSE>(P, P.stamp + 2 * i + 1, cs, s_slc, s_slp, nbar, nrec);
+    grid_sync(P.bar, ++nbar, P.trace);                                          // F done
+    for (int s = gt; s < L; s += nthr) P.sl_cnt[s] = 0u;
+    eval_slack_blocks(P, sr);
+    if (i + 1 < P.num_cand) eval_save(P, i + 1);
+  }
+  grid_sync(P.bar, ++nbar, P.trace);
+  for (int w = gt; w < nw; w += nthr) P.ep_blk[w] = 0u;
   grid_exit(P.bar);
 }
 
@@ -803,7 +961,9 @@ __device__ __forceinline__ void sl_bwd_head(const SLParams& P, SLHeavyTab* tab, 
   if (ax | ay) asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %1};" ::"l"(P.acc + 2 * size_t(h)), "l"(0ull));
   const float2 ab = make_float2(sd.x + float(double((long long)ax) * kAccInv),
                                 sd.y + float(double((long long)ay) * kAccInv));
-  if (ab.x == 0.f && ab.y == 0.f) return;   // nothing flows through this head
+  // nothing flows through this head: its arcs keep the zero prefill (scattered zero stores in
+  // caller arc order cost 2.5x the whole backward on B200: measured, profiles/r02_summary.md)
+  if (ab.x == 0.f && ab.y == 0.f) return;
   for (int k = 0; k < nf; ++k) {
     const int x = x0 + k;
     int32_t arc, farc, sh, bw, f;
@@ -973,6 +1133,21 @@ static SLParams sl_params(DevGraph& g) {
   P.hseed = g.hseed;
   P.acc = g.acc_h;
   P.store_fold = 0;
+  P.hd_eop = g.hd_eop;
+  P.ep_blk = nullptr;
+  P.slack_nb = slack_blocks(g.num_ep, g.sl_grid > 0 ? g.sl_grid : 148);
+  P.num_ep = g.num_ep;
+  P.ep_pin = g.ep_pin;
+  P.ep_rat = g.ep_rat;
+  P.slack = g.slack;
+  P.rf_star = g.rf_star;
+  P.partials = g.partials;
+  P.arc_pos = g.arc_pos;
+  P.arc_xpos = g.arc_xpos;
+  P.arc_head = g.arc_head;
+  P.fin_ms = g.fin_ms;
+  P.ext_ms_w = g.ext_ms;
+  P.ext_fms_w = g.ext_fms;
   return P;
 }
 
@@ -980,6 +1155,8 @@ template <class K>
 static cudaError_t sl_smem_attr(K kernel, size_t bytes) {
   return cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(bytes));
 }
+
+constexpr size_t kEvalSmem = sizeof(int4) * kSliceCap + sizeof(int32_t) * (kSliceCap + 4);
 
 int query_sl_grid(int device, int* grid_f, int* grid_b) {
   int sms = 0;
@@ -990,6 +1167,8 @@ int query_sl_grid(int device, int* grid_f, int* grid_b) {
   if (e == cudaSuccess) e = sl_smem_attr(fwdl_kernel<true, 1>, kFStageBytes);
   if (e == cudaSuccess) e = sl_smem_attr(fwdl_kernel<false, 2>, kFStageBytes);
   if (e == cudaSuccess) e = sl_smem_attr(fwdl_kernel<true, 2>, kFStageBytes);
+  if (e == cudaSuccess) e = sl_smem_attr(eval_kernel<false>, kEvalSmem);
+  if (e == cudaSuccess) e = sl_smem_attr(eval_kernel<true>, kEvalSmem);
   if (e == cudaSuccess) e = sl_smem_attr(bwdl_kernel<false>, kBStageBytes);
   if (e == cudaSuccess) e = sl_smem_attr(bwdl_kernel<true>, kBStageBytes);
   if (e != cudaSuccess) return int(e);
@@ -1083,7 +1262,56 @@ int launch_forward_cone(DevGraph& g, float n_sigma, float tau, void* stream) {
   const bool staged = g.pending_updates * 1000 > g.e;
   const void* fn = staged ? (lse ? (const void*)fwdl_kernel<true, 1> : (const void*)fwdl_kernel<false, 1>)
                           : (lse ? (const void*)fwdl_kernel<true, 2> : (const void*)fwdl_kernel<false, 2>);
+  if (g.slack_valid) P.ep_blk = g.ep_blk;   // insta_forward follows with the slack of the flagged blocks only
   const int err = launch_coop(fn, g.sl_grid, kSLFwdThreads, kFStageBytes, P, st, "cone");
+  g.folded_valid = false;
+  return err;
+}
+
+// All candidates in one persistent launch (eval_kernel).  cand_ptr: host; the
+// arc arrays on the device.  Stamps past the graph's epoch, 2 per candidate.
+int launch_eval_candidates(DevGraph& g, int num, const int32_t* cand_ptr, const int32_t* arc_ids, const float* mean,
+                           const float* sigma, double* out, void* stream) {
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (num <= 0) return 0;
+  const int total = cand_ptr[num];
+  cudaError_t e = cudaSuccess;
+  if (g.cand_ptr_cap < num + 1) {
+    if (g.cand_ptr_d) cudaFree(g.cand_ptr_d);
+    g.cand_ptr_d = nullptr;
+    g.cand_ptr_cap = 0;
+    e = cudaMalloc(&g.cand_ptr_d, sizeof(int32_t) * size_t(num + 1));
+    if (e != cudaSuccess) return int(e);
+    g.cand_ptr_cap = num + 1;
+  }
+  if (g.cand_cap < total) {   // float4 per candidate arc (saved records)
+    if (g.cand_old) cudaFree(g.cand_old);
+    g.cand_old = nullptr;
+    g.cand_cap = 0;
+    e = cudaMalloc(reinterpret_cast<void**>(&g.cand_old), sizeof(float4) * size_t(std::max(total, 1)));
+    if (e != cudaSuccess) return int(e);
+    g.cand_cap = total;
+  }
+  e = cudaMemcpyAsync(g.cand_ptr_d, cand_ptr, sizeof(int32_t) * size_t(num + 1), cudaMemcpyHostToDevice, st);
+  if (e != cudaSuccess) return int(e);
+  SLParams P = sl_params(g);
+  P.n_sigma = g.last_n_sigma;
+  P.tau = g.last_tau;
+  P.inv_tau = g.last_tau > 0.f ? 1.0 / double(g.last_tau) : 0.0;
+  P.par = g.pass_fwd & 1u;
+  P.stamp = g.inc_epoch + 1;
+  g.inc_epoch += 2 * uint32_t(num);
+  P.ep_blk = g.ep_blk;
+  P.cand_ptr = g.cand_ptr_d;
+  P.cand_arc = arc_ids;
+  P.cand_m = reinterpret_cast<const float2*>(mean);
+  P.cand_s = reinterpret_cast<const float2*>(sigma);
+  P.cand_old = reinterpret_cast<float4*>(g.cand_old);
+  P.cand_out = out;
+  P.num_cand = num;
+  const bool lse = g.last_tau > 0.f;
+  const int err = launch_coop(lse ? (const void*)eval_kernel<true> : (const void*)eval_kernel<false>, g.sl_grid,
+                              kSLFwdThreads, kEvalSmem, P, st, "eval");
   g.folded_valid = false;
   return err;
 }

@@ -396,6 +396,124 @@ __global__ void __launch_bounds__(256, 8) tk_one_kernel(TkParams P) {
   }
 }
 
+// K in (32, kTkWideMax]: a warp per (pin, rf) with its queue in shared memory
+// (kTkWideCap entries: the K queue slots plus one chunk of new candidates,
+// padded to a power of two).  Candidates arrive 32 at a time (one parent
+// queue's slots, unique startpoints, in Alg 1's k order); when the queue is
+// full, those whose (A, t) key is below its last slot are pruned (they can
+// neither enter nor beat their startpoint's entry); each survivor looks up its
+// startpoint in the queue (a found one replaces its entry only with a larger
+// key, else it is dropped), new ones are appended, and the queue is re-sorted
+// by key (warp bitonic sort in shared memory) and cut to K.  This maintains
+// the R19 closed form (the K best startpoints by their best candidate's key),
+// so the result equals the literal sequential Alg 2 bit for bit.
+constexpr int kTkWideMax = 128, kTkWideCap = 256, kTkWideWarps = 4;
+struct TkWideSm {
+  double A[kTkWideCap], mu[kTkWideCap], var[kTkWideCap];
+  int t[kTkWideCap], sp[kTkWideCap];
+};
+
+__device__ __forceinline__ void tk_sm_put(TkWideSm& Q, int j, const TkEnt& c) {
+  Q.A[j] = c.A;
+  Q.mu[j] = c.mu;
+  Q.var[j] = c.var;
+  Q.t[j] = c.t;
+  Q.sp[j] = c.sp;
+}
+
+__device__ __forceinline__ void tk_sm_swap(TkWideSm& Q, int i, int j) {
+  const double a = Q.A[i], m = Q.mu[i], v = Q.var[i];
+  const int t = Q.t[i], sp = Q.sp[i];
+  Q.A[i] = Q.A[j];
+  Q.mu[i] = Q.mu[j];
+  Q.var[i] = Q.var[j];
+  Q.t[i] = Q.t[j];
+  Q.sp[i] = Q.sp[j];
+  Q.A[j] = a;
+  Q.mu[j] = m;
+  Q.var[j] = v;
+  Q.t[j] = t;
+  Q.sp[j] = sp;
+}
+
+// descending (A, t) order of Q[0, n): bitonic over the next power of two, the tail padded empty
+__device__ __forceinline__ void tk_sm_sort(TkWideSm& Q, int n, int lane) {
+  int P2 = 1;
+  while (P2 < n) P2 <<= 1;
+  for (int j = n + lane; j < P2; j += 32) tk_sm_put(Q, j, tk_empty());
+  __syncwarp();
+  for (int size = 2; size <= P2; size <<= 1) {
+    for (int stride = size >> 1; stride > 0; stride >>= 1) {
+      for (int p = lane; p < (P2 >> 1); p += 32) {
+        const int i = 2 * p - (p & (stride - 1)), j = i + stride;
+        const bool desc = (i & size) == 0;
+        const bool sw = desc ? key_gt(Q.A[j], Q.t[j], Q.A[i], Q.t[i]) : key_gt(Q.A[i], Q.t[i], Q.A[j], Q.t[j]);
+        if (sw) tk_sm_swap(Q, i, j);
+      }
+      __syncwarp();
+    }
+  }
+}
+
+__global__ void __launch_bounds__(32 * kTkWideWarps) tk_wide_kernel(TkParams P) {
+  __shared__ TkWideSm S[kTkWideWarps];
+  const int lane = threadIdx.x & 31;
+  TkWideSm& Q = S[threadIdx.x >> 5];
+  const long long grp = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
+  if (grp >= 2LL * (P.hi - P.lo)) return;   // uniform within the warp
+  const int i = __ldg(P.list + P.lo + int(grp >> 1)), rf = int(grp & 1), K = P.K;
+  const int b0 = __ldg(P.fanin_ptr + i), b1 = __ldg(P.fanin_ptr + i + 1), nf = b1 - b0;
+  int n = 0;
+  for (int r = b0; r < b1; ++r) {   // fanin arcs in row order (Alg 1 l.7-8)
+    const int32_t w = __ldg(P.fin_src + r);
+    const int u = int(uint32_t(w) >> kUnateShift);
+    const float4 ms = __ldg(P.fin_ms + r);
+    const double am = double(rf ? ms.y : ms.x), se = double(rf ? ms.w : ms.z);
+    for (int si = 0; si < n_src_tr(u); ++si) {
+      const size_t ps0 = (size_t(w & kSrcMask) * 2 + src_tr(rf, u, si)) * K;
+      for (int k0 = 0; k0 < K; k0 += 32) {
+        const int k = k0 + lane;
+        const int csp = k < K ? __ldg(P.qsp + ps0 + k) : -1;
+        const double2 pv = k < K ? __ldg(P.q + ps0 + k) : make_double2(0.0, 0.0);
+        TkEnt c;
+        c.sp = csp;
+        c.t = (k * nf + (r - b0)) * 2 + si;          // Alg 1 order: k outer, arcs, s
+        c.mu = pv.x + am;                            // Eq 1 (l.12)
+        c.var = pv.y + se * se;                      // Eq 2 (l.13)
+        c.A = csp >= 0 ? c.mu + P.ns * double(sigma_of(c.var)) : -INFINITY;   // Eq 3 (l.14)
+        bool live = csp >= 0;
+        if (n == K) live = live && key_gt(c.A, c.t, Q.A[K - 1], Q.t[K - 1]);
+        if (!__ballot_sync(0xffffffffu, live)) continue;
+        int f = -1;
+        if (live)
+          for (int j = 0; j < n; ++j)
+            if (Q.sp[j] == csp) {
+              f = j;
+              break;
+            }
+        const bool rep = live && f >= 0 && key_gt(c.A, c.t, Q.A[f], Q.t[f]);
+        const bool ins = live && f < 0;
+        __syncwarp();
+        if (rep) tk_sm_put(Q, f, c);
+        const unsigned mi = __ballot_sync(0xffffffffu, ins);
+        if (ins) tk_sm_put(Q, n + __popc(mi & ((1u << lane) - 1u)), c);
+        const bool changed = __ballot_sync(0xffffffffu, rep || ins) != 0u;
+        __syncwarp();
+        if (!changed) continue;
+        const int n2 = n + __popc(mi);
+        tk_sm_sort(Q, n2, lane);
+        n = min(n2, K);
+      }
+    }
+  }
+  for (int k = lane; k < K; k += 32) {
+    const size_t o = (size_t(i) * 2 + rf) * K + k;
+    const bool v = k < n;
+    P.q[o] = v ? make_double2(Q.mu[k], Q.var[k]) : make_double2(0.0, 0.0);
+    P.qsp[o] = v ? Q.sp[k] : -1;
+  }
+}
+
 // CPPR slack: warp per endpoint; slack = min over (rf, k) of
 // RAT(ep, SP_k)[rf] - A_k[rf], the first minimum in (rf, k) order wins.
 __global__ void __launch_bounds__(256)
@@ -613,6 +731,16 @@ int launch_topk_forward(DevGraph& g, int K, float n_sigma, void* stream) {
   P.fin_ms = g.fin_ms;
   P.q = g.tk_q;
   P.qsp = g.tk_sp;
+  if (K > 32) {   // wide queues: a warp per (pin, rf), every pin of a level in one launch
+    for (int l = 1; l < g.num_levels; ++l) {
+      P.lo = g.tk_one_ptr[l];
+      P.hi = g.tk_one_ptr[l + 1];
+      if (P.hi <= P.lo) continue;
+      const long long warps = 2LL * (P.hi - P.lo);
+      tk_wide_kernel<<<unsigned((warps + kTkWideWarps - 1) / kTkWideWarps), 32 * kTkWideWarps, 0, st>>>(P);
+    }
+    return int(cudaGetLastError());
+  }
   const int G = pow2_group(K);
   // The two parts of a level are independent: the bandwidth-bound single-arc
   // kernel runs on a side stream next to the ALU-bound merging kernel on the

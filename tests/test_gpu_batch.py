@@ -141,14 +141,26 @@ def test_eval_candidates_cone(tau):
     insta_forward on its materialized graph bit for bit, and the graph returns to its base state."""
     g = synth.generate("C2")
     scs = [synth.sizing_scenario(g, s) for s in range(512, 512 + 24)]
+    # an empty candidate (the base state) and one listing an arc twice with the same record
+    scs.insert(3, dict(n_sigma=3.0, derate_cell=1.0, derate_net=1.0, delta_arc=np.zeros(0, np.int32),
+                       delta_mean=np.zeros((0, 2), np.float32), delta_sigma=np.zeros((0, 2), np.float32)))
+    d = scs[5]
+    scs.insert(6, dict(d, delta_arc=np.concatenate([d["delta_arc"], d["delta_arc"][:1]]),
+                       delta_mean=np.concatenate([d["delta_mean"], d["delta_mean"][:1]]),
+                       delta_sigma=np.concatenate([d["delta_sigma"], d["delta_sigma"][:1]])))
     G = insta.Graph(g)
     base = G.forward(3.0, tau)
     A0 = G.arrivals()[0].cpu().numpy()
+    sl0 = G.slack()[0].cpu().numpy()
     d0 = G.backward().cpu().numpy()
     summ = G.eval_candidates(scs).cpu().numpy()
     assert np.array_equal(G.arrivals()[0].cpu().numpy(), A0)
+    assert np.array_equal(G.slack()[0].cpu().numpy(), sl0)
     assert np.array_equal(G.backward().cpu().numpy(), d0)
     assert G.summary().tns == base.tns
+    assert summ[3, 1] == base.tns and summ[3, 0] == base.wns
+    # a second batch on the restored state gives the same summaries
+    assert np.array_equal(G.eval_candidates(scs[:8]).cpu().numpy(), summ[:8])
     G.close()
     for k, sc in enumerate(scs):
         H = insta.Graph(materialize(g, sc))

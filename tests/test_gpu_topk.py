@@ -49,7 +49,7 @@ def _table64(t):
     return None if t is None else (t[0], t[1], np.asarray(t[2], np.float64))
 
 
-@pytest.mark.parametrize("K", [1, 2, 3, 4, 8, 32])
+@pytest.mark.parametrize("K", [1, 2, 3, 4, 8, 32, 33, 64, 128])
 @pytest.mark.parametrize("seed", range(6))
 def test_topk_dyadic_tiny_bit_exact(K, seed):
     g = bf.tiny_dag(seed, n_pins=9, p_edge=0.5, sigma0=True, dyadic=True, n_ep=5)
@@ -63,7 +63,7 @@ def test_topk_dyadic_tiny_bit_exact(K, seed):
     assert gq.summary.tns == os_["tns"]
 
 
-@pytest.mark.parametrize("K", [1, 3, 8, 32])
+@pytest.mark.parametrize("K", [1, 3, 8, 32, 33, 64, 128])
 def test_topk_dyadic_c1_bit_exact_with_cppr(K):
     g = synth.generate("C1", dyadic=True)
     table = synth.cppr_rat_table(g, dyadic=True)
@@ -86,7 +86,7 @@ def _near_tie_rows(oq, eps=1e-3):
     return (np.nan_to_num(d, nan=np.inf, posinf=np.inf) <= eps).any(axis=2)
 
 
-@pytest.mark.parametrize("cfg,K", [("C1", 1), ("C1", 8), ("C1", 32), ("C2", 4), ("C2", 16)])
+@pytest.mark.parametrize("cfg,K", [("C1", 1), ("C1", 8), ("C1", 32), ("C1", 128), ("C2", 4), ("C2", 16), ("C2", 64)])
 def test_topk_sigma_parity(cfg, K):
     g = synth.generate(cfg)
     table = synth.cppr_rat_table(g)
@@ -149,7 +149,7 @@ def test_topk_errors():
     with pytest.raises(insta.InstaError, match="E_ARG"):
         G.topk_forward(0, NS)
     with pytest.raises(insta.InstaError, match="E_ARG"):
-        G.topk_forward(33, NS)
+        G.topk_forward(129, NS)
     non_source = int(g.arc_to[0])
     with pytest.raises(insta.InstaError, match="E_ARG"):
         G.set_cppr_rat(np.array([0] + [1] * g.num_endpoints), np.array([non_source]), np.array([[1.0, 1.0]]))
@@ -193,4 +193,12 @@ def test_topk_c4_invariants():
     # (entry 0 is NOT bounded below by the hard arrival when sigma > 0: the hard state of a pin need not be
     # its startpoint's best-key entry, and sqrt(var + std^2) can reorder them downstream)
     assert summ.num_violations > 0 and np.isfinite(summ.tns)
+    del q, A, sp, valid, both, s_sorted, dup
+    # K = 128 (the paper's CPPR study) at full size: its first 8 slots are the K = 8 queue (the
+    # queue is a key-ordered top-K set), so its CPPR slack can only be lower, endpoint by endpoint
+    sl8 = sl.clone()
+    G.topk_forward(128, NS)
+    summ128, sl128, _ = G.topk_slack()
+    assert (sl128 <= sl8).all()
+    assert summ128.tns <= summ.tns and summ128.num_violations >= summ.num_violations
     G.close()
