@@ -116,8 +116,8 @@ def survey_bytes(N, E, P, lse):
 
 
 def sched0_bytes(sc, N, E, n_src, P, nnz_arcs, lse):
-    """Bytes the default schedule's kernels move (this layout): forward (stage-folded
-    dataflow kernel, folded pins kept in registers) 8 B/head (row, pin) + per entry 20 B (source
+    """Bytes the default schedule's kernels move (this layout): forward (entry-parallel
+    sweep fwdx_kernel, folded pins kept in registers) 8 B/head (row, pin) + per entry 20 B (source
     word, record of e) + a 32 B source-record gather + 20 B/folded pin (word, record of e') + a 32 B
     record store per head + arg-max 4 B/head (hard) or Eq 6 weights 16 B/entry (LSE) + 16 B/startpoint
     + 41 B/endpoint (slack); backward (sweep) 8 B/arc zero fill + 25 B/endpoint seeds + per head
@@ -334,7 +334,7 @@ def main():
         except Exception:
             traffic = None
     roofline = {
-        "bound": "hbm", "kernel": ("fwd_kernel<stage-folded dataflow> + slack_kernel (insta_forward)" if dom == "fwd"
+        "bound": "hbm", "kernel": ("fwdx_kernel<entry-parallel sweep, parity dataflow> + slack_kernel (insta_forward)" if dom == "fwd"
                                    else "bwd_prep_kernel + bwdl_kernel<sweep> (insta_backward)"),
         "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak, "peak_kind": peak_kind,
         "traffic": traffic, "traffic_source": "profiles/traffic.json: ncu --set full dram__bytes_read.sum + "
@@ -732,9 +732,9 @@ def main():
             "config": {"workload": f"{cfg.name}: synthetic 3nm-shaped timing graph, {N} pins, {E} arcs, "
                                    f"{P} endpoints, {G.num_levels} levels",
                        "pins": N, "arcs": E, "endpoints": P, "levels": G.num_levels, "tau": args.tau,
-                       "n_sigma": 3.0, "schedule": {0: "dataflow forward + sweep backward", 1: "per-level",
+                       "n_sigma": 3.0, "schedule": {0: "entry-parallel dataflow sweep forward + sweep backward", 1: "per-level",
                                                     2: "dataflow forward + dataflow backward",
-                                                    3: "sweep forward + sweep backward"}[args.schedule],
+                                                    3: "entry-parallel sweep forward (level barriers) + sweep backward"}[args.schedule],
                        "super_levels": sched["num_super_levels"], "folded_pins": sched["num_folded"],
                        "parallelism": f"replicas x{world}",
                        "l2": "working set > 126 MB L2 (no flush between passes; the `cold` leg flushes)",

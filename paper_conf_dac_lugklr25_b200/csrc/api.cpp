@@ -68,7 +68,7 @@ void free_graph(insta::DevGraph& d) {
                   d.cl_rf,     d.cl_summary, d.cl_hv_list, d.cl_hv_of, d.cl_hv_sum, d.tl_partials, d.sz_tmp,
                   d.sl_ptr,    d.ext_sh,    d.hd_csl,    d.chg,       d.acc_h,     d.sl_bar,    d.sl_cnt,
                   d.hwin,      d.ew,        d.fwin,      d.efw,       d.sl_slice,  d.hfo_ptr,   d.hfo,       d.hd_hsrc,
-                  d.cand_old,  d.ep_blk,    d.cand_ptr_d, d.pl_ptr,    d.pl_ent,    d.pl_arc,    d.pl_wide};
+                  d.cand_old,  d.xscr,  d.ep_blk,    d.cand_ptr_d, d.pl_ptr,    d.pl_ent,    d.pl_arc,    d.pl_wide};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   if (d.b_stage_h) cudaFreeHost(d.b_stage_h);
@@ -336,6 +336,7 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
       for (int64_t c = 0; c < G; ++c) {
         const int32_t a = int32_t(lo + nh * c / G), b = int32_t(lo + nh * (c + 1) / G);
         slc[size_t(sv) * G + c] = make_int4(a, b, fold.hd_ptr[a], fold.hd_ptr[b]);
+        if (sv > 0) d.sl_max_x = std::max(d.sl_max_x, fold.hd_ptr[b] - fold.hd_ptr[a]);
       }
     }
     UP(d.sl_slice, slc.data(), slc.size());
@@ -435,6 +436,18 @@ static insta_status read_summary(insta::DevGraph& d, void* stream, insta_summary
   return INSTA_OK;
 }
 
+// schedule 0's full pass: 2 (default) = entry-parallel sweep without grid barriers (sweep.cu
+// fwdx_kernel, parity dataflow), 1 = the same with level barriers, 0 = the warp-round dataflow
+// kernel of schedule 2 (kernels.cu); INSTA_FWDX overrides (measurements only)
+static int fwdx_mode() {
+  static int m = -1;
+  if (m < 0) {
+    const char* v = getenv("INSTA_FWDX");
+    m = v ? atoi(v) : 2;
+  }
+  return m;
+}
+
 insta_status insta_forward(insta_graph* g, const insta_opts* o, void* cuda_stream,
                            insta_summary* out) {
   if (!g) return fail(INSTA_E_ARG, "forward: NULL graph");
@@ -465,10 +478,11 @@ insta_status insta_forward(insta_graph* g, const insta_opts* o, void* cuda_strea
       d.last_tau = opt.tau;
       err = insta::launch_slack_delta(d, cuda_stream);   // only the slack blocks the cone reached
     }
-  } else if (opt.schedule == 3 || (opt.schedule == 0 && d.parity_mixed)) {
-    // level-synchronous sweep forward (sweep.cu); also the default's full pass
-    // right after a cone pass, whose mixed record parity cannot order a dataflow pass
-    err = insta::launch_forward_sl(d, opt.n_sigma, opt.tau, cuda_stream);
+  } else if (opt.schedule == 3 || (opt.schedule == 0 && (d.parity_mixed || fwdx_mode() != 0))) {
+    // entry-parallel sweep forward (sweep.cu fwdx_kernel): level barriers for schedule 3 and
+    // right after a cone pass (mixed record parity cannot order a dataflow pass)
+    const bool flow = opt.schedule == 0 && !d.parity_mixed && fwdx_mode() == 2;
+    err = insta::launch_forward_sl(d, opt.n_sigma, opt.tau, cuda_stream, flow);
     if (!err) {
       d.last_n_sigma = opt.n_sigma;
       d.last_tau = opt.tau;

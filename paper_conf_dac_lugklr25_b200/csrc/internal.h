@@ -216,6 +216,8 @@ struct DevGraph {
   std::vector<int32_t> h_sl_ptr;   // [SL+1] host copy of the super-level head ranges
   int32_t* sl_ptr = nullptr;       // [SL+1]
   int4* sl_slice = nullptr;        // [SL][sl_grid] per-CTA slices {a, b, xa, xb} of every super-level
+  int32_t sl_max_x = 0;            // most entries in one slice (fwdx_kernel: candidate buffer size)
+  void* xscr = nullptr;            // fwdx_kernel: per-CTA candidate buffers for slices beyond shared memory
   int32_t* ext_sh = nullptr;       // [X] source head of each entry
   int32_t* hd_csl = nullptr;       // [H] consumer super-level range of each head
   int32_t* hfo_ptr = nullptr;      // [H+1] consumer heads of each head
@@ -354,7 +356,7 @@ int launch_update_arcs(DevGraph& g, int64_t n, const int32_t* ids, const float* 
 int launch_arrivals(DevGraph& g, float* A, float* mean, float* sigma, void* stream);
 // sweep.cu: level-synchronous thread-per-head passes (schedule 0)
 int query_sl_grid(int device, int* grid_fwd, int* grid_bwd);
-int launch_forward_sl(DevGraph& g, float n_sigma, float tau, void* stream);
+int launch_forward_sl(DevGraph& g, float n_sigma, float tau, void* stream, bool flow = false);
 int launch_forward_cone(DevGraph& g, float n_sigma, float tau, void* stream);
 int launch_eval_candidates(DevGraph& g, int num, const int32_t* cand_ptr, const int32_t* arc_ids, const float* mean,
                            const float* sigma, double* out, void* stream);

@@ -139,6 +139,10 @@ struct SLParams {
   float4* cand_old;                      // [arcs of all candidates] saved records
   double* cand_out;                      // [n][3]
   int32_t num_cand;
+  // entry-parallel forward (fwdx_kernel): per-CTA candidate buffers in global memory
+  // for slices with more than kXCap entries ([grid][xscr_cap] XCand pairs, then bytes)
+  void* xscr;
+  int32_t xscr_cap;
 };
 
 // --------------------------------------------------------------------------
@@ -711,6 +715,370 @@ __global__ void __launch_bounds__(kSLFwdThreads, 1) fwdl_kernel(SLParams P) {
 }
 
 // --------------------------------------------------------------------------
+// Entry-parallel forward (fwdx_kernel; the default full pass).
+//
+// fwdl_kernel runs a head's whole merge on one thread: the gathers, every
+// folded pin (merge1) and every candidate of both transitions form one serial
+// chain of ~600 instructions, which (ncu: 12 warps / SM, 27 cycles per issued
+// instruction, 60 % of the samples in the CTA barrier waiting for the slowest
+// thread) is what a level costs.  Here a level is two short phases:
+//   (1) entry phase, a thread per entry: gather the source record, evaluate the
+//       folded pin (merge1), form both transitions' candidates (Eq 1-3) and
+//       reduce a non-unate arc's pair (strict ">": the second replaces the first
+//       only if greater), into a shared-memory slot {A0, A1, mu, var} per rf;
+//   (2) head phase, a thread per head: the first arg-max over its entries' slots
+//       in fanin order (strict ">", Alg 2 l.4 / P:L97), the LSE normalizer in
+//       candidate order (Eq 4), the store and the Eq 6 weights.
+// The candidate values are those of make_cand, the arg-max is the one of the
+// sequential scan (a pair pre-reduced with strict ">" then compared with strict
+// ">" selects the same first maximum), the sums run in the same order: the
+// arrivals, arg-max words and weights equal fwdl_kernel's bit for bit.
+// kFlow: no grid barrier -- a gather re-polls a record until its parity is this
+// pass's (the dataflow synchronization of schedule 2); the CTA barriers between
+// the phases and levels stay (they order the shared stage only).
+// --------------------------------------------------------------------------
+// threads per CTA (one CTA per SM): hard mode 768 (<= 80 registers), LSE 512 (its
+// exponentials and weights need more registers; measured best of 384-768 at C4)
+#ifndef INSTA_SX_THREADS
+#define INSTA_SX_THREADS 768
+#endif
+#ifndef INSTA_SX_THREADS_LSE
+#define INSTA_SX_THREADS_LSE 512
+#endif
+constexpr int kSXThreads = INSTA_SX_THREADS;
+constexpr int kSXThreadsLSE = INSTA_SX_THREADS_LSE;
+__host__ __device__ constexpr int sx_threads(bool lse) { return lse ? kSXThreadsLSE : kSXThreads; }
+constexpr int kXCap = 2048;   // entries of a slice held in shared memory
+#ifndef INSTA_SX_PREFETCH
+#define INSTA_SX_PREFETCH 1
+#endif
+constexpr bool kSXPrefetch = INSTA_SX_PREFETCH != 0;   // L2 prefetch of the next level's arc records
+// head merge specialized for 1-4 entries: LSE only (measured: hard mode is faster with the generic loop)
+#ifndef INSTA_SX_HEADN
+#define INSTA_SX_HEADN 2
+#endif
+template <bool kLSE>
+__device__ __forceinline__ constexpr bool sx_headn() { return INSTA_SX_HEADN == 1 || (INSTA_SX_HEADN == 2 && kLSE); }
+struct XCand {
+  double A0, A1, mu, var;     // corners of the s0 / non-unate second candidate; the pair's winner
+};
+constexpr size_t kXOff = (kFStageBytes + 127) & ~size_t(127);
+constexpr size_t kXStageBytes = kXOff + sizeof(XCand) * 2 * kXCap + kXCap;
+
+// L2 prefetch of a byte range (TMA bulk prefetch; 16-byte aligned, size a multiple of 16)
+__device__ __forceinline__ void prefetch_l2(const void* p, uint32_t bytes) {
+  if (bytes) asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
+}
+
+// the arc records of entries [xa, xb) (the next level's slice): off the dependency chain
+__device__ __forceinline__ void sx_prefetch_rec(const SLParams& P, int xa, int xb) {
+  if (xb <= xa) return;
+  prefetch_l2(P.ext_ms + xa, uint32_t(xb - xa) * 16u);
+  prefetch_l2(P.ext_fms + xa, uint32_t(xb - xa) * 16u);
+}
+
+template <bool kFlow>
+__device__ __forceinline__ void sx_await(const SLParams& P, int j, Raw& r) {
+  if (!kFlow) return;
+  uint32_t n = 0;
+  while (!raw_ready(r, P.par)) {
+    if (++n > (1u << 26)) __trap();   // bounded: never a silent hang
+    r = ld_raw(P.state + j);
+  }
+}
+
+// entry x (slot of the slice): folded pin, candidates of both transitions
+template <bool kLSE>
+__device__ __forceinline__ void sx_entry(const SLParams& P, int x, int32_t w, int32_t f, const float4& ms,
+                                         const float4& fms, Raw r, XCand* xc, uint8_t* xs) {
+  if ((w >> kFoldBit) & 1) r = sl_fold<kLSE>(P, f, fms, x, r);
+  const Gath st = unpack(r);
+  const int u = int(uint32_t(w) >> kUnateShift);
+  const double ns = double(P.n_sigma);
+  uint32_t sb = 0u;
+#pragma unroll
+  for (int rf = 0; rf < 2; ++rf) {
+    const Cand c0 = make_cand(st, ms, rf, src_tr(rf, u, 0), ns);
+    XCand o;
+    o.A0 = c0.A;
+    o.A1 = c0.A;
+    o.mu = c0.mu;
+    o.var = c0.var;
+    if (u == 2) {
+      const Cand c1 = make_cand(st, ms, rf, rf ^ 1, ns);
+      o.A1 = c1.A;
+      if (c1.A > c0.A) {   // strict: s = rf wins ties (merge_rf order)
+        o.mu = c1.mu;
+        o.var = c1.var;
+        sb |= 1u << rf;
+      }
+    }
+    xc[rf] = o;
+  }
+  *xs = uint8_t(sb);
+}
+
+// head h with exactly NF entries (compile-time: every slot load is issued before
+// the scan; heads of a slice are ordered by shape, fold.cpp, so a warp's heads
+// take the same case).  The same operations in the same order as sx_head.
+template <bool kLSE, int NF>
+__device__ __forceinline__ void sx_head_n(const SLParams& P, int h, int x0, int pin, const int32_t* w,
+                                          const XCand* xc, const uint8_t* xs) {
+  const double ns = double(P.n_sigma);
+  XCand c[NF][2];
+  uint32_t sb[NF];
+  int u[NF];
+#pragma unroll
+  for (int k = 0; k < NF; ++k) {
+    sb[k] = xs[k];
+    u[k] = int(uint32_t(w[k]) >> kUnateShift);
+    c[k][0] = xc[2 * k];
+    c[k][1] = xc[2 * k + 1];
+  }
+  double mu[2], var[2], best[2];
+  float sum[2];
+  int win[2];
+#pragma unroll
+  for (int rf = 0; rf < 2; ++rf) {
+    double b = ((sb[0] >> rf) & 1u) ? c[0][rf].A1 : c[0][rf].A0;
+    int bk = 0;
+    double bm = c[0][rf].mu, bv = c[0][rf].var;
+#pragma unroll
+    for (int k = 1; k < NF; ++k) {
+      const double A = ((sb[k] >> rf) & 1u) ? c[k][rf].A1 : c[k][rf].A0;
+      if (A > b) {   // Alg 2 l.4: replace only if strictly greater
+        b = A;
+        bk = k;
+        bm = c[k][rf].mu;
+        bv = c[k][rf].var;
+      }
+    }
+    int uw = u[0];
+    uint32_t sbw = sb[0];
+#pragma unroll
+    for (int k = 1; k < NF; ++k)
+      if (bk == k) {
+        uw = u[k];
+        sbw = sb[k];
+      }
+    const int sw = ((sbw >> rf) & 1u) ? (rf ^ 1) : src_tr(rf, uw, 0);
+    mu[rf] = bm;
+    var[rf] = bv;
+    best[rf] = b;
+    win[rf] = bk | (sw << 15);
+    sum[rf] = 0.f;
+    if (kLSE) {
+      float s = 0.f;
+#pragma unroll
+      for (int k = 0; k < NF; ++k) {
+        s += lse_w(c[k][rf].A0, b, P.inv_tau);
+        if (u[k] == 2) s += lse_w(c[k][rf].A1, b, P.inv_tau);
+      }
+      sum[rf] = s;
+      mu[rf] = lse_arrival(b, double(P.tau), s) - ns * double(sigma_of(bv));
+    }
+  }
+  st_state(P.state + pin, mu[0], mu[1], var[0], var[1], P.par);
+  if (!kLSE) {
+    P.hwin[h] = win[0] | (win[1] << 16);
+  } else {
+    const float inv0 = 1.f / sum[0], inv1 = 1.f / sum[1];
+#pragma unroll
+    for (int k = 0; k < NF; ++k) {
+      float wt[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
+#pragma unroll
+      for (int rf = 0; rf < 2; ++rf) {
+        const float inv = rf ? inv1 : inv0;
+        wt[rf][src_tr(rf, u[k], 0)] = lse_w(c[k][rf].A0, best[rf], P.inv_tau) * inv;
+        if (u[k] == 2) wt[rf][rf ^ 1] = lse_w(c[k][rf].A1, best[rf], P.inv_tau) * inv;
+      }
+      P.ew[x0 + k] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
+    }
+  }
+}
+
+// head h with entries [x0, x0 + nf): words w[k], slots xc[2k + rf], pair bits xs[k]
+template <bool kLSE>
+__device__ __forceinline__ void sx_head(const SLParams& P, int h, int x0, int nf, int pin, const int32_t* w,
+                                        const XCand* xc, const uint8_t* xs) {
+  const double ns = double(P.n_sigma);
+  double mu[2], var[2], best[2];
+  float sum[2];
+  int win[2];
+#pragma unroll
+  for (int rf = 0; rf < 2; ++rf) {
+    double b = 0.0;
+    int bk = 0;
+    for (int k = 0; k < nf; ++k) {
+      const XCand& c = xc[2 * k + rf];
+      const double A = ((xs[k] >> rf) & 1u) ? c.A1 : c.A0;
+      if (k == 0 || A > b) {   // Alg 2 l.4: replace only if strictly greater
+        b = A;
+        bk = k;
+      }
+    }
+    const XCand& cw = xc[2 * bk + rf];
+    const int uw = int(uint32_t(w[bk]) >> kUnateShift);
+    const int sw = ((xs[bk] >> rf) & 1u) ? (rf ^ 1) : src_tr(rf, uw, 0);
+    mu[rf] = cw.mu;
+    var[rf] = cw.var;
+    best[rf] = b;
+    win[rf] = bk | (sw << 15);
+    sum[rf] = 0.f;
+    if (kLSE) {   // Eq 4 over the candidates in merge order; reading R1 for sigma
+      float s = 0.f;
+      for (int k = 0; k < nf; ++k) {
+        s += lse_w(xc[2 * k + rf].A0, b, P.inv_tau);
+        if ((uint32_t(w[k]) >> kUnateShift) == 2u) s += lse_w(xc[2 * k + rf].A1, b, P.inv_tau);
+      }
+      sum[rf] = s;
+      mu[rf] = lse_arrival(b, double(P.tau), s) - ns * double(sigma_of(cw.var));
+    }
+  }
+  st_state(P.state + pin, mu[0], mu[1], var[0], var[1], P.par);
+  if (!kLSE) {
+    P.hwin[h] = win[0] | (win[1] << 16);
+  } else {
+    const float inv0 = 1.f / sum[0], inv1 = 1.f / sum[1];
+    for (int k = 0; k < nf; ++k) {   // Eq 6 weights (arc_weights)
+      const int u = int(uint32_t(w[k]) >> kUnateShift);
+      float wt[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
+#pragma unroll
+      for (int rf = 0; rf < 2; ++rf) {
+        const float inv = rf ? inv1 : inv0;
+        wt[rf][src_tr(rf, u, 0)] = lse_w(xc[2 * k + rf].A0, best[rf], P.inv_tau) * inv;
+        if (u == 2) wt[rf][rf ^ 1] = lse_w(xc[2 * k + rf].A1, best[rf], P.inv_tau) * inv;
+      }
+      P.ew[x0 + k] = make_float4(wt[0][0], wt[0][1], wt[1][0], wt[1][1]);
+    }
+  }
+}
+
+// one level of fwdx_kernel: (1) entry phase, CTA barrier, (2) head phase.  xc / xs are indexed by entry
+// id (shared memory, or the CTA's global buffer for a slice beyond kXCap entries).
+template <bool kLSE, bool kFlow>
+__device__ __forceinline__ void sx_level(const SLParams& P, int a, int b, int xa, int xb, const int32_t* Pt,
+                                         const int32_t* Pn, const int32_t* Wx, const int32_t* Fx, XCand* xc,
+                                         uint8_t* xs, unsigned long long* ph) {
+  const int tid = threadIdx.x, nt = blockDim.x;
+  // (1) entries: two per thread in flight (loads of both issued before either is used)
+  for (int x = xa + tid; x < xb; x += 2 * nt) {
+    const int y = x + nt;
+    const bool two = y < xb;
+    const int32_t w0 = Wx[x], w1 = two ? Wx[y] : 0;
+    const float4 m0 = P.ext_ms[x];
+    const float4 m1 = two ? P.ext_ms[y] : make_float4(0.f, 0.f, 0.f, 0.f);
+    const bool f0 = (w0 >> kFoldBit) & 1, f1 = two && ((w1 >> kFoldBit) & 1);
+    const int32_t g0 = f0 ? Fx[x] : 0, g1 = f1 ? Fx[y] : 0;
+    const float4 n0 = f0 ? P.ext_fms[x] : m0;
+    const float4 n1 = f1 ? P.ext_fms[y] : m1;
+    Raw r0 = ld_raw(P.state + (w0 & kSrcMask));
+    Raw r1;
+    if (two) r1 = ld_raw(P.state + (w1 & kSrcMask));
+    sx_await<kFlow>(P, w0 & kSrcMask, r0);
+#ifdef INSTA_SL_PHASES
+    if (ph && x == xa) ph[4] = gtimer() + ((r0.a | __float_as_uint(m0.x)) & 0ull);
+#endif
+    sx_entry<kLSE>(P, x, w0, g0, m0, n0, r0, xc + 2 * x, xs + x);
+    if (two) {
+      sx_await<kFlow>(P, w1 & kSrcMask, r1);
+      sx_entry<kLSE>(P, y, w1, g1, m1, n1, r1, xc + 2 * y, xs + y);
+    }
+  }
+  __syncthreads();
+#ifdef INSTA_SL_PHASES
+  if (ph) ph[6] = gtimer();   // debug: every entry of the CTA's slice done
+#endif
+  // (2) heads
+  for (int h = a + tid; h < b; h += nt) {
+    const int x0 = Pt[h], nf = Pt[h + 1] - x0;
+    switch (sx_headn<kLSE>() ? nf : 0) {
+      case 1: sx_head_n<kLSE, 1>(P, h, x0, Pn[h], Wx + x0, xc + 2 * x0, xs + x0); break;
+      case 2: sx_head_n<kLSE, 2>(P, h, x0, Pn[h], Wx + x0, xc + 2 * x0, xs + x0); break;
+      case 3: sx_head_n<kLSE, 3>(P, h, x0, Pn[h], Wx + x0, xc + 2 * x0, xs + x0); break;
+      case 4: sx_head_n<kLSE, 4>(P, h, x0, Pn[h], Wx + x0, xc + 2 * x0, xs + x0); break;
+      default: sx_head<kLSE>(P, h, x0, nf, Pn[h], Wx + x0, xc + 2 * x0, xs + x0); break;
+    }
+  }
+}
+
+template <bool kLSE, bool kFlow>
+__global__ void __launch_bounds__(sx_threads(kLSE), 1) fwdx_kernel(SLParams P) {
+  extern __shared__ __align__(128) unsigned char sl_smem[];
+  const int gt = blockIdx.x * blockDim.x + threadIdx.x;
+  const int nthr = gridDim.x * blockDim.x;
+  const int tid = threadIdx.x;
+  const int L = P.num_sl;
+  FStageSet* S = reinterpret_cast<FStageSet*>(sl_smem);
+  int4* s_slc = reinterpret_cast<int4*>(sl_smem + kFSlcOff);
+  XCand* xc_s = reinterpret_cast<XCand*>(sl_smem + kXOff);
+  uint8_t* xs_s = reinterpret_cast<uint8_t*>(xc_s + 2 * kXCap);
+  XCand* xc_g = P.xscr ? reinterpret_cast<XCand*>(P.xscr) + size_t(blockIdx.x) * 2 * P.xscr_cap : nullptr;
+  uint8_t* xs_g = P.xscr ? reinterpret_cast<uint8_t*>(reinterpret_cast<XCand*>(P.xscr) + size_t(gridDim.x) * 2 *
+                                                      P.xscr_cap) + size_t(blockIdx.x) * P.xscr_cap
+                         : nullptr;
+  uint32_t nbar = 0;
+  load_slices(P, s_slc);
+  __syncthreads();
+  if (tid == 0) {
+    mbar_init(&S->full[0]);
+    mbar_init(&S->full[1]);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    if (L > 1) {
+      const int4 c = slice_of(P, s_slc, 1);
+      fwd_issue(P, S, 1, c.x, c.y, c.z, c.w);
+      sx_prefetch_rec(P, c.z, c.w);
+    }
+  }
+  for (int s = gt; s < L; s += nthr) P.sl_cnt[s] = 0u;   // a full pass supersedes pending flags
+  // startpoints: clock arrival distribution, mean and variance per rf
+  for (int i = gt; i < P.num_src; i += nthr) {
+    const float4 v = __ldg(P.src_ms + i);
+    st_state(P.state + i, double(v.x), double(v.y), double(v.z) * double(v.z), double(v.w) * double(v.w), P.par);
+  }
+  uint32_t phase[2] = {0u, 0u};
+  unsigned long long* ph = nullptr;
+  for (int s = 1; s < L; ++s) {
+    const int bf = s & 1;
+    __syncthreads();   // level s - 1 is done with buffer bf ^ 1 and the candidate slots
+#ifdef INSTA_SL_PHASES
+    if (ph) ph[5] = gtimer();   // debug: the CTA finished level s - 1
+#endif
+    if (tid == 0 && s + 1 < L) {
+      const int4 c = slice_of(P, s_slc, s + 1);
+      fwd_issue(P, S, bf ^ 1, c.x, c.y, c.z, c.w);
+      if (kSXPrefetch) sx_prefetch_rec(P, c.z, c.w);
+    }
+    if (!kFlow) grid_sync(P.bar, ++nbar, P.trace);   // levels < s are complete
+#ifdef INSTA_SL_PHASES
+    if (P.trace && tid == 0) {   // debug: per (level, CTA) timestamps
+      ph = P.trace + 512 + size_t(L + 8) * 2 * gridDim.x + (size_t(s) * gridDim.x + blockIdx.x) * 8;
+      ph[0] = gtimer();
+    }
+#endif
+    const int4 sc = slice_of(P, s_slc, s);
+    const int a = sc.x, b = sc.y, xa = sc.z, xb = sc.w;
+    mbar_wait(&S->full[bf], phase[bf]);
+    phase[bf] ^= 1u;
+#ifdef INSTA_SL_PHASES
+    if (ph) ph[2] = gtimer();
+#endif
+    if (b <= a) continue;
+    const bool ok = S->ok[bf] != 0;
+    const Window wp = window(a, b + 1, 4), wh = window(a, b, 4), wx = window(xa, xb, 4);
+    // topology of the slice, indexed by head / entry id: staged, or global
+    const int32_t* Pt = ok ? S->ptr[bf] + wp.off - a : P.hd_ptr;
+    const int32_t* Pn = ok ? S->pin[bf] + wh.off - a : P.hd_pin;
+    const int32_t* Wx = ok ? S->w[bf] + wx.off - xa : P.ext_w;
+    const int32_t* Fx = ok ? S->f[bf] + wx.off - xa : P.ext_f;
+    const bool fit = xb - xa <= kXCap;
+    if (fit) sx_level<kLSE, kFlow>(P, a, b, xa, xb, Pt, Pn, Wx, Fx, xc_s - 2 * ptrdiff_t(xa), xs_s - ptrdiff_t(xa), ph);
+    else sx_level<kLSE, kFlow>(P, a, b, xa, xb, Pt, Pn, Wx, Fx, xc_g - 2 * ptrdiff_t(xa), xs_g - ptrdiff_t(xa), ph);
+  }
+  grid_exit(P.bar);
+}
+
+// --------------------------------------------------------------------------
 // One-cell what-if candidates (insta_eval_candidates; SURVEY §8(f) C5
 // INSTA-Size "estimate the timing of each candidate"), all in ONE persistent
 // launch.  Per candidate i (stamps 2i / 2i + 1 past the graph's epoch):
@@ -1167,6 +1535,10 @@ int query_sl_grid(int device, int* grid_f, int* grid_b) {
   if (e == cudaSuccess) e = sl_smem_attr(fwdl_kernel<true, 1>, kFStageBytes);
   if (e == cudaSuccess) e = sl_smem_attr(fwdl_kernel<false, 2>, kFStageBytes);
   if (e == cudaSuccess) e = sl_smem_attr(fwdl_kernel<true, 2>, kFStageBytes);
+  if (e == cudaSuccess) e = sl_smem_attr(fwdx_kernel<false, false>, kXStageBytes);
+  if (e == cudaSuccess) e = sl_smem_attr(fwdx_kernel<true, false>, kXStageBytes);
+  if (e == cudaSuccess) e = sl_smem_attr(fwdx_kernel<false, true>, kXStageBytes);
+  if (e == cudaSuccess) e = sl_smem_attr(fwdx_kernel<true, true>, kXStageBytes);
   if (e == cudaSuccess) e = sl_smem_attr(eval_kernel<false>, kEvalSmem);
   if (e == cudaSuccess) e = sl_smem_attr(eval_kernel<true>, kEvalSmem);
   if (e == cudaSuccess) e = sl_smem_attr(bwdl_kernel<false>, kBStageBytes);
@@ -1179,6 +1551,13 @@ int query_sl_grid(int device, int* grid_f, int* grid_b) {
   const size_t sf[] = {kFStageBytes, kFStageBytes, kFStageBytes, kFStageBytes, kFStageBytes, kFStageBytes};
   for (int i = 0; i < 6; ++i) {
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kf[i], kSLFwdThreads, sf[i]);
+    if (e != cudaSuccess) return int(e);
+    occ = std::min(occ, b);
+  }
+  const void* kx[] = {(const void*)fwdx_kernel<false, false>, (const void*)fwdx_kernel<true, false>,
+                      (const void*)fwdx_kernel<false, true>, (const void*)fwdx_kernel<true, true>};
+  for (int i = 0; i < 4; ++i) {
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kx[i], sx_threads(i & 1), kXStageBytes);
     if (e != cudaSuccess) return int(e);
     occ = std::min(occ, b);
   }
@@ -1225,7 +1604,7 @@ static int launch_coop(const void* fn, int grid, int threads, size_t smem, SLPar
   return err;
 }
 
-int launch_forward_sl(DevGraph& g, float n_sigma, float tau, void* stream) {
+int launch_forward_sl(DevGraph& g, float n_sigma, float tau, void* stream, bool flow) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   if (g.n == 0) return 0;
   SLParams P = sl_params(g);
@@ -1235,8 +1614,17 @@ int launch_forward_sl(DevGraph& g, float n_sigma, float tau, void* stream) {
   P.par = (++g.pass_fwd) & 1u;
   ++g.inc_epoch;   // a full pass supersedes pending incremental marks
   const bool lse = tau > 0.f;
-  const int err = launch_coop(lse ? (const void*)fwdl_kernel<true, 0> : (const void*)fwdl_kernel<false, 0>, g.sl_grid,
-                              kSLFwdThreads, kFStageBytes, P, st, lse ? "fwd_lse" : "fwd");
+  if (g.sl_max_x > kXCap && !g.xscr) {   // candidate buffers of slices beyond shared memory
+    const cudaError_t e =
+        cudaMalloc(&g.xscr, size_t(g.sl_grid) * size_t(g.sl_max_x) * (2 * sizeof(XCand) + 1));
+    if (e != cudaSuccess) return int(e);
+  }
+  P.xscr = g.sl_max_x > kXCap ? g.xscr : nullptr;
+  P.xscr_cap = g.sl_max_x;
+  // flow: no grid barrier (parity dataflow); needs uniform record parity (no cone pass since the last full pass)
+  const void* fn = flow ? (lse ? (const void*)fwdx_kernel<true, true> : (const void*)fwdx_kernel<false, true>)
+                        : (lse ? (const void*)fwdx_kernel<true, false> : (const void*)fwdx_kernel<false, false>);
+  const int err = launch_coop(fn, g.sl_grid, sx_threads(lse), kXStageBytes, P, st, lse ? "fwd_lse" : "fwd");
   if (!err) g.parity_mixed = false;
   g.folded_valid = false;
   return err;

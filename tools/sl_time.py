@@ -49,6 +49,8 @@ with torch.cuda.stream(st):
                 raw = np.fromfile(p, np.uint64).astype(np.int64)
                 t = raw[:512]
                 t = t[t > 0]
+                if t.size == 0:
+                    continue
                 d = np.diff(t) / 1e3
                 print(name, "total us", (t[-1] - t[0]) / 1e3, "per barrier us:", " ".join(f"{x:.1f}" for x in d))
                 arr = raw[512:]
