@@ -685,6 +685,39 @@ def main():
                 out[f"{frac:g}"] = row
         return out
 
+    # reverse-cone incremental backward: after each cone pass, insta_backward_update
+    # on the kept gradient vs a full insta_backward into another buffer (bit-identical results; CUDA events)
+    def bwd_series(GG, gg, fracs_steps, seed0):
+        out = {}
+        H = GG.schedule()["num_heads"]
+        dk = torch.zeros((gg.num_arcs, 2), dtype=torch.float32, device=dev)
+        df = torch.empty_like(dk)
+        with torch.cuda.stream(stream):
+            GG.forward(3.0, 0.0, 0, stream=stream)
+            GG.backward_update(dk, stream=stream)
+            for frac, nst in fracs_steps:
+                tu, tf, hr, same = [], [], [], True
+                for k in range(nst):
+                    ids, m, sg = (torch.as_tensor(x, device=dev) for x in synth.sizing_step(gg, seed0 + k, frac=frac))
+                    GG.update_arcs(ids, m, sg, incremental=True, stream=stream)
+                    GG.forward(3.0, 0.0, 0, sync=False, stream=stream, cone_max=10 ** 12)
+                    e = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
+                    e[0].record(stream)
+                    inc = GG.backward_update(dk, stream=stream)   # default policy (full past E/5e4 arcs)
+                    e[1].record(stream)
+                    GG.backward(out=df, stream=stream)
+                    e[2].record(stream)
+                    stream.synchronize()
+                    tu.append(e[0].elapsed_time(e[1]))
+                    tf.append(e[1].elapsed_time(e[2]))
+                    hr.append(GG.last_backward_stats() / H if inc else 1.0)
+                    same = same and bool(torch.equal(dk.view(torch.int32), df.view(torch.int32)))
+                out[f"{frac:g}"] = {"arcs_per_step": int(round(frac * gg.num_arcs)) or 1, "steps": nst,
+                                    "update_ms_median": float(np.median(tu[1:])), "full_ms_median": float(np.median(tf[1:])),
+                                    "heads_rerun_frac": float(np.median(hr)), "incremental_steps": int(sum(x < 1.0 for x in hr)),
+                                    "bit_identical": same}
+        return out
+
     incremental = None
     if args.incremental and world == 1:
         big = 10 ** 12
@@ -693,6 +726,11 @@ def main():
                        "what": "per step: insta_update_arcs + insta_forward (CUDA events); incremental = default "
                                "policy (cone pass for <= max(64, E/1e5) updated arcs), full = the same updates "
                                "then a full pass"}
+        incremental["C4_backward_update"] = bwd_series(G, g, [(1e-7, 12), (1e-6, 12), (1e-5, 12), (1e-4, 8)], 8000)
+        incremental["C4_backward_update_what"] = (
+            "per step: a 1-cell .. 1e-4 sizing update + cone forward (untimed), then insta_backward_update on the "
+            "kept TNS gradient (reverse cone; update_ms) vs insta_backward into another buffer (full_ms), CUDA "
+            "events; heads_rerun_frac = work heads whose Eq 6 chain was re-run")
         try:
             g3 = synth.generate("C3")
             G3 = insta.Graph(g3, device=local)

@@ -188,6 +188,33 @@ insta_status insta_arrivals(insta_graph* g, float* A, float* mean, float* sigma,
 insta_status insta_backward(insta_graph* g, const float* ep_seed, float* d_arc_mean,
                             float* d_arc_sigma, float* d_src, void* cuda_stream);
 
+/* The TNS gradient kept current across incremental forwards (SURVEY §8(f)
+ * NEXT 3: the reverse-cone backward of INSTA-Size; incremental
+ * evaluation P:L229).  d_arc_mean: DEVICE float[num_arcs][2], the caller's
+ * gradient buffer, owned by the caller.  The first call -- or any call after a
+ * full forward, a forward with other tau / n_sigma, or with another buffer --
+ * runs the full backward (default TNS seeds, as insta_backward with ep_seed =
+ * NULL; also when more than max(64, num_arcs / 50000) arcs were re-annotated
+ * since the snapshot: the reverse cone then spans every level and the full
+ * backward is faster) and keeps a snapshot of its fixed-point adjoint sums, adjoints, seeds,
+ * arg-max words and Eq 6 weights on the device (16 B + 8 B + 8 B + 4 B per work
+ * head, 4 B (hard) or 32 B (LSE) per entry; allocated on first use).  A later
+ * call after insta_forward cone passes only (insta_update_arcs(incremental=1)
+ * below the cone threshold) re-runs the Eq 6 chain in the reverse cone of what
+ * changed -- heads whose seed, arg-max or weights differ from the snapshot and,
+ * level by level, every head a changed share reaches -- and updates
+ * d_arc_mean in place: the buffer must still hold the previous call's result.
+ * Bit-identical to insta_backward (the adjoints are integer sums of the same
+ * fixed-point shares).  *incremental (HOST, may be NULL) = 1 if the update ran
+ * incrementally, 0 if it ran the full backward.  Needs a schedule 0/3 forward
+ * (INSTA_E_STATE otherwise); no sigma channel or source gradient. */
+insta_status insta_backward_update(insta_graph* g, float* d_arc_mean, void* cuda_stream,
+                                   int32_t* incremental);
+
+/* Work heads whose Eq 6 chain the last incremental insta_backward_update re-ran
+ * (HOST int64 out).  Synchronizes. */
+insta_status insta_last_backward_stats(insta_graph* g, int64_t* heads_rerun);
+
 /* Re-annotate n arcs ("re-annotate ... then re-propagate"):
  * arc_ids DEVICE int32[n] (caller ids, unique) -- or NULL with n == num_arcs
  * to re-annotate every arc in caller order -- mean/sigma DEVICE float[n][2].

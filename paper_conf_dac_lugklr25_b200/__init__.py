@@ -202,6 +202,21 @@ class Graph:
         outs = (d_mean,) + ((d_sig,) if want_sigma else ()) + ((d_src,) if want_src else ())
         return outs if len(outs) > 1 else d_mean
 
+    def backward_update(self, out, stream=None) -> bool:
+        """insta_backward_update: the TNS gradient in `out` (float32[E,2] device tensor holding the
+        previous call's result) brought up to date after incremental forwards, in the reverse cone
+        of the change; the first call (or one after a full forward) runs the full backward.
+        Returns True if the update ran incrementally."""
+        inc = ctypes.c_int32(0)
+        check(self.lib.insta_backward_update(self._h, _dptr(out), self._st(stream), ctypes.byref(inc)),
+              "insta_backward_update")
+        return bool(inc.value)
+
+    def last_backward_stats(self) -> int:
+        v = ctypes.c_int64()
+        check(self.lib.insta_last_backward_stats(self._h, ctypes.byref(v)), "insta_last_backward_stats")
+        return int(v.value)
+
     def update_arcs(self, arc_ids, mean, sigma, incremental: bool = True, stream=None):
         """insta_update_arcs: re-annotate arcs (device or host arrays; copied to the device)."""
         t = self._torch

@@ -69,6 +69,8 @@ SIGNATURES = {
     "insta_backward": (ctypes.c_int, [c_vp, c_vp, c_vp, c_vp, c_vp, c_vp]),
     "insta_update_arcs": (ctypes.c_int, [c_vp, ctypes.c_int64, c_vp, c_vp, c_vp, ctypes.c_int32, c_vp]),
     "insta_last_forward_stats": (ctypes.c_int, [c_vp, c_vp]),
+    "insta_backward_update": (ctypes.c_int, [c_vp, c_vp, c_vp, c_vp]),
+    "insta_last_backward_stats": (ctypes.c_int, [c_vp, c_vp]),
     "insta_forward_batch": (ctypes.c_int, [c_vp, ctypes.c_int32, ctypes.POINTER(insta_scenario), ctypes.c_float,
                                            c_vp, c_vp, c_vp]),
     "insta_eval_candidates": (ctypes.c_int, [c_vp, ctypes.c_int32, c_vp, c_vp, c_vp, c_vp, c_vp, c_vp]),

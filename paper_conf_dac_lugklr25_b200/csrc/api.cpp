@@ -68,7 +68,7 @@ void free_graph(insta::DevGraph& d) {
                   d.cl_rf,     d.cl_summary, d.cl_hv_list, d.cl_hv_of, d.cl_hv_sum, d.tl_partials, d.sz_tmp,
                   d.sl_ptr,    d.ext_sh,    d.hd_csl,    d.chg,       d.acc_h,     d.sl_bar,    d.sl_cnt,
                   d.hwin,      d.ew,        d.fwin,      d.efw,       d.sl_slice,  d.hfo_ptr,   d.hfo,       d.hd_hsrc,
-                  d.cand_old,  d.xscr,  d.ep_blk,    d.cand_ptr_d, d.pl_ptr,    d.pl_ent,    d.pl_arc,    d.pl_wide};
+                  d.cand_old,  d.xscr,  d.acc_b, d.hab_b, d.hseed_b, d.hwin_b, d.fwin_b, d.ew_b, d.efw_b, d.btouch, d.bdirty, d.bl_cnt, d.ep_blk,    d.cand_ptr_d, d.pl_ptr,    d.pl_ent,    d.pl_arc,    d.pl_wide};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   if (d.b_stage_h) cudaFreeHost(d.b_stage_h);
@@ -500,6 +500,7 @@ insta_status insta_forward(insta_graph* g, const insta_opts* o, void* cuda_strea
   }
   if (err) return cuda_fail(err, "forward");
   if (!inc) {
+    d.binc_touch_all = true;   // every head's arg-max / weights may differ from the backward snapshot
     d.sweep_valid = sweep_sched;
     d.canon_valid = !sweep_sched;
   } else if (sweep_sched) {
@@ -573,6 +574,48 @@ insta_status insta_backward(insta_graph* g, const float* ep_seed, float* d_arc_m
   return INSTA_OK;
 }
 
+insta_status insta_backward_update(insta_graph* g, float* d_arc_mean, void* cuda_stream, int32_t* incremental) {
+  if (!g) return fail(INSTA_E_ARG, "backward_update: NULL graph");
+  insta::DevGraph& d = g->d;
+  if (!d_arc_mean && d.e > 0) return fail(INSTA_E_ARG, "backward_update: d_arc_mean is required");
+  if (!d.fwd_valid) return fail(INSTA_E_STATE, "backward_update: no valid forward (call insta_forward)");
+  if (d.bwd_schedule != 0 && d.bwd_schedule != 3)
+    return fail(INSTA_E_STATE, "backward_update: needs a schedule-0/3 forward (the sweep backward's accumulators)");
+  if (double(d.num_ep) >= 0x1p30)
+    return fail(INSTA_E_ARG, "backward_update: too many endpoints for the sweep accumulators");
+  cudaSetDevice(d.device);
+  // incremental only from a snapshot of the same buffer and options, with cone passes only since
+  // and few re-annotated arcs: the reverse cone costs a grid barrier per super-level it spans,
+  // so past ~E/5e4 updated arcs (C4: 426) the full backward is the faster one (bench
+  // incremental.C4_backward_update: 1e-5 of the arcs 0.10 vs 0.37 ms, 1e-4 0.49 vs 0.37 ms)
+  const int64_t upd_max = std::max<int64_t>(64, d.e / 50000);
+  const bool full = !d.binc_valid || d.binc_touch_all || d.binc_dmean != d_arc_mean ||
+                    d.binc_tau != d.last_tau || d.binc_nsig != d.last_n_sigma || d.binc_updates > upd_max;
+  int err = insta::launch_backward_update(d, d_arc_mean, full, cuda_stream);
+  if (err) {
+    d.binc_valid = false;
+    return cuda_fail(err, "backward_update");
+  }
+  d.binc_valid = true;
+  d.binc_touch_all = false;
+  d.binc_updates = 0;
+  d.binc_dmean = d_arc_mean;
+  d.binc_tau = d.last_tau;
+  d.binc_nsig = d.last_n_sigma;
+  if (incremental) *incremental = full ? 0 : 1;
+  return INSTA_OK;
+}
+
+insta_status insta_last_backward_stats(insta_graph* g, int64_t* heads_rerun) {
+  if (!g || !heads_rerun) return fail(INSTA_E_ARG, "last_backward_stats: NULL argument");
+  insta::DevGraph& d = g->d;
+  unsigned long long v = 0;
+  const cudaError_t e = cudaMemcpy(&v, d.counters + 2, sizeof v, cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) return cuda_fail(int(e), "last_backward_stats");
+  *heads_rerun = int64_t(v);
+  return INSTA_OK;
+}
+
 insta_status insta_update_arcs(insta_graph* g, int64_t n, const int32_t* arc_ids,
                                const float* mean, const float* sigma, int32_t incremental,
                                void* cuda_stream) {
@@ -590,6 +633,7 @@ insta_status insta_update_arcs(insta_graph* g, int64_t n, const int32_t* arc_ids
   if (incremental && !d.pending_full) d.pending_incremental = true;
   else d.pending_full = true;
   d.pending_updates += n;
+  d.binc_updates += n;
   return INSTA_OK;
 }
 

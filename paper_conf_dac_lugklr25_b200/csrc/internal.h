@@ -217,6 +217,27 @@ struct DevGraph {
   int32_t* sl_ptr = nullptr;       // [SL+1]
   int4* sl_slice = nullptr;        // [SL][sl_grid] per-CTA slices {a, b, xa, xb} of every super-level
   int32_t sl_max_x = 0;            // most entries in one slice (fwdx_kernel: candidate buffer size)
+  // incremental backward (insta_backward_update, sweep.cu bwdi_kernel): the state of the last
+  // snapshot backward -- per head its accumulated fixed-point sum and adjoint, its seed and
+  // arg-max word; per entry the folded arg-max / Eq 6 weights -- and the heads touched since
+  long long* acc_b = nullptr;      // [H][2]
+  float2* hab_b = nullptr;         // [H]
+  float2* hseed_b = nullptr;       // [H]
+  int32_t* hwin_b = nullptr;       // [H]
+  int32_t* fwin_b = nullptr;       // [X]
+  float4* ew_b = nullptr;          // [X] (LSE)
+  float4* efw_b = nullptr;         // [X] (LSE)
+  uint32_t* btouch = nullptr;      // [H] == bepoch: recomputed by a cone pass since the snapshot
+  uint32_t* bdirty = nullptr;      // [H] == bstamp: re-run the head's Eq 6 chain
+  uint32_t* bl_cnt = nullptr;      // [SL] levels holding a dirty head
+  uint32_t bepoch = 1, bstamp = 0;
+  bool binc_valid = false;         // the snapshot describes the last update's gradient
+  bool binc_touch_all = true;      // a full forward since the snapshot (every head may differ)
+  float binc_tau = 0.f, binc_nsig = 0.f;
+  float* binc_dmean = nullptr;     // the caller's gradient buffer the snapshot belongs to
+  int64_t binc_heads = 0;          // heads re-run by the last update (stats)
+  bool bsnap_req = false;          // the next sweep backward writes the snapshot
+  int64_t binc_updates = 0;        // arcs re-annotated since the snapshot
   void* xscr = nullptr;            // fwdx_kernel: per-CTA candidate buffers for slices beyond shared memory
   int32_t* ext_sh = nullptr;       // [X] source head of each entry
   int32_t* hd_csl = nullptr;       // [H] consumer super-level range of each head
@@ -351,12 +372,14 @@ int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float*
 int launch_gather_arcs(DevGraph& g, int n, const int32_t* ids, float* mean, float* sigma, void* stream);
 // sum |ep_seed| on the device (synchronizes)
 int seed_abs_sum(DevGraph& g, const float* seed, double* host_out, void* stream);
+int launch_seeds(DevGraph& g, void* stream);   // TNS endpoint seeds (hseed) from the current slacks
 int launch_update_arcs(DevGraph& g, int64_t n, const int32_t* ids, const float* mean,
                        const float* sigma, int incremental, void* stream);
 int launch_arrivals(DevGraph& g, float* A, float* mean, float* sigma, void* stream);
 // sweep.cu: level-synchronous thread-per-head passes (schedule 0)
 int query_sl_grid(int device, int* grid_fwd, int* grid_bwd);
 int launch_forward_sl(DevGraph& g, float n_sigma, float tau, void* stream, bool flow = false);
+int launch_backward_update(DevGraph& g, float* d_arc_mean, bool snapshot_only, void* stream);
 int launch_forward_cone(DevGraph& g, float n_sigma, float tau, void* stream);
 int launch_eval_candidates(DevGraph& g, int num, const int32_t* cand_ptr, const int32_t* arc_ids, const float* mean,
                            const float* sigma, double* out, void* stream);

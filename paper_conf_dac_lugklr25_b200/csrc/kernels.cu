@@ -1859,6 +1859,15 @@ int launch_forward(DevGraph& g, float n_sigma, float tau, int schedule, void* st
   return launch_slack(g, stream);
 }
 
+int launch_seeds(DevGraph& g, void* stream) {
+  if (g.num_ep == 0) return 0;
+  PrepParams Z{};
+  const int blocks = int(std::min<size_t>((size_t(g.num_ep) + 255) / 256, size_t(g.grid > 0 ? g.grid : 148) * 8));
+  bwd_prep_kernel<<<blocks, 256, 0, static_cast<cudaStream_t>(stream)>>>(g.num_ep, g.ep_pin, g.ep_head, g.slack,
+                                                                         g.rf_star, nullptr, g.seed, g.hseed, Z);
+  return int(cudaGetLastError());
+}
+
 int launch_backward(DevGraph& g, const float* ep_seed, float* d_arc_mean, float* d_arc_sigma, float* d_src,
                     void* stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);

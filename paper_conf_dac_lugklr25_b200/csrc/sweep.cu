@@ -143,6 +143,19 @@ struct SLParams {
   // for slices with more than kXCap entries ([grid][xscr_cap] XCand pairs, then bytes)
   void* xscr;
   int32_t xscr_cap;
+  // incremental backward (bwdi_kernel) and the snapshot written by a full backward
+  long long* acc_b;
+  float2* hab_b;
+  float2* hseed_b;
+  int32_t* hwin_b;
+  int32_t* fwin_b;
+  float4* ew_b;
+  float4* efw_b;
+  uint32_t* btouch;   // cone passes stamp the heads they recompute (== bepoch)
+  uint32_t bepoch;
+  uint32_t* bdirty;
+  uint32_t* bl_cnt;
+  uint32_t bstamp;
 };
 
 // --------------------------------------------------------------------------
@@ -161,7 +174,7 @@ __device__ __forceinline__ void grid_sync_ctr(uint32_t* bar, uint32_t target, un
     for (;;) {
       asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(bar) : "memory");
       if (v >= target) break;
-      if (++npoll > (1u << 26)) __trap();   // bounded: never a silent hang
+      if (++npoll > (1u << 23)) __trap();   // bounded: never a silent hang
     }
 #endif
     if (trace && blockIdx.x == 0) trace[target / gridDim.x] = gtimer();
@@ -461,6 +474,7 @@ __device__ __forceinline__ int sl_fwd_head(const SLParams& P, int h, const HeadT
     default: npins = sl_fwd_wide<kLSE>(P, t, R, F); break;
   }
   if (!kLSE) P.hwin[h] = R.win | (F.win << 16);
+  if (kInc && P.btouch) P.btouch[h] = P.bepoch;   // its arg-max / weights may differ from the backward snapshot
   if (kInc) {
     if (rec_changed(old, R.mu, F.mu, R.var, F.var)) {
       st_state(P.state + t.pin, R.mu, F.mu, R.var, F.var, P.par);
@@ -782,7 +796,7 @@ __device__ __forceinline__ void sx_await(const SLParams& P, int j, Raw& r) {
   if (!kFlow) return;
   uint32_t n = 0;
   while (!raw_ready(r, P.par)) {
-    if (++n > (1u << 26)) __trap();   // bounded: never a silent hang
+    if (++n > (1u << 23)) __trap();   // bounded: never a silent hang
     r = ld_raw(P.state + j);
   }
 }
@@ -1329,6 +1343,10 @@ __device__ __forceinline__ void sl_bwd_head(const SLParams& P, SLHeavyTab* tab, 
   if (ax | ay) asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %1};" ::"l"(P.acc + 2 * size_t(h)), "l"(0ull));
   const float2 ab = make_float2(sd.x + float(double((long long)ax) * kAccInv),
                                 sd.y + float(double((long long)ay) * kAccInv));
+  if (P.acc_b) {   // snapshot for insta_backward_update
+    asm volatile("st.global.v2.u64 [%0], {%1, %2};" ::"l"(P.acc_b + 2 * size_t(h)), "l"(ax), "l"(ay) : "memory");
+    P.hab_b[h] = ab;
+  }
   // nothing flows through this head: its arcs keep the zero prefill (scattered zero stores in
   // caller arc order cost 2.5x the whole backward on B200: measured, profiles/r02_summary.md)
   if (ab.x == 0.f && ab.y == 0.f) return;
@@ -1438,10 +1456,210 @@ __global__ void __launch_bounds__(kSLBwdThreads, 1) bwdl_kernel(SLParams P) {
     ld2_u64(P.acc + 2 * size_t(h), ax, ay);
     if (ax | ay) asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %1};" ::"l"(P.acc + 2 * size_t(h)), "l"(0ull));
     const float2 sd = P.hseed[h];
+    if (P.acc_b) {
+      asm volatile("st.global.v2.u64 [%0], {%1, %2};" ::"l"(P.acc_b + 2 * size_t(h)), "l"(ax), "l"(ay) : "memory");
+      P.hab_b[h] = make_float2(sd.x + float(double((long long)ax) * kAccInv), sd.y + float(double((long long)ay) * kAccInv));
+    }
     if (P.d_src)
       reinterpret_cast<float2*>(P.d_src)[__ldg(P.order + h)] =
           make_float2(sd.x + float(double((long long)ax) * kAccInv), sd.y + float(double((long long)ay) * kAccInv));
   }
+  grid_exit(P.bar);
+}
+
+// --------------------------------------------------------------------------
+// Incremental backward (insta_backward_update; SURVEY §8(f) NEXT 3
+// INSTA-Size, P:L229 incremental evaluation).
+//
+// The sweep backward accumulates every head's adjoint as an integer sum of
+// fixed-point shares (push_adj), so a later backward can be reached exactly by
+// deltas: a snapshot backward keeps, per head, its accumulated sum (acc_b), its
+// adjoint (hab_b), seed and arg-max word, and per entry the folded arg-max /
+// Eq 6 weights.  After cone passes (which stamp the heads they recompute), the
+// update (1) recomputes the endpoint seeds, (2) marks every touched head whose
+// seed, arg-max or weights differ from the snapshot, then (3) walks the flagged
+// super-levels in reverse: a marked head adds the deltas pushed to it to its
+// sum, forms its adjoint exactly as the full backward does, rewrites dL/d(mean)
+// of its arcs, and pushes fix(new share) - fix(old share) to each source --
+// marking the source when that difference is nonzero.  Integer addition is
+// exact and order-free, so every sum, adjoint and gradient equals the full
+// backward's bit for bit; the work is the reverse cone of the change, cut off
+// where the shares stop changing.
+// --------------------------------------------------------------------------
+__device__ __forceinline__ long long fixp(float v) { return __double2ll_rn(double(v) * kAccScale); }
+
+// sl_sink with the store of dL/d(mean) optional and unconditional (zeros included)
+template <bool kLSE>
+__device__ __forceinline__ float2 bi_sink(const SLParams& P, float2 ab, int sel, float4 w4, int32_t arcid, bool store) {
+  const float abr[2] = {ab.x, ab.y};
+  float w[2][2];
+  if (kLSE) {
+    w[0][0] = w4.x;
+    w[0][1] = w4.y;
+    w[1][0] = w4.z;
+    w[1][1] = w4.w;
+  } else {
+#pragma unroll
+    for (int rf = 0; rf < 2; ++rf) {
+      w[rf][0] = ((sel >> (2 * rf)) & 1) ? 1.f : 0.f;
+      w[rf][1] = ((sel >> (2 * rf + 1)) & 1) ? 1.f : 0.f;
+    }
+  }
+  float gm[2], gs[2] = {0.f, 0.f};
+#pragma unroll
+  for (int rf = 0; rf < 2; ++rf) {
+    const float a0 = w[rf][0] * abr[rf], a1 = w[rf][1] * abr[rf];
+    gm[rf] = a0 + a1;
+    gs[0] += a0;
+    gs[1] += a1;
+  }
+  // the full backward stores a nonzero pair as is and leaves the zero prefill otherwise
+  if (store)
+    reinterpret_cast<float2*>(P.d_mean)[arcid] =
+        (gm[0] != 0.f || gm[1] != 0.f) ? make_float2(gm[0], gm[1]) : make_float2(0.f, 0.f);
+  return make_float2(gs[0], gs[1]);
+}
+
+__device__ __forceinline__ void bi_mark(const SLParams& P, const int32_t* s_slp, int h) {
+  P.bdirty[h] = P.bstamp;
+  atomicOr(P.bl_cnt + sl_of(P, s_slp, h), 1u);
+}
+
+// (2) heads recomputed since the snapshot whose seed, arg-max or weights differ
+template <bool kLSE>
+__global__ void __launch_bounds__(256) bdiff_kernel(SLParams P) {
+  __shared__ int32_t s_slp[kSliceCap + 4];
+  for (int v = threadIdx.x; v <= min(P.num_sl, kSliceCap); v += blockDim.x) s_slp[v] = __ldg(P.sl_ptr + v);
+  __syncthreads();
+  for (int h = blockIdx.x * blockDim.x + threadIdx.x; h < P.num_heads; h += gridDim.x * blockDim.x) {
+    if (__ldcg(P.btouch + h) != P.bepoch) continue;
+    const float2 a = P.hseed[h], b = P.hseed_b[h];
+    bool chg = __float_as_uint(a.x) != __float_as_uint(b.x) || __float_as_uint(a.y) != __float_as_uint(b.y);
+    if (!kLSE) chg |= __ldcg(P.hwin + h) != P.hwin_b[h];
+    const int x0 = __ldg(P.hd_ptr + h), x1 = __ldg(P.hd_ptr + h + 1);
+    for (int x = x0; x < x1 && !chg; ++x) {
+      if (kLSE) {
+        const float4 u = __ldcg(P.ew + x), v = P.ew_b[x];
+        chg |= __float_as_uint(u.x) != __float_as_uint(v.x) || __float_as_uint(u.y) != __float_as_uint(v.y) ||
+               __float_as_uint(u.z) != __float_as_uint(v.z) || __float_as_uint(u.w) != __float_as_uint(v.w);
+      }
+      if (__ldg(P.ext_farc + x) >= 0 && (uint32_t(__ldg(P.ext_f + x)) >> kUnateShift) == 2u) {   // non-unate folded arc
+        if (kLSE) {
+          const float4 u = __ldcg(P.efw + x), v = P.efw_b[x];
+          chg |= __float_as_uint(u.x) != __float_as_uint(v.x) || __float_as_uint(u.y) != __float_as_uint(v.y) ||
+                 __float_as_uint(u.z) != __float_as_uint(v.z) || __float_as_uint(u.w) != __float_as_uint(v.w);
+        } else {
+          chg |= __ldcg(P.fwin + x) != P.fwin_b[x];
+        }
+      }
+    }
+    if (chg) bi_mark(P, s_slp, h);
+  }
+}
+
+// (3) one marked head: its adjoint from the snapshot sum plus the pushed deltas,
+// its arcs' gradients, and the share deltas to its sources; the snapshot follows
+template <bool kLSE>
+__device__ __forceinline__ int bi_head(const SLParams& P, const int32_t* s_slp, int h) {
+  unsigned long long dx, dy;
+  ld2_u64(P.acc + 2 * size_t(h), dx, dy);
+  if (dx | dy) asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %1};" ::"l"(P.acc + 2 * size_t(h)), "l"(0ull));
+  const long long tx = P.acc_b[2 * size_t(h)] + (long long)dx, ty = P.acc_b[2 * size_t(h) + 1] + (long long)dy;
+  P.acc_b[2 * size_t(h)] = tx;
+  P.acc_b[2 * size_t(h) + 1] = ty;
+  const float2 sd = P.hseed[h];
+  const float2 ab = make_float2(sd.x + float(double(tx) * kAccInv), sd.y + float(double(ty) * kAccInv));
+  const float2 ao = P.hab_b[h];
+  P.hab_b[h] = ab;
+  P.hseed_b[h] = sd;
+  if (h < P.num_src) return 0;   // a startpoint: no arcs
+  int32_t wn = 0, wo = 0;
+  if (!kLSE) {
+    wn = __ldcg(P.hwin + h);
+    wo = P.hwin_b[h];
+    P.hwin_b[h] = wn;
+  }
+  const int x0 = __ldg(P.hd_ptr + h), nf = __ldg(P.hd_ptr + h + 1) - x0;
+  for (int k = 0; k < nf; ++k) {
+    const int x = x0 + k;
+    const int32_t arc = __ldg(P.ext_arc + x), farc = __ldg(P.ext_farc + x), sh = __ldg(P.ext_sh + x);
+    float4 w4n = make_float4(0.f, 0.f, 0.f, 0.f), w4o = w4n;
+    if (kLSE) {
+      w4n = __ldcg(P.ew + x);
+      w4o = P.ew_b[x];
+      P.ew_b[x] = w4n;
+    }
+    float2 gn = bi_sink<kLSE>(P, ab, kLSE ? 0 : sel_of(wn, k), w4n, arc, true);
+    float2 go = bi_sink<kLSE>(P, ao, kLSE ? 0 : sel_of(wo, k), w4o, arc, false);
+    if (farc >= 0) {   // through the folded pin (as sl_bwd_head)
+      const int u2 = int(uint32_t(__ldg(P.ext_f + x)) >> kUnateShift);
+      int fsn = 0, fso = 0;
+      float4 fwn = make_float4(0.f, 0.f, 0.f, 0.f), fwo = fwn;
+      if (u2 != 2) {
+        if (kLSE) fwn = fwo = unate_w(u2);
+        else fsn = fso = unate_sel(u2);
+      } else if (kLSE) {
+        fwn = __ldcg(P.efw + x);
+        fwo = P.efw_b[x];
+        P.efw_b[x] = fwn;
+      } else {
+        const int32_t a = __ldcg(P.fwin + x), b = P.fwin_b[x];
+        P.fwin_b[x] = a;
+        fsn = sel_of(a, 0);
+        fso = sel_of(b, 0);
+      }
+      gn = bi_sink<kLSE>(P, gn, fsn, fwn, farc, true);
+      go = bi_sink<kLSE>(P, go, fso, fwo, farc, false);
+    }
+    const long long ddx = fixp(gn.x) - fixp(go.x), ddy = fixp(gn.y) - fixp(go.y);
+    if (ddx | ddy) {
+      unsigned long long* a = reinterpret_cast<unsigned long long*>(P.acc) + 2 * size_t(sh);
+      red_u64(a, (unsigned long long)ddx);
+      red_u64(a + 1, (unsigned long long)ddy);
+      if (__ldcg(P.bdirty + sh) != P.bstamp) bi_mark(P, s_slp, sh);
+    }
+  }
+  return 1;
+}
+
+template <bool kLSE>
+__global__ void __launch_bounds__(kSLBwdThreads, 1) bwdi_kernel(SLParams P) {
+  __shared__ int4 s_slc[kSliceCap];
+  __shared__ int32_t s_slp[kSliceCap + 4];
+  __shared__ int32_t s_next;
+  const int tid = threadIdx.x, L = P.num_sl;
+  uint32_t nbar = 0, nrun = 0;
+  load_slices(P, s_slc);
+  for (int v = tid; v <= min(P.num_sl, kSliceCap); v += blockDim.x) s_slp[v] = __ldg(P.sl_ptr + v);
+  __syncthreads();
+  int s = L;   // levels >= s are done
+  for (;;) {
+    // next flagged level below s: every flag there is final (set by levels >= s, before the last barrier)
+    if (tid < 32) {
+      int nx = -1;
+      for (int top = s - 1; top >= 0; top -= 32) {
+        const int lv = top - tid;
+        const uint32_t f = lv >= 0 ? __ldcg(P.bl_cnt + lv) : 0u;
+        const uint32_t hit = __ballot_sync(0xffffffffu, f != 0u);
+        if (hit) {
+          nx = top - (__ffs(hit) - 1);
+          break;
+        }
+      }
+      if (tid == 0) s_next = nx;
+    }
+    __syncthreads();
+    s = s_next;
+    __syncthreads();
+    if (s < 0) break;
+    const int4 sc = slice_of(P, s_slc, s);
+    for (int h = sc.x + tid; h < sc.y; h += blockDim.x)
+      if (__ldcg(P.bdirty + h) == P.bstamp) nrun += uint32_t(bi_head<kLSE>(P, s_slp, h));
+    grid_sync(P.bar, ++nbar, P.trace);   // level s is complete: its pushes and marks are visible
+  }
+  for (int v = blockIdx.x * blockDim.x + tid; v < L; v += gridDim.x * blockDim.x) P.bl_cnt[v] = 0u;
+  const uint32_t n = __reduce_add_sync(0xffffffffu, nrun);
+  if ((tid & 31) == 0 && n) atomicAdd(P.counters + 2, (unsigned long long)n);
   grid_exit(P.bar);
 }
 
@@ -1516,6 +1734,8 @@ static SLParams sl_params(DevGraph& g) {
   P.fin_ms = g.fin_ms;
   P.ext_ms_w = g.ext_ms;
   P.ext_fms_w = g.ext_fms;
+  P.btouch = g.btouch;   // cone passes stamp the heads they recompute (incremental backward)
+  P.bepoch = g.bepoch;
   return P;
 }
 
@@ -1710,9 +1930,80 @@ int launch_backward_sl(DevGraph& g, float* d_arc_mean, float* d_src, void* strea
   SLParams P = sl_params(g);
   P.d_mean = d_arc_mean;
   P.d_src = d_src;
+  if (g.bsnap_req) {   // snapshot for insta_backward_update
+    P.acc_b = g.acc_b;
+    P.hab_b = g.hab_b;
+  }
   const bool lse = g.last_tau > 0.f;
   return launch_coop(lse ? (const void*)bwdl_kernel<true> : (const void*)bwdl_kernel<false>, g.sl_grid_b,
                      kSLBwdThreads, kBStageBytes, P, st, lse ? "bwd_lse" : "bwd");
+}
+
+// insta_backward_update: a snapshot backward (full sweep backward + snapshot), or the
+// incremental update from the snapshot (seeds, diff of the touched heads, reverse cone)
+int launch_backward_update(DevGraph& g, float* d_arc_mean, bool full, void* stream) {
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (g.n == 0) return 0;
+  const bool lse = g.last_tau > 0.f;
+  const size_t H = size_t(std::max(g.num_heads, 1)), X = size_t(std::max<int64_t>(g.num_ext, 1));
+  cudaError_t e = cudaSuccess;
+  if (!g.acc_b) {   // snapshot arrays, allocated on first use
+    e = cudaMalloc(&g.acc_b, sizeof(long long) * 2 * H);
+    if (e == cudaSuccess) e = cudaMalloc(&g.hab_b, sizeof(float2) * H);
+    if (e == cudaSuccess) e = cudaMalloc(&g.hseed_b, sizeof(float2) * H);
+    if (e == cudaSuccess) e = cudaMalloc(&g.hwin_b, sizeof(int32_t) * H);
+    if (e == cudaSuccess) e = cudaMalloc(&g.fwin_b, sizeof(int32_t) * X);
+    if (e == cudaSuccess) e = cudaMalloc(&g.ew_b, sizeof(float4) * X);
+    if (e == cudaSuccess) e = cudaMalloc(&g.efw_b, sizeof(float4) * X);
+    if (e == cudaSuccess) e = cudaMalloc(&g.btouch, sizeof(uint32_t) * H);
+    if (e == cudaSuccess) e = cudaMalloc(&g.bdirty, sizeof(uint32_t) * H);
+    if (e == cudaSuccess) e = cudaMalloc(&g.bl_cnt, sizeof(uint32_t) * size_t(std::max(g.num_slevels, 1)));
+    if (e == cudaSuccess) e = cudaMemsetAsync(g.btouch, 0, sizeof(uint32_t) * H, st);
+    if (e == cudaSuccess) e = cudaMemsetAsync(g.bdirty, 0, sizeof(uint32_t) * H, st);
+    if (e == cudaSuccess) e = cudaMemsetAsync(g.bl_cnt, 0, sizeof(uint32_t) * size_t(std::max(g.num_slevels, 1)), st);
+    if (e != cudaSuccess) return int(e);
+  }
+  SLParams P = sl_params(g);
+  P.d_mean = d_arc_mean;
+  P.acc_b = g.acc_b;
+  P.hab_b = g.hab_b;
+  P.hseed_b = g.hseed_b;
+  P.hwin_b = g.hwin_b;
+  P.fwin_b = g.fwin_b;
+  P.ew_b = g.ew_b;
+  P.efw_b = g.efw_b;
+  P.btouch = g.btouch;
+  P.bepoch = g.bepoch;
+  P.bdirty = g.bdirty;
+  P.bl_cnt = g.bl_cnt;
+  P.bstamp = ++g.bstamp;
+  if (full) {   // the full backward (seeds, zero fills, sweep) writing acc_b / hab_b, then weights and seeds
+    g.bsnap_req = true;
+    int err = launch_backward(g, nullptr, d_arc_mean, nullptr, nullptr, stream);
+    g.bsnap_req = false;
+    if (err) return err;
+    e = cudaMemcpyAsync(g.hseed_b, g.hseed, sizeof(float2) * H, cudaMemcpyDeviceToDevice, st);
+    if (e == cudaSuccess && !lse) e = cudaMemcpyAsync(g.hwin_b, g.hwin, sizeof(int32_t) * H, cudaMemcpyDeviceToDevice, st);
+    if (e == cudaSuccess && !lse) e = cudaMemcpyAsync(g.fwin_b, g.fwin, sizeof(int32_t) * X, cudaMemcpyDeviceToDevice, st);
+    if (e == cudaSuccess && lse) e = cudaMemcpyAsync(g.ew_b, g.ew, sizeof(float4) * X, cudaMemcpyDeviceToDevice, st);
+    if (e == cudaSuccess && lse) e = cudaMemcpyAsync(g.efw_b, g.efw, sizeof(float4) * X, cudaMemcpyDeviceToDevice, st);
+    g.binc_heads = g.num_heads;
+  } else {
+    e = cudaMemsetAsync(g.counters + 2, 0, sizeof(unsigned long long), st);
+    if (e != cudaSuccess) return int(e);
+    int err = launch_seeds(g, stream);   // endpoint seeds from the current slacks (TNS)
+    if (err) return err;
+    const int blocks = int(std::min<size_t>((H + 255) / 256, size_t(std::max(g.sl_grid, 1)) * 8));
+    if (lse) bdiff_kernel<true><<<blocks, 256, 0, st>>>(P);
+    else bdiff_kernel<false><<<blocks, 256, 0, st>>>(P);
+    err = int(cudaGetLastError());
+    if (err) return err;
+    err = launch_coop(lse ? (const void*)bwdi_kernel<true> : (const void*)bwdi_kernel<false>, g.sl_grid_b,
+                      kSLBwdThreads, 0, P, st, "bwdi");
+    if (err) return err;
+  }
+  ++g.bepoch;   // heads touched from now on differ from this snapshot
+  return int(e);
 }
 
 int launch_fold_fill(DevGraph& g, void* stream) {

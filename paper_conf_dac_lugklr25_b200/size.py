@@ -11,7 +11,8 @@ it (`library_options`).
 
 Host orchestration only: every timing step runs in libinsta.so through the C
 ABI -- insta_forward (incremental cone pass after insta_update_arcs),
-insta_backward, insta_stage_gradients, insta_select_stages.
+insta_backward_update (the reverse-cone incremental backward), insta_stage_gradients,
+insta_select_stages.
 """
 from __future__ import annotations
 
@@ -95,8 +96,11 @@ def insta_size(G, g, iterations: int = 2, per_iter: int = 25, threshold: float =
     s = G.forward(n_sigma, tau)
     tns0 = tns = s.tns
     history, trials, commits = [], 0, 0
+    d = G._torch.zeros((g.num_arcs, 2), dtype=G._torch.float32, device=G.device)
     for it in range(iterations):
-        d = G.backward()
+        # the TNS gradient, kept current by the reverse-cone backward after the previous
+        # iteration's cone passes (insta_backward_update; bit-identical to insta_backward)
+        G.backward_update(d)
         sg = G.stage_gradients(d)
         order = G.select_stages(sg, threshold).cpu().numpy()
         blocked = set()
