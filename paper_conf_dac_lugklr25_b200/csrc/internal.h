@@ -300,6 +300,8 @@ struct DevGraph {
   std::vector<int32_t> cl_hv_ptr;  // [L+1]
   // insta_eval_candidates: previous records of a candidate's arcs
   float* cand_old = nullptr;       // [cand_cap][4] {mean R, F, sigma R, F}
+  void* elog = nullptr;            // eval_kernel undo log: changed head records / arg-max words (hard mode)
+  int32_t elog_cap = 0;
   int32_t cand_cap = 0;
   // INSTA-Size selection scratch (size.cu)
   void* sz_tmp = nullptr;

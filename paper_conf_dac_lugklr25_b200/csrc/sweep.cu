@@ -156,6 +156,17 @@ struct SLParams {
   uint32_t* bdirty;
   uint32_t* bl_cnt;
   uint32_t bstamp;
+  // eval_kernel undo log (hard mode): a cone pass records what it overwrites
+  struct EvLog* elog;        // [elog_cap] head entries
+  int2* flog;                // [elog_cap] {entry, old arg-max word} of non-unate folded pins
+  uint32_t* elog_n;          // [2] entry counts of this candidate
+  int32_t elog_cap;
+};
+
+// one undo record: a recomputed head's previous record and arg-max word
+struct EvLog {
+  Raw rec;
+  int32_t pin, h, win, pad;
 };
 
 // --------------------------------------------------------------------------
@@ -307,8 +318,18 @@ __device__ __forceinline__ Raw sl_fold(const SLParams& P, int32_t f, const float
     else P.wts[__ldg(P.ext_fq + x)] = m.wt;
   }
   if (u2 == 2) {
-    if (!kLSE) P.fwin[x] = m.win;
-    else P.efw[x] = m.wt;
+    if (!kLSE) {
+      if (P.elog) {   // eval_kernel: record the word this cone pass overwrites
+        const int32_t o = P.fwin[x];
+        if (o != m.win) {
+          const uint32_t k = atomicAdd(P.elog_n + 1, 1u);
+          if (k < uint32_t(P.elog_cap)) P.flog[k] = make_int2(x, o);
+        }
+      }
+      P.fwin[x] = m.win;
+    } else {
+      P.efw[x] = m.wt;
+    }
   }
   return m.stored(P.par);
 }
@@ -473,7 +494,25 @@ __device__ __forceinline__ int sl_fwd_head(const SLParams& P, int h, const HeadT
     case 4: npins = sl_fwd_core<kLSE, 4>(P, t, E, R, F, ph); break;
     default: npins = sl_fwd_wide<kLSE>(P, t, R, F); break;
   }
-  if (!kLSE) P.hwin[h] = R.win | (F.win << 16);
+  if (!kLSE) {
+    const int32_t nw = R.win | (F.win << 16);
+    if (kInc && P.elog) {   // eval_kernel: record what this cone pass overwrites (undo log)
+      const int32_t ow = P.hwin[h];
+      if (ow != nw || rec_changed(old, R.mu, F.mu, R.var, F.var)) {
+        const uint32_t k = atomicAdd(P.elog_n, 1u);
+        if (k < uint32_t(P.elog_cap)) {
+          EvLog e;
+          e.rec = old;
+          e.pin = t.pin;
+          e.h = h;
+          e.win = ow;
+          e.pad = 0;
+          P.elog[k] = e;
+        }
+      }
+    }
+    P.hwin[h] = nw;
+  }
   if (kInc && P.btouch) P.btouch[h] = P.bepoch;   // its arg-max / weights may differ from the backward snapshot
   if (kInc) {
     if (rec_changed(old, R.mu, F.mu, R.var, F.var)) {
@@ -1167,6 +1206,7 @@ __global__ void __launch_bounds__(kSLFwdThreads, 1) eval_kernel(SLParams P) {
     grid_sync(P.bar, ++nbar, P.trace);                                          // A done
     for (int w = gt; w < nw; w += nthr) P.ep_blk[w] = 0u;                      // read in D, G of i - 1
     for (int k = tid; k < 2 * kMarkWords; k += blockDim.x) cs.mark[k] = cs.pub[k] = 0u;
+    if (P.elog && gt < 2) P.elog_n[gt] = 0u;                                    // read in E of i - 1
     eval_apply<kLSE>(P, i, false, P.stamp + 2 * i);
     grid_sync(P.bar, ++nbar, P.trace);                                          // B done
     cone_levels<kLSE>(P, P.stamp + 2 * i, cs, s_slc, s_slp, nbar, nrec);
@@ -1177,9 +1217,27 @@ __global__ void __launch_bounds__(kSLFwdThreads, 1) eval_kernel(SLParams P) {
     if (blockIdx.x == 0) slack_final(P.slack_nb, P.partials, P.cand_out + 3 * size_t(i), sr);
     for (int k = tid; k < 2 * kMarkWords; k += blockDim.x) cs.mark[k] = cs.pub[k] = 0u;
     eval_apply<kLSE>(P, i, true, P.stamp + 2 * i + 1);
-    grid_sync(P.bar, ++nbar, P.trace);                                          // E done
-    cone_levels<kLSE>(P, P.stamp + 2 * i + 1, cs, s_slc, s_slp, nbar, nrec);
-    grid_sync(P.bar, ++nbar, P.trace);                                          // F done
+    const uint32_t n0 = P.elog ? __ldcg(P.elog_n) : 0u, n1 = P.elog ? __ldcg(P.elog_n + 1) : 0u;
+    if (P.elog && n0 <= uint32_t(P.elog_cap) && n1 <= uint32_t(P.elog_cap)) {
+      // undo log: every record and arg-max word the cone pass overwrote, written back (each head /
+      // entry appears once: a cone pass recomputes a head at most once)
+      for (uint32_t k = gt; k < n0; k += nthr) {
+        const EvLog e = P.elog[k];
+        asm volatile("st.relaxed.gpu.global.v4.b64 [%0], {%1, %2, %3, %4};" ::"l"(P.state + e.pin), "l"(e.rec.a),
+                     "l"(e.rec.b), "l"(e.rec.c), "l"(e.rec.d)
+                     : "memory");
+        P.hwin[e.h] = e.win;
+      }
+      for (uint32_t k = gt; k < n1; k += nthr) {
+        const int2 f = P.flog[k];
+        P.fwin[f.x] = f.y;
+      }
+      grid_sync(P.bar, ++nbar, P.trace);                                        // E, F done
+    } else {   // no log (LSE) or it overflowed: the cone pass again reverts every record
+      grid_sync(P.bar, ++nbar, P.trace);                                        // E done
+      cone_levels<kLSE>(P, P.stamp + 2 * i + 1, cs, s_slc, s_slp, nbar, nrec);
+      grid_sync(P.bar, ++nbar, P.trace);                                        // F done
+    }
     for (int s = gt; s < L; s += nthr) P.sl_cnt[s] = 0u;
     eval_slack_blocks(P, sr);
     if (i + 1 < P.num_cand) eval_save(P, i + 1);
@@ -1917,6 +1975,18 @@ int launch_eval_candidates(DevGraph& g, int num, const int32_t* cand_ptr, const 
   P.cand_old = reinterpret_cast<float4*>(g.cand_old);
   P.cand_out = out;
   P.num_cand = num;
+  if (!(g.last_tau > 0.f)) {   // hard mode: undo log instead of a second cone pass per candidate
+    if (!g.elog) {
+      const int cap = std::max(1024, std::min(g.num_heads, 1 << 20));
+      e = cudaMalloc(&g.elog, sizeof(EvLog) * size_t(cap) + sizeof(int2) * size_t(cap) + 16);
+      if (e != cudaSuccess) return int(e);
+      g.elog_cap = cap;
+    }
+    P.elog = reinterpret_cast<EvLog*>(g.elog);
+    P.flog = reinterpret_cast<int2*>(P.elog + g.elog_cap);
+    P.elog_n = reinterpret_cast<uint32_t*>(P.flog + g.elog_cap);
+    P.elog_cap = g.elog_cap;
+  }
   const bool lse = g.last_tau > 0.f;
   const int err = launch_coop(lse ? (const void*)eval_kernel<true> : (const void*)eval_kernel<false>, g.sl_grid,
                               kSLFwdThreads, kEvalSmem, P, st, "eval");
