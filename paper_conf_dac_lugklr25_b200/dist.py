@@ -1,9 +1,12 @@
 """Scenario sharding across GPUs: one process per GPU.
 
 A single graph does not shard (serial level dependency), so the
-multi-GPU path is independent scenarios: rank r evaluates a contiguous block of
-the scenario list on its own replica of the graph, OCV scenarios with the TNS
-gradient and sizing candidates forward-only.  The only exchange happens once,
+multi-GPU path is independent scenarios: rank r evaluates, on its own replica
+of the graph, a contiguous block of the gradient (OCV) scenarios and a
+contiguous block of the forward-only (sizing-candidate) scenarios -- the two
+classes are split separately, so every rank gets the same mix (an OCV scenario
+with its backward costs ~15x a one-cell candidate on the cone pass; one block
+of the whole list would put all OCV work on the first half of the ranks).  The only exchange happens once,
 at the end: an all_gather of the per-scenario summaries {wns, tns, #viol} and
 an all_reduce(SUM) of the gradient sum over scenarios.  With the nccl backend
 these run over NVLink; the host logic is backend-agnostic (gloo tests).
@@ -27,10 +30,12 @@ def evaluate_sharded(evaluate, scenarios, n_grad: int, num_arcs: int, rank: int,
     `device`), identical on every rank."""
     import torch
     n = len(scenarios)
-    lo, hi, per = scenario_block(n, rank, world)
-    mine = list(range(lo, hi))
-    g_idx = [s for s in mine if s < n_grad]
-    f_idx = [s for s in mine if s >= n_grad]
+    n_f = n - n_grad
+    glo, ghi, gper = scenario_block(n_grad, rank, world)
+    flo, fhi, fper = scenario_block(n_f, rank, world)
+    g_idx = list(range(glo, ghi))
+    f_idx = [n_grad + s for s in range(flo, fhi)]
+    per = gper + fper
     summ = torch.zeros((per, 3), dtype=torch.float64, device=device)
     grad = torch.zeros((num_arcs, 2), dtype=torch.float32, device=device)
     if g_idx:
@@ -42,13 +47,18 @@ def evaluate_sharded(evaluate, scenarios, n_grad: int, num_arcs: int, rank: int,
     work = dist.all_reduce(grad, op=dist.ReduceOp.SUM, async_op=True) if world > 1 else None
     if f_idx:
         s_f, _ = evaluate([scenarios[s] for s in f_idx], False)
-        summ[len(g_idx): len(g_idx) + len(f_idx)] = s_f
+        summ[gper: gper + len(f_idx)] = s_f
     if world > 1:
         parts = [torch.empty_like(summ) for _ in range(world)]
         dist.all_gather(parts, summ)
-        allsum = torch.cat(parts)
+        out = torch.empty((n, 3), dtype=torch.float64, device=device)
+        for r, part in enumerate(parts):   # back to scenario order
+            a, b, _ = scenario_block(n_grad, r, world)
+            c, d, _ = scenario_block(n_f, r, world)
+            out[a:b] = part[: b - a]
+            out[n_grad + c: n_grad + d] = part[gper: gper + d - c]
         work.wait()
-        summ = allsum[:n]
+        summ = out
     else:
-        summ = summ[:n]
+        summ = torch.cat([summ[: len(g_idx)], summ[gper: gper + len(f_idx)]])
     return summ, grad

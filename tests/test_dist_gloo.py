@@ -51,7 +51,7 @@ def _worker(rank, world, port, out):
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     g = synth.generate("C1")
-    scs = synth.c5_scenarios(g, n=10, n_ocv=5)
+    scs = synth.c5_scenarios(g, n=11, n_ocv=5)
     summ, grad = idist.evaluate_sharded(oracle_eval(g), scs, 5, g.num_arcs, rank, world, "cpu", dist)
     if rank == 0:
         np.save(out + "_summ.npy", summ.numpy())
@@ -73,7 +73,7 @@ def test_scenario_blocks_cover_exactly_once():
 
 def test_sharded_equals_unsharded(tmp_path):
     g = synth.generate("C1")
-    scs = synth.c5_scenarios(g, n=10, n_ocv=5)
+    scs = synth.c5_scenarios(g, n=11, n_ocv=5)   # 5 OCV + 6 sizing: uneven blocks in both classes
     ref_summ, ref_grad = idist.evaluate_sharded(oracle_eval(g), scs, 5, g.num_arcs, 0, 1, "cpu")
     out = str(tmp_path / "r")
     port = 29500 + (os.getpid() % 1000)
@@ -84,3 +84,12 @@ def test_sharded_equals_unsharded(tmp_path):
     assert np.allclose(grad, ref_grad.numpy(), rtol=1e-6, atol=1e-6)
     # OCV scenarios carry gradients, sizing candidates do not: the sum must be nonzero
     assert np.abs(grad).sum() > 0
+
+
+def test_each_rank_gets_both_classes():
+    # 1024 scenarios, 512 OCV: every rank of 2/4/8 evaluates 512/N of each class
+    for w in (2, 4, 8):
+        for r in range(w):
+            a, b, _ = idist.scenario_block(512, r, w)
+            c, d, _ = idist.scenario_block(512, r, w)
+            assert b - a == 512 // w and d - c == 512 // w
