@@ -68,7 +68,7 @@ void free_graph(insta::DevGraph& d) {
                   d.cl_rf,     d.cl_summary, d.cl_hv_list, d.cl_hv_of, d.cl_hv_sum, d.tl_partials, d.sz_tmp,
                   d.sl_ptr,    d.ext_sh,    d.hd_csl,    d.chg,       d.acc_h,     d.sl_bar,    d.sl_cnt,
                   d.hwin,      d.ew,        d.fwin,      d.efw,       d.sl_slice,  d.hfo_ptr,   d.hfo,       d.hd_hsrc,
-                  d.cand_old,  d.elog,  d.hcnt,  d.bcnt,  d.xscr,  d.acc_b, d.hab_b, d.hseed_b, d.hwin_b, d.fwin_b, d.ew_b, d.efw_b, d.btouch, d.bdirty, d.bl_cnt, d.ep_blk,    d.cand_ptr_d, d.pl_ptr,    d.pl_ent,    d.pl_arc,    d.pl_wide};
+                  d.cand_old,  d.elog,  d.xscr,  d.acc_b, d.hab_b, d.hseed_b, d.hwin_b, d.fwin_b, d.ew_b, d.efw_b, d.btouch, d.bdirty, d.bl_cnt, d.ep_blk,    d.cand_ptr_d, d.pl_ptr,    d.pl_ent,    d.pl_arc,    d.pl_wide};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   if (d.b_stage_h) cudaFreeHost(d.b_stage_h);
@@ -342,12 +342,6 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
     UP(d.sl_slice, slc.data(), slc.size());
   }
   UP(d.ext_sh, fold.ext_sh.data(), fold.ext_sh.size());
-  {   // dataflow backward: every head waits for one share per entry it is the source of
-    std::vector<int32_t> hc(fold.hd_pin.size(), 0);
-    for (const int32_t v : fold.ext_sh) ++hc[size_t(v)];
-    UP(d.hcnt, hc.data(), hc.size());
-    ZERO(d.bcnt, fold.hd_pin.size());
-  }
   UP(d.hd_csl, fold.hd_csl.data(), fold.hd_csl.size());
   UP(d.hfo_ptr, fold.hfo_ptr.data(), fold.hfo_ptr.size());
   UP(d.hfo, fold.hfo.data(), fold.hfo.size());

@@ -240,8 +240,6 @@ struct DevGraph {
   int64_t binc_updates = 0;        // arcs re-annotated since the snapshot
   void* xscr = nullptr;            // fwdx_kernel: per-CTA candidate buffers for slices beyond shared memory
   int32_t* ext_sh = nullptr;       // [X] source head of each entry
-  int32_t* hcnt = nullptr;         // [H] entries whose source is the head (dataflow backward: shares to wait for)
-  uint32_t* bcnt = nullptr;        // [H] shares arrived in this pass (zero between passes)
   int32_t* hd_csl = nullptr;       // [H] consumer super-level range of each head
   int32_t* hfo_ptr = nullptr;      // [H+1] consumer heads of each head
   int32_t* hfo = nullptr;

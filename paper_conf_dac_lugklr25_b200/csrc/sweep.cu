@@ -157,8 +157,6 @@ struct SLParams {
   uint32_t* bl_cnt;
   uint32_t bstamp;
   // eval_kernel undo log (hard mode): a cone pass records what it overwrites
-  const int32_t* __restrict__ hcnt;   // dataflow backward: shares each head waits for
-  uint32_t* bcnt;                     // shares arrived (zero between passes)
   struct EvLog* elog;        // [elog_cap] head entries
   int2* flog;                // [elog_cap] {entry, old arg-max word} of non-unate folded pins
   uint32_t* elog_n;          // [2] entry counts of this candidate
@@ -1256,18 +1254,14 @@ constexpr int kSLHeavyTab = 256;
 struct SLHeavyTab {
   int32_t key[kSLHeavyTab];
   unsigned long long acc[kSLHeavyTab][2];
-  uint32_t n[kSLHeavyTab];   // dataflow backward: shares combined in the slot
 };
 
 __device__ __forceinline__ void red_u64(unsigned long long* a, unsigned long long v) {
   asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(a), "l"(v));
 }
 
-// kFlow: returns true if the share went into the CTA table (its arrival is counted by the
-// flush), false if the caller counts it (after a fence) -- a zero share is counted too
-template <bool kFlow = false>
-__device__ __forceinline__ bool push_adj(const SLParams& P, SLHeavyTab* tab, int sh, bool heavy, float gx, float gy) {
-  if (!kFlow && gx == 0.f && gy == 0.f) return false;
+__device__ __forceinline__ void push_adj(const SLParams& P, SLHeavyTab* tab, int sh, bool heavy, float gx, float gy) {
+  if (gx == 0.f && gy == 0.f) return;
   const unsigned long long vx = (unsigned long long)__double2ll_rn(double(gx) * kAccScale);
   const unsigned long long vy = (unsigned long long)__double2ll_rn(double(gy) * kAccScale);
   if (heavy) {   // a driver with > kHeavyFanout sinks: combine in shared memory first
@@ -1275,55 +1269,28 @@ __device__ __forceinline__ bool push_adj(const SLParams& P, SLHeavyTab* tab, int
     for (int probe = 0; probe < 8; ++probe, hh = (hh + 1) & (kSLHeavyTab - 1)) {
       const int prev = atomicCAS(&tab->key[hh], -1, sh);
       if (prev == -1 || prev == sh) {
-        if (vx | vy) {
-          atomicAdd(&tab->acc[hh][0], vx);
-          atomicAdd(&tab->acc[hh][1], vy);
-        }
-        if (kFlow) atomicAdd(&tab->n[hh], 1u);
-        return true;
+        atomicAdd(&tab->acc[hh][0], vx);
+        atomicAdd(&tab->acc[hh][1], vy);
+        return;
       }
     }
   }
-  if (vx | vy) {
-    unsigned long long* a = reinterpret_cast<unsigned long long*>(P.acc) + 2 * size_t(sh);
-    red_u64(a, vx);
-    red_u64(a + 1, vy);
-  }
-  return false;
+  unsigned long long* a = reinterpret_cast<unsigned long long*>(P.acc) + 2 * size_t(sh);
+  red_u64(a, vx);
+  red_u64(a + 1, vy);
 }
 
-__device__ __forceinline__ void red_u32(uint32_t* a, uint32_t v) {
-  asm volatile("red.relaxed.gpu.global.add.u32 [%0], %1;" ::"l"(a), "r"(v) : "memory");
-}
-
-template <bool kFlow = false>
 __device__ __forceinline__ void heavy_flush(const SLParams& P, SLHeavyTab* tab) {
   for (int k = threadIdx.x; k < kSLHeavyTab; k += blockDim.x) {
     const int sh = tab->key[k];
     if (sh >= 0) {
       unsigned long long* a = reinterpret_cast<unsigned long long*>(P.acc) + 2 * size_t(sh);
-      if (tab->acc[k][0]) red_u64(a, tab->acc[k][0]);
-      if (tab->acc[k][1]) red_u64(a + 1, tab->acc[k][1]);
-      if (kFlow) {   // the arrivals after the shares (release order)
-        __threadfence();
-        red_u32(P.bcnt + sh, tab->n[k]);
-        tab->n[k] = 0u;
-      }
+      red_u64(a, tab->acc[k][0]);
+      red_u64(a + 1, tab->acc[k][1]);
       tab->key[k] = -1;
       tab->acc[k][0] = 0ull;
       tab->acc[k][1] = 0ull;
     }
-  }
-}
-
-// dataflow backward: wait until every share to head h has arrived (bounded)
-__device__ __forceinline__ void await_shares(const SLParams& P, int h) {
-  const uint32_t want = uint32_t(__ldg(P.hcnt + h));
-  uint32_t n = 0, v;
-  for (;;) {
-    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(P.bcnt + h) : "memory");
-    if (v >= want) break;
-    if (++n > (1u << 23)) __trap();   // bounded: never a silent hang
   }
 }
 
@@ -1426,14 +1393,12 @@ __device__ __forceinline__ void bwd_issue(const SLParams& P, BStageSet* S, int b
 // cleared), then the Eq 6 sink side of every entry (through the folded pin
 // when there is one) and the share pushed to the entry's source head.
 // T: the staged slice (entry words at xr + k, weights at xw + k) or nullptr (global).
-template <bool kLSE, bool kFlow = false>
+template <bool kLSE>
 __device__ __forceinline__ void sl_bwd_head(const SLParams& P, SLHeavyTab* tab, int h, int x0, int nf, float2 sd,
                                             int32_t win, const BStage* T, int xr, int xw) {
-  if (kFlow) await_shares(P, h);
   unsigned long long ax, ay;
   ld2_u64(P.acc + 2 * size_t(h), ax, ay);
   if (ax | ay) asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %1};" ::"l"(P.acc + 2 * size_t(h)), "l"(0ull));
-  if (kFlow && __ldg(P.hcnt + h)) P.bcnt[h] = 0u;   // every share has arrived: ready for the next pass
   const float2 ab = make_float2(sd.x + float(double((long long)ax) * kAccInv),
                                 sd.y + float(double((long long)ay) * kAccInv));
   if (P.acc_b) {   // snapshot for insta_backward_update
@@ -1441,19 +1406,8 @@ __device__ __forceinline__ void sl_bwd_head(const SLParams& P, SLHeavyTab* tab, 
     P.hab_b[h] = ab;
   }
   // nothing flows through this head: its arcs keep the zero prefill (scattered zero stores in
-  // caller arc order cost 2.5x the whole backward on B200: measured, profiles/r02_summary.md);
-  // the dataflow pass still counts one (zero) share per entry
-  uint32_t direct = 0u;   // kFlow: entries whose share the caller counts
-  if (ab.x == 0.f && ab.y == 0.f) {
-    if (kFlow) {
-      for (int k = 0; k < nf; ++k) {
-        const int32_t sh = T ? T->sh[xr + k] : __ldg(P.ext_sh + x0 + k);
-        const int32_t bw = T ? T->bw[xr + k] : __ldg(P.ext_bw + x0 + k);
-        if (!push_adj<true>(P, tab, sh, (bw >> kHeavyBit) & 1, 0.f, 0.f)) red_u32(P.bcnt + sh, 1u);
-      }
-    }
-    return;
-  }
+  // caller arc order cost 2.5x the whole backward on B200: measured, profiles/r02_summary.md)
+  if (ab.x == 0.f && ab.y == 0.f) return;
   for (int k = 0; k < nf; ++k) {
     const int x = x0 + k;
     int32_t arc, farc, sh, bw, f;
@@ -1488,24 +1442,11 @@ __device__ __forceinline__ void sl_bwd_head(const SLParams& P, SLHeavyTab* tab, 
       }
       gs = sl_sink<kLSE>(P, gs, fsel, fw, farc);
     }
-    const bool tabled = push_adj<kFlow>(P, tab, sh, (bw >> kHeavyBit) & 1, gs.x, gs.y);
-    if (kFlow && !tabled) {
-      if (k < 32) {
-        direct |= 1u << k;
-      } else {   // (wide heads only) counted at once
-        __threadfence();
-        red_u32(P.bcnt + sh, 1u);
-      }
-    }
-  }
-  if (kFlow && direct) {   // the arrivals, after this head's shares are visible (one fence per head)
-    __threadfence();
-    for (int k = 0; k < min(nf, 32); ++k)
-      if ((direct >> k) & 1u) red_u32(P.bcnt + (T ? T->sh[xr + k] : __ldg(P.ext_sh + x0 + k)), 1u);
+    push_adj(P, tab, sh, (bw >> kHeavyBit) & 1, gs.x, gs.y);
   }
 }
 
-template <bool kLSE, bool kFlow = false>
+template <bool kLSE>
 __global__ void __launch_bounds__(kSLBwdThreads, 1) bwdl_kernel(SLParams P) {
   extern __shared__ __align__(128) unsigned char sl_smem[];
   BStageSet* S = reinterpret_cast<BStageSet*>(sl_smem);
@@ -1515,7 +1456,6 @@ __global__ void __launch_bounds__(kSLBwdThreads, 1) bwdl_kernel(SLParams P) {
     tab.key[k] = -1;
     tab.acc[k][0] = 0ull;
     tab.acc[k][1] = 0ull;
-    tab.n[k] = 0u;
   }
   const int L = P.num_sl;
   uint32_t nbar = 0;
@@ -1540,7 +1480,7 @@ __global__ void __launch_bounds__(kSLBwdThreads, 1) bwdl_kernel(SLParams P) {
       const int4 c = slice_of(P, s_slc, s - 1);
       bwd_issue<kLSE>(P, S, bf ^ 1, c.x, c.y, c.z, c.w);
     }
-    if (!kFlow && s < L - 1) grid_sync(P.bar, ++nbar, P.trace);   // levels > s are complete
+    if (s < L - 1) grid_sync(P.bar, ++nbar, P.trace);   // levels > s are complete
     mbar_wait(&S->full[bf], phase[bf]);
     phase[bf] ^= 1u;
     const int4 sc = slice_of(P, s_slc, s);
@@ -1555,25 +1495,21 @@ __global__ void __launch_bounds__(kSLBwdThreads, 1) bwdl_kernel(SLParams P) {
           const int r = h - a;
           const int x0 = T.ptr[wp.off + r], nf = T.ptr[wp.off + r + 1] - x0;
           const int32_t win = kLSE ? 0 : T.win[wh.off + r];
-          sl_bwd_head<kLSE, kFlow>(P, &tab, h, x0, nf, T.seed[ws.off + r], win, &T, wx.off + x0 - xa, x0 - xa);
+          sl_bwd_head<kLSE>(P, &tab, h, x0, nf, T.seed[ws.off + r], win, &T, wx.off + x0 - xa, x0 - xa);
         }
       } else {
         for (int h = a + tid; h < b; h += blockDim.x) {
           const int x0 = __ldg(P.hd_ptr + h), nf = __ldg(P.hd_ptr + h + 1) - x0;
-          sl_bwd_head<kLSE, kFlow>(P, &tab, h, x0, nf, P.hseed[h], kLSE ? 0 : __ldcg(P.hwin + h), nullptr, 0, 0);
+          sl_bwd_head<kLSE>(P, &tab, h, x0, nf, P.hseed[h], kLSE ? 0 : __ldcg(P.hwin + h), nullptr, 0, 0);
         }
       }
     }
     __syncthreads();
-    heavy_flush<kFlow>(P, &tab);
+    heavy_flush(P, &tab);
   }
   // level 0 (startpoints, hd_pin[h] = h): dL/d(source mean)
-  if (!kFlow && L > 1) grid_sync(P.bar, ++nbar, P.trace);
+  if (L > 1) grid_sync(P.bar, ++nbar, P.trace);
   for (int h = blockIdx.x * blockDim.x + tid; h < P.num_src; h += gridDim.x * blockDim.x) {
-    if (kFlow) {
-      await_shares(P, h);
-      if (__ldg(P.hcnt + h)) P.bcnt[h] = 0u;
-    }
     unsigned long long ax, ay;
     ld2_u64(P.acc + 2 * size_t(h), ax, ay);
     if (ax | ay) asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %1};" ::"l"(P.acc + 2 * size_t(h)), "l"(0ull));
@@ -1856,8 +1792,6 @@ static SLParams sl_params(DevGraph& g) {
   P.fin_ms = g.fin_ms;
   P.ext_ms_w = g.ext_ms;
   P.ext_fms_w = g.ext_fms;
-  P.hcnt = g.hcnt;
-  P.bcnt = g.bcnt;
   P.btouch = g.btouch;   // cone passes stamp the heads they recompute (incremental backward)
   P.bepoch = g.bepoch;
   return P;
@@ -1885,10 +1819,8 @@ int query_sl_grid(int device, int* grid_f, int* grid_b) {
   if (e == cudaSuccess) e = sl_smem_attr(fwdx_kernel<true, true>, kXStageBytes);
   if (e == cudaSuccess) e = sl_smem_attr(eval_kernel<false>, kEvalSmem);
   if (e == cudaSuccess) e = sl_smem_attr(eval_kernel<true>, kEvalSmem);
-  if (e == cudaSuccess) e = sl_smem_attr(bwdl_kernel<false, false>, kBStageBytes);
-  if (e == cudaSuccess) e = sl_smem_attr(bwdl_kernel<true, false>, kBStageBytes);
-  if (e == cudaSuccess) e = sl_smem_attr(bwdl_kernel<false, true>, kBStageBytes);
-  if (e == cudaSuccess) e = sl_smem_attr(bwdl_kernel<true, true>, kBStageBytes);
+  if (e == cudaSuccess) e = sl_smem_attr(bwdl_kernel<false>, kBStageBytes);
+  if (e == cudaSuccess) e = sl_smem_attr(bwdl_kernel<true>, kBStageBytes);
   if (e != cudaSuccess) return int(e);
   int occ = 1 << 30, b = 0;
   const void* kf[] = {(const void*)fwdl_kernel<false, 0>, (const void*)fwdl_kernel<true, 0>,
@@ -1910,9 +1842,8 @@ int query_sl_grid(int device, int* grid_f, int* grid_b) {
   if (occ <= 0) return int(cudaErrorLaunchOutOfResources);
   *grid_f = sms;   // one CTA per SM (the stage and the barrier arrival are per CTA)
   occ = 1 << 30;
-  const void* kb[] = {(const void*)bwdl_kernel<false, false>, (const void*)bwdl_kernel<true, false>,
-                      (const void*)bwdl_kernel<false, true>, (const void*)bwdl_kernel<true, true>};
-  for (int i = 0; i < 4; ++i) {
+  const void* kb[] = {(const void*)bwdl_kernel<false>, (const void*)bwdl_kernel<true>};
+  for (int i = 0; i < 2; ++i) {
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kb[i], kSLBwdThreads, kBStageBytes);
     if (e != cudaSuccess) return int(e);
     occ = std::min(occ, b);
@@ -2063,19 +1994,6 @@ int launch_eval_candidates(DevGraph& g, int num, const int32_t* cand_ptr, const 
   return err;
 }
 
-// the sweep backward: 0 (default) = a grid barrier per super-level; 1 = arrival counters per head
-// instead (a head waits for one counted share per entry it sources; a fence per head orders its
-// shares before its counts): parity-green but slower at C4, 0.445 vs 0.382 ms -- the per-head fence
-// and the doubled atomic traffic cost more than the barrier (INSTA_BWD_FLOW=1; measurements only)
-static bool bwd_flow() {
-  static int m = -1;
-  if (m < 0) {
-    const char* v = getenv("INSTA_BWD_FLOW");
-    m = v ? atoi(v) : 0;
-  }
-  return m != 0;
-}
-
 int launch_backward_sl(DevGraph& g, float* d_arc_mean, float* d_src, void* stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   if (g.n == 0) return 0;
@@ -2087,9 +2005,8 @@ int launch_backward_sl(DevGraph& g, float* d_arc_mean, float* d_src, void* strea
     P.hab_b = g.hab_b;
   }
   const bool lse = g.last_tau > 0.f;
-  const void* fn = bwd_flow() ? (lse ? (const void*)bwdl_kernel<true, true> : (const void*)bwdl_kernel<false, true>)
-                              : (lse ? (const void*)bwdl_kernel<true, false> : (const void*)bwdl_kernel<false, false>);
-  return launch_coop(fn, g.sl_grid_b, kSLBwdThreads, kBStageBytes, P, st, lse ? "bwd_lse" : "bwd");
+  return launch_coop(lse ? (const void*)bwdl_kernel<true> : (const void*)bwdl_kernel<false>, g.sl_grid_b,
+                     kSLBwdThreads, kBStageBytes, P, st, lse ? "bwd_lse" : "bwd");
 }
 
 // insta_backward_update: a snapshot backward (full sweep backward + snapshot), or the
