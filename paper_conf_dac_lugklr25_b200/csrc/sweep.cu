@@ -805,7 +805,11 @@ constexpr int kXCap = 2048;   // entries of a slice held in shared memory
 #ifndef INSTA_SX_PREFETCH
 #define INSTA_SX_PREFETCH 1
 #endif
-constexpr bool kSXPrefetch = INSTA_SX_PREFETCH != 0;   // L2 prefetch of the next level's arc records
+constexpr bool kSXPrefetch = INSTA_SX_PREFETCH != 0;   // L2 prefetch of a later level's arc records
+#ifndef INSTA_SX_AHEAD
+#define INSTA_SX_AHEAD 1
+#endif
+constexpr int kSXAhead = INSTA_SX_AHEAD;               // how many levels ahead
 // head merge specialized for 1-4 entries: LSE only (measured: hard mode is faster with the generic loop)
 #ifndef INSTA_SX_HEADN
 #define INSTA_SX_HEADN 2
@@ -1080,7 +1084,10 @@ __global__ void __launch_bounds__(sx_threads(kLSE), 1) fwdx_kernel(SLParams P) {
     if (L > 1) {
       const int4 c = slice_of(P, s_slc, 1);
       fwd_issue(P, S, 1, c.x, c.y, c.z, c.w);
-      sx_prefetch_rec(P, c.z, c.w);
+      for (int a = 1; a <= kSXAhead && a < L; ++a) {
+        const int4 d = slice_of(P, s_slc, a);
+        sx_prefetch_rec(P, d.z, d.w);
+      }
     }
   }
   for (int s = gt; s < L; s += nthr) P.sl_cnt[s] = 0u;   // a full pass supersedes pending flags
@@ -1100,7 +1107,10 @@ __global__ void __launch_bounds__(sx_threads(kLSE), 1) fwdx_kernel(SLParams P) {
     if (tid == 0 && s + 1 < L) {
       const int4 c = slice_of(P, s_slc, s + 1);
       fwd_issue(P, S, bf ^ 1, c.x, c.y, c.z, c.w);
-      if (kSXPrefetch) sx_prefetch_rec(P, c.z, c.w);
+      if (kSXPrefetch && s + kSXAhead < L) {
+        const int4 d = slice_of(P, s_slc, s + kSXAhead);
+        sx_prefetch_rec(P, d.z, d.w);
+      }
     }
     if (!kFlow) grid_sync(P.bar, ++nbar, P.trace);   // levels < s are complete
 #ifdef INSTA_SL_PHASES
