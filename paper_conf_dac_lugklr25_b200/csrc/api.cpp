@@ -67,7 +67,7 @@ void free_graph(insta::DevGraph& d) {
                   d.cl_mv,     d.cl_pre,    d.cl_g,      d.cl_fo_ptr,  d.cl_fo_q,   d.cl_slack,
                   d.cl_rf,     d.cl_summary, d.cl_hv_list, d.cl_hv_of, d.cl_hv_sum, d.tl_partials, d.sz_tmp,
                   d.sl_ptr,    d.ext_sh,    d.hd_csl,    d.chg,       d.acc_h,     d.sl_bar,    d.sl_cnt,
-                  d.hwin,      d.ew,        d.fwin,      d.efw,       d.sl_slice,  d.hfo_ptr,   d.hfo,       d.hd_hsrc,
+                  d.hwin,      d.ew,        d.fwin,      d.efw,       d.sl_slice,  d.hfo_ptr,   d.hfo,       d.hfo_sl,    d.hd_hsrc,
                   d.cand_old,  d.elog,  d.xscr,  d.acc_b, d.hab_b, d.hseed_b, d.hwin_b, d.fwin_b, d.ew_b, d.efw_b, d.btouch, d.bdirty, d.bl_cnt, d.ep_blk,    d.cand_ptr_d, d.pl_ptr,    d.pl_ent,    d.pl_arc,    d.pl_wide};
   for (void* p : ptrs)
     if (p) cudaFree(p);
@@ -345,6 +345,13 @@ insta_status insta_graph_create(const insta_graph_desc* desc, insta_graph** out)
   UP(d.hd_csl, fold.hd_csl.data(), fold.hd_csl.size());
   UP(d.hfo_ptr, fold.hfo_ptr.data(), fold.hfo_ptr.size());
   UP(d.hfo, fold.hfo.data(), fold.hfo.size());
+  {   // the super-level of every consumer head in the rows (heads are in super-level order)
+    std::vector<int32_t> hsl(fold.hd_pin.size(), 0), fsl(fold.hfo.size(), 0);
+    for (int32_t sv = 0; sv + 1 < int32_t(fold.slevel_ptr.size()); ++sv)
+      for (int32_t hh = fold.slevel_ptr[sv]; hh < fold.slevel_ptr[sv + 1]; ++hh) hsl[size_t(hh)] = sv;
+    for (size_t r = 0; r < fold.hfo.size(); ++r) fsl[r] = hsl[size_t(fold.hfo[r])];
+    UP(d.hfo_sl, fsl.data(), fsl.size());
+  }
   UP(d.hd_hsrc, fold.hd_hsrc.data(), fold.hd_hsrc.size());
   ZERO(d.chg, nN);
   ZERO(d.acc_h, 2 * fold.hd_pin.size());

@@ -243,6 +243,7 @@ struct DevGraph {
   int32_t* hd_csl = nullptr;       // [H] consumer super-level range of each head
   int32_t* hfo_ptr = nullptr;      // [H+1] consumer heads of each head
   int32_t* hfo = nullptr;
+  int32_t* hfo_sl = nullptr;       // super-level of each hfo entry (cone pass: the level to flag)
   uint8_t* hd_hsrc = nullptr;      // [H] a source with a long consumer row
   uint32_t* chg = nullptr;         // [n] cone pass: stamp of the pass that changed the pin's record
   long long* acc_h = nullptr;      // [H][2] fixed-point adjoint accumulators (zero between passes)

@@ -101,6 +101,7 @@ struct SLParams {
   const int32_t* __restrict__ hd_csl;     // [H] consumer super-level range (min | max << 16, -1 none)
   const int32_t* __restrict__ hfo_ptr;    // [H+1] consumer heads (deduplicated rows)
   const int32_t* __restrict__ hfo;
+  const int32_t* __restrict__ hfo_sl;     // super-level of each hfo entry
   const uint8_t* __restrict__ hd_hsrc;    // [H] a source of the head has a long consumer row
   uint32_t* chg;                          // [n] == stamp: the pin's record changed in this cone pass
   uint32_t* sl_cnt;                      // [SL] level marked (cleared by the pass)
@@ -302,6 +303,18 @@ __device__ __forceinline__ void fwd_issue(const SLParams& P, FStageSet* S, int b
   }
 }
 
+// L2 prefetch of a byte range (TMA bulk prefetch; 16-byte aligned, size a multiple of 16)
+__device__ __forceinline__ void prefetch_l2(const void* p, uint32_t bytes) {
+  if (bytes) asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
+}
+
+// the arc records of entries [xa, xb) (the next level's slice): off the dependency chain
+__device__ __forceinline__ void sx_prefetch_rec(const SLParams& P, int xa, int xb) {
+  if (xb <= xa) return;
+  prefetch_l2(P.ext_ms + xa, uint32_t(xb - xa) * 16u);
+  prefetch_l2(P.ext_fms + xa, uint32_t(xb - xa) * 16u);
+}
+
 // Folded pin p (fold.cpp) on its single fanin arc e' = (j -> p) (word f,
 // record fms, entry x): merge1, the nf = 1 merge (bit-identical to merge_rf),
 // on j's words rj.  Returns p's words as a store would leave them (parity
@@ -340,9 +353,16 @@ __device__ __forceinline__ Raw sl_fold(const SLParams& P, int32_t f, const float
 // consumer row changed -- the level's heads with such a source check it.
 constexpr int kMarkWords = 64;   // levels >= 32 * kMarkWords are flagged in global directly
 
+// (read before the atomic: most marks find the bit set already -- the heads of a level mark the
+// same few levels, and same-word shared atomics serialize: ncu / trace, ~20 us per level at C3 1 %)
 __device__ __forceinline__ void mark_level(const SLParams& P, uint32_t* s_mark, int s, uint32_t kind) {
-  if (s < 32 * kMarkWords) atomicOr(s_mark + (kind - 1) * kMarkWords + (s >> 5), 1u << (s & 31));
-  else atomicOr(P.sl_cnt + s, kind);
+  if (s < 32 * kMarkWords) {
+    uint32_t* w = s_mark + (kind - 1) * kMarkWords + (s >> 5);
+    const uint32_t b = 1u << (s & 31);
+    if (!(*reinterpret_cast<volatile uint32_t*>(w) & b)) atomicOr(w, b);
+  } else if (!(__ldcg(P.sl_cnt + s) & kind)) {
+    atomicOr(P.sl_cnt + s, kind);
+  }
 }
 
 // flag levels [lo, hi] (kind 2)
@@ -355,7 +375,7 @@ __device__ __forceinline__ void mark_range(const SLParams& P, uint32_t* s_mark, 
     uint32_t m = 0xffffffffu;
     if (w == (lo >> 5)) m &= 0xffffffffu << (lo & 31);
     if (w == (hi >> 5)) m &= 0xffffffffu >> (31 - (hi & 31));
-    atomicOr(s_mark + kMarkWords + w, m);
+    if ((*reinterpret_cast<volatile uint32_t*>(s_mark + kMarkWords + w) & m) != m) atomicOr(s_mark + kMarkWords + w, m);
   }
 }
 
@@ -524,20 +544,24 @@ __device__ __forceinline__ int sl_fwd_head(const SLParams& P, int h, const HeadT
         const int k = __ldg(P.hd_eop + h);
         if (k >= 0) {
           const int b = (k / kRedThreads) % P.slack_nb;
-          atomicOr(P.ep_blk + (b >> 5), 1u << (b & 31));
+          // (read first: a few words take every endpoint's flag, global atomics on them serialize)
+          if (!((__ldcg(P.ep_blk + (b >> 5)) >> (b & 31)) & 1u)) atomicOr(P.ep_blk + (b >> 5), 1u << (b & 31));
         }
       }
       const int r0 = __ldg(P.hfo_ptr + h), r1 = __ldg(P.hfo_ptr + h + 1);
       if (r1 - r0 <= kConeRow) {
         for (int r = r0; r < r1; r += 8) {   // the row's loads in flight together
-          int32_t q[8];
+          int32_t q[8], lv[8];
 #pragma unroll
-          for (int j = 0; j < 8; ++j) q[j] = r + j < r1 ? __ldg(P.hfo + r + j) : -1;
+          for (int j = 0; j < 8; ++j) {
+            q[j] = r + j < r1 ? __ldg(P.hfo + r + j) : -1;
+            lv[j] = r + j < r1 ? __ldg(P.hfo_sl + r + j) : 0;
+          }
 #pragma unroll
           for (int j = 0; j < 8; ++j) {
             if (q[j] >= 0) {
               P.dirty[q[j]] = stamp;
-              mark_level(P, s_mark, sl_of(P, s_slp, q[j]), 1u);
+              mark_level(P, s_mark, lv[j], 1u);
             }
           }
         }
@@ -691,6 +715,7 @@ __global__ void __launch_bounds__(kSLFwdThreads, 1) fwdl_kernel(SLParams P) {
       if (tid == 0 && s + 1 < L) {   // rows and entry words of level s + 1
         const int4 c = slice_of(P, s_slc, s + 1);
         fwd_issue(P, S, bf ^ 1, c.x, c.y, c.z, c.w);
+        if (kInc) sx_prefetch_rec(P, c.z, c.w);   // and its arc records to L2 (off the dirty heads' chain)
       }
       if (need_bar) grid_sync(P.bar, ++nbar, P.trace);   // levels < s are complete
       unsigned long long* ph = nullptr;
@@ -740,7 +765,13 @@ __global__ void __launch_bounds__(kSLFwdThreads, 1) fwdl_kernel(SLParams P) {
         }
         if (kInc) {
           if (!head_dirty(P, h, E.w, t.nf, lvl, P.stamp)) continue;
+#ifdef INSTA_SL_PHASES
+          if (ph && !ph[3]) ph[3] = gtimer();   // debug: the first dirty head found
+#endif
           nrec += uint32_t(sl_fwd_head<kLSE, true>(P, h, t, E, cs.mark, s_slp, P.stamp, ph));
+#ifdef INSTA_SL_PHASES
+          if (ph && !ph[7]) ph[7] = gtimer();   // debug: its recompute and marks done
+#endif
         } else {
           (void)sl_fwd_head<kLSE, false>(P, h, t, E, cs.mark, s_slp, P.stamp, ph);
         }
@@ -821,18 +852,6 @@ struct XCand {
 };
 constexpr size_t kXOff = (kFStageBytes + 127) & ~size_t(127);
 constexpr size_t kXStageBytes = kXOff + sizeof(XCand) * 2 * kXCap + kXCap;
-
-// L2 prefetch of a byte range (TMA bulk prefetch; 16-byte aligned, size a multiple of 16)
-__device__ __forceinline__ void prefetch_l2(const void* p, uint32_t bytes) {
-  if (bytes) asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
-}
-
-// the arc records of entries [xa, xb) (the next level's slice): off the dependency chain
-__device__ __forceinline__ void sx_prefetch_rec(const SLParams& P, int xa, int xb) {
-  if (xb <= xa) return;
-  prefetch_l2(P.ext_ms + xa, uint32_t(xb - xa) * 16u);
-  prefetch_l2(P.ext_fms + xa, uint32_t(xb - xa) * 16u);
-}
 
 template <bool kFlow>
 __device__ __forceinline__ void sx_await(const SLParams& P, int j, Raw& r) {
@@ -1775,6 +1794,7 @@ static SLParams sl_params(DevGraph& g) {
   P.hd_csl = g.hd_csl;
   P.hfo_ptr = g.hfo_ptr;
   P.hfo = g.hfo;
+  P.hfo_sl = g.hfo_sl;
   P.hd_hsrc = g.hd_hsrc;
   P.chg = g.chg;
   P.sl_cnt = g.sl_cnt;
