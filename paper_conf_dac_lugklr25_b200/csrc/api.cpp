@@ -68,7 +68,7 @@ void free_graph(insta::DevGraph& d) {
                   d.cl_rf,     d.cl_summary, d.cl_hv_list, d.cl_hv_of, d.cl_hv_sum, d.tl_partials, d.sz_tmp,
                   d.sl_ptr,    d.ext_sh,    d.hd_csl,    d.chg,       d.acc_h,     d.sl_bar,    d.sl_cnt,
                   d.hwin,      d.ew,        d.fwin,      d.efw,       d.sl_slice,  d.hfo_ptr,   d.hfo,       d.hfo_sl,    d.hd_hsrc,
-                  d.cand_old,  d.elog,  d.xscr,  d.acc_b, d.hab_b, d.hseed_b, d.hwin_b, d.fwin_b, d.ew_b, d.efw_b, d.btouch, d.bdirty, d.bl_cnt, d.ep_blk,    d.cand_ptr_d, d.pl_ptr,    d.pl_ent,    d.pl_arc,    d.pl_wide};
+                  d.cand_old,  d.elog,  d.xscr,  d.acc_b, d.hab_b, d.hseed_b, d.hwin_b, d.fwin_b, d.ew_b, d.efw_b, d.btouch, d.bdirty, d.bl_cnt, d.ep_blk,    d.cand_ptr_d, d.pl_ptr,    d.pl_ent,    d.pl_arc,    d.pl_wide,   d.pl_xy};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   if (d.b_stage_h) cudaFreeHost(d.b_stage_h);

@@ -314,6 +314,8 @@ struct DevGraph {
   int32_t* pl_ent = nullptr;       // [2e] other end (caller pin) | 1 << 31 if the pin is the arc's sink
   int32_t* pl_arc = nullptr;       // [2e] caller arc id
   int32_t* pl_wide = nullptr;      // caller pins with more than kPlWide incident arcs
+  void* pl_xy = nullptr;           // Eq 7: positions packed per pin (scratch)
+  int32_t pl_xy_cap = 0;
   int32_t num_pl_wide = -1;        // -1: not built
   // CPPR required times per (endpoint, startpoint) (insta_set_cppr_rat)
   int32_t* rat_ptr = nullptr;      // [P+1] or NULL (no table)

@@ -40,6 +40,7 @@ struct TlParams {
   const int32_t* __restrict__ wide;
   const float* __restrict__ x;            // caller order
   const float* __restrict__ y;
+  const float2* __restrict__ xy;          // (x, y) packed per pin (tl_pack_kernel): one 8-byte gather per arc end
   const float* __restrict__ w;            // caller arc order
   double* partials;
   float* gx;
@@ -48,18 +49,43 @@ struct TlParams {
 
 __device__ __forceinline__ double sgn(double d) { return d > 0.0 ? 1.0 : (d < 0.0 ? -1.0 : 0.0); }
 
-// incident arcs k0, k0 + step, ... < k1 of pin (xi, yi): gradient sums and the driver-side loss
+// incident arcs k0, k0 + step, ... < k1 of pin (xi, yi): gradient sums and the driver-side loss.
+// Four arcs per round: their row words, then their gathers, all in flight before any is used
+// (the same sums in the same order as one arc at a time).
 __device__ __forceinline__ void tl_row(const TlParams& P, double xi, double yi, int k0, int k1, int step,
                                        double& gx, double& gy, double& loss) {
-  for (int k = k0; k < k1; k += step) {
-    const int32_t e = __ldg(P.ent + k);
-    const int o = e & 0x7fffffff;
-    const double wk = double(__ldg(P.w + __ldg(P.arc + k)));
-    const double dx = xi - double(__ldg(P.x + o)), dy = yi - double(__ldg(P.y + o));
-    gx += wk * sgn(dx);
-    gy += wk * sgn(dy);
-    if (e >= 0) loss += (fabs(dx) + fabs(dy)) * wk;   // counted once, at the driver
+  for (int k = k0; k < k1; k += 4 * step) {
+    int32_t e[4], a[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int kk = k + j * step;
+      e[j] = kk < k1 ? __ldg(P.ent + kk) : 0;
+      a[j] = kk < k1 ? __ldg(P.arc + kk) : 0;
+    }
+    float2 po[4];
+    float wv[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const bool v = k + j * step < k1;
+      po[j] = v ? __ldg(P.xy + (e[j] & 0x7fffffff)) : make_float2(0.f, 0.f);
+      wv[j] = v ? __ldg(P.w + a[j]) : 0.f;
+    }
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      if (k + j * step < k1) {
+        const double wk = double(wv[j]);
+        const double dx = xi - double(po[j].x), dy = yi - double(po[j].y);
+        gx += wk * sgn(dx);
+        gy += wk * sgn(dy);
+        if (e[j] >= 0) loss += (fabs(dx) + fabs(dy)) * wk;   // counted once, at the driver
+      }
+    }
   }
+}
+
+__global__ void tl_pack_kernel(int n, const float* __restrict__ x, const float* __restrict__ y, float2* xy) {
+  for (int p = blockIdx.x * blockDim.x + threadIdx.x; p < n; p += gridDim.x * blockDim.x)
+    xy[p] = make_float2(__ldg(x + p), __ldg(y + p));
 }
 
 __device__ __forceinline__ double block_sum(double v, double* s) {
@@ -80,7 +106,8 @@ __global__ void __launch_bounds__(kTlThreads) tl_pin_kernel(TlParams P, int want
   if (p < P.n) {
     const int k0 = __ldg(P.ptr + p), k1 = __ldg(P.ptr + p + 1);
     if (k1 - k0 <= kPlWide) {
-      const double xi = double(__ldg(P.x + p)), yi = double(__ldg(P.y + p));
+      const float2 pi = __ldg(P.xy + p);
+      const double xi = double(pi.x), yi = double(pi.y);
       double gx = 0.0, gy = 0.0;
       tl_row(P, xi, yi, k0, k1, 1, gx, gy, loss);
       if (want_grad) {
@@ -196,8 +223,16 @@ int launch_timing_loss(DevGraph& g, const float* x, const float* y, const float*
   P.ent = g.pl_ent;
   P.arc = g.pl_arc;
   P.wide = g.pl_wide;
+  if (g.pl_xy_cap < g.n) {   // packed positions (scratch)
+    if (g.pl_xy) cudaFree(g.pl_xy);
+    g.pl_xy = nullptr;
+    cudaError_t e = cudaMalloc(&g.pl_xy, sizeof(float2) * size_t(std::max(g.n, 1)));
+    if (e != cudaSuccess) return int(e);
+    g.pl_xy_cap = g.n;
+  }
   P.x = x;
   P.y = y;
+  P.xy = reinterpret_cast<const float2*>(g.pl_xy);
   P.w = w;
   P.partials = g.tl_partials;
   P.gx = gx;
@@ -208,6 +243,8 @@ int launch_timing_loss(DevGraph& g, const float* x, const float* y, const float*
     if (loss) cudaMemsetAsync(loss, 0, sizeof(double), st);
     return int(cudaGetLastError());
   }
+  if (g.n > 0)
+    tl_pack_kernel<<<std::min((g.n + 255) / 256, 148 * 8), 256, 0, st>>>(g.n, x, y, reinterpret_cast<float2*>(g.pl_xy));
   if (nb > 0) tl_pin_kernel<<<nb, kTlThreads, 0, st>>>(P, want_grad);
   if (P.num_wide > 0) tl_wide_kernel<<<unsigned((32LL * P.num_wide + 255) / 256), 256, 0, st>>>(P, want_grad);
   if (loss) tl_final_kernel<<<1, 1024, 0, st>>>(np, P.lambda, g.tl_partials, loss);

@@ -514,6 +514,78 @@ __global__ void __launch_bounds__(32 * kTkWideWarps) tk_wide_kernel(TkParams P) 
   }
 }
 
+// Single-arc pins at K > 32 (a unate fanin arc: 11.2M of 15M pins at C4): the queue is the
+// parent's, each slot shifted by the arc (Eq 1-3) -- one parent's startpoints are unique, so
+// (R19) only the order by key (A desc, t = 2k asc) can change.  A warp per (pin, rf), K / 32
+// slots per lane; the usual case (already in key order, one ballot over adjacent pairs) is
+// written straight back, otherwise the warp sorts in shared memory (tk_sm_sort) -- the same
+// queue the merging kernel builds for one arc, bit for bit.
+__global__ void __launch_bounds__(32 * kTkWideWarps) tk_one_wide_kernel(TkParams P) {
+  __shared__ TkWideSm S[kTkWideWarps];
+  const int lane = threadIdx.x & 31;
+  TkWideSm& Q = S[threadIdx.x >> 5];
+  const long long grp = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
+  if (grp >= 2LL * (P.hi - P.lo)) return;   // uniform within the warp
+  const int i = __ldg(P.list + P.lo + int(grp >> 1)), rf = int(grp & 1), K = P.K;
+  const int a = __ldg(P.fanin_ptr + i);
+  const int32_t w = __ldg(P.fin_src + a);
+  const float4 ms = __ldg(P.fin_ms + a);
+  const size_t ps = (size_t(w & kSrcMask) * 2 + src_tr(rf, int(uint32_t(w) >> kUnateShift), 0)) * K;
+  const double am = double(rf ? ms.y : ms.x), se = double(rf ? ms.w : ms.z);
+  constexpr int kPer = kTkWideMax / 32;
+  TkEnt c[kPer];
+#pragma unroll
+  for (int j = 0; j < kPer; ++j) {
+    const int k = 32 * j + lane;
+    const int csp = k < K ? __ldg(P.qsp + ps + k) : -1;
+    const double2 pv = k < K ? __ldg(P.q + ps + k) : make_double2(0.0, 0.0);
+    c[j].sp = csp;
+    c[j].mu = pv.x + am;                                 // Eq 1
+    c[j].var = pv.y + se * se;                           // Eq 2
+    c[j].A = csp >= 0 ? c[j].mu + P.ns * double(sigma_of(c[j].var)) : -INFINITY;   // Eq 3
+    c[j].t = csp >= 0 ? 2 * k : INT_MAX;                 // single arc: t = 2k
+  }
+  // in key order already?  pairs (k, k + 1) within a row of 32 and across rows
+  bool bad = false;
+#pragma unroll
+  for (int j = 0; j < kPer; ++j) {
+    const double nA = __shfl_down_sync(0xffffffffu, c[j].A, 1);
+    const int nt = __shfl_down_sync(0xffffffffu, c[j].t, 1);
+    const double xA = j + 1 < kPer ? __shfl_sync(0xffffffffu, c[j + 1 < kPer ? j + 1 : j].A, 0) : -INFINITY;
+    const int xt = j + 1 < kPer ? __shfl_sync(0xffffffffu, c[j + 1 < kPer ? j + 1 : j].t, 0) : INT_MAX;
+    const int k = 32 * j + lane;
+    if (lane < 31 && k + 1 < K) bad |= key_gt(nA, nt, c[j].A, c[j].t);
+    if (lane == 31 && k + 1 < K && j + 1 < kPer) bad |= key_gt(xA, xt, c[j].A, c[j].t);
+  }
+  if (__ballot_sync(0xffffffffu, bad)) {   // reorder by key in shared memory
+#pragma unroll
+    for (int j = 0; j < kPer; ++j)
+      if (32 * j + lane < K) tk_sm_put(Q, 32 * j + lane, c[j]);
+    __syncwarp();
+    tk_sm_sort(Q, K, lane);
+#pragma unroll
+    for (int j = 0; j < kPer; ++j) {
+      const int k = 32 * j + lane;
+      if (k < K) {
+        c[j].A = Q.A[k];
+        c[j].mu = Q.mu[k];
+        c[j].var = Q.var[k];
+        c[j].t = Q.t[k];
+        c[j].sp = Q.sp[k];
+      }
+    }
+  }
+#pragma unroll
+  for (int j = 0; j < kPer; ++j) {
+    const int k = 32 * j + lane;
+    if (k < K) {
+      const size_t o = (size_t(i) * 2 + rf) * K + k;
+      P.q[o] = c[j].sp >= 0 ? make_double2(c[j].mu, c[j].var) : make_double2(0.0, 0.0);
+      P.qsp[o] = c[j].sp;
+    }
+  }
+}
+
 // CPPR slack: warp per endpoint; slack = min over (rf, k) of
 // RAT(ep, SP_k)[rf] - A_k[rf], the first minimum in (rf, k) order wins.
 __global__ void __launch_bounds__(256)
@@ -731,13 +803,18 @@ int launch_topk_forward(DevGraph& g, int K, float n_sigma, void* stream) {
   P.fin_ms = g.fin_ms;
   P.q = g.tk_q;
   P.qsp = g.tk_sp;
-  if (K > 32) {   // wide queues: a warp per (pin, rf), every pin of a level in one launch
+  if (K > 32) {   // wide queues: a warp per (pin, rf); single-arc pins, then the merging pins of a level
     for (int l = 1; l < g.num_levels; ++l) {
       P.lo = g.tk_one_ptr[l];
+      P.hi = g.tk_multi_ptr[l];
+      if (P.hi > P.lo)
+        tk_one_wide_kernel<<<unsigned((2LL * (P.hi - P.lo) + kTkWideWarps - 1) / kTkWideWarps),
+                             32 * kTkWideWarps, 0, st>>>(P);
+      P.lo = g.tk_multi_ptr[l];
       P.hi = g.tk_one_ptr[l + 1];
-      if (P.hi <= P.lo) continue;
-      const long long warps = 2LL * (P.hi - P.lo);
-      tk_wide_kernel<<<unsigned((warps + kTkWideWarps - 1) / kTkWideWarps), 32 * kTkWideWarps, 0, st>>>(P);
+      if (P.hi > P.lo)
+        tk_wide_kernel<<<unsigned((2LL * (P.hi - P.lo) + kTkWideWarps - 1) / kTkWideWarps), 32 * kTkWideWarps, 0,
+                         st>>>(P);
     }
     return int(cudaGetLastError());
   }
