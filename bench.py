@@ -525,14 +525,16 @@ def main():
                 torch.distributed.barrier()
             b0, b1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             b0.record(stream)
-            summ_all, grad_sum = idist.evaluate_sharded(ev, scs, n_ocv, E, rank, world, dev, dd)
+            ctiming = {}
+            summ_all, grad_sum = idist.evaluate_sharded(ev, scs, n_ocv, E, rank, world, dev, dd, timing=ctiming)
             b1.record(stream)
             torch.cuda.synchronize(dev)
             bms = b0.elapsed_time(b1)
+        coll_ms = None
         if world > 1:
-            t = torch.tensor([bms], dtype=torch.float64, device=dev)
+            t = torch.tensor([bms, ctiming.get("collective_ms", 0.0)], dtype=torch.float64, device=dev)
             torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-            bms = float(t.item())
+            bms, coll_ms = (float(x) for x in t.tolist())
         sa = summ_all.cpu().numpy()
         split = None
         if world == 1:   # the two halves timed separately (and the sizing half on the batched kernels too)
@@ -555,7 +557,7 @@ def main():
                    "evals": nsc, "ms": bms, "evals_per_s": nsc / (bms * 1e-3),
                    "pins_per_s": nsc * N / (bms * 1e-3), "n_gpus": world,
                    "collectives": "all_gather(per-scenario summaries) + all_reduce(SUM, gradient sum)" if world > 1
-                   else "none (1 rank)",
+                   else "none (1 rank)", "collective_ms": coll_ms,
                    "tns_min": float(sa[:, 1].min()), "tns_max": float(sa[:, 1].max())}
 
     # ---------------- Top-K unique-startpoint propagation + CPPR slack -------------

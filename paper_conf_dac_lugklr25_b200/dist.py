@@ -21,13 +21,16 @@ def scenario_block(n: int, rank: int, world: int):
     return lo, min(n, lo + per), per
 
 
-def evaluate_sharded(evaluate, scenarios, n_grad: int, num_arcs: int, rank: int, world: int, device, dist=None):
+def evaluate_sharded(evaluate, scenarios, n_grad: int, num_arcs: int, rank: int, world: int, device, dist=None,
+                     timing: dict | None = None):
     """Evaluate `scenarios` sharded over `world` ranks.
 
     evaluate(list_of_scenarios, want_grad) -> (summaries [k, 3] float64 tensor, grad [E, 2] float32 or None)
     Scenarios with index < n_grad contribute to the gradient sum.  Returns
     (summaries [n, 3] float64 on `device`, grad_sum [num_arcs, 2] float32 on
-    `device`), identical on every rank."""
+    `device`), identical on every rank.  timing (optional dict): 'collective_ms' = device time from the
+    end of this rank's evaluations to the gathered result (the all_gather plus what is left of the
+    overlapped all_reduce; CUDA events on the current stream)."""
     import torch
     n = len(scenarios)
     n_f = n - n_grad
@@ -48,6 +51,10 @@ def evaluate_sharded(evaluate, scenarios, n_grad: int, num_arcs: int, rank: int,
     if f_idx:
         s_f, _ = evaluate([scenarios[s] for s in f_idx], False)
         summ[gper: gper + len(f_idx)] = s_f
+    ev0 = ev1 = None
+    if timing is not None and world > 1 and torch.cuda.is_available() and str(device).startswith("cuda"):
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ev0.record()
     if world > 1:
         parts = [torch.empty_like(summ) for _ in range(world)]
         dist.all_gather(parts, summ)
@@ -59,6 +66,10 @@ def evaluate_sharded(evaluate, scenarios, n_grad: int, num_arcs: int, rank: int,
             out[n_grad + c: n_grad + d] = part[gper: gper + d - c]
         work.wait()
         summ = out
+        if ev0 is not None:
+            ev1.record()
+            ev1.synchronize()
+            timing["collective_ms"] = ev0.elapsed_time(ev1)
     else:
         summ = torch.cat([summ[: len(g_idx)], summ[gper: gper + len(f_idx)]])
     return summ, grad
