@@ -511,3 +511,43 @@ def test_appendix_a_gpu(mode):
         e, r = map(int, k.split(","))
         want_s[e, r] = v
     assert np.allclose(dm, want_m, atol=1e-3) and np.allclose(ds, want_s, atol=1e-3)
+
+
+def _wide_level(n_heads, wide_fanin, seed=5):
+    """One level of n_heads single-input endpoint heads (more than 1024 per CTA slice: the entry-
+    parallel forward reads that slice's topology from global) plus one head with wide_fanin inputs
+    (more entries than a slice's shared-memory candidate buffer: the CTA's global buffer)."""
+    rng = np.random.default_rng(seed)
+    n_src = n_heads + wide_fanin
+    N = n_src + n_heads + 1
+    src = np.arange(n_src)
+    af = np.concatenate([src[:n_heads], src[n_heads:]]).astype(np.int32)
+    at = np.concatenate([n_src + np.arange(n_heads), np.full(wide_fanin, N - 1)]).astype(np.int32)
+    E = len(af)
+    un = rng.integers(0, 3, E).astype(np.uint8)
+    mean = rng.uniform(1, 20, (E, 2)).astype(np.float32)
+    sig = rng.uniform(0, 2, (E, 2)).astype(np.float32)
+    eps = np.arange(n_src, N, dtype=np.int32)
+    rat = rng.uniform(40, 60, (len(eps), 2)).astype(np.float32)
+    return types.SimpleNamespace(num_pins=N, arc_from=af, arc_to=at, arc_unate=un,
+                                 arc_class=np.zeros(E, np.uint8), arc_mean=mean, arc_sigma=sig,
+                                 src_mean=rng.uniform(0, 30, (N, 2)).astype(np.float32),
+                                 src_sigma=rng.uniform(0, 3, (N, 2)).astype(np.float32), ep_pin=eps, ep_rat=rat)
+
+
+@pytest.mark.parametrize("tau", [0.0, 1.0])
+def test_forward_unstaged_and_global_candidate_paths(tau):
+    # 160k heads in one level (1081 per CTA > the 1024-row stage) and a 3000-input head (> 2048
+    # candidate slots and > 2560 staged entries): schedule 0 (flow) and 3 (barriers) equal the
+    # per-level schedule bit for bit and the oracle within tolerance
+    g = _wide_level(160_000, 3000)
+    a = run_gpu(g, tau, 0)
+    b = run_gpu(g, tau, 3)
+    c = run_gpu(g, tau, 1)
+    for x in (a, b):
+        assert np.array_equal(x.A, c.A) and np.array_equal(x.mu, c.mu) and np.array_equal(x.sigma, c.sigma)
+        assert np.array_equal(x.slack, c.slack)
+        assert grads_match(x.d_mean, c.d_mean, tau)
+    f, s, o = run_oracle(g, tau)
+    assert not tol_ok(a.A, f["A"]).any()
+    assert abs(a.summary.tns - s["tns"]) <= 1e-5 * abs(s["tns"]) + 1e-3
