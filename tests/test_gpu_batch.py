@@ -167,3 +167,26 @@ def test_eval_candidates_cone(tau):
         s = H.forward(3.0, tau)
         H.close()
         assert summ[k, 0] == s.wns and summ[k, 1] == s.tns and summ[k, 2] == s.num_violations, k
+
+
+@pytest.mark.parametrize("tau", [0.0, 1.0])
+def test_batch_and_candidates_against_oracle_c2(tau):
+    """C2 (200k pins): OCV scenarios (insta_forward_batch) and one-cell sizing candidates
+    (insta_eval_candidates) against the fp64 oracle on each materialized graph -- TNS / WNS within
+    the slack tolerance, violation counts equal."""
+    g = synth.generate("C2")
+    ocv = scenarios(g, 6, seed=11)
+    cand = [synth.sizing_scenario(g, s) for s in range(700, 706)]
+    G = insta.Graph(g)
+    s_ocv = G.forward_batch(ocv, tau=tau, want_grad=False)[0].cpu().numpy()
+    G.forward(3.0, tau)
+    s_cand = G.eval_candidates(cand).cpu().numpy()
+    G.close()
+    for summ, scs in ((s_ocv, ocv), (s_cand, cand)):
+        for k, sc in enumerate(scs):
+            h = materialize(g, sc)
+            f = oracle.forward(h, sc["n_sigma"], tau)
+            o = oracle.slack(h, f["A"])
+            assert summ[k, 1] == pytest.approx(o["tns"], rel=1e-5, abs=1e-3), (k, summ[k], o["tns"])
+            assert summ[k, 0] == pytest.approx(o["wns"], rel=1e-4, abs=1e-3)
+            assert abs(summ[k, 2] - o["num_viol"]) <= 1   # a slack within rounding of 0 may flip
