@@ -726,7 +726,7 @@ def main():
         c4 = inc_series(G, g, [(1e-7, 20), (1e-5, 20), (1e-4, 10)], [("incremental", 0), ("full", 0)], 7000)
         incremental = {"C4_small_updates": c4,
                        "what": "per step: insta_update_arcs + insta_forward (CUDA events); incremental = default "
-                               "policy (cone pass for <= max(64, E/1e5) updated arcs), full = the same updates "
+                               "policy (cone pass for <= max(64, E/5e4) updated arcs), full = the same updates "
                                "then a full pass"}
         incremental["C4_backward_update"] = bwd_series(G, g, [(1e-7, 12), (1e-6, 12), (1e-5, 12), (1e-4, 8)], 8000)
         incremental["C4_backward_update_what"] = (

@@ -86,7 +86,7 @@ typedef struct {
  * the cone pass (only heads whose inputs changed are
  * recomputed) when at most this many arcs were re-annotated, else a full pass
  * (for large batches the cone of a random update reaches every level, and the
- * dataflow full pass is faster).  0 = default limit max(64, num_arcs / 1e5);
+ * dataflow full pass is faster).  0 = default limit max(64, num_arcs / 5e4) (the measured crossover);
  * < 0 = never. */
 typedef struct {
   float n_sigma;

@@ -473,7 +473,7 @@ insta_status insta_forward(insta_graph* g, const insta_opts* o, void* cuda_strea
   // must be in the layout this schedule's backward reads -- head/entry order for 0 and 3,
   // canonical for 2)
   const bool sweep_sched = opt.schedule == 0 || opt.schedule == 3;
-  const int64_t cone_max = opt.cone_max != 0 ? opt.cone_max : std::max<int64_t>(64, d.e / 100000);
+  const int64_t cone_max = opt.cone_max != 0 ? opt.cone_max : std::max<int64_t>(64, d.e / 50000);   // crossover measured: tools/cone_cross.py
   const bool inc = d.pending_incremental && !d.pending_full && opt.schedule != 1 &&
                    opt.n_sigma == d.last_n_sigma && opt.tau == d.last_tau &&
                    (sweep_sched ? d.sweep_valid && d.pending_updates <= cone_max : d.canon_valid);
