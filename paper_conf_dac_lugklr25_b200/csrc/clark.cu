@@ -165,15 +165,20 @@ __global__ void cl_slack_kernel(int num_ep, double ns, const int32_t* __restrict
 __global__ void __launch_bounds__(1024) cl_reduce_kernel(int num_ep, const double* __restrict__ slack, double* out) {
   __shared__ double s_t[1024], s_w[1024], s_n[1024];
   const int t = threadIdx.x;
-  const int ch = (num_ep + 1023) / 1024;
   double tns = 0.0, wns = 0.0, nv = 0.0;
-  for (int e = t * ch; e < min(num_ep, (t + 1) * ch); ++e) {
-    const double s = slack[e];
-    if (s < 0.0) {
-      tns += s;
-      nv += 1.0;
+  // thread t sums endpoints t, t + 1024, ... (coalesced; four loads in flight), fixed order
+  for (int e0 = t; e0 < num_ep; e0 += 4 * 1024) {
+    double v[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) v[j] = e0 + j * 1024 < num_ep ? slack[e0 + j * 1024] : 0.0;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      if (v[j] < 0.0) {
+        tns += v[j];
+        nv += 1.0;
+      }
+      wns = fmin(wns, v[j]);
     }
-    wns = fmin(wns, s);
   }
   s_t[t] = tns;
   s_w[t] = wns;
@@ -233,20 +238,35 @@ __device__ __forceinline__ double2 cl_pull(const ClParams& P, int rf, int k0, in
 
 // Pins with a wide fanout row (> kClWide): a warp per (pin, rf) pulls the row
 // (lanes strided, fixed shuffle tree) into hv_sum before the level's fold kernel.
+// A CTA of kClPullThreads per (pin, rf): thread t sums entries t, t + 128, ... in row order, then a
+// fixed shuffle tree per warp and the warps in order -- deterministic; a 20k-sink net takes ~160
+// rounds of one thread instead of ~625 of one warp lane (the warp-per-pin pull was 1.8 of the 6.1 ms
+// backward at C4).
 constexpr int kClWide = 32;
-__global__ void cl_pull_wide_kernel(ClParams P) {
-  const long long x = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
-  const int lane = threadIdx.x & 31;
+constexpr int kClPullThreads = 128;
+__global__ void __launch_bounds__(kClPullThreads) cl_pull_wide_kernel(ClParams P) {
+  __shared__ double2 s_w[kClPullThreads / 32];
+  const long long x = blockIdx.x;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   if (x >= 2LL * (P.hv_hi - P.hv_lo)) return;
   const int h = P.hv_lo + int(x >> 1), rf = int(x & 1);
   const int i = __ldg(P.hv_list + h);
-  double2 s = cl_pull(P, rf, __ldg(P.fo_ptr + i) + lane, __ldg(P.fo_ptr + i + 1), 32);
+  double2 s = cl_pull(P, rf, __ldg(P.fo_ptr + i) + int(threadIdx.x), __ldg(P.fo_ptr + i + 1), kClPullThreads);
 #pragma unroll
   for (int d = 16; d > 0; d >>= 1) {
     s.x += __shfl_down_sync(0xffffffffu, s.x, d);
     s.y += __shfl_down_sync(0xffffffffu, s.y, d);
   }
-  if (lane == 0) P.hv_sum[size_t(h) * 2 + rf] = s;
+  if (lane == 0) s_w[warp] = s;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double2 t = s_w[0];
+    for (int w = 1; w < kClPullThreads / 32; ++w) {
+      t.x += s_w[w].x;
+      t.y += s_w[w].y;
+    }
+    P.hv_sum[size_t(h) * 2 + rf] = t;
+  }
 }
 
 // Backward of one level, a thread per (pin, rf): (1) the adjoint of (pin, rf)
@@ -442,8 +462,8 @@ int launch_clark_backward(DevGraph& g, const float* ep_seed, float* d_mean, floa
     P.hi = lp[l + 1];
     P.hv_lo = g.cl_hv_ptr[l];
     P.hv_hi = g.cl_hv_ptr[l + 1];
-    if (P.hv_hi > P.hv_lo)   // a warp per (wide pin, rf)
-      cl_pull_wide_kernel<<<unsigned((64LL * (P.hv_hi - P.hv_lo) + 255) / 256), 256, 0, st>>>(P);
+    if (P.hv_hi > P.hv_lo)   // a CTA per (wide pin, rf)
+      cl_pull_wide_kernel<<<unsigned(2LL * (P.hv_hi - P.hv_lo)), kClPullThreads, 0, st>>>(P);
     const long long threads = 2LL * (P.hi - P.lo);
     if (threads > 0) cl_bwd_kernel<<<unsigned((threads + 255) / 256), 256, 0, st>>>(P);
   }
