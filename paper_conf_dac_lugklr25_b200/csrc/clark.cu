@@ -273,7 +273,10 @@ __global__ void __launch_bounds__(kClPullThreads) cl_pull_wide_kernel(ClParams P
 // = the pulled fanout slots (+ the endpoint seed); (2) reverse the fold with
 // Clark's Jacobian at (prefix, candidate), write each candidate's adjoint slot
 // and the arc gradients.
-__global__ void cl_bwd_kernel(ClParams P) {
+#ifndef CL_BWD_MINB
+#define CL_BWD_MINB 4   // resident 256-thread blocks per SM (<= 64 registers): latency-bound gathers want warps
+#endif
+__global__ void __launch_bounds__(256, CL_BWD_MINB) cl_bwd_kernel(ClParams P) {
   const long long x = blockIdx.x * (long long)blockDim.x + threadIdx.x;
   if (x >= 2LL * (P.hi - P.lo)) return;
   const int i = P.lo + int(x >> 1), rf = int(x & 1);
