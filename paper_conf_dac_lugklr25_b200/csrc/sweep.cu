@@ -1,47 +1,46 @@
-// sweep.cu -- level-synchronous, thread-per-head passes of the INSTA hot path
-// (schedule 0, the default).
+// sweep.cu -- the persistent passes of the INSTA hot path on the stage-folded
+// schedule (schedule 0, the default).
 //
 // The stage-folded schedule (fold.cpp) groups the pins into "heads" by
 // super-level; a netlist's cell input pins are folded into the work of the
 // cell output that consumes them, so one (net arc, cell arc) stage costs one
 // dependent step (C4: 162 timing levels -> 82 super-levels, every head has at
 // most 4 entries).  ONE persistent cooperative launch runs a whole pass: CTA c
-// owns the c-th contiguous slice of every super-level's heads (one thread per
-// head), and a grid barrier separates consecutive super-levels.  The paper
-// launches one kernel per timing level with a thread per output pin (P:L113,
-// L123); this keeps the thread-per-pin mapping but replaces the launch chain by
-// one barrier per super-level and halves the chain length by folding.
+// owns the c-th contiguous slice of every super-level's heads and entries.  The
+// paper launches one kernel per timing level with a thread per output pin
+// (P:L113, L123); this replaces the launch chain by one persistent launch and
+// halves the chain length by folding.
 //
 // Topology staging: a CTA's slice of a level is contiguous in every head- and
-// entry-ordered array, so one thread stages the slice of level s + 1 with TMA
-// bulk copies (cp.async.bulk + mbarrier) while level s is processed; after the
-// barrier only the source-state gathers (forward) or the accumulator reads
-// (backward) are on the dependency chain.  What the backward reads is stored
-// by the forward in head / entry order (arg-max word per head, Eq 6 weights
-// per entry), so it is staged the same way.
+// entry-ordered array, so one thread stages the slice of the next level with
+// TMA bulk copies (cp.async.bulk + mbarrier) while the current one runs.
 //
-//  * forward (fwdl_kernel): Eq 1-3 candidates and the K = 1 merge of
-//    Alg 1 / Alg 2 (first arg-max, strict ">") or the LSE smooth max
-//    of Eq 4, the same device functions as the other schedules
-//    (device_common.cuh), hence the same arrivals bit for bit.  Folded pins are
-//    evaluated in registers; their records are not stored (their only consumer
-//    is the head's thread): insta_arrivals and the sigma-channel backward
-//    materialize them on demand (fold_fill_kernel).
-//  * cone pass (mode 1): the same kernel visits only heads
-//    whose dirty stamp is this pass's -- stamped by insta_update_arcs for the
-//    arcs they evaluate, or by a recomputed source head whose record changed
-//    bitwise -- and skips the barrier of a super-level with no dirty head.
+//  * forward, full pass (fwdx_kernel): per super-level an entry phase (a thread
+//    per entry: gather, folded pin, both transitions' Eq 1-3 candidates into
+//    shared-memory slots) and a head phase (a thread per head: the first
+//    arg-max of Alg 1 / Alg 2, strict ">", or the LSE smooth max
+//    of Eq 4; the store); kFlow: no grid barrier, gathers re-poll
+//    until the record carries this pass's parity (dataflow), the next level's
+//    arc records prefetched to L2.  Folded pins are evaluated in registers and
+//    not stored: insta_arrivals and the sigma channel materialize them on
+//    demand (fold_fill_kernel).
+//  * cone pass (fwdl_kernel, modes 1 / 2): visits only
+//    super-levels flagged by a stamped or changed source, recomputes the dirty
+//    heads (thread per head), compares each new record with the previous one
+//    bitwise and marks the consumers of a changed one; a level with no flag is
+//    skipped without a barrier.
+//  * candidate evaluation (eval_kernel; C5 sizing candidates): apply, cone
+//    pass, the flagged slack blocks, undo log, per candidate in one launch.
 //  * backward (bwdl_kernel): Eq 6 weights chained in reverse super-level order
-//    (P:L138, L152).  Push form: every entry adds its source's adjoint share
-//    into that source head's accumulator with integer atomics (fixed point,
-//    2^-32 ps units; integer addition is exact and order-independent, so the
-//    result is deterministic), and a head reads (and clears) its accumulator
-//    after the barrier that closes its consumers' levels.  Heavy drivers'
-//    shares are first combined per CTA in shared memory.
+//    (P:L138, L152), push form with int64 fixed-point accumulators (2^-32 ps;
+//    exact, order-independent, deterministic), a grid barrier per level.
+//  * incremental backward (bdiff_kernel + bwdi_kernel; NEXT 3): fixed-point
+//    share deltas over the reverse cone of what changed since a snapshot --
+//    bit-identical to the full backward.
 //
-// Every 64-bit state word still carries the pass parity in its LSB (stored
-// values are truncated by <= 1 ulp exactly as in the dataflow schedule 2, so
-// all schedules produce the same arrivals bit for bit).
+// Every 64-bit state word carries the pass parity in its LSB (stored values
+// are truncated by <= 1 ulp identically in every schedule), so all schedules
+// produce the same arrivals bit for bit.
 #include <cuda_runtime.h>
 
 #include <algorithm>
