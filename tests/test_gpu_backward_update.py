@@ -95,3 +95,21 @@ def test_update_policy_many_arcs_runs_full():
     assert G.backward_update(out) is False
     assert np.array_equal(bits(out), bits(G.backward()))
     G.close()
+
+
+@pytest.mark.slow
+def test_update_c4_one_cell_steps():
+    """C4 (15M pins) at the headline scale: one-cell sizing steps through the cone pass, the kept
+    TNS gradient brought up to date by the reverse cone equals a full backward bit for bit."""
+    g = synth.generate("C4")
+    G = insta.Graph(g)
+    G.forward(3.0, 0.0)
+    out = torch.zeros((g.num_arcs, 2), dtype=torch.float32, device="cuda")
+    assert G.backward_update(out) is False
+    for step in range(3):
+        ids, m, s = synth.sizing_step(g, 60 + step, frac=1e-6)
+        G.update_arcs(ids, m, s, incremental=True)
+        G.forward(3.0, 0.0)
+        assert G.backward_update(out) is True
+        assert np.array_equal(bits(out), bits(G.backward())), step
+    G.close()
