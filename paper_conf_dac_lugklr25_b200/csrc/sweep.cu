@@ -61,10 +61,10 @@ namespace insta {
 #define INSTA_SL_FWD_THREADS 384
 #endif
 #ifndef INSTA_SL_BWD_THREADS
-#define INSTA_SL_BWD_THREADS 1024
+#define INSTA_SL_BWD_THREADS 768
 #endif
 constexpr int kSLFwdThreads = INSTA_SL_FWD_THREADS;   // forward: ~128-168 registers per thread, 1 CTA / SM
-constexpr int kSLBwdThreads = INSTA_SL_BWD_THREADS;   // backward: <= 64 registers, 1 CTA / SM
+constexpr int kSLBwdThreads = INSTA_SL_BWD_THREADS;   // backward: 1 CTA / SM (768 measured best of 512 / 768 / 1024)
 constexpr int kSLNf = 4;                              // entries per head held in registers (netlists: <= 4)
 constexpr double kAccScale = 4294967296.0;            // 2^32: fixed-point unit of the backward accumulators
 constexpr double kAccInv = 1.0 / 4294967296.0;
